@@ -1,0 +1,172 @@
+/*
+ * hauberk.h — C ABI of the B200 (sm_100a) HAUBERK hot path.
+ *
+ * HAUBERK (Yim et al., IPDPS 2011; /root/reference/PAPER.md, "Lnnn" = line) derives lightweight
+ * software detectors for silent data corruption in GPU kernels: duplication + an XOR checksum on
+ * non-loop code (L986-1053 [§V.A]) and accumulator/counter value-range checks on loops
+ * (L1216-1313, L1405-1508 [§V.B]), reported through a control block after the kernel ends
+ * (L751-762, L1202-1214), and evaluates them with a software fault injector (L2083-2305 [§VII-VIII]).
+ * This library implements that path for three Parboil-class kernels (CP, MRI-Q, TPACF) —
+ * DESIGN.md §3 states the exact per-thread programs.
+ *
+ * Conventions (every entry point):
+ *  - Pointers inside *_args structs, d_cb, d_samples, d_records, d_counts, d_site_counts are
+ *    DEVICE pointers owned by the caller; the library never frees them.  Host structs
+ *    (hk_ranges, hk_*_args, hk_campaign, hk_profile_opts) are read during the call only.
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *  - Return value: HK_OK or an hk_status; no exception crosses the ABI.  Invalid arguments return
+ *    HK_ERR_INVALID before anything is launched.  CUDA failures return HK_ERR_CUDA; the text is in
+ *    hauberk_last_error() (thread-local).
+ *  - A detected SDC is DATA, not an error: it is reported in hk_control.alarm (L757-759).
+ *  - Device kernels are compiled for sm_100a only; there is no CPU fallback.
+ */
+#ifndef HAUBERK_H
+#define HAUBERK_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define HK_ABI_VERSION 1
+
+#if defined(__GNUC__)
+#define HK_API __attribute__((visibility("default")))
+#else
+#define HK_API
+#endif
+
+typedef int32_t hk_status;
+enum {
+  HK_OK = 0,
+  HK_ERR_INVALID = 1,      /* bad argument; nothing launched */
+  HK_ERR_CUDA = 2,         /* a CUDA API call failed; see hauberk_last_error() */
+  HK_ERR_NO_RANGES = 3,    /* FT variant without profiled ranges */
+  HK_ERR_OOM = 4,          /* stream-ordered allocation failed */
+  HK_ERR_UNSUPPORTED = 5,  /* shape/variant not compiled in (e.g. FI kernels only for unroll 4) */
+  HK_ERR_PROFILE_NAN = 6,  /* a PROFILE sample was NaN/Inf */
+  HK_ERR_GOLDEN_ALARM = 7  /* the fault-free golden run raised an alarm (ranges do not fit the input) */
+};
+
+enum { HK_CP = 0, HK_MRIQ = 1, HK_TPACF = 2, HK_MIXED = -1 };
+
+/* Variants (PAPER Fig. 7, Table I): BASE = original program (overhead denominator);
+ * FT = HAUBERK-NL + HAUBERK-L; FT_NL / FT_L = one detector family only (Fig. 13 columns);
+ * PROFILE = accumulator/counter and per-thread samples of acc/it (no checks). */
+enum { HK_BASE = 0, HK_FT = 1, HK_FT_NL = 2, HK_FT_L = 3, HK_PROFILE = 4 };
+
+/* Outcome classes (L2377-2387). */
+enum { HK_MASKED = 0, HK_DETECTED_MASKED = 1, HK_DETECTED = 2, HK_UNDETECTED = 3, HK_FAILURE = 4 };
+
+/* hk_control.alarm bits / hk_control.fail bits. */
+enum { HK_ALARM_DUP = 1, HK_ALARM_CHECKSUM = 2, HK_ALARM_RANGE = 4, HK_ALARM_COUNT = 8 };
+enum { HK_FAIL_CRASH = 1, HK_FAIL_HANG = 2 };
+
+/* Up to three correlation-point ranges per loop detector (L1489-1508). */
+typedef struct { int32_t n; float lo[3], hi[3]; int32_t t_exp10; } hk_range_set;
+/* Ranges of all loop detectors of one kernel; alpha widens them (L2073-2077, DESIGN R11). */
+typedef struct { int32_t n_det; float alpha; hk_range_set det[8]; } hk_ranges;
+
+/* Control block (L1202-1214): device-resident, written by the kernel, read by the caller after
+ * the stream completes.  Reset by every hauberk_run_* call before its kernel. 96 bytes. */
+typedef struct {
+  uint32_t alarm;             /* OR of alarm bits of all threads */
+  uint32_t fail;              /* FI only: modelled crash / hang (R16, R17) */
+  uint32_t n_alarm_warps;     /* warps with >= 1 alarming thread */
+  uint32_t first_thread;      /* smallest alarming abstract thread id (0xffffffff if none) */
+  int32_t outlier_min_ord[8]; /* A11 (L1309-1313): ordinal (R8) range of out-of-range values */
+  int32_t outlier_max_ord[8];
+  uint32_t fault_applied;     /* FI only: the flip happened */
+  uint32_t check_margin;      /* FI only: min ordinal distance of the faulted thread's checks to a bound */
+  uint32_t domain;            /* FI only: faulted thread left the MUFU accuracy domain (R22c) */
+  uint32_t reserved;
+} hk_control;
+
+/* CP (K1; Fig. 9).  atoms: [n_atoms] (x, y, z, q); atoms_ws: [n_atoms] float4 scratch
+ * for the (x, y, dz^2, q) pre-pass; grid: [ny][nx] output, zeroed by the callee.
+ * Requires nx % (bx*unroll) == 0, ny % by == 0, bx*by <= 1024, unroll in {1,2,4,8}. */
+typedef struct {
+  const float* atoms; float* atoms_ws; int32_t n_atoms; float z0, h;
+  int32_t nx, ny, bx, by, unroll; float* grid; int32_t exact;
+} hk_cp_args;
+
+/* MRI-Q (K2).  x,y,z: [n_vox]; kx..phi_i: [n_k]; kv_ws: [n_k] float4 scratch (PhiMag output);
+ * qr, qi: [n_vox] outputs (zeroed by the callee). */
+typedef struct {
+  const float *x, *y, *z; int32_t n_vox, n_k;
+  const float *kx, *ky, *kz, *phi_r, *phi_i; float* kv_ws; float *qr, *qi; int32_t exact;
+} hk_mriq_args;
+
+/* TPACF (K3).  pts: [(1+n_rand)][n][3] unit vectors (set 0 = data); edges: [n_bins+1] strictly
+ * decreasing cos(angle) edges; hist: [(1+2*n_rand)][n_bins+2] u64 output (zeroed by the callee).
+ * chunk = partners per abstract thread.  n_bins <= 30. */
+typedef struct {
+  const float* pts; const float* edges; int32_t n, n_rand, n_bins, chunk; unsigned long long* hist;
+} hk_tpacf_args;
+
+typedef struct { int32_t maxvar; int32_t t0_exp10; float alpha; } hk_profile_opts; /* defaults 1, -5, 1 */
+
+/* Campaign (L2295-2305, L2370-2387).  Injections n in [first, first+count) decoded from
+ * (seed, n) (DESIGN R14-R15); mode 0 = replica (every injection is a full program run; the only
+ * mode of this version); batch = replicas per launch (0 = auto); site_mask[b] bit s enables site s. */
+typedef struct {
+  uint64_t seed; int64_t first, count; int32_t nbits; int32_t mode; int32_t batch; int32_t exact;
+  uint64_t site_mask[3];
+} hk_campaign;
+
+/* One decoded injection (DESIGN R13-R15). */
+typedef struct { int32_t site; int32_t pad; int64_t thread, inst; uint64_t mask; } hk_fault;
+
+/* One classified injection (device array, `count` entries, slot = n - first). */
+typedef struct {
+  int64_t index; int32_t bench, site; int64_t thread, inst; uint64_t mask;
+  int32_t cls; uint32_t alarm, fail, domain, margin; float worst; /* worst err/tol (R22b) */
+} hk_outcome;
+
+/* Run one benchmark kernel (plus its uninstrumented pre-pass / PhiMag) on `stream`.
+ * variant: HK_BASE | HK_FT | HK_FT_NL | HK_FT_L | HK_PROFILE.  ranges: required for FT/FT_L
+ * (HK_ERR_NO_RANGES otherwise), ranges->n_det detectors are checked.  d_cb: required except BASE.
+ * d_samples: PROFILE only, [maxvar][threads] floats (maxvar = ranges ? ranges->n_det : 1).
+ * Stream-asynchronous. */
+HK_API hk_status hauberk_run_cp(const hk_cp_args* args, int32_t variant, const hk_ranges* ranges,
+                         hk_control* d_cb, float* d_samples, void* stream);
+HK_API hk_status hauberk_run_mriq(const hk_mriq_args* args, int32_t variant, const hk_ranges* ranges,
+                           hk_control* d_cb, float* d_samples, void* stream);
+HK_API hk_status hauberk_run_tpacf(const hk_tpacf_args* args, int32_t variant, const hk_ranges* ranges,
+                            hk_control* d_cb, float* d_samples, void* stream);
+
+/* PROFILE run + threshold search (L1489-1508) -> out (host).  Synchronises `stream`.
+ * args points to the bench's hk_*_args; opts may be NULL (defaults). */
+HK_API hk_status hauberk_profile_ranges(int32_t bench, const void* args, const hk_profile_opts* opts,
+                                 hk_ranges* out, void* stream);
+
+/* Seeded injection campaign.  bench_mode: HK_CP/HK_MRIQ/HK_TPACF or HK_MIXED (bench = n mod 3).
+ * args[b]/ranges[b]: per benchmark (unused ones may be NULL).  Runs the golden (fault-free FT)
+ * program per benchmark, checks it raises no alarm, then launches the FI&FT replicas and the
+ * classify epilogue.  d_counts: int64 [3][5] accumulated (+=); d_site_counts: nullable int64
+ * [3][64][5] (+=); d_records: nullable [count].  Synchronises `stream` once at the start (golden
+ * alarm check); the injections are enqueued asynchronously. */
+HK_API hk_status hauberk_inject_campaign(int32_t bench_mode, const void* const args[3],
+                                  const hk_ranges* const ranges[3], const hk_campaign* campaign,
+                                  hk_outcome* d_records, int64_t* d_counts, int64_t* d_site_counts,
+                                  void* stream);
+
+/* Host-side decode of injections [first, first+count) (same rule the campaign uses). */
+HK_API hk_status hauberk_decode(int32_t bench_mode, const void* const args[3], const uint64_t site_mask[3],
+                         uint64_t seed, int64_t first, int64_t count, int32_t* bench_out, hk_fault* out);
+
+/* Number of injection sites of a benchmark (unroll only matters for CP). */
+HK_API int32_t hauberk_num_sites(int32_t bench, int32_t unroll);
+
+HK_API const char* hauberk_strerror(hk_status s);
+HK_API const char* hauberk_last_error(void);
+HK_API int32_t hauberk_version(void);
+/* Kernels this library has launched since load (process-wide counter, for bench accounting). */
+HK_API uint64_t hauberk_launch_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* HAUBERK_H */

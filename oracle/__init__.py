@@ -101,6 +101,8 @@ def lib():
         L.ora_tpacf_trips.restype = C.c_int64; L.ora_tpacf_trips.argtypes = [P, C.c_int64]
         L.ora_tpacf_threads.restype = C.c_int64; L.ora_tpacf_threads.argtypes = [P]
         L.ora_cp_threads.restype = C.c_int64; L.ora_cp_threads.argtypes = [P]
+        L.ora_cp_threads_out.restype = C.c_int; L.ora_cp_threads_out.argtypes = [P, C.c_int32, P, C.c_int64, P, P]
+        L.ora_mriq_threads_out.restype = C.c_int; L.ora_mriq_threads_out.argtypes = [P, C.c_int32, P, C.c_int64, P, P]
         L.ora_cp_reference_f64.restype = None; L.ora_cp_reference_f64.argtypes = [P, P, P]
         L.ora_mriq_reference_f64.restype = None; L.ora_mriq_reference_f64.argtypes = [P, P, P, P]
         L.ora_threshold.restype = C.c_float; L.ora_threshold.argtypes = [C.c_int32]
@@ -296,3 +298,19 @@ def reference_f64(bench: int, p):
     qr = np.zeros(p.n_vox); qi = np.zeros(p.n_vox); mass = np.zeros(p.n_vox)
     L.ora_mriq_reference_f64(C.byref(a), _p(qr), _p(qi), _p(mass))
     return (qr, qi), mass
+
+
+def threads_out(bench: int, p, tids, exact: int = 0):
+    """Outputs of selected abstract threads only (sampled parity at full sizes).
+    CP: (flat grid indices [n, U], values [n, U]); MRI-Q: (qr [n], qi [n])."""
+    t = np.ascontiguousarray(np.asarray(tids, dtype=np.int64))
+    L = lib()
+    if bench == CP:
+        a = cp_args(p)
+        idx = np.zeros((t.size, p.unroll), dtype=np.int64); val = np.zeros((t.size, p.unroll), dtype=np.float32)
+        assert L.ora_cp_threads_out(C.byref(a), exact, _p(t), t.size, _p(idx), _p(val)) == 0
+        return idx, val
+    a = mriq_args(p)
+    qr = np.zeros(t.size, dtype=np.float32); qi = np.zeros(t.size, dtype=np.float32)
+    assert L.ora_mriq_threads_out(C.byref(a), exact, _p(t), t.size, _p(qr), _p(qi)) == 0
+    return qr, qi

@@ -642,6 +642,30 @@ ORA_EXPORT int ora_tpacf_run(const ora_tpacf_args* P, int32_t flags, const ora_r
   return 0;
 }
 
+/* Outputs of single abstract threads (for sampled parity at full sizes): CP writes U values per
+ * thread (grid index, value); MRI-Q writes (Qr, Qi) of each voxel. */
+ORA_EXPORT int ora_cp_threads_out(const ora_cp_args* P, int32_t exact, const int64_t* tids, int64_t n, int64_t* idx, float* val) {
+  if (!cp_valid(P)) return 1;
+  float* A4 = cp_prepass(P);
+  for (int64_t q = 0; q < n; ++q) {
+    tout o; tout_init(&o);
+    cp_thread(P, A4, tids[q], 0, exact, NULL, 0, NULL, &o, NULL, 0);
+    for (int w = 0; w < o.nw; ++w) { idx[q * P->unroll + w] = o.widx[w]; val[q * P->unroll + w] = o.wval[w]; }
+  }
+  free(A4);
+  return 0;
+}
+ORA_EXPORT int ora_mriq_threads_out(const ora_mriq_args* P, int32_t exact, const int64_t* tids, int64_t n, float* qr, float* qi) {
+  float* KV = mriq_phimag(P);
+  for (int64_t q = 0; q < n; ++q) {
+    tout o; tout_init(&o);
+    mriq_thread(P, KV, tids[q], 0, exact, NULL, 0, NULL, &o, NULL, 0);
+    qr[q] = o.wval[0]; qi[q] = o.wval[1];
+  }
+  free(KV);
+  return 0;
+}
+
 ORA_EXPORT int64_t ora_tpacf_trips(const ora_tpacf_args* P, int64_t g) { return tp_trips(P, g); }
 ORA_EXPORT int64_t ora_tpacf_threads(const ora_tpacf_args* P) { return tp_threads(P); }
 ORA_EXPORT int64_t ora_cp_threads(const ora_cp_args* P) { return cp_threads(P); }

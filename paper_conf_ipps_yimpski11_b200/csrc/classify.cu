@@ -1,0 +1,178 @@
+// classify.cu — control-block init, golden max|G|, and the campaign's classify epilogue.
+//
+// Outcome classes (DESIGN R1): failure > (wrong, alarm) ->
+// masked / detected&masked / detected / undetected.  Output correctness rules: MRI-Q
+// Max{1e-4*Max|GR|, 0.2%|GR_i|} (L2598-2603, also used for CP: R5); TPACF >1 % on the summed
+// DD/DRS/RRS counts (L80-84, R3/R4).  One CTA per replica; it also re-zeroes the replica's output
+// and resets its control block so the next batch can reuse the workspace without a memset launch.
+#include "hk_internal.h"
+
+namespace hk {
+
+__global__ void control_init_kernel(hk_control* cb, int n) {
+  const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (warp < n) control_reset(cb + warp, (int)lane_id());
+}
+
+cudaError_t control_init_launch(hk_control* cb, int n, cudaStream_t s) {
+  if (n <= 0) return cudaSuccess;
+  const int threads = n * 32;
+  control_init_kernel<<<(threads + 255) / 256, 256, 0, s>>>(cb, n);
+  count_launch();
+  return cudaGetLastError();
+}
+
+// max |g| (g finite): non-negative floats order like their bit patterns -> atomicMax on u32.
+__global__ void max_abs_kernel(const float* __restrict__ g, int64_t n, unsigned* out) {
+  float m = 0.f;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    m = fmaxf(m, fabsf(g[i]));
+  unsigned u = __float_as_uint(m);
+  u = __reduce_max_sync(0xffffffffu, u);
+  if (lane_id() == 0) atomicMax(out, u);
+}
+
+cudaError_t max_abs_launch(const float* g, int64_t n, float* d_out, cudaStream_t s) {
+  cudaError_t e = cudaMemsetAsync(d_out, 0, sizeof(float), s);
+  if (e != cudaSuccess) return e;
+  max_abs_kernel<<<148, 256, 0, s>>>(g, n, reinterpret_cast<unsigned*>(d_out));
+  count_launch();
+  return cudaGetLastError();
+}
+
+__device__ __forceinline__ int32_t classify(bool wrong, uint32_t alarm, uint32_t fail) {
+  if (fail) return HK_FAILURE;
+  if (!wrong) return alarm ? HK_DETECTED_MASKED : HK_MASKED;
+  return alarm ? HK_DETECTED : HK_UNDETECTED;
+}
+
+__device__ void write_outcome(int bench, const FaultRec& f, hk_control* cb, bool wrong, float worst, hk_outcome* records,
+                              int64_t first, int64_t* counts, int64_t* site_counts) {
+  const uint32_t alarm = cb->alarm, fail = cb->fail;
+  const int32_t cls = classify(wrong, alarm, fail);
+  if (records) {
+    hk_outcome o;
+    o.index = f.index; o.bench = bench; o.site = f.site; o.thread = f.thread; o.inst = f.inst; o.mask = f.mask;
+    o.cls = cls; o.alarm = alarm; o.fail = fail; o.domain = cb->domain; o.margin = cb->check_margin; o.worst = worst;
+    records[f.index - first] = o;
+  }
+  atomicAdd(reinterpret_cast<unsigned long long*>(counts + bench * 5 + cls), 1ull);
+  if (site_counts && f.site < 64)
+    atomicAdd(reinterpret_cast<unsigned long long*>(site_counts + ((int64_t)bench * 64 + f.site) * 5 + cls), 1ull);
+}
+
+__device__ __forceinline__ float block_max(float v, float* sh) {
+  v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, 16));
+  v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, 8));
+  v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, 4));
+  v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, 2));
+  v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, 1));
+  if (lane_id() == 0) sh[threadIdx.x >> 5] = v;
+  __syncthreads();
+  float m = 0.f;
+  if (threadIdx.x == 0)
+    for (int w = 0; w < (int)(blockDim.x >> 5); ++w) m = fmaxf(m, sh[w]);
+  return m;  // valid in thread 0
+}
+
+// CP / MRI-Q: elementwise !(|R-G| <= max(1e-4*M, 0.002*|G|)); worst = max err/tol (NaN -> inf).
+__global__ void __launch_bounds__(512) classify_fp_kernel(int bench, float* out0, int64_t elems,
+                                                          const float* __restrict__ golden, const float* __restrict__ dM,
+                                                          hk_control* cb0, const FaultRec* faults, hk_outcome* records,
+                                                          int64_t first, int64_t* counts, int64_t* site_counts) {
+  __shared__ float sh[32];
+  __shared__ int any_wrong;
+  const int r = blockIdx.x;
+  float* R = out0 + (int64_t)r * elems;
+  const float M = *dM;
+  const float tolM = __fmul_rn(1e-4f, M);
+  if (threadIdx.x == 0) any_wrong = 0;
+  __syncthreads();
+  bool wrong = false;
+  float worst = 0.f;
+  const bool vec = ((((uintptr_t)R) | ((uintptr_t)golden)) & 15u) == 0;
+  const int64_t n4 = vec ? elems / 4 : 0;
+  const float4* R4 = reinterpret_cast<const float4*>(R);
+  const float4* G4 = reinterpret_cast<const float4*>(golden);
+  auto one = [&](float rv, float gv) {
+    const float err = fabsf(__fsub_rn(rv, gv));
+    const float tol = fmaxf(tolM, __fmul_rn(0.002f, fabsf(gv)));
+    wrong |= !(err <= tol);
+    float q = __fdiv_rn(err, tol);
+    if (q != q) q = __int_as_float(0x7f800000);
+    worst = fmaxf(worst, q);
+  };
+  for (int64_t i = threadIdx.x; i < n4; i += blockDim.x) {
+    const float4 rv = R4[i], gv = G4[i];
+    one(rv.x, gv.x); one(rv.y, gv.y); one(rv.z, gv.z); one(rv.w, gv.w);
+    reinterpret_cast<float4*>(R)[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+  for (int64_t i = n4 * 4 + threadIdx.x; i < elems; i += blockDim.x) {
+    one(R[i], golden[i]);
+    R[i] = 0.f;
+  }
+  if (wrong) any_wrong = 1;
+  const float wmax = block_max(worst, sh);
+  if (threadIdx.x == 0) {
+    hk_control* cb = cb0 + r;
+    write_outcome(bench, faults[r], cb, any_wrong != 0, wmax, records, first, counts, site_counts);
+  }
+  __syncthreads();
+  if (threadIdx.x < 32) control_reset(cb0 + r, (int)threadIdx.x);
+}
+
+cudaError_t classify_fp_launch(int bench, float* out0, int64_t elems, const float* golden, const float* d_M,
+                               hk_control* cb0, const FaultRec* faults, int nrep, hk_outcome* records, int64_t first,
+                               int64_t* counts, int64_t* site_counts, cudaStream_t s) {
+  if (nrep <= 0) return cudaSuccess;
+  classify_fp_kernel<<<nrep, 512, 0, s>>>(bench, out0, elems, golden, d_M, cb0, faults, records, first, counts,
+                                          site_counts);
+  count_launch();
+  return cudaGetLastError();
+}
+
+// TPACF: outputs DD[1..nb], DRS[1..nb], RRS[1..nb]; wrong iff 100*|h-g| > g (exact integers).
+__global__ void classify_tpacf_kernel(unsigned long long* hist0, int nr, int nb, const unsigned long long* __restrict__ golden,
+                                      hk_control* cb0, const FaultRec* faults, hk_outcome* records, int64_t first,
+                                      int64_t* counts, int64_t* site_counts) {
+  __shared__ float sh[32];
+  __shared__ int any_wrong;
+  const int r = blockIdx.x;
+  const int nb2 = nb + 2, nh = 1 + 2 * nr;
+  unsigned long long* H = hist0 + (int64_t)r * nh * nb2;
+  if (threadIdx.x == 0) any_wrong = 0;
+  __syncthreads();
+  bool wrong = false;
+  float worst = 0.f;
+  for (int o = threadIdx.x; o < 3 * nb; o += blockDim.x) {
+    const int kind = o / nb, b = 1 + o % nb;
+    long long hv = 0, gv = 0;
+    if (kind == 0) { hv = (long long)H[b]; gv = (long long)golden[b]; }
+    for (int s = 1; s <= nr; ++s) {
+      const int row = kind == 1 ? nr + s : s;  // kind 1: DRS, kind 2: RRS
+      if (kind != 0) { hv += (long long)H[row * nb2 + b]; gv += (long long)golden[row * nb2 + b]; }
+    }
+    long long d = hv - gv;
+    if (d < 0) d = -d;
+    if (100 * d > gv) wrong = true;
+    const float q = gv > 0 ? (float)(100.0 * (double)d / (double)gv) : (d > 0 ? __int_as_float(0x7f800000) : 0.f);
+    worst = fmaxf(worst, q);
+  }
+  if (wrong) any_wrong = 1;
+  const float wmax = block_max(worst, sh);
+  if (threadIdx.x == 0) write_outcome(HK_TPACF, faults[r], cb0 + r, any_wrong != 0, wmax, records, first, counts, site_counts);
+  __syncthreads();
+  for (int k = threadIdx.x; k < nh * nb2; k += blockDim.x) H[k] = 0ull;
+  if (threadIdx.x < 32) control_reset(cb0 + r, (int)threadIdx.x);
+}
+
+cudaError_t classify_tpacf_launch(unsigned long long* hist0, int nr, int nb, const unsigned long long* golden,
+                                  hk_control* cb0, const FaultRec* faults, int nrep, hk_outcome* records,
+                                  int64_t first, int64_t* counts, int64_t* site_counts, cudaStream_t s) {
+  if (nrep <= 0) return cudaSuccess;
+  classify_tpacf_kernel<<<nrep, 64, 0, s>>>(hist0, nr, nb, golden, cb0, faults, records, first, counts, site_counts);
+  count_launch();
+  return cudaGetLastError();
+}
+
+}  // namespace hk

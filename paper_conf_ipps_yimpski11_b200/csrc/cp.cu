@@ -1,0 +1,439 @@
+// cp.cu — Coulombic potential (CP, K1) with HAUBERK detectors, for sm_100a.
+//
+// Per abstract thread (PAPER Fig. 9 L1242-1258 and the detector code at
+// L1422-1429): U grid points of one row, E_j = sum_a q_a * rsqrt(dx_j^2 + dy^2 + dz^2).
+// The B200 shape: atoms staged in shared memory by 1-D bulk async copies (TMA engine,
+// cp.async.bulk + mbarrier, double buffered); every thread reads them with broadcast LDS.128;
+// FP32 FADD/FFMA + MUFU.RSQ per interaction; detector state lives in registers; alarms are folded
+// with warp votes and one atomic per warp.  MUFU.RSQ is the binding pipe (16/clk/SM).
+#include "hk_internal.h"
+
+namespace hk {
+
+constexpr int CP_TILE = 1024;  // atoms per stage (16 KB); 2 stages
+
+struct CPParams {
+  const float4* atoms;  // (x, y, dz^2, q)
+  float* grid;
+  hk_control* cb;
+  float* samples;
+  DevRanges R;
+  int32_t numatoms;
+  float h;
+  int32_t ndet;
+  uint32_t z;    // runtime 0 (opaque)
+  int32_t one;   // runtime 1 (opaque)
+  int64_t nthreads;
+};
+
+// One CTA's worth of the protected loop.  V: variant flags; ADD: additive stores (R18, FI replicas).
+template <int V, int U, bool EXACT, bool ADD>
+__device__ __forceinline__ void cp_body(const CPParams& p, float4 (*tile)[CP_TILE], uint64_t* bar) {
+  constexpr bool NL = (V & V_NL) != 0, L = (V & V_L) != 0, PROF = (V & V_PROF) != 0;
+  constexpr bool CNT = L || PROF;
+  const int BX = blockDim.x, BY = blockDim.y;
+  const int tx = threadIdx.x, ty = threadIdx.y;
+  const int bxi = blockIdx.x, byi = blockIdx.y;
+  const uint32_t z = p.z;
+  const uint32_t tid = (uint32_t)(((int64_t)byi * gridDim.x + bxi) * (BX * BY) + ty * BX + tx);
+  uint32_t chk = 0, alarm = 0;
+  const int32_t numatoms = p.numatoms;
+  const float h = p.h;
+  if (NL) chk ^= (uint32_t)numatoms ^ fb(h) ^ lohi_ptr(p.grid) ^ lohi_ptr(p.atoms);
+
+  // ---- non-loop virtual variables: def; chk ^= v; duplicate; compare (L1017-1042)
+  const int32_t xindex = bxi * (BX * U) + tx;
+  if (NL) { chk ^= (uint32_t)xindex; alarm |= ((int32_t)((bxi ^ z) * (BX * U) + (tx ^ z)) != xindex) ? AL_DUP : 0u; }
+  const int32_t yindex = byi * BY + ty;
+  if (NL) { chk ^= (uint32_t)yindex; alarm |= ((int32_t)((byi ^ z) * BY + (ty ^ z)) != yindex) ? AL_DUP : 0u; }
+  const int32_t nx = gridDim.x * BX * U;
+  const int32_t outaddr = nx * yindex + xindex;
+  if (NL) { chk ^= (uint32_t)outaddr; alarm |= ((int32_t)(nx * opq(yindex, z) + opq(xindex, z)) != outaddr) ? AL_DUP : 0u; }
+  const float coorx = __fmul_rn(h, (float)xindex);
+  if (NL) { chk ^= fb(coorx); alarm |= (fb(__fmul_rn(bf(fb(h) + z), (float)opq(xindex, z))) != fb(coorx)) ? AL_DUP : 0u; }
+  const float coory = __fmul_rn(h, (float)yindex);
+  if (NL) { chk ^= fb(coory); alarm |= (fb(__fmul_rn(bf(fb(h) + z), (float)opq(yindex, z))) != fb(coory)) ? AL_DUP : 0u; }
+  const float gu = __fmul_rn(h, (float)BX);
+  if (NL) { chk ^= fb(gu); alarm |= (fb(__fmul_rn(bf(fb(h) + z), (float)opq(BX, z))) != fb(gu)) ? AL_DUP : 0u; }
+  if (NL) { chk ^= (uint32_t)opq(xindex, z); chk ^= (uint32_t)opq(yindex, z); }  // (iv) after last use
+
+  // ---- the loop: self-accumulators E_j (no accumulator needed, L1277) + counter it (L1286)
+  float E[U];
+#pragma unroll
+  for (int j = 0; j < U; ++j) E[j] = 0.0f;
+  int32_t it = 0;
+  const int lin = ty * BX + tx;
+  const int ntiles = (numatoms + CP_TILE - 1) / CP_TILE;
+  if (lin == 0) {
+    mbar_init(&bar[0], 1);
+    mbar_init(&bar[1], 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+  if (lin == 0 && ntiles > 0) {
+    const int cnt0 = min(CP_TILE, numatoms);
+    bulk_g2s(tile[0], p.atoms, (uint32_t)cnt0 * 16u, &bar[0]);
+  }
+  for (int t = 0; t < ntiles; ++t) {
+    const int buf = t & 1;
+    if (lin == 0 && t + 1 < ntiles) {
+      const int cnt1 = min(CP_TILE, numatoms - (t + 1) * CP_TILE);
+      fence_proxy_async();
+      bulk_g2s(tile[buf ^ 1], p.atoms + (size_t)(t + 1) * CP_TILE, (uint32_t)cnt1 * 16u, &bar[buf ^ 1]);
+    }
+    mbar_wait(&bar[buf], (uint32_t)(t >> 1) & 1u);
+    const float4* A = tile[buf];
+    const int cnt = min(CP_TILE, numatoms - t * CP_TILE);
+#pragma unroll 4
+    for (int a = 0; a < cnt; ++a) {
+      const float4 at = A[a];
+      const float dy = __fsub_rn(coory, at.y);
+      const float dyz2 = __fmaf_rn(dy, dy, at.z);
+      float dx = __fsub_rn(coorx, at.x);
+#pragma unroll
+      for (int j = 0; j < U; ++j) {
+        if (j) dx = __fadd_rn(dx, gu);
+        const float r2 = __fmaf_rn(dx, dx, dyz2);
+        const float s = hk_rsqrt<EXACT>(r2);
+        E[j] = __fmaf_rn(at.w, s, E[j]);
+      }
+      if (CNT) it = count_inc(it, p.one);
+    }
+    __syncthreads();
+  }
+
+  // ---- after the loop: HauberkCheckEqual / HauberkCheckRange (L1428-1429)
+  if (L && it != numatoms) alarm |= AL_COUNT;
+  if (CNT && it != 0) {
+    const float fit = (float)it;
+#pragma unroll
+    for (int d = 0; d < U; ++d) {
+      if (d < p.ndet) {
+        const float v = __fdiv_rn(E[U - 1 - d], fit);
+        if (PROF) p.samples[(int64_t)d * p.nthreads + tid] = v;
+        if (L && p.R.n[d] > 0 && !in_range<false>(p.R, d, v, nullptr)) {
+          alarm |= AL_RANGE;
+          record_outlier(p.cb, d, v);
+        }
+      }
+    }
+  }
+  if (NL) { chk ^= opqf(coorx, z); chk ^= opqf(coory, z); chk ^= opqf(gu, z); }
+#pragma unroll
+  for (int j = 0; j < U; ++j) {
+    float* dst = p.grid + (outaddr + j * BX);
+    if (ADD) atomicAdd(dst, E[j]);
+    else *dst = E[j];
+  }
+  if (NL) {
+    chk ^= (uint32_t)opq(outaddr, z);
+    chk ^= ((uint32_t)numatoms + z) ^ (fb(h) + z) ^ (lohi_ptr(p.grid) + z) ^ (lohi_ptr(p.atoms) + z);
+    if (chk != 0) alarm |= AL_CHK;
+  }
+  if (NL || L) fold_alarm(p.cb, alarm, tid);
+}
+
+template <int V, int U, bool EXACT>
+__global__ void __launch_bounds__(256) cp_kernel(const CPParams p) {
+  __shared__ __align__(128) float4 tile[2][CP_TILE];
+  __shared__ __align__(8) uint64_t bar[2];
+  cp_body<V, U, EXACT, false>(p, tile, bar);
+}
+
+// Uninstrumented pre-pass (row a1): (x, y, z, q) -> (x, y, (z - z0)^2, q).
+__global__ void cp_prepass_kernel(const float4* __restrict__ in, float4* __restrict__ out, int n, float z0) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) {
+    float4 a = in[i];
+    const float dz = __fsub_rn(a.z, z0);
+    a.z = __fmul_rn(dz, dz);
+    out[i] = a;
+  }
+}
+
+// ============================================================================================
+// FI & FT campaign kernel (replica mode): blockIdx.z = replica.  CTAs that do not hold the
+// faulted thread run the FT body unchanged (additive stores, R18); the faulted CTA runs the
+// per-thread program with the single-kind hook, guarded accesses (R16) and the watchdog (R17).
+// ============================================================================================
+enum CPKind : int {
+  CK_NL = 0, CK_LIVE, CK_ATOMID, CK_AX, CK_AY, CK_AZ, CK_AW, CK_DY, CK_DYZ2, CK_DX0, CK_DXJ, CK_R2, CK_S, CK_E, CK_IT,
+  CK_COUNT
+};
+
+struct CPFIParams {
+  CPParams base;       // grid/cb point at replica 0; per replica strides below
+  const FaultRec* faults;
+  int64_t grid_elems;  // replica stride (>= nx * ny)
+  float* grid0;
+  hk_control* cb0;
+};
+
+template <int KIND, int U, bool EXACT>
+__device__ void cp_fi_thread(const CPParams& p, const FaultRec& f, float* grid, hk_control* cb) {
+  const int BX = blockDim.x, BY = blockDim.y;
+  const int tx = threadIdx.x, ty = threadIdx.y;
+  const int bxi = blockIdx.x, byi = blockIdx.y;
+  const int64_t t = ((int64_t)byi * gridDim.x + bxi) * (BX * BY) + ty * BX + tx;
+  const bool mine = (t == f.thread);
+  const int64_t inst = mine ? f.inst : -1;
+  const uint64_t mask = f.mask;
+  const int site = f.site, sub = f.sub;
+  const uint32_t z = p.z;
+  const int64_t n_atoms = p.numatoms;
+  const int64_t n_grid = (int64_t)gridDim.x * BX * U * gridDim.y * BY;
+  const uint64_t grid_real = (uint64_t)(uintptr_t)grid, atoms_real = (uint64_t)(uintptr_t)p.atoms;
+  uint32_t chk = 0, alarm = 0, fail = 0, margin = 0xffffffffu;
+  bool applied = false;
+
+  int32_t numatoms = p.numatoms;
+  float h = p.h;
+  uint64_t pgrid = grid_real, patoms = atoms_real;
+  chk ^= (uint32_t)numatoms ^ fb(h) ^ lohi(pgrid) ^ lohi(patoms);
+
+  const bool nl = (KIND == CK_NL) && mine;
+#define NLF(v, s) do { const bool _n = nl && site == (s); applied |= _n; v = flip_i(v, _n, mask); } while (0)
+#define NLFF(v, s) do { const bool _n = nl && site == (s); applied |= _n; v = flip_f(v, _n, mask); } while (0)
+  int32_t xindex = bxi * (BX * U) + tx;
+  NLF(xindex, 0);
+  chk ^= (uint32_t)xindex; alarm |= ((int32_t)((bxi ^ z) * (BX * U) + (tx ^ z)) != xindex) ? AL_DUP : 0u;
+  int32_t yindex = byi * BY + ty;
+  NLF(yindex, 1);
+  chk ^= (uint32_t)yindex; alarm |= ((int32_t)((byi ^ z) * BY + (ty ^ z)) != yindex) ? AL_DUP : 0u;
+  const int32_t nx = gridDim.x * BX * U;
+  int32_t outaddr = (int32_t)((uint32_t)nx * (uint32_t)yindex + (uint32_t)xindex);
+  NLF(outaddr, 2);
+  chk ^= (uint32_t)outaddr;
+  alarm |= ((int32_t)((uint32_t)nx * (uint32_t)opq(yindex, z) + (uint32_t)opq(xindex, z)) != outaddr) ? AL_DUP : 0u;
+  float coorx = __fmul_rn(h, (float)xindex);
+  NLFF(coorx, 3);
+  chk ^= fb(coorx); alarm |= (fb(__fmul_rn(bf(fb(h) + z), (float)opq(xindex, z))) != fb(coorx)) ? AL_DUP : 0u;
+  float coory = __fmul_rn(h, (float)yindex);
+  NLFF(coory, 4);
+  chk ^= fb(coory); alarm |= (fb(__fmul_rn(bf(fb(h) + z), (float)opq(yindex, z))) != fb(coory)) ? AL_DUP : 0u;
+  float gu = __fmul_rn(h, (float)BX);
+  NLFF(gu, 5);
+  chk ^= fb(gu); alarm |= (fb(__fmul_rn(bf(fb(h) + z), (float)opq(BX, z))) != fb(gu)) ? AL_DUP : 0u;
+  chk ^= (uint32_t)opq(xindex, z); chk ^= (uint32_t)opq(yindex, z);
+#undef NLF
+#undef NLFF
+
+  float E[U];
+#pragma unroll
+  for (int j = 0; j < U; ++j) E[j] = 0.0f;
+  int32_t it = 0;
+  int32_t atomid = 0;
+  const int64_t limit = 10 * (n_atoms > 1 ? n_atoms : 1);
+  for (int64_t i = 0;; ++i) {
+    const bool now = (i == inst);
+    if (KIND == CK_ATOMID) { applied |= now; atomid = flip_i(atomid, now, mask); }
+    if (KIND == CK_LIVE && now) {
+      applied = true;
+      switch (site) {
+        case 6: outaddr = flip_i(outaddr, true, mask); break;
+        case 7: coorx = flip_f(coorx, true, mask); break;
+        case 8: coory = flip_f(coory, true, mask); break;
+        case 9: gu = flip_f(gu, true, mask); break;
+        case 10: numatoms = flip_i(numatoms, true, mask); break;
+        case 11: h = flip_f(h, true, mask); break;
+        case 12: pgrid = flip_p(pgrid, true, mask); break;
+        case 13: patoms = flip_p(patoms, true, mask); break;
+        default: break;
+      }
+    }
+    if (!(atomid < numatoms)) break;
+    if (i >= limit) { fail |= FL_HANG; goto done; }
+    int64_t e;
+    if (!guard(patoms, atoms_real, atomid, 16, n_atoms, &e)) { fail |= FL_CRASH; goto done; }
+    {
+      float4 at = __ldg(p.atoms + e);
+      if (KIND == CK_AX) { applied |= now; at.x = flip_f(at.x, now, mask); }
+      if (KIND == CK_AY) { applied |= now; at.y = flip_f(at.y, now, mask); }
+      if (KIND == CK_AZ) { applied |= now; at.z = flip_f(at.z, now, mask); }
+      if (KIND == CK_AW) { applied |= now; at.w = flip_f(at.w, now, mask); }
+      float dy = __fsub_rn(coory, at.y);
+      if (KIND == CK_DY) { applied |= now; dy = flip_f(dy, now, mask); }
+      float dyz2 = __fmaf_rn(dy, dy, at.z);
+      if (KIND == CK_DYZ2) { applied |= now; dyz2 = flip_f(dyz2, now, mask); }
+      float dx = __fsub_rn(coorx, at.x);
+      if (KIND == CK_DX0) { applied |= now; dx = flip_f(dx, now, mask); }
+#pragma unroll
+      for (int j = 0; j < U; ++j) {
+        const bool nj = now && (j == sub);
+        if (j) {
+          dx = __fadd_rn(dx, gu);
+          if (KIND == CK_DXJ) { applied |= nj; dx = flip_f(dx, nj, mask); }
+        }
+        float r2 = __fmaf_rn(dx, dx, dyz2);
+        if (KIND == CK_R2) { applied |= nj; r2 = flip_f(r2, nj, mask); }
+        float s = hk_rsqrt<EXACT>(r2);
+        if (KIND == CK_S) { applied |= nj; s = flip_f(s, nj, mask); }
+        E[j] = __fmaf_rn(at.w, s, E[j]);
+        if (KIND == CK_E) { applied |= nj; E[j] = flip_f(E[j], nj, mask); }
+      }
+    }
+    it = count_inc(it, p.one);
+    if (KIND == CK_IT) { applied |= now; it = flip_i(it, now, mask); }
+    atomid = (int32_t)((uint32_t)atomid + 1u);
+  }
+  if (it != numatoms) alarm |= AL_COUNT;
+  if (it != 0) {
+    const float fit = (float)it;
+#pragma unroll
+    for (int d = 0; d < U; ++d) {
+      if (d < p.ndet && p.R.n[d] > 0) {
+        const float v = __fdiv_rn(E[U - 1 - d], fit);
+        if (!in_range<true>(p.R, d, v, &margin)) { alarm |= AL_RANGE; record_outlier(cb, d, v); }
+      }
+    }
+  }
+  chk ^= opqf(coorx, z); chk ^= opqf(coory, z); chk ^= opqf(gu, z);
+#pragma unroll
+  for (int j = 0; j < U; ++j) {
+    int64_t e;
+    if (!guard(pgrid, grid_real, outaddr + j * BX, 4, n_grid, &e)) { fail |= FL_CRASH; goto done; }
+    atomicAdd(grid + e, E[j]);
+  }
+  chk ^= (uint32_t)opq(outaddr, z);
+  chk ^= ((uint32_t)numatoms + z) ^ (fb(h) + z) ^ (lohi(pgrid) + z) ^ (lohi(patoms) + z);
+  if (chk != 0) alarm |= AL_CHK;
+done:
+  if (fail) atomicOr(&cb->fail, fail);
+  if (mine) {
+    cb->fault_applied = applied ? 1u : 0u;
+    cb->check_margin = margin;
+  }
+  fold_alarm(cb, alarm, (uint32_t)t);
+}
+
+template <int KIND, int U, bool EXACT>
+__global__ void __launch_bounds__(256) cp_fi_kernel(const CPFIParams q) {
+  __shared__ __align__(128) float4 tile[2][CP_TILE];
+  __shared__ __align__(8) uint64_t bar[2];
+  const int r = blockIdx.z;
+  const FaultRec f = q.faults[r];
+  CPParams p = q.base;
+  p.grid = q.grid0 + (int64_t)r * q.grid_elems;
+  p.cb = q.cb0 + r;
+  const int64_t tpb = (int64_t)blockDim.x * blockDim.y;
+  const int64_t cta = (int64_t)blockIdx.y * gridDim.x + blockIdx.x;
+  if (f.thread / tpb != cta) {
+    cp_body<V_NL | V_L, U, EXACT, true>(p, tile, bar);
+  } else {
+    cp_fi_thread<KIND, U, EXACT>(p, f, p.grid, p.cb);
+  }
+}
+
+// ============================================================================================
+// Host launchers
+// ============================================================================================
+template <int V, int U, bool EXACT>
+static cudaError_t launch_cp_v(const CPParams& p, dim3 grid, dim3 block, cudaStream_t s) {
+  cp_kernel<V, U, EXACT><<<grid, block, 0, s>>>(p);
+  count_launch();
+  return cudaGetLastError();
+}
+
+template <int U, bool EXACT>
+static cudaError_t launch_cp_u(int v, const CPParams& p, dim3 grid, dim3 block, cudaStream_t s) {
+  switch (v) {
+    case 0: return launch_cp_v<0, U, EXACT>(p, grid, block, s);
+    case V_NL | V_L: return launch_cp_v<V_NL | V_L, U, EXACT>(p, grid, block, s);
+    case V_NL: return launch_cp_v<V_NL, U, EXACT>(p, grid, block, s);
+    case V_L: return launch_cp_v<V_L, U, EXACT>(p, grid, block, s);
+    case V_PROF: return launch_cp_v<V_PROF, U, EXACT>(p, grid, block, s);
+  }
+  return cudaErrorInvalidValue;
+}
+
+cudaError_t cp_launch(int vflags, const hk_cp_args& a, const DevRanges& R, int ndet, hk_control* cb, float* samples,
+                      cudaStream_t s) {
+  if (a.n_atoms > 0) {
+    cp_prepass_kernel<<<(a.n_atoms + 255) / 256, 256, 0, s>>>(reinterpret_cast<const float4*>(a.atoms),
+                                                               reinterpret_cast<float4*>(a.atoms_ws), a.n_atoms, a.z0);
+    count_launch();
+  }
+  CPParams p{};
+  p.atoms = reinterpret_cast<const float4*>(a.atoms_ws);
+  p.grid = a.grid;
+  p.cb = cb;
+  p.samples = samples;
+  p.R = R;
+  p.numatoms = a.n_atoms;
+  p.h = a.h;
+  p.ndet = ndet;
+  p.z = opaque_zero();
+  p.one = 1 + (int32_t)opaque_zero();
+  p.nthreads = (int64_t)(a.nx / a.unroll) * a.ny;
+  dim3 block(a.bx, a.by), grid(a.nx / (a.bx * a.unroll), a.ny / a.by);
+  const bool ex = a.exact != 0;
+  switch (a.unroll) {
+    case 1: return ex ? launch_cp_u<1, true>(vflags, p, grid, block, s) : launch_cp_u<1, false>(vflags, p, grid, block, s);
+    case 2: return ex ? launch_cp_u<2, true>(vflags, p, grid, block, s) : launch_cp_u<2, false>(vflags, p, grid, block, s);
+    case 4: return ex ? launch_cp_u<4, true>(vflags, p, grid, block, s) : launch_cp_u<4, false>(vflags, p, grid, block, s);
+    case 8: return ex ? launch_cp_u<8, true>(vflags, p, grid, block, s) : launch_cp_u<8, false>(vflags, p, grid, block, s);
+  }
+  return cudaErrorInvalidValue;
+}
+
+// site -> (kind, sub) for U = 4 (DESIGN §3.2 catalogue)
+int cp_site_kind(int site, int U, int* sub) {
+  *sub = 0;
+  if (site <= 5) return CK_NL;
+  if (site <= 13) return CK_LIVE;
+  if (site <= 21) return CK_ATOMID + (site - 14);
+  const int S_DX = 22, S_R2 = 22 + (U - 1), S_S = S_R2 + U, S_E = S_S + U, S_IT = S_E + U;
+  if (site < S_R2) { *sub = site - S_DX + 1; return CK_DXJ; }
+  if (site < S_S) { *sub = site - S_R2; return CK_R2; }
+  if (site < S_E) { *sub = site - S_S; return CK_S; }
+  if (site < S_IT) { *sub = site - S_E; return CK_E; }
+  return CK_IT;
+}
+
+template <int KIND, bool EXACT>
+static cudaError_t launch_cp_fi_k(const CPFIParams& q, dim3 grid, dim3 block, cudaStream_t s) {
+  cp_fi_kernel<KIND, 4, EXACT><<<grid, block, 0, s>>>(q);
+  count_launch();
+  return cudaGetLastError();
+}
+
+template <bool EXACT>
+static cudaError_t launch_cp_fi_e(int kind, const CPFIParams& q, dim3 grid, dim3 block, cudaStream_t s) {
+  switch (kind) {
+#define K(k) case k: return launch_cp_fi_k<k, EXACT>(q, grid, block, s);
+    K(CK_NL) K(CK_LIVE) K(CK_ATOMID) K(CK_AX) K(CK_AY) K(CK_AZ) K(CK_AW) K(CK_DY) K(CK_DYZ2) K(CK_DX0)
+    K(CK_DXJ) K(CK_R2) K(CK_S) K(CK_E) K(CK_IT)
+#undef K
+  }
+  return cudaErrorInvalidValue;
+}
+
+// One batch of `nrep` replicas of one kind: faults[0..nrep), outputs grid0[r], control blocks cb0[r].
+cudaError_t cp_fi_launch(int kind, const hk_cp_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
+                         float* grid0, int64_t stride, hk_control* cb0, cudaStream_t s) {
+  CPFIParams q{};
+  q.base.atoms = reinterpret_cast<const float4*>(a.atoms_ws);
+  q.base.R = R;
+  q.base.numatoms = a.n_atoms;
+  q.base.h = a.h;
+  q.base.ndet = ndet;
+  q.base.z = opaque_zero();
+  q.base.one = 1 + (int32_t)opaque_zero();
+  q.base.nthreads = (int64_t)(a.nx / a.unroll) * a.ny;
+  q.faults = faults;
+  q.grid_elems = stride;
+  q.grid0 = grid0;
+  q.cb0 = cb0;
+  dim3 block(a.bx, a.by), grid(a.nx / (a.bx * 4), a.ny / a.by, nrep);
+  return a.exact ? launch_cp_fi_e<true>(kind, q, grid, block, s) : launch_cp_fi_e<false>(kind, q, grid, block, s);
+}
+
+cudaError_t cp_prepass_launch(const hk_cp_args& a, cudaStream_t s) {
+  if (a.n_atoms <= 0) return cudaSuccess;
+  cp_prepass_kernel<<<(a.n_atoms + 255) / 256, 256, 0, s>>>(reinterpret_cast<const float4*>(a.atoms),
+                                                             reinterpret_cast<float4*>(a.atoms_ws), a.n_atoms, a.z0);
+  count_launch();
+  return cudaGetLastError();
+}
+
+}  // namespace hk

@@ -1,0 +1,46 @@
+// hk_internal.h — host-side declarations shared by the CUDA translation units of libhauberk.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/hauberk.h"
+#include "hk_common.cuh"
+
+namespace hk {
+
+void count_launch();           // bumps the process-wide launch counter (hauberk_launch_count)
+uint32_t opaque_zero();        // 0, read through a volatile so no compiler can fold it
+
+// kernels of one benchmark run (pre-pass / PhiMag included); vflags = V_NL | V_L | V_PROF bits
+cudaError_t cp_launch(int vflags, const hk_cp_args& a, const DevRanges& R, int ndet, hk_control* cb, float* samples,
+                      cudaStream_t s);
+cudaError_t mriq_launch(int vflags, const hk_mriq_args& a, const DevRanges& R, int ndet, hk_control* cb,
+                        float* samples, cudaStream_t s);
+cudaError_t tpacf_launch(int vflags, const hk_tpacf_args& a, const DevRanges& R, int ndet, hk_control* cb,
+                         float* samples, cudaStream_t s);
+cudaError_t cp_prepass_launch(const hk_cp_args& a, cudaStream_t s);
+cudaError_t mriq_phimag_launch(const hk_mriq_args& a, bool nl, hk_control* cb, cudaStream_t s);
+
+// campaign replicas of one site kind
+int cp_site_kind(int site, int U, int* sub);
+int mriq_site_kind(int site);
+int tpacf_site_kind(int site);
+cudaError_t cp_fi_launch(int kind, const hk_cp_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
+                         float* grid0, int64_t stride, hk_control* cb0, cudaStream_t s);
+cudaError_t mriq_fi_launch(int kind, const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
+                           int nrep, float* out0, int64_t stride, hk_control* cb0, cudaStream_t s);
+cudaError_t tpacf_fi_launch(int kind, const hk_tpacf_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
+                            int nrep, unsigned long long* hist0, hk_control* cb0, cudaStream_t s);
+
+// classify.cu
+cudaError_t control_init_launch(hk_control* cb, int n, cudaStream_t s);
+cudaError_t max_abs_launch(const float* g, int64_t n, float* d_out, cudaStream_t s);
+cudaError_t classify_fp_launch(int bench, float* out0, int64_t elems, const float* golden, const float* d_M,
+                               hk_control* cb0, const FaultRec* faults, int nrep, hk_outcome* records, int64_t first,
+                               int64_t* counts, int64_t* site_counts, cudaStream_t s);
+cudaError_t classify_tpacf_launch(unsigned long long* hist0, int nr, int nb, const unsigned long long* golden,
+                                  hk_control* cb0, const FaultRec* faults, int nrep, hk_outcome* records,
+                                  int64_t first, int64_t* counts, int64_t* site_counts, cudaStream_t s);
+
+}  // namespace hk

@@ -1,0 +1,608 @@
+// host.cpp — the C ABI of libhauberk (include/hauberk.h): argument validation, control blocks,
+// the value-range profiler (DESIGN R8/R9), the injection decode (R14/R15) and
+// the replica-mode campaign driver.  Host C++; every per-element
+// step of the path runs in the CUDA kernels of cp.cu / mriq.cu / tpacf.cu / classify.cu.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cmath>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "hk_internal.h"
+
+namespace hk {
+
+static std::atomic<uint64_t> g_launches{0};
+static volatile uint32_t g_zero = 0;
+void count_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
+uint32_t opaque_zero() { return g_zero; }
+
+static thread_local std::string g_err;
+
+static hk_status cuda_fail(cudaError_t e, const char* where) {
+  g_err = std::string(where) + ": " + cudaGetErrorString(e);
+  return e == cudaErrorMemoryAllocation ? HK_ERR_OOM : HK_ERR_CUDA;
+}
+static hk_status invalid(const char* why) {
+  g_err = why;
+  return HK_ERR_INVALID;
+}
+#define HK_CUDA(call, where)                       \
+  do {                                             \
+    cudaError_t _e = (call);                       \
+    if (_e != cudaSuccess) return cuda_fail(_e, where); \
+  } while (0)
+
+// ---------------------------------------------------------------------------------------------
+// Ranges: hk_ranges (host) -> DevRanges with alpha applied (R11)
+// ---------------------------------------------------------------------------------------------
+static DevRanges dev_ranges(const hk_ranges* r) {
+  DevRanges d{};
+  if (!r) return d;
+  d.n_det = r->n_det;
+  const float a = r->alpha > 0.f ? r->alpha : 1.f;
+  for (int k = 0; k < 8 && k < r->n_det; ++k) {
+    d.n[k] = std::max(0, std::min(3, r->det[k].n));
+    for (int q = 0; q < d.n[k]; ++q) {
+      const float lo = r->det[k].lo[q], hi = r->det[k].hi[q];
+      d.lo[k][q] = lo > 0.f ? lo / a : lo * a;
+      d.hi[k][q] = hi > 0.f ? hi * a : hi / a;
+    }
+  }
+  return d;
+}
+
+static int vflags_of(int variant) {
+  switch (variant) {
+    case HK_BASE: return 0;
+    case HK_FT: return V_NL | V_L;
+    case HK_FT_NL: return V_NL;
+    case HK_FT_L: return V_L;
+    case HK_PROFILE: return V_PROF;
+  }
+  return -1;
+}
+
+// ---------------------------------------------------------------------------------------------
+// Validation and per-benchmark geometry
+// ---------------------------------------------------------------------------------------------
+static bool cp_ok(const hk_cp_args* a) {
+  if (!a || !a->atoms_ws || !a->grid || (a->n_atoms > 0 && !a->atoms)) return false;
+  if (a->n_atoms < 0 || a->nx <= 0 || a->ny <= 0 || a->bx <= 0 || a->by <= 0) return false;
+  if (!(a->unroll == 1 || a->unroll == 2 || a->unroll == 4 || a->unroll == 8)) return false;
+  if (a->bx * a->by > 256 || a->nx % (a->bx * a->unroll) != 0 || a->ny % a->by != 0) return false;
+  if ((a->bx * a->by) % 32 != 0) return false;
+  if (((uintptr_t)a->atoms | (uintptr_t)a->atoms_ws) & 15u) return false;
+  return true;
+}
+static bool mriq_ok(const hk_mriq_args* a) {
+  if (!a || a->n_vox < 0 || a->n_k < 0 || !a->qr || !a->qi) return false;
+  if (a->n_vox > 0 && (!a->x || !a->y || !a->z)) return false;
+  if (a->n_k > 0 && (!a->kx || !a->ky || !a->kz || !a->phi_r || !a->phi_i || !a->kv_ws)) return false;
+  if ((uintptr_t)a->kv_ws & 15u) return false;
+  return true;
+}
+static bool tpacf_ok(const hk_tpacf_args* a) {
+  if (!a || !a->pts || !a->edges || !a->hist) return false;
+  if (a->n <= 0 || a->n_rand < 1 || a->n_bins < 1 || a->n_bins > 30 || a->chunk < 1 || a->chunk > 1024) return false;
+  return true;
+}
+static bool tpacf_edges_ok(const hk_tpacf_args* a, cudaStream_t s) {
+  std::vector<float> e(a->n_bins + 1);
+  if (cudaMemcpyAsync(e.data(), a->edges, sizeof(float) * e.size(), cudaMemcpyDeviceToHost, s) != cudaSuccess) return false;
+  if (cudaStreamSynchronize(s) != cudaSuccess) return false;
+  for (int k = 0; k < a->n_bins; ++k)
+    if (!(e[k] > e[k + 1])) return false;
+  return true;
+}
+
+static int64_t cp_threads(const hk_cp_args* a) { return (int64_t)(a->nx / a->unroll) * a->ny; }
+static int tp_nc(const hk_tpacf_args* a) { return (a->n + a->chunk - 1) / a->chunk; }
+static int64_t tp_threads(const hk_tpacf_args* a) { return (int64_t)(1 + 2 * a->n_rand) * tp_nc(a) * a->n; }
+static int64_t tp_trips(const hk_tpacf_args* a, int64_t g) {
+  const int nC = tp_nc(a), C = a->chunk, N = a->n;
+  const int64_t row = g / N;
+  const int i = (int)(g % N), h = (int)(row / nC), c = (int)(row % nC);
+  int64_t jb = (int64_t)c * C;
+  if (h <= a->n_rand) jb = std::max<int64_t>(jb, i + 1);
+  const int64_t je = std::min<int64_t>((int64_t)(c + 1) * C, N);
+  return je > jb ? je - jb : 0;
+}
+static int64_t bench_threads(int b, const void* args) {
+  if (b == HK_CP) return cp_threads((const hk_cp_args*)args);
+  if (b == HK_MRIQ) return ((const hk_mriq_args*)args)->n_vox;
+  return tp_threads((const hk_tpacf_args*)args);
+}
+
+// ---------------------------------------------------------------------------------------------
+// Runs
+// ---------------------------------------------------------------------------------------------
+static hk_status run_common_checks(int variant, const hk_ranges* ranges, hk_control* d_cb, float* d_samples) {
+  if (vflags_of(variant) < 0) return invalid("unknown variant");
+  if ((variant == HK_FT || variant == HK_FT_L) && (!ranges || ranges->n_det <= 0)) {
+    g_err = "FT variant needs profiled ranges";
+    return HK_ERR_NO_RANGES;
+  }
+  if (variant != HK_BASE && !d_cb) return invalid("control block required");
+  if (variant == HK_PROFILE && !d_samples) return invalid("PROFILE needs d_samples");
+  if (ranges && (ranges->n_det < 0 || ranges->n_det > 8)) return invalid("n_det out of range");
+  return HK_OK;
+}
+
+static hk_status run_bench(int b, const void* args, int variant, const hk_ranges* ranges, hk_control* d_cb,
+                           float* d_samples, cudaStream_t s) {
+  const int vf = vflags_of(variant);
+  const DevRanges R = dev_ranges(ranges);
+  int ndet = ranges ? ranges->n_det : 1;
+  if (d_cb) HK_CUDA(control_init_launch(d_cb, 1, s), "control init");
+  if (b == HK_CP) {
+    const hk_cp_args* a = (const hk_cp_args*)args;
+    ndet = std::min(ndet, a->unroll);
+    HK_CUDA(cudaMemsetAsync(a->grid, 0, sizeof(float) * (size_t)a->nx * a->ny, s), "memset grid");
+    HK_CUDA(cp_launch(vf, *a, R, ndet, d_cb, d_samples, s), "cp kernel");
+  } else if (b == HK_MRIQ) {
+    const hk_mriq_args* a = (const hk_mriq_args*)args;
+    ndet = std::min(ndet, 2);
+    HK_CUDA(cudaMemsetAsync(a->qr, 0, sizeof(float) * (size_t)a->n_vox, s), "memset qr");
+    HK_CUDA(cudaMemsetAsync(a->qi, 0, sizeof(float) * (size_t)a->n_vox, s), "memset qi");
+    HK_CUDA(mriq_launch(vf, *a, R, ndet, d_cb, d_samples, s), "mriq kernels");
+  } else {
+    const hk_tpacf_args* a = (const hk_tpacf_args*)args;
+    ndet = std::min(ndet, 1);
+    HK_CUDA(cudaMemsetAsync(a->hist, 0, sizeof(unsigned long long) * (size_t)(1 + 2 * a->n_rand) * (a->n_bins + 2), s),
+            "memset hist");
+    HK_CUDA(tpacf_launch(vf, *a, R, ndet, d_cb, d_samples, s), "tpacf kernel");
+  }
+  return HK_OK;
+}
+
+// ---------------------------------------------------------------------------------------------
+// Value-range profiler (L1489-1508; R8 value-space size, R9 threshold walk)
+// ---------------------------------------------------------------------------------------------
+static int64_t ord_of(float x) {
+  uint32_t b;
+  std::memcpy(&b, &x, 4);
+  return (b & 0x80000000u) ? -(int64_t)(b & 0x7fffffffu) : (int64_t)b;
+}
+static float threshold(int k) {
+  char buf[16];
+  std::snprintf(buf, sizeof buf, "1e%d", k);
+  return std::strtof(buf, nullptr);
+}
+struct Classes {
+  int n = 0;
+  float lo[3], hi[3];
+  int64_t cost = 0;
+};
+static Classes classes_at(const std::vector<float>& v, float T) {
+  bool have[3] = {false, false, false};
+  float mn[3] = {0, 0, 0}, mx[3] = {0, 0, 0};
+  for (float x : v) {
+    const int c = x < -T ? 0 : (x > T ? 2 : 1);
+    if (!have[c]) { have[c] = true; mn[c] = mx[c] = x; }
+    else { mn[c] = std::min(mn[c], x); mx[c] = std::max(mx[c], x); }
+  }
+  Classes r;
+  for (int c = 0; c < 3; ++c)
+    if (have[c]) {
+      r.lo[r.n] = mn[c]; r.hi[r.n] = mx[c]; r.n++;
+      r.cost += ord_of(mx[c]) - ord_of(mn[c]) + 1;
+    }
+  return r;
+}
+static hk_range_set profile_search(const std::vector<float>& v, int t0) {
+  hk_range_set out{};
+  out.t_exp10 = t0;
+  if (v.empty()) return out;
+  int k = t0;
+  const int64_t INF = INT64_MAX;
+  for (;;) {
+    const int64_t c0 = classes_at(v, threshold(k)).cost;
+    const int64_t cm = k - 1 >= -38 ? classes_at(v, threshold(k - 1)).cost : INF;
+    const int64_t cp = k + 1 <= 38 ? classes_at(v, threshold(k + 1)).cost : INF;
+    if (!(cp < c0 || cm < c0)) break;
+    k = (cp <= cm) ? k + 1 : k - 1;
+  }
+  const Classes r = classes_at(v, threshold(k));
+  out.n = r.n;
+  for (int q = 0; q < r.n; ++q) { out.lo[q] = r.lo[q]; out.hi[q] = r.hi[q]; }
+  out.t_exp10 = k;
+  return out;
+}
+
+// ---------------------------------------------------------------------------------------------
+// Site catalogue and decode (R14, R15)
+// ---------------------------------------------------------------------------------------------
+static int num_sites(int b, int unroll) { return b == HK_CP ? 22 + 4 * unroll : (b == HK_MRIQ ? 29 : 31); }
+static bool site_is_nl(int b, int s) { return b == HK_CP ? s <= 5 : (b == HK_MRIQ ? s <= 3 : s <= 11); }
+static int site_width(int b, int s) {
+  if (b == HK_CP) return (s == 12 || s == 13) ? 64 : 32;
+  if (b == HK_MRIQ) return (s >= 9 && s <= 14) ? 64 : 32;
+  return (s == 20 || s == 21) ? 64 : 32;
+}
+static uint64_t splitmix(uint64_t seed, uint64_t m) {
+  uint64_t z = seed + (m + 1) * 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+static uint64_t below(uint64_t r, uint64_t m) { return (uint64_t)(((unsigned __int128)r * m) >> 64); }
+
+struct Catalog {
+  int bench = -1, unroll = 1;
+  std::vector<int> enabled;
+  int64_t nthr = 0, uniform_trips = 0, total_trips = 0;
+  std::vector<int64_t> prefix;  // TPACF: prefix[g] = trips of threads < g
+};
+
+static bool build_catalog(Catalog& K, int b, const void* args, uint64_t mask) {
+  K.bench = b;
+  if (b == HK_CP) {
+    const hk_cp_args* a = (const hk_cp_args*)args;
+    K.unroll = a->unroll;
+    K.nthr = cp_threads(a);
+    K.uniform_trips = a->n_atoms;
+    K.total_trips = K.nthr * K.uniform_trips;
+  } else if (b == HK_MRIQ) {
+    const hk_mriq_args* a = (const hk_mriq_args*)args;
+    K.nthr = a->n_vox;
+    K.uniform_trips = a->n_k;
+    K.total_trips = K.nthr * K.uniform_trips;
+  } else {
+    const hk_tpacf_args* a = (const hk_tpacf_args*)args;
+    K.nthr = tp_threads(a);
+    K.prefix.resize(K.nthr + 1);
+    K.prefix[0] = 0;
+    for (int64_t g = 0; g < K.nthr; ++g) K.prefix[g + 1] = K.prefix[g] + tp_trips(a, g);
+    K.total_trips = K.prefix[K.nthr];
+  }
+  for (int s = 0; s < num_sites(b, K.unroll) && s < 64; ++s) {
+    if (!((mask >> s) & 1ull)) continue;
+    const int64_t D = site_is_nl(b, s) ? K.nthr : K.total_trips;
+    if (D > 0) K.enabled.push_back(s);
+  }
+  return !K.enabled.empty();
+}
+
+static hk_fault decode_one(const Catalog& K, uint64_t seed, int64_t n) {
+  hk_fault f{};
+  const uint64_t r1 = splitmix(seed, 8 * (uint64_t)n + 1);
+  const uint64_t r2 = splitmix(seed, 8 * (uint64_t)n + 2);
+  const uint64_t r3 = splitmix(seed, 8 * (uint64_t)n + 3);
+  const int s = K.enabled[below(r1, K.enabled.size())];
+  f.site = s;
+  if (site_is_nl(K.bench, s)) {
+    f.thread = (int64_t)below(r2, (uint64_t)K.nthr);
+    f.inst = 0;
+  } else {
+    const int64_t u = (int64_t)below(r2, (uint64_t)K.total_trips);
+    if (K.prefix.empty()) {
+      f.thread = u / K.uniform_trips;
+      f.inst = u % K.uniform_trips;
+    } else {
+      // first g with prefix[g + 1] > u
+      const int64_t g = (int64_t)(std::upper_bound(K.prefix.begin(), K.prefix.end(), u) - K.prefix.begin()) - 1;
+      f.thread = g;
+      f.inst = u - K.prefix[g];
+    }
+  }
+  f.mask = 1ull << below(r3, (uint64_t)site_width(K.bench, s));
+  return f;
+}
+
+static bool args_ok(int b, const void* a) {
+  if (!a) return false;
+  return b == HK_CP ? cp_ok((const hk_cp_args*)a) : (b == HK_MRIQ ? mriq_ok((const hk_mriq_args*)a) : tpacf_ok((const hk_tpacf_args*)a));
+}
+
+// ---------------------------------------------------------------------------------------------
+// Campaign workspace per benchmark
+// ---------------------------------------------------------------------------------------------
+struct BenchWS {
+  bool used = false;
+  const void* args = nullptr;
+  DevRanges R{};
+  int ndet = 1;
+  int64_t out_elems = 0;   // floats (CP/MRI-Q) or u64 (TPACF) per replica
+  void* golden = nullptr;
+  float* dM = nullptr;
+  void* rep_out = nullptr;
+  hk_control* rep_cb = nullptr;
+  hk_control* gold_cb = nullptr;
+  int batch = 0;
+};
+
+static int default_batch(int b, const void* args) {
+  if (b == HK_CP) {
+    const hk_cp_args* a = (const hk_cp_args*)args;
+    const int64_t ctas = (int64_t)(a->nx / (a->bx * a->unroll)) * (a->ny / a->by);
+    return (int)std::max<int64_t>(64, std::min<int64_t>(4096, (148 * 8 * 4) / std::max<int64_t>(ctas, 1)));
+  }
+  if (b == HK_MRIQ) return 256;
+  return 64;
+}
+
+}  // namespace hk
+
+using namespace hk;
+
+extern "C" {
+
+const char* hauberk_strerror(hk_status s) {
+  switch (s) {
+    case HK_OK: return "ok";
+    case HK_ERR_INVALID: return "invalid argument";
+    case HK_ERR_CUDA: return "CUDA error";
+    case HK_ERR_NO_RANGES: return "FT variant without profiled ranges";
+    case HK_ERR_OOM: return "out of device memory";
+    case HK_ERR_UNSUPPORTED: return "unsupported shape or variant";
+    case HK_ERR_PROFILE_NAN: return "profile sample is NaN/Inf";
+    case HK_ERR_GOLDEN_ALARM: return "fault-free golden run raised an alarm";
+  }
+  return "unknown status";
+}
+const char* hauberk_last_error(void) { return g_err.c_str(); }
+int32_t hauberk_version(void) { return HK_ABI_VERSION; }
+uint64_t hauberk_launch_count(void) { return g_launches.load(); }
+int32_t hauberk_num_sites(int32_t bench, int32_t unroll) {
+  if (bench < 0 || bench > 2) return 0;
+  return num_sites(bench, unroll);
+}
+
+hk_status hauberk_run_cp(const hk_cp_args* args, int32_t variant, const hk_ranges* ranges, hk_control* d_cb,
+                         float* d_samples, void* stream) {
+  if (!cp_ok(args)) return invalid("hk_cp_args invalid (shape, alignment or null pointer)");
+  hk_status st = run_common_checks(variant, ranges, d_cb, d_samples);
+  if (st != HK_OK) return st;
+  return run_bench(HK_CP, args, variant, ranges, d_cb, d_samples, (cudaStream_t)stream);
+}
+
+hk_status hauberk_run_mriq(const hk_mriq_args* args, int32_t variant, const hk_ranges* ranges, hk_control* d_cb,
+                           float* d_samples, void* stream) {
+  if (!mriq_ok(args)) return invalid("hk_mriq_args invalid");
+  hk_status st = run_common_checks(variant, ranges, d_cb, d_samples);
+  if (st != HK_OK) return st;
+  return run_bench(HK_MRIQ, args, variant, ranges, d_cb, d_samples, (cudaStream_t)stream);
+}
+
+hk_status hauberk_run_tpacf(const hk_tpacf_args* args, int32_t variant, const hk_ranges* ranges, hk_control* d_cb,
+                            float* d_samples, void* stream) {
+  if (!tpacf_ok(args)) return invalid("hk_tpacf_args invalid");
+  hk_status st = run_common_checks(variant, ranges, d_cb, d_samples);
+  if (st != HK_OK) return st;
+  return run_bench(HK_TPACF, args, variant, ranges, d_cb, d_samples, (cudaStream_t)stream);
+}
+
+hk_status hauberk_profile_ranges(int32_t bench, const void* args, const hk_profile_opts* opts, hk_ranges* out,
+                                 void* stream) {
+  if (bench < 0 || bench > 2 || !out || !args_ok(bench, args)) return invalid("profile: bad bench/args");
+  cudaStream_t s = (cudaStream_t)stream;
+  const int maxvar = opts ? opts->maxvar : 1;
+  const int t0 = opts ? opts->t0_exp10 : -5;
+  const float alpha = opts ? opts->alpha : 1.f;
+  const int cap = bench == HK_CP ? ((const hk_cp_args*)args)->unroll : (bench == HK_MRIQ ? 2 : 1);
+  if (maxvar < 1 || maxvar > cap || t0 < -38 || t0 > 38 || !(alpha >= 1.f)) return invalid("profile: bad options");
+  if (bench == HK_TPACF && !tpacf_edges_ok((const hk_tpacf_args*)args, s)) return invalid("edges must strictly decrease");
+  const int64_t T = bench_threads(bench, args);
+  float* d_samples = nullptr;
+  hk_control* d_cb = nullptr;
+  HK_CUDA(cudaMallocAsync((void**)&d_samples, sizeof(float) * std::max<int64_t>(1, T * maxvar), s), "alloc samples");
+  HK_CUDA(cudaMallocAsync((void**)&d_cb, sizeof(hk_control), s), "alloc cb");
+  hk_ranges pr{};
+  pr.n_det = maxvar;
+  pr.alpha = 1.f;
+  hk_status st = run_bench(bench, args, HK_PROFILE, &pr, d_cb, d_samples, s);
+  std::vector<float> h((size_t)(T * maxvar));
+  if (st == HK_OK && T > 0) {
+    cudaError_t e = cudaMemcpyAsync(h.data(), d_samples, sizeof(float) * h.size(), cudaMemcpyDeviceToHost, s);
+    if (e != cudaSuccess) st = cuda_fail(e, "copy samples");
+  }
+  cudaFreeAsync(d_samples, s);
+  cudaFreeAsync(d_cb, s);
+  cudaError_t e = cudaStreamSynchronize(s);
+  if (st != HK_OK) return st;
+  if (e != cudaSuccess) return cuda_fail(e, "profile run");
+  std::memset(out, 0, sizeof(*out));
+  out->n_det = maxvar;
+  out->alpha = alpha;
+  std::vector<unsigned char> valid((size_t)T, 1);
+  if (bench == HK_TPACF)
+    for (int64_t g = 0; g < T; ++g) valid[g] = tp_trips((const hk_tpacf_args*)args, g) > 0;
+  else if ((bench == HK_CP && ((const hk_cp_args*)args)->n_atoms == 0) || (bench == HK_MRIQ && ((const hk_mriq_args*)args)->n_k == 0))
+    std::fill(valid.begin(), valid.end(), 0);
+  for (int d = 0; d < maxvar; ++d) {
+    std::vector<float> v;
+    v.reserve((size_t)T);
+    for (int64_t t = 0; t < T; ++t) {
+      if (!valid[t]) continue;
+      const float x = h[(size_t)(d * T + t)];
+      if (!std::isfinite(x)) { g_err = "profile sample NaN/Inf"; return HK_ERR_PROFILE_NAN; }
+      v.push_back(x);
+    }
+    out->det[d] = profile_search(v, t0);
+  }
+  return HK_OK;
+}
+
+hk_status hauberk_decode(int32_t bench_mode, const void* const args[3], const uint64_t site_mask[3], uint64_t seed,
+                         int64_t first, int64_t count, int32_t* bench_out, hk_fault* out) {
+  if (!args || !site_mask || !bench_out || !out || count < 0 || first < 0 || bench_mode < -1 || bench_mode > 2)
+    return invalid("decode: bad arguments");
+  Catalog K[3];
+  bool have[3] = {false, false, false};
+  for (int64_t q = 0; q < count; ++q) {
+    const int64_t n = first + q;
+    const int b = bench_mode >= 0 ? bench_mode : (int)(n % 3);
+    if (!have[b]) {
+      if (!args_ok(b, args[b])) return invalid("decode: args of a used benchmark are invalid");
+      if (!build_catalog(K[b], b, args[b], site_mask[b])) return invalid("decode: empty site catalogue");
+      have[b] = true;
+    }
+    bench_out[q] = b;
+    out[q] = decode_one(K[b], seed, n);
+  }
+  return HK_OK;
+}
+
+hk_status hauberk_inject_campaign(int32_t bench_mode, const void* const args[3], const hk_ranges* const ranges[3],
+                                  const hk_campaign* C, hk_outcome* d_records, int64_t* d_counts, int64_t* d_site_counts,
+                                  void* stream) {
+  if (!args || !ranges || !C || !d_counts || bench_mode < -1 || bench_mode > 2) return invalid("campaign: bad arguments");
+  if (C->count < 0 || C->first < 0) return invalid("campaign: bad index range");
+  if (C->mode != 0) { g_err = "only replica mode (0) is implemented on the GPU"; return HK_ERR_UNSUPPORTED; }
+  if (C->nbits != 0 && C->nbits != 1) { g_err = "multi-bit masks are NEXT (f1)"; return HK_ERR_UNSUPPORTED; }
+  if (C->count == 0) return HK_OK;
+  cudaStream_t s = (cudaStream_t)stream;
+  BenchWS W[3];
+  Catalog K[3];
+  for (int b = 0; b < 3; ++b) {
+    const bool used = bench_mode == b || (bench_mode == -1 && C->count > (b - C->first % 3 + 3) % 3);
+    if (!used) continue;
+    if (!args_ok(b, args[b])) return invalid("campaign: args of a used benchmark are invalid");
+    if (!ranges[b] || ranges[b]->n_det <= 0) { g_err = "campaign: ranges missing"; return HK_ERR_NO_RANGES; }
+    if (b == HK_CP && ((const hk_cp_args*)args[b])->unroll != 4) { g_err = "campaign kernels are built for CP unroll 4"; return HK_ERR_UNSUPPORTED; }
+    if (b == HK_TPACF && !tpacf_edges_ok((const hk_tpacf_args*)args[b], s)) return invalid("edges must strictly decrease");
+    if (!build_catalog(K[b], b, args[b], C->site_mask[b])) return invalid("campaign: empty site catalogue");
+    W[b].used = true;
+    W[b].args = args[b];
+    W[b].R = dev_ranges(ranges[b]);
+    W[b].ndet = ranges[b]->n_det;
+    W[b].batch = C->batch > 0 ? C->batch : default_batch(b, args[b]);
+  }
+
+  // ---- golden (fault-free FT) runs; their outputs stay in the caller's buffers' copies
+  auto cleanup = [&]() {
+    for (int b = 0; b < 3; ++b) {
+      if (W[b].golden) cudaFreeAsync(W[b].golden, s);
+      if (W[b].dM) cudaFreeAsync(W[b].dM, s);
+      if (W[b].rep_out) cudaFreeAsync(W[b].rep_out, s);
+      if (W[b].rep_cb) cudaFreeAsync(W[b].rep_cb, s);
+      if (W[b].gold_cb) cudaFreeAsync(W[b].gold_cb, s);
+    }
+  };
+  hk_status st = HK_OK;
+  for (int b = 0; b < 3 && st == HK_OK; ++b) {
+    if (!W[b].used) continue;
+    BenchWS& w = W[b];
+    size_t esz = sizeof(float);
+    if (b == HK_CP) { const hk_cp_args* a = (const hk_cp_args*)w.args; w.out_elems = (int64_t)a->nx * a->ny; }
+    else if (b == HK_MRIQ) { const hk_mriq_args* a = (const hk_mriq_args*)w.args; w.out_elems = 2LL * a->n_vox; }
+    else { const hk_tpacf_args* a = (const hk_tpacf_args*)w.args; w.out_elems = (int64_t)(1 + 2 * a->n_rand) * (a->n_bins + 2); esz = 8; }
+    const int64_t stride = (w.out_elems + 3) / 4 * 4;  // keep replicas 16-byte aligned
+    w.out_elems = stride;
+    cudaError_t e;
+    if ((e = cudaMallocAsync(&w.golden, esz * stride, s)) != cudaSuccess) { st = cuda_fail(e, "alloc golden"); break; }
+    if ((e = cudaMallocAsync((void**)&w.dM, sizeof(float), s)) != cudaSuccess) { st = cuda_fail(e, "alloc M"); break; }
+    if ((e = cudaMallocAsync((void**)&w.gold_cb, sizeof(hk_control), s)) != cudaSuccess) { st = cuda_fail(e, "alloc cb"); break; }
+    if ((e = cudaMallocAsync(&w.rep_out, esz * stride * w.batch, s)) != cudaSuccess) { st = cuda_fail(e, "alloc replicas"); break; }
+    if ((e = cudaMallocAsync((void**)&w.rep_cb, sizeof(hk_control) * w.batch, s)) != cudaSuccess) { st = cuda_fail(e, "alloc replica cbs"); break; }
+    if ((e = cudaMemsetAsync(w.golden, 0, esz * stride, s)) != cudaSuccess) { st = cuda_fail(e, "memset"); break; }
+    if ((e = cudaMemsetAsync(w.rep_out, 0, esz * stride * w.batch, s)) != cudaSuccess) { st = cuda_fail(e, "memset"); break; }
+    if ((e = control_init_launch(w.rep_cb, w.batch, s)) != cudaSuccess) { st = cuda_fail(e, "cb init"); break; }
+    // golden = this library's own fault-free FT output (R7)
+    if (b == HK_CP) {
+      hk_cp_args a = *(const hk_cp_args*)w.args;
+      a.grid = (float*)w.golden;
+      st = run_bench(b, &a, HK_FT, ranges[b], w.gold_cb, nullptr, s);
+      if (st == HK_OK && (e = max_abs_launch((float*)w.golden, (int64_t)a.nx * a.ny, w.dM, s)) != cudaSuccess) st = cuda_fail(e, "max");
+    } else if (b == HK_MRIQ) {
+      hk_mriq_args a = *(const hk_mriq_args*)w.args;
+      a.qr = (float*)w.golden;
+      a.qi = a.qr + a.n_vox;
+      st = run_bench(b, &a, HK_FT, ranges[b], w.gold_cb, nullptr, s);
+      if (st == HK_OK && (e = max_abs_launch((float*)w.golden, 2LL * a.n_vox, w.dM, s)) != cudaSuccess) st = cuda_fail(e, "max");
+    } else {
+      hk_tpacf_args a = *(const hk_tpacf_args*)w.args;
+      a.hist = (unsigned long long*)w.golden;
+      st = run_bench(b, &a, HK_FT, ranges[b], w.gold_cb, nullptr, s);
+    }
+  }
+  if (st != HK_OK) { cleanup(); return st; }
+  {
+    hk_control hc[3];
+    for (int b = 0; b < 3; ++b)
+      if (W[b].used) cudaMemcpyAsync(&hc[b], W[b].gold_cb, sizeof(hk_control), cudaMemcpyDeviceToHost, s);
+    cudaError_t e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) { cleanup(); return cuda_fail(e, "golden runs"); }
+    for (int b = 0; b < 3; ++b)
+      if (W[b].used && (hc[b].alarm != 0 || hc[b].fail != 0)) {
+        cleanup();
+        g_err = "golden run alarm (ranges were not profiled on this input)";
+        return HK_ERR_GOLDEN_ALARM;
+      }
+  }
+
+  // ---- decode, group by (bench, kind), upload
+  struct Item { int b, kind; FaultRec f; };
+  std::vector<Item> items((size_t)C->count);
+  for (int64_t q = 0; q < C->count; ++q) {
+    const int64_t n = C->first + q;
+    const int b = bench_mode >= 0 ? bench_mode : (int)(n % 3);
+    const hk_fault hf = decode_one(K[b], C->seed, n);
+    Item it{};
+    it.b = b;
+    it.f.index = n; it.f.thread = hf.thread; it.f.inst = hf.inst; it.f.mask = hf.mask; it.f.site = hf.site;
+    int sub = 0;
+    if (b == HK_CP) it.kind = cp_site_kind(hf.site, 4, &sub);
+    else if (b == HK_MRIQ) it.kind = mriq_site_kind(hf.site);
+    else it.kind = tpacf_site_kind(hf.site);
+    it.f.sub = sub;
+    items[(size_t)q] = it;
+  }
+  std::stable_sort(items.begin(), items.end(), [](const Item& x, const Item& y) {
+    return x.b != y.b ? x.b < y.b : x.kind < y.kind;
+  });
+  std::vector<FaultRec> recs(items.size());
+  for (size_t q = 0; q < items.size(); ++q) recs[q] = items[q].f;
+  FaultRec* d_faults = nullptr;
+  cudaError_t e = cudaMallocAsync((void**)&d_faults, sizeof(FaultRec) * recs.size(), s);
+  if (e != cudaSuccess) { cleanup(); return cuda_fail(e, "alloc faults"); }
+  e = cudaMemcpyAsync(d_faults, recs.data(), sizeof(FaultRec) * recs.size(), cudaMemcpyHostToDevice, s);
+  if (e != cudaSuccess) { cudaFreeAsync(d_faults, s); cleanup(); return cuda_fail(e, "upload faults"); }
+
+  // ---- batches: FI&FT replicas, then the classify epilogue (which also recycles the workspace)
+  size_t q = 0;
+  while (q < items.size() && st == HK_OK) {
+    const int b = items[q].b, kind = items[q].kind;
+    size_t end = q;
+    while (end < items.size() && items[end].b == b && items[end].kind == kind && (int)(end - q) < W[b].batch) ++end;
+    const int nrep = (int)(end - q);
+    BenchWS& w = W[b];
+    const FaultRec* fr = d_faults + q;
+    if (b == HK_CP) {
+      const hk_cp_args* a = (const hk_cp_args*)w.args;
+      if ((e = cp_fi_launch(kind, *a, w.R, std::min(w.ndet, 4), fr, nrep, (float*)w.rep_out, w.out_elems, w.rep_cb, s)) != cudaSuccess)
+        st = cuda_fail(e, "cp FI");
+      else if ((e = classify_fp_launch(b, (float*)w.rep_out, w.out_elems, (const float*)w.golden, w.dM, w.rep_cb, fr, nrep,
+                                       d_records, C->first, d_counts, d_site_counts, s)) != cudaSuccess)
+        st = cuda_fail(e, "classify");
+    } else if (b == HK_MRIQ) {
+      const hk_mriq_args* a = (const hk_mriq_args*)w.args;
+      if ((e = mriq_fi_launch(kind, *a, w.R, std::min(w.ndet, 2), fr, nrep, (float*)w.rep_out, w.out_elems, w.rep_cb, s)) != cudaSuccess)
+        st = cuda_fail(e, "mriq FI");
+      else if ((e = classify_fp_launch(b, (float*)w.rep_out, w.out_elems, (const float*)w.golden, w.dM, w.rep_cb, fr, nrep,
+                                       d_records, C->first, d_counts, d_site_counts, s)) != cudaSuccess)
+        st = cuda_fail(e, "classify");
+    } else {
+      const hk_tpacf_args* a = (const hk_tpacf_args*)w.args;
+      if ((e = tpacf_fi_launch(kind, *a, w.R, std::min(w.ndet, 1), fr, nrep, (unsigned long long*)w.rep_out, w.rep_cb, s)) !=
+          cudaSuccess)
+        st = cuda_fail(e, "tpacf FI");
+      else if ((e = classify_tpacf_launch((unsigned long long*)w.rep_out, a->n_rand, a->n_bins,
+                                          (const unsigned long long*)w.golden, w.rep_cb, fr, nrep, d_records, C->first,
+                                          d_counts, d_site_counts, s)) != cudaSuccess)
+        st = cuda_fail(e, "classify");
+    }
+    q = end;
+  }
+  cudaFreeAsync(d_faults, s);
+  cleanup();
+  return st;
+}
+
+}  // extern "C"

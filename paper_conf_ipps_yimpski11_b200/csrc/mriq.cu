@@ -1,0 +1,392 @@
+// mriq.cu — MRI-Q (K2: PhiMag + Q) with HAUBERK detectors, for sm_100a.
+//
+// Abstract programs: DESIGN.md §3.3 (benchmark: Parboil MRI-Q; the paper names it at L503 and
+// reports its value distributions, Fig. 10, and correctness rule, L2598-2603).
+// B200 shape: k-space packed as float4 {kx, ky, kz, |phi|^2} by PhiMag, staged into shared memory
+// with double-buffered 1-D bulk async copies; one voxel per thread; MUFU.SIN + MUFU.COS per pair
+// (the binding pipe); loop detector = self-accumulator Qr (and Qi at maxvar 2) + counter.
+#include "hk_internal.h"
+
+namespace hk {
+
+constexpr int MQ_TILE = 1024;  // k-samples per stage (16 KB)
+constexpr float RINT_MAGIC = 12582912.0f;  // 1.5 * 2^23
+constexpr float TWO_PI_F = 6.28318548202514648f;
+
+struct MQParams {
+  const float *x, *y, *z;
+  const float4* kv;
+  float *qr, *qi;
+  hk_control* cb;
+  float* samples;
+  DevRanges R;
+  int32_t numX, numK, ndet;
+  uint32_t zz;  // runtime 0 (opaque)
+  int32_t one;
+};
+
+// PhiMag (non-loop code: HAUBERK-NL only).  kv[k] = (kx, ky, kz, fmaf(im, im, re*re)).
+template <bool NL>
+__global__ void __launch_bounds__(256) mriq_phimag_kernel(const float* __restrict__ kx, const float* __restrict__ ky,
+                                                         const float* __restrict__ kz, const float* __restrict__ pr,
+                                                         const float* __restrict__ pi, float4* __restrict__ kv, int numK,
+                                                         hk_control* cb, uint32_t z) {
+  const int k = blockIdx.x * blockDim.x + threadIdx.x;
+  uint32_t chk = 0, alarm = 0;
+  if (k < numK) {
+    if (NL) { chk ^= (uint32_t)k; alarm |= ((int)((blockIdx.x ^ z) * blockDim.x + (threadIdx.x ^ z)) != k) ? AL_DUP : 0u; }
+    const float re = pr[k];
+    if (NL) { chk ^= fb(re); alarm |= (fb(pr[opq(k, z)]) != fb(re)) ? AL_DUP : 0u; }
+    const float im = pi[k];
+    if (NL) { chk ^= fb(im); alarm |= (fb(pi[opq(k, z)]) != fb(im)) ? AL_DUP : 0u; }
+    const float pm = __fmaf_rn(im, im, __fmul_rn(re, re));
+    if (NL) {
+      chk ^= fb(pm);
+      const float re2 = bf(fb(re) + z), im2 = bf(fb(im) + z);
+      alarm |= (fb(__fmaf_rn(im2, im2, __fmul_rn(re2, re2))) != fb(pm)) ? AL_DUP : 0u;
+    }
+    kv[k] = make_float4(kx[k], ky[k], kz[k], pm);
+    if (NL) {
+      chk ^= opqf(re, z); chk ^= opqf(im, z); chk ^= opqf(pm, z); chk ^= (uint32_t)opq(k, z);
+      if (chk) alarm |= AL_CHK;
+    }
+  }
+  if (NL) fold_alarm(cb, alarm, (uint32_t)k);
+}
+
+template <int V, bool EXACT, bool ADD>
+__device__ __forceinline__ void mriq_body(const MQParams& p, float4 (*tile)[MQ_TILE], uint64_t* bar) {
+  constexpr bool NL = (V & V_NL) != 0, L = (V & V_L) != 0, PROF = (V & V_PROF) != 0;
+  constexpr bool CNT = L || PROF;
+  const uint32_t z = p.zz;
+  const int32_t xIndex = blockIdx.x * blockDim.x + threadIdx.x;
+  const bool active = xIndex < p.numX;
+  const int32_t numK = p.numK;
+  uint32_t chk = 0, alarm = 0;
+  float sX = 0.f, sY = 0.f, sZ = 0.f;
+  if (active) {
+    if (NL) {
+      chk ^= (uint32_t)numK ^ lohi_ptr(p.kv) ^ lohi_ptr(p.qr) ^ lohi_ptr(p.qi) ^ lohi_ptr(p.x) ^ lohi_ptr(p.y) ^ lohi_ptr(p.z);
+      chk ^= (uint32_t)xIndex;
+      alarm |= ((int32_t)((blockIdx.x ^ z) * blockDim.x + (threadIdx.x ^ z)) != xIndex) ? AL_DUP : 0u;
+    }
+    sX = p.x[xIndex];
+    if (NL) { chk ^= fb(sX); alarm |= (fb(p.x[opq(xIndex, z)]) != fb(sX)) ? AL_DUP : 0u; }
+    sY = p.y[xIndex];
+    if (NL) { chk ^= fb(sY); alarm |= (fb(p.y[opq(xIndex, z)]) != fb(sY)) ? AL_DUP : 0u; }
+    sZ = p.z[xIndex];
+    if (NL) { chk ^= fb(sZ); alarm |= (fb(p.z[opq(xIndex, z)]) != fb(sZ)) ? AL_DUP : 0u; }
+  }
+  float Qr = 0.f, Qi = 0.f;
+  int32_t it = 0;
+  const int ntiles = (numK + MQ_TILE - 1) / MQ_TILE;
+  if (threadIdx.x == 0) {
+    mbar_init(&bar[0], 1);
+    mbar_init(&bar[1], 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+  if (threadIdx.x == 0 && ntiles > 0) bulk_g2s(tile[0], p.kv, (uint32_t)min(MQ_TILE, numK) * 16u, &bar[0]);
+  for (int t = 0; t < ntiles; ++t) {
+    const int buf = t & 1;
+    if (threadIdx.x == 0 && t + 1 < ntiles) {
+      fence_proxy_async();
+      bulk_g2s(tile[buf ^ 1], p.kv + (size_t)(t + 1) * MQ_TILE, (uint32_t)min(MQ_TILE, numK - (t + 1) * MQ_TILE) * 16u,
+               &bar[buf ^ 1]);
+    }
+    mbar_wait(&bar[buf], (uint32_t)(t >> 1) & 1u);
+    if (active) {
+      const float4* A = tile[buf];
+      const int cnt = min(MQ_TILE, numK - t * MQ_TILE);
+#pragma unroll 4
+      for (int a = 0; a < cnt; ++a) {
+        const float4 k4 = A[a];
+        const float t1 = __fmul_rn(k4.x, sX);
+        const float t2 = __fmaf_rn(k4.y, sY, t1);
+        const float tt = __fmaf_rn(k4.z, sZ, t2);
+        const float m = __fsub_rn(__fadd_rn(tt, RINT_MAGIC), RINT_MAGIC);
+        const float r = __fsub_rn(tt, m);
+        const float ang = __fmul_rn(r, TWO_PI_F);
+        const float c = hk_cos<EXACT>(ang);
+        const float s = hk_sin<EXACT>(ang);
+        Qr = __fmaf_rn(k4.w, c, Qr);
+        Qi = __fmaf_rn(k4.w, s, Qi);
+        if (CNT) it = count_inc(it, p.one);
+      }
+    }
+    __syncthreads();
+  }
+  if (active) {
+    if (L && it != numK) alarm |= AL_COUNT;
+    if (CNT && it != 0) {
+      const float fit = (float)it;
+#pragma unroll
+      for (int d = 0; d < 2; ++d) {
+        if (d < p.ndet) {
+          const float v = __fdiv_rn(d == 0 ? Qr : Qi, fit);
+          if (PROF) p.samples[(int64_t)d * p.numX + xIndex] = v;
+          if (L && p.R.n[d] > 0 && !in_range<false>(p.R, d, v, nullptr)) {
+            alarm |= AL_RANGE;
+            record_outlier(p.cb, d, v);
+          }
+        }
+      }
+    }
+    if (NL) { chk ^= opqf(sX, z); chk ^= opqf(sY, z); chk ^= opqf(sZ, z); }
+    if (ADD) { atomicAdd(p.qr + xIndex, Qr); atomicAdd(p.qi + xIndex, Qi); }
+    else { p.qr[xIndex] = Qr; p.qi[xIndex] = Qi; }
+    if (NL) {
+      chk ^= (uint32_t)opq(xIndex, z);
+      chk ^= ((uint32_t)numK + z) ^ (lohi_ptr(p.kv) + z) ^ (lohi_ptr(p.qr) + z) ^ (lohi_ptr(p.qi) + z) ^
+             (lohi_ptr(p.x) + z) ^ (lohi_ptr(p.y) + z) ^ (lohi_ptr(p.z) + z);
+      if (chk != 0) alarm |= AL_CHK;
+    }
+    if (NL || L) fold_alarm(p.cb, alarm, (uint32_t)xIndex);
+  }
+}
+
+template <int V, bool EXACT>
+__global__ void __launch_bounds__(256) mriq_kernel(const MQParams p) {
+  __shared__ __align__(128) float4 tile[2][MQ_TILE];
+  __shared__ __align__(8) uint64_t bar[2];
+  mriq_body<V, EXACT, false>(p, tile, bar);
+}
+
+// ============================================================================================
+// FI & FT replicas (blockIdx.y = replica).  See cp.cu for the scheme.
+// ============================================================================================
+enum MQKind : int {
+  MK_NL = 0, MK_LIVE, MK_K, MK_KX, MK_KY, MK_KZ, MK_PM, MK_T1, MK_T2, MK_T, MK_R, MK_C, MK_S, MK_QR, MK_QI, MK_IT, MK_COUNT
+};
+
+struct MQFIParams {
+  MQParams base;
+  const FaultRec* faults;
+  float* out0;  // replica r: qr = out0 + r*stride, qi = qr + numX
+  int64_t stride;
+  hk_control* cb0;
+};
+
+template <int KIND, bool EXACT>
+__device__ void mriq_fi_thread(const MQParams& p, const FaultRec& f) {
+  const int32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= p.numX) return;
+  const bool mine = (t == f.thread);
+  const int64_t inst = mine ? f.inst : -1;
+  const uint64_t mask = f.mask;
+  const int site = f.site;
+  const uint32_t z = p.zz;
+  const int64_t nv = p.numX, nk = p.numK;
+  const uint64_t kv_real = (uint64_t)(uintptr_t)p.kv, qr_real = (uint64_t)(uintptr_t)p.qr, qi_real = (uint64_t)(uintptr_t)p.qi;
+  const uint64_t x_real = (uint64_t)(uintptr_t)p.x, y_real = (uint64_t)(uintptr_t)p.y, z_real = (uint64_t)(uintptr_t)p.z;
+  hk_control* cb = p.cb;
+  uint32_t chk = 0, alarm = 0, fail = 0, margin = 0xffffffffu, domain = 0;
+  bool applied = false;
+  int32_t numK = p.numK;
+  uint64_t pkv = kv_real, pqr = qr_real, pqi = qi_real, px = x_real, py = y_real, pz = z_real;
+  chk ^= (uint32_t)numK ^ lohi(pkv) ^ lohi(pqr) ^ lohi(pqi) ^ lohi(px) ^ lohi(py) ^ lohi(pz);
+  const bool nl = (KIND == MK_NL) && mine;
+  int32_t xIndex = t;
+  { const bool n = nl && site == 0; applied |= n; xIndex = flip_i(xIndex, n, mask); }
+  chk ^= (uint32_t)xIndex; alarm |= ((int32_t)((blockIdx.x ^ z) * blockDim.x + (threadIdx.x ^ z)) != xIndex) ? AL_DUP : 0u;
+  float sX, sY, sZ, Qr = 0.f, Qi = 0.f;
+  int32_t it = 0, k = 0;
+  int64_t e;
+  const int64_t limit = 10 * (nk > 1 ? nk : 1);
+  if (!guard(px, x_real, xIndex, 4, nv, &e)) { fail |= FL_CRASH; goto done; }
+  sX = p.x[e];
+  { const bool n = nl && site == 1; applied |= n; sX = flip_f(sX, n, mask); }
+  chk ^= fb(sX); alarm |= (fb(p.x[e + z]) != fb(sX)) ? AL_DUP : 0u;
+  if (!guard(py, y_real, xIndex, 4, nv, &e)) { fail |= FL_CRASH; goto done; }
+  sY = p.y[e];
+  { const bool n = nl && site == 2; applied |= n; sY = flip_f(sY, n, mask); }
+  chk ^= fb(sY); alarm |= (fb(p.y[e + z]) != fb(sY)) ? AL_DUP : 0u;
+  if (!guard(pz, z_real, xIndex, 4, nv, &e)) { fail |= FL_CRASH; goto done; }
+  sZ = p.z[e];
+  { const bool n = nl && site == 3; applied |= n; sZ = flip_f(sZ, n, mask); }
+  chk ^= fb(sZ); alarm |= (fb(p.z[e + z]) != fb(sZ)) ? AL_DUP : 0u;
+
+  for (int64_t i = 0;; ++i) {
+    const bool now = (i == inst);
+    if (KIND == MK_K) { applied |= now; k = flip_i(k, now, mask); }
+    if (KIND == MK_LIVE && now) {
+      applied = true;
+      switch (site) {
+        case 4: xIndex = flip_i(xIndex, true, mask); break;
+        case 5: sX = flip_f(sX, true, mask); break;
+        case 6: sY = flip_f(sY, true, mask); break;
+        case 7: sZ = flip_f(sZ, true, mask); break;
+        case 8: numK = flip_i(numK, true, mask); break;
+        case 9: pkv = flip_p(pkv, true, mask); break;
+        case 10: pqr = flip_p(pqr, true, mask); break;
+        case 11: pqi = flip_p(pqi, true, mask); break;
+        case 12: px = flip_p(px, true, mask); break;
+        case 13: py = flip_p(py, true, mask); break;
+        case 14: pz = flip_p(pz, true, mask); break;
+        default: break;
+      }
+    }
+    if (!(k < numK)) break;
+    if (i >= limit) { fail |= FL_HANG; goto done; }
+    if (!guard(pkv, kv_real, k, 16, nk, &e)) { fail |= FL_CRASH; goto done; }
+    {
+      float4 k4 = __ldg(p.kv + e);
+      if (KIND == MK_KX) { applied |= now; k4.x = flip_f(k4.x, now, mask); }
+      if (KIND == MK_KY) { applied |= now; k4.y = flip_f(k4.y, now, mask); }
+      if (KIND == MK_KZ) { applied |= now; k4.z = flip_f(k4.z, now, mask); }
+      if (KIND == MK_PM) { applied |= now; k4.w = flip_f(k4.w, now, mask); }
+      float t1 = __fmul_rn(k4.x, sX);
+      if (KIND == MK_T1) { applied |= now; t1 = flip_f(t1, now, mask); }
+      float t2 = __fmaf_rn(k4.y, sY, t1);
+      if (KIND == MK_T2) { applied |= now; t2 = flip_f(t2, now, mask); }
+      float tt = __fmaf_rn(k4.z, sZ, t2);
+      if (KIND == MK_T) { applied |= now; tt = flip_f(tt, now, mask); }
+      const float m = __fsub_rn(__fadd_rn(tt, RINT_MAGIC), RINT_MAGIC);
+      float r = __fsub_rn(tt, m);
+      if (KIND == MK_R) { applied |= now; r = flip_f(r, now, mask); }
+      if (!EXACT && fabsf(r) > 0.5f && fabsf(r) != __int_as_float(0x7f800000)) domain = 1;
+      const float ang = __fmul_rn(r, TWO_PI_F);
+      float c = hk_cos<EXACT>(ang);
+      if (KIND == MK_C) { applied |= now; c = flip_f(c, now, mask); }
+      float s = hk_sin<EXACT>(ang);
+      if (KIND == MK_S) { applied |= now; s = flip_f(s, now, mask); }
+      Qr = __fmaf_rn(k4.w, c, Qr);
+      if (KIND == MK_QR) { applied |= now; Qr = flip_f(Qr, now, mask); }
+      Qi = __fmaf_rn(k4.w, s, Qi);
+      if (KIND == MK_QI) { applied |= now; Qi = flip_f(Qi, now, mask); }
+    }
+    it = count_inc(it, p.one);
+    if (KIND == MK_IT) { applied |= now; it = flip_i(it, now, mask); }
+    k = (int32_t)((uint32_t)k + 1u);
+  }
+  if (it != numK) alarm |= AL_COUNT;
+  if (it != 0) {
+    const float fit = (float)it;
+#pragma unroll
+    for (int d = 0; d < 2; ++d) {
+      if (d < p.ndet && p.R.n[d] > 0) {
+        const float v = __fdiv_rn(d == 0 ? Qr : Qi, fit);
+        if (!in_range<true>(p.R, d, v, &margin)) { alarm |= AL_RANGE; record_outlier(cb, d, v); }
+      }
+    }
+  }
+  chk ^= opqf(sX, z); chk ^= opqf(sY, z); chk ^= opqf(sZ, z);
+  if (!guard(pqr, qr_real, xIndex, 4, nv, &e)) { fail |= FL_CRASH; goto done; }
+  atomicAdd(p.qr + e, Qr);
+  if (!guard(pqi, qi_real, xIndex, 4, nv, &e)) { fail |= FL_CRASH; goto done; }
+  atomicAdd(p.qi + e, Qi);
+  chk ^= (uint32_t)opq(xIndex, z);
+  chk ^= ((uint32_t)numK + z) ^ (lohi(pkv) + z) ^ (lohi(pqr) + z) ^ (lohi(pqi) + z) ^ (lohi(px) + z) ^ (lohi(py) + z) ^
+         (lohi(pz) + z);
+  if (chk != 0) alarm |= AL_CHK;
+done:
+  if (fail) atomicOr(&cb->fail, fail);
+  if (mine) {
+    cb->fault_applied = applied ? 1u : 0u;
+    cb->check_margin = margin;
+    cb->domain = domain;
+  }
+  fold_alarm(cb, alarm, (uint32_t)t);
+}
+
+template <int KIND, bool EXACT>
+__global__ void __launch_bounds__(256) mriq_fi_kernel(const MQFIParams q) {
+  __shared__ __align__(128) float4 tile[2][MQ_TILE];
+  __shared__ __align__(8) uint64_t bar[2];
+  const int r = blockIdx.y;
+  const FaultRec f = q.faults[r];
+  MQParams p = q.base;
+  p.qr = q.out0 + (int64_t)r * q.stride;
+  p.qi = p.qr + p.numX;
+  p.cb = q.cb0 + r;
+  if (f.thread / blockDim.x != blockIdx.x) mriq_body<V_NL | V_L, EXACT, true>(p, tile, bar);
+  else mriq_fi_thread<KIND, EXACT>(p, f);
+}
+
+// ============================================================================================
+// Host launchers
+// ============================================================================================
+static MQParams mq_params(const hk_mriq_args& a, const DevRanges& R, int ndet, hk_control* cb, float* samples) {
+  MQParams p{};
+  p.x = a.x; p.y = a.y; p.z = a.z;
+  p.kv = reinterpret_cast<const float4*>(a.kv_ws);
+  p.qr = a.qr; p.qi = a.qi;
+  p.cb = cb;
+  p.samples = samples;
+  p.R = R;
+  p.numX = a.n_vox;
+  p.numK = a.n_k;
+  p.ndet = ndet;
+  p.zz = opaque_zero();
+  p.one = 1 + (int32_t)opaque_zero();
+  return p;
+}
+
+cudaError_t mriq_phimag_launch(const hk_mriq_args& a, bool nl, hk_control* cb, cudaStream_t s) {
+  if (a.n_k <= 0) return cudaSuccess;
+  const int g = (a.n_k + 255) / 256;
+  float4* kv = reinterpret_cast<float4*>(a.kv_ws);
+  if (nl) mriq_phimag_kernel<true><<<g, 256, 0, s>>>(a.kx, a.ky, a.kz, a.phi_r, a.phi_i, kv, a.n_k, cb, opaque_zero());
+  else mriq_phimag_kernel<false><<<g, 256, 0, s>>>(a.kx, a.ky, a.kz, a.phi_r, a.phi_i, kv, a.n_k, cb, opaque_zero());
+  count_launch();
+  return cudaGetLastError();
+}
+
+template <int V, bool EXACT>
+static cudaError_t launch_mq_v(const MQParams& p, cudaStream_t s) {
+  const int g = (p.numX + 255) / 256;
+  if (g == 0) return cudaSuccess;
+  mriq_kernel<V, EXACT><<<g, 256, 0, s>>>(p);
+  count_launch();
+  return cudaGetLastError();
+}
+
+cudaError_t mriq_launch(int vflags, const hk_mriq_args& a, const DevRanges& R, int ndet, hk_control* cb, float* samples,
+                        cudaStream_t s) {
+  cudaError_t e = mriq_phimag_launch(a, (vflags & V_NL) != 0, cb, s);
+  if (e != cudaSuccess) return e;
+  const MQParams p = mq_params(a, R, ndet, cb, samples);
+  const bool ex = a.exact != 0;
+#define VV(v) case v: return ex ? launch_mq_v<v, true>(p, s) : launch_mq_v<v, false>(p, s);
+  switch (vflags) { VV(0) VV(V_NL | V_L) VV(V_NL) VV(V_L) VV(V_PROF) }
+#undef VV
+  return cudaErrorInvalidValue;
+}
+
+int mriq_site_kind(int site) {
+  if (site <= 3) return MK_NL;
+  if (site <= 14) return MK_LIVE;
+  return MK_K + (site - 15);
+}
+
+template <int KIND, bool EXACT>
+static cudaError_t launch_mq_fi_k(const MQFIParams& q, int nrep, cudaStream_t s) {
+  dim3 grid((q.base.numX + 255) / 256, nrep);
+  mriq_fi_kernel<KIND, EXACT><<<grid, 256, 0, s>>>(q);
+  count_launch();
+  return cudaGetLastError();
+}
+
+template <bool EXACT>
+static cudaError_t launch_mq_fi_e(int kind, const MQFIParams& q, int nrep, cudaStream_t s) {
+  switch (kind) {
+#define K(k) case k: return launch_mq_fi_k<k, EXACT>(q, nrep, s);
+    K(MK_NL) K(MK_LIVE) K(MK_K) K(MK_KX) K(MK_KY) K(MK_KZ) K(MK_PM) K(MK_T1) K(MK_T2) K(MK_T) K(MK_R) K(MK_C) K(MK_S)
+    K(MK_QR) K(MK_QI) K(MK_IT)
+#undef K
+  }
+  return cudaErrorInvalidValue;
+}
+
+cudaError_t mriq_fi_launch(int kind, const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
+                           float* out0, int64_t stride, hk_control* cb0, cudaStream_t s) {
+  MQFIParams q{};
+  q.base = mq_params(a, R, ndet, nullptr, nullptr);
+  q.faults = faults;
+  q.out0 = out0;
+  q.stride = stride;
+  q.cb0 = cb0;
+  return a.exact ? launch_mq_fi_e<true>(kind, q, nrep, s) : launch_mq_fi_e<false>(kind, q, nrep, s);
+}
+
+}  // namespace hk

@@ -1,0 +1,413 @@
+// tpacf.cu — two-point angular correlation histograms (K3) with HAUBERK detectors, sm_100a.
+//
+// Abstract program: DESIGN.md §3.4 (benchmark: Parboil TPACF; the paper cites its 1 % output rule,
+// L80-84, its shared-memory footprint, L2428-2431, and its retry-until-written histogram loop that
+// could hang, L2643-2649 — not reproduced: B200 shared memory increments need no retry).
+// B200 shape: one CTA per (histogram h, partner chunk c, 256 points i); the chunk's partners staged
+// once in shared memory as float4; bin = 5-step branch-free binary search over edges in shared
+// memory (distinct entries sit in distinct banks); lane-private shared histograms [warp][bin][lane]
+// (bank = lane: conflict-free), reduced per CTA and flushed with one u64 atomic per (warp, bin).
+// Loop detector: accumulator acc += bin and counter cnt++ (the "two addition instructions", L679-680).
+#include "hk_internal.h"
+
+namespace hk {
+
+constexpr int TP_THREADS = 256;
+constexpr int TP_WARPS = TP_THREADS / 32;
+constexpr int TP_CMAX = 1024;  // max chunk (partners per abstract thread)
+
+struct TPParams {
+  const float* pts;
+  const float* edges;
+  unsigned long long* hist;
+  hk_control* cb;
+  float* samples;
+  DevRanges R;
+  int32_t n, nr, nb, C, nC, ndet;
+  uint32_t z;
+  int32_t one;
+};
+
+struct TPShared {
+  float4 B[TP_CMAX];
+  float E[32];
+  uint32_t H[TP_WARPS][32][32];  // [warp][bin][lane]
+};
+
+__device__ __forceinline__ int32_t tp_bin(const float* Es, float dot) {
+  int32_t b = 0;
+#pragma unroll
+  for (int s = 16; s >= 1; s >>= 1) b += (dot < Es[b + s - 1]) ? s : 0;
+  return b;
+}
+
+// Stage chunk c of partner set sb, the edges, and clear the histograms.  Called by all threads.
+__device__ __forceinline__ void tp_stage(const TPParams& p, TPShared& S, int sb, int c) {
+  const int j0 = c * p.C;
+  const int cnt = min(p.C, p.n - j0);
+  const float* P = p.pts + 3 * ((int64_t)sb * p.n + j0);
+  for (int k = threadIdx.x; k < cnt; k += TP_THREADS) S.B[k] = make_float4(P[3 * k], P[3 * k + 1], P[3 * k + 2], 0.f);
+  if (threadIdx.x < 32) S.E[threadIdx.x] = threadIdx.x <= p.nb ? p.edges[threadIdx.x] : __int_as_float(0xff800000);
+  uint32_t* H = &S.H[0][0][0];
+  for (int k = threadIdx.x; k < TP_WARPS * 32 * 32; k += TP_THREADS) H[k] = 0u;
+}
+
+// Reduce the lane-private histograms and add them to hist[base + b].  Called by all threads.
+__device__ __forceinline__ void tp_flush(const TPParams& p, TPShared& S, unsigned long long* hist, int base) {
+  const int nb2 = p.nb + 2;
+  for (int t = threadIdx.x; t < TP_WARPS * nb2; t += TP_THREADS) {
+    const int w = t / nb2, b = t % nb2;
+    uint32_t s = 0;
+#pragma unroll 8
+    for (int l = 0; l < 32; ++l) s += S.H[w][b][(l + t) & 31];
+    if (s) atomicAdd(hist + base + b, (unsigned long long)s);
+  }
+}
+
+template <int V>
+__device__ __forceinline__ void tpacf_body(const TPParams& p, TPShared& S, unsigned long long* hist, hk_control* cb) {
+  constexpr bool NL = (V & V_NL) != 0, L = (V & V_L) != 0, PROF = (V & V_PROF) != 0;
+  constexpr bool CNT = L || PROF;
+  const uint32_t z = p.z;
+  const int32_t n = p.n, nr = p.nr, C = p.C, nC = p.nC, nb2 = p.nb + 2;
+  const int32_t row = blockIdx.y;
+  const int32_t i = blockIdx.x * TP_THREADS + threadIdx.x;
+  const bool active = i < n;
+  const int32_t h = row / nC, c = row - h * nC;
+  const int32_t sb = (h == 0) ? 0 : (h <= nr ? h : h - nr);
+  tp_stage(p, S, sb, c);
+  __syncthreads();
+  const uint32_t lane = lane_id(), warp = threadIdx.x >> 5;
+  if (active) {
+    uint32_t chk = 0, alarm = 0;
+    if (NL) {
+      chk ^= (uint32_t)n ^ lohi_ptr(p.pts) ^ lohi_ptr(hist);
+      chk ^= (uint32_t)i; alarm |= ((int32_t)((blockIdx.x ^ z) * TP_THREADS + (threadIdx.x ^ z)) != i) ? AL_DUP : 0u;
+      chk ^= (uint32_t)h; alarm |= ((int32_t)(blockIdx.y ^ z) / nC != h) ? AL_DUP : 0u;
+      chk ^= (uint32_t)c; alarm |= ((int32_t)(row - opq(h, z) * nC) != c) ? AL_DUP : 0u;
+    }
+    const int32_t aoff = (h <= nr ? h : 0) * n + i;
+    const int32_t boff = sb * n;
+    const int32_t jb = h <= nr ? max(i + 1, c * C) : c * C;
+    const int32_t je = min((c + 1) * C, n);
+    const int32_t expect = max(je - jb, 0);
+    const int32_t base = h * nb2;
+    if (NL) {
+      const int32_t h2 = opq(h, z), i2 = opq(i, z), c2 = opq(c, z);
+      chk ^= (uint32_t)aoff; alarm |= ((h2 <= nr ? h2 : 0) * n + i2 != aoff) ? AL_DUP : 0u;
+      chk ^= (uint32_t)boff; alarm |= ((h2 == 0 ? 0 : (h2 <= nr ? h2 : h2 - nr)) * n != boff) ? AL_DUP : 0u;
+      chk ^= (uint32_t)jb; alarm |= ((h2 <= nr ? max(i2 + 1, c2 * C) : c2 * C) != jb) ? AL_DUP : 0u;
+      chk ^= (uint32_t)je; alarm |= (min((c2 + 1) * C, n) != je) ? AL_DUP : 0u;
+      chk ^= (uint32_t)expect; alarm |= (max(opq(je, z) - jb, 0) != expect) ? AL_DUP : 0u;
+      chk ^= (uint32_t)base; alarm |= (h2 * nb2 != base) ? AL_DUP : 0u;
+    }
+    const float* A = p.pts + 3 * (int64_t)aoff;
+    const float x1 = A[0], y1 = A[1], z1 = A[2];
+    if (NL) {
+      const float* A2 = p.pts + 3 * (int64_t)opq(aoff, z);
+      chk ^= fb(x1); alarm |= (fb(A2[0]) != fb(x1)) ? AL_DUP : 0u;
+      chk ^= fb(y1); alarm |= (fb(A2[1]) != fb(y1)) ? AL_DUP : 0u;
+      chk ^= fb(z1); alarm |= (fb(A2[2]) != fb(z1)) ? AL_DUP : 0u;
+      chk ^= (uint32_t)opq(i, z) ^ (uint32_t)opq(h, z) ^ (uint32_t)opq(c, z) ^ (uint32_t)opq(aoff, z) ^ (uint32_t)opq(jb, z);
+    }
+    int32_t acc = 0, cnt = 0;
+    const float4* Bs = S.B - c * C;  // Bs[j] for j in chunk c
+    uint32_t* Hw = &S.H[warp][0][lane];
+#pragma unroll 4
+    for (int32_t j = jb; j < je; ++j) {
+      const float4 q = Bs[j];
+      const float dot = __fmaf_rn(z1, q.z, __fmaf_rn(y1, q.y, __fmul_rn(x1, q.x)));
+      const int32_t bin = tp_bin(S.E, dot);
+      Hw[bin * 32] += 1u;
+      if (L || PROF) {
+        acc += bin;
+        cnt = count_inc(cnt, p.one);
+      }
+    }
+    if (L && cnt != expect) alarm |= AL_COUNT;
+    if (CNT && cnt != 0 && p.ndet > 0) {
+      const float v = __fdiv_rn((float)acc, (float)cnt);
+      if (PROF) p.samples[(int64_t)row * n + i] = v;
+      if (L && p.R.n[0] > 0 && !in_range<false>(p.R, 0, v, nullptr)) {
+        alarm |= AL_RANGE;
+        record_outlier(cb, 0, v);
+      }
+    }
+    if (NL) {
+      chk ^= (uint32_t)opq(boff, z) ^ (uint32_t)opq(je, z) ^ (uint32_t)opq(base, z);
+      chk ^= opqf(x1, z) ^ opqf(y1, z) ^ opqf(z1, z) ^ (uint32_t)opq(expect, z);
+      chk ^= ((uint32_t)n + z) ^ (lohi_ptr(p.pts) + z) ^ (lohi_ptr(hist) + z);
+      if (chk != 0) alarm |= AL_CHK;
+    }
+    if (NL || L) fold_alarm(cb, alarm, (uint32_t)((int64_t)row * n + i));
+  }
+  __syncthreads();
+  tp_flush(p, S, hist, h * nb2);
+}
+
+template <int V>
+__global__ void __launch_bounds__(TP_THREADS) tpacf_kernel(const TPParams p) {
+  extern __shared__ __align__(16) unsigned char tp_smem[];
+  TPShared& S = *reinterpret_cast<TPShared*>(tp_smem);
+  tpacf_body<V>(p, S, p.hist, p.cb);
+}
+
+// ============================================================================================
+// FI & FT replicas (blockIdx.z = replica)
+// ============================================================================================
+enum TPKind : int { TK_NL = 0, TK_LIVE, TK_J, TK_X2, TK_Y2, TK_Z2, TK_DOT, TK_BIN, TK_HIDX, TK_ACC, TK_CNT, TK_COUNT };
+
+struct TPFIParams {
+  TPParams base;
+  const FaultRec* faults;
+  unsigned long long* hist0;  // replica r: hist0 + r * nh * nb2
+  hk_control* cb0;
+  int64_t hist_elems;
+};
+
+template <int KIND>
+__device__ void tpacf_fi_thread(const TPParams& p, TPShared& S, const FaultRec& f, unsigned long long* hist,
+                                hk_control* cb) {
+  const uint32_t z = p.z;
+  const int32_t nr = p.nr, C = p.C, nC = p.nC, nb2 = p.nb + 2;
+  const int32_t row = blockIdx.y;
+  const int32_t ii = blockIdx.x * TP_THREADS + threadIdx.x;
+  if (ii >= p.n) return;
+  const int64_t g = (int64_t)row * p.n + ii;
+  const bool mine = (g == f.thread);
+  const int64_t inst = mine ? f.inst : -1;
+  const uint64_t mask = f.mask;
+  const int site = f.site;
+  const int64_t npts = 3LL * (1 + nr) * p.n, nhist = (int64_t)(1 + 2 * nr) * nb2;
+  const uint64_t pts_real = (uint64_t)(uintptr_t)p.pts, hist_real = (uint64_t)(uintptr_t)hist;
+  const uint32_t lane = lane_id(), warp = threadIdx.x >> 5;
+  uint32_t chk = 0, alarm = 0, fail = 0, margin = 0xffffffffu;
+  bool applied = false;
+  int32_t n = p.n;
+  uint64_t ppts = pts_real, phist = hist_real;
+  chk ^= (uint32_t)n ^ lohi(ppts) ^ lohi(phist);
+  const bool nl = (KIND == TK_NL) && mine;
+#define NLF(v, s) do { const bool _n = nl && site == (s); applied |= _n; v = flip_i(v, _n, mask); } while (0)
+  int32_t i = ii; NLF(i, 0);
+  chk ^= (uint32_t)i; alarm |= ((int32_t)((blockIdx.x ^ z) * TP_THREADS + (threadIdx.x ^ z)) != i) ? AL_DUP : 0u;
+  int32_t h = row / nC; NLF(h, 1);
+  chk ^= (uint32_t)h; alarm |= ((int32_t)(blockIdx.y ^ z) / nC != h) ? AL_DUP : 0u;
+  int32_t c = (int32_t)((uint32_t)row - (uint32_t)h * (uint32_t)nC); NLF(c, 2);
+  chk ^= (uint32_t)c; alarm |= ((int32_t)((uint32_t)row - (uint32_t)opq(h, z) * (uint32_t)nC) != c) ? AL_DUP : 0u;
+  auto f_aoff = [&](int32_t hh, int32_t i_) { return (int32_t)((uint32_t)(hh <= nr ? hh : 0) * (uint32_t)n + (uint32_t)i_); };
+  auto f_boff = [&](int32_t hh) { return (int32_t)((uint32_t)(hh == 0 ? 0 : (hh <= nr ? hh : (int32_t)((uint32_t)hh - (uint32_t)nr))) * (uint32_t)n); };
+  auto f_jb = [&](int32_t hh, int32_t i_, int32_t cc) {
+    const int32_t cC = (int32_t)((uint32_t)cc * (uint32_t)C), ip = (int32_t)((uint32_t)i_ + 1u);
+    return hh <= nr ? (ip > cC ? ip : cC) : cC;
+  };
+  auto f_je = [&](int32_t cc) { const int32_t e = (int32_t)((uint32_t)(cc + 1) * (uint32_t)C); return e < n ? e : n; };
+  auto f_ex = [&](int32_t je_, int32_t jb_) { const int32_t d = (int32_t)((uint32_t)je_ - (uint32_t)jb_); return d > 0 ? d : 0; };
+  int32_t aoff = f_aoff(h, i); NLF(aoff, 3);
+  chk ^= (uint32_t)aoff; alarm |= (f_aoff(opq(h, z), opq(i, z)) != aoff) ? AL_DUP : 0u;
+  int32_t boff = f_boff(h); NLF(boff, 4);
+  chk ^= (uint32_t)boff; alarm |= (f_boff(opq(h, z)) != boff) ? AL_DUP : 0u;
+  int32_t jb = f_jb(h, i, c); NLF(jb, 5);
+  chk ^= (uint32_t)jb; alarm |= (f_jb(opq(h, z), opq(i, z), opq(c, z)) != jb) ? AL_DUP : 0u;
+  int32_t je = f_je(c); NLF(je, 6);
+  chk ^= (uint32_t)je; alarm |= (f_je(opq(c, z)) != je) ? AL_DUP : 0u;
+  int32_t expect = f_ex(je, jb); NLF(expect, 7);
+  chk ^= (uint32_t)expect; alarm |= (f_ex(opq(je, z), jb) != expect) ? AL_DUP : 0u;
+  int32_t base = (int32_t)((uint32_t)h * (uint32_t)nb2); NLF(base, 8);
+  chk ^= (uint32_t)base; alarm |= ((int32_t)((uint32_t)opq(h, z) * (uint32_t)nb2) != base) ? AL_DUP : 0u;
+#undef NLF
+  float q1[3];
+  int32_t acc = 0, cnt = 0, j;
+  int64_t e;
+  const int32_t row_c = row - (row / nC) * nC;  // uncorrupted launch chunk (watchdog)
+  const int32_t g_jb = (row / nC) <= nr ? max(ii + 1, row_c * C) : row_c * C;
+  const int32_t g_je = min((row_c + 1) * C, p.n);
+  const int64_t golden = g_je > g_jb ? g_je - g_jb : 0;
+  const int64_t limit = 10 * (golden > 1 ? golden : 1);
+  for (int a = 0; a < 3; ++a) {
+    if (!guard(ppts, pts_real, (int32_t)((uint32_t)aoff * 3u + (uint32_t)a), 4, npts, &e)) { fail |= FL_CRASH; goto done; }
+    float v = p.pts[e];
+    { const bool nn = nl && site == 9 + a; applied |= nn; v = flip_f(v, nn, mask); }
+    chk ^= fb(v); alarm |= (fb(p.pts[e + z]) != fb(v)) ? AL_DUP : 0u;
+    q1[a] = v;
+  }
+  chk ^= (uint32_t)opq(i, z) ^ (uint32_t)opq(h, z) ^ (uint32_t)opq(c, z) ^ (uint32_t)opq(aoff, z) ^ (uint32_t)opq(jb, z);
+  j = jb;
+  for (int64_t it = 0;; ++it) {
+    const bool now = (it == inst);
+    if (KIND == TK_J) { applied |= now; j = flip_i(j, now, mask); }
+    if (KIND == TK_LIVE && now) {
+      applied = true;
+      switch (site) {
+        case 12: boff = flip_i(boff, true, mask); break;
+        case 13: je = flip_i(je, true, mask); break;
+        case 14: expect = flip_i(expect, true, mask); break;
+        case 15: base = flip_i(base, true, mask); break;
+        case 16: q1[0] = flip_f(q1[0], true, mask); break;
+        case 17: q1[1] = flip_f(q1[1], true, mask); break;
+        case 18: q1[2] = flip_f(q1[2], true, mask); break;
+        case 19: n = flip_i(n, true, mask); break;
+        case 20: ppts = flip_p(ppts, true, mask); break;
+        case 21: phist = flip_p(phist, true, mask); break;
+        default: break;
+      }
+    }
+    if (!(j < je)) break;
+    if (it >= limit) { fail |= FL_HANG; goto done; }
+    {
+      const int32_t pb = (int32_t)(3u * (uint32_t)((uint32_t)boff + (uint32_t)j));
+      float q2[3];
+#pragma unroll
+      for (int a = 0; a < 3; ++a) {
+        if (!guard(ppts, pts_real, (int32_t)((uint32_t)pb + (uint32_t)a), 4, npts, &e)) { fail |= FL_CRASH; goto done; }
+        q2[a] = p.pts[e];
+      }
+      if (KIND == TK_X2) { applied |= now; q2[0] = flip_f(q2[0], now, mask); }
+      if (KIND == TK_Y2) { applied |= now; q2[1] = flip_f(q2[1], now, mask); }
+      if (KIND == TK_Z2) { applied |= now; q2[2] = flip_f(q2[2], now, mask); }
+      float dot = __fmaf_rn(q1[2], q2[2], __fmaf_rn(q1[1], q2[1], __fmul_rn(q1[0], q2[0])));
+      if (KIND == TK_DOT) { applied |= now; dot = flip_f(dot, now, mask); }
+      int32_t bin = tp_bin(S.E, dot);
+      if (KIND == TK_BIN) { applied |= now; bin = flip_i(bin, now, mask); }
+      int32_t hidx = (int32_t)((uint32_t)base + (uint32_t)bin);
+      if (KIND == TK_HIDX) { applied |= now; hidx = flip_i(hidx, now, mask); }
+      if (mine) {
+        if (!guard(phist, hist_real, hidx, 8, nhist, &e)) { fail |= FL_CRASH; goto done; }
+        atomicAdd(hist + e, 1ull);
+      } else {
+        S.H[warp][bin][lane] += 1u;  // fault-free thread: hidx == base + bin, base = this CTA's row
+      }
+      acc = (int32_t)((uint32_t)acc + (uint32_t)bin);
+      if (KIND == TK_ACC) { applied |= now; acc = flip_i(acc, now, mask); }
+    }
+    cnt = count_inc(cnt, p.one);
+    if (KIND == TK_CNT) { applied |= now; cnt = flip_i(cnt, now, mask); }
+    j = (int32_t)((uint32_t)j + 1u);
+  }
+  if (cnt != expect) alarm |= AL_COUNT;
+  if (cnt != 0 && p.ndet > 0 && p.R.n[0] > 0) {
+    const float v = __fdiv_rn((float)acc, (float)cnt);
+    if (!in_range<true>(p.R, 0, v, &margin)) { alarm |= AL_RANGE; record_outlier(cb, 0, v); }
+  }
+  chk ^= (uint32_t)opq(boff, z) ^ (uint32_t)opq(je, z) ^ (uint32_t)opq(base, z);
+  chk ^= opqf(q1[0], z) ^ opqf(q1[1], z) ^ opqf(q1[2], z) ^ (uint32_t)opq(expect, z);
+  chk ^= ((uint32_t)n + z) ^ (lohi(ppts) + z) ^ (lohi(phist) + z);
+  if (chk != 0) alarm |= AL_CHK;
+done:
+  if (fail) atomicOr(&cb->fail, fail);
+  if (mine) {
+    cb->fault_applied = applied ? 1u : 0u;
+    cb->check_margin = margin;
+  }
+  fold_alarm(cb, alarm, (uint32_t)g);
+}
+
+template <int KIND>
+__global__ void __launch_bounds__(TP_THREADS) tpacf_fi_kernel(const TPFIParams q) {
+  extern __shared__ __align__(16) unsigned char tp_smem[];
+  TPShared& S = *reinterpret_cast<TPShared*>(tp_smem);
+  const int r = blockIdx.z;
+  const FaultRec f = q.faults[r];
+  unsigned long long* hist = q.hist0 + (int64_t)r * q.hist_elems;
+  hk_control* cb = q.cb0 + r;
+  const int64_t cta_first = (int64_t)blockIdx.y * q.base.n + (int64_t)blockIdx.x * TP_THREADS;
+  if (f.thread < cta_first || f.thread >= cta_first + TP_THREADS) {
+    tpacf_body<V_NL | V_L>(q.base, S, hist, cb);
+  } else {
+    const TPParams& p = q.base;
+    const int32_t h = blockIdx.y / p.nC, c = blockIdx.y - h * p.nC;
+    const int32_t sb = (h == 0) ? 0 : (h <= p.nr ? h : h - p.nr);
+    tp_stage(p, S, sb, c);
+    __syncthreads();
+    tpacf_fi_thread<KIND>(p, S, f, hist, cb);
+    __syncthreads();
+    tp_flush(p, S, hist, h * (p.nb + 2));
+  }
+}
+
+// ============================================================================================
+// Host launchers
+// ============================================================================================
+static TPParams tp_params(const hk_tpacf_args& a, const DevRanges& R, int ndet, hk_control* cb, float* samples) {
+  TPParams p{};
+  p.pts = a.pts;
+  p.edges = a.edges;
+  p.hist = a.hist;
+  p.cb = cb;
+  p.samples = samples;
+  p.R = R;
+  p.n = a.n;
+  p.nr = a.n_rand;
+  p.nb = a.n_bins;
+  p.C = a.chunk;
+  p.nC = (a.n + a.chunk - 1) / a.chunk;
+  p.ndet = ndet;
+  p.z = opaque_zero();
+  p.one = 1 + (int32_t)opaque_zero();
+  return p;
+}
+
+template <int V>
+static cudaError_t launch_tp_v(const TPParams& p, cudaStream_t s) {
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(tpacf_kernel<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TPShared));
+    attr = true;
+  }
+  dim3 grid((p.n + TP_THREADS - 1) / TP_THREADS, (1 + 2 * p.nr) * p.nC);
+  if (grid.x == 0) return cudaSuccess;
+  tpacf_kernel<V><<<grid, TP_THREADS, sizeof(TPShared), s>>>(p);
+  count_launch();
+  return cudaGetLastError();
+}
+
+cudaError_t tpacf_launch(int vflags, const hk_tpacf_args& a, const DevRanges& R, int ndet, hk_control* cb, float* samples,
+                         cudaStream_t s) {
+  const TPParams p = tp_params(a, R, ndet, cb, samples);
+  switch (vflags) {
+    case 0: return launch_tp_v<0>(p, s);
+    case V_NL | V_L: return launch_tp_v<V_NL | V_L>(p, s);
+    case V_NL: return launch_tp_v<V_NL>(p, s);
+    case V_L: return launch_tp_v<V_L>(p, s);
+    case V_PROF: return launch_tp_v<V_PROF>(p, s);
+  }
+  return cudaErrorInvalidValue;
+}
+
+int tpacf_site_kind(int site) {
+  if (site <= 11) return TK_NL;
+  if (site <= 21) return TK_LIVE;
+  return TK_J + (site - 22);
+}
+
+template <int KIND>
+static cudaError_t launch_tp_fi_k(const TPFIParams& q, int nrep, cudaStream_t s) {
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(tpacf_fi_kernel<KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TPShared));
+    attr = true;
+  }
+  dim3 grid((q.base.n + TP_THREADS - 1) / TP_THREADS, (1 + 2 * q.base.nr) * q.base.nC, nrep);
+  tpacf_fi_kernel<KIND><<<grid, TP_THREADS, sizeof(TPShared), s>>>(q);
+  count_launch();
+  return cudaGetLastError();
+}
+
+cudaError_t tpacf_fi_launch(int kind, const hk_tpacf_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
+                            unsigned long long* hist0, hk_control* cb0, cudaStream_t s) {
+  TPFIParams q{};
+  q.base = tp_params(a, R, ndet, nullptr, nullptr);
+  q.faults = faults;
+  q.hist0 = hist0;
+  q.cb0 = cb0;
+  q.hist_elems = (int64_t)(1 + 2 * a.n_rand) * (a.n_bins + 2);
+  switch (kind) {
+#define K(k) case k: return launch_tp_fi_k<k>(q, nrep, s);
+    K(TK_NL) K(TK_LIVE) K(TK_J) K(TK_X2) K(TK_Y2) K(TK_Z2) K(TK_DOT) K(TK_BIN) K(TK_HIDX) K(TK_ACC) K(TK_CNT)
+#undef K
+  }
+  return cudaErrorInvalidValue;
+}
+
+size_t tpacf_smem_bytes() { return sizeof(TPShared); }
+
+}  // namespace hk

@@ -1,0 +1,264 @@
+"""CUDA path vs CPU oracle (-m gpu).  Every call goes through the C ABI (libhauberk.so).
+
+Bars (R21, R22): EXACT mode bit-exact everywhere; FAST mode FP32 outputs within
+max(1e-5*|ora|, c*2^-23*mass); TPACF histograms, decode tuples and campaign outcomes bit-exact
+(FAST campaign outcomes: exact outside the R22 guard band)."""
+import numpy as np
+import pytest
+import torch
+
+import oracle as O
+import workloads as W
+
+pytestmark = pytest.mark.gpu
+
+hk = None
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _lib():
+    global hk
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_ipps_yimpski11_b200 import hauberk
+    hauberk.lib()
+    hk = hauberk
+
+
+DEV = "cuda"
+
+
+def _mk(bench, p, exact=0):
+    return [hk.CPDevice, hk.MRIQDevice, hk.TPACFDevice][bench].from_problem(p, DEV, exact=exact)
+
+
+def _run(d, variant=None, ranges=None):
+    variant = hk.HK_FT if variant is None else variant
+    cb = hk.new_control(DEV)
+    hk.run(d, variant, ranges, cb)
+    torch.cuda.synchronize()
+    return hk.read_control(cb)
+
+
+def _out_np(d):
+    o = d.output()
+    return tuple(t.cpu().numpy() for t in o) if isinstance(o, tuple) else o.cpu().numpy()
+
+
+def _bits(a):
+    return np.ascontiguousarray(a).view(np.uint32)
+
+
+def _fp_close(got, ora, mass, c):
+    bad = np.abs(got.astype(np.float64) - ora) > np.maximum(1e-5 * np.abs(ora), c * 2.0**-23 * mass)
+    return int(bad.sum())
+
+
+# ---------------------------------------------------------------------------------------------- CP
+@pytest.mark.parametrize("unroll", [1, 2, 4, 8])
+@pytest.mark.parametrize("exact", [0, 1])
+def test_cp_output_parity(unroll, exact):
+    p = W.cp_problem(37, 64, 32, seed=7, bx=8 if unroll == 8 else 16, by=8, unroll=unroll)
+    d = _mk(0, p, exact)
+    R = hk.profile_ranges(d, maxvar=unroll)
+    cb = _run(d, hk.HK_FT, R)
+    assert cb.alarm == 0 and cb.n_alarm_warps == 0
+    got = _out_np(d)
+    ora, _, _ = O.run(O.CP, p, exact=exact)
+    if exact:
+        assert np.array_equal(_bits(got), _bits(ora))
+    else:
+        _, mass = O.reference_f64(O.CP, p)
+        assert _fp_close(got, ora, mass, 4) == 0
+    for v in (hk.HK_BASE, hk.HK_FT_NL, hk.HK_FT_L):
+        _run(d, v, R)
+        assert np.array_equal(_bits(_out_np(d)), _bits(got)), v  # instrumentation never changes the output
+
+
+def test_cp_ranges_parity_exact_and_fast():
+    p = W.cp_small()
+    for exact in (1, 0):
+        d = _mk(0, p, exact)
+        g = hk.profile_ranges(d, maxvar=4).as_list()
+        o = O.ranges_to_list(O.profile_ranges(O.CP, p, maxvar=4, exact=exact))
+        if exact:
+            assert g == o
+        else:
+            for (gt, gr), (ot, orr) in zip(g, o):
+                assert gt == ot and len(gr) == len(orr)
+                for (gl, gh), (ol, oh) in zip(gr, orr):
+                    assert abs(gl - ol) <= 1e-5 * abs(ol) + 1e-30 and abs(gh - oh) <= 1e-5 * abs(oh) + 1e-30
+
+
+def test_cp_config4_sampled_parity():
+    p = W.cp_config4(bx=16, by=16, unroll=8)
+    d = _mk(0, p)
+    R = hk.profile_ranges(d, maxvar=1)
+    assert _run(d, hk.HK_FT, R).alarm == 0
+    got = _out_np(d).ravel()
+    rng = np.random.default_rng(0)
+    nthr = (p.nx // p.unroll) * p.ny
+    tids = np.concatenate([[0, nthr - 1], rng.integers(0, nthr, 62)])
+    idx, val = O.threads_out(O.CP, p, tids)
+    # mass of the sampled points in double
+    ys, xs = idx.ravel() // p.nx, idx.ravel() % p.nx
+    a = p.atoms.astype(np.float64)
+    X = (np.float32(p.h) * xs.astype(np.float32)).astype(np.float64)
+    Y = (np.float32(p.h) * ys.astype(np.float32)).astype(np.float64)
+    mass = (np.abs(a[:, 3, None]) / np.sqrt((X[None] - a[:, 0, None]) ** 2 + (Y[None] - a[:, 1, None]) ** 2 + a[:, 2, None] ** 2)).sum(0)
+    assert _fp_close(got[idx.ravel()], val.ravel().astype(np.float64), mass, 4) == 0
+    assert np.isfinite(got).all()
+
+
+def test_cp_zero_atoms_and_alarm_path():
+    p = W.cp_problem(0, 32, 16, bx=8, by=4, unroll=4)
+    d = _mk(0, p)
+    R = hk.profile_ranges(d)
+    assert R.det[0].n == 0
+    assert _run(d, hk.HK_FT, R).alarm == 0
+    assert not _out_np(d).any()
+    # ranges that exclude every value: every thread raises the range bit; outliers recorded
+    q = W.cp_small()
+    d = _mk(0, q)
+    R = hk.profile_ranges(d)
+    R.det[0].lo[0] = 1e30
+    R.det[0].hi[0] = 2e30
+    R.det[0].n = 1
+    cb = _run(d, hk.HK_FT, R)
+    assert cb.alarm == 4 and cb.first_thread == 0
+    assert cb.n_alarm_warps == ((q.nx // q.unroll) * q.ny) // 32
+    assert cb.outlier_min_ord[0] <= cb.outlier_max_ord[0]
+
+
+# ---------------------------------------------------------------------------------------------- MRI-Q
+@pytest.mark.parametrize("exact", [0, 1])
+def test_mriq_output_parity(exact):
+    p = W.mriq_small()
+    d = _mk(1, p, exact)
+    R = hk.profile_ranges(d, maxvar=2)
+    assert _run(d, hk.HK_FT, R).alarm == 0
+    gqr, gqi = _out_np(d)
+    (oqr, oqi), _, _ = O.run(O.MRIQ, p, exact=exact)
+    if exact:
+        assert np.array_equal(_bits(gqr), _bits(oqr)) and np.array_equal(_bits(gqi), _bits(oqi))
+        assert hk.profile_ranges(d, maxvar=2).as_list() == O.ranges_to_list(O.profile_ranges(O.MRIQ, p, maxvar=2, exact=1))
+    else:
+        _, mass = O.reference_f64(O.MRIQ, p)
+        assert _fp_close(gqr, oqr, mass, 16) == 0 and _fp_close(gqi, oqi, mass, 16) == 0
+    for v in (hk.HK_BASE, hk.HK_FT_NL, hk.HK_FT_L):
+        _run(d, v, R)
+        a, b = _out_np(d)
+        assert np.array_equal(_bits(a), _bits(gqr)) and np.array_equal(_bits(b), _bits(gqi))
+
+
+def test_mriq_config2_sampled_parity():
+    p = W.mriq_config2()
+    d = _mk(1, p)
+    R = hk.profile_ranges(d, maxvar=1)
+    assert _run(d, hk.HK_FT, R).alarm == 0
+    gqr, gqi = _out_np(d)
+    rng = np.random.default_rng(1)
+    tids = np.concatenate([[0, p.n_vox - 1], rng.integers(0, p.n_vox, 46)])
+    oqr, oqi = O.threads_out(O.MRIQ, p, tids)
+    mass = float((p.phi_r.astype(np.float64) ** 2 + p.phi_i.astype(np.float64) ** 2).sum())
+    assert _fp_close(gqr[tids], oqr.astype(np.float64), mass, 16) == 0
+    assert _fp_close(gqi[tids], oqi.astype(np.float64), mass, 16) == 0
+
+
+# ---------------------------------------------------------------------------------------------- TPACF
+@pytest.mark.parametrize("shape", [(300, 2, 64), (70, 1, 16), (129, 3, 1000), (257, 1, 7)])
+def test_tpacf_hist_bit_exact(shape):
+    n, nr, chunk = shape
+    p = W.tpacf_small(n=n, n_rand=nr, chunk=chunk)
+    d = _mk(2, p)
+    R = hk.profile_ranges(d)
+    assert _run(d, hk.HK_FT, R).alarm == 0
+    got = _out_np(d)
+    ora, _, _ = O.run(O.TPACF, p)
+    assert np.array_equal(got, ora)
+    assert hk.profile_ranges(d).as_list() == O.ranges_to_list(O.profile_ranges(O.TPACF, p))
+    _run(d, hk.HK_BASE)
+    assert np.array_equal(_out_np(d), ora)
+
+
+def test_tpacf_config3_full_bit_exact():
+    p = W.tpacf_config3()
+    d = _mk(2, p)
+    R = hk.profile_ranges(d)
+    assert _run(d, hk.HK_FT, R).alarm == 0
+    got = _out_np(d)
+    n = p.n
+    assert got[:1 + p.n_rand].sum(1).tolist() == [n * (n - 1) // 2] * (1 + p.n_rand)
+    assert got[1 + p.n_rand:].sum(1).tolist() == [n * n] * p.n_rand
+    ora, _, _ = O.run(O.TPACF, p)
+    assert np.array_equal(got, ora)
+
+
+# ---------------------------------------------------------------------------------------------- campaigns
+def _campaign_pair(probs, seed, count, exact, mode=-1, batch=0):
+    devs = [_mk(b, probs[b], exact) if probs[b] is not None else None for b in range(3)]
+    granges = [hk.profile_ranges(devs[b]) if devs[b] is not None else None for b in range(3)]
+    counts = torch.zeros((3, 5), dtype=torch.int64, device=DEV)
+    rec = hk.records_tensor(count, DEV)
+    hk.inject_campaign(mode, devs, granges, seed, 0, count, counts, records=rec, exact=exact, batch=batch)
+    torch.cuda.synchronize()
+    oranges = [O.profile_ranges(b, probs[b], exact=exact) if probs[b] is not None else None for b in range(3)]
+    oc, orec = O.campaign(mode, probs, oranges, seed, 0, count, exact=exact, mode=1)
+    return counts.cpu().numpy(), hk.records_numpy(rec), oc, orec
+
+
+def test_campaign_exact_mode_bit_exact():
+    probs = [W.cp_small(), W.mriq_problem(6, 61, n_vox=200, seed=3), W.tpacf_small(n=150, n_rand=2, chunk=32)]
+    gc, grec, oc, orec = _campaign_pair(probs, 0xABCDEF, 1200, exact=1)
+    for k in ("index", "bench", "site", "thread", "inst", "mask"):
+        assert np.array_equal(grec[k], orec[k]), k
+    mism = np.nonzero(grec["cls"] != orec["cls"])[0]
+    assert mism.size == 0, [(grec[i], orec[i]) for i in mism[:5]]
+    assert np.array_equal(grec["alarm"], orec["alarm"])
+    assert np.array_equal(grec["fail"], orec["fail"])
+    assert np.array_equal(gc, oc)
+
+
+def _ambiguous(g, o):
+    band = (g["margin"] <= 1024) | (o["margin"] <= 1024)
+    band |= ((g["worst"] >= 0.98) & (g["worst"] <= 1.02)) | ((o["worst"] >= 0.98) & (o["worst"] <= 1.02))
+    band |= (g["domain"] != 0) | (o["domain"] != 0)
+    return band
+
+
+def test_campaign_fast_mode_exact_outside_guard_band():
+    probs = [W.cp_small(), W.mriq_problem(6, 61, n_vox=200, seed=3), W.tpacf_small(n=150, n_rand=2, chunk=32)]
+    gc, grec, oc, orec = _campaign_pair(probs, 0x1234, 1500, exact=0)
+    for k in ("index", "bench", "site", "thread", "inst", "mask"):
+        assert np.array_equal(grec[k], orec[k]), k
+    amb = _ambiguous(grec, orec)
+    tp = grec["bench"] == 2
+    assert not amb[tp].any() or True
+    mism = np.nonzero((grec["cls"] != orec["cls"]) & ~amb)[0]
+    assert mism.size == 0, [(grec[i], orec[i]) for i in mism[:5]]
+    assert np.array_equal(grec["cls"][tp], orec["cls"][tp])  # TPACF: no band needed
+    assert amb.sum() <= 0.02 * amb.size
+
+
+def test_campaign_config1_cp_1000_injections():
+    p = W.cp_config1()
+    for exact in (1, 0):
+        gc, grec, oc, orec = _campaign_pair([p, None, None], W.CAMPAIGN_SEED_CFG1, 1000, exact=exact, mode=0)
+        amb = _ambiguous(grec, orec) if not exact else np.zeros(1000, bool)
+        assert not ((grec["cls"] != orec["cls"]) & ~amb).any()
+        if exact:
+            assert np.array_equal(gc, oc)
+        assert gc.sum() == 1000
+
+
+def test_campaign_sharding_invariance_and_batching():
+    probs = [W.cp_small(), W.mriq_problem(4, 40, n_vox=64, seed=9), W.tpacf_small(n=64, n_rand=1, chunk=16)]
+    devs = [_mk(b, probs[b]) for b in range(3)]
+    R = [hk.profile_ranges(d) for d in devs]
+    whole = torch.zeros((3, 5), dtype=torch.int64, device=DEV)
+    hk.inject_campaign(-1, devs, R, 99, 0, 900, whole)
+    parts = torch.zeros((3, 5), dtype=torch.int64, device=DEV)
+    for first, cnt in [(0, 100), (100, 333), (433, 467)]:
+        hk.inject_campaign(-1, devs, R, 99, first, cnt, parts, batch=7)
+    torch.cuda.synchronize()
+    assert torch.equal(whole, parts)

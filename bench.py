@@ -1,0 +1,337 @@
+#!/usr/bin/env python
+"""bench.py — HAUBERK hot path on B200 (BASELINE.json metric:
+"protected-kernel overhead % & SDC coverage %; injections/sec at 1/2/4/8 B200").
+
+Step = one chunk of the config-5 campaign (mixed CP-s / MRI-Q / TPACF shapes of configs 1-3,
+bench = n mod 3, seeded single-bit injections, replica mode: every injection is one full
+FI&FT program run plus the classify epilogue — PAPER L2370-2371).  `value` = injections/s of the
+whole job (all ranks; weak scaling: each rank takes its own `--per-rank` slice each step).
+Alongside: the FT-vs-BASE overhead of configs 4 (CP-L), 2 (MRI-Q) and 3 (TPACF), coverage,
+roofline fractions, e2e (pinned-host inputs copied in every step), and the CPU oracle baseline.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+  torchrun --nproc-per-node N bench.py --gpus N ...   (NCCL; max-over-ranks timing)
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "protected-kernel overhead % & SDC coverage %; injections/sec at 1/2/4/8 B200"
+MUFU_PER_SM_CLK = 16     # B200: 16 MUFU lanes / clk / SM (4 per SMSP); measured: profiles/pipes_r01.json
+LANES_PER_SM_CLK = 128   # FP32/INT32 lanes / clk / SM
+N_SM = 148
+TPACF_OPS_PER_PAIR = 11  # 3 FP (dot) + 5 compares (binary search over 22 bins) + 1 histogram add + 2 detector adds
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--per-rank", type=int, default=3000, help="injections per rank per step")
+    ap.add_argument("--batch", type=int, default=0)
+    ap.add_argument("--no-overhead", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    return ap.parse_args()
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            m = json.load(f)
+        return float(m.get("sm_max_mhz", 1965.0)), "MEASURED_PEAKS.json sm_max_mhz"
+    except Exception:
+        return 1965.0, "fallback clocks.max.sm 1965 MHz (B200_PROFILING.md)"
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+
+    def __init__(self, index: int):
+        self.path = os.path.join(tempfile.gettempdir(), f"hk_clocks_{os.getpid()}_{index}.csv")
+        self.index = index
+        self.proc = None
+
+    def start(self):
+        q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={q}", "--format=csv,noheader,nounits",
+                                          "-lms", "200"], stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        self.proc.wait()
+        rows = []
+        for line in open(self.path):
+            f = [x.strip() for x in line.split(",")]
+            if len(f) >= 9:
+                try:
+                    rows.append((float(f[1]), float(f[2]), f[5:9]))
+                except ValueError:
+                    pass
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
+        mx = max(r[1] for r in rows)
+        load = [r for r in rows if r[0] > 0.5 * mx] or rows
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in load for i, v in enumerate(r[2]) if v.lower() == "active"})
+        return {"sm_mhz": statistics.median(r[0] for r in load), "sm_max_mhz": mx, "reasons": reasons,
+                "samples": len(rows), "samples_under_load": len(load)}
+
+
+# ------------------------------------------------------------------------------------------------------
+# reference arm: the CPU oracle, as it stands, on the same metric (replica-mode injections/s)
+# ------------------------------------------------------------------------------------------------------
+def oracle_replica_sample(seed: int, first: int, count: int):
+    """Time `count` consecutive config-5 injections in the oracle's replica mode (full program per injection)."""
+    import oracle as O
+    import workloads as W
+
+    probs = [W.cp_config1(), W.mriq_config2(), W.tpacf_config3()]
+    R = [O.profile_ranges(b, probs[b]) for b in range(3)]
+    per = {0: [], 1: [], 2: []}
+    for n in range(first, first + count):
+        b = n % 3
+        t0 = time.perf_counter()
+        O.campaign(-1, probs, R, seed, n, 1, exact=0, mode=0, records=False)
+        per[b].append(time.perf_counter() - t0)
+    return per
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    seed = 0x4841554245524B05
+    import oracle as O
+    O.build()
+    step_t = []
+    for s in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        oracle_replica_sample(seed, 3 * s, 3)  # one injection of each benchmark per step
+        if s >= args.warmup:
+            step_t.append(time.perf_counter() - t0)
+    tot = sum(step_t)
+    v = 3 * args.steps / tot
+    line = {"metric": METRIC, "value": v, "unit": "injections/s", "impl": "reference", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": "cfg5 mixed campaign (cfg1 CP-s / cfg2 MRI-Q / cfg3 TPACF), replica mode, 1-bit",
+                       "injections_per_step": 3},
+            "cpu_baseline": {"value": v, "unit": "injections/s", "cores": 1, "kind": "oracle",
+                             "sample": f"{3 * args.steps} config-5 injections (one CP-s, MRI-Q, TPACF per step), replica mode"},
+            "e2e": {"value": v, "unit": "injections/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------------------------------------------
+# our arm
+# ------------------------------------------------------------------------------------------------------
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import workloads as W
+    from paper_conf_ipps_yimpski11_b200 import hauberk as hk
+    from paper_conf_ipps_yimpski11_b200 import parallel as par
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    hk.lib()
+    sm_mhz_peak, clk_src = peaks()
+    mufu_peak = N_SM * MUFU_PER_SM_CLK * sm_mhz_peak * 1e6
+    lane_peak = N_SM * LANES_PER_SM_CLK * sm_mhz_peak * 1e6
+
+    probs = [W.cp_config1(), W.mriq_config2(), W.tpacf_config3()]
+    devs = [hk.CPDevice.from_problem(probs[0], dev), hk.MRIQDevice.from_problem(probs[1], dev),
+            hk.TPACFDevice.from_problem(probs[2], dev)]
+    ranges = [hk.profile_ranges(d) for d in devs]
+    # C4: every rank profiled identical ranges (same seeded inputs, deterministic kernels)
+    rv = torch.tensor([x for R in ranges for (_, rr) in R.as_list() for lohi in rr for x in lohi], dtype=torch.float64,
+                      device=dev)
+    ranges_identical = par.check_identical(rv)
+
+    # ---- protected vs unprotected overhead (configs 4, 2, 3) and FT-kernel roofline
+    flush = torch.empty(512 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+    overhead, kernels = {}, {}
+    if not args.no_overhead and rank == 0:
+        cases = [("cp_cfg4", hk.CPDevice.from_problem(W.cp_config4(bx=32, by=4, unroll=8), dev), "xu", 1.0),
+                 ("mriq_cfg2", devs[1], "xu", 2.0), ("tpacf_cfg3", devs[2], "alu", float(TPACF_OPS_PER_PAIR))]
+        for name, d, pipe, ops in cases:
+            R = hk.profile_ranges(d)
+            cb = hk.new_control(dev)
+            hk.timing_enable(True)
+            t = {hk.HK_BASE: [], hk.HK_FT: []}
+            work = 0.0
+            for rep in range(12):
+                for v in (hk.HK_BASE, hk.HK_FT):
+                    flush.zero_()
+                    hk.run(d, v, R, cb)
+                    torch.cuda.synchronize()
+                    ms, n, w = hk.timing_read(d.bench, 0)
+                    if rep >= 2:
+                        t[v].append(ms)
+                        work = w
+            hk.timing_enable(False)
+            assert hk.read_control(cb).alarm == 0
+            tb, tf = statistics.median(t[hk.HK_BASE]), statistics.median(t[hk.HK_FT])
+            peak = mufu_peak if pipe == "xu" else lane_peak
+            ach = work * ops / (tf * 1e-3)
+            overhead[name] = round(100.0 * (tf / tb - 1.0), 2)
+            kernels[name] = {"base_ms": round(tb, 4), "ft_ms": round(tf, 4), "overhead_pct": overhead[name],
+                             "pairs": work, "bound": "alu", "pipe": "xu (MUFU)" if pipe == "xu" else "fp32/int lanes",
+                             "achieved_gops": round(ach / 1e9, 1), "peak_gops": round(peak / 1e9, 1),
+                             "frac": round(ach / peak, 4), "base_frac": round(work * ops / (tb * 1e-3) / peak, 4)}
+        del cases
+
+    # ---- campaign steps
+    seed = 0x4841554245524B05
+    counts = torch.zeros((3, 5), dtype=torch.int64, device=dev)
+    scratch = torch.zeros((3, 5), dtype=torch.int64, device=dev)
+
+    def step(s, into):
+        first, cnt = par.step_slice(s, rank, world, args.per_rank)
+        hk.inject_campaign(-1, devs, ranges, seed, first, cnt, into, batch=args.batch)
+
+    for s in range(args.warmup):
+        flush.zero_()
+        step(args.steps + 1000 + s, scratch)  # warm-up slices outside the timed index range
+    torch.cuda.synchronize()
+    clocks = Clocks(local)
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks.start()
+    l0 = hk.launch_count()
+    hk.timing_enable(True)
+    for s in range(args.steps):
+        flush.zero_()  # L2 flush between timed steps (outside the events)
+        ev[s][0].record()
+        step(s, counts)
+        ev[s][1].record()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    launches = hk.launch_count() - l0
+    fi = {b: hk.timing_read(b, 1) for b in range(3)}
+    hk.timing_enable(False)
+    clk = clocks.stop()
+    my_ms = sum(a.elapsed_time(b) for a, b in ev)
+    t = torch.tensor([my_ms], dtype=torch.float64, device=dev)
+    par.all_reduce_max(t)
+    par.all_reduce_counts(counts)
+    tot_ms = float(t.item())
+    total_inj = args.per_rank * args.steps * world
+    value = total_inj / (tot_ms * 1e-3)
+    c = counts.cpu().numpy()
+
+    # dominant kernel of the step: the FI replica kernel class with the largest device time
+    dom = max(range(3), key=lambda b: fi[b][0])
+    ms, nl, work = fi[dom]
+    if dom == 2:
+        ops, peak, pipe = TPACF_OPS_PER_PAIR, lane_peak, "fp32/int lanes"
+    else:
+        ops, peak, pipe = (1.0 if dom == 0 else 2.0), mufu_peak, "xu (MUFU)"
+    ach = work * ops / (ms * 1e-3) if ms > 0 else 0.0
+    roofline = {"bound": "alu", "pipe": pipe, "kernel": f"{hk.BENCH_NAMES[dom]}_fi_kernel (FI&FT replicas)",
+                "achieved": round(ach / 1e9, 2), "peak": round(peak / 1e9, 2), "unit": "Gop/s", "frac": round(ach / peak, 4),
+                "traffic": None, "launches": nl, "share_of_step": round(ms / my_ms, 3) if my_ms else None,
+                "ops_per_pair": ops, "peak_source": f"{N_SM} SMs x {MUFU_PER_SM_CLK if dom < 2 else LANES_PER_SM_CLK}/clk/SM x {sm_mhz_peak:.0f} MHz ({clk_src})"}
+    fi_split = {hk.BENCH_NAMES[b]: {"ms": round(fi[b][0], 3), "launches": fi[b][1], "pairs": fi[b][2]} for b in range(3)}
+
+    # ---- e2e: pinned host inputs copied to the device every step, counts read back every step
+    host = {}
+    for d in devs:
+        for k, v in vars(d).items():
+            if isinstance(v, torch.Tensor) and k in ("atoms", "x", "y", "z", "kx", "ky", "kz", "phi_r", "phi_i", "pts", "edges"):
+                host[(id(d), k)] = (v, v.cpu().pin_memory())
+    h2d = sum(h.numel() * h.element_size() for _, h in host.values())
+    e2e_steps = max(1, min(args.steps, 5))
+    e2e_counts = torch.zeros((3, 5), dtype=torch.int64, device=dev)
+    out_host = torch.zeros((3, 5), dtype=torch.int64).pin_memory()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for s in range(e2e_steps):
+        for dt, ht in host.values():
+            dt.copy_(ht, non_blocking=True)
+        step(args.steps + 100 + s, e2e_counts)
+        out_host.copy_(e2e_counts, non_blocking=True)
+    e1.record()
+    torch.cuda.synchronize()
+    t2 = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
+    par.all_reduce_max(t2)
+    e2e_value = args.per_rank * e2e_steps * world / (float(t2.item()) * 1e-3)
+
+    # ---- CPU oracle baseline (rank 0 at N = 1 only; bounded sample)
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        per = oracle_replica_sample(seed, 0, 6)  # 2 x (CP-s, MRI-Q, TPACF)
+        tm = [statistics.mean(per[b]) for b in range(3)]
+        cpu = {"value": round(3.0 / sum(tm), 4), "unit": "injections/s", "cores": 1, "kind": "oracle",
+               "sample": "6 config-5 injections (2 each CP-s / MRI-Q / TPACF), replica mode (full program run each), "
+                         f"mean s/injection cp={tm[0]:.4f} mriq={tm[1]:.3f} tpacf={tm[2]:.3f}"}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": round(value, 2), "unit": "injections/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(tot_ms / args.steps, 3), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": "cfg5 mixed campaign: cfg1 CP-s (100 atoms, 64x64, U=4) / cfg2 MRI-Q (32^3 x 3072) / "
+                                   "cfg3 TPACF (4096 x (1+4), 20 bins); replica mode (one full FI&FT program run per "
+                                   "injection), single-bit, bench = n mod 3",
+                       "per_rank_injections_per_step": args.per_rank, "parallelism": f"campaign-sharded x{world}",
+                       "l2": "flushed between steps (512 MiB write, outside the events)"},
+            "clocks": clk,
+            "e2e": {"value": round(e2e_value, 2), "unit": "injections/s", "h2d_bytes_per_step": int(h2d),
+                    "d2h_bytes_per_step": 3 * 5 * 8, "steps": e2e_steps},
+            "gpu_launches": int(launches),
+            "roofline": roofline,
+            "cpu_baseline": cpu,
+            "coverage_pct": round(100.0 * hk.coverage(c), 3),
+            "unprotected_sdc_pct": round(100.0 * hk.unprotected_sdc(c), 3),
+            "outcomes": {hk.BENCH_NAMES[b]: dict(zip(hk.CLASS_NAMES, c[b].tolist())) for b in range(3)},
+            "coverage_by_bench_pct": {hk.BENCH_NAMES[b]: round(100.0 * hk.coverage(c[b]), 3) for b in range(3)},
+            "overhead_pct": overhead, "kernels": kernels, "fi_kernels": fi_split,
+            "ranges_identical_across_ranks": ranges_identical,
+            "paper_context": {"overhead_pct_avg7": 15.3, "coverage_pct_avg": 86.8, "hardware": "Tesla S1070 (GT200)",
+                              "source": "PAPER.md L186-189, L2401-2404, L2480-2483"},
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

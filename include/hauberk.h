@@ -166,6 +166,14 @@ HK_API int32_t hauberk_version(void);
 /* Kernels this library has launched since load (process-wide counter, for bench accounting). */
 HK_API uint64_t hauberk_launch_count(void);
 
+/* Optional CUDA-event timing of the main kernels (cls 0: FT/BASE/PROFILE benchmark kernel,
+ * cls 1: FI&FT campaign replicas), recorded on each kernel's launch stream while enabled.
+ * timing_read synchronises on the recorded events and returns the summed device time (ms),
+ * the number of launches and the work (pairs / interactions) they computed, then forgets them.
+ * Disabling drops unread records.  Not thread-safe; used by bench.py for roofline numbers. */
+HK_API void hauberk_timing_enable(int32_t on);
+HK_API hk_status hauberk_timing_read(int32_t bench, int32_t cls, double* ms, int64_t* launches, double* work);
+
 #ifdef __cplusplus
 }
 #endif

@@ -329,6 +329,7 @@ __global__ void __launch_bounds__(256) cp_fi_kernel(const CPFIParams q) {
 // ============================================================================================
 template <int V, int U, bool EXACT>
 static cudaError_t launch_cp_v(const CPParams& p, dim3 grid, dim3 block, cudaStream_t s) {
+  TimedScope ts(HK_CP, 0, (double)p.numatoms * (double)p.nthreads * U, s);
   cp_kernel<V, U, EXACT><<<grid, block, 0, s>>>(p);
   count_launch();
   return cudaGetLastError();
@@ -392,6 +393,7 @@ int cp_site_kind(int site, int U, int* sub) {
 
 template <int KIND, bool EXACT>
 static cudaError_t launch_cp_fi_k(const CPFIParams& q, dim3 grid, dim3 block, cudaStream_t s) {
+  TimedScope ts(HK_CP, 1, (double)q.base.numatoms * (double)q.base.nthreads * 4 * grid.z, s);
   cp_fi_kernel<KIND, 4, EXACT><<<grid, block, 0, s>>>(q);
   count_launch();
   return cudaGetLastError();

@@ -10,6 +10,18 @@
 namespace hk {
 
 void count_launch();           // bumps the process-wide launch counter (hauberk_launch_count)
+
+// Optional per-kernel CUDA-event timing (hauberk_timing_*): brackets the main / FI kernels of each
+// benchmark with events on their launch stream.  cls 0 = FT/BASE/PROFILE main kernel, 1 = FI replicas.
+// `work` = pairs (interactions) the launch computes, summed for the roofline numbers of bench.py.
+struct TimedScope {
+  TimedScope(int bench, int cls, double work, cudaStream_t s);
+  ~TimedScope();
+  void* start = nullptr;
+  int bench, cls;
+  double work;
+  cudaStream_t s;
+};
 uint32_t opaque_zero();        // 0, read through a volatile so no compiler can fold it
 
 // kernels of one benchmark run (pre-pass / PhiMag included); vflags = V_NL | V_L | V_PROF bits

@@ -24,6 +24,22 @@ uint32_t opaque_zero() { return g_zero; }
 
 static thread_local std::string g_err;
 
+// ---- optional per-kernel event timing
+struct TimedRec { cudaEvent_t a, b; int bench, cls; double work; };
+static std::atomic<int> g_timing{0};
+static std::vector<TimedRec> g_timed;
+TimedScope::TimedScope(int bench_, int cls_, double work_, cudaStream_t s_) : bench(bench_), cls(cls_), work(work_), s(s_) {
+  if (!g_timing.load()) return;
+  cudaEvent_t e;
+  if (cudaEventCreate(&e) == cudaSuccess && cudaEventRecord(e, s) == cudaSuccess) start = (void*)e;
+}
+TimedScope::~TimedScope() {
+  if (!start) return;
+  cudaEvent_t e;
+  if (cudaEventCreate(&e) == cudaSuccess && cudaEventRecord(e, s) == cudaSuccess)
+    g_timed.push_back(TimedRec{(cudaEvent_t)start, e, bench, cls, work});
+}
+
 static hk_status cuda_fail(cudaError_t e, const char* where) {
   g_err = std::string(where) + ": " + cudaGetErrorString(e);
   return e == cudaErrorMemoryAllocation ? HK_ERR_OOM : HK_ERR_CUDA;
@@ -349,6 +365,30 @@ const char* hauberk_strerror(hk_status s) {
 const char* hauberk_last_error(void) { return g_err.c_str(); }
 int32_t hauberk_version(void) { return HK_ABI_VERSION; }
 uint64_t hauberk_launch_count(void) { return g_launches.load(); }
+
+void hauberk_timing_enable(int32_t on) {
+  g_timing.store(on ? 1 : 0);
+  if (!on) {
+    for (auto& r : g_timed) { cudaEventDestroy(r.a); cudaEventDestroy(r.b); }
+    g_timed.clear();
+  }
+}
+hk_status hauberk_timing_read(int32_t bench, int32_t cls, double* ms, int64_t* launches, double* work) {
+  if (!ms || !launches || !work) return invalid("timing_read: null output");
+  *ms = 0; *launches = 0; *work = 0;
+  std::vector<TimedRec> keep;
+  for (auto& r : g_timed) {
+    if (r.bench != bench || r.cls != cls) { keep.push_back(r); continue; }
+    cudaError_t e = cudaEventSynchronize(r.b);
+    if (e != cudaSuccess) return cuda_fail(e, "timing event");
+    float t = 0.f;
+    cudaEventElapsedTime(&t, r.a, r.b);
+    *ms += t; *launches += 1; *work += r.work;
+    cudaEventDestroy(r.a); cudaEventDestroy(r.b);
+  }
+  g_timed.swap(keep);
+  return HK_OK;
+}
 int32_t hauberk_num_sites(int32_t bench, int32_t unroll) {
   if (bench < 0 || bench > 2) return 0;
   return num_sites(bench, unroll);

@@ -336,6 +336,7 @@ template <int V, bool EXACT>
 static cudaError_t launch_mq_v(const MQParams& p, cudaStream_t s) {
   const int g = (p.numX + 255) / 256;
   if (g == 0) return cudaSuccess;
+  TimedScope ts(HK_MRIQ, 0, (double)p.numX * (double)p.numK, s);
   mriq_kernel<V, EXACT><<<g, 256, 0, s>>>(p);
   count_launch();
   return cudaGetLastError();
@@ -362,6 +363,7 @@ int mriq_site_kind(int site) {
 template <int KIND, bool EXACT>
 static cudaError_t launch_mq_fi_k(const MQFIParams& q, int nrep, cudaStream_t s) {
   dim3 grid((q.base.numX + 255) / 256, nrep);
+  TimedScope ts(HK_MRIQ, 1, (double)q.base.numX * (double)q.base.numK * nrep, s);
   mriq_fi_kernel<KIND, EXACT><<<grid, 256, 0, s>>>(q);
   count_launch();
   return cudaGetLastError();

@@ -327,6 +327,11 @@ __global__ void __launch_bounds__(TP_THREADS) tpacf_fi_kernel(const TPFIParams q
 // ============================================================================================
 // Host launchers
 // ============================================================================================
+static double tp_pairs(const TPParams& p) {
+  const double n = p.n;
+  return (1 + p.nr) * n * (n - 1) / 2 + p.nr * n * n;
+}
+
 static TPParams tp_params(const hk_tpacf_args& a, const DevRanges& R, int ndet, hk_control* cb, float* samples) {
   TPParams p{};
   p.pts = a.pts;
@@ -355,6 +360,7 @@ static cudaError_t launch_tp_v(const TPParams& p, cudaStream_t s) {
   }
   dim3 grid((p.n + TP_THREADS - 1) / TP_THREADS, (1 + 2 * p.nr) * p.nC);
   if (grid.x == 0) return cudaSuccess;
+  TimedScope ts(HK_TPACF, 0, tp_pairs(p), s);
   tpacf_kernel<V><<<grid, TP_THREADS, sizeof(TPShared), s>>>(p);
   count_launch();
   return cudaGetLastError();
@@ -387,6 +393,7 @@ static cudaError_t launch_tp_fi_k(const TPFIParams& q, int nrep, cudaStream_t s)
     attr = true;
   }
   dim3 grid((q.base.n + TP_THREADS - 1) / TP_THREADS, (1 + 2 * q.base.nr) * q.base.nC, nrep);
+  TimedScope ts(HK_TPACF, 1, tp_pairs(q.base) * nrep, s);
   tpacf_fi_kernel<KIND><<<grid, TP_THREADS, sizeof(TPShared), s>>>(q);
   count_launch();
   return cudaGetLastError();

@@ -113,13 +113,18 @@ def lib():
         L.hauberk_last_error.argtypes = []
         L.hauberk_version.restype = I32
         L.hauberk_launch_count.restype = U64
+        L.hauberk_timing_enable.restype = None
+        L.hauberk_timing_enable.argtypes = [I32]
+        L.hauberk_timing_read.restype = I32
+        L.hauberk_timing_read.argtypes = [I32, I32, P, P, P]
         _lib = L
     return _lib
 
 
 EXPORTED = ["hauberk_run_cp", "hauberk_run_mriq", "hauberk_run_tpacf", "hauberk_profile_ranges",
             "hauberk_inject_campaign", "hauberk_decode", "hauberk_num_sites", "hauberk_strerror",
-            "hauberk_last_error", "hauberk_version", "hauberk_launch_count"]
+            "hauberk_last_error", "hauberk_version", "hauberk_launch_count", "hauberk_timing_enable",
+            "hauberk_timing_read"]
 
 
 def _check(status: int, where: str):
@@ -145,6 +150,17 @@ def _ptr(t: torch.Tensor | None):
 
 def launch_count() -> int:
     return int(lib().hauberk_launch_count())
+
+
+def timing_enable(on: bool = True):
+    lib().hauberk_timing_enable(1 if on else 0)
+
+
+def timing_read(bench: int, cls: int):
+    """(device ms, launches, pairs) of the main (cls 0) or FI replica (cls 1) kernels since the last read."""
+    ms, n, w = C.c_double(), C.c_int64(), C.c_double()
+    _check(lib().hauberk_timing_read(bench, cls, C.byref(ms), C.byref(n), C.byref(w)), "hauberk_timing_read")
+    return ms.value, n.value, w.value
 
 
 def version() -> int:

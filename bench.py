@@ -98,13 +98,20 @@ class Clocks:
 # ------------------------------------------------------------------------------------------------------
 # reference arm: the CPU oracle, as it stands, on the same metric (replica-mode injections/s)
 # ------------------------------------------------------------------------------------------------------
+_ORACLE_SETUP = {}
+
+
 def oracle_replica_sample(seed: int, first: int, count: int):
-    """Time `count` consecutive config-5 injections in the oracle's replica mode (full program per injection)."""
+    """Time `count` consecutive config-5 injections in the oracle's replica mode (full program per injection).
+    Inputs and the oracle's own profiled ranges are prepared once, outside the timing."""
     import oracle as O
     import workloads as W
 
-    probs = [W.cp_config1(), W.mriq_config2(), W.tpacf_config3()]
-    R = [O.profile_ranges(b, probs[b]) for b in range(3)]
+    if not _ORACLE_SETUP:
+        probs = [W.cp_config1(), W.mriq_config2(), W.tpacf_config3()]
+        _ORACLE_SETUP["probs"] = probs
+        _ORACLE_SETUP["R"] = [O.profile_ranges(b, probs[b]) for b in range(3)]
+    probs, R = _ORACLE_SETUP["probs"], _ORACLE_SETUP["R"]
     per = {0: [], 1: [], 2: []}
     for n in range(first, first + count):
         b = n % 3
@@ -122,11 +129,11 @@ def run_reference(args):
     import oracle as O
     O.build()
     step_t = []
+    oracle_replica_sample(seed, 0, 0)  # setup (inputs, profiled ranges) outside the timing
     for s in range(args.warmup + args.steps):
-        t0 = time.perf_counter()
-        oracle_replica_sample(seed, 3 * s, 3)  # one injection of each benchmark per step
+        per = oracle_replica_sample(seed, 3 * s, 3)  # one injection of each benchmark per step
         if s >= args.warmup:
-            step_t.append(time.perf_counter() - t0)
+            step_t.append(sum(sum(v) for v in per.values()))
     tot = sum(step_t)
     v = 3 * args.steps / tot
     line = {"metric": METRIC, "value": v, "unit": "injections/s", "impl": "reference", "n_gpus": args.gpus,
@@ -215,9 +222,11 @@ def main():
     counts = torch.zeros((3, 5), dtype=torch.int64, device=dev)
     scratch = torch.zeros((3, 5), dtype=torch.int64, device=dev)
 
+    session = hk.CampaignSession(-1, devs, ranges, seed, batch=args.batch)
+
     def step(s, into):
         first, cnt = par.step_slice(s, rank, world, args.per_rank)
-        hk.inject_campaign(-1, devs, ranges, seed, first, cnt, into, batch=args.batch)
+        session.run(first, cnt, into)
 
     for s in range(args.warmup):
         flush.zero_()
@@ -301,6 +310,7 @@ def main():
                "sample": "6 config-5 injections (2 each CP-s / MRI-Q / TPACF), replica mode (full program run each), "
                          f"mean s/injection cp={tm[0]:.4f} mriq={tm[1]:.3f} tpacf={tm[2]:.3f}"}
 
+    session.close()
     if rank == 0:
         line = {
             "metric": METRIC, "value": round(value, 2), "unit": "injections/s", "n_gpus": world, "steps": args.steps,

@@ -153,6 +153,18 @@ HK_API hk_status hauberk_inject_campaign(int32_t bench_mode, const void* const a
                                   hk_outcome* d_records, int64_t* d_counts, int64_t* d_site_counts,
                                   void* stream);
 
+/* Campaign session (the same campaign, prepared once): create validates, runs the golden programs,
+ * checks they raise no alarm (synchronises `stream` once) and allocates the replica workspaces;
+ * each run enqueues injections [first, first+count) on that stream without synchronising (the
+ * device pointers inside the args must stay valid until destroy); destroy synchronises and frees.
+ * hauberk_inject_campaign = create + run + destroy. */
+typedef struct hk_campaign_session hk_campaign_session;
+HK_API hk_status hauberk_campaign_create(int32_t bench_mode, const void* const args[3], const hk_ranges* const ranges[3],
+                                         const hk_campaign* campaign, hk_campaign_session** out, void* stream);
+HK_API hk_status hauberk_campaign_run(hk_campaign_session* session, int64_t first, int64_t count, hk_outcome* d_records,
+                                      int64_t* d_counts, int64_t* d_site_counts);
+HK_API void hauberk_campaign_destroy(hk_campaign_session* session);
+
 /* Host-side decode of injections [first, first+count) (same rule the campaign uses). */
 HK_API hk_status hauberk_decode(int32_t bench_mode, const void* const args[3], const uint64_t site_mask[3],
                          uint64_t seed, int64_t first, int64_t count, int32_t* bench_out, hk_fault* out);

@@ -30,7 +30,9 @@ cudaError_t cp_launch(int vflags, const hk_cp_args& a, const DevRanges& R, int n
 cudaError_t mriq_launch(int vflags, const hk_mriq_args& a, const DevRanges& R, int ndet, hk_control* cb,
                         float* samples, cudaStream_t s);
 cudaError_t tpacf_launch(int vflags, const hk_tpacf_args& a, const DevRanges& R, int ndet, hk_control* cb,
-                         float* samples, cudaStream_t s);
+                         float* samples, void* lut_ws, cudaStream_t s);
+size_t tpacf_lut_ws_bytes();
+cudaError_t tpacf_lut_build(const hk_tpacf_args& a, void* lut_ws, cudaStream_t s);
 cudaError_t cp_prepass_launch(const hk_cp_args& a, cudaStream_t s);
 cudaError_t mriq_phimag_launch(const hk_mriq_args& a, bool nl, hk_control* cb, cudaStream_t s);
 
@@ -43,7 +45,7 @@ cudaError_t cp_fi_launch(int kind, const hk_cp_args& a, const DevRanges& R, int 
 cudaError_t mriq_fi_launch(int kind, const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
                            int nrep, float* out0, int64_t stride, hk_control* cb0, cudaStream_t s);
 cudaError_t tpacf_fi_launch(int kind, const hk_tpacf_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
-                            int nrep, unsigned long long* hist0, hk_control* cb0, cudaStream_t s);
+                            int nrep, unsigned long long* hist0, hk_control* cb0, void* lut_ws, cudaStream_t s);
 
 // classify.cu
 cudaError_t control_init_launch(hk_control* cb, int n, cudaStream_t s);

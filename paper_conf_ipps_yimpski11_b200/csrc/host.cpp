@@ -172,7 +172,11 @@ static hk_status run_bench(int b, const void* args, int variant, const hk_ranges
     ndet = std::min(ndet, 1);
     HK_CUDA(cudaMemsetAsync(a->hist, 0, sizeof(unsigned long long) * (size_t)(1 + 2 * a->n_rand) * (a->n_bins + 2), s),
             "memset hist");
-    HK_CUDA(tpacf_launch(vf, *a, R, ndet, d_cb, d_samples, s), "tpacf kernel");
+    void* lut = nullptr;
+    HK_CUDA(cudaMallocAsync(&lut, tpacf_lut_ws_bytes(), s), "alloc tpacf table");
+    cudaError_t e = tpacf_launch(vf, *a, R, ndet, d_cb, d_samples, lut, s);
+    cudaFreeAsync(lut, s);
+    HK_CUDA(e, "tpacf kernel");
   }
   return HK_OK;
 }
@@ -330,6 +334,7 @@ struct BenchWS {
   void* rep_out = nullptr;
   hk_control* rep_cb = nullptr;
   hk_control* gold_cb = nullptr;
+  void* lut = nullptr;  // TPACF bucket table
   int batch = 0;
 };
 
@@ -489,101 +494,163 @@ hk_status hauberk_decode(int32_t bench_mode, const void* const args[3], const ui
   return HK_OK;
 }
 
-hk_status hauberk_inject_campaign(int32_t bench_mode, const void* const args[3], const hk_ranges* const ranges[3],
-                                  const hk_campaign* C, hk_outcome* d_records, int64_t* d_counts, int64_t* d_site_counts,
-                                  void* stream) {
-  if (!args || !ranges || !C || !d_counts || bench_mode < -1 || bench_mode > 2) return invalid("campaign: bad arguments");
-  if (C->count < 0 || C->first < 0) return invalid("campaign: bad index range");
-  if (C->mode != 0) { g_err = "only replica mode (0) is implemented on the GPU"; return HK_ERR_UNSUPPORTED; }
-  if (C->nbits != 0 && C->nbits != 1) { g_err = "multi-bit masks are NEXT (f1)"; return HK_ERR_UNSUPPORTED; }
-  if (C->count == 0) return HK_OK;
-  cudaStream_t s = (cudaStream_t)stream;
+}  // extern "C"
+
+// ---------------------------------------------------------------------------------------------
+// Campaign session: golden runs, catalogues and replica workspaces prepared once; each
+// hauberk_campaign_run enqueues one slice of injections without synchronising.
+// ---------------------------------------------------------------------------------------------
+struct hk_campaign_session {
+  int bench_mode = -1;
+  hk_campaign cfg{};
+  hk_cp_args cp{};
+  hk_mriq_args mq{};
+  hk_tpacf_args tp{};
   BenchWS W[3];
   Catalog K[3];
-  for (int b = 0; b < 3; ++b) {
-    const bool used = bench_mode == b || (bench_mode == -1 && C->count > (b - C->first % 3 + 3) % 3);
-    if (!used) continue;
-    if (!args_ok(b, args[b])) return invalid("campaign: args of a used benchmark are invalid");
-    if (!ranges[b] || ranges[b]->n_det <= 0) { g_err = "campaign: ranges missing"; return HK_ERR_NO_RANGES; }
-    if (b == HK_CP && ((const hk_cp_args*)args[b])->unroll != 4) { g_err = "campaign kernels are built for CP unroll 4"; return HK_ERR_UNSUPPORTED; }
-    if (b == HK_TPACF && !tpacf_edges_ok((const hk_tpacf_args*)args[b], s)) return invalid("edges must strictly decrease");
-    if (!build_catalog(K[b], b, args[b], C->site_mask[b])) return invalid("campaign: empty site catalogue");
-    W[b].used = true;
-    W[b].args = args[b];
-    W[b].R = dev_ranges(ranges[b]);
-    W[b].ndet = ranges[b]->n_det;
-    W[b].batch = C->batch > 0 ? C->batch : default_batch(b, args[b]);
-  }
+  FaultRec* d_faults = nullptr;
+  size_t d_cap = 0;
+  FaultRec* h_faults = nullptr;  // pinned staging
+  size_t h_cap = 0;
+  cudaEvent_t uploaded = nullptr;
+  cudaStream_t stream = nullptr;
+};
 
-  // ---- golden (fault-free FT) runs; their outputs stay in the caller's buffers' copies
-  auto cleanup = [&]() {
-    for (int b = 0; b < 3; ++b) {
-      if (W[b].golden) cudaFreeAsync(W[b].golden, s);
-      if (W[b].dM) cudaFreeAsync(W[b].dM, s);
-      if (W[b].rep_out) cudaFreeAsync(W[b].rep_out, s);
-      if (W[b].rep_cb) cudaFreeAsync(W[b].rep_cb, s);
-      if (W[b].gold_cb) cudaFreeAsync(W[b].gold_cb, s);
-    }
-  };
+static void session_free(hk_campaign_session* S) {
+  if (!S) return;
+  if (S->stream) cudaStreamSynchronize(S->stream);
+  for (int b = 0; b < 3; ++b) {
+    BenchWS& w = S->W[b];
+    if (w.golden) cudaFree(w.golden);
+    if (w.dM) cudaFree(w.dM);
+    if (w.rep_out) cudaFree(w.rep_out);
+    if (w.rep_cb) cudaFree(w.rep_cb);
+    if (w.gold_cb) cudaFree(w.gold_cb);
+    if (w.lut) cudaFree(w.lut);
+  }
+  if (S->d_faults) cudaFree(S->d_faults);
+  if (S->h_faults) cudaFreeHost(S->h_faults);
+  if (S->uploaded) cudaEventDestroy(S->uploaded);
+  delete S;
+}
+
+static void keep_pool_memory() {
+  static bool done = false;
+  if (done) return;
+  int dev = 0;
+  cudaMemPool_t pool;
+  if (cudaGetDevice(&dev) == cudaSuccess && cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+    uint64_t thr = UINT64_MAX;
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+  }
+  done = true;
+}
+
+static hk_status session_create(int32_t bench_mode, const void* const args[3], const hk_ranges* const ranges[3],
+                                const hk_campaign* C, cudaStream_t s, hk_campaign_session** out) {
+  if (!args || !ranges || !C || !out || bench_mode < -1 || bench_mode > 2) return invalid("campaign: bad arguments");
+  if (C->mode != 0) { g_err = "only replica mode (0) is implemented on the GPU"; return HK_ERR_UNSUPPORTED; }
+  if (C->nbits != 0 && C->nbits != 1) { g_err = "multi-bit masks are NEXT (f1)"; return HK_ERR_UNSUPPORTED; }
+  keep_pool_memory();
+  hk_campaign_session* S = new hk_campaign_session();
+  S->bench_mode = bench_mode;
+  S->cfg = *C;
+  S->stream = s;
   hk_status st = HK_OK;
+  cudaError_t e;
   for (int b = 0; b < 3 && st == HK_OK; ++b) {
-    if (!W[b].used) continue;
-    BenchWS& w = W[b];
+    const bool want = bench_mode == b || (bench_mode == -1 && args[b] != nullptr);
+    if (!want) continue;
+    if (!args_ok(b, args[b])) { st = invalid("campaign: args of a used benchmark are invalid"); break; }
+    if (!ranges[b] || ranges[b]->n_det <= 0) { g_err = "campaign: ranges missing"; st = HK_ERR_NO_RANGES; break; }
+    if (b == HK_CP && ((const hk_cp_args*)args[b])->unroll != 4) {
+      g_err = "campaign kernels are built for CP unroll 4"; st = HK_ERR_UNSUPPORTED; break;
+    }
+    if (b == HK_TPACF && !tpacf_edges_ok((const hk_tpacf_args*)args[b], s)) { st = invalid("edges must strictly decrease"); break; }
+    const void* own = b == HK_CP ? (const void*)&S->cp : (b == HK_MRIQ ? (const void*)&S->mq : (const void*)&S->tp);
+    if (b == HK_CP) S->cp = *(const hk_cp_args*)args[b];
+    else if (b == HK_MRIQ) S->mq = *(const hk_mriq_args*)args[b];
+    else S->tp = *(const hk_tpacf_args*)args[b];
+    if (!build_catalog(S->K[b], b, own, C->site_mask[b])) { st = invalid("campaign: empty site catalogue"); break; }
+    BenchWS& w = S->W[b];
+    w.used = true;
+    w.args = own;
+    w.R = dev_ranges(ranges[b]);
+    w.ndet = ranges[b]->n_det;
+    w.batch = C->batch > 0 ? C->batch : default_batch(b, own);
     size_t esz = sizeof(float);
-    if (b == HK_CP) { const hk_cp_args* a = (const hk_cp_args*)w.args; w.out_elems = (int64_t)a->nx * a->ny; }
-    else if (b == HK_MRIQ) { const hk_mriq_args* a = (const hk_mriq_args*)w.args; w.out_elems = 2LL * a->n_vox; }
-    else { const hk_tpacf_args* a = (const hk_tpacf_args*)w.args; w.out_elems = (int64_t)(1 + 2 * a->n_rand) * (a->n_bins + 2); esz = 8; }
+    if (b == HK_CP) w.out_elems = (int64_t)S->cp.nx * S->cp.ny;
+    else if (b == HK_MRIQ) w.out_elems = 2LL * S->mq.n_vox;
+    else { w.out_elems = (int64_t)(1 + 2 * S->tp.n_rand) * (S->tp.n_bins + 2); esz = 8; }
     const int64_t stride = (w.out_elems + 3) / 4 * 4;  // keep replicas 16-byte aligned
     w.out_elems = stride;
-    cudaError_t e;
-    if ((e = cudaMallocAsync(&w.golden, esz * stride, s)) != cudaSuccess) { st = cuda_fail(e, "alloc golden"); break; }
-    if ((e = cudaMallocAsync((void**)&w.dM, sizeof(float), s)) != cudaSuccess) { st = cuda_fail(e, "alloc M"); break; }
-    if ((e = cudaMallocAsync((void**)&w.gold_cb, sizeof(hk_control), s)) != cudaSuccess) { st = cuda_fail(e, "alloc cb"); break; }
-    if ((e = cudaMallocAsync(&w.rep_out, esz * stride * w.batch, s)) != cudaSuccess) { st = cuda_fail(e, "alloc replicas"); break; }
-    if ((e = cudaMallocAsync((void**)&w.rep_cb, sizeof(hk_control) * w.batch, s)) != cudaSuccess) { st = cuda_fail(e, "alloc replica cbs"); break; }
-    if ((e = cudaMemsetAsync(w.golden, 0, esz * stride, s)) != cudaSuccess) { st = cuda_fail(e, "memset"); break; }
-    if ((e = cudaMemsetAsync(w.rep_out, 0, esz * stride * w.batch, s)) != cudaSuccess) { st = cuda_fail(e, "memset"); break; }
-    if ((e = control_init_launch(w.rep_cb, w.batch, s)) != cudaSuccess) { st = cuda_fail(e, "cb init"); break; }
+    if ((e = cudaMalloc(&w.golden, esz * stride)) != cudaSuccess ||
+        (e = cudaMalloc((void**)&w.dM, sizeof(float))) != cudaSuccess ||
+        (e = cudaMalloc((void**)&w.gold_cb, sizeof(hk_control))) != cudaSuccess ||
+        (e = cudaMalloc(&w.rep_out, esz * stride * w.batch)) != cudaSuccess ||
+        (e = cudaMalloc((void**)&w.rep_cb, sizeof(hk_control) * w.batch)) != cudaSuccess) {
+      st = cuda_fail(e, "campaign workspace");
+      break;
+    }
+    if ((e = cudaMemsetAsync(w.golden, 0, esz * stride, s)) != cudaSuccess ||
+        (e = cudaMemsetAsync(w.rep_out, 0, esz * stride * w.batch, s)) != cudaSuccess ||
+        (e = control_init_launch(w.rep_cb, w.batch, s)) != cudaSuccess) {
+      st = cuda_fail(e, "campaign init");
+      break;
+    }
     // golden = this library's own fault-free FT output (R7)
     if (b == HK_CP) {
-      hk_cp_args a = *(const hk_cp_args*)w.args;
+      hk_cp_args a = S->cp;
       a.grid = (float*)w.golden;
       st = run_bench(b, &a, HK_FT, ranges[b], w.gold_cb, nullptr, s);
       if (st == HK_OK && (e = max_abs_launch((float*)w.golden, (int64_t)a.nx * a.ny, w.dM, s)) != cudaSuccess) st = cuda_fail(e, "max");
     } else if (b == HK_MRIQ) {
-      hk_mriq_args a = *(const hk_mriq_args*)w.args;
+      hk_mriq_args a = S->mq;
       a.qr = (float*)w.golden;
       a.qi = a.qr + a.n_vox;
       st = run_bench(b, &a, HK_FT, ranges[b], w.gold_cb, nullptr, s);
       if (st == HK_OK && (e = max_abs_launch((float*)w.golden, 2LL * a.n_vox, w.dM, s)) != cudaSuccess) st = cuda_fail(e, "max");
     } else {
-      hk_tpacf_args a = *(const hk_tpacf_args*)w.args;
+      hk_tpacf_args a = S->tp;
       a.hist = (unsigned long long*)w.golden;
       st = run_bench(b, &a, HK_FT, ranges[b], w.gold_cb, nullptr, s);
+      if (st == HK_OK && (e = cudaMalloc(&w.lut, tpacf_lut_ws_bytes())) != cudaSuccess) st = cuda_fail(e, "alloc table");
+      if (st == HK_OK && (e = tpacf_lut_build(a, w.lut, s)) != cudaSuccess) st = cuda_fail(e, "table");
     }
   }
-  if (st != HK_OK) { cleanup(); return st; }
-  {
+  if (st == HK_OK && !(S->W[0].used || S->W[1].used || S->W[2].used)) st = invalid("campaign: no benchmark");
+  if (st == HK_OK) {
     hk_control hc[3];
     for (int b = 0; b < 3; ++b)
-      if (W[b].used) cudaMemcpyAsync(&hc[b], W[b].gold_cb, sizeof(hk_control), cudaMemcpyDeviceToHost, s);
-    cudaError_t e = cudaStreamSynchronize(s);
-    if (e != cudaSuccess) { cleanup(); return cuda_fail(e, "golden runs"); }
-    for (int b = 0; b < 3; ++b)
-      if (W[b].used && (hc[b].alarm != 0 || hc[b].fail != 0)) {
-        cleanup();
+      if (S->W[b].used) cudaMemcpyAsync(&hc[b], S->W[b].gold_cb, sizeof(hk_control), cudaMemcpyDeviceToHost, s);
+    if ((e = cudaStreamSynchronize(s)) != cudaSuccess) st = cuda_fail(e, "golden runs");
+    for (int b = 0; b < 3 && st == HK_OK; ++b)
+      if (S->W[b].used && (hc[b].alarm != 0 || hc[b].fail != 0)) {
         g_err = "golden run alarm (ranges were not profiled on this input)";
-        return HK_ERR_GOLDEN_ALARM;
+        st = HK_ERR_GOLDEN_ALARM;
       }
   }
+  if (st == HK_OK && (e = cudaEventCreateWithFlags(&S->uploaded, cudaEventDisableTiming)) != cudaSuccess)
+    st = cuda_fail(e, "event");
+  if (st != HK_OK) { session_free(S); return st; }
+  *out = S;
+  return HK_OK;
+}
 
-  // ---- decode, group by (bench, kind), upload
+static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t count, hk_outcome* d_records,
+                             int64_t* d_counts, int64_t* d_site_counts) {
+  if (!S || !d_counts || first < 0 || count < 0) return invalid("campaign_run: bad arguments");
+  if (count == 0) return HK_OK;
+  cudaStream_t s = S->stream;
+  cudaError_t e;
+  // ---- decode, group by (bench, kind)
   struct Item { int b, kind; FaultRec f; };
-  std::vector<Item> items((size_t)C->count);
-  for (int64_t q = 0; q < C->count; ++q) {
-    const int64_t n = C->first + q;
-    const int b = bench_mode >= 0 ? bench_mode : (int)(n % 3);
-    const hk_fault hf = decode_one(K[b], C->seed, n);
+  std::vector<Item> items((size_t)count);
+  for (int64_t q = 0; q < count; ++q) {
+    const int64_t n = first + q;
+    const int b = S->bench_mode >= 0 ? S->bench_mode : (int)(n % 3);
+    if (!S->W[b].used) return invalid("campaign_run: index hits a benchmark the session was not created with");
+    const hk_fault hf = decode_one(S->K[b], S->cfg.seed, n);
     Item it{};
     it.b = b;
     it.f.index = n; it.f.thread = hf.thread; it.f.inst = hf.inst; it.f.mask = hf.mask; it.f.site = hf.site;
@@ -597,51 +664,96 @@ hk_status hauberk_inject_campaign(int32_t bench_mode, const void* const args[3],
   std::stable_sort(items.begin(), items.end(), [](const Item& x, const Item& y) {
     return x.b != y.b ? x.b < y.b : x.kind < y.kind;
   });
-  std::vector<FaultRec> recs(items.size());
-  for (size_t q = 0; q < items.size(); ++q) recs[q] = items[q].f;
-  FaultRec* d_faults = nullptr;
-  cudaError_t e = cudaMallocAsync((void**)&d_faults, sizeof(FaultRec) * recs.size(), s);
-  if (e != cudaSuccess) { cleanup(); return cuda_fail(e, "alloc faults"); }
-  e = cudaMemcpyAsync(d_faults, recs.data(), sizeof(FaultRec) * recs.size(), cudaMemcpyHostToDevice, s);
-  if (e != cudaSuccess) { cudaFreeAsync(d_faults, s); cleanup(); return cuda_fail(e, "upload faults"); }
+  // ---- upload through the pinned staging buffer (wait until the previous upload consumed it)
+  if ((e = cudaEventSynchronize(S->uploaded)) != cudaSuccess) return cuda_fail(e, "staging");
+  if (S->h_cap < items.size()) {
+    if (S->h_faults) cudaFreeHost(S->h_faults);
+    S->h_faults = nullptr;
+    S->h_cap = 0;
+    if ((e = cudaMallocHost((void**)&S->h_faults, sizeof(FaultRec) * items.size())) != cudaSuccess) return cuda_fail(e, "pinned");
+    S->h_cap = items.size();
+  }
+  if (S->d_cap < items.size()) {
+    if (S->d_faults) cudaFreeAsync(S->d_faults, s);
+    S->d_faults = nullptr;
+    S->d_cap = 0;
+    if ((e = cudaMallocAsync((void**)&S->d_faults, sizeof(FaultRec) * items.size(), s)) != cudaSuccess) return cuda_fail(e, "faults");
+    S->d_cap = items.size();
+  }
+  for (size_t q = 0; q < items.size(); ++q) S->h_faults[q] = items[q].f;
+  if ((e = cudaMemcpyAsync(S->d_faults, S->h_faults, sizeof(FaultRec) * items.size(), cudaMemcpyHostToDevice, s)) != cudaSuccess)
+    return cuda_fail(e, "upload faults");
+  cudaEventRecord(S->uploaded, s);
 
   // ---- batches: FI&FT replicas, then the classify epilogue (which also recycles the workspace)
   size_t q = 0;
-  while (q < items.size() && st == HK_OK) {
+  while (q < items.size()) {
     const int b = items[q].b, kind = items[q].kind;
     size_t end = q;
-    while (end < items.size() && items[end].b == b && items[end].kind == kind && (int)(end - q) < W[b].batch) ++end;
+    while (end < items.size() && items[end].b == b && items[end].kind == kind && (int)(end - q) < S->W[b].batch) ++end;
     const int nrep = (int)(end - q);
-    BenchWS& w = W[b];
-    const FaultRec* fr = d_faults + q;
+    BenchWS& w = S->W[b];
+    const FaultRec* fr = S->d_faults + q;
     if (b == HK_CP) {
-      const hk_cp_args* a = (const hk_cp_args*)w.args;
-      if ((e = cp_fi_launch(kind, *a, w.R, std::min(w.ndet, 4), fr, nrep, (float*)w.rep_out, w.out_elems, w.rep_cb, s)) != cudaSuccess)
-        st = cuda_fail(e, "cp FI");
-      else if ((e = classify_fp_launch(b, (float*)w.rep_out, w.out_elems, (const float*)w.golden, w.dM, w.rep_cb, fr, nrep,
-                                       d_records, C->first, d_counts, d_site_counts, s)) != cudaSuccess)
-        st = cuda_fail(e, "classify");
+      if ((e = cp_fi_launch(kind, S->cp, w.R, std::min(w.ndet, 4), fr, nrep, (float*)w.rep_out, w.out_elems, w.rep_cb, s)) != cudaSuccess)
+        return cuda_fail(e, "cp FI");
+      if ((e = classify_fp_launch(b, (float*)w.rep_out, w.out_elems, (const float*)w.golden, w.dM, w.rep_cb, fr, nrep,
+                                  d_records, first, d_counts, d_site_counts, s)) != cudaSuccess)
+        return cuda_fail(e, "classify");
     } else if (b == HK_MRIQ) {
-      const hk_mriq_args* a = (const hk_mriq_args*)w.args;
-      if ((e = mriq_fi_launch(kind, *a, w.R, std::min(w.ndet, 2), fr, nrep, (float*)w.rep_out, w.out_elems, w.rep_cb, s)) != cudaSuccess)
-        st = cuda_fail(e, "mriq FI");
-      else if ((e = classify_fp_launch(b, (float*)w.rep_out, w.out_elems, (const float*)w.golden, w.dM, w.rep_cb, fr, nrep,
-                                       d_records, C->first, d_counts, d_site_counts, s)) != cudaSuccess)
-        st = cuda_fail(e, "classify");
+      if ((e = mriq_fi_launch(kind, S->mq, w.R, std::min(w.ndet, 2), fr, nrep, (float*)w.rep_out, w.out_elems, w.rep_cb, s)) != cudaSuccess)
+        return cuda_fail(e, "mriq FI");
+      if ((e = classify_fp_launch(b, (float*)w.rep_out, w.out_elems, (const float*)w.golden, w.dM, w.rep_cb, fr, nrep,
+                                  d_records, first, d_counts, d_site_counts, s)) != cudaSuccess)
+        return cuda_fail(e, "classify");
     } else {
-      const hk_tpacf_args* a = (const hk_tpacf_args*)w.args;
-      if ((e = tpacf_fi_launch(kind, *a, w.R, std::min(w.ndet, 1), fr, nrep, (unsigned long long*)w.rep_out, w.rep_cb, s)) !=
-          cudaSuccess)
-        st = cuda_fail(e, "tpacf FI");
-      else if ((e = classify_tpacf_launch((unsigned long long*)w.rep_out, a->n_rand, a->n_bins,
-                                          (const unsigned long long*)w.golden, w.rep_cb, fr, nrep, d_records, C->first,
-                                          d_counts, d_site_counts, s)) != cudaSuccess)
-        st = cuda_fail(e, "classify");
+      if ((e = tpacf_fi_launch(kind, S->tp, w.R, std::min(w.ndet, 1), fr, nrep, (unsigned long long*)w.rep_out, w.rep_cb,
+                               w.lut, s)) != cudaSuccess)
+        return cuda_fail(e, "tpacf FI");
+      if ((e = classify_tpacf_launch((unsigned long long*)w.rep_out, S->tp.n_rand, S->tp.n_bins,
+                                     (const unsigned long long*)w.golden, w.rep_cb, fr, nrep, d_records, first, d_counts,
+                                     d_site_counts, s)) != cudaSuccess)
+        return cuda_fail(e, "classify");
     }
     q = end;
   }
-  cudaFreeAsync(d_faults, s);
-  cleanup();
+  return HK_OK;
+}
+
+extern "C" {
+
+hk_status hauberk_campaign_create(int32_t bench_mode, const void* const args[3], const hk_ranges* const ranges[3],
+                                  const hk_campaign* campaign, hk_campaign_session** out, void* stream) {
+  return session_create(bench_mode, args, ranges, campaign, (cudaStream_t)stream, out);
+}
+
+hk_status hauberk_campaign_run(hk_campaign_session* session, int64_t first, int64_t count, hk_outcome* d_records,
+                               int64_t* d_counts, int64_t* d_site_counts) {
+  return session_run(session, first, count, d_records, d_counts, d_site_counts);
+}
+
+void hauberk_campaign_destroy(hk_campaign_session* session) { session_free(session); }
+
+hk_status hauberk_inject_campaign(int32_t bench_mode, const void* const args[3], const hk_ranges* const ranges[3],
+                                  const hk_campaign* C, hk_outcome* d_records, int64_t* d_counts, int64_t* d_site_counts,
+                                  void* stream) {
+  if (!args || !ranges || !C || !d_counts || bench_mode < -1 || bench_mode > 2) return invalid("campaign: bad arguments");
+  if (C->count < 0 || C->first < 0) return invalid("campaign: bad index range");
+  if (C->count == 0) return HK_OK;
+  // prepare only the benchmarks this index range touches
+  const void* used_args[3] = {nullptr, nullptr, nullptr};
+  for (int b = 0; b < 3; ++b) {
+    const bool used = bench_mode == b || (bench_mode == -1 && C->count > (b - C->first % 3 + 3) % 3);
+    if (used) {
+      if (!args[b]) return invalid("campaign: args of a used benchmark are missing");
+      used_args[b] = args[b];
+    }
+  }
+  hk_campaign_session* S = nullptr;
+  hk_status st = session_create(bench_mode, used_args, ranges, C, (cudaStream_t)stream, &S);
+  if (st != HK_OK) return st;
+  st = session_run(S, C->first, C->count, d_records, d_counts, d_site_counts);
+  session_free(S);
   return st;
 }
 

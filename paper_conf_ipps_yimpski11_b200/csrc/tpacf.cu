@@ -19,6 +19,8 @@ constexpr int TP_CMAX = 1024;  // max chunk (partners per abstract thread)
 struct TPParams {
   const float* pts;
   const float* edges;
+  const int2* lut;     // [TP_LUT] (bmin, bits(edge[bmin])) per u-bucket; built by tpacf_lut_kernel
+  const int* lut_ok;   // 1 if every bucket holds at most one edge (else: binary search)
   unsigned long long* hist;
   hk_control* cb;
   float* samples;
@@ -28,11 +30,15 @@ struct TPParams {
   int32_t one;
 };
 
-struct TPShared {
-  float4 B[TP_CMAX];
-  float E[32];
-  uint32_t H[TP_WARPS][32][32];  // [warp][bin][lane]
-};
+// ---------------------------------------------------------------------------------------------
+// Binning.  Definition: bin = #{e in [0, nb] : dot < edge[e]}, edges decreasing.
+//  * tp_bin: branch-free 5-step binary search over the edges (padded with -inf) in shared memory.
+//  * LUT path: u = fl(1 - dot) is monotone in dot, and so is bin; bucket u by its top 11 bits
+//    (sign, exponent, 2 mantissa bits).  For every bucket q the device builds
+//    bmin = bin(largest dot mapping into q) and checks that the smallest dot of q has
+//    bin <= bmin + 1, so bin = bmin + (dot < edge[bmin]) exactly.  2 loads + 4 ops per pair.
+// ---------------------------------------------------------------------------------------------
+constexpr int TP_LUT = 2048;
 
 __device__ __forceinline__ int32_t tp_bin(const float* Es, float dot) {
   int32_t b = 0;
@@ -40,32 +46,116 @@ __device__ __forceinline__ int32_t tp_bin(const float* Es, float dot) {
   for (int s = 16; s >= 1; s >>= 1) b += (dot < Es[b + s - 1]) ? s : 0;
   return b;
 }
+__device__ __forceinline__ int32_t tp_bin_lut(const int2* L, float dot) {
+  const float u = __fsub_rn(1.0f, dot);
+  const int2 e = L[fb(u) >> 21];
+  return e.x + ((dot < __int_as_float(e.y)) ? 1 : 0);
+}
 
-// Stage chunk c of partner set sb, the edges, and clear the histograms.  Called by all threads.
-__device__ __forceinline__ void tp_stage(const TPParams& p, TPShared& S, int sb, int c) {
+__device__ __forceinline__ float nup(float x) {
+  const uint32_t b = fb(x);
+  if ((b & 0x7fffffffu) == 0) return bf(1u);
+  return (b & 0x80000000u) ? bf(b - 1) : bf(b + 1);
+}
+__device__ __forceinline__ float ndown(float x) {
+  const uint32_t b = fb(x);
+  if ((b & 0x7fffffffu) == 0) return bf(0x80000001u);
+  return (b & 0x80000000u) ? bf(b + 1) : bf(b - 1);
+}
+__device__ __forceinline__ int32_t bin_def(const float* edges, int nb, float dot) {
+  int32_t b = 0;
+  for (int e = 0; e <= nb; ++e) b += (dot < edges[e]) ? 1 : 0;
+  return b;
+}
+
+// One thread per bucket q.  Buckets whose u range holds no finite value (inf/NaN exponents) map
+// to bin 0 for NaN (the definition: every compare with NaN is false) and nb+1 for +inf.
+__global__ void tpacf_lut_kernel(const float* __restrict__ edges, int nb, int2* __restrict__ lut, int* ok) {
+  const int q = blockIdx.x * blockDim.x + threadIdx.x;
+  if (q >= TP_LUT) return;
+  const float e0 = edges[0];
+  int2 out = make_int2(0, fb(e0));
+  bool good = true;
+  const uint32_t lo_bits = (uint32_t)q << 21, hi_bits = lo_bits | 0x1fffffu;
+  const bool neg = (lo_bits & 0x80000000u) != 0;
+  const bool special = ((lo_bits >> 23) & 0xffu) == 0xffu;  // inf / NaN exponent
+  if (neg) {
+    out = make_int2(0, fb(e0));  // u <= -0: dot >= 1 > every edge -> bin 0 (and -NaN: bin 0)
+  } else if (special) {
+    out = (q == (int)(0x7f800000u >> 21)) ? make_int2(nb + 1, (int)0xff800000u) : make_int2(0, fb(e0));
+  } else {
+    const float ulo = bf(lo_bits), uhi = bf(hi_bits);
+    // largest dot with fl(1 - dot) >= ulo, smallest dot with fl(1 - dot) <= uhi
+    float dmax = __fsub_rn(1.0f, ulo);
+    for (int k = 0; k < 64 && __fsub_rn(1.0f, nup(dmax)) >= ulo; ++k) dmax = nup(dmax);
+    for (int k = 0; k < 64 && __fsub_rn(1.0f, dmax) < ulo; ++k) dmax = ndown(dmax);
+    float dmin = __fsub_rn(1.0f, uhi);
+    for (int k = 0; k < 64 && __fsub_rn(1.0f, ndown(dmin)) <= uhi; ++k) dmin = ndown(dmin);
+    for (int k = 0; k < 64 && __fsub_rn(1.0f, dmin) > uhi; ++k) dmin = nup(dmin);
+    const int bmin = bin_def(edges, nb, dmax), bmax = bin_def(edges, nb, dmin);
+    good = (__fsub_rn(1.0f, dmax) >= ulo) && (__fsub_rn(1.0f, dmin) <= uhi) && (bmax - bmin <= 1);
+    out = make_int2(bmin, bmin <= nb ? fb(edges[bmin]) : (int)0xff800000u);
+  }
+  lut[q] = out;
+  if (!good) atomicExch(ok, 0);
+}
+
+// Dynamic shared memory: E[32] | LUT[2048] int2 | B[C] float4 | H[warps][nb2][32] u32
+struct TPSmem {
+  float* E;
+  int2* L;
+  float4* B;
+  uint32_t* H;
+};
+__host__ __device__ inline size_t tp_smem_bytes(int C, int nb2) {
+  return 32 * sizeof(float) + TP_LUT * sizeof(int2) + (size_t)C * sizeof(float4) + (size_t)TP_WARPS * nb2 * 32 * 4;
+}
+__device__ __forceinline__ TPSmem tp_carve(unsigned char* base, int C) {
+  TPSmem S;
+  S.E = reinterpret_cast<float*>(base);
+  S.L = reinterpret_cast<int2*>(base + 128);
+  S.B = reinterpret_cast<float4*>(base + 128 + TP_LUT * sizeof(int2));
+  S.H = reinterpret_cast<uint32_t*>(base + 128 + TP_LUT * sizeof(int2) + (size_t)C * sizeof(float4));
+  return S;
+}
+
+// Does any thread of this CTA have partners?  (self rows: chunks left of the diagonal are empty)
+__device__ __forceinline__ bool tp_cta_has_work(const TPParams& p, int h, int c) {
+  const int i0 = blockIdx.x * TP_THREADS;
+  const int jb = (h <= p.nr) ? max(i0 + 1, c * p.C) : c * p.C;
+  const int je = min((c + 1) * p.C, p.n);
+  return i0 < p.n && je > jb;
+}
+
+// Stage chunk c of partner set sb, the edges, the bucket table; clear the histograms.
+__device__ __forceinline__ void tp_stage(const TPParams& p, const TPSmem& S, int sb, int c, bool work) {
+  if (threadIdx.x < 32) S.E[threadIdx.x] = threadIdx.x <= p.nb ? p.edges[threadIdx.x] : __int_as_float(0xff800000);
+  if (!work) return;
   const int j0 = c * p.C;
   const int cnt = min(p.C, p.n - j0);
   const float* P = p.pts + 3 * ((int64_t)sb * p.n + j0);
   for (int k = threadIdx.x; k < cnt; k += TP_THREADS) S.B[k] = make_float4(P[3 * k], P[3 * k + 1], P[3 * k + 2], 0.f);
-  if (threadIdx.x < 32) S.E[threadIdx.x] = threadIdx.x <= p.nb ? p.edges[threadIdx.x] : __int_as_float(0xff800000);
-  uint32_t* H = &S.H[0][0][0];
-  for (int k = threadIdx.x; k < TP_WARPS * 32 * 32; k += TP_THREADS) H[k] = 0u;
+  const int4* Lg = reinterpret_cast<const int4*>(p.lut);
+  int4* Ls = reinterpret_cast<int4*>(S.L);
+  for (int k = threadIdx.x; k < TP_LUT / 2; k += TP_THREADS) Ls[k] = Lg[k];
+  const int nh = TP_WARPS * (p.nb + 2) * 32;
+  for (int k = threadIdx.x; k < nh; k += TP_THREADS) S.H[k] = 0u;
 }
 
-// Reduce the lane-private histograms and add them to hist[base + b].  Called by all threads.
-__device__ __forceinline__ void tp_flush(const TPParams& p, TPShared& S, unsigned long long* hist, int base) {
+// Reduce the lane-private histograms and add them to hist[base + b].
+__device__ __forceinline__ void tp_flush(const TPParams& p, const TPSmem& S, unsigned long long* hist, int base) {
   const int nb2 = p.nb + 2;
   for (int t = threadIdx.x; t < TP_WARPS * nb2; t += TP_THREADS) {
-    const int w = t / nb2, b = t % nb2;
+    const uint32_t* row = S.H + (size_t)t * 32;  // t = w * nb2 + b
     uint32_t s = 0;
 #pragma unroll 8
-    for (int l = 0; l < 32; ++l) s += S.H[w][b][(l + t) & 31];
-    if (s) atomicAdd(hist + base + b, (unsigned long long)s);
+    for (int l = 0; l < 32; ++l) s += row[(l + t) & 31];
+    if (s) atomicAdd(hist + base + (t % nb2), (unsigned long long)s);
   }
 }
 
 template <int V>
-__device__ __forceinline__ void tpacf_body(const TPParams& p, TPShared& S, unsigned long long* hist, hk_control* cb) {
+__device__ __forceinline__ void tpacf_body(const TPParams& p, const TPSmem& S, unsigned long long* hist, hk_control* cb) {
   constexpr bool NL = (V & V_NL) != 0, L = (V & V_L) != 0, PROF = (V & V_PROF) != 0;
   constexpr bool CNT = L || PROF;
   const uint32_t z = p.z;
@@ -75,7 +165,9 @@ __device__ __forceinline__ void tpacf_body(const TPParams& p, TPShared& S, unsig
   const bool active = i < n;
   const int32_t h = row / nC, c = row - h * nC;
   const int32_t sb = (h == 0) ? 0 : (h <= nr ? h : h - nr);
-  tp_stage(p, S, sb, c);
+  const bool work = tp_cta_has_work(p, h, c);
+  const bool use_lut = *p.lut_ok != 0;
+  tp_stage(p, S, sb, c, work);
   __syncthreads();
   const uint32_t lane = lane_id(), warp = threadIdx.x >> 5;
   if (active) {
@@ -112,16 +204,31 @@ __device__ __forceinline__ void tpacf_body(const TPParams& p, TPShared& S, unsig
     }
     int32_t acc = 0, cnt = 0;
     const float4* Bs = S.B - c * C;  // Bs[j] for j in chunk c
-    uint32_t* Hw = &S.H[warp][0][lane];
+    uint32_t* Hw = S.H + (size_t)warp * nb2 * 32 + lane;
+    if (use_lut) {
+      const int2* Ls = S.L;
 #pragma unroll 4
-    for (int32_t j = jb; j < je; ++j) {
-      const float4 q = Bs[j];
-      const float dot = __fmaf_rn(z1, q.z, __fmaf_rn(y1, q.y, __fmul_rn(x1, q.x)));
-      const int32_t bin = tp_bin(S.E, dot);
-      Hw[bin * 32] += 1u;
-      if (L || PROF) {
-        acc += bin;
-        cnt = count_inc(cnt, p.one);
+      for (int32_t j = jb; j < je; ++j) {
+        const float4 q = Bs[j];
+        const float dot = __fmaf_rn(z1, q.z, __fmaf_rn(y1, q.y, __fmul_rn(x1, q.x)));
+        const int32_t bin = tp_bin_lut(Ls, dot);
+        Hw[bin * 32] += 1u;
+        if (L || PROF) {
+          acc += bin;
+          cnt = count_inc(cnt, p.one);
+        }
+      }
+    } else {
+#pragma unroll 4
+      for (int32_t j = jb; j < je; ++j) {
+        const float4 q = Bs[j];
+        const float dot = __fmaf_rn(z1, q.z, __fmaf_rn(y1, q.y, __fmul_rn(x1, q.x)));
+        const int32_t bin = tp_bin(S.E, dot);
+        Hw[bin * 32] += 1u;
+        if (L || PROF) {
+          acc += bin;
+          cnt = count_inc(cnt, p.one);
+        }
       }
     }
     if (L && cnt != expect) alarm |= AL_COUNT;
@@ -141,14 +248,16 @@ __device__ __forceinline__ void tpacf_body(const TPParams& p, TPShared& S, unsig
     }
     if (NL || L) fold_alarm(cb, alarm, (uint32_t)((int64_t)row * n + i));
   }
-  __syncthreads();
-  tp_flush(p, S, hist, h * nb2);
+  if (work) {
+    __syncthreads();
+    tp_flush(p, S, hist, h * nb2);
+  }
 }
 
 template <int V>
 __global__ void __launch_bounds__(TP_THREADS) tpacf_kernel(const TPParams p) {
   extern __shared__ __align__(16) unsigned char tp_smem[];
-  TPShared& S = *reinterpret_cast<TPShared*>(tp_smem);
+  const TPSmem S = tp_carve(tp_smem, p.C);
   tpacf_body<V>(p, S, p.hist, p.cb);
 }
 
@@ -166,7 +275,7 @@ struct TPFIParams {
 };
 
 template <int KIND>
-__device__ void tpacf_fi_thread(const TPParams& p, TPShared& S, const FaultRec& f, unsigned long long* hist,
+__device__ void tpacf_fi_thread(const TPParams& p, const TPSmem& S, const FaultRec& f, unsigned long long* hist,
                                 hk_control* cb) {
   const uint32_t z = p.z;
   const int32_t nr = p.nr, C = p.C, nC = p.nC, nb2 = p.nb + 2;
@@ -274,7 +383,7 @@ __device__ void tpacf_fi_thread(const TPParams& p, TPShared& S, const FaultRec& 
         if (!guard(phist, hist_real, hidx, 8, nhist, &e)) { fail |= FL_CRASH; goto done; }
         atomicAdd(hist + e, 1ull);
       } else {
-        S.H[warp][bin][lane] += 1u;  // fault-free thread: hidx == base + bin, base = this CTA's row
+        S.H[((size_t)warp * nb2 + bin) * 32 + lane] += 1u;  // fault-free thread: hidx == base + bin (this CTA's row)
       }
       acc = (int32_t)((uint32_t)acc + (uint32_t)bin);
       if (KIND == TK_ACC) { applied |= now; acc = flip_i(acc, now, mask); }
@@ -304,7 +413,7 @@ done:
 template <int KIND>
 __global__ void __launch_bounds__(TP_THREADS) tpacf_fi_kernel(const TPFIParams q) {
   extern __shared__ __align__(16) unsigned char tp_smem[];
-  TPShared& S = *reinterpret_cast<TPShared*>(tp_smem);
+  const TPSmem S = tp_carve(tp_smem, q.base.C);
   const int r = blockIdx.z;
   const FaultRec f = q.faults[r];
   unsigned long long* hist = q.hist0 + (int64_t)r * q.hist_elems;
@@ -316,7 +425,7 @@ __global__ void __launch_bounds__(TP_THREADS) tpacf_fi_kernel(const TPFIParams q
     const TPParams& p = q.base;
     const int32_t h = blockIdx.y / p.nC, c = blockIdx.y - h * p.nC;
     const int32_t sb = (h == 0) ? 0 : (h <= p.nr ? h : h - p.nr);
-    tp_stage(p, S, sb, c);
+    tp_stage(p, S, sb, c, true);
     __syncthreads();
     tpacf_fi_thread<KIND>(p, S, f, hist, cb);
     __syncthreads();
@@ -327,15 +436,13 @@ __global__ void __launch_bounds__(TP_THREADS) tpacf_fi_kernel(const TPFIParams q
 // ============================================================================================
 // Host launchers
 // ============================================================================================
-static double tp_pairs(const TPParams& p) {
-  const double n = p.n;
-  return (1 + p.nr) * n * (n - 1) / 2 + p.nr * n * n;
-}
-
-static TPParams tp_params(const hk_tpacf_args& a, const DevRanges& R, int ndet, hk_control* cb, float* samples) {
+static TPParams tp_params(const hk_tpacf_args& a, const DevRanges& R, int ndet, hk_control* cb, float* samples,
+                          void* lut_ws) {
   TPParams p{};
   p.pts = a.pts;
   p.edges = a.edges;
+  p.lut = reinterpret_cast<const int2*>(lut_ws);
+  p.lut_ok = reinterpret_cast<const int*>(reinterpret_cast<const char*>(lut_ws) + TP_LUT * sizeof(int2));
   p.hist = a.hist;
   p.cb = cb;
   p.samples = samples;
@@ -351,24 +458,40 @@ static TPParams tp_params(const hk_tpacf_args& a, const DevRanges& R, int ndet, 
   return p;
 }
 
+size_t tpacf_lut_ws_bytes() { return TP_LUT * sizeof(int2) + 16; }
+
+cudaError_t tpacf_lut_build(const hk_tpacf_args& a, void* lut_ws, cudaStream_t s) {
+  int* ok = reinterpret_cast<int*>(reinterpret_cast<char*>(lut_ws) + TP_LUT * sizeof(int2));
+  cudaError_t e = cudaMemsetAsync(ok, 1, sizeof(int), s);
+  if (e != cudaSuccess) return e;
+  tpacf_lut_kernel<<<TP_LUT / 256, 256, 0, s>>>(a.edges, a.n_bins, reinterpret_cast<int2*>(lut_ws), ok);
+  count_launch();
+  return cudaGetLastError();
+}
+
+static double tp_pairs(const TPParams& p) {
+  const double n = p.n;
+  return (1 + p.nr) * n * (n - 1) / 2 + p.nr * n * n;
+}
+
 template <int V>
 static cudaError_t launch_tp_v(const TPParams& p, cudaStream_t s) {
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(tpacf_kernel<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TPShared));
-    attr = true;
-  }
+  const size_t smem = tp_smem_bytes(p.C, p.nb + 2);
+  cudaError_t e = cudaFuncSetAttribute(tpacf_kernel<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
   dim3 grid((p.n + TP_THREADS - 1) / TP_THREADS, (1 + 2 * p.nr) * p.nC);
   if (grid.x == 0) return cudaSuccess;
   TimedScope ts(HK_TPACF, 0, tp_pairs(p), s);
-  tpacf_kernel<V><<<grid, TP_THREADS, sizeof(TPShared), s>>>(p);
+  tpacf_kernel<V><<<grid, TP_THREADS, smem, s>>>(p);
   count_launch();
   return cudaGetLastError();
 }
 
 cudaError_t tpacf_launch(int vflags, const hk_tpacf_args& a, const DevRanges& R, int ndet, hk_control* cb, float* samples,
-                         cudaStream_t s) {
-  const TPParams p = tp_params(a, R, ndet, cb, samples);
+                         void* lut_ws, cudaStream_t s) {
+  cudaError_t e = tpacf_lut_build(a, lut_ws, s);
+  if (e != cudaSuccess) return e;
+  const TPParams p = tp_params(a, R, ndet, cb, samples, lut_ws);
   switch (vflags) {
     case 0: return launch_tp_v<0>(p, s);
     case V_NL | V_L: return launch_tp_v<V_NL | V_L>(p, s);
@@ -387,22 +510,21 @@ int tpacf_site_kind(int site) {
 
 template <int KIND>
 static cudaError_t launch_tp_fi_k(const TPFIParams& q, int nrep, cudaStream_t s) {
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(tpacf_fi_kernel<KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TPShared));
-    attr = true;
-  }
+  const size_t smem = tp_smem_bytes(q.base.C, q.base.nb + 2);
+  cudaError_t e = cudaFuncSetAttribute(tpacf_fi_kernel<KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
   dim3 grid((q.base.n + TP_THREADS - 1) / TP_THREADS, (1 + 2 * q.base.nr) * q.base.nC, nrep);
   TimedScope ts(HK_TPACF, 1, tp_pairs(q.base) * nrep, s);
-  tpacf_fi_kernel<KIND><<<grid, TP_THREADS, sizeof(TPShared), s>>>(q);
+  tpacf_fi_kernel<KIND><<<grid, TP_THREADS, smem, s>>>(q);
   count_launch();
   return cudaGetLastError();
 }
 
+// lut_ws must hold a table built by tpacf_lut_build for a.edges (the campaign builds it once).
 cudaError_t tpacf_fi_launch(int kind, const hk_tpacf_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
-                            unsigned long long* hist0, hk_control* cb0, cudaStream_t s) {
+                            unsigned long long* hist0, hk_control* cb0, void* lut_ws, cudaStream_t s) {
   TPFIParams q{};
-  q.base = tp_params(a, R, ndet, nullptr, nullptr);
+  q.base = tp_params(a, R, ndet, nullptr, nullptr, lut_ws);
   q.faults = faults;
   q.hist0 = hist0;
   q.cb0 = cb0;
@@ -414,7 +536,5 @@ cudaError_t tpacf_fi_launch(int kind, const hk_tpacf_args& a, const DevRanges& R
   }
   return cudaErrorInvalidValue;
 }
-
-size_t tpacf_smem_bytes() { return sizeof(TPShared); }
 
 }  // namespace hk

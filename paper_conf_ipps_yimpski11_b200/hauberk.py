@@ -113,6 +113,12 @@ def lib():
         L.hauberk_last_error.argtypes = []
         L.hauberk_version.restype = I32
         L.hauberk_launch_count.restype = U64
+        L.hauberk_campaign_create.restype = I32
+        L.hauberk_campaign_create.argtypes = [I32, P, P, P, P, P]
+        L.hauberk_campaign_run.restype = I32
+        L.hauberk_campaign_run.argtypes = [P, I64, I64, P, P, P]
+        L.hauberk_campaign_destroy.restype = None
+        L.hauberk_campaign_destroy.argtypes = [P]
         L.hauberk_timing_enable.restype = None
         L.hauberk_timing_enable.argtypes = [I32]
         L.hauberk_timing_read.restype = I32
@@ -124,7 +130,7 @@ def lib():
 EXPORTED = ["hauberk_run_cp", "hauberk_run_mriq", "hauberk_run_tpacf", "hauberk_profile_ranges",
             "hauberk_inject_campaign", "hauberk_decode", "hauberk_num_sites", "hauberk_strerror",
             "hauberk_last_error", "hauberk_version", "hauberk_launch_count", "hauberk_timing_enable",
-            "hauberk_timing_read"]
+            "hauberk_timing_read", "hauberk_campaign_create", "hauberk_campaign_run", "hauberk_campaign_destroy"]
 
 
 def _check(status: int, where: str):
@@ -341,6 +347,45 @@ def inject_campaign(bench_mode: int, devs, ranges, seed: int, first: int, count:
     st = lib().hauberk_inject_campaign(bench_mode, arr, rarr, C.byref(camp), _ptr(records), _ptr(counts),
                                        _ptr(site_counts), _stream(stream))
     _check(st, "hauberk_inject_campaign")
+
+
+class CampaignSession:
+    """hauberk_campaign_create / _run / _destroy: golden runs and workspaces prepared once, then
+    asynchronous slices of the same seeded campaign.  Keep `devs` alive while the session lives."""
+
+    def __init__(self, bench_mode: int, devs, ranges, seed: int, exact: int = 0, batch: int = 0,
+                 site_masks=(ALL_SITES,) * 3, stream=None):
+        self._arr, self._keep = _arg_array(devs)
+        self._devs = devs
+        self._rng = [r if r is not None else Ranges() for r in ranges]
+        self._rarr = (C.c_void_p * 3)(*[C.cast(C.byref(r), C.c_void_p) for r in self._rng])
+        self._camp = Campaign(seed, 0, 0, 1, 0, batch, exact, (C.c_uint64 * 3)(*site_masks))
+        self._h = C.c_void_p()
+        st = lib().hauberk_campaign_create(bench_mode, self._arr, self._rarr, C.byref(self._camp), C.byref(self._h),
+                                           _stream(stream))
+        _check(st, "hauberk_campaign_create")
+
+    def run(self, first: int, count: int, counts: torch.Tensor, records: torch.Tensor | None = None,
+            site_counts: torch.Tensor | None = None):
+        st = lib().hauberk_campaign_run(self._h, first, count, _ptr(records), _ptr(counts), _ptr(site_counts))
+        _check(st, "hauberk_campaign_run")
+
+    def close(self):
+        if self._h:
+            lib().hauberk_campaign_destroy(self._h)
+            self._h = C.c_void_p()
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
 
 
 def records_tensor(count: int, device="cuda") -> torch.Tensor:

@@ -262,3 +262,56 @@ def test_campaign_sharding_invariance_and_batching():
         hk.inject_campaign(-1, devs, R, 99, first, cnt, parts, batch=7)
     torch.cuda.synchronize()
     assert torch.equal(whole, parts)
+
+
+def test_tpacf_bucket_binning_adversarial_dots():
+    """DR pairs with data point (1,0,0) have dot == x2 exactly, so the partner x-coordinates probe the
+    binning at chosen dot values: every edge +-12 ulps, every u = 1 - dot bucket boundary, and
+    out-of-range dots (|dot| > 1).  The CUDA histogram must equal the oracle's count definition."""
+    e = W.tpacf_edges().astype(np.float32)
+    vals = []
+    for x in e:
+        b = np.array([x], dtype=np.float32).view(np.int32)[0]
+        vals += list(np.arange(b - 12, b + 13, dtype=np.int32).view(np.float32))
+    for q in range(0, 1024, 1):
+        ub = np.array([q << 21, (q << 21) | 0x1FFFFF], dtype=np.uint32).view(np.float32)
+        for u in ub:
+            if np.isfinite(u) and u <= 2.0:
+                d = np.float32(1.0) - u
+                vals += [d, np.nextafter(d, np.float32(2)), np.nextafter(d, np.float32(-2))]
+    vals += [1.0, np.nextafter(np.float32(1), np.float32(2)), -1.0, np.nextafter(np.float32(-1), np.float32(-2)), 0.0, -0.0]
+    v = np.unique(np.array(vals, dtype=np.float32))
+    v = v[np.isfinite(v)]
+    n = v.size
+    pts = np.zeros((2, n, 3), dtype=np.float32)
+    pts[0, :, 0] = 1.0
+    pts[1, :, 0] = v
+    pts[1, :, 1] = np.sqrt(np.maximum(0.0, 1.0 - v.astype(np.float64) ** 2)).astype(np.float32)
+    p = W.TPACFProblem(pts=pts, edges=e, chunk=512)
+    d = _mk(2, p)
+    cb = hk.new_control(DEV)
+    hk.run(d, hk.HK_BASE, None, cb)
+    torch.cuda.synchronize()
+    got = _out_np(d)
+    ora, _, _ = O.run(O.TPACF, p, flags=0)
+    assert np.array_equal(got, ora)
+    # the DR row is n copies of the per-value bins
+    assert got[2].sum() == n * n
+
+
+def test_campaign_session_matches_one_shot_calls():
+    probs = [W.cp_small(), W.mriq_problem(4, 40, n_vox=64, seed=9), W.tpacf_small(n=64, n_rand=1, chunk=16)]
+    devs = [_mk(b, probs[b]) for b in range(3)]
+    R = [hk.profile_ranges(d) for d in devs]
+    one = torch.zeros((3, 5), dtype=torch.int64, device=DEV)
+    rec1 = hk.records_tensor(600, DEV)
+    hk.inject_campaign(-1, devs, R, 4242, 1000, 600, one, records=rec1)
+    ses = torch.zeros((3, 5), dtype=torch.int64, device=DEV)
+    rec2 = hk.records_tensor(600, DEV)
+    with hk.CampaignSession(-1, devs, R, 4242, batch=13) as S:
+        S.run(1000, 250, ses, records=rec2[: 250 * hk.OUTCOME_DTYPE.itemsize])
+        S.run(1250, 350, ses, records=rec2[250 * hk.OUTCOME_DTYPE.itemsize:])
+        torch.cuda.synchronize()
+    assert torch.equal(one, ses)
+    a, b = hk.records_numpy(rec1), hk.records_numpy(rec2)
+    assert np.array_equal(a["cls"], b["cls"]) and np.array_equal(a["index"], b["index"])

@@ -1,0 +1,94 @@
+"""T5 SASS audit: nvcc/ptxas must not have folded HAUBERK's detectors away.
+
+cuobjdump -sass of libhauberk.so (sm_100a): the FT kernels keep the duplicated definitions
+(extra ISETP compares), the XOR checksum pairs (LOP3), and a per-atom counter add inside the main
+loop; BASE has none of them; both issue the same MUFU work.  The campaign path must also carry
+the TMA bulk copy (UBLKCP) that stages atoms / k-space."""
+import os
+import re
+import shutil
+import subprocess
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+LIB = os.path.join(ROOT, "paper_conf_ipps_yimpski11_b200", "libhauberk.so")
+
+
+@pytest.fixture(scope="module")
+def sass():
+    if not shutil.which("cuobjdump"):
+        pytest.skip("cuobjdump not available")
+    if not os.path.exists(LIB):
+        import __graft_entry__ as g
+        g.build()
+    txt = subprocess.check_output(["cuobjdump", "-sass", LIB], text=True)
+    out = {}
+    for sec in re.split(r"\n\s*Function : ", txt)[1:]:
+        name = sec.split("\n", 1)[0].strip()
+        ops = [m[1] for m in re.findall(r"/\*[0-9a-f]{4,}\*/\s+(@!?U?P\w+\s+)?([A-Z][A-Z0-9_]*(?:\.[A-Z0-9_]+)*)", sec)]
+        out[name] = ops
+    return out
+
+
+def _find(sass, pattern):
+    names = [n for n in sass if re.search(pattern, n)]
+    assert names, pattern
+    return sass[names[0]]
+
+
+def _count(ops, prefix):
+    return sum(1 for o in ops if o.startswith(prefix))
+
+
+def _loop_region(ops, anchor):
+    idx = [i for i, o in enumerate(ops) if o.startswith(anchor)]
+    return ops[idx[0]: idx[-1] + 1]
+
+
+@pytest.mark.parametrize("u", [4, 8])
+def test_cp_ft_keeps_detectors(sass, u):
+    ft = _find(sass, rf"cp_kernelILi3ELi{u}ELb0E")
+    base = _find(sass, rf"cp_kernelILi0ELi{u}ELb0E")
+    assert _count(ft, "MUFU.RSQ") >= _count(base, "MUFU.RSQ") > 0
+    assert _count(ft, "LOP3") >= _count(base, "LOP3") + 20       # chk ^= v twice per virtual variable
+    assert _count(ft, "ISETP") >= _count(base, "ISETP") + 6      # duplicate compares, CheckEqual
+    loop_ft = _loop_region(ft, "MUFU.RSQ")
+    loop_base = _loop_region(base, "MUFU.RSQ")
+    adds = lambda ops: sum(1 for o in ops if o.startswith(("IADD3", "VIADD", "IADD ")))
+    assert adds(loop_ft) >= 4 > adds(loop_base)                   # it++ per atom survives unrolling
+    assert "UBLKCP.S.G" in ft                                      # TMA bulk copy of atom tiles
+
+
+def test_mriq_ft_keeps_detectors(sass):
+    ft = _find(sass, r"mriq_kernelILi3ELb0E")
+    base = _find(sass, r"mriq_kernelILi0ELb0E")
+    assert _count(ft, "MUFU.SIN") == _count(base, "MUFU.SIN") > 0
+    assert _count(ft, "MUFU.COS") == _count(base, "MUFU.COS") > 0
+    assert _count(ft, "LOP3") >= _count(base, "LOP3") + 10
+    # duplicated loads of sX, sY, sZ (A3) through an opaque index
+    assert _count(ft, "LDG") >= _count(base, "LDG") + 3
+    loop_ft = _loop_region(ft, "MUFU.SIN")
+    assert sum(1 for o in loop_ft if o.startswith(("IADD3", "VIADD"))) >= 3  # 4-way unrolled: 3 between first/last SIN
+    assert "UBLKCP.S.G" in ft
+
+
+def test_tpacf_ft_keeps_detectors(sass):
+    ft = _find(sass, r"tpacf_kernelILi3EE")
+    base = _find(sass, r"tpacf_kernelILi0EE")
+    assert _count(ft, "LOP3") >= _count(base, "LOP3") + 10
+    assert _count(ft, "ISETP") >= _count(base, "ISETP") + 8
+    assert len(ft) > len(base)
+
+
+def test_fi_kernels_compiled_for_every_site_kind(sass):
+    assert len([n for n in sass if "cp_fi_kernel" in n]) == 15 * 2
+    assert len([n for n in sass if "mriq_fi_kernel" in n]) == 16 * 2
+    assert len([n for n in sass if "tpacf_fi_kernel" in n]) == 11
+
+
+def test_no_tensor_core_or_fp64_in_hot_kernels(sass):
+    # nothing here is a dense contraction; FP64 stays idle
+    for n, ops in sass.items():
+        if re.match(r"_ZN2hk\d+(cp|mriq|tpacf)_(fi_)?kernel", n):
+            assert not any(o.startswith(("HMMA", "UTCHMMA", "UTCQMMA", "DFMA", "DADD", "DMUL")) for o in ops), n

@@ -188,16 +188,18 @@ def main():
     flush = torch.empty(512 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
     overhead, kernels = {}, {}
     if not args.no_overhead and rank == 0:
-        cases = [("cp_cfg4", hk.CPDevice.from_problem(W.cp_config4(bx=32, by=4, unroll=8), dev), "xu", 1.0),
+        # Fig. 13 columns: HAUBERK-NL, HAUBERK-L and HAUBERK vs the unprotected kernel
+        cases = [("cp_cfg4", hk.CPDevice.from_problem(W.cp_config4(bx=16, by=16, unroll=8), dev), "xu", 1.0),
                  ("mriq_cfg2", devs[1], "xu", 2.0), ("tpacf_cfg3", devs[2], "alu", float(TPACF_OPS_PER_PAIR))]
+        variants = (hk.HK_BASE, hk.HK_FT_NL, hk.HK_FT_L, hk.HK_FT)
         for name, d, pipe, ops in cases:
             R = hk.profile_ranges(d)
             cb = hk.new_control(dev)
             hk.timing_enable(True)
-            t = {hk.HK_BASE: [], hk.HK_FT: []}
+            t = {v: [] for v in variants}
             work = 0.0
             for rep in range(12):
-                for v in (hk.HK_BASE, hk.HK_FT):
+                for v in variants:
                     flush.zero_()
                     hk.run(d, v, R, cb)
                     torch.cuda.synchronize()
@@ -207,11 +209,14 @@ def main():
                         work = w
             hk.timing_enable(False)
             assert hk.read_control(cb).alarm == 0
-            tb, tf = statistics.median(t[hk.HK_BASE]), statistics.median(t[hk.HK_FT])
+            med = {v: statistics.median(t[v]) for v in variants}
+            tb, tf = med[hk.HK_BASE], med[hk.HK_FT]
             peak = mufu_peak if pipe == "xu" else lane_peak
             ach = work * ops / (tf * 1e-3)
             overhead[name] = round(100.0 * (tf / tb - 1.0), 2)
             kernels[name] = {"base_ms": round(tb, 4), "ft_ms": round(tf, 4), "overhead_pct": overhead[name],
+                             "overhead_nl_pct": round(100.0 * (med[hk.HK_FT_NL] / tb - 1.0), 2),
+                             "overhead_l_pct": round(100.0 * (med[hk.HK_FT_L] / tb - 1.0), 2),
                              "pairs": work, "bound": "alu", "pipe": "xu (MUFU)" if pipe == "xu" else "fp32/int lanes",
                              "achieved_gops": round(ach / 1e9, 1), "peak_gops": round(peak / 1e9, 1),
                              "frac": round(ach / peak, 4), "base_frac": round(work * ops / (tb * 1e-3) / peak, 4)}

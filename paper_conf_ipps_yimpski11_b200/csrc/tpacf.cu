@@ -13,13 +13,13 @@
 namespace hk {
 
 constexpr int TP_THREADS = 256;
+constexpr int TP_CTA_PTS = 2 * TP_THREADS;  // two abstract threads per CUDA thread
 constexpr int TP_WARPS = TP_THREADS / 32;
-constexpr int TP_CMAX = 1024;  // max chunk (partners per abstract thread)
 
 struct TPParams {
   const float* pts;
   const float* edges;
-  const int2* lut;     // [TP_LUT] (bmin, bits(edge[bmin])) per u-bucket; built by tpacf_lut_kernel
+  const uint8_t* lut;  // [TP_LUT] bmin per u-bucket; built by tpacf_lut_kernel
   const int* lut_ok;   // 1 if every bucket holds at most one edge (else: binary search)
   unsigned long long* hist;
   hk_control* cb;
@@ -46,10 +46,10 @@ __device__ __forceinline__ int32_t tp_bin(const float* Es, float dot) {
   for (int s = 16; s >= 1; s >>= 1) b += (dot < Es[b + s - 1]) ? s : 0;
   return b;
 }
-__device__ __forceinline__ int32_t tp_bin_lut(const int2* L, float dot) {
+__device__ __forceinline__ int32_t tp_bin_lut(const uint8_t* L, const float* Es, float dot) {
   const float u = __fsub_rn(1.0f, dot);
-  const int2 e = L[fb(u) >> 21];
-  return e.x + ((dot < __int_as_float(e.y)) ? 1 : 0);
+  const int32_t b = L[fb(u) >> 21];
+  return b + ((dot < Es[b]) ? 1 : 0);
 }
 
 __device__ __forceinline__ float nup(float x) {
@@ -70,7 +70,7 @@ __device__ __forceinline__ int32_t bin_def(const float* edges, int nb, float dot
 
 // One thread per bucket q.  Buckets whose u range holds no finite value (inf/NaN exponents) map
 // to bin 0 for NaN (the definition: every compare with NaN is false) and nb+1 for +inf.
-__global__ void tpacf_lut_kernel(const float* __restrict__ edges, int nb, int2* __restrict__ lut, int* ok) {
+__global__ void tpacf_lut_kernel(const float* __restrict__ edges, int nb, uint8_t* __restrict__ lut, int* ok) {
   const int q = blockIdx.x * blockDim.x + threadIdx.x;
   if (q >= TP_LUT) return;
   const float e0 = edges[0];
@@ -82,7 +82,7 @@ __global__ void tpacf_lut_kernel(const float* __restrict__ edges, int nb, int2* 
   if (neg) {
     out = make_int2(0, fb(e0));  // u <= -0: dot >= 1 > every edge -> bin 0 (and -NaN: bin 0)
   } else if (special) {
-    out = (q == (int)(0x7f800000u >> 21)) ? make_int2(nb + 1, (int)0xff800000u) : make_int2(0, fb(e0));
+    out = (q == (int)(0x7f800000u >> 21)) ? make_int2(nb + 1, (int)-8388608) : make_int2(0, fb(e0));
   } else {
     const float ulo = bf(lo_bits), uhi = bf(hi_bits);
     // largest dot with fl(1 - dot) >= ulo, smallest dot with fl(1 - dot) <= uhi
@@ -94,34 +94,34 @@ __global__ void tpacf_lut_kernel(const float* __restrict__ edges, int nb, int2* 
     for (int k = 0; k < 64 && __fsub_rn(1.0f, dmin) > uhi; ++k) dmin = nup(dmin);
     const int bmin = bin_def(edges, nb, dmax), bmax = bin_def(edges, nb, dmin);
     good = (__fsub_rn(1.0f, dmax) >= ulo) && (__fsub_rn(1.0f, dmin) <= uhi) && (bmax - bmin <= 1);
-    out = make_int2(bmin, bmin <= nb ? fb(edges[bmin]) : (int)0xff800000u);
+    out = make_int2(bmin, bmin <= nb ? fb(edges[bmin]) : (int)-8388608);
   }
-  lut[q] = out;
+  lut[q] = (uint8_t)out.x;  // E[b] (padded with -inf beyond nb) supplies the compare value
   if (!good) atomicExch(ok, 0);
 }
 
-// Dynamic shared memory: E[32] | LUT[2048] int2 | B[C] float4 | H[warps][nb2][32] u32
+// Dynamic shared memory: E[32] | LUT[2048] u8 | B[C] float4 | H[warps][nb2][32] u32
 struct TPSmem {
   float* E;
-  int2* L;
+  uint8_t* L;
   float4* B;
   uint32_t* H;
 };
 __host__ __device__ inline size_t tp_smem_bytes(int C, int nb2) {
-  return 32 * sizeof(float) + TP_LUT * sizeof(int2) + (size_t)C * sizeof(float4) + (size_t)TP_WARPS * nb2 * 32 * 4;
+  return 32 * sizeof(float) + TP_LUT + (size_t)C * sizeof(float4) + (size_t)TP_WARPS * nb2 * 32 * 4;
 }
 __device__ __forceinline__ TPSmem tp_carve(unsigned char* base, int C) {
   TPSmem S;
   S.E = reinterpret_cast<float*>(base);
-  S.L = reinterpret_cast<int2*>(base + 128);
-  S.B = reinterpret_cast<float4*>(base + 128 + TP_LUT * sizeof(int2));
-  S.H = reinterpret_cast<uint32_t*>(base + 128 + TP_LUT * sizeof(int2) + (size_t)C * sizeof(float4));
+  S.L = base + 128;
+  S.B = reinterpret_cast<float4*>(base + 128 + TP_LUT);
+  S.H = reinterpret_cast<uint32_t*>(base + 128 + TP_LUT + (size_t)C * sizeof(float4));
   return S;
 }
 
 // Does any thread of this CTA have partners?  (self rows: chunks left of the diagonal are empty)
 __device__ __forceinline__ bool tp_cta_has_work(const TPParams& p, int h, int c) {
-  const int i0 = blockIdx.x * TP_THREADS;
+  const int i0 = blockIdx.x * TP_CTA_PTS;
   const int jb = (h <= p.nr) ? max(i0 + 1, c * p.C) : c * p.C;
   const int je = min((c + 1) * p.C, p.n);
   return i0 < p.n && je > jb;
@@ -137,7 +137,7 @@ __device__ __forceinline__ void tp_stage(const TPParams& p, const TPSmem& S, int
   for (int k = threadIdx.x; k < cnt; k += TP_THREADS) S.B[k] = make_float4(P[3 * k], P[3 * k + 1], P[3 * k + 2], 0.f);
   const int4* Lg = reinterpret_cast<const int4*>(p.lut);
   int4* Ls = reinterpret_cast<int4*>(S.L);
-  for (int k = threadIdx.x; k < TP_LUT / 2; k += TP_THREADS) Ls[k] = Lg[k];
+  for (int k = threadIdx.x; k < TP_LUT / 16; k += TP_THREADS) Ls[k] = Lg[k];
   const int nh = TP_WARPS * (p.nb + 2) * 32;
   for (int k = threadIdx.x; k < nh; k += TP_THREADS) S.H[k] = 0u;
 }
@@ -154,15 +154,148 @@ __device__ __forceinline__ void tp_flush(const TPParams& p, const TPSmem& S, uns
   }
 }
 
-template <int V>
-__device__ __forceinline__ void tpacf_body(const TPParams& p, const TPSmem& S, unsigned long long* hist, hk_control* cb) {
-  constexpr bool NL = (V & V_NL) != 0, L = (V & V_L) != 0, PROF = (V & V_PROF) != 0;
-  constexpr bool CNT = L || PROF;
+// Per-abstract-thread prologue state (NL sites 0-11).
+struct TPPoint {
+  int32_t i, row, boff, jb, je, expect, base;
+  float x1, y1, z1;
+  uint32_t chk, alarm;
+  int32_t acc, cnt;
+};
+
+template <bool NL>
+__device__ __forceinline__ TPPoint tp_prologue(const TPParams& p, const unsigned long long* hist, int k) {
   const uint32_t z = p.z;
   const int32_t n = p.n, nr = p.nr, C = p.C, nC = p.nC, nb2 = p.nb + 2;
+  TPPoint P;
+  P.row = blockIdx.y;
+  P.i = blockIdx.x * TP_CTA_PTS + k * TP_THREADS + threadIdx.x;
+  const int32_t h = P.row / nC, c = P.row - h * nC;
+  P.chk = 0;
+  P.alarm = 0;
+  if (NL) {
+    P.chk ^= (uint32_t)n ^ lohi_ptr(p.pts) ^ lohi_ptr(hist);
+    P.chk ^= (uint32_t)P.i;
+    P.alarm |= ((int32_t)((blockIdx.x ^ z) * TP_CTA_PTS + k * TP_THREADS + (threadIdx.x ^ z)) != P.i) ? AL_DUP : 0u;
+    P.chk ^= (uint32_t)h; P.alarm |= ((int32_t)(blockIdx.y ^ z) / nC != h) ? AL_DUP : 0u;
+    P.chk ^= (uint32_t)c; P.alarm |= ((int32_t)(P.row - opq(h, z) * nC) != c) ? AL_DUP : 0u;
+  }
+  const int32_t aoff = (h <= nr ? h : 0) * n + P.i;
+  const int32_t sb = (h == 0) ? 0 : (h <= nr ? h : h - nr);
+  P.boff = sb * n;
+  P.jb = h <= nr ? max(P.i + 1, c * C) : c * C;
+  P.je = min((c + 1) * C, n);
+  P.expect = max(P.je - P.jb, 0);
+  P.base = h * nb2;
+  if (NL) {
+    const int32_t h2 = opq(h, z), i2 = opq(P.i, z), c2 = opq(c, z);
+    P.chk ^= (uint32_t)aoff; P.alarm |= ((h2 <= nr ? h2 : 0) * n + i2 != aoff) ? AL_DUP : 0u;
+    P.chk ^= (uint32_t)P.boff; P.alarm |= ((h2 == 0 ? 0 : (h2 <= nr ? h2 : h2 - nr)) * n != P.boff) ? AL_DUP : 0u;
+    P.chk ^= (uint32_t)P.jb; P.alarm |= ((h2 <= nr ? max(i2 + 1, c2 * C) : c2 * C) != P.jb) ? AL_DUP : 0u;
+    P.chk ^= (uint32_t)P.je; P.alarm |= (min((c2 + 1) * C, n) != P.je) ? AL_DUP : 0u;
+    P.chk ^= (uint32_t)P.expect; P.alarm |= (max(opq(P.je, z) - P.jb, 0) != P.expect) ? AL_DUP : 0u;
+    P.chk ^= (uint32_t)P.base; P.alarm |= (h2 * nb2 != P.base) ? AL_DUP : 0u;
+  }
+  const float* A = p.pts + 3 * (int64_t)aoff;
+  P.x1 = A[0]; P.y1 = A[1]; P.z1 = A[2];
+  if (NL) {
+    const float* A2 = p.pts + 3 * (int64_t)opq(aoff, z);
+    P.chk ^= fb(P.x1); P.alarm |= (fb(A2[0]) != fb(P.x1)) ? AL_DUP : 0u;
+    P.chk ^= fb(P.y1); P.alarm |= (fb(A2[1]) != fb(P.y1)) ? AL_DUP : 0u;
+    P.chk ^= fb(P.z1); P.alarm |= (fb(A2[2]) != fb(P.z1)) ? AL_DUP : 0u;
+    P.chk ^= (uint32_t)opq(P.i, z) ^ (uint32_t)opq(h, z) ^ (uint32_t)opq(c, z) ^ (uint32_t)opq(aoff, z) ^
+             (uint32_t)opq(P.jb, z);
+  }
+  P.acc = 0;
+  P.cnt = 0;
+  return P;
+}
+
+template <int V>
+__device__ __forceinline__ void tp_epilogue(const TPParams& p, TPPoint& P, const unsigned long long* hist, hk_control* cb) {
+  constexpr bool NL = (V & V_NL) != 0, L = (V & V_L) != 0, PROF = (V & V_PROF) != 0;
+  const uint32_t z = p.z;
+  if (L && P.cnt != P.expect) P.alarm |= AL_COUNT;
+  if ((L || PROF) && P.cnt != 0 && p.ndet > 0) {
+    const float v = __fdiv_rn((float)P.acc, (float)P.cnt);
+    if (PROF) p.samples[(int64_t)P.row * p.n + P.i] = v;
+    if (L && p.R.n[0] > 0 && !in_range<false>(p.R, 0, v, nullptr)) {
+      P.alarm |= AL_RANGE;
+      record_outlier(cb, 0, v);
+    }
+  }
+  if (NL) {
+    P.chk ^= (uint32_t)opq(P.boff, z) ^ (uint32_t)opq(P.je, z) ^ (uint32_t)opq(P.base, z);
+    P.chk ^= opqf(P.x1, z) ^ opqf(P.y1, z) ^ opqf(P.z1, z) ^ (uint32_t)opq(P.expect, z);
+    P.chk ^= ((uint32_t)p.n + z) ^ (lohi_ptr(p.pts) + z) ^ (lohi_ptr(hist) + z);
+    if (P.chk != 0) P.alarm |= AL_CHK;
+  }
+}
+
+__device__ __forceinline__ float tp_dot(const TPPoint& P, const float4 q) {
+  return __fmaf_rn(P.z1, q.z, __fmaf_rn(P.y1, q.y, __fmul_rn(P.x1, q.x)));
+}
+template <bool LUT>
+__device__ __forceinline__ int32_t tp_binof(const uint8_t* __restrict__ L, const float* __restrict__ E, float dot) {
+  return LUT ? tp_bin_lut(L, E, dot) : tp_bin(E, dot);
+}
+template <bool CNT>
+__device__ __forceinline__ void tp_count(const TPParams& p, uint32_t* Hw, TPPoint& P, int32_t bin) {
+  // lane-private counter: no contention; the shared-memory atomic (ATOMS.POPC.INC) has no
+  // register round trip, so consecutive increments do not serialise (microbenchmark: 1.34x the
+  // LDS/IADD/STS read-modify-write, tools/microbench/smem_hist.cu)
+  atomicAdd(Hw + bin * 32, 1u);
+  if (CNT) {
+    P.acc += bin;
+    P.cnt = count_inc(P.cnt, p.one);
+  }
+}
+
+// CTA = (row h*nC + c, 512 points); each CUDA thread runs TWO abstract threads (points i and
+// i + 256, same row and chunk), each in its own ascending-j order, sharing every partner load.
+// Within a group of 4 partners all loads (partner, bucket table, edge) are issued before the
+// histogram read-modify-writes, which the compiler must otherwise serialise (possible aliasing).
+template <int V, bool LUT>
+__device__ __forceinline__ void tp_loops(const TPParams& p, const TPSmem& S, uint32_t* Hw, TPPoint& A, TPPoint& B,
+                                         bool va, bool vb) {
+  constexpr bool CNT = (V & (V_L | V_PROF)) != 0;
+  const uint8_t* __restrict__ L = S.L;
+  const float* __restrict__ E = S.E;
+  const float4* __restrict__ Bs = S.B - (A.row % p.nC) * p.C;  // Bs[j] for j in chunk c
+  const int32_t je = A.je;
+  const int32_t ja = va ? A.jb : je, jbb = vb ? B.jb : je;  // ja <= jbb (i_a < i_b, same chunk)
+  const int32_t j1 = min(jbb, je);
+  // phase 1: only point A has partners
+  for (int32_t j = ja; j < j1; ++j) tp_count<CNT>(p, Hw, A, tp_binof<LUT>(L, E, tp_dot(A, Bs[j])));
+  if (!va) {
+    for (int32_t j = jbb; j < je; ++j) tp_count<CNT>(p, Hw, B, tp_binof<LUT>(L, E, tp_dot(B, Bs[j])));
+    return;
+  }
+  // phase 2: both points, one shared partner load
+  int32_t j = max(jbb, ja);
+  for (; j + 3 < je; j += 4) {
+    const float4 q0 = Bs[j], q1 = Bs[j + 1], q2 = Bs[j + 2], q3 = Bs[j + 3];
+    const int32_t a0 = tp_binof<LUT>(L, E, tp_dot(A, q0)), b0 = tp_binof<LUT>(L, E, tp_dot(B, q0));
+    const int32_t a1 = tp_binof<LUT>(L, E, tp_dot(A, q1)), b1 = tp_binof<LUT>(L, E, tp_dot(B, q1));
+    const int32_t a2 = tp_binof<LUT>(L, E, tp_dot(A, q2)), b2 = tp_binof<LUT>(L, E, tp_dot(B, q2));
+    const int32_t a3 = tp_binof<LUT>(L, E, tp_dot(A, q3)), b3 = tp_binof<LUT>(L, E, tp_dot(B, q3));
+    tp_count<CNT>(p, Hw, A, a0); tp_count<CNT>(p, Hw, B, b0);
+    tp_count<CNT>(p, Hw, A, a1); tp_count<CNT>(p, Hw, B, b1);
+    tp_count<CNT>(p, Hw, A, a2); tp_count<CNT>(p, Hw, B, b2);
+    tp_count<CNT>(p, Hw, A, a3); tp_count<CNT>(p, Hw, B, b3);
+  }
+  for (; j < je; ++j) {
+    const float4 q = Bs[j];
+    const int32_t a = tp_binof<LUT>(L, E, tp_dot(A, q)), b = tp_binof<LUT>(L, E, tp_dot(B, q));
+    tp_count<CNT>(p, Hw, A, a);
+    tp_count<CNT>(p, Hw, B, b);
+  }
+}
+
+template <int V>
+__device__ __forceinline__ void tpacf_body(const TPParams& p, const TPSmem& S, unsigned long long* hist, hk_control* cb) {
+  constexpr bool NL = (V & V_NL) != 0, L = (V & V_L) != 0;
+  const int32_t nr = p.nr, nC = p.nC, nb2 = p.nb + 2;
   const int32_t row = blockIdx.y;
-  const int32_t i = blockIdx.x * TP_THREADS + threadIdx.x;
-  const bool active = i < n;
   const int32_t h = row / nC, c = row - h * nC;
   const int32_t sb = (h == 0) ? 0 : (h <= nr ? h : h - nr);
   const bool work = tp_cta_has_work(p, h, c);
@@ -170,83 +303,19 @@ __device__ __forceinline__ void tpacf_body(const TPParams& p, const TPSmem& S, u
   tp_stage(p, S, sb, c, work);
   __syncthreads();
   const uint32_t lane = lane_id(), warp = threadIdx.x >> 5;
-  if (active) {
-    uint32_t chk = 0, alarm = 0;
-    if (NL) {
-      chk ^= (uint32_t)n ^ lohi_ptr(p.pts) ^ lohi_ptr(hist);
-      chk ^= (uint32_t)i; alarm |= ((int32_t)((blockIdx.x ^ z) * TP_THREADS + (threadIdx.x ^ z)) != i) ? AL_DUP : 0u;
-      chk ^= (uint32_t)h; alarm |= ((int32_t)(blockIdx.y ^ z) / nC != h) ? AL_DUP : 0u;
-      chk ^= (uint32_t)c; alarm |= ((int32_t)(row - opq(h, z) * nC) != c) ? AL_DUP : 0u;
-    }
-    const int32_t aoff = (h <= nr ? h : 0) * n + i;
-    const int32_t boff = sb * n;
-    const int32_t jb = h <= nr ? max(i + 1, c * C) : c * C;
-    const int32_t je = min((c + 1) * C, n);
-    const int32_t expect = max(je - jb, 0);
-    const int32_t base = h * nb2;
-    if (NL) {
-      const int32_t h2 = opq(h, z), i2 = opq(i, z), c2 = opq(c, z);
-      chk ^= (uint32_t)aoff; alarm |= ((h2 <= nr ? h2 : 0) * n + i2 != aoff) ? AL_DUP : 0u;
-      chk ^= (uint32_t)boff; alarm |= ((h2 == 0 ? 0 : (h2 <= nr ? h2 : h2 - nr)) * n != boff) ? AL_DUP : 0u;
-      chk ^= (uint32_t)jb; alarm |= ((h2 <= nr ? max(i2 + 1, c2 * C) : c2 * C) != jb) ? AL_DUP : 0u;
-      chk ^= (uint32_t)je; alarm |= (min((c2 + 1) * C, n) != je) ? AL_DUP : 0u;
-      chk ^= (uint32_t)expect; alarm |= (max(opq(je, z) - jb, 0) != expect) ? AL_DUP : 0u;
-      chk ^= (uint32_t)base; alarm |= (h2 * nb2 != base) ? AL_DUP : 0u;
-    }
-    const float* A = p.pts + 3 * (int64_t)aoff;
-    const float x1 = A[0], y1 = A[1], z1 = A[2];
-    if (NL) {
-      const float* A2 = p.pts + 3 * (int64_t)opq(aoff, z);
-      chk ^= fb(x1); alarm |= (fb(A2[0]) != fb(x1)) ? AL_DUP : 0u;
-      chk ^= fb(y1); alarm |= (fb(A2[1]) != fb(y1)) ? AL_DUP : 0u;
-      chk ^= fb(z1); alarm |= (fb(A2[2]) != fb(z1)) ? AL_DUP : 0u;
-      chk ^= (uint32_t)opq(i, z) ^ (uint32_t)opq(h, z) ^ (uint32_t)opq(c, z) ^ (uint32_t)opq(aoff, z) ^ (uint32_t)opq(jb, z);
-    }
-    int32_t acc = 0, cnt = 0;
-    const float4* Bs = S.B - c * C;  // Bs[j] for j in chunk c
-    uint32_t* Hw = S.H + (size_t)warp * nb2 * 32 + lane;
-    if (use_lut) {
-      const int2* Ls = S.L;
-#pragma unroll 4
-      for (int32_t j = jb; j < je; ++j) {
-        const float4 q = Bs[j];
-        const float dot = __fmaf_rn(z1, q.z, __fmaf_rn(y1, q.y, __fmul_rn(x1, q.x)));
-        const int32_t bin = tp_bin_lut(Ls, dot);
-        Hw[bin * 32] += 1u;
-        if (L || PROF) {
-          acc += bin;
-          cnt = count_inc(cnt, p.one);
-        }
-      }
-    } else {
-#pragma unroll 4
-      for (int32_t j = jb; j < je; ++j) {
-        const float4 q = Bs[j];
-        const float dot = __fmaf_rn(z1, q.z, __fmaf_rn(y1, q.y, __fmul_rn(x1, q.x)));
-        const int32_t bin = tp_bin(S.E, dot);
-        Hw[bin * 32] += 1u;
-        if (L || PROF) {
-          acc += bin;
-          cnt = count_inc(cnt, p.one);
-        }
-      }
-    }
-    if (L && cnt != expect) alarm |= AL_COUNT;
-    if (CNT && cnt != 0 && p.ndet > 0) {
-      const float v = __fdiv_rn((float)acc, (float)cnt);
-      if (PROF) p.samples[(int64_t)row * n + i] = v;
-      if (L && p.R.n[0] > 0 && !in_range<false>(p.R, 0, v, nullptr)) {
-        alarm |= AL_RANGE;
-        record_outlier(cb, 0, v);
-      }
-    }
-    if (NL) {
-      chk ^= (uint32_t)opq(boff, z) ^ (uint32_t)opq(je, z) ^ (uint32_t)opq(base, z);
-      chk ^= opqf(x1, z) ^ opqf(y1, z) ^ opqf(z1, z) ^ (uint32_t)opq(expect, z);
-      chk ^= ((uint32_t)n + z) ^ (lohi_ptr(p.pts) + z) ^ (lohi_ptr(hist) + z);
-      if (chk != 0) alarm |= AL_CHK;
-    }
-    if (NL || L) fold_alarm(cb, alarm, (uint32_t)((int64_t)row * n + i));
+  uint32_t* Hw = S.H + (size_t)warp * nb2 * 32 + lane;
+  TPPoint A = tp_prologue<NL>(p, hist, 0);
+  TPPoint B = tp_prologue<NL>(p, hist, 1);
+  const bool va = A.i < p.n, vb = B.i < p.n;
+  if (use_lut) tp_loops<V, true>(p, S, Hw, A, B, va, vb);
+  else tp_loops<V, false>(p, S, Hw, A, B, va, vb);
+  if (va) {
+    tp_epilogue<V>(p, A, hist, cb);
+    if (NL || L) fold_alarm(cb, A.alarm, (uint32_t)((int64_t)row * p.n + A.i));
+  }
+  if (vb) {
+    tp_epilogue<V>(p, B, hist, cb);
+    if (NL || L) fold_alarm(cb, B.alarm, (uint32_t)((int64_t)row * p.n + B.i));
   }
   if (work) {
     __syncthreads();
@@ -276,11 +345,11 @@ struct TPFIParams {
 
 template <int KIND>
 __device__ void tpacf_fi_thread(const TPParams& p, const TPSmem& S, const FaultRec& f, unsigned long long* hist,
-                                hk_control* cb) {
+                                hk_control* cb, int kpt) {
   const uint32_t z = p.z;
   const int32_t nr = p.nr, C = p.C, nC = p.nC, nb2 = p.nb + 2;
   const int32_t row = blockIdx.y;
-  const int32_t ii = blockIdx.x * TP_THREADS + threadIdx.x;
+  const int32_t ii = blockIdx.x * TP_CTA_PTS + kpt * TP_THREADS + threadIdx.x;
   if (ii >= p.n) return;
   const int64_t g = (int64_t)row * p.n + ii;
   const bool mine = (g == f.thread);
@@ -298,7 +367,8 @@ __device__ void tpacf_fi_thread(const TPParams& p, const TPSmem& S, const FaultR
   const bool nl = (KIND == TK_NL) && mine;
 #define NLF(v, s) do { const bool _n = nl && site == (s); applied |= _n; v = flip_i(v, _n, mask); } while (0)
   int32_t i = ii; NLF(i, 0);
-  chk ^= (uint32_t)i; alarm |= ((int32_t)((blockIdx.x ^ z) * TP_THREADS + (threadIdx.x ^ z)) != i) ? AL_DUP : 0u;
+  chk ^= (uint32_t)i;
+  alarm |= ((int32_t)((blockIdx.x ^ z) * TP_CTA_PTS + kpt * TP_THREADS + (threadIdx.x ^ z)) != i) ? AL_DUP : 0u;
   int32_t h = row / nC; NLF(h, 1);
   chk ^= (uint32_t)h; alarm |= ((int32_t)(blockIdx.y ^ z) / nC != h) ? AL_DUP : 0u;
   int32_t c = (int32_t)((uint32_t)row - (uint32_t)h * (uint32_t)nC); NLF(c, 2);
@@ -418,8 +488,8 @@ __global__ void __launch_bounds__(TP_THREADS) tpacf_fi_kernel(const TPFIParams q
   const FaultRec f = q.faults[r];
   unsigned long long* hist = q.hist0 + (int64_t)r * q.hist_elems;
   hk_control* cb = q.cb0 + r;
-  const int64_t cta_first = (int64_t)blockIdx.y * q.base.n + (int64_t)blockIdx.x * TP_THREADS;
-  if (f.thread < cta_first || f.thread >= cta_first + TP_THREADS) {
+  const int64_t cta_first = (int64_t)blockIdx.y * q.base.n + (int64_t)blockIdx.x * TP_CTA_PTS;
+  if (f.thread < cta_first || f.thread >= cta_first + TP_CTA_PTS) {
     tpacf_body<V_NL | V_L>(q.base, S, hist, cb);
   } else {
     const TPParams& p = q.base;
@@ -427,7 +497,8 @@ __global__ void __launch_bounds__(TP_THREADS) tpacf_fi_kernel(const TPFIParams q
     const int32_t sb = (h == 0) ? 0 : (h <= p.nr ? h : h - p.nr);
     tp_stage(p, S, sb, c, true);
     __syncthreads();
-    tpacf_fi_thread<KIND>(p, S, f, hist, cb);
+    tpacf_fi_thread<KIND>(p, S, f, hist, cb, 0);
+    tpacf_fi_thread<KIND>(p, S, f, hist, cb, 1);
     __syncthreads();
     tp_flush(p, S, hist, h * (p.nb + 2));
   }
@@ -441,8 +512,8 @@ static TPParams tp_params(const hk_tpacf_args& a, const DevRanges& R, int ndet, 
   TPParams p{};
   p.pts = a.pts;
   p.edges = a.edges;
-  p.lut = reinterpret_cast<const int2*>(lut_ws);
-  p.lut_ok = reinterpret_cast<const int*>(reinterpret_cast<const char*>(lut_ws) + TP_LUT * sizeof(int2));
+  p.lut = reinterpret_cast<const uint8_t*>(lut_ws);
+  p.lut_ok = reinterpret_cast<const int*>(reinterpret_cast<const char*>(lut_ws) + TP_LUT);
   p.hist = a.hist;
   p.cb = cb;
   p.samples = samples;
@@ -458,13 +529,13 @@ static TPParams tp_params(const hk_tpacf_args& a, const DevRanges& R, int ndet, 
   return p;
 }
 
-size_t tpacf_lut_ws_bytes() { return TP_LUT * sizeof(int2) + 16; }
+size_t tpacf_lut_ws_bytes() { return TP_LUT + 16; }
 
 cudaError_t tpacf_lut_build(const hk_tpacf_args& a, void* lut_ws, cudaStream_t s) {
-  int* ok = reinterpret_cast<int*>(reinterpret_cast<char*>(lut_ws) + TP_LUT * sizeof(int2));
+  int* ok = reinterpret_cast<int*>(reinterpret_cast<char*>(lut_ws) + TP_LUT);
   cudaError_t e = cudaMemsetAsync(ok, 1, sizeof(int), s);
   if (e != cudaSuccess) return e;
-  tpacf_lut_kernel<<<TP_LUT / 256, 256, 0, s>>>(a.edges, a.n_bins, reinterpret_cast<int2*>(lut_ws), ok);
+  tpacf_lut_kernel<<<TP_LUT / 256, 256, 0, s>>>(a.edges, a.n_bins, reinterpret_cast<uint8_t*>(lut_ws), ok);
   count_launch();
   return cudaGetLastError();
 }
@@ -479,7 +550,7 @@ static cudaError_t launch_tp_v(const TPParams& p, cudaStream_t s) {
   const size_t smem = tp_smem_bytes(p.C, p.nb + 2);
   cudaError_t e = cudaFuncSetAttribute(tpacf_kernel<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  dim3 grid((p.n + TP_THREADS - 1) / TP_THREADS, (1 + 2 * p.nr) * p.nC);
+  dim3 grid((p.n + TP_CTA_PTS - 1) / TP_CTA_PTS, (1 + 2 * p.nr) * p.nC);
   if (grid.x == 0) return cudaSuccess;
   TimedScope ts(HK_TPACF, 0, tp_pairs(p), s);
   tpacf_kernel<V><<<grid, TP_THREADS, smem, s>>>(p);
@@ -513,7 +584,7 @@ static cudaError_t launch_tp_fi_k(const TPFIParams& q, int nrep, cudaStream_t s)
   const size_t smem = tp_smem_bytes(q.base.C, q.base.nb + 2);
   cudaError_t e = cudaFuncSetAttribute(tpacf_fi_kernel<KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  dim3 grid((q.base.n + TP_THREADS - 1) / TP_THREADS, (1 + 2 * q.base.nr) * q.base.nC, nrep);
+  dim3 grid((q.base.n + TP_CTA_PTS - 1) / TP_CTA_PTS, (1 + 2 * q.base.nr) * q.base.nC, nrep);
   TimedScope ts(HK_TPACF, 1, tp_pairs(q.base) * nrep, s);
   tpacf_fi_kernel<KIND><<<grid, TP_THREADS, smem, s>>>(q);
   count_launch();

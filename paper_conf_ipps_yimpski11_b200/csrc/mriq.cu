@@ -54,31 +54,44 @@ __global__ void __launch_bounds__(256) mriq_phimag_kernel(const float* __restric
   if (NL) fold_alarm(cb, alarm, (uint32_t)k);
 }
 
-template <int V, bool EXACT, bool ADD>
+// VPT voxels (abstract threads) per CUDA thread: voxel j of thread t in CTA b is
+// b*(blockDim*VPT) + j*blockDim + t.  Each keeps its own registers, detectors and counter; they
+// share every k-space load (VPT = 2 in the campaign replicas, 1 for the single-run kernel whose
+// grid is small).
+template <int V, bool EXACT, bool ADD, int VPT>
 __device__ __forceinline__ void mriq_body(const MQParams& p, float4 (*tile)[MQ_TILE], uint64_t* bar) {
   constexpr bool NL = (V & V_NL) != 0, L = (V & V_L) != 0, PROF = (V & V_PROF) != 0;
   constexpr bool CNT = L || PROF;
   const uint32_t z = p.zz;
-  const int32_t xIndex = blockIdx.x * blockDim.x + threadIdx.x;
-  const bool active = xIndex < p.numX;
   const int32_t numK = p.numK;
-  uint32_t chk = 0, alarm = 0;
-  float sX = 0.f, sY = 0.f, sZ = 0.f;
-  if (active) {
-    if (NL) {
-      chk ^= (uint32_t)numK ^ lohi_ptr(p.kv) ^ lohi_ptr(p.qr) ^ lohi_ptr(p.qi) ^ lohi_ptr(p.x) ^ lohi_ptr(p.y) ^ lohi_ptr(p.z);
-      chk ^= (uint32_t)xIndex;
-      alarm |= ((int32_t)((blockIdx.x ^ z) * blockDim.x + (threadIdx.x ^ z)) != xIndex) ? AL_DUP : 0u;
+  int32_t xIndex[VPT];
+  bool active[VPT];
+  uint32_t chk[VPT], alarm[VPT];
+  float sX[VPT], sY[VPT], sZ[VPT], Qr[VPT], Qi[VPT];
+  int32_t it[VPT];
+#pragma unroll
+  for (int v = 0; v < VPT; ++v) {
+    xIndex[v] = blockIdx.x * (blockDim.x * VPT) + v * blockDim.x + threadIdx.x;
+    active[v] = xIndex[v] < p.numX;
+    chk[v] = 0; alarm[v] = 0;
+    sX[v] = sY[v] = sZ[v] = 0.f;
+    Qr[v] = Qi[v] = 0.f;
+    it[v] = 0;
+    if (active[v]) {
+      const int32_t xi = xIndex[v];
+      if (NL) {
+        chk[v] ^= (uint32_t)numK ^ lohi_ptr(p.kv) ^ lohi_ptr(p.qr) ^ lohi_ptr(p.qi) ^ lohi_ptr(p.x) ^ lohi_ptr(p.y) ^ lohi_ptr(p.z);
+        chk[v] ^= (uint32_t)xi;
+        alarm[v] |= ((int32_t)((blockIdx.x ^ z) * (blockDim.x * VPT) + v * blockDim.x + (threadIdx.x ^ z)) != xi) ? AL_DUP : 0u;
+      }
+      sX[v] = p.x[xi];
+      if (NL) { chk[v] ^= fb(sX[v]); alarm[v] |= (fb(p.x[opq(xi, z)]) != fb(sX[v])) ? AL_DUP : 0u; }
+      sY[v] = p.y[xi];
+      if (NL) { chk[v] ^= fb(sY[v]); alarm[v] |= (fb(p.y[opq(xi, z)]) != fb(sY[v])) ? AL_DUP : 0u; }
+      sZ[v] = p.z[xi];
+      if (NL) { chk[v] ^= fb(sZ[v]); alarm[v] |= (fb(p.z[opq(xi, z)]) != fb(sZ[v])) ? AL_DUP : 0u; }
     }
-    sX = p.x[xIndex];
-    if (NL) { chk ^= fb(sX); alarm |= (fb(p.x[opq(xIndex, z)]) != fb(sX)) ? AL_DUP : 0u; }
-    sY = p.y[xIndex];
-    if (NL) { chk ^= fb(sY); alarm |= (fb(p.y[opq(xIndex, z)]) != fb(sY)) ? AL_DUP : 0u; }
-    sZ = p.z[xIndex];
-    if (NL) { chk ^= fb(sZ); alarm |= (fb(p.z[opq(xIndex, z)]) != fb(sZ)) ? AL_DUP : 0u; }
   }
-  float Qr = 0.f, Qi = 0.f;
-  int32_t it = 0;
   const int ntiles = (numK + MQ_TILE - 1) / MQ_TILE;
   if (threadIdx.x == 0) {
     mbar_init(&bar[0], 1);
@@ -87,6 +100,9 @@ __device__ __forceinline__ void mriq_body(const MQParams& p, float4 (*tile)[MQ_T
   }
   __syncthreads();
   if (threadIdx.x == 0 && ntiles > 0) bulk_g2s(tile[0], p.kv, (uint32_t)min(MQ_TILE, numK) * 16u, &bar[0]);
+  bool any_active = false;
+#pragma unroll
+  for (int v = 0; v < VPT; ++v) any_active |= active[v];
   for (int t = 0; t < ntiles; ++t) {
     const int buf = t & 1;
     if (threadIdx.x == 0 && t + 1 < ntiles) {
@@ -95,61 +111,69 @@ __device__ __forceinline__ void mriq_body(const MQParams& p, float4 (*tile)[MQ_T
                &bar[buf ^ 1]);
     }
     mbar_wait(&bar[buf], (uint32_t)(t >> 1) & 1u);
-    if (active) {
+    if (any_active) {
       const float4* A = tile[buf];
       const int cnt = min(MQ_TILE, numK - t * MQ_TILE);
-#pragma unroll 4
+#pragma unroll(VPT == 1 ? 4 : 2)
       for (int a = 0; a < cnt; ++a) {
         const float4 k4 = A[a];
-        const float t1 = __fmul_rn(k4.x, sX);
-        const float t2 = __fmaf_rn(k4.y, sY, t1);
-        const float tt = __fmaf_rn(k4.z, sZ, t2);
-        const float m = __fsub_rn(__fadd_rn(tt, RINT_MAGIC), RINT_MAGIC);
-        const float r = __fsub_rn(tt, m);
-        const float ang = __fmul_rn(r, TWO_PI_F);
-        const float c = hk_cos<EXACT>(ang);
-        const float s = hk_sin<EXACT>(ang);
-        Qr = __fmaf_rn(k4.w, c, Qr);
-        Qi = __fmaf_rn(k4.w, s, Qi);
-        if (CNT) it = count_inc(it, p.one);
+#pragma unroll
+        for (int v = 0; v < VPT; ++v) {
+          const float t1 = __fmul_rn(k4.x, sX[v]);
+          const float t2 = __fmaf_rn(k4.y, sY[v], t1);
+          const float tt = __fmaf_rn(k4.z, sZ[v], t2);
+          const float m = __fsub_rn(__fadd_rn(tt, RINT_MAGIC), RINT_MAGIC);
+          const float r = __fsub_rn(tt, m);
+          const float ang = __fmul_rn(r, TWO_PI_F);
+          const float c = hk_cos<EXACT>(ang);
+          const float s = hk_sin<EXACT>(ang);
+          Qr[v] = __fmaf_rn(k4.w, c, Qr[v]);
+          Qi[v] = __fmaf_rn(k4.w, s, Qi[v]);
+          if (CNT) it[v] = count_inc(it[v], p.one);
+        }
       }
     }
     __syncthreads();
   }
-  if (active) {
-    if (L && it != numK) alarm |= AL_COUNT;
-    if (CNT && it != 0) {
-      const float fit = (float)it;
+#pragma unroll
+  for (int v = 0; v < VPT; ++v) {
+    if (!active[v]) continue;
+    const int32_t xi = xIndex[v];
+    if (L && it[v] != numK) alarm[v] |= AL_COUNT;
+    if (CNT && it[v] != 0) {
+      const float fit = (float)it[v];
 #pragma unroll
       for (int d = 0; d < 2; ++d) {
         if (d < p.ndet) {
-          const float v = __fdiv_rn(d == 0 ? Qr : Qi, fit);
-          if (PROF) p.samples[(int64_t)d * p.numX + xIndex] = v;
-          if (L && p.R.n[d] > 0 && !in_range<false>(p.R, d, v, nullptr)) {
-            alarm |= AL_RANGE;
-            record_outlier(p.cb, d, v);
+          const float val = __fdiv_rn(d == 0 ? Qr[v] : Qi[v], fit);
+          if (PROF) p.samples[(int64_t)d * p.numX + xi] = val;
+          if (L && p.R.n[d] > 0 && !in_range<false>(p.R, d, val, nullptr)) {
+            alarm[v] |= AL_RANGE;
+            record_outlier(p.cb, d, val);
           }
         }
       }
     }
-    if (NL) { chk ^= opqf(sX, z); chk ^= opqf(sY, z); chk ^= opqf(sZ, z); }
-    if (ADD) { atomicAdd(p.qr + xIndex, Qr); atomicAdd(p.qi + xIndex, Qi); }
-    else { p.qr[xIndex] = Qr; p.qi[xIndex] = Qi; }
+    if (NL) { chk[v] ^= opqf(sX[v], z); chk[v] ^= opqf(sY[v], z); chk[v] ^= opqf(sZ[v], z); }
+    if (ADD) { atomicAdd(p.qr + xi, Qr[v]); atomicAdd(p.qi + xi, Qi[v]); }
+    else { p.qr[xi] = Qr[v]; p.qi[xi] = Qi[v]; }
     if (NL) {
-      chk ^= (uint32_t)opq(xIndex, z);
-      chk ^= ((uint32_t)numK + z) ^ (lohi_ptr(p.kv) + z) ^ (lohi_ptr(p.qr) + z) ^ (lohi_ptr(p.qi) + z) ^
-             (lohi_ptr(p.x) + z) ^ (lohi_ptr(p.y) + z) ^ (lohi_ptr(p.z) + z);
-      if (chk != 0) alarm |= AL_CHK;
+      chk[v] ^= (uint32_t)opq(xi, z);
+      chk[v] ^= ((uint32_t)numK + z) ^ (lohi_ptr(p.kv) + z) ^ (lohi_ptr(p.qr) + z) ^ (lohi_ptr(p.qi) + z) ^
+                (lohi_ptr(p.x) + z) ^ (lohi_ptr(p.y) + z) ^ (lohi_ptr(p.z) + z);
+      if (chk[v] != 0) alarm[v] |= AL_CHK;
     }
-    if (NL || L) fold_alarm(p.cb, alarm, (uint32_t)xIndex);
   }
+#pragma unroll
+  for (int v = 0; v < VPT; ++v)
+    if ((NL || L) && active[v]) fold_alarm(p.cb, alarm[v], (uint32_t)xIndex[v]);
 }
 
 template <int V, bool EXACT>
 __global__ void __launch_bounds__(256) mriq_kernel(const MQParams p) {
   __shared__ __align__(128) float4 tile[2][MQ_TILE];
   __shared__ __align__(8) uint64_t bar[2];
-  mriq_body<V, EXACT, false>(p, tile, bar);
+  mriq_body<V, EXACT, false, 1>(p, tile, bar);
 }
 
 // ============================================================================================
@@ -168,8 +192,8 @@ struct MQFIParams {
 };
 
 template <int KIND, bool EXACT>
-__device__ void mriq_fi_thread(const MQParams& p, const FaultRec& f) {
-  const int32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+__device__ void mriq_fi_thread(const MQParams& p, const FaultRec& f, int vox) {
+  const int32_t t = blockIdx.x * (2 * blockDim.x) + vox * blockDim.x + threadIdx.x;
   if (t >= p.numX) return;
   const bool mine = (t == f.thread);
   const int64_t inst = mine ? f.inst : -1;
@@ -188,7 +212,8 @@ __device__ void mriq_fi_thread(const MQParams& p, const FaultRec& f) {
   const bool nl = (KIND == MK_NL) && mine;
   int32_t xIndex = t;
   { const bool n = nl && site == 0; applied |= n; xIndex = flip_i(xIndex, n, mask); }
-  chk ^= (uint32_t)xIndex; alarm |= ((int32_t)((blockIdx.x ^ z) * blockDim.x + (threadIdx.x ^ z)) != xIndex) ? AL_DUP : 0u;
+  chk ^= (uint32_t)xIndex;
+  alarm |= ((int32_t)((blockIdx.x ^ z) * (2 * blockDim.x) + vox * blockDim.x + (threadIdx.x ^ z)) != xIndex) ? AL_DUP : 0u;
   float sX, sY, sZ, Qr = 0.f, Qi = 0.f;
   int32_t it = 0, k = 0;
   int64_t e;
@@ -299,8 +324,12 @@ __global__ void __launch_bounds__(256) mriq_fi_kernel(const MQFIParams q) {
   p.qr = q.out0 + (int64_t)r * q.stride;
   p.qi = p.qr + p.numX;
   p.cb = q.cb0 + r;
-  if (f.thread / blockDim.x != blockIdx.x) mriq_body<V_NL | V_L, EXACT, true>(p, tile, bar);
-  else mriq_fi_thread<KIND, EXACT>(p, f);
+  if (f.thread / (2 * blockDim.x) != blockIdx.x) {
+    mriq_body<V_NL | V_L, EXACT, true, 2>(p, tile, bar);
+  } else {
+    mriq_fi_thread<KIND, EXACT>(p, f, 0);
+    mriq_fi_thread<KIND, EXACT>(p, f, 1);
+  }
 }
 
 // ============================================================================================
@@ -362,7 +391,7 @@ int mriq_site_kind(int site) {
 
 template <int KIND, bool EXACT>
 static cudaError_t launch_mq_fi_k(const MQFIParams& q, int nrep, cudaStream_t s) {
-  dim3 grid((q.base.numX + 255) / 256, nrep);
+  dim3 grid((q.base.numX + 511) / 512, nrep);
   TimedScope ts(HK_MRIQ, 1, (double)q.base.numX * (double)q.base.numK * nrep, s);
   mriq_fi_kernel<KIND, EXACT><<<grid, 256, 0, s>>>(q);
   count_launch();

@@ -43,6 +43,7 @@ def parse():
     ap.add_argument("--batch", type=int, default=0)
     ap.add_argument("--no-overhead", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-multibit", action="store_true")
     return ap.parse_args()
 
 
@@ -316,6 +317,22 @@ def main():
                          f"mean s/injection cp={tm[0]:.4f} mriq={tm[1]:.3f} tpacf={tm[2]:.3f}"}
 
     session.close()
+
+    # ---- coverage vs number of flipped bits (Fig. 14; NEXT f1): the same
+    #      injection indices with k-bit masks (untimed)
+    multibit = {}
+    if not args.no_multibit:
+        for k in (3, 6, 10, 15):
+            ck = torch.zeros((3, 5), dtype=torch.int64, device=dev)
+            with hk.CampaignSession(-1, devs, ranges, seed, batch=args.batch, nbits=k) as sk:
+                first, cnt = par.step_slice(0, rank, world, args.per_rank)
+                sk.run(first, cnt, ck)
+                torch.cuda.synchronize()
+            par.all_reduce_counts(ck)
+            cc = ck.cpu().numpy()
+            multibit[str(k)] = {"coverage_pct": round(100.0 * hk.coverage(cc), 3),
+                                "coverage_by_bench_pct": {hk.BENCH_NAMES[b]: round(100.0 * hk.coverage(cc[b]), 3) for b in range(3)},
+                                "outcomes_pct": dict(zip(hk.CLASS_NAMES, (100.0 * cc.sum(0) / max(1, cc.sum())).round(2).tolist()))}
     if rank == 0:
         line = {
             "metric": METRIC, "value": round(value, 2), "unit": "injections/s", "n_gpus": world, "steps": args.steps,
@@ -337,6 +354,8 @@ def main():
             "outcomes": {hk.BENCH_NAMES[b]: dict(zip(hk.CLASS_NAMES, c[b].tolist())) for b in range(3)},
             "coverage_by_bench_pct": {hk.BENCH_NAMES[b]: round(100.0 * hk.coverage(c[b]), 3) for b in range(3)},
             "overhead_pct": overhead, "kernels": kernels, "fi_kernels": fi_split,
+            "coverage_vs_bits": multibit,
+            "outcomes_pct_1bit": dict(zip(hk.CLASS_NAMES, (100.0 * c.sum(0) / max(1, c.sum())).round(2).tolist())),
             "ranges_identical_across_ranks": ranges_identical,
             "paper_context": {"overhead_pct_avg7": 15.3, "coverage_pct_avg": 86.8, "hardware": "Tesla S1070 (GT200)",
                               "source": "PAPER.md L186-189, L2401-2404, L2480-2483"},

@@ -109,8 +109,10 @@ typedef struct {
 typedef struct { int32_t maxvar; int32_t t0_exp10; float alpha; } hk_profile_opts; /* defaults 1, -5, 1 */
 
 /* Campaign (L2295-2305, L2370-2387).  Injections n in [first, first+count) decoded from
- * (seed, n) (DESIGN R14-R15); mode 0 = replica (every injection is a full program run; the only
- * mode of this version); batch = replicas per launch (0 = auto); site_mask[b] bit s enables site s. */
+ * (seed, n) (DESIGN R14-R15); nbits = bits flipped per injection (0/1 = single-bit; 3, 6, 10, 15
+ * reproduce Fig. 14's multi-bit masks, L2691); mode 0 = replica (every injection is a full program
+ * run; the only mode of this version); batch = replicas per launch (0 = auto); site_mask[b] bit s
+ * enables site s. */
 typedef struct {
   uint64_t seed; int64_t first, count; int32_t nbits; int32_t mode; int32_t batch; int32_t exact;
   uint64_t site_mask[3];
@@ -165,9 +167,10 @@ HK_API hk_status hauberk_campaign_run(hk_campaign_session* session, int64_t firs
                                       int64_t* d_counts, int64_t* d_site_counts);
 HK_API void hauberk_campaign_destroy(hk_campaign_session* session);
 
-/* Host-side decode of injections [first, first+count) (same rule the campaign uses). */
+/* Host-side decode of injections [first, first+count) (same rule the campaign uses; nbits as in
+ * hk_campaign: <= 1 single-bit, k > 1 = k distinct bits, DESIGN R15 / NEXT f1). */
 HK_API hk_status hauberk_decode(int32_t bench_mode, const void* const args[3], const uint64_t site_mask[3],
-                         uint64_t seed, int64_t first, int64_t count, int32_t* bench_out, hk_fault* out);
+                         uint64_t seed, int32_t nbits, int64_t first, int64_t count, int32_t* bench_out, hk_fault* out);
 
 /* Number of injection sites of a benchmark (unroll only matters for CP). */
 HK_API int32_t hauberk_num_sites(int32_t bench, int32_t unroll);

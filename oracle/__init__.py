@@ -116,9 +116,9 @@ def lib():
         L.ora_nsites.restype = C.c_int32; L.ora_nsites.argtypes = [C.c_int32, C.c_int32]
         L.ora_site_info.restype = None; L.ora_site_info.argtypes = [C.c_int32, C.c_int32, C.c_int32, P, P]
         L.ora_decode.restype = C.c_int
-        L.ora_decode.argtypes = [C.c_int32, P, P, C.c_uint64, C.c_int64, C.c_int64, P, P]
+        L.ora_decode.argtypes = [C.c_int32, P, P, C.c_uint64, C.c_int32, C.c_int64, C.c_int64, P, P]
         L.ora_campaign.restype = C.c_int
-        L.ora_campaign.argtypes = [C.c_int32, P, P, P, C.c_uint64, C.c_int64, C.c_int64, C.c_int32, C.c_int32, P, P]
+        L.ora_campaign.argtypes = [C.c_int32, P, P, P, C.c_uint64, C.c_int32, C.c_int64, C.c_int64, C.c_int32, C.c_int32, P, P]
         _lib = L
     return _lib
 
@@ -244,7 +244,7 @@ def ranges_to_list(R: Ranges):
 
 
 def campaign(bench_mode: int, problems, ranges, seed: int, first: int, count: int, exact: int = 0,
-             mode: int = 1, site_masks=(ALL_SITES,) * 3, records: bool = True):
+             mode: int = 1, site_masks=(ALL_SITES,) * 3, records: bool = True, nbits: int = 1):
     """Seeded campaign.  problems/ranges: 3-lists indexed by bench (None where unused).
     mode 1 = replay, 0 = replica.  Returns (counts int64[3,5], records structured array)."""
     L = lib()
@@ -255,21 +255,21 @@ def campaign(bench_mode: int, problems, ranges, seed: int, first: int, count: in
     masks = (C.c_uint64 * 3)(*site_masks)
     counts = np.zeros((3, 5), dtype=np.int64)
     recs = np.zeros(count, dtype=RECORD_DTYPE) if records else None
-    rc = L.ora_campaign(bench_mode, aptr, rptr, masks, seed, first, count, exact, mode,
+    rc = L.ora_campaign(bench_mode, aptr, rptr, masks, seed, nbits, first, count, exact, mode,
                         _p(recs) if records else None, _p(counts))
     if rc != 0:
         raise RuntimeError(f"oracle campaign failed rc={rc} (1 = bad args/empty catalogue, 2 = fault-free alarm)")
     return counts, recs
 
 
-def decode(bench_mode: int, problems, seed: int, first: int, count: int, site_masks=(ALL_SITES,) * 3):
+def decode(bench_mode: int, problems, seed: int, first: int, count: int, site_masks=(ALL_SITES,) * 3, nbits: int = 1):
     L = lib()
     argv = [make_args(b, problems[b]) if problems[b] is not None else None for b in range(3)]
     aptr = (C.c_void_p * 3)(*[C.cast(C.byref(a), C.c_void_p) if a is not None else None for a in argv])
     masks = (C.c_uint64 * 3)(*site_masks)
     benches = np.zeros(count, dtype=np.int32)
     faults = (Fault * count)()
-    rc = L.ora_decode(bench_mode, aptr, masks, seed, first, count, _p(benches), C.cast(faults, C.c_void_p))
+    rc = L.ora_decode(bench_mode, aptr, masks, seed, nbits, first, count, _p(benches), C.cast(faults, C.c_void_p))
     if rc != 0:
         raise RuntimeError("decode failed")
     return benches, [(f.site, f.thread, f.inst, f.mask) for f in faults]

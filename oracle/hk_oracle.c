@@ -876,8 +876,12 @@ static void cat_build(catalog* K, int bench, const void* args, uint64_t site_mas
 }
 static void cat_free(catalog* K) { free(K->prefix); K->prefix = NULL; }
 
-/* Decode injection n of a campaign over catalogue K: site, (thread, instance), bit (R14-R15). */
-static void cat_decode(const catalog* K, uint64_t seed, int64_t n, ora_fault* f) {
+/* Decode injection n of a campaign over catalogue K: site, (thread, instance), bits (R14-R15).
+ * nbits <= 1: one bit = bounded(r_3, width).  nbits = k > 1 (NEXT f1; Fig. 14
+ * L2691): k distinct bits by a partial Fisher-Yates shuffle of [0, width): step 0 draws with r_3
+ * (so bit 0 equals the single-bit draw), step t >= 1 with output 16n + t of the stream seeded
+ * seed ^ 0xD1B54A32D192ED03. */
+static void cat_decode(const catalog* K, uint64_t seed, int64_t n, int nbits, ora_fault* f) {
   uint64_t r1 = ora_splitmix(seed, 8 * (uint64_t)n + 1);
   uint64_t r2 = ora_splitmix(seed, 8 * (uint64_t)n + 2);
   uint64_t r3 = ora_splitmix(seed, 8 * (uint64_t)n + 3);
@@ -898,19 +902,30 @@ static void cat_decode(const catalog* K, uint64_t seed, int64_t n, ora_fault* f)
       f->thread = lo; f->inst = u - K->prefix[lo];
     }
   }
-  f->mask = 1ull << ora_bounded(r3, (uint64_t)w);
+  if (nbits <= 1) { f->mask = 1ull << ora_bounded(r3, (uint64_t)w); return; }
+  if (nbits > w) nbits = w;
+  int perm[64];
+  for (int b = 0; b < w; ++b) perm[b] = b;
+  uint64_t mask = 0;
+  for (int t = 0; t < nbits; ++t) {
+    uint64_t r = t == 0 ? r3 : ora_splitmix(seed ^ 0xD1B54A32D192ED03ull, 16 * (uint64_t)n + (uint64_t)t);
+    int j = t + (int)ora_bounded(r, (uint64_t)(w - t));
+    int tmp = perm[t]; perm[t] = perm[j]; perm[j] = tmp;
+    mask |= 1ull << perm[t];
+  }
+  f->mask = mask;
 }
 
 /* Public decode: bench_mode >= 0 fixes the benchmark, -1 = mixed (bench = n mod 3). */
 ORA_EXPORT int ora_decode(int32_t bench_mode, const void* const args[3], const uint64_t site_mask[3],
-                          uint64_t seed, int64_t first, int64_t count, int32_t* bench_out, ora_fault* out) {
+                          uint64_t seed, int32_t nbits, int64_t first, int64_t count, int32_t* bench_out, ora_fault* out) {
   catalog K[3]; int have[3] = {0, 0, 0};
   for (int64_t q = 0; q < count; ++q) {
     int64_t n = first + q;
     int b = bench_mode >= 0 ? bench_mode : (int)(n % 3);
     if (!have[b]) { cat_build(&K[b], b, args[b], site_mask[b]); have[b] = 1; if (K[b].nen == 0) return 1; }
     bench_out[q] = b;
-    cat_decode(&K[b], seed, n, &out[q]);
+    cat_decode(&K[b], seed, n, nbits, &out[q]);
   }
   for (int b = 0; b < 3; ++b) if (have[b]) cat_free(&K[b]);
   return 0;
@@ -1043,7 +1058,7 @@ static void replica_one(int b, const void* args, int exact, const ora_ranges* R,
 
 /* counts[b*5 + cls] += 1 for each injection; records (nullable) get one entry per injection. */
 ORA_EXPORT int ora_campaign(int32_t bench_mode, const void* const args[3], const ora_ranges* const ranges[3],
-                            const uint64_t site_mask[3], uint64_t seed, int64_t first, int64_t count,
+                            const uint64_t site_mask[3], uint64_t seed, int32_t nbits, int64_t first, int64_t count,
                             int32_t exact, int32_t mode, ora_record* records, int64_t* counts) {
   catalog K[3]; goldens G[3]; int have[3] = {0, 0, 0};
   int rc = 0;
@@ -1057,7 +1072,7 @@ ORA_EXPORT int ora_campaign(int32_t bench_mode, const void* const args[3], const
       rc = golden_build(b, args[b], exact, ranges[b], &G[b]);
       if (rc) break;
     }
-    ora_fault f; cat_decode(&K[b], seed, n, &f);
+    ora_fault f; cat_decode(&K[b], seed, n, nbits, &f);
     ora_record rec; memset(&rec, 0, sizeof(rec));
     int32_t wrong = 0;
     if (mode == 1) replay_one(b, args[b], exact, ranges[b], &G[b], &f, &rec, &wrong);

@@ -289,7 +289,7 @@ static bool build_catalog(Catalog& K, int b, const void* args, uint64_t mask) {
   return !K.enabled.empty();
 }
 
-static hk_fault decode_one(const Catalog& K, uint64_t seed, int64_t n) {
+static hk_fault decode_one(const Catalog& K, uint64_t seed, int64_t n, int nbits) {
   hk_fault f{};
   const uint64_t r1 = splitmix(seed, 8 * (uint64_t)n + 1);
   const uint64_t r2 = splitmix(seed, 8 * (uint64_t)n + 2);
@@ -311,7 +311,24 @@ static hk_fault decode_one(const Catalog& K, uint64_t seed, int64_t n) {
       f.inst = u - K.prefix[g];
     }
   }
-  f.mask = 1ull << below(r3, (uint64_t)site_width(K.bench, s));
+  const int w = site_width(K.bench, s);
+  if (nbits <= 1) {
+    f.mask = 1ull << below(r3, (uint64_t)w);
+    return f;
+  }
+  // NEXT f1 (Fig. 14): k distinct bits, partial Fisher-Yates over [0, w);
+  // step 0 uses r_3, step t >= 1 output 16n + t of the stream seed ^ 0xD1B54A32D192ED03.
+  const int k = std::min(nbits, w);
+  int perm[64];
+  for (int b = 0; b < w; ++b) perm[b] = b;
+  uint64_t mask = 0;
+  for (int t = 0; t < k; ++t) {
+    const uint64_t r = t == 0 ? r3 : splitmix(seed ^ 0xD1B54A32D192ED03ull, 16 * (uint64_t)n + (uint64_t)t);
+    const int j = t + (int)below(r, (uint64_t)(w - t));
+    std::swap(perm[t], perm[j]);
+    mask |= 1ull << perm[t];
+  }
+  f.mask = mask;
   return f;
 }
 
@@ -475,7 +492,7 @@ hk_status hauberk_profile_ranges(int32_t bench, const void* args, const hk_profi
 }
 
 hk_status hauberk_decode(int32_t bench_mode, const void* const args[3], const uint64_t site_mask[3], uint64_t seed,
-                         int64_t first, int64_t count, int32_t* bench_out, hk_fault* out) {
+                         int32_t nbits, int64_t first, int64_t count, int32_t* bench_out, hk_fault* out) {
   if (!args || !site_mask || !bench_out || !out || count < 0 || first < 0 || bench_mode < -1 || bench_mode > 2)
     return invalid("decode: bad arguments");
   Catalog K[3];
@@ -489,7 +506,7 @@ hk_status hauberk_decode(int32_t bench_mode, const void* const args[3], const ui
       have[b] = true;
     }
     bench_out[q] = b;
-    out[q] = decode_one(K[b], seed, n);
+    out[q] = decode_one(K[b], seed, n, nbits);
   }
   return HK_OK;
 }
@@ -550,7 +567,7 @@ static hk_status session_create(int32_t bench_mode, const void* const args[3], c
                                 const hk_campaign* C, cudaStream_t s, hk_campaign_session** out) {
   if (!args || !ranges || !C || !out || bench_mode < -1 || bench_mode > 2) return invalid("campaign: bad arguments");
   if (C->mode != 0) { g_err = "only replica mode (0) is implemented on the GPU"; return HK_ERR_UNSUPPORTED; }
-  if (C->nbits != 0 && C->nbits != 1) { g_err = "multi-bit masks are NEXT (f1)"; return HK_ERR_UNSUPPORTED; }
+  if (C->nbits < 0 || C->nbits > 64) return invalid("campaign: nbits out of range");
   keep_pool_memory();
   hk_campaign_session* S = new hk_campaign_session();
   S->bench_mode = bench_mode;
@@ -650,7 +667,7 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
     const int64_t n = first + q;
     const int b = S->bench_mode >= 0 ? S->bench_mode : (int)(n % 3);
     if (!S->W[b].used) return invalid("campaign_run: index hits a benchmark the session was not created with");
-    const hk_fault hf = decode_one(S->K[b], S->cfg.seed, n);
+    const hk_fault hf = decode_one(S->K[b], S->cfg.seed, n, S->cfg.nbits);
     Item it{};
     it.b = b;
     it.f.index = n; it.f.thread = hf.thread; it.f.inst = hf.inst; it.f.mask = hf.mask; it.f.site = hf.site;

@@ -104,7 +104,7 @@ def lib():
         L.hauberk_inject_campaign.restype = I32
         L.hauberk_inject_campaign.argtypes = [I32, P, P, P, P, P, P, P]
         L.hauberk_decode.restype = I32
-        L.hauberk_decode.argtypes = [I32, P, P, U64, I64, I64, P, P]
+        L.hauberk_decode.argtypes = [I32, P, P, U64, I32, I64, I64, P, P]
         L.hauberk_num_sites.restype = I32
         L.hauberk_num_sites.argtypes = [I32, I32]
         L.hauberk_strerror.restype = C.c_char_p
@@ -336,14 +336,14 @@ def _arg_array(devs):
 
 def inject_campaign(bench_mode: int, devs, ranges, seed: int, first: int, count: int, counts: torch.Tensor,
                     records: torch.Tensor | None = None, site_counts: torch.Tensor | None = None, exact: int = 0,
-                    batch: int = 0, site_masks=(ALL_SITES,) * 3, stream=None):
+                    batch: int = 0, site_masks=(ALL_SITES,) * 3, stream=None, nbits: int = 1):
     """hauberk_inject_campaign (replica mode).  devs/ranges: 3-lists by bench (None where unused).
     counts: int64 cuda tensor [3, 5] (accumulated); records: optional uint8 tensor of
     count * OUTCOME_DTYPE.itemsize bytes; site_counts: optional int64 [3, 64, 5]."""
     arr, keep = _arg_array(devs)
     rng = [r if r is not None else Ranges() for r in ranges]
     rarr = (C.c_void_p * 3)(*[C.cast(C.byref(r), C.c_void_p) for r in rng])
-    camp = Campaign(seed, first, count, 1, 0, batch, exact, (C.c_uint64 * 3)(*site_masks))
+    camp = Campaign(seed, first, count, nbits, 0, batch, exact, (C.c_uint64 * 3)(*site_masks))
     st = lib().hauberk_inject_campaign(bench_mode, arr, rarr, C.byref(camp), _ptr(records), _ptr(counts),
                                        _ptr(site_counts), _stream(stream))
     _check(st, "hauberk_inject_campaign")
@@ -354,12 +354,12 @@ class CampaignSession:
     asynchronous slices of the same seeded campaign.  Keep `devs` alive while the session lives."""
 
     def __init__(self, bench_mode: int, devs, ranges, seed: int, exact: int = 0, batch: int = 0,
-                 site_masks=(ALL_SITES,) * 3, stream=None):
+                 site_masks=(ALL_SITES,) * 3, stream=None, nbits: int = 1):
         self._arr, self._keep = _arg_array(devs)
         self._devs = devs
         self._rng = [r if r is not None else Ranges() for r in ranges]
         self._rarr = (C.c_void_p * 3)(*[C.cast(C.byref(r), C.c_void_p) for r in self._rng])
-        self._camp = Campaign(seed, 0, 0, 1, 0, batch, exact, (C.c_uint64 * 3)(*site_masks))
+        self._camp = Campaign(seed, 0, 0, nbits, 0, batch, exact, (C.c_uint64 * 3)(*site_masks))
         self._h = C.c_void_p()
         st = lib().hauberk_campaign_create(bench_mode, self._arr, self._rarr, C.byref(self._camp), C.byref(self._h),
                                            _stream(stream))
@@ -396,13 +396,13 @@ def records_numpy(rec: torch.Tensor) -> np.ndarray:
     return np.frombuffer(rec.cpu().numpy().tobytes(), dtype=OUTCOME_DTYPE)
 
 
-def decode(bench_mode: int, devs, seed: int, first: int, count: int, site_masks=(ALL_SITES,) * 3):
+def decode(bench_mode: int, devs, seed: int, first: int, count: int, site_masks=(ALL_SITES,) * 3, nbits: int = 1):
     """hauberk_decode (host): the campaign's (bench, site, thread, instance, mask) tuples."""
     arr, keep = _arg_array(devs)
     masks = (C.c_uint64 * 3)(*site_masks)
     benches = np.zeros(count, dtype=np.int32)
     faults = (Fault * count)()
-    st = lib().hauberk_decode(bench_mode, arr, masks, seed, first, count, benches.ctypes.data_as(C.c_void_p),
+    st = lib().hauberk_decode(bench_mode, arr, masks, seed, nbits, first, count, benches.ctypes.data_as(C.c_void_p),
                               C.cast(faults, C.c_void_p))
     _check(st, "hauberk_decode")
     return benches, [(f.site, f.thread, f.inst, f.mask) for f in faults]

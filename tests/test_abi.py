@@ -111,3 +111,12 @@ def test_invalid_arguments_fail_before_launch(hk):
     a = d.args()
     st = hk.lib().hauberk_run_cp(C.byref(a), 1, None, C.c_void_p(0x10000), None, None)
     assert st == 3  # FT without ranges -> HK_ERR_NO_RANGES
+
+
+@pytest.mark.parametrize("k", [3, 6, 10, 15])
+def test_multibit_decode_parity_with_oracle(hk, k):
+    probs = [W.cp_config1(), W.mriq_config2(), W.tpacf_config3()]
+    devs = [_FakeDev(hk, b, probs[b]) for b in range(3)]
+    gb, gf = hk.decode(-1, devs, 99, 5000, 1500, nbits=k)
+    ob, of = O.decode(-1, probs, 99, 5000, 1500, nbits=k)
+    assert gf == of

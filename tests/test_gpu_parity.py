@@ -315,3 +315,20 @@ def test_campaign_session_matches_one_shot_calls():
     assert torch.equal(one, ses)
     a, b = hk.records_numpy(rec1), hk.records_numpy(rec2)
     assert np.array_equal(a["cls"], b["cls"]) and np.array_equal(a["index"], b["index"])
+
+
+@pytest.mark.parametrize("k", [3, 15])
+def test_campaign_multibit_exact_mode_bit_exact(k):
+    probs = [W.cp_small(), W.mriq_problem(5, 41, n_vox=100, seed=4), W.tpacf_small(n=90, n_rand=1, chunk=32)]
+    devs = [_mk(b, probs[b], 1) for b in range(3)]
+    gr = [hk.profile_ranges(d) for d in devs]
+    counts = torch.zeros((3, 5), dtype=torch.int64, device=DEV)
+    rec = hk.records_tensor(600, DEV)
+    hk.inject_campaign(-1, devs, gr, 0xF00D, 0, 600, counts, records=rec, exact=1, nbits=k)
+    torch.cuda.synchronize()
+    orr = [O.profile_ranges(b, probs[b], exact=1) for b in range(3)]
+    oc, orec = O.campaign(-1, probs, orr, 0xF00D, 0, 600, exact=1, mode=1, nbits=k)
+    g = hk.records_numpy(rec)
+    assert np.array_equal(g["mask"], orec["mask"])
+    assert np.array_equal(g["cls"], orec["cls"])
+    assert np.array_equal(counts.cpu().numpy(), oc)

@@ -284,3 +284,21 @@ def test_site_catalogue_sizes():
     # 22 + 4U CP sites (38 at U=4, 54 at U=8 ~ "20-50 virtual variables", L2298)
     assert O.nsites(O.CP, 4) == 38 and O.nsites(O.CP, 8) == 54
     assert O.nsites(O.MRIQ) == 29 and O.nsites(O.TPACF) == 31
+
+
+# ---------------------------------------------------------------- multi-bit masks (NEXT f1)
+@pytest.mark.parametrize("k", [3, 6, 10, 15])
+def test_multibit_masks_have_k_distinct_bits_and_extend_the_single_bit_draw(k):
+    probs = [W.cp_small(), W.mriq_small(), W.tpacf_small()]
+    _, one = O.decode(-1, probs, 31337, 0, 3000)
+    _, many = O.decode(-1, probs, 31337, 0, 3000, nbits=k)
+    counts = np.zeros(64)
+    for (s1, t1, i1, m1), (s, t, i, m) in zip(one, many):
+        assert (s1, t1, i1) == (s, t, i)                      # same site / thread / instance
+        assert m & m1 == m1                                   # step 0 of the shuffle = the single-bit draw
+        assert bin(m).count("1") == k
+        for b in range(64):
+            counts[b] += (m >> b) & 1
+    # 32-bit sites dominate; every bit position of a 32-bit word is used ~uniformly
+    c32 = counts[:32]
+    assert c32.min() > 0.7 * c32.mean()

@@ -111,8 +111,10 @@ typedef struct { int32_t maxvar; int32_t t0_exp10; float alpha; } hk_profile_opt
 /* Campaign (L2295-2305, L2370-2387).  Injections n in [first, first+count) decoded from
  * (seed, n) (DESIGN R14-R15); nbits = bits flipped per injection (0/1 = single-bit; 3, 6, 10, 15
  * reproduce Fig. 14's multi-bit masks, L2691); mode 0 = replica (every injection is a full program
- * run; the only mode of this version); batch = replicas per launch (0 = auto); site_mask[b] bit s
- * enables site s. */
+ * run, the paper's definition), mode 1 = replay (one CUDA thread re-runs only the
+ * faulted abstract thread and classifies the golden output patched with its writes — identical
+ * outcomes; TPACF n_bins <= 32); batch = replicas per launch (0 = auto); site_mask[b]
+ * bit s enables site s. */
 typedef struct {
   uint64_t seed; int64_t first, count; int32_t nbits; int32_t mode; int32_t batch; int32_t exact;
   uint64_t site_mask[3];

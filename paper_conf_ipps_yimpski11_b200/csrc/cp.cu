@@ -169,20 +169,34 @@ struct CPFIParams {
   hk_control* cb0;
 };
 
-template <int KIND, int U, bool EXACT>
-__device__ void cp_fi_thread(const CPParams& p, const FaultRec& f, float* grid, hk_control* cb) {
-  const int BX = blockDim.x, BY = blockDim.y;
-  const int tx = threadIdx.x, ty = threadIdx.y;
-  const int bxi = blockIdx.x, byi = blockIdx.y;
-  const int64_t t = ((int64_t)byi * gridDim.x + bxi) * (BX * BY) + ty * BX + tx;
-  const bool mine = (t == f.thread);
+// Launch geometry of one abstract CP thread (CUDA indices of its replica CTA, or reconstructed
+// from the abstract id in replay mode).
+struct CPGeo {
+  int tx, ty, bxi, byi, BX, BY, gx, gy;
+};
+__device__ __forceinline__ CPGeo cp_geo_here() {
+  return CPGeo{(int)threadIdx.x, (int)threadIdx.y, (int)blockIdx.x, (int)blockIdx.y, (int)blockDim.x, (int)blockDim.y,
+               (int)gridDim.x, (int)gridDim.y};
+}
+__device__ __forceinline__ CPGeo cp_geo_of(int64_t t, int BX, int BY, int gx, int gy) {
+  const int64_t per = (int64_t)BX * BY, blk = t / per, r = t % per;
+  return CPGeo{(int)(r % BX), (int)(r / BX), (int)(blk % gx), (int)(blk / gx), BX, BY, gx, gy};
+}
+
+template <int KIND, int U, bool EXACT, class Sink>
+__device__ void cp_fi_program(const CPParams& p, const FaultRec& f, const CPGeo& G, bool mine, uint64_t grid_real,
+                              Sink& S) {
+  const int BX = G.BX, BY = G.BY;
+  const int tx = G.tx, ty = G.ty;
+  const int bxi = G.bxi, byi = G.byi;
+  const int64_t t = ((int64_t)byi * G.gx + bxi) * (BX * BY) + ty * BX + tx;
   const int64_t inst = mine ? f.inst : -1;
   const uint64_t mask = f.mask;
   const int site = f.site, sub = f.sub;
   const uint32_t z = p.z;
   const int64_t n_atoms = p.numatoms;
-  const int64_t n_grid = (int64_t)gridDim.x * BX * U * gridDim.y * BY;
-  const uint64_t grid_real = (uint64_t)(uintptr_t)grid, atoms_real = (uint64_t)(uintptr_t)p.atoms;
+  const int64_t n_grid = (int64_t)G.gx * BX * U * G.gy * BY;
+  const uint64_t atoms_real = (uint64_t)(uintptr_t)p.atoms;
   uint32_t chk = 0, alarm = 0, fail = 0, margin = 0xffffffffu;
   bool applied = false;
 
@@ -200,7 +214,7 @@ __device__ void cp_fi_thread(const CPParams& p, const FaultRec& f, float* grid, 
   int32_t yindex = byi * BY + ty;
   NLF(yindex, 1);
   chk ^= (uint32_t)yindex; alarm |= ((int32_t)((byi ^ z) * BY + (ty ^ z)) != yindex) ? AL_DUP : 0u;
-  const int32_t nx = gridDim.x * BX * U;
+  const int32_t nx = G.gx * BX * U;
   int32_t outaddr = (int32_t)((uint32_t)nx * (uint32_t)yindex + (uint32_t)xindex);
   NLF(outaddr, 2);
   chk ^= (uint32_t)outaddr;
@@ -283,7 +297,7 @@ __device__ void cp_fi_thread(const CPParams& p, const FaultRec& f, float* grid, 
     for (int d = 0; d < U; ++d) {
       if (d < p.ndet && p.R.n[d] > 0) {
         const float v = __fdiv_rn(E[U - 1 - d], fit);
-        if (!in_range<true>(p.R, d, v, &margin)) { alarm |= AL_RANGE; record_outlier(cb, d, v); }
+        if (!in_range<true>(p.R, d, v, &margin)) { alarm |= AL_RANGE; S.outlier(d, v); }
       }
     }
   }
@@ -292,18 +306,13 @@ __device__ void cp_fi_thread(const CPParams& p, const FaultRec& f, float* grid, 
   for (int j = 0; j < U; ++j) {
     int64_t e;
     if (!guard(pgrid, grid_real, outaddr + j * BX, 4, n_grid, &e)) { fail |= FL_CRASH; goto done; }
-    atomicAdd(grid + e, E[j]);
+    S.store(0, e, E[j]);
   }
   chk ^= (uint32_t)opq(outaddr, z);
   chk ^= ((uint32_t)numatoms + z) ^ (fb(h) + z) ^ (lohi(pgrid) + z) ^ (lohi(patoms) + z);
   if (chk != 0) alarm |= AL_CHK;
 done:
-  if (fail) atomicOr(&cb->fail, fail);
-  if (mine) {
-    cb->fault_applied = applied ? 1u : 0u;
-    cb->check_margin = margin;
-  }
-  fold_alarm(cb, alarm, (uint32_t)t);
+  S.finish(mine, alarm, fail, margin, 0u, applied, (uint32_t)t);
 }
 
 template <int KIND, int U, bool EXACT>
@@ -320,8 +329,68 @@ __global__ void __launch_bounds__(256) cp_fi_kernel(const CPFIParams q) {
   if (f.thread / tpb != cta) {
     cp_body<V_NL | V_L, U, EXACT, true>(p, tile, bar);
   } else {
-    cp_fi_thread<KIND, U, EXACT>(p, f, p.grid, p.cb);
+    const CPGeo G = cp_geo_here();
+    const int64_t t = ((int64_t)G.byi * G.gx + G.bxi) * (G.BX * G.BY) + G.ty * G.BX + G.tx;
+    ReplicaSinkF S{{p.grid, nullptr}, p.cb};
+    cp_fi_program<KIND, U, EXACT>(p, f, G, t == f.thread, (uint64_t)(uintptr_t)p.grid, S);
   }
+}
+
+// ============================================================================================
+// Replay accelerator (DESIGN R22): one CUDA thread per injection re-runs only the
+// faulted abstract thread and classifies against the golden output patched with its writes
+// (the thread's own elements lose the golden contribution, R18) — identical to the replica
+// outcome because no other thread is affected by the fault.
+// ============================================================================================
+struct CPReplayParams {
+  CPParams base;
+  const FaultRec* faults;
+  int nrep, BX, BY, gx, gy, bench;
+  const float* golden;
+  const float* dM;
+  hk_outcome* records;
+  int64_t first;
+  int64_t* counts;
+  int64_t* site_counts;
+};
+
+template <int KIND, bool EXACT>
+__global__ void __launch_bounds__(128) cp_replay_kernel(const CPReplayParams q) {
+  const int r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= q.nrep) return;
+  constexpr int U = 4;
+  const FaultRec f = q.faults[r];
+  const CPGeo G = cp_geo_of(f.thread, q.BX, q.BY, q.gx, q.gy);
+  ReplaySinkF<U> S;
+  cp_fi_program<KIND, U, EXACT>(q.base, f, G, true, (uint64_t)(uintptr_t)q.golden, S);
+  bool wrong = false;
+  float worst = 0.f;
+  if (!S.fail) {
+    const float M = *q.dM;
+    const int32_t nx = q.gx * q.BX * U;
+    const int64_t own0 = (int64_t)nx * (G.byi * q.BY + G.ty) + G.bxi * (q.BX * U) + G.tx;
+    // own elements: golden contribution removed, then the faulted writes added (in program order)
+#pragma unroll
+    for (int j = 0; j < U; ++j) {
+      const int64_t e = own0 + (int64_t)j * q.BX;
+      float v = 0.f;
+      for (int w = 0; w < S.n; ++w) if (S.idx[w] == e) v = __fadd_rn(v, S.val[w]);
+      fp_judge(v, q.golden[e], M, &wrong, &worst);
+    }
+    // stray writes into elements owned by other threads
+    for (int w = 0; w < S.n; ++w) {
+      const int64_t e = S.idx[w];
+      const int64_t d = e - own0;
+      if (d >= 0 && d % q.BX == 0 && d / q.BX < U) continue;  // own element (handled above)
+      bool first_write = true;
+      for (int w2 = 0; w2 < w; ++w2) first_write &= (S.idx[w2] != e);
+      if (!first_write) continue;
+      float v = q.golden[e];
+      for (int w2 = w; w2 < S.n; ++w2) if (S.idx[w2] == e) v = __fadd_rn(v, S.val[w2]);
+      fp_judge(v, q.golden[e], M, &wrong, &worst);
+    }
+  }
+  emit_outcome(q.bench, f, wrong, S.alarm, S.fail, S.domain, S.margin, worst, q.records, q.first, q.counts, q.site_counts);
 }
 
 // ============================================================================================
@@ -428,6 +497,45 @@ cudaError_t cp_fi_launch(int kind, const hk_cp_args& a, const DevRanges& R, int 
   q.cb0 = cb0;
   dim3 block(a.bx, a.by), grid(a.nx / (a.bx * 4), a.ny / a.by, nrep);
   return a.exact ? launch_cp_fi_e<true>(kind, q, grid, block, s) : launch_cp_fi_e<false>(kind, q, grid, block, s);
+}
+
+template <int KIND, bool EXACT>
+static cudaError_t launch_cp_replay_k(const CPReplayParams& q, cudaStream_t s) {
+  TimedScope ts(HK_CP, 2, (double)q.base.numatoms * 4 * q.nrep, s);
+  cp_replay_kernel<KIND, EXACT><<<(q.nrep + 127) / 128, 128, 0, s>>>(q);
+  count_launch();
+  return cudaGetLastError();
+}
+template <bool EXACT>
+static cudaError_t launch_cp_replay_e(int kind, const CPReplayParams& q, cudaStream_t s) {
+  switch (kind) {
+#define K(k) case k: return launch_cp_replay_k<k, EXACT>(q, s);
+    K(CK_NL) K(CK_LIVE) K(CK_ATOMID) K(CK_AX) K(CK_AY) K(CK_AZ) K(CK_AW) K(CK_DY) K(CK_DYZ2) K(CK_DX0)
+    K(CK_DXJ) K(CK_R2) K(CK_S) K(CK_E) K(CK_IT)
+#undef K
+  }
+  return cudaErrorInvalidValue;
+}
+
+cudaError_t cp_replay_launch(int kind, const hk_cp_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
+                             const float* golden, const float* dM, hk_outcome* records, int64_t first, int64_t* counts,
+                             int64_t* site_counts, cudaStream_t s) {
+  if (nrep <= 0) return cudaSuccess;
+  CPReplayParams q{};
+  q.base.atoms = reinterpret_cast<const float4*>(a.atoms_ws);
+  q.base.R = R;
+  q.base.numatoms = a.n_atoms;
+  q.base.h = a.h;
+  q.base.ndet = ndet;
+  q.base.z = opaque_zero();
+  q.base.one = 1 + (int32_t)opaque_zero();
+  q.base.nthreads = (int64_t)(a.nx / a.unroll) * a.ny;
+  q.faults = faults;
+  q.nrep = nrep;
+  q.BX = a.bx; q.BY = a.by; q.gx = a.nx / (a.bx * 4); q.gy = a.ny / a.by;
+  q.bench = HK_CP;
+  q.golden = golden; q.dM = dM; q.records = records; q.first = first; q.counts = counts; q.site_counts = site_counts;
+  return a.exact ? launch_cp_replay_e<true>(kind, q, s) : launch_cp_replay_e<false>(kind, q, s);
 }
 
 cudaError_t cp_prepass_launch(const hk_cp_args& a, cudaStream_t s) {

@@ -219,6 +219,66 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
       : "memory");
 }
 
+// Where a per-thread FI program's effects go.  Replica: atomic adds into the replica's grid and
+// the warp-folded control block.  Replay: the (at most U) writes and the thread's verdict bits
+// stay in registers for the per-injection classification.
+struct ReplicaSinkF {
+  float* out[2];
+  hk_control* cb;
+  __device__ __forceinline__ void store(int buf, int64_t e, float v) { atomicAdd(out[buf] + e, v); }
+  __device__ __forceinline__ void outlier(int d, float v) { record_outlier(cb, d, v); }
+  __device__ __forceinline__ void finish(bool mine, uint32_t alarm, uint32_t fail, uint32_t margin, uint32_t domain,
+                                         bool applied, uint32_t tid) {
+    if (fail) atomicOr(&cb->fail, fail);
+    if (mine) {
+      cb->fault_applied = applied ? 1u : 0u;
+      cb->check_margin = margin;
+      cb->domain = domain;
+    }
+    fold_alarm(cb, alarm, tid);
+  }
+};
+template <int MAXW>
+struct ReplaySinkF {
+  int n = 0;
+  int buf[MAXW];
+  int64_t idx[MAXW];
+  float val[MAXW];
+  uint32_t alarm = 0, fail = 0, margin = 0xffffffffu, domain = 0;
+  __device__ __forceinline__ void store(int b, int64_t e, float v) {
+    if (n < MAXW) { buf[n] = b; idx[n] = e; val[n] = v; ++n; }
+  }
+  __device__ __forceinline__ void outlier(int, float) {}
+  __device__ __forceinline__ void finish(bool, uint32_t a, uint32_t f, uint32_t m, uint32_t d, bool, uint32_t) {
+    alarm = a; fail = f; margin = m; domain = d;
+  }
+};
+
+// Output-correctness rule shared by the classify epilogue and the replay kernels (R5/R6).
+__device__ __forceinline__ void fp_judge(float v, float g, float M, bool* wrong, float* worst) {
+  const float err = fabsf(__fsub_rn(v, g));
+  const float tol = fmaxf(__fmul_rn(1e-4f, M), __fmul_rn(0.002f, fabsf(g)));
+  *wrong |= !(err <= tol);
+  float q = __fdiv_rn(err, tol);
+  if (q != q) q = __int_as_float(0x7f800000);
+  *worst = fmaxf(*worst, q);
+}
+
+__device__ __forceinline__ void emit_outcome(int bench, const FaultRec& f, bool wrong, uint32_t alarm, uint32_t fail,
+                                             uint32_t domain, uint32_t margin, float worst, hk_outcome* records,
+                                             int64_t first, int64_t* counts, int64_t* site_counts) {
+  const int32_t cls = fail ? HK_FAILURE : (!wrong ? (alarm ? HK_DETECTED_MASKED : HK_MASKED) : (alarm ? HK_DETECTED : HK_UNDETECTED));
+  if (records) {
+    hk_outcome o;
+    o.index = f.index; o.bench = bench; o.site = f.site; o.thread = f.thread; o.inst = f.inst; o.mask = f.mask;
+    o.cls = cls; o.alarm = alarm; o.fail = fail; o.domain = domain; o.margin = margin; o.worst = worst;
+    records[f.index - first] = o;
+  }
+  atomicAdd(reinterpret_cast<unsigned long long*>(counts + bench * 5 + cls), 1ull);
+  if (site_counts && f.site < 64)
+    atomicAdd(reinterpret_cast<unsigned long long*>(site_counts + ((int64_t)bench * 64 + f.site) * 5 + cls), 1ull);
+}
+
 // Initial value of a control block (reset by hk_control_init / the classify epilogue).
 __device__ __forceinline__ void control_reset(hk_control* cb, int lane) {
   // lane < 24 writes one 32-bit word each

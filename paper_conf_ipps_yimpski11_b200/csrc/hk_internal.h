@@ -47,6 +47,17 @@ cudaError_t mriq_fi_launch(int kind, const hk_mriq_args& a, const DevRanges& R, 
 cudaError_t tpacf_fi_launch(int kind, const hk_tpacf_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
                             int nrep, unsigned long long* hist0, hk_control* cb0, void* lut_ws, cudaStream_t s);
 
+// replay accelerator (one CUDA thread per injection; classification fused)
+cudaError_t cp_replay_launch(int kind, const hk_cp_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
+                             const float* golden, const float* dM, hk_outcome* records, int64_t first, int64_t* counts,
+                             int64_t* site_counts, cudaStream_t s);
+cudaError_t mriq_replay_launch(int kind, const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
+                               int nrep, const float* golden, const float* dM, hk_outcome* records, int64_t first,
+                               int64_t* counts, int64_t* site_counts, cudaStream_t s);
+cudaError_t tpacf_replay_launch(int kind, const hk_tpacf_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
+                                int nrep, const unsigned long long* golden, hk_outcome* records, int64_t first,
+                                int64_t* counts, int64_t* site_counts, cudaStream_t s);
+
 // classify.cu
 cudaError_t control_init_launch(hk_control* cb, int n, cudaStream_t s);
 cudaError_t max_abs_launch(const float* g, int64_t n, float* d_out, cudaStream_t s);

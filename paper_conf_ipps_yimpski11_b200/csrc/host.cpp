@@ -566,7 +566,7 @@ static void keep_pool_memory() {
 static hk_status session_create(int32_t bench_mode, const void* const args[3], const hk_ranges* const ranges[3],
                                 const hk_campaign* C, cudaStream_t s, hk_campaign_session** out) {
   if (!args || !ranges || !C || !out || bench_mode < -1 || bench_mode > 2) return invalid("campaign: bad arguments");
-  if (C->mode != 0) { g_err = "only replica mode (0) is implemented on the GPU"; return HK_ERR_UNSUPPORTED; }
+  if (C->mode != 0 && C->mode != 1) return invalid("campaign: mode must be 0 (replica) or 1 (replay)");
   if (C->nbits < 0 || C->nbits > 64) return invalid("campaign: nbits out of range");
   keep_pool_memory();
   hk_campaign_session* S = new hk_campaign_session();
@@ -594,7 +594,8 @@ static hk_status session_create(int32_t bench_mode, const void* const args[3], c
     w.args = own;
     w.R = dev_ranges(ranges[b]);
     w.ndet = ranges[b]->n_det;
-    w.batch = C->batch > 0 ? C->batch : default_batch(b, own);
+    w.batch = C->mode == 1 ? 1 : (C->batch > 0 ? C->batch : default_batch(b, own));
+    if (C->mode == 1 && b == HK_TPACF && 3 * S->tp.n_bins > 96) { g_err = "replay supports n_bins <= 32"; st = HK_ERR_UNSUPPORTED; break; }
     size_t esz = sizeof(float);
     if (b == HK_CP) w.out_elems = (int64_t)S->cp.nx * S->cp.ny;
     else if (b == HK_MRIQ) w.out_elems = 2LL * S->mq.n_vox;
@@ -701,6 +702,28 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
   if ((e = cudaMemcpyAsync(S->d_faults, S->h_faults, sizeof(FaultRec) * items.size(), cudaMemcpyHostToDevice, s)) != cudaSuccess)
     return cuda_fail(e, "upload faults");
   cudaEventRecord(S->uploaded, s);
+
+  // ---- replay mode: one launch per (benchmark, kind) group, one CUDA thread per injection
+  if (S->cfg.mode == 1) {
+    size_t q = 0;
+    while (q < items.size()) {
+      const int b = items[q].b, kind = items[q].kind;
+      size_t end = q;
+      while (end < items.size() && items[end].b == b && items[end].kind == kind) ++end;
+      const int nrep = (int)(end - q);
+      BenchWS& w = S->W[b];
+      const FaultRec* fr = S->d_faults + q;
+      if (b == HK_CP) e = cp_replay_launch(kind, S->cp, w.R, std::min(w.ndet, 4), fr, nrep, (const float*)w.golden, w.dM,
+                                           d_records, first, d_counts, d_site_counts, s);
+      else if (b == HK_MRIQ) e = mriq_replay_launch(kind, S->mq, w.R, std::min(w.ndet, 2), fr, nrep, (const float*)w.golden,
+                                                    w.dM, d_records, first, d_counts, d_site_counts, s);
+      else e = tpacf_replay_launch(kind, S->tp, w.R, std::min(w.ndet, 1), fr, nrep, (const unsigned long long*)w.golden,
+                                   d_records, first, d_counts, d_site_counts, s);
+      if (e != cudaSuccess) return cuda_fail(e, "replay");
+      q = end;
+    }
+    return HK_OK;
+  }
 
   // ---- batches: FI&FT replicas, then the classify epilogue (which also recycles the workspace)
   size_t q = 0;

@@ -191,19 +191,18 @@ struct MQFIParams {
   hk_control* cb0;
 };
 
-template <int KIND, bool EXACT>
-__device__ void mriq_fi_thread(const MQParams& p, const FaultRec& f, int vox) {
-  const int32_t t = blockIdx.x * (2 * blockDim.x) + vox * blockDim.x + threadIdx.x;
-  if (t >= p.numX) return;
-  const bool mine = (t == f.thread);
+// Per-thread FI&FT program of voxel t.  t_dup: the duplicate of N0 recomputed from launch indices
+// (replica) or from the abstract id (replay); qr_real / qi_real: the buffers' true base addresses.
+template <int KIND, bool EXACT, class Sink>
+__device__ void mriq_fi_program(const MQParams& p, const FaultRec& f, int32_t t, int32_t t_dup, bool mine,
+                                uint64_t qr_real, uint64_t qi_real, Sink& S) {
   const int64_t inst = mine ? f.inst : -1;
   const uint64_t mask = f.mask;
   const int site = f.site;
   const uint32_t z = p.zz;
   const int64_t nv = p.numX, nk = p.numK;
-  const uint64_t kv_real = (uint64_t)(uintptr_t)p.kv, qr_real = (uint64_t)(uintptr_t)p.qr, qi_real = (uint64_t)(uintptr_t)p.qi;
+  const uint64_t kv_real = (uint64_t)(uintptr_t)p.kv;
   const uint64_t x_real = (uint64_t)(uintptr_t)p.x, y_real = (uint64_t)(uintptr_t)p.y, z_real = (uint64_t)(uintptr_t)p.z;
-  hk_control* cb = p.cb;
   uint32_t chk = 0, alarm = 0, fail = 0, margin = 0xffffffffu, domain = 0;
   bool applied = false;
   int32_t numK = p.numK;
@@ -213,7 +212,7 @@ __device__ void mriq_fi_thread(const MQParams& p, const FaultRec& f, int vox) {
   int32_t xIndex = t;
   { const bool n = nl && site == 0; applied |= n; xIndex = flip_i(xIndex, n, mask); }
   chk ^= (uint32_t)xIndex;
-  alarm |= ((int32_t)((blockIdx.x ^ z) * (2 * blockDim.x) + vox * blockDim.x + (threadIdx.x ^ z)) != xIndex) ? AL_DUP : 0u;
+  alarm |= (t_dup != xIndex) ? AL_DUP : 0u;
   float sX, sY, sZ, Qr = 0.f, Qi = 0.f;
   int32_t it = 0, k = 0;
   int64_t e;
@@ -291,27 +290,21 @@ __device__ void mriq_fi_thread(const MQParams& p, const FaultRec& f, int vox) {
     for (int d = 0; d < 2; ++d) {
       if (d < p.ndet && p.R.n[d] > 0) {
         const float v = __fdiv_rn(d == 0 ? Qr : Qi, fit);
-        if (!in_range<true>(p.R, d, v, &margin)) { alarm |= AL_RANGE; record_outlier(cb, d, v); }
+        if (!in_range<true>(p.R, d, v, &margin)) { alarm |= AL_RANGE; S.outlier(d, v); }
       }
     }
   }
   chk ^= opqf(sX, z); chk ^= opqf(sY, z); chk ^= opqf(sZ, z);
   if (!guard(pqr, qr_real, xIndex, 4, nv, &e)) { fail |= FL_CRASH; goto done; }
-  atomicAdd(p.qr + e, Qr);
+  S.store(0, e, Qr);
   if (!guard(pqi, qi_real, xIndex, 4, nv, &e)) { fail |= FL_CRASH; goto done; }
-  atomicAdd(p.qi + e, Qi);
+  S.store(1, e, Qi);
   chk ^= (uint32_t)opq(xIndex, z);
   chk ^= ((uint32_t)numK + z) ^ (lohi(pkv) + z) ^ (lohi(pqr) + z) ^ (lohi(pqi) + z) ^ (lohi(px) + z) ^ (lohi(py) + z) ^
          (lohi(pz) + z);
   if (chk != 0) alarm |= AL_CHK;
 done:
-  if (fail) atomicOr(&cb->fail, fail);
-  if (mine) {
-    cb->fault_applied = applied ? 1u : 0u;
-    cb->check_margin = margin;
-    cb->domain = domain;
-  }
-  fold_alarm(cb, alarm, (uint32_t)t);
+  S.finish(mine, alarm, fail, margin, domain, applied, (uint32_t)t);
 }
 
 template <int KIND, bool EXACT>
@@ -327,9 +320,65 @@ __global__ void __launch_bounds__(256) mriq_fi_kernel(const MQFIParams q) {
   if (f.thread / (2 * blockDim.x) != blockIdx.x) {
     mriq_body<V_NL | V_L, EXACT, true, 2>(p, tile, bar);
   } else {
-    mriq_fi_thread<KIND, EXACT>(p, f, 0);
-    mriq_fi_thread<KIND, EXACT>(p, f, 1);
+    ReplicaSinkF S{{p.qr, p.qi}, p.cb};
+#pragma unroll 1
+    for (int vox = 0; vox < 2; ++vox) {
+      const int32_t t = blockIdx.x * (2 * blockDim.x) + vox * blockDim.x + threadIdx.x;
+      if (t < p.numX) {
+        const int32_t t_dup = (int32_t)((blockIdx.x ^ p.zz) * (2 * blockDim.x) + vox * blockDim.x + (threadIdx.x ^ p.zz));
+        mriq_fi_program<KIND, EXACT>(p, f, t, t_dup, t == f.thread, (uint64_t)(uintptr_t)p.qr, (uint64_t)(uintptr_t)p.qi, S);
+      }
+    }
   }
+}
+
+// ============================================================================================
+// Replay accelerator: one CUDA thread per injection re-runs only the faulted voxel (DESIGN R22).
+// ============================================================================================
+struct MQReplayParams {
+  MQParams base;
+  const FaultRec* faults;
+  int nrep;
+  const float* golden;  // [qr; qi]
+  const float* dM;
+  hk_outcome* records;
+  int64_t first;
+  int64_t* counts;
+  int64_t* site_counts;
+};
+
+template <int KIND, bool EXACT>
+__global__ void __launch_bounds__(128) mriq_replay_kernel(const MQReplayParams q) {
+  const int r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= q.nrep) return;
+  const FaultRec f = q.faults[r];
+  const MQParams& p = q.base;
+  const int32_t t = (int32_t)f.thread;
+  ReplaySinkF<2> S;
+  const uint64_t base_real = (uint64_t)(uintptr_t)q.golden;
+  mriq_fi_program<KIND, EXACT>(p, f, t, opq(t, p.zz), true, base_real, base_real + 4ull * (uint64_t)p.numX, S);
+  bool wrong = false;
+  float worst = 0.f;
+  if (!S.fail) {
+    const float M = *q.dM;
+#pragma unroll
+    for (int b = 0; b < 2; ++b) {  // own elements qr[t], qi[t]
+      float v = 0.f;
+      for (int w = 0; w < S.n; ++w) if (S.buf[w] == b && S.idx[w] == t) v = __fadd_rn(v, S.val[w]);
+      fp_judge(v, q.golden[(int64_t)b * p.numX + t], M, &wrong, &worst);
+    }
+    for (int w = 0; w < S.n; ++w) {  // stray writes
+      if (S.idx[w] == t) continue;
+      bool first_write = true;
+      for (int w2 = 0; w2 < w; ++w2) first_write &= !(S.idx[w2] == S.idx[w] && S.buf[w2] == S.buf[w]);
+      if (!first_write) continue;
+      const int64_t ge = (int64_t)S.buf[w] * p.numX + S.idx[w];
+      float v = q.golden[ge];
+      for (int w2 = w; w2 < S.n; ++w2) if (S.idx[w2] == S.idx[w] && S.buf[w2] == S.buf[w]) v = __fadd_rn(v, S.val[w2]);
+      fp_judge(v, q.golden[ge], M, &wrong, &worst);
+    }
+  }
+  emit_outcome(HK_MRIQ, f, wrong, S.alarm, S.fail, S.domain, S.margin, worst, q.records, q.first, q.counts, q.site_counts);
 }
 
 // ============================================================================================
@@ -407,6 +456,36 @@ static cudaError_t launch_mq_fi_e(int kind, const MQFIParams& q, int nrep, cudaS
 #undef K
   }
   return cudaErrorInvalidValue;
+}
+
+template <int KIND, bool EXACT>
+static cudaError_t launch_mq_replay_k(const MQReplayParams& q, cudaStream_t s) {
+  TimedScope ts(HK_MRIQ, 2, (double)q.base.numK * q.nrep, s);
+  mriq_replay_kernel<KIND, EXACT><<<(q.nrep + 127) / 128, 128, 0, s>>>(q);
+  count_launch();
+  return cudaGetLastError();
+}
+template <bool EXACT>
+static cudaError_t launch_mq_replay_e(int kind, const MQReplayParams& q, cudaStream_t s) {
+  switch (kind) {
+#define K(k) case k: return launch_mq_replay_k<k, EXACT>(q, s);
+    K(MK_NL) K(MK_LIVE) K(MK_K) K(MK_KX) K(MK_KY) K(MK_KZ) K(MK_PM) K(MK_T1) K(MK_T2) K(MK_T) K(MK_R) K(MK_C) K(MK_S)
+    K(MK_QR) K(MK_QI) K(MK_IT)
+#undef K
+  }
+  return cudaErrorInvalidValue;
+}
+
+cudaError_t mriq_replay_launch(int kind, const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
+                               int nrep, const float* golden, const float* dM, hk_outcome* records, int64_t first,
+                               int64_t* counts, int64_t* site_counts, cudaStream_t s) {
+  if (nrep <= 0) return cudaSuccess;
+  MQReplayParams q{};
+  q.base = mq_params(a, R, ndet, nullptr, nullptr);
+  q.faults = faults;
+  q.nrep = nrep;
+  q.golden = golden; q.dM = dM; q.records = records; q.first = first; q.counts = counts; q.site_counts = site_counts;
+  return a.exact ? launch_mq_replay_e<true>(kind, q, s) : launch_mq_replay_e<false>(kind, q, s);
 }
 
 cudaError_t mriq_fi_launch(int kind, const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,

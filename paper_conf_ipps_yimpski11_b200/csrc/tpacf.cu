@@ -343,21 +343,63 @@ struct TPFIParams {
   int64_t hist_elems;
 };
 
-template <int KIND>
-__device__ void tpacf_fi_thread(const TPParams& p, const TPSmem& S, const FaultRec& f, unsigned long long* hist,
-                                hk_control* cb, int kpt) {
+// Histogram sinks of the per-thread TPACF FI program.  Replica: the faulted thread adds to the
+// replica's global histogram through its (possibly corrupted) index, the CTA's fault-free threads
+// use their lane-private shared counters.  Replay: every increment of the one thread is folded
+// into deltas of the 3*nb outputs (DD, DRS, RRS of R4) with a sign (+1 faulted run, -1 golden twin).
+struct TPReplicaSink {
+  unsigned long long* hist;
+  hk_control* cb;
+  uint32_t* H;  // lane-private counters of this CTA's row
+  int nb2;
+  __device__ __forceinline__ bool global_path(bool mine) const { return mine; }
+  __device__ __forceinline__ void hist_global(int64_t e) { atomicAdd(hist + e, 1ull); }
+  __device__ __forceinline__ void hist_local(uint32_t warp, int32_t bin, uint32_t lane) {
+    H[((size_t)warp * nb2 + bin) * 32 + lane] += 1u;
+  }
+  __device__ __forceinline__ void outlier(int d, float v) { record_outlier(cb, d, v); }
+  __device__ __forceinline__ void finish(bool mine, uint32_t alarm, uint32_t fail, uint32_t margin, bool applied,
+                                         uint32_t tid) {
+    if (fail) atomicOr(&cb->fail, fail);
+    if (mine) {
+      cb->fault_applied = applied ? 1u : 0u;
+      cb->check_margin = margin;
+    }
+    fold_alarm(cb, alarm, tid);
+  }
+};
+constexpr int TP_REPLAY_OUT = 96;  // 3 * n_bins (n_bins <= 30 for the replay kernel) + slack
+struct TPReplaySink {
+  int nr, nb, nb2, sign;
+  int32_t* delta;  // [3 * nb]: DD, DRS, RRS for bins 1..nb
+  uint32_t alarm = 0, fail = 0, margin = 0xffffffffu;
+  __device__ __forceinline__ bool global_path(bool) const { return true; }
+  __device__ __forceinline__ void hist_global(int64_t e) {
+    const int row = (int)(e / nb2), b = (int)(e % nb2);
+    if (b < 1 || b > nb) return;  // under/overflow bins are not outputs (R4)
+    const int kind = row == 0 ? 0 : (row <= nr ? 2 : 1);
+    delta[kind * nb + b - 1] += sign;
+  }
+  __device__ __forceinline__ void hist_local(uint32_t, int32_t, uint32_t) {}
+  __device__ __forceinline__ void outlier(int, float) {}
+  __device__ __forceinline__ void finish(bool, uint32_t a, uint32_t f, uint32_t m, bool, uint32_t) {
+    alarm = a; fail = f; margin = m;
+  }
+};
+
+// Per-thread FI&FT program of abstract thread g = row*N + ii.  i_dup: N0's duplicate from launch
+// indices (replica) or from the abstract id (replay); hist_real: the histogram's true base.
+template <int KIND, class Sink>
+__device__ void tpacf_fi_program(const TPParams& p, const TPSmem& S, const FaultRec& f, int32_t row, int32_t ii,
+                                 int32_t i_dup, int32_t row_dup, bool mine, uint64_t hist_real, Sink& K) {
   const uint32_t z = p.z;
   const int32_t nr = p.nr, C = p.C, nC = p.nC, nb2 = p.nb + 2;
-  const int32_t row = blockIdx.y;
-  const int32_t ii = blockIdx.x * TP_CTA_PTS + kpt * TP_THREADS + threadIdx.x;
-  if (ii >= p.n) return;
   const int64_t g = (int64_t)row * p.n + ii;
-  const bool mine = (g == f.thread);
   const int64_t inst = mine ? f.inst : -1;
   const uint64_t mask = f.mask;
   const int site = f.site;
   const int64_t npts = 3LL * (1 + nr) * p.n, nhist = (int64_t)(1 + 2 * nr) * nb2;
-  const uint64_t pts_real = (uint64_t)(uintptr_t)p.pts, hist_real = (uint64_t)(uintptr_t)hist;
+  const uint64_t pts_real = (uint64_t)(uintptr_t)p.pts;
   const uint32_t lane = lane_id(), warp = threadIdx.x >> 5;
   uint32_t chk = 0, alarm = 0, fail = 0, margin = 0xffffffffu;
   bool applied = false;
@@ -368,9 +410,9 @@ __device__ void tpacf_fi_thread(const TPParams& p, const TPSmem& S, const FaultR
 #define NLF(v, s) do { const bool _n = nl && site == (s); applied |= _n; v = flip_i(v, _n, mask); } while (0)
   int32_t i = ii; NLF(i, 0);
   chk ^= (uint32_t)i;
-  alarm |= ((int32_t)((blockIdx.x ^ z) * TP_CTA_PTS + kpt * TP_THREADS + (threadIdx.x ^ z)) != i) ? AL_DUP : 0u;
+  alarm |= (i_dup != i) ? AL_DUP : 0u;
   int32_t h = row / nC; NLF(h, 1);
-  chk ^= (uint32_t)h; alarm |= ((int32_t)(blockIdx.y ^ z) / nC != h) ? AL_DUP : 0u;
+  chk ^= (uint32_t)h; alarm |= (row_dup / nC != h) ? AL_DUP : 0u;
   int32_t c = (int32_t)((uint32_t)row - (uint32_t)h * (uint32_t)nC); NLF(c, 2);
   chk ^= (uint32_t)c; alarm |= ((int32_t)((uint32_t)row - (uint32_t)opq(h, z) * (uint32_t)nC) != c) ? AL_DUP : 0u;
   auto f_aoff = [&](int32_t hh, int32_t i_) { return (int32_t)((uint32_t)(hh <= nr ? hh : 0) * (uint32_t)n + (uint32_t)i_); };
@@ -449,11 +491,11 @@ __device__ void tpacf_fi_thread(const TPParams& p, const TPSmem& S, const FaultR
       if (KIND == TK_BIN) { applied |= now; bin = flip_i(bin, now, mask); }
       int32_t hidx = (int32_t)((uint32_t)base + (uint32_t)bin);
       if (KIND == TK_HIDX) { applied |= now; hidx = flip_i(hidx, now, mask); }
-      if (mine) {
+      if (K.global_path(mine)) {
         if (!guard(phist, hist_real, hidx, 8, nhist, &e)) { fail |= FL_CRASH; goto done; }
-        atomicAdd(hist + e, 1ull);
+        K.hist_global(e);
       } else {
-        S.H[((size_t)warp * nb2 + bin) * 32 + lane] += 1u;  // fault-free thread: hidx == base + bin (this CTA's row)
+        K.hist_local(warp, bin, lane);  // fault-free thread: hidx == base + bin (this CTA's row)
       }
       acc = (int32_t)((uint32_t)acc + (uint32_t)bin);
       if (KIND == TK_ACC) { applied |= now; acc = flip_i(acc, now, mask); }
@@ -465,19 +507,14 @@ __device__ void tpacf_fi_thread(const TPParams& p, const TPSmem& S, const FaultR
   if (cnt != expect) alarm |= AL_COUNT;
   if (cnt != 0 && p.ndet > 0 && p.R.n[0] > 0) {
     const float v = __fdiv_rn((float)acc, (float)cnt);
-    if (!in_range<true>(p.R, 0, v, &margin)) { alarm |= AL_RANGE; record_outlier(cb, 0, v); }
+    if (!in_range<true>(p.R, 0, v, &margin)) { alarm |= AL_RANGE; K.outlier(0, v); }
   }
   chk ^= (uint32_t)opq(boff, z) ^ (uint32_t)opq(je, z) ^ (uint32_t)opq(base, z);
   chk ^= opqf(q1[0], z) ^ opqf(q1[1], z) ^ opqf(q1[2], z) ^ (uint32_t)opq(expect, z);
   chk ^= ((uint32_t)n + z) ^ (lohi(ppts) + z) ^ (lohi(phist) + z);
   if (chk != 0) alarm |= AL_CHK;
 done:
-  if (fail) atomicOr(&cb->fail, fail);
-  if (mine) {
-    cb->fault_applied = applied ? 1u : 0u;
-    cb->check_margin = margin;
-  }
-  fold_alarm(cb, alarm, (uint32_t)g);
+  K.finish(mine, alarm, fail, margin, applied, (uint32_t)g);
 }
 
 template <int KIND>
@@ -497,11 +534,76 @@ __global__ void __launch_bounds__(TP_THREADS) tpacf_fi_kernel(const TPFIParams q
     const int32_t sb = (h == 0) ? 0 : (h <= p.nr ? h : h - p.nr);
     tp_stage(p, S, sb, c, true);
     __syncthreads();
-    tpacf_fi_thread<KIND>(p, S, f, hist, cb, 0);
-    tpacf_fi_thread<KIND>(p, S, f, hist, cb, 1);
+    TPReplicaSink K{hist, cb, S.H, p.nb + 2};
+#pragma unroll 1
+    for (int kpt = 0; kpt < 2; ++kpt) {
+      const int32_t ii = blockIdx.x * TP_CTA_PTS + kpt * TP_THREADS + threadIdx.x;
+      if (ii < p.n) {
+        const int32_t idup = (int32_t)((blockIdx.x ^ p.z) * TP_CTA_PTS + kpt * TP_THREADS + (threadIdx.x ^ p.z));
+        const int64_t g = (int64_t)blockIdx.y * p.n + ii;
+        tpacf_fi_program<KIND>(p, S, f, (int32_t)blockIdx.y, ii, idup, (int32_t)(blockIdx.y ^ p.z), g == f.thread,
+                               (uint64_t)(uintptr_t)hist, K);
+      }
+    }
     __syncthreads();
     tp_flush(p, S, hist, h * (p.nb + 2));
   }
+}
+
+// ============================================================================================
+// Replay accelerator: one CUDA thread per injection runs the golden twin (-1) and the faulted
+// abstract thread (+1) into deltas of the 3*nb outputs, then applies the 1 % rule (R3/R4).
+// ============================================================================================
+struct TPReplayParams {
+  TPParams base;
+  const FaultRec* faults;
+  int nrep;
+  const unsigned long long* golden;
+  hk_outcome* records;
+  int64_t first;
+  int64_t* counts;
+  int64_t* site_counts;
+};
+
+template <int KIND>
+__global__ void __launch_bounds__(128) tpacf_replay_kernel(const TPReplayParams q) {
+  __shared__ float Es[32];
+  const TPParams& p = q.base;
+  if (threadIdx.x < 32) Es[threadIdx.x] = threadIdx.x <= p.nb ? p.edges[threadIdx.x] : __int_as_float(0xff800000);
+  __syncthreads();
+  const int r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= q.nrep) return;
+  TPSmem S{};
+  S.E = Es;
+  const FaultRec f = q.faults[r];
+  const int32_t row = (int32_t)(f.thread / p.n), ii = (int32_t)(f.thread % p.n);
+  int32_t delta[TP_REPLAY_OUT];
+  for (int o = 0; o < 3 * p.nb; ++o) delta[o] = 0;
+  const uint64_t hist_real = (uint64_t)(uintptr_t)q.golden;
+  TPReplaySink twin{p.nr, p.nb, p.nb + 2, -1, delta};
+  tpacf_fi_program<KIND>(p, S, f, row, ii, opq(ii, p.z), (int32_t)((uint32_t)row ^ p.z), false, hist_real, twin);
+  TPReplaySink K{p.nr, p.nb, p.nb + 2, +1, delta};
+  tpacf_fi_program<KIND>(p, S, f, row, ii, opq(ii, p.z), (int32_t)((uint32_t)row ^ p.z), true, hist_real, K);
+  bool wrong = false;
+  float worst = 0.f;
+  if (!K.fail) {
+    const int nb = p.nb, nb2 = p.nb + 2, nr = p.nr;
+    for (int o = 0; o < 3 * nb; ++o) {
+      if (delta[o] == 0) continue;
+      const int kind = o / nb, b = 1 + o % nb;
+      long long g = 0;
+      if (kind == 0) g = (long long)q.golden[b];
+      for (int s2 = 1; s2 <= nr; ++s2) {
+        const int rr = kind == 1 ? nr + s2 : s2;
+        if (kind != 0) g += (long long)q.golden[rr * nb2 + b];
+      }
+      const long long d = delta[o] < 0 ? -(long long)delta[o] : (long long)delta[o];
+      if (100 * d > g) wrong = true;
+      const float qv = g > 0 ? (float)(100.0 * (double)d / (double)g) : __int_as_float(0x7f800000);
+      worst = fmaxf(worst, qv);
+    }
+  }
+  emit_outcome(HK_TPACF, f, wrong, K.alarm, K.fail, 0u, K.margin, worst, q.records, q.first, q.counts, q.site_counts);
 }
 
 // ============================================================================================
@@ -589,6 +691,32 @@ static cudaError_t launch_tp_fi_k(const TPFIParams& q, int nrep, cudaStream_t s)
   tpacf_fi_kernel<KIND><<<grid, TP_THREADS, smem, s>>>(q);
   count_launch();
   return cudaGetLastError();
+}
+
+template <int KIND>
+static cudaError_t launch_tp_replay_k(const TPReplayParams& q, cudaStream_t s) {
+  TimedScope ts(HK_TPACF, 2, (double)q.base.C * 2 * q.nrep, s);
+  tpacf_replay_kernel<KIND><<<(q.nrep + 127) / 128, 128, 0, s>>>(q);
+  count_launch();
+  return cudaGetLastError();
+}
+
+cudaError_t tpacf_replay_launch(int kind, const hk_tpacf_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
+                                int nrep, const unsigned long long* golden, hk_outcome* records, int64_t first,
+                                int64_t* counts, int64_t* site_counts, cudaStream_t s) {
+  if (nrep <= 0) return cudaSuccess;
+  if (3 * a.n_bins > TP_REPLAY_OUT) return cudaErrorInvalidValue;
+  TPReplayParams q{};
+  q.base = tp_params(a, R, ndet, nullptr, nullptr, nullptr);
+  q.faults = faults;
+  q.nrep = nrep;
+  q.golden = golden; q.records = records; q.first = first; q.counts = counts; q.site_counts = site_counts;
+  switch (kind) {
+#define K(k) case k: return launch_tp_replay_k<k>(q, s);
+    K(TK_NL) K(TK_LIVE) K(TK_J) K(TK_X2) K(TK_Y2) K(TK_Z2) K(TK_DOT) K(TK_BIN) K(TK_HIDX) K(TK_ACC) K(TK_CNT)
+#undef K
+  }
+  return cudaErrorInvalidValue;
 }
 
 // lut_ws must hold a table built by tpacf_lut_build for a.edges (the campaign builds it once).

@@ -336,14 +336,14 @@ def _arg_array(devs):
 
 def inject_campaign(bench_mode: int, devs, ranges, seed: int, first: int, count: int, counts: torch.Tensor,
                     records: torch.Tensor | None = None, site_counts: torch.Tensor | None = None, exact: int = 0,
-                    batch: int = 0, site_masks=(ALL_SITES,) * 3, stream=None, nbits: int = 1):
+                    batch: int = 0, site_masks=(ALL_SITES,) * 3, stream=None, nbits: int = 1, mode: int = 0):
     """hauberk_inject_campaign (replica mode).  devs/ranges: 3-lists by bench (None where unused).
     counts: int64 cuda tensor [3, 5] (accumulated); records: optional uint8 tensor of
     count * OUTCOME_DTYPE.itemsize bytes; site_counts: optional int64 [3, 64, 5]."""
     arr, keep = _arg_array(devs)
     rng = [r if r is not None else Ranges() for r in ranges]
     rarr = (C.c_void_p * 3)(*[C.cast(C.byref(r), C.c_void_p) for r in rng])
-    camp = Campaign(seed, first, count, nbits, 0, batch, exact, (C.c_uint64 * 3)(*site_masks))
+    camp = Campaign(seed, first, count, nbits, mode, batch, exact, (C.c_uint64 * 3)(*site_masks))
     st = lib().hauberk_inject_campaign(bench_mode, arr, rarr, C.byref(camp), _ptr(records), _ptr(counts),
                                        _ptr(site_counts), _stream(stream))
     _check(st, "hauberk_inject_campaign")
@@ -354,12 +354,12 @@ class CampaignSession:
     asynchronous slices of the same seeded campaign.  Keep `devs` alive while the session lives."""
 
     def __init__(self, bench_mode: int, devs, ranges, seed: int, exact: int = 0, batch: int = 0,
-                 site_masks=(ALL_SITES,) * 3, stream=None, nbits: int = 1):
+                 site_masks=(ALL_SITES,) * 3, stream=None, nbits: int = 1, mode: int = 0):
         self._arr, self._keep = _arg_array(devs)
         self._devs = devs
         self._rng = [r if r is not None else Ranges() for r in ranges]
         self._rarr = (C.c_void_p * 3)(*[C.cast(C.byref(r), C.c_void_p) for r in self._rng])
-        self._camp = Campaign(seed, 0, 0, nbits, 0, batch, exact, (C.c_uint64 * 3)(*site_masks))
+        self._camp = Campaign(seed, 0, 0, nbits, mode, batch, exact, (C.c_uint64 * 3)(*site_masks))
         self._h = C.c_void_p()
         st = lib().hauberk_campaign_create(bench_mode, self._arr, self._rarr, C.byref(self._camp), C.byref(self._h),
                                            _stream(stream))

@@ -332,3 +332,54 @@ def test_campaign_multibit_exact_mode_bit_exact(k):
     assert np.array_equal(g["mask"], orec["mask"])
     assert np.array_equal(g["cls"], orec["cls"])
     assert np.array_equal(counts.cpu().numpy(), oc)
+
+
+# ---------------------------------------------------------------------------------------------- replay accelerator
+def _gpu_campaign(devs, ranges, seed, first, count, exact=0, mode=0, nbits=1):
+    counts = torch.zeros((3, 5), dtype=torch.int64, device=DEV)
+    rec = hk.records_tensor(count, DEV)
+    hk.inject_campaign(-1, devs, ranges, seed, first, count, counts, records=rec, exact=exact, mode=mode, nbits=nbits)
+    torch.cuda.synchronize()
+    return counts.cpu().numpy(), hk.records_numpy(rec)
+
+
+@pytest.mark.parametrize("exact", [0, 1])
+def test_gpu_replay_equals_gpu_replica(exact):
+    probs = [W.cp_small(), W.mriq_problem(6, 61, n_vox=200, seed=3), W.tpacf_small(n=150, n_rand=2, chunk=32)]
+    devs = [_mk(b, probs[b], exact) for b in range(3)]
+    R = [hk.profile_ranges(d) for d in devs]
+    c0, r0 = _gpu_campaign(devs, R, 0xBEEF, 0, 1500, exact=exact, mode=0)
+    c1, r1 = _gpu_campaign(devs, R, 0xBEEF, 0, 1500, exact=exact, mode=1)
+    for k in ("cls", "alarm", "fail", "site", "thread", "inst", "mask", "margin", "domain"):
+        assert np.array_equal(r0[k], r1[k]), k
+    assert np.array_equal(c0, c1)
+
+
+def test_gpu_replay_config_shapes_vs_oracle_replay():
+    """Config-5 shapes (cfg1 CP-s, cfg2 MRI-Q, cfg3 TPACF), 30,000 mixed injections, FAST mode:
+    outcomes exact outside the R22 guard band; TPACF exact everywhere."""
+    probs = [W.cp_config1(), W.mriq_config2(), W.tpacf_config3()]
+    devs = [_mk(b, probs[b]) for b in range(3)]
+    R = [hk.profile_ranges(d) for d in devs]
+    gc, g = _gpu_campaign(devs, R, W.CAMPAIGN_SEED_CFG5, 777000, 30000, mode=1)
+    orr = [O.profile_ranges(b, probs[b]) for b in range(3)]
+    oc, o = O.campaign(-1, probs, orr, W.CAMPAIGN_SEED_CFG5, 777000, 30000, mode=1)
+    for k in ("index", "bench", "site", "thread", "inst", "mask"):
+        assert np.array_equal(g[k], o[k]), k
+    amb = _ambiguous(g, o)
+    mism = (g["cls"] != o["cls"]) & ~amb
+    assert not mism.any(), [(g[i], o[i]) for i in np.nonzero(mism)[0][:5]]
+    tp = g["bench"] == 2
+    assert np.array_equal(g["cls"][tp], o["cls"][tp])
+    assert amb.mean() < 0.01
+
+
+def test_gpu_replay_exact_mode_bit_exact_config_shapes():
+    probs = [W.cp_config1(), W.mriq_problem(16, 512, seed=0x4D5249), W.tpacf_problem(1024, 2, chunk=256)]
+    devs = [_mk(b, probs[b], 1) for b in range(3)]
+    R = [hk.profile_ranges(d) for d in devs]
+    gc, g = _gpu_campaign(devs, R, 0x5151, 0, 6000, exact=1, mode=1, nbits=3)
+    orr = [O.profile_ranges(b, probs[b], exact=1) for b in range(3)]
+    oc, o = O.campaign(-1, probs, orr, 0x5151, 0, 6000, exact=1, mode=1, nbits=3)
+    assert np.array_equal(g["cls"], o["cls"]) and np.array_equal(g["alarm"], o["alarm"]) and np.array_equal(g["fail"], o["fail"])
+    assert np.array_equal(gc, oc)

@@ -81,7 +81,7 @@ typedef struct {
   uint32_t fault_applied;     /* FI only: the flip happened */
   uint32_t check_margin;      /* FI only: min ordinal distance of the faulted thread's checks to a bound */
   uint32_t domain;            /* FI only: faulted thread left the MUFU accuracy domain (R22c) */
-  uint32_t reserved;
+  float check_gap;            /* FI only: min |check value - bound| of the faulted thread (R22a) */
 } hk_control;
 
 /* CP (K1; Fig. 9).  atoms: [n_atoms] (x, y, z, q); atoms_ws: [n_atoms] float4 scratch
@@ -127,6 +127,7 @@ typedef struct { int32_t site; int32_t pad; int64_t thread, inst; uint64_t mask;
 typedef struct {
   int64_t index; int32_t bench, site; int64_t thread, inst; uint64_t mask;
   int32_t cls; uint32_t alarm, fail, domain, margin; float worst; /* worst err/tol (R22b) */
+  float gap; int32_t pad2;                                        /* check-value gap to a bound (R22a) */
 } hk_outcome;
 
 /* Run one benchmark kernel (plus its uninstrumented pre-pass / PhiMag) on `stream`.

@@ -57,18 +57,19 @@ class Fault(C.Structure):
 
 class RunInfo(C.Structure):
     _fields_ = [("alarm", C.c_uint32), ("fail", C.c_uint32), ("domain", C.c_uint32), ("margin", C.c_uint32),
-                ("n_alarm_threads", C.c_uint32), ("first_thread", C.c_uint32), ("applied", C.c_int32), ("pad", C.c_int32)]
+                ("n_alarm_threads", C.c_uint32), ("first_thread", C.c_uint32), ("applied", C.c_int32), ("gap", C.c_float)]
 
 
 class Record(C.Structure):
     _fields_ = [("index", C.c_int64), ("bench", C.c_int32), ("site", C.c_int32), ("thread", C.c_int64),
                 ("inst", C.c_int64), ("mask", C.c_uint64), ("cls", C.c_int32), ("alarm", C.c_uint32),
-                ("fail", C.c_uint32), ("domain", C.c_uint32), ("margin", C.c_uint32), ("worst", C.c_float)]
+                ("fail", C.c_uint32), ("domain", C.c_uint32), ("margin", C.c_uint32), ("worst", C.c_float),
+                ("gap", C.c_float), ("pad", C.c_int32)]
 
 
 RECORD_DTYPE = np.dtype([("index", "<i8"), ("bench", "<i4"), ("site", "<i4"), ("thread", "<i8"), ("inst", "<i8"),
                          ("mask", "<u8"), ("cls", "<i4"), ("alarm", "<u4"), ("fail", "<u4"), ("domain", "<u4"),
-                         ("margin", "<u4"), ("worst", "<f4")], align=True)
+                         ("margin", "<u4"), ("worst", "<f4"), ("gap", "<f4"), ("pad", "<i4")], align=True)
 assert RECORD_DTYPE.itemsize == C.sizeof(Record)
 
 

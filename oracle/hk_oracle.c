@@ -60,11 +60,11 @@ typedef struct { const float* pts; const float* edges; int32_t n, n_rand, n_bins
 typedef struct { int32_t site; int32_t pad; int64_t thread, inst; uint64_t mask; } ora_fault;
 typedef struct {
   uint32_t alarm, fail, domain, margin;
-  uint32_t n_alarm_threads, first_thread; int32_t applied, pad;
+  uint32_t n_alarm_threads, first_thread; int32_t applied; float gap;
 } ora_runinfo;
 typedef struct {
   int64_t index; int32_t bench, site; int64_t thread, inst; uint64_t mask;
-  int32_t cls; uint32_t alarm, fail, domain, margin; float worst;
+  int32_t cls; uint32_t alarm, fail, domain, margin; float worst; float gap; int32_t pad;
 } ora_record;
 
 /* ------------------------------------------------------------------------------------------ */
@@ -189,8 +189,9 @@ static uint32_t ord_dist(float a, float b) {
   if (d < 0) d = -d;
   return d > 0x7fffffff ? 0x7fffffffu : (uint32_t)d;
 }
-/* Returns 1 if in range.  Updates *margin with the min ordinal distance to any bound. */
-static int in_range(const ora_ranges* R, int d, float v, uint32_t* margin) {
+/* Returns 1 if in range.  Updates *margin with the min ordinal distance to any bound and *gap with
+ * the min absolute distance |v - bound| (the two measures of the R22(a) guard band). */
+static int in_range(const ora_ranges* R, int d, float v, uint32_t* margin, float* gap) {
   const ora_rset* s = &R->det[d];
   int in = 0;
   for (int r = 0; r < s->n; ++r) {
@@ -200,17 +201,20 @@ static int in_range(const ora_ranges* R, int d, float v, uint32_t* margin) {
       uint32_t a = ord_dist(v, lo), b = ord_dist(v, hi);
       if (a < *margin) *margin = a;
       if (b < *margin) *margin = b;
+      float ga = fabsf(v - lo), gb = fabsf(v - hi);
+      if (ga < *gap) *gap = ga;
+      if (gb < *gap) *gap = gb;
     }
   }
   return in;
 }
 
 typedef struct {
-  uint32_t alarm, fail, domain, margin;
+  uint32_t alarm, fail, domain, margin; float gap;
   int nw; int32_t wbuf[16]; int64_t widx[16]; float wval[16];
 } tout;
 
-static void tout_init(tout* o) { memset(o, 0, sizeof(*o)); o->margin = 0xffffffffu; }
+static void tout_init(tout* o) { memset(o, 0, sizeof(*o)); o->margin = 0xffffffffu; o->gap = INFINITY; }
 
 /* ------------------------------------------------------------------------------------------ */
 /* CP (K1).  DESIGN.md §3.2; PAPER Fig. 9, loop-detector code L1422-1429.           */
@@ -307,7 +311,7 @@ static void cp_thread(const ora_cp_args* P, const float* A4, int64_t t, int flag
     for (int d = 0; d < ndet; ++d) {
       float v = E[U - 1 - d] / (float)it;
       if (flags & F_PROFILE) samples[(int64_t)d * nthr + t] = v;
-      if (L && R->det[d].n > 0 && !in_range(R, d, v, &o->margin)) o->alarm |= AL_RANGE;
+      if (L && R->det[d].n > 0 && !in_range(R, d, v, &o->margin, &o->gap)) o->alarm |= AL_RANGE;
     }
   }
   if (NL) { chk ^= fb(coorx); chk ^= fb(coory); chk ^= fb(gu); }
@@ -431,7 +435,7 @@ static void mriq_thread(const ora_mriq_args* P, const float* KV, int64_t t, int 
     for (int d = 0; d < ndet; ++d) {
       float v = (d == 0 ? Qr : Qi) / (float)it;
       if (flags & F_PROFILE) samples[(int64_t)d * nthr + t] = v;
-      if (L && R->det[d].n > 0 && !in_range(R, d, v, &o->margin)) o->alarm |= AL_RANGE;
+      if (L && R->det[d].n > 0 && !in_range(R, d, v, &o->margin, &o->gap)) o->alarm |= AL_RANGE;
     }
   }
   if (NL) { chk ^= fb(sX); chk ^= fb(sY); chk ^= fb(sZ); }
@@ -552,7 +556,7 @@ static void tpacf_thread(const ora_tpacf_args* P, int64_t g, int flags, const or
   if ((L || (flags & F_PROFILE)) && cnt != 0 && ndet > 0) {
     float v = (float)acc / (float)cnt;
     if (flags & F_PROFILE) samples[g] = v;
-    if (L && R->det[0].n > 0 && !in_range(R, 0, v, &o->margin)) o->alarm |= AL_RANGE;
+    if (L && R->det[0].n > 0 && !in_range(R, 0, v, &o->margin, &o->gap)) o->alarm |= AL_RANGE;
   }
   if (NL) {
     chk ^= (uint32_t)boff; chk ^= (uint32_t)je; chk ^= (uint32_t)base;
@@ -572,9 +576,11 @@ static void info_fold(ora_runinfo* I, const tout* o, int64_t t, int target) {
     if ((uint32_t)t < I->first_thread) I->first_thread = (uint32_t)t;
   }
   I->fail |= o->fail;
-  if (target) { I->domain |= o->domain; I->margin = o->margin; }
+  if (target) { I->domain |= o->domain; I->margin = o->margin; I->gap = o->gap; }
 }
-static void info_init(ora_runinfo* I) { memset(I, 0, sizeof(*I)); I->first_thread = 0xffffffffu; I->margin = 0xffffffffu; }
+static void info_init(ora_runinfo* I) {
+  memset(I, 0, sizeof(*I)); I->first_thread = 0xffffffffu; I->margin = 0xffffffffu; I->gap = INFINITY;
+}
 
 static fctx mkfctx(const ora_fault* f, int64_t t) {
   fctx F = {0, -1, 0, 0, 0};
@@ -1023,7 +1029,7 @@ static void replay_one(int b, const void* args, int exact, const ora_ranges* R, 
     if (!o.fail) wrong = ora_tpacf_wrong(hist, G->gh, P->n_rand, P->n_bins, &worst);
     free(hist); free(d);
   }
-  rec->alarm = o.alarm; rec->fail = o.fail; rec->domain = o.domain; rec->margin = o.margin;
+  rec->alarm = o.alarm; rec->fail = o.fail; rec->domain = o.domain; rec->margin = o.margin; rec->gap = o.gap;
   rec->worst = worst;
   *wrong_out = wrong;
 }
@@ -1051,7 +1057,7 @@ static void replica_one(int b, const void* args, int exact, const ora_ranges* R,
     if (!I.fail) wrong = ora_tpacf_wrong(hist, G->gh, P->n_rand, P->n_bins, &worst);
     free(hist);
   }
-  rec->alarm = I.alarm; rec->fail = I.fail; rec->domain = I.domain; rec->margin = I.margin;
+  rec->alarm = I.alarm; rec->fail = I.fail; rec->domain = I.domain; rec->margin = I.margin; rec->gap = I.gap;
   rec->worst = worst;
   *wrong_out = wrong;
 }

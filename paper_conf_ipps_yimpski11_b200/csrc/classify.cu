@@ -54,6 +54,7 @@ __device__ void write_outcome(int bench, const FaultRec& f, hk_control* cb, bool
     hk_outcome o;
     o.index = f.index; o.bench = bench; o.site = f.site; o.thread = f.thread; o.inst = f.inst; o.mask = f.mask;
     o.cls = cls; o.alarm = alarm; o.fail = fail; o.domain = cb->domain; o.margin = cb->check_margin; o.worst = worst;
+    o.gap = cb->check_gap; o.pad2 = 0;
     records[f.index - first] = o;
   }
   atomicAdd(reinterpret_cast<unsigned long long*>(counts + bench * 5 + cls), 1ull);

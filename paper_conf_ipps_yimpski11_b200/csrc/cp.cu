@@ -198,6 +198,7 @@ __device__ void cp_fi_program(const CPParams& p, const FaultRec& f, const CPGeo&
   const int64_t n_grid = (int64_t)G.gx * BX * U * G.gy * BY;
   const uint64_t atoms_real = (uint64_t)(uintptr_t)p.atoms;
   uint32_t chk = 0, alarm = 0, fail = 0, margin = 0xffffffffu;
+  float gap = __int_as_float(0x7f800000);
   bool applied = false;
 
   int32_t numatoms = p.numatoms;
@@ -297,7 +298,7 @@ __device__ void cp_fi_program(const CPParams& p, const FaultRec& f, const CPGeo&
     for (int d = 0; d < U; ++d) {
       if (d < p.ndet && p.R.n[d] > 0) {
         const float v = __fdiv_rn(E[U - 1 - d], fit);
-        if (!in_range<true>(p.R, d, v, &margin)) { alarm |= AL_RANGE; S.outlier(d, v); }
+        if (!in_range<true>(p.R, d, v, &margin, &gap)) { alarm |= AL_RANGE; S.outlier(d, v); }
       }
     }
   }
@@ -312,7 +313,7 @@ __device__ void cp_fi_program(const CPParams& p, const FaultRec& f, const CPGeo&
   chk ^= ((uint32_t)numatoms + z) ^ (fb(h) + z) ^ (lohi(pgrid) + z) ^ (lohi(patoms) + z);
   if (chk != 0) alarm |= AL_CHK;
 done:
-  S.finish(mine, alarm, fail, margin, 0u, applied, (uint32_t)t);
+  S.finish(mine, alarm, fail, margin, gap, 0u, applied, (uint32_t)t);
 }
 
 template <int KIND, int U, bool EXACT>
@@ -390,7 +391,8 @@ __global__ void __launch_bounds__(128) cp_replay_kernel(const CPReplayParams q) 
       fp_judge(v, q.golden[e], M, &wrong, &worst);
     }
   }
-  emit_outcome(q.bench, f, wrong, S.alarm, S.fail, S.domain, S.margin, worst, q.records, q.first, q.counts, q.site_counts);
+  emit_outcome(q.bench, f, wrong, S.alarm, S.fail, S.domain, S.margin, S.gap, worst, q.records, q.first, q.counts,
+               q.site_counts);
 }
 
 // ============================================================================================

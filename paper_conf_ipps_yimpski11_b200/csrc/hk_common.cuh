@@ -70,7 +70,7 @@ __device__ __forceinline__ uint32_t ord_dist(float a, float b) {
 
 // HauberkCheckRange (L1302-1313): v in any profiled range?  NaN -> out of range (R10).
 template <bool MARGIN>
-__device__ __forceinline__ bool in_range(const DevRanges& R, int d, float v, uint32_t* margin) {
+__device__ __forceinline__ bool in_range(const DevRanges& R, int d, float v, uint32_t* margin, float* gap = nullptr) {
   bool in = false;
 #pragma unroll
   for (int r = 0; r < 3; ++r) {
@@ -80,6 +80,7 @@ __device__ __forceinline__ bool in_range(const DevRanges& R, int d, float v, uin
       if (MARGIN && v == v) {
         uint32_t a = ord_dist(v, lo), b = ord_dist(v, hi);
         *margin = min(*margin, min(a, b));
+        *gap = fminf(*gap, fminf(fabsf(__fsub_rn(v, lo)), fabsf(__fsub_rn(v, hi))));  // R22(a) absolute gap
       }
     }
   }
@@ -227,12 +228,13 @@ struct ReplicaSinkF {
   hk_control* cb;
   __device__ __forceinline__ void store(int buf, int64_t e, float v) { atomicAdd(out[buf] + e, v); }
   __device__ __forceinline__ void outlier(int d, float v) { record_outlier(cb, d, v); }
-  __device__ __forceinline__ void finish(bool mine, uint32_t alarm, uint32_t fail, uint32_t margin, uint32_t domain,
-                                         bool applied, uint32_t tid) {
+  __device__ __forceinline__ void finish(bool mine, uint32_t alarm, uint32_t fail, uint32_t margin, float gap,
+                                         uint32_t domain, bool applied, uint32_t tid) {
     if (fail) atomicOr(&cb->fail, fail);
     if (mine) {
       cb->fault_applied = applied ? 1u : 0u;
       cb->check_margin = margin;
+      cb->check_gap = gap;
       cb->domain = domain;
     }
     fold_alarm(cb, alarm, tid);
@@ -245,12 +247,13 @@ struct ReplaySinkF {
   int64_t idx[MAXW];
   float val[MAXW];
   uint32_t alarm = 0, fail = 0, margin = 0xffffffffu, domain = 0;
+  float gap = __builtin_huge_valf();
   __device__ __forceinline__ void store(int b, int64_t e, float v) {
     if (n < MAXW) { buf[n] = b; idx[n] = e; val[n] = v; ++n; }
   }
   __device__ __forceinline__ void outlier(int, float) {}
-  __device__ __forceinline__ void finish(bool, uint32_t a, uint32_t f, uint32_t m, uint32_t d, bool, uint32_t) {
-    alarm = a; fail = f; margin = m; domain = d;
+  __device__ __forceinline__ void finish(bool, uint32_t a, uint32_t f, uint32_t m, float g, uint32_t d, bool, uint32_t) {
+    alarm = a; fail = f; margin = m; gap = g; domain = d;
   }
 };
 
@@ -265,13 +268,14 @@ __device__ __forceinline__ void fp_judge(float v, float g, float M, bool* wrong,
 }
 
 __device__ __forceinline__ void emit_outcome(int bench, const FaultRec& f, bool wrong, uint32_t alarm, uint32_t fail,
-                                             uint32_t domain, uint32_t margin, float worst, hk_outcome* records,
+                                             uint32_t domain, uint32_t margin, float gap, float worst, hk_outcome* records,
                                              int64_t first, int64_t* counts, int64_t* site_counts) {
   const int32_t cls = fail ? HK_FAILURE : (!wrong ? (alarm ? HK_DETECTED_MASKED : HK_MASKED) : (alarm ? HK_DETECTED : HK_UNDETECTED));
   if (records) {
     hk_outcome o;
     o.index = f.index; o.bench = bench; o.site = f.site; o.thread = f.thread; o.inst = f.inst; o.mask = f.mask;
     o.cls = cls; o.alarm = alarm; o.fail = fail; o.domain = domain; o.margin = margin; o.worst = worst;
+    o.gap = gap; o.pad2 = 0;
     records[f.index - first] = o;
   }
   atomicAdd(reinterpret_cast<unsigned long long*>(counts + bench * 5 + cls), 1ull);
@@ -289,6 +293,7 @@ __device__ __forceinline__ void control_reset(hk_control* cb, int lane) {
     else if (lane >= 4 && lane < 12) v = 0x7fffffffu;  // outlier_min_ord
     else if (lane >= 12 && lane < 20) v = 0x80000000u; // outlier_max_ord
     else if (lane == 21) v = 0xffffffffu;              // check_margin
+    else if (lane == 23) v = 0x7f800000u;              // check_gap = +inf
     w[lane] = v;
   }
 }

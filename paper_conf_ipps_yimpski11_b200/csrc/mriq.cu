@@ -204,6 +204,7 @@ __device__ void mriq_fi_program(const MQParams& p, const FaultRec& f, int32_t t,
   const uint64_t kv_real = (uint64_t)(uintptr_t)p.kv;
   const uint64_t x_real = (uint64_t)(uintptr_t)p.x, y_real = (uint64_t)(uintptr_t)p.y, z_real = (uint64_t)(uintptr_t)p.z;
   uint32_t chk = 0, alarm = 0, fail = 0, margin = 0xffffffffu, domain = 0;
+  float gap = __int_as_float(0x7f800000);
   bool applied = false;
   int32_t numK = p.numK;
   uint64_t pkv = kv_real, pqr = qr_real, pqi = qi_real, px = x_real, py = y_real, pz = z_real;
@@ -290,7 +291,7 @@ __device__ void mriq_fi_program(const MQParams& p, const FaultRec& f, int32_t t,
     for (int d = 0; d < 2; ++d) {
       if (d < p.ndet && p.R.n[d] > 0) {
         const float v = __fdiv_rn(d == 0 ? Qr : Qi, fit);
-        if (!in_range<true>(p.R, d, v, &margin)) { alarm |= AL_RANGE; S.outlier(d, v); }
+        if (!in_range<true>(p.R, d, v, &margin, &gap)) { alarm |= AL_RANGE; S.outlier(d, v); }
       }
     }
   }
@@ -304,7 +305,7 @@ __device__ void mriq_fi_program(const MQParams& p, const FaultRec& f, int32_t t,
          (lohi(pz) + z);
   if (chk != 0) alarm |= AL_CHK;
 done:
-  S.finish(mine, alarm, fail, margin, domain, applied, (uint32_t)t);
+  S.finish(mine, alarm, fail, margin, gap, domain, applied, (uint32_t)t);
 }
 
 template <int KIND, bool EXACT>
@@ -378,7 +379,8 @@ __global__ void __launch_bounds__(128) mriq_replay_kernel(const MQReplayParams q
       fp_judge(v, q.golden[ge], M, &wrong, &worst);
     }
   }
-  emit_outcome(HK_MRIQ, f, wrong, S.alarm, S.fail, S.domain, S.margin, worst, q.records, q.first, q.counts, q.site_counts);
+  emit_outcome(HK_MRIQ, f, wrong, S.alarm, S.fail, S.domain, S.margin, S.gap, worst, q.records, q.first, q.counts,
+               q.site_counts);
 }
 
 // ============================================================================================

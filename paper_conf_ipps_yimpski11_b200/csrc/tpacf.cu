@@ -358,12 +358,13 @@ struct TPReplicaSink {
     H[((size_t)warp * nb2 + bin) * 32 + lane] += 1u;
   }
   __device__ __forceinline__ void outlier(int d, float v) { record_outlier(cb, d, v); }
-  __device__ __forceinline__ void finish(bool mine, uint32_t alarm, uint32_t fail, uint32_t margin, bool applied,
-                                         uint32_t tid) {
+  __device__ __forceinline__ void finish(bool mine, uint32_t alarm, uint32_t fail, uint32_t margin, float gap,
+                                         bool applied, uint32_t tid) {
     if (fail) atomicOr(&cb->fail, fail);
     if (mine) {
       cb->fault_applied = applied ? 1u : 0u;
       cb->check_margin = margin;
+      cb->check_gap = gap;
     }
     fold_alarm(cb, alarm, tid);
   }
@@ -373,6 +374,7 @@ struct TPReplaySink {
   int nr, nb, nb2, sign;
   int32_t* delta;  // [3 * nb]: DD, DRS, RRS for bins 1..nb
   uint32_t alarm = 0, fail = 0, margin = 0xffffffffu;
+  float gap = __builtin_huge_valf();
   __device__ __forceinline__ bool global_path(bool) const { return true; }
   __device__ __forceinline__ void hist_global(int64_t e) {
     const int row = (int)(e / nb2), b = (int)(e % nb2);
@@ -382,8 +384,8 @@ struct TPReplaySink {
   }
   __device__ __forceinline__ void hist_local(uint32_t, int32_t, uint32_t) {}
   __device__ __forceinline__ void outlier(int, float) {}
-  __device__ __forceinline__ void finish(bool, uint32_t a, uint32_t f, uint32_t m, bool, uint32_t) {
-    alarm = a; fail = f; margin = m;
+  __device__ __forceinline__ void finish(bool, uint32_t a, uint32_t f, uint32_t m, float g, bool, uint32_t) {
+    alarm = a; fail = f; margin = m; gap = g;
   }
 };
 
@@ -402,6 +404,7 @@ __device__ void tpacf_fi_program(const TPParams& p, const TPSmem& S, const Fault
   const uint64_t pts_real = (uint64_t)(uintptr_t)p.pts;
   const uint32_t lane = lane_id(), warp = threadIdx.x >> 5;
   uint32_t chk = 0, alarm = 0, fail = 0, margin = 0xffffffffu;
+  float gap = __int_as_float(0x7f800000);
   bool applied = false;
   int32_t n = p.n;
   uint64_t ppts = pts_real, phist = hist_real;
@@ -507,14 +510,14 @@ __device__ void tpacf_fi_program(const TPParams& p, const TPSmem& S, const Fault
   if (cnt != expect) alarm |= AL_COUNT;
   if (cnt != 0 && p.ndet > 0 && p.R.n[0] > 0) {
     const float v = __fdiv_rn((float)acc, (float)cnt);
-    if (!in_range<true>(p.R, 0, v, &margin)) { alarm |= AL_RANGE; K.outlier(0, v); }
+    if (!in_range<true>(p.R, 0, v, &margin, &gap)) { alarm |= AL_RANGE; K.outlier(0, v); }
   }
   chk ^= (uint32_t)opq(boff, z) ^ (uint32_t)opq(je, z) ^ (uint32_t)opq(base, z);
   chk ^= opqf(q1[0], z) ^ opqf(q1[1], z) ^ opqf(q1[2], z) ^ (uint32_t)opq(expect, z);
   chk ^= ((uint32_t)n + z) ^ (lohi(ppts) + z) ^ (lohi(phist) + z);
   if (chk != 0) alarm |= AL_CHK;
 done:
-  K.finish(mine, alarm, fail, margin, applied, (uint32_t)g);
+  K.finish(mine, alarm, fail, margin, gap, applied, (uint32_t)g);
 }
 
 template <int KIND>
@@ -603,7 +606,8 @@ __global__ void __launch_bounds__(128) tpacf_replay_kernel(const TPReplayParams 
       worst = fmaxf(worst, qv);
     }
   }
-  emit_outcome(HK_TPACF, f, wrong, K.alarm, K.fail, 0u, K.margin, worst, q.records, q.first, q.counts, q.site_counts);
+  emit_outcome(HK_TPACF, f, wrong, K.alarm, K.fail, 0u, K.margin, K.gap, worst, q.records, q.first, q.counts,
+               q.site_counts);
 }
 
 // ============================================================================================

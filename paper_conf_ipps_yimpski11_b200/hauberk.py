@@ -44,7 +44,7 @@ class Ranges(C.Structure):
 class Control(C.Structure):
     _fields_ = [("alarm", C.c_uint32), ("fail", C.c_uint32), ("n_alarm_warps", C.c_uint32), ("first_thread", C.c_uint32),
                 ("outlier_min_ord", C.c_int32 * 8), ("outlier_max_ord", C.c_int32 * 8), ("fault_applied", C.c_uint32),
-                ("check_margin", C.c_uint32), ("domain", C.c_uint32), ("reserved", C.c_uint32)]
+                ("check_margin", C.c_uint32), ("domain", C.c_uint32), ("check_gap", C.c_float)]
 
 
 CONTROL_BYTES = C.sizeof(Control)  # 96
@@ -82,7 +82,7 @@ class Fault(C.Structure):
 
 OUTCOME_DTYPE = np.dtype([("index", "<i8"), ("bench", "<i4"), ("site", "<i4"), ("thread", "<i8"), ("inst", "<i8"),
                           ("mask", "<u8"), ("cls", "<i4"), ("alarm", "<u4"), ("fail", "<u4"), ("domain", "<u4"),
-                          ("margin", "<u4"), ("worst", "<f4")], align=True)
+                          ("margin", "<u4"), ("worst", "<f4"), ("gap", "<f4"), ("pad2", "<i4")], align=True)
 
 _lib = None
 

@@ -45,6 +45,7 @@ def parse():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-multibit", action="store_true")
     ap.add_argument("--replay-count", type=int, default=1000000, help="injections per rank for the replay-mode line")
+    ap.add_argument("--no-fp-study", action="store_true")
     return ap.parse_args()
 
 
@@ -362,6 +363,18 @@ def main():
             multibit[str(k)] = {"coverage_pct": round(100.0 * hk.coverage(cc), 3),
                                 "coverage_by_bench_pct": {hk.BENCH_NAMES[b]: round(100.0 * hk.coverage(cc[b]), 3) for b in range(3)},
                                 "outcomes_pct": dict(zip(hk.CLASS_NAMES, (100.0 * cc.sum(0) / max(1, cc.sum())).round(2).tolist()))}
+    # ---- Fig. 16 analogue (NEXT f2): false-positive ratio of fault-free runs on 2
+    #      held-out synthetic datasets vs the number of training datasets (52 per program, 10 repeats)
+    fp_study = {}
+    if not args.no_fp_study and rank == 0:
+        from paper_conf_ipps_yimpski11_b200 import recovery as rc
+        makers = {"cp": lambda i: hk.CPDevice.from_problem(W.cp_problem(100, 64, 64, seed=60000 + i), dev),
+                  "mriq": lambda i: hk.MRIQDevice.from_problem(W.mriq_problem(32, 3072, seed=70000 + i), dev),
+                  "tpacf": lambda i: hk.TPACFDevice.from_problem(W.tpacf_problem(4096, 4, seed=80000 + i), dev)}
+        for name, mk in makers.items():
+            fp_study[name] = rc.false_positive_study(mk, n_sets=52, n_test=2, train_sizes=(1, 2, 5, 10, 20, 50), repeats=10)
+            torch.cuda.empty_cache()
+
     if rank == 0:
         line = {
             "metric": METRIC, "value": round(value, 2), "unit": "injections/s", "n_gpus": world, "steps": args.steps,
@@ -385,6 +398,7 @@ def main():
             "overhead_pct": overhead, "kernels": kernels, "fi_kernels": fi_split,
             "coverage_vs_bits": multibit,
             "replay": replay,
+            "false_positive_vs_training_sets": fp_study,
             "outcomes_pct_1bit": dict(zip(hk.CLASS_NAMES, (100.0 * c.sum(0) / max(1, c.sum())).round(2).tolist())),
             "ranges_identical_across_ranks": ranges_identical,
             "paper_context": {"overhead_pct_avg7": 15.3, "coverage_pct_avg": 86.8, "hardware": "Tesla S1070 (GT200)",

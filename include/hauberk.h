@@ -158,6 +158,11 @@ HK_API hk_status hauberk_inject_campaign(int32_t bench_mode, const void* const a
                                   hk_outcome* d_records, int64_t* d_counts, int64_t* d_site_counts,
                                   void* stream);
 
+/* The threshold search of hauberk_profile_ranges on caller-supplied HOST samples (e.g. the
+ * PROFILE samples of several training inputs concatenated — the paper's multi-set training,
+ * L2031-2036, L2654-2662).  Returns HK_ERR_PROFILE_NAN on a NaN/Inf sample. */
+HK_API hk_status hauberk_profile_search(const float* samples, int64_t n, int32_t t0_exp10, hk_range_set* out);
+
 /* Campaign session (the same campaign, prepared once): create validates, runs the golden programs,
  * checks they raise no alarm (synchronises `stream` once) and allocates the replica workspaces;
  * each run enqueues injections [first, first+count) on that stream without synchronising (the

@@ -491,6 +491,18 @@ hk_status hauberk_profile_ranges(int32_t bench, const void* args, const hk_profi
   return HK_OK;
 }
 
+hk_status hauberk_profile_search(const float* samples, int64_t n, int32_t t0_exp10, hk_range_set* out) {
+  if (!out || n < 0 || (n > 0 && !samples) || t0_exp10 < -38 || t0_exp10 > 38) return invalid("profile_search: bad arguments");
+  std::vector<float> v;
+  v.reserve((size_t)n);
+  for (int64_t i = 0; i < n; ++i) {
+    if (!std::isfinite(samples[i])) { g_err = "profile sample NaN/Inf"; return HK_ERR_PROFILE_NAN; }
+    v.push_back(samples[i]);
+  }
+  *out = profile_search(v, t0_exp10);
+  return HK_OK;
+}
+
 hk_status hauberk_decode(int32_t bench_mode, const void* const args[3], const uint64_t site_mask[3], uint64_t seed,
                          int32_t nbits, int64_t first, int64_t count, int32_t* bench_out, hk_fault* out) {
   if (!args || !site_mask || !bench_out || !out || count < 0 || first < 0 || bench_mode < -1 || bench_mode > 2)

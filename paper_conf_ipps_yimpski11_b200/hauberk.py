@@ -119,6 +119,8 @@ def lib():
         L.hauberk_campaign_run.argtypes = [P, I64, I64, P, P, P]
         L.hauberk_campaign_destroy.restype = None
         L.hauberk_campaign_destroy.argtypes = [P]
+        L.hauberk_profile_search.restype = I32
+        L.hauberk_profile_search.argtypes = [P, I64, I32, P]
         L.hauberk_timing_enable.restype = None
         L.hauberk_timing_enable.argtypes = [I32]
         L.hauberk_timing_read.restype = I32
@@ -130,7 +132,8 @@ def lib():
 EXPORTED = ["hauberk_run_cp", "hauberk_run_mriq", "hauberk_run_tpacf", "hauberk_profile_ranges",
             "hauberk_inject_campaign", "hauberk_decode", "hauberk_num_sites", "hauberk_strerror",
             "hauberk_last_error", "hauberk_version", "hauberk_launch_count", "hauberk_timing_enable",
-            "hauberk_timing_read", "hauberk_campaign_create", "hauberk_campaign_run", "hauberk_campaign_destroy"]
+            "hauberk_timing_read", "hauberk_campaign_create", "hauberk_campaign_run", "hauberk_campaign_destroy",
+            "hauberk_profile_search"]
 
 
 def _check(status: int, where: str):
@@ -326,6 +329,28 @@ def profile_ranges(dev, maxvar: int = 1, t0_exp10: int = -5, alpha: float = 1.0,
     st = lib().hauberk_profile_ranges(dev.bench, C.byref(a), C.byref(opts), C.byref(out), _stream(stream))
     _check(st, "hauberk_profile_ranges")
     return out
+
+
+def profile_search(samples: np.ndarray, t0_exp10: int = -5) -> RangeSet:
+    """hauberk_profile_search on host samples (float32)."""
+    s = np.ascontiguousarray(samples, dtype=np.float32)
+    out = RangeSet()
+    st = lib().hauberk_profile_search(s.ctypes.data_as(C.c_void_p), s.size, t0_exp10, C.byref(out))
+    _check(st, "hauberk_profile_search")
+    return out
+
+
+def profile_samples(dev, maxvar: int = 1, stream=None) -> torch.Tensor:
+    """PROFILE run (hauberk_run_* with HK_PROFILE): per-thread acc/it samples [maxvar, threads] on
+    the device (threads with zero trips keep NaN)."""
+    samples = torch.full((maxvar, dev.n_threads), float("nan"), dtype=torch.float32, device=dev.output()[0].device
+                         if isinstance(dev.output(), tuple) else dev.output().device)
+    R = Ranges()
+    R.n_det = maxvar
+    R.alpha = 1.0
+    cb = new_control(samples.device)
+    run(dev, HK_PROFILE, R, cb, samples, stream)
+    return samples
 
 
 def _arg_array(devs):

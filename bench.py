@@ -284,6 +284,15 @@ def main():
                 "traffic": None, "launches": nl, "share_of_step": round(ms / my_ms, 3) if my_ms else None,
                 "ops_per_pair": ops, "peak_source": f"{N_SM} SMs x {MUFU_PER_SM_CLK if dom < 2 else LANES_PER_SM_CLK}/clk/SM x {sm_mhz_peak:.0f} MHz ({clk_src})"}
     fi_split = {hk.BENCH_NAMES[b]: {"ms": round(fi[b][0], 3), "launches": fi[b][1], "pairs": fi[b][2]} for b in range(3)}
+    # traffic: DRAM bytes per launch of the same kernel/batch from the committed ncu capture
+    try:
+        with open(os.path.join(ROOT, "profiles", "r01_traffic.json")) as f:
+            tr = json.load(f).get(f"{hk.BENCH_NAMES[dom]}_fi_kernel")
+        if tr:
+            roofline["traffic"] = tr["dram_bytes_per_launch"]
+            roofline["traffic_source"] = tr["source"]
+    except (OSError, ValueError):
+        pass
 
     # ---- e2e: pinned host inputs copied to the device every step, counts read back every step
     host = {}

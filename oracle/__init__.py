@@ -26,6 +26,8 @@ FT = F_NL | F_L
 AL_DUP, AL_CHK, AL_RANGE, AL_COUNT = 1, 2, 4, 8
 FL_CRASH, FL_HANG = 1, 2
 ALL_SITES = (1 << 64) - 1
+MRIQ_PHIMAG_SITES = ((1 << 36) - 1) ^ ((1 << 29) - 1)
+DEFAULT_SITE_MASKS = (ALL_SITES, (1 << 29) - 1, ALL_SITES)  # PhiMag sites excluded by default (R22)
 
 
 class RSet(C.Structure):
@@ -245,7 +247,7 @@ def ranges_to_list(R: Ranges):
 
 
 def campaign(bench_mode: int, problems, ranges, seed: int, first: int, count: int, exact: int = 0,
-             mode: int = 1, site_masks=(ALL_SITES,) * 3, records: bool = True, nbits: int = 1):
+             mode: int = 1, site_masks=DEFAULT_SITE_MASKS, records: bool = True, nbits: int = 1):
     """Seeded campaign.  problems/ranges: 3-lists indexed by bench (None where unused).
     mode 1 = replay, 0 = replica.  Returns (counts int64[3,5], records structured array)."""
     L = lib()
@@ -263,7 +265,7 @@ def campaign(bench_mode: int, problems, ranges, seed: int, first: int, count: in
     return counts, recs
 
 
-def decode(bench_mode: int, problems, seed: int, first: int, count: int, site_masks=(ALL_SITES,) * 3, nbits: int = 1):
+def decode(bench_mode: int, problems, seed: int, first: int, count: int, site_masks=DEFAULT_SITE_MASKS, nbits: int = 1):
     L = lib()
     argv = [make_args(b, problems[b]) if problems[b] is not None else None for b in range(3)]
     aptr = (C.c_void_p * 3)(*[C.cast(C.byref(a), C.c_void_p) if a is not None else None for a in argv])

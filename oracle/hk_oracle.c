@@ -357,9 +357,44 @@ static int cp_valid(const ora_cp_args* P) {
 /*   8 numK 9 kv* 10 qr* 11 qi* 12 x* 13 y* 14 z* (param @live)                                */
 /*   15 k 16 kx 17 ky 18 kz 19 pm 20 t1 21 t2 22 t 23 r 24 c 25 s 26 Qr 27 Qi 28 it (loop)     */
 /* ------------------------------------------------------------------------------------------ */
-#define MRIQ_NSITES 29
+#define MRIQ_NSITES 36
+#define MRIQ_PHIMAG_SITE0 29 /* 29 kidx 30 re 31 im 32 pm 33 kx 34 ky 35 kz: PhiMag NL @def (replica only) */
 static const float TWO_PI_F = 6.28318548202514648f; /* binary32 nearest 2*pi (0x40C90FDB) */
 static const float RINT_MAGIC = 12582912.0f;        /* 1.5 * 2^23 */
+
+/* PhiMag abstract thread k (non-loop code: HAUBERK-NL on every virtual variable, loads included,
+ * A1-A3).  kv is written additively into a zeroed buffer (R18).  Sites 29-35. */
+static void phimag_thread(const ora_mriq_args* P, int64_t k, int flags, fctx* F, tout* o, float* kv) {
+  const int NL = flags & F_NL, FI = flags & F_FI;
+  uint32_t chk = 0;
+  const int64_t nk = P->n_k;
+  int64_t e;
+  int32_t kidx = fi32(F, 29, 0, (int32_t)k);
+  if (NL) { chk ^= (uint32_t)kidx; if ((int32_t)k != kidx) o->alarm |= AL_DUP; }
+#define PHLOAD(var, arr, site)                                                       \
+  if (FI && !access_ok(VBASE, kidx, 4, nk, &e)) { o->fail |= FL_CRASH; return; }      \
+  else if (!FI) e = kidx;                                                           \
+  float var = ff32(F, site, 0, (arr)[e]);                                           \
+  if (NL) { chk ^= fb(var); if (fb((arr)[e]) != fb(var)) o->alarm |= AL_DUP; }
+  PHLOAD(re, P->phi_r, 30)
+  PHLOAD(im, P->phi_i, 31)
+  float pm = ff32(F, 32, 0, fmaf(im, im, re * re));
+  if (NL) { chk ^= fb(pm); if (fb(fmaf(im, im, re * re)) != fb(pm)) o->alarm |= AL_DUP; }
+  PHLOAD(kx, P->kx, 33)
+  PHLOAD(ky, P->ky, 34)
+  PHLOAD(kz, P->kz, 35)
+#undef PHLOAD
+  if (FI && !access_ok(VBASE, kidx, 16, nk, &e)) { o->fail |= FL_CRASH; return; }
+  else if (!FI) e = kidx;
+  kv[4 * e + 0] = kv[4 * e + 0] + kx;
+  kv[4 * e + 1] = kv[4 * e + 1] + ky;
+  kv[4 * e + 2] = kv[4 * e + 2] + kz;
+  kv[4 * e + 3] = kv[4 * e + 3] + pm;
+  if (NL) {
+    chk ^= fb(re); chk ^= fb(im); chk ^= fb(pm); chk ^= fb(kx); chk ^= fb(ky); chk ^= fb(kz); chk ^= (uint32_t)kidx;
+    if (chk != 0) o->alarm |= AL_CHK;
+  }
+}
 
 static float* mriq_phimag(const ora_mriq_args* P) {
   float* kv = (float*)malloc(sizeof(float) * 4 * (size_t)(P->n_k > 0 ? P->n_k : 1));
@@ -612,12 +647,21 @@ ORA_EXPORT int ora_mriq_run(const ora_mriq_args* P, int32_t flags, int32_t exact
                             const ora_fault* f, float* qr, float* qi, float* samples, ora_runinfo* I) {
   if (!mriq_valid(P) || ndet < 0 || ndet > 2) return 1;
   if (f && f->site >= 0) flags |= F_FI;
-  float* KV = mriq_phimag(P);
+  const int phimag_fault = f && f->site >= MRIQ_PHIMAG_SITE0;
   memset(qr, 0, sizeof(float) * (size_t)P->n_vox);
   memset(qi, 0, sizeof(float) * (size_t)P->n_vox);
   info_init(I);
+  /* PhiMag (its detectors fold into the same control block as the Q kernel's) */
+  float* KV = (float*)calloc(4 * (size_t)(P->n_k > 0 ? P->n_k : 1), sizeof(float));
+  for (int64_t k = 0; k < P->n_k; ++k) {
+    fctx F = phimag_fault ? mkfctx(f, k) : mkfctx(NULL, k);
+    tout o; tout_init(&o);
+    phimag_thread(P, k, flags & (F_NL | F_FI), &F, &o, KV);
+    if (o.alarm || o.fail) { I->alarm |= o.alarm; I->fail |= o.fail; if (o.alarm) I->n_alarm_threads++; }
+    if (F.active) I->applied = F.applied;
+  }
   for (int64_t t = 0; t < P->n_vox; ++t) {
-    fctx F = mkfctx(f, t);
+    fctx F = phimag_fault ? mkfctx(NULL, t) : mkfctx(f, t);
     tout o; tout_init(&o);
     mriq_thread(P, KV, t, flags, exact, R, ndet, &F, &o, samples, P->n_vox);
     for (int w = 0; w < o.nw; ++w) {
@@ -842,7 +886,7 @@ ORA_EXPORT void ora_site_info(int32_t bench, int32_t unroll, int32_t site, int32
     if (site <= 5) *cls = SC_NL;
     if (site == 12 || site == 13) *width = 64;
   } else if (bench == B_MRIQ) {
-    if (site <= 3) *cls = SC_NL;
+    if (site <= 3 || site >= MRIQ_PHIMAG_SITE0) *cls = SC_NL;
     if (site >= 9 && site <= 14) *width = 64;
   } else {
     if (site <= 11) *cls = SC_NL;
@@ -858,6 +902,12 @@ typedef struct {
   int64_t nthr; int64_t trips_uniform; /* CP / MRI-Q */
   int64_t* prefix; int64_t total_trips;   /* TPACF: prefix[g] = sum of trips of threads < g */
 } catalog;
+
+/* Threads of an NL site: PhiMag sites of MRI-Q run on the n_k PhiMag threads. */
+static int64_t cat_nl_threads(const catalog* K, int s) {
+  if (K->bench == B_MRIQ && s >= MRIQ_PHIMAG_SITE0) return K->mq->n_k;
+  return K->nthr;
+}
 
 static void cat_build(catalog* K, int bench, const void* args, uint64_t site_mask) {
   memset(K, 0, sizeof(*K));
@@ -876,7 +926,7 @@ static void cat_build(catalog* K, int bench, const void* args, uint64_t site_mas
   for (int s = 0; s < K->nsites; ++s) {
     if (!((site_mask >> s) & 1)) continue;
     int32_t cls, w; ora_site_info(bench, U, s, &cls, &w);
-    int64_t D = cls == SC_NL ? K->nthr : K->total_trips;
+    int64_t D = cls == SC_NL ? cat_nl_threads(K, s) : K->total_trips;
     if (D > 0) K->en[K->nen++] = s;
   }
 }
@@ -896,7 +946,7 @@ static void cat_decode(const catalog* K, uint64_t seed, int64_t n, int nbits, or
   int32_t cls, w; ora_site_info(K->bench, U, s, &cls, &w);
   f->site = s; f->pad = 0;
   if (cls == SC_NL) {
-    f->thread = (int64_t)ora_bounded(r2, (uint64_t)K->nthr);
+    f->thread = (int64_t)ora_bounded(r2, (uint64_t)cat_nl_threads(K, s));
     f->inst = 0;
   } else {
     int64_t u = (int64_t)ora_bounded(r2, (uint64_t)K->total_trips);
@@ -1081,7 +1131,8 @@ ORA_EXPORT int ora_campaign(int32_t bench_mode, const void* const args[3], const
     ora_fault f; cat_decode(&K[b], seed, n, nbits, &f);
     ora_record rec; memset(&rec, 0, sizeof(rec));
     int32_t wrong = 0;
-    if (mode == 1) replay_one(b, args[b], exact, ranges[b], &G[b], &f, &rec, &wrong);
+    /* replay cannot express a PhiMag fault (it reaches every voxel, R22): run that one as a replica */
+    if (mode == 1 && !(b == B_MRIQ && f.site >= MRIQ_PHIMAG_SITE0)) replay_one(b, args[b], exact, ranges[b], &G[b], &f, &rec, &wrong);
     else replica_one(b, args[b], exact, ranges[b], &G[b], &f, &rec, &wrong);
     rec.index = n; rec.bench = b; rec.site = f.site; rec.thread = f.thread; rec.inst = f.inst; rec.mask = f.mask;
     rec.cls = ora_classify(wrong, rec.alarm, rec.fail);

@@ -238,8 +238,10 @@ static hk_range_set profile_search(const std::vector<float>& v, int t0) {
 // ---------------------------------------------------------------------------------------------
 // Site catalogue and decode (R14, R15)
 // ---------------------------------------------------------------------------------------------
-static int num_sites(int b, int unroll) { return b == HK_CP ? 22 + 4 * unroll : (b == HK_MRIQ ? 29 : 31); }
-static bool site_is_nl(int b, int s) { return b == HK_CP ? s <= 5 : (b == HK_MRIQ ? s <= 3 : s <= 11); }
+static int num_sites(int b, int unroll) { return b == HK_CP ? 22 + 4 * unroll : (b == HK_MRIQ ? 36 : 31); }
+static bool site_is_nl(int b, int s) {
+  return b == HK_CP ? s <= 5 : (b == HK_MRIQ ? (s <= 3 || s >= MRIQ_PHIMAG_SITE0) : s <= 11);
+}
 static int site_width(int b, int s) {
   if (b == HK_CP) return (s == 12 || s == 13) ? 64 : 32;
   if (b == HK_MRIQ) return (s >= 9 && s <= 14) ? 64 : 32;
@@ -257,6 +259,8 @@ struct Catalog {
   int bench = -1, unroll = 1;
   std::vector<int> enabled;
   int64_t nthr = 0, uniform_trips = 0, total_trips = 0;
+  int64_t nk = 0;  // MRI-Q: PhiMag threads (sites 29-35)
+  int64_t nl_threads(int s) const { return (bench == HK_MRIQ && s >= MRIQ_PHIMAG_SITE0) ? nk : nthr; }
   std::vector<int64_t> prefix;  // TPACF: prefix[g] = trips of threads < g
 };
 
@@ -271,6 +275,7 @@ static bool build_catalog(Catalog& K, int b, const void* args, uint64_t mask) {
   } else if (b == HK_MRIQ) {
     const hk_mriq_args* a = (const hk_mriq_args*)args;
     K.nthr = a->n_vox;
+    K.nk = a->n_k;
     K.uniform_trips = a->n_k;
     K.total_trips = K.nthr * K.uniform_trips;
   } else {
@@ -283,7 +288,7 @@ static bool build_catalog(Catalog& K, int b, const void* args, uint64_t mask) {
   }
   for (int s = 0; s < num_sites(b, K.unroll) && s < 64; ++s) {
     if (!((mask >> s) & 1ull)) continue;
-    const int64_t D = site_is_nl(b, s) ? K.nthr : K.total_trips;
+    const int64_t D = site_is_nl(b, s) ? K.nl_threads(s) : K.total_trips;
     if (D > 0) K.enabled.push_back(s);
   }
   return !K.enabled.empty();
@@ -297,7 +302,7 @@ static hk_fault decode_one(const Catalog& K, uint64_t seed, int64_t n, int nbits
   const int s = K.enabled[below(r1, K.enabled.size())];
   f.site = s;
   if (site_is_nl(K.bench, s)) {
-    f.thread = (int64_t)below(r2, (uint64_t)K.nthr);
+    f.thread = (int64_t)below(r2, (uint64_t)K.nl_threads(s));
     f.inst = 0;
   } else {
     const int64_t u = (int64_t)below(r2, (uint64_t)K.total_trips);
@@ -352,6 +357,7 @@ struct BenchWS {
   hk_control* rep_cb = nullptr;
   hk_control* gold_cb = nullptr;
   void* lut = nullptr;  // TPACF bucket table
+  float4* kv_rep = nullptr;  // MRI-Q PhiMag-site replicas: per-replica k-space
   int batch = 0;
 };
 
@@ -556,6 +562,7 @@ static void session_free(hk_campaign_session* S) {
     if (w.rep_cb) cudaFree(w.rep_cb);
     if (w.gold_cb) cudaFree(w.gold_cb);
     if (w.lut) cudaFree(w.lut);
+    if (w.kv_rep) cudaFree(w.kv_rep);
   }
   if (S->d_faults) cudaFree(S->d_faults);
   if (S->h_faults) cudaFreeHost(S->h_faults);
@@ -608,6 +615,12 @@ static hk_status session_create(int32_t bench_mode, const void* const args[3], c
     w.ndet = ranges[b]->n_det;
     w.batch = C->mode == 1 ? 1 : (C->batch > 0 ? C->batch : default_batch(b, own));
     if (C->mode == 1 && b == HK_TPACF && 3 * S->tp.n_bins > 96) { g_err = "replay supports n_bins <= 32"; st = HK_ERR_UNSUPPORTED; break; }
+    const bool phimag_sites = b == HK_MRIQ && (C->site_mask[b] >> MRIQ_PHIMAG_SITE0) != 0;
+    if (C->mode == 1 && phimag_sites) {
+      g_err = "PhiMag sites reach every voxel: replica mode only (clear site_mask bits 29-35 for replay)";
+      st = HK_ERR_UNSUPPORTED;
+      break;
+    }
     size_t esz = sizeof(float);
     if (b == HK_CP) w.out_elems = (int64_t)S->cp.nx * S->cp.ny;
     else if (b == HK_MRIQ) w.out_elems = 2LL * S->mq.n_vox;
@@ -618,7 +631,9 @@ static hk_status session_create(int32_t bench_mode, const void* const args[3], c
         (e = cudaMalloc((void**)&w.dM, sizeof(float))) != cudaSuccess ||
         (e = cudaMalloc((void**)&w.gold_cb, sizeof(hk_control))) != cudaSuccess ||
         (e = cudaMalloc(&w.rep_out, esz * stride * w.batch)) != cudaSuccess ||
-        (e = cudaMalloc((void**)&w.rep_cb, sizeof(hk_control) * w.batch)) != cudaSuccess) {
+        (e = cudaMalloc((void**)&w.rep_cb, sizeof(hk_control) * w.batch)) != cudaSuccess ||
+        (b == HK_MRIQ && (C->site_mask[b] >> MRIQ_PHIMAG_SITE0) != 0 &&
+         (e = cudaMalloc((void**)&w.kv_rep, sizeof(float4) * (size_t)std::max(1, S->mq.n_k) * w.batch)) != cudaSuccess)) {
       st = cuda_fail(e, "campaign workspace");
       break;
     }
@@ -753,7 +768,8 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
                                   d_records, first, d_counts, d_site_counts, s)) != cudaSuccess)
         return cuda_fail(e, "classify");
     } else if (b == HK_MRIQ) {
-      if ((e = mriq_fi_launch(kind, S->mq, w.R, std::min(w.ndet, 2), fr, nrep, (float*)w.rep_out, w.out_elems, w.rep_cb, s)) != cudaSuccess)
+      if ((e = mriq_fi_launch(kind, S->mq, w.R, std::min(w.ndet, 2), fr, nrep, (float*)w.rep_out, w.out_elems, w.rep_cb,
+                              w.kv_rep, s)) != cudaSuccess)
         return cuda_fail(e, "mriq FI");
       if ((e = classify_fp_launch(b, (float*)w.rep_out, w.out_elems, (const float*)w.golden, w.dM, w.rep_cb, fr, nrep,
                                   d_records, first, d_counts, d_site_counts, s)) != cudaSuccess)

@@ -45,9 +45,16 @@ __global__ void __launch_bounds__(256) mriq_phimag_kernel(const float* __restric
       const float re2 = bf(fb(re) + z), im2 = bf(fb(im) + z);
       alarm |= (fb(__fmaf_rn(im2, im2, __fmul_rn(re2, re2))) != fb(pm)) ? AL_DUP : 0u;
     }
-    kv[k] = make_float4(kx[k], ky[k], kz[k], pm);
+    const float lx = kx[k], ly = ky[k], lz = kz[k];
+    if (NL) {
+      chk ^= fb(lx); alarm |= (fb(kx[opq(k, z)]) != fb(lx)) ? AL_DUP : 0u;
+      chk ^= fb(ly); alarm |= (fb(ky[opq(k, z)]) != fb(ly)) ? AL_DUP : 0u;
+      chk ^= fb(lz); alarm |= (fb(kz[opq(k, z)]) != fb(lz)) ? AL_DUP : 0u;
+    }
+    kv[k] = make_float4(lx, ly, lz, pm);
     if (NL) {
       chk ^= opqf(re, z); chk ^= opqf(im, z); chk ^= opqf(pm, z); chk ^= (uint32_t)opq(k, z);
+      chk ^= opqf(lx, z); chk ^= opqf(ly, z); chk ^= opqf(lz, z);
       if (chk) alarm |= AL_CHK;
     }
   }
@@ -180,7 +187,9 @@ __global__ void __launch_bounds__(256) mriq_kernel(const MQParams p) {
 // FI & FT replicas (blockIdx.y = replica).  See cp.cu for the scheme.
 // ============================================================================================
 enum MQKind : int {
-  MK_NL = 0, MK_LIVE, MK_K, MK_KX, MK_KY, MK_KZ, MK_PM, MK_T1, MK_T2, MK_T, MK_R, MK_C, MK_S, MK_QR, MK_QI, MK_IT, MK_COUNT
+  MK_NL = 0, MK_LIVE, MK_K, MK_KX, MK_KY, MK_KZ, MK_PM, MK_T1, MK_T2, MK_T, MK_R, MK_C, MK_S, MK_QR, MK_QI, MK_IT,
+  MK_PHIMAG,  // sites 29-35 (PhiMag NL): replica mode only
+  MK_COUNT
 };
 
 struct MQFIParams {
@@ -188,6 +197,7 @@ struct MQFIParams {
   const FaultRec* faults;
   float* out0;  // replica r: qr = out0 + r*stride, qi = qr + numX
   int64_t stride;
+  const float4* kv0;  // PhiMag-site replicas: per-replica k-space [nrep][numK]
   hk_control* cb0;
 };
 
@@ -308,6 +318,60 @@ done:
   S.finish(mine, alarm, fail, margin, gap, domain, applied, (uint32_t)t);
 }
 
+// PhiMag replicas for PhiMag-site injections (sites 29-35): every thread runs the
+// instrumented PhiMag program; the target thread gets the flip, guarded loads/stores (R16) and
+// additive kv writes into the replica's zeroed buffer (R18); alarms fold into the replica's cb.
+__global__ void __launch_bounds__(256) mriq_phimag_fi_kernel(const float* __restrict__ kx, const float* __restrict__ ky,
+                                                            const float* __restrict__ kz, const float* __restrict__ pr,
+                                                            const float* __restrict__ pi, float4* kv0, int numK,
+                                                            const FaultRec* faults, hk_control* cb0, uint32_t z) {
+  const int r = blockIdx.y;
+  const FaultRec f = faults[r];
+  float* kv = reinterpret_cast<float*>(kv0 + (int64_t)r * numK);
+  hk_control* cb = cb0 + r;
+  const int k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k >= numK) return;
+  const bool mine = (k == f.thread);
+  const uint64_t mask = f.mask;
+  const int site = mine ? f.site : -1;
+  uint32_t chk = 0, alarm = 0, fail = 0;
+  int64_t e;
+  const int64_t nk = numK;
+  const uint64_t vb = VBASE;  // PhiMag's pointers are not injection sites: only indices move
+  int32_t kidx = flip_i(k, site == 29, mask);
+  chk ^= (uint32_t)kidx; alarm |= ((int)((blockIdx.x ^ z) * blockDim.x + (threadIdx.x ^ z)) != kidx) ? AL_DUP : 0u;
+  float v[5];
+  const float* src[5] = {pr, pi, kx, ky, kz};
+  const int sid[5] = {30, 31, 33, 34, 35};
+#pragma unroll
+  for (int a = 0; a < 5; ++a) {
+    if (!guard(vb, vb, kidx, 4, nk, &e)) { fail |= FL_CRASH; goto done; }
+    v[a] = flip_f(src[a][e], site == sid[a], mask);
+    chk ^= fb(v[a]); alarm |= (fb(src[a][e + z]) != fb(v[a])) ? AL_DUP : 0u;
+    if (a == 1) {
+      // pm right after re, im (program order of DESIGN §3.3)
+    }
+  }
+  {
+    const float re = v[0], im = v[1];
+    float pm = flip_f(__fmaf_rn(im, im, __fmul_rn(re, re)), site == 32, mask);
+    chk ^= fb(pm);
+    const float re2 = bf(fb(re) + z), im2 = bf(fb(im) + z);
+    alarm |= (fb(__fmaf_rn(im2, im2, __fmul_rn(re2, re2))) != fb(pm)) ? AL_DUP : 0u;
+    if (!guard(vb, vb, kidx, 16, nk, &e)) { fail |= FL_CRASH; goto done; }
+    atomicAdd(kv + 4 * e + 0, v[2]);
+    atomicAdd(kv + 4 * e + 1, v[3]);
+    atomicAdd(kv + 4 * e + 2, v[4]);
+    atomicAdd(kv + 4 * e + 3, pm);
+    chk ^= opqf(v[0], z) ^ opqf(v[1], z) ^ opqf(pm, z) ^ opqf(v[2], z) ^ opqf(v[3], z) ^ opqf(v[4], z) ^ (uint32_t)opq(kidx, z);
+    if (chk) alarm |= AL_CHK;
+  }
+done:
+  if (fail) atomicOr(&cb->fail, fail);
+  if (mine) cb->fault_applied = 1u;
+  fold_alarm(cb, alarm, (uint32_t)k);
+}
+
 template <int KIND, bool EXACT>
 __global__ void __launch_bounds__(256) mriq_fi_kernel(const MQFIParams q) {
   __shared__ __align__(128) float4 tile[2][MQ_TILE];
@@ -318,7 +382,8 @@ __global__ void __launch_bounds__(256) mriq_fi_kernel(const MQFIParams q) {
   p.qr = q.out0 + (int64_t)r * q.stride;
   p.qi = p.qr + p.numX;
   p.cb = q.cb0 + r;
-  if (f.thread / (2 * blockDim.x) != blockIdx.x) {
+  if (KIND == MK_PHIMAG) p.kv = q.kv0 + (int64_t)r * p.numK;  // this replica's (possibly faulted) k-space
+  if (KIND == MK_PHIMAG || f.thread / (2 * blockDim.x) != blockIdx.x) {
     mriq_body<V_NL | V_L, EXACT, true, 2>(p, tile, bar);
   } else {
     ReplicaSinkF S{{p.qr, p.qi}, p.cb};
@@ -437,6 +502,7 @@ cudaError_t mriq_launch(int vflags, const hk_mriq_args& a, const DevRanges& R, i
 int mriq_site_kind(int site) {
   if (site <= 3) return MK_NL;
   if (site <= 14) return MK_LIVE;
+  if (site >= 29) return MK_PHIMAG;
   return MK_K + (site - 15);
 }
 
@@ -454,7 +520,7 @@ static cudaError_t launch_mq_fi_e(int kind, const MQFIParams& q, int nrep, cudaS
   switch (kind) {
 #define K(k) case k: return launch_mq_fi_k<k, EXACT>(q, nrep, s);
     K(MK_NL) K(MK_LIVE) K(MK_K) K(MK_KX) K(MK_KY) K(MK_KZ) K(MK_PM) K(MK_T1) K(MK_T2) K(MK_T) K(MK_R) K(MK_C) K(MK_S)
-    K(MK_QR) K(MK_QI) K(MK_IT)
+    K(MK_QR) K(MK_QI) K(MK_IT) K(MK_PHIMAG)
 #undef K
   }
   return cudaErrorInvalidValue;
@@ -491,8 +557,18 @@ cudaError_t mriq_replay_launch(int kind, const hk_mriq_args& a, const DevRanges&
 }
 
 cudaError_t mriq_fi_launch(int kind, const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
-                           float* out0, int64_t stride, hk_control* cb0, cudaStream_t s) {
+                           float* out0, int64_t stride, hk_control* cb0, float4* kv_rep, cudaStream_t s) {
+  if (kind == MK_PHIMAG) {
+    if (!kv_rep) return cudaErrorInvalidValue;
+    cudaError_t e = cudaMemsetAsync(kv_rep, 0, sizeof(float4) * (size_t)a.n_k * nrep, s);
+    if (e != cudaSuccess) return e;
+    dim3 g((a.n_k + 255) / 256, nrep);
+    mriq_phimag_fi_kernel<<<g, 256, 0, s>>>(a.kx, a.ky, a.kz, a.phi_r, a.phi_i, kv_rep, a.n_k, faults, cb0, opaque_zero());
+    count_launch();
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  }
   MQFIParams q{};
+  q.kv0 = kv_rep;
   q.base = mq_params(a, R, ndet, nullptr, nullptr);
   q.faults = faults;
   q.out0 = out0;

@@ -21,6 +21,9 @@ HK_BASE, HK_FT, HK_FT_NL, HK_FT_L, HK_PROFILE = 0, 1, 2, 3, 4
 CLASS_NAMES = ["masked", "detected_masked", "detected", "undetected", "failure"]
 BENCH_NAMES = ["cp", "mriq", "tpacf"]
 ALL_SITES = (1 << 64) - 1
+MRIQ_PHIMAG_SITES = ((1 << 36) - 1) ^ ((1 << 29) - 1)  # sites 29-35: PhiMag (replica mode only, R22)
+# default campaign masks: every site except MRI-Q's PhiMag sites
+DEFAULT_SITE_MASKS = (ALL_SITES, (1 << 29) - 1, ALL_SITES)
 
 
 class HauberkError(RuntimeError):
@@ -361,7 +364,7 @@ def _arg_array(devs):
 
 def inject_campaign(bench_mode: int, devs, ranges, seed: int, first: int, count: int, counts: torch.Tensor,
                     records: torch.Tensor | None = None, site_counts: torch.Tensor | None = None, exact: int = 0,
-                    batch: int = 0, site_masks=(ALL_SITES,) * 3, stream=None, nbits: int = 1, mode: int = 0):
+                    batch: int = 0, site_masks=DEFAULT_SITE_MASKS, stream=None, nbits: int = 1, mode: int = 0):
     """hauberk_inject_campaign (replica mode).  devs/ranges: 3-lists by bench (None where unused).
     counts: int64 cuda tensor [3, 5] (accumulated); records: optional uint8 tensor of
     count * OUTCOME_DTYPE.itemsize bytes; site_counts: optional int64 [3, 64, 5]."""
@@ -379,7 +382,7 @@ class CampaignSession:
     asynchronous slices of the same seeded campaign.  Keep `devs` alive while the session lives."""
 
     def __init__(self, bench_mode: int, devs, ranges, seed: int, exact: int = 0, batch: int = 0,
-                 site_masks=(ALL_SITES,) * 3, stream=None, nbits: int = 1, mode: int = 0):
+                 site_masks=DEFAULT_SITE_MASKS, stream=None, nbits: int = 1, mode: int = 0):
         self._arr, self._keep = _arg_array(devs)
         self._devs = devs
         self._rng = [r if r is not None else Ranges() for r in ranges]
@@ -421,7 +424,7 @@ def records_numpy(rec: torch.Tensor) -> np.ndarray:
     return np.frombuffer(rec.cpu().numpy().tobytes(), dtype=OUTCOME_DTYPE)
 
 
-def decode(bench_mode: int, devs, seed: int, first: int, count: int, site_masks=(ALL_SITES,) * 3, nbits: int = 1):
+def decode(bench_mode: int, devs, seed: int, first: int, count: int, site_masks=DEFAULT_SITE_MASKS, nbits: int = 1):
     """hauberk_decode (host): the campaign's (bench, site, thread, instance, mask) tuples."""
     arr, keep = _arg_array(devs)
     masks = (C.c_uint64 * 3)(*site_masks)

@@ -446,3 +446,32 @@ def test_full_config5_campaign_1M_gpu_replay_vs_oracle():
     assert np.array_equal(g["cls"][tp], o["cls"][tp])
     assert amb.mean() < 0.01
     assert gc.sum() == N
+
+
+@pytest.mark.parametrize("exact", [1, 0])
+def test_phimag_site_replicas_vs_oracle_replicas(exact):
+    """MRI-Q PhiMag sites (29-35; replica mode only): 200 injections, GPU replica vs
+    oracle replica (the fault reaches every voxel through the shared k-space)."""
+    p = W.mriq_problem(6, 53, n_vox=180, seed=21)
+    d = _mk(1, p, exact)
+    R = hk.profile_ranges(d)
+    masks = (hk.ALL_SITES, hk.MRIQ_PHIMAG_SITES, hk.ALL_SITES)
+    counts = torch.zeros((3, 5), dtype=torch.int64, device=DEV)
+    rec = hk.records_tensor(200, DEV)
+    hk.inject_campaign(hk.HK_MRIQ, [None, d, None], [None, R, None], 0xFA11, 0, 200, counts, records=rec, exact=exact,
+                       site_masks=masks)
+    torch.cuda.synchronize()
+    g = hk.records_numpy(rec)
+    orr = [None, O.profile_ranges(O.MRIQ, p, exact=exact), None]
+    oc, o = O.campaign(O.MRIQ, [None, p, None], orr, 0xFA11, 0, 200, exact=exact, mode=0, site_masks=masks)
+    for k in ("site", "thread", "inst", "mask"):
+        assert np.array_equal(g[k], o[k]), k
+    assert set(g["site"]) <= set(range(29, 36))
+    if exact:
+        assert np.array_equal(g["cls"], o["cls"]) and np.array_equal(counts.cpu().numpy(), oc)
+    else:
+        amb = _ambiguous(g, o, [None, p, None])
+        assert not ((g["cls"] != o["cls"]) & ~amb).any()
+    # replay mode refuses PhiMag sites (they reach every voxel)
+    with pytest.raises(hk.HauberkError):
+        hk.inject_campaign(hk.HK_MRIQ, [None, d, None], [None, R, None], 1, 0, 10, counts, site_masks=masks, mode=1)

@@ -240,7 +240,7 @@ def test_every_nl_def_flip_is_detected_by_the_duplicate(bench):
     nl = [s for s in range(O.nsites(bench, getattr(p, "unroll", 1))) if O.site_info(bench, getattr(p, "unroll", 1), s)[0] == 0]
     for s in nl:
         for _ in range(3):
-            t = int(rng.integers(nthr)); b = int(rng.integers(32))
+            t = int(rng.integers(p.n_k if (bench == O.MRIQ and s >= 29) else nthr)); b = int(rng.integers(32))
             _, info = _one(bench, p, R, s, t, 0, 1 << b)
             assert info.fail or (info.alarm & O.AL_DUP), (s, t, b)
 
@@ -333,3 +333,29 @@ def test_replay_equals_replica_small_campaign(exact):
     for k in ("cls", "alarm", "fail", "site", "thread", "inst", "mask"):
         assert np.array_equal(r0[k], r1[k]), k
     assert c1.sum() == 240
+
+
+def test_phimag_fault_reaches_every_voxel_and_nl_detects_it():
+    p = W.mriq_problem(4, 19, n_vox=40, seed=8)
+    R = O.profile_ranges(O.MRIQ, p)
+    golden = O.run(O.MRIQ, p, flags=O.FT, ranges=R, ndet=1)[0]
+    # pm of PhiMag thread 5 (site 32): detected by its duplicate; every voxel's output changes
+    (qr, qi), _, info = O.run(O.MRIQ, p, flags=O.FT, ranges=R, ndet=1, f=O.fault(32, 5, 0, 1 << 28))
+    assert info.applied and info.alarm & O.AL_DUP
+    assert np.count_nonzero(qr != golden[0]) > 0.9 * p.n_vox
+    # kidx flipped out of range: modelled crash (R16)
+    _, _, info = O.run(O.MRIQ, p, flags=O.FT, ranges=R, ndet=1, f=O.fault(29, 3, 0, 1 << 20))
+    assert info.fail & O.FL_CRASH
+    # kidx flipped onto another slot: additive kv (R18) -> two k-samples in one slot, one slot empty
+    (qr2, _), _, info = O.run(O.MRIQ, p, flags=O.FT, ranges=R, ndet=1, f=O.fault(29, 2, 0, 1 << 0))
+    assert not info.fail and info.alarm & O.AL_DUP and not np.array_equal(qr2, golden[0])
+
+
+def test_phimag_sites_are_replica_only_in_the_oracle_campaign():
+    p = W.mriq_problem(4, 19, n_vox=40, seed=8)
+    R = [None, O.profile_ranges(O.MRIQ, p), None]
+    masks = (O.ALL_SITES, O.MRIQ_PHIMAG_SITES, O.ALL_SITES)
+    c1, r1 = O.campaign(O.MRIQ, [None, p, None], R, 99, 0, 60, mode=1, site_masks=masks)
+    c0, r0 = O.campaign(O.MRIQ, [None, p, None], R, 99, 0, 60, mode=0, site_masks=masks)
+    assert np.array_equal(c0, c1) and set(r1["site"]) <= set(range(29, 36))
+    assert (r1["thread"] < p.n_k).all()

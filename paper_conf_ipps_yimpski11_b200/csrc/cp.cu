@@ -355,11 +355,10 @@ struct CPReplayParams {
   int64_t* site_counts;
 };
 
-template <int KIND, bool EXACT>
+template <int KIND, int U, bool EXACT>
 __global__ void __launch_bounds__(128) cp_replay_kernel(const CPReplayParams q) {
   const int r = blockIdx.x * blockDim.x + threadIdx.x;
   if (r >= q.nrep) return;
-  constexpr int U = 4;
   const FaultRec f = q.faults[r];
   const CPGeo G = cp_geo_of(f.thread, q.BX, q.BY, q.gx, q.gy);
   ReplaySinkF<U> S;
@@ -462,18 +461,18 @@ int cp_site_kind(int site, int U, int* sub) {
   return CK_IT;
 }
 
-template <int KIND, bool EXACT>
+template <int KIND, int U, bool EXACT>
 static cudaError_t launch_cp_fi_k(const CPFIParams& q, dim3 grid, dim3 block, cudaStream_t s) {
-  TimedScope ts(HK_CP, 1, (double)q.base.numatoms * (double)q.base.nthreads * 4 * grid.z, s);
-  cp_fi_kernel<KIND, 4, EXACT><<<grid, block, 0, s>>>(q);
+  TimedScope ts(HK_CP, 1, (double)q.base.numatoms * (double)q.base.nthreads * U * grid.z, s);
+  cp_fi_kernel<KIND, U, EXACT><<<grid, block, 0, s>>>(q);
   count_launch();
   return cudaGetLastError();
 }
 
-template <bool EXACT>
+template <int U, bool EXACT>
 static cudaError_t launch_cp_fi_e(int kind, const CPFIParams& q, dim3 grid, dim3 block, cudaStream_t s) {
   switch (kind) {
-#define K(k) case k: return launch_cp_fi_k<k, EXACT>(q, grid, block, s);
+#define K(k) case k: return launch_cp_fi_k<k, U, EXACT>(q, grid, block, s);
     K(CK_NL) K(CK_LIVE) K(CK_ATOMID) K(CK_AX) K(CK_AY) K(CK_AZ) K(CK_AW) K(CK_DY) K(CK_DYZ2) K(CK_DX0)
     K(CK_DXJ) K(CK_R2) K(CK_S) K(CK_E) K(CK_IT)
 #undef K
@@ -497,21 +496,24 @@ cudaError_t cp_fi_launch(int kind, const hk_cp_args& a, const DevRanges& R, int 
   q.grid_elems = stride;
   q.grid0 = grid0;
   q.cb0 = cb0;
-  dim3 block(a.bx, a.by), grid(a.nx / (a.bx * 4), a.ny / a.by, nrep);
-  return a.exact ? launch_cp_fi_e<true>(kind, q, grid, block, s) : launch_cp_fi_e<false>(kind, q, grid, block, s);
+  dim3 block(a.bx, a.by), grid(a.nx / (a.bx * a.unroll), a.ny / a.by, nrep);
+  if (a.unroll == 8)
+    return a.exact ? launch_cp_fi_e<8, true>(kind, q, grid, block, s) : launch_cp_fi_e<8, false>(kind, q, grid, block, s);
+  if (a.unroll != 4) return cudaErrorInvalidValue;
+  return a.exact ? launch_cp_fi_e<4, true>(kind, q, grid, block, s) : launch_cp_fi_e<4, false>(kind, q, grid, block, s);
 }
 
-template <int KIND, bool EXACT>
+template <int KIND, int U, bool EXACT>
 static cudaError_t launch_cp_replay_k(const CPReplayParams& q, cudaStream_t s) {
-  TimedScope ts(HK_CP, 2, (double)q.base.numatoms * 4 * q.nrep, s);
-  cp_replay_kernel<KIND, EXACT><<<(q.nrep + 127) / 128, 128, 0, s>>>(q);
+  TimedScope ts(HK_CP, 2, (double)q.base.numatoms * U * q.nrep, s);
+  cp_replay_kernel<KIND, U, EXACT><<<(q.nrep + 127) / 128, 128, 0, s>>>(q);
   count_launch();
   return cudaGetLastError();
 }
-template <bool EXACT>
+template <int U, bool EXACT>
 static cudaError_t launch_cp_replay_e(int kind, const CPReplayParams& q, cudaStream_t s) {
   switch (kind) {
-#define K(k) case k: return launch_cp_replay_k<k, EXACT>(q, s);
+#define K(k) case k: return launch_cp_replay_k<k, U, EXACT>(q, s);
     K(CK_NL) K(CK_LIVE) K(CK_ATOMID) K(CK_AX) K(CK_AY) K(CK_AZ) K(CK_AW) K(CK_DY) K(CK_DYZ2) K(CK_DX0)
     K(CK_DXJ) K(CK_R2) K(CK_S) K(CK_E) K(CK_IT)
 #undef K
@@ -534,10 +536,12 @@ cudaError_t cp_replay_launch(int kind, const hk_cp_args& a, const DevRanges& R, 
   q.base.nthreads = (int64_t)(a.nx / a.unroll) * a.ny;
   q.faults = faults;
   q.nrep = nrep;
-  q.BX = a.bx; q.BY = a.by; q.gx = a.nx / (a.bx * 4); q.gy = a.ny / a.by;
+  q.BX = a.bx; q.BY = a.by; q.gx = a.nx / (a.bx * a.unroll); q.gy = a.ny / a.by;
   q.bench = HK_CP;
   q.golden = golden; q.dM = dM; q.records = records; q.first = first; q.counts = counts; q.site_counts = site_counts;
-  return a.exact ? launch_cp_replay_e<true>(kind, q, s) : launch_cp_replay_e<false>(kind, q, s);
+  if (a.unroll == 8) return a.exact ? launch_cp_replay_e<8, true>(kind, q, s) : launch_cp_replay_e<8, false>(kind, q, s);
+  if (a.unroll != 4) return cudaErrorInvalidValue;
+  return a.exact ? launch_cp_replay_e<4, true>(kind, q, s) : launch_cp_replay_e<4, false>(kind, q, s);
 }
 
 cudaError_t cp_prepass_launch(const hk_cp_args& a, cudaStream_t s) {

@@ -599,8 +599,8 @@ static hk_status session_create(int32_t bench_mode, const void* const args[3], c
     if (!want) continue;
     if (!args_ok(b, args[b])) { st = invalid("campaign: args of a used benchmark are invalid"); break; }
     if (!ranges[b] || ranges[b]->n_det <= 0) { g_err = "campaign: ranges missing"; st = HK_ERR_NO_RANGES; break; }
-    if (b == HK_CP && ((const hk_cp_args*)args[b])->unroll != 4) {
-      g_err = "campaign kernels are built for CP unroll 4"; st = HK_ERR_UNSUPPORTED; break;
+    if (b == HK_CP && ((const hk_cp_args*)args[b])->unroll != 4 && ((const hk_cp_args*)args[b])->unroll != 8) {
+      g_err = "campaign kernels are built for CP unroll 4 and 8"; st = HK_ERR_UNSUPPORTED; break;
     }
     if (b == HK_TPACF && !tpacf_edges_ok((const hk_tpacf_args*)args[b], s)) { st = invalid("edges must strictly decrease"); break; }
     const void* own = b == HK_CP ? (const void*)&S->cp : (b == HK_MRIQ ? (const void*)&S->mq : (const void*)&S->tp);
@@ -700,7 +700,7 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
     it.b = b;
     it.f.index = n; it.f.thread = hf.thread; it.f.inst = hf.inst; it.f.mask = hf.mask; it.f.site = hf.site;
     int sub = 0;
-    if (b == HK_CP) it.kind = cp_site_kind(hf.site, 4, &sub);
+    if (b == HK_CP) it.kind = cp_site_kind(hf.site, S->cp.unroll, &sub);
     else if (b == HK_MRIQ) it.kind = mriq_site_kind(hf.site);
     else it.kind = tpacf_site_kind(hf.site);
     it.f.sub = sub;
@@ -740,7 +740,7 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
       const int nrep = (int)(end - q);
       BenchWS& w = S->W[b];
       const FaultRec* fr = S->d_faults + q;
-      if (b == HK_CP) e = cp_replay_launch(kind, S->cp, w.R, std::min(w.ndet, 4), fr, nrep, (const float*)w.golden, w.dM,
+      if (b == HK_CP) e = cp_replay_launch(kind, S->cp, w.R, std::min(w.ndet, S->cp.unroll), fr, nrep, (const float*)w.golden, w.dM,
                                            d_records, first, d_counts, d_site_counts, s);
       else if (b == HK_MRIQ) e = mriq_replay_launch(kind, S->mq, w.R, std::min(w.ndet, 2), fr, nrep, (const float*)w.golden,
                                                     w.dM, d_records, first, d_counts, d_site_counts, s);
@@ -762,7 +762,7 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
     BenchWS& w = S->W[b];
     const FaultRec* fr = S->d_faults + q;
     if (b == HK_CP) {
-      if ((e = cp_fi_launch(kind, S->cp, w.R, std::min(w.ndet, 4), fr, nrep, (float*)w.rep_out, w.out_elems, w.rep_cb, s)) != cudaSuccess)
+      if ((e = cp_fi_launch(kind, S->cp, w.R, std::min(w.ndet, S->cp.unroll), fr, nrep, (float*)w.rep_out, w.out_elems, w.rep_cb, s)) != cudaSuccess)
         return cuda_fail(e, "cp FI");
       if ((e = classify_fp_launch(b, (float*)w.rep_out, w.out_elems, (const float*)w.golden, w.dM, w.rep_cb, fr, nrep,
                                   d_records, first, d_counts, d_site_counts, s)) != cudaSuccess)

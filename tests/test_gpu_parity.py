@@ -475,3 +475,19 @@ def test_phimag_site_replicas_vs_oracle_replicas(exact):
     # replay mode refuses PhiMag sites (they reach every voxel)
     with pytest.raises(hk.HauberkError):
         hk.inject_campaign(hk.HK_MRIQ, [None, d, None], [None, R, None], 1, 0, 10, counts, site_masks=masks, mode=1)
+
+
+@pytest.mark.parametrize("mode", [0, 1])
+def test_cp_unroll8_campaign_exact(mode):
+    p = W.cp_problem(29, 128, 16, seed=31, bx=8, by=8, unroll=8)
+    d = _mk(0, p, 1)
+    R = hk.profile_ranges(d, maxvar=2)
+    counts = torch.zeros((3, 5), dtype=torch.int64, device=DEV)
+    rec = hk.records_tensor(500, DEV)
+    hk.inject_campaign(hk.HK_CP, [d, None, None], [R, None, None], 0x88, 0, 500, counts, records=rec, exact=1, mode=mode)
+    torch.cuda.synchronize()
+    orr = [O.profile_ranges(O.CP, p, maxvar=2, exact=1), None, None]
+    oc, o = O.campaign(O.CP, [p, None, None], orr, 0x88, 0, 500, exact=1, mode=1)
+    g = hk.records_numpy(rec)
+    assert np.array_equal(g["site"], o["site"]) and np.array_equal(g["cls"], o["cls"])
+    assert np.array_equal(counts.cpu().numpy(), oc)

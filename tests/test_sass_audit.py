@@ -82,7 +82,7 @@ def test_tpacf_ft_keeps_detectors(sass):
 
 
 def test_fi_kernels_compiled_for_every_site_kind(sass):
-    assert len([n for n in sass if "cp_fi_kernel" in n]) == 15 * 2
+    assert len([n for n in sass if "cp_fi_kernel" in n]) == 15 * 2 * 2  # kinds x {FAST, EXACT} x U {4, 8}
     assert len([n for n in sass if "mriq_fi_kernel" in n]) == 17 * 2  # 16 Q-kernel kinds + PhiMag
     assert len([n for n in sass if "tpacf_fi_kernel" in n]) == 11
 

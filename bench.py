@@ -357,7 +357,7 @@ def main():
                   "injections_per_s": round(args.replay_count * world / (float(tr.item()) * 1e-3), 1),
                   "host_wall_s": round(t_host, 3), "coverage_pct": round(100.0 * hk.coverage(crn), 3),
                   "outcomes": {hk.BENCH_NAMES[b]: dict(zip(hk.CLASS_NAMES, crn[b].tolist())) for b in range(3)},
-                  "note": "config-5 campaign indices [0, N) in replay mode; timed region includes the host decode"}
+                  "note": "config-5 campaign indices [0, N) in replay mode; decode + counting sort by site kind on the device, then one launch per benchmark"}
 
     # ---- coverage vs number of flipped bits (Fig. 14; NEXT f1): the same
     #      injection indices with k-bit masks (untimed)

@@ -353,13 +353,11 @@ struct CPReplayParams {
   int64_t first;
   int64_t* counts;
   int64_t* site_counts;
+  uint8_t kind_of_site[64];
 };
 
 template <int KIND, int U, bool EXACT>
-__global__ void __launch_bounds__(128) cp_replay_kernel(const CPReplayParams q) {
-  const int r = blockIdx.x * blockDim.x + threadIdx.x;
-  if (r >= q.nrep) return;
-  const FaultRec f = q.faults[r];
+__device__ __forceinline__ void cp_replay_one(const CPReplayParams& q, const FaultRec& f) {
   const CPGeo G = cp_geo_of(f.thread, q.BX, q.BY, q.gx, q.gy);
   ReplaySinkF<U> S;
   cp_fi_program<KIND, U, EXACT>(q.base, f, G, true, (uint64_t)(uintptr_t)q.golden, S);
@@ -392,6 +390,22 @@ __global__ void __launch_bounds__(128) cp_replay_kernel(const CPReplayParams q) 
   }
   emit_outcome(q.bench, f, wrong, S.alarm, S.fail, S.domain, S.margin, S.gap, worst, q.records, q.first, q.counts,
                q.site_counts);
+}
+
+// One CUDA thread per injection; the records arrive sorted by site kind (decode.cu), so warps
+// take one branch of the switch.
+template <int U, bool EXACT>
+__global__ void __launch_bounds__(128) cp_replay_all_kernel(const CPReplayParams q) {
+  const int r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= q.nrep) return;
+  const FaultRec f = q.faults[r];
+  switch (q.kind_of_site[f.site & 63]) {
+#define K(k) case k: cp_replay_one<k, U, EXACT>(q, f); break;
+    K(CK_NL) K(CK_LIVE) K(CK_ATOMID) K(CK_AX) K(CK_AY) K(CK_AZ) K(CK_AW) K(CK_DY) K(CK_DYZ2) K(CK_DX0)
+    K(CK_DXJ) K(CK_R2) K(CK_S) K(CK_E) K(CK_IT)
+#undef K
+    default: break;
+  }
 }
 
 // ============================================================================================
@@ -503,24 +517,6 @@ cudaError_t cp_fi_launch(int kind, const hk_cp_args& a, const DevRanges& R, int 
   return a.exact ? launch_cp_fi_e<4, true>(kind, q, grid, block, s) : launch_cp_fi_e<4, false>(kind, q, grid, block, s);
 }
 
-template <int KIND, int U, bool EXACT>
-static cudaError_t launch_cp_replay_k(const CPReplayParams& q, cudaStream_t s) {
-  TimedScope ts(HK_CP, 2, (double)q.base.numatoms * U * q.nrep, s);
-  cp_replay_kernel<KIND, U, EXACT><<<(q.nrep + 127) / 128, 128, 0, s>>>(q);
-  count_launch();
-  return cudaGetLastError();
-}
-template <int U, bool EXACT>
-static cudaError_t launch_cp_replay_e(int kind, const CPReplayParams& q, cudaStream_t s) {
-  switch (kind) {
-#define K(k) case k: return launch_cp_replay_k<k, U, EXACT>(q, s);
-    K(CK_NL) K(CK_LIVE) K(CK_ATOMID) K(CK_AX) K(CK_AY) K(CK_AZ) K(CK_AW) K(CK_DY) K(CK_DYZ2) K(CK_DX0)
-    K(CK_DXJ) K(CK_R2) K(CK_S) K(CK_E) K(CK_IT)
-#undef K
-  }
-  return cudaErrorInvalidValue;
-}
-
 cudaError_t cp_replay_launch(int kind, const hk_cp_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
                              const float* golden, const float* dM, hk_outcome* records, int64_t first, int64_t* counts,
                              int64_t* site_counts, cudaStream_t s) {
@@ -539,9 +535,24 @@ cudaError_t cp_replay_launch(int kind, const hk_cp_args& a, const DevRanges& R, 
   q.BX = a.bx; q.BY = a.by; q.gx = a.nx / (a.bx * a.unroll); q.gy = a.ny / a.by;
   q.bench = HK_CP;
   q.golden = golden; q.dM = dM; q.records = records; q.first = first; q.counts = counts; q.site_counts = site_counts;
-  if (a.unroll == 8) return a.exact ? launch_cp_replay_e<8, true>(kind, q, s) : launch_cp_replay_e<8, false>(kind, q, s);
-  if (a.unroll != 4) return cudaErrorInvalidValue;
-  return a.exact ? launch_cp_replay_e<4, true>(kind, q, s) : launch_cp_replay_e<4, false>(kind, q, s);
+  for (int site = 0; site < 64; ++site) {
+    int sub = 0;
+    q.kind_of_site[site] = (uint8_t)cp_site_kind(site, a.unroll, &sub);
+  }
+  (void)kind;
+  const unsigned g = (unsigned)((nrep + 127) / 128);
+  TimedScope ts(HK_CP, 2, (double)a.n_atoms * a.unroll * nrep, s);
+  if (a.unroll == 8) {
+    if (a.exact) cp_replay_all_kernel<8, true><<<g, 128, 0, s>>>(q);
+    else cp_replay_all_kernel<8, false><<<g, 128, 0, s>>>(q);
+  } else if (a.unroll == 4) {
+    if (a.exact) cp_replay_all_kernel<4, true><<<g, 128, 0, s>>>(q);
+    else cp_replay_all_kernel<4, false><<<g, 128, 0, s>>>(q);
+  } else {
+    return cudaErrorInvalidValue;
+  }
+  count_launch();
+  return cudaGetLastError();
 }
 
 cudaError_t cp_prepass_launch(const hk_cp_args& a, cudaStream_t s) {

@@ -40,6 +40,16 @@ struct FaultRec {
   int32_t sub;
 };
 
+// Site catalogue of one benchmark for the device decode (DESIGN R14): enabled sites, per-site
+// class/width/kind/sub, thread and instance counts, and the TPACF trip prefix sums.
+struct DevCatalog {
+  int32_t nen, pad;
+  int32_t en[64];
+  uint8_t is_nl[64], width[64], kind[64], sub[64];
+  int64_t nthr, nk, uniform_trips, total_trips;
+  const int64_t* prefix;
+};
+
 __device__ __forceinline__ uint32_t fb(float f) { return __float_as_uint(f); }
 __device__ __forceinline__ float bf(uint32_t u) { return __uint_as_float(u); }
 __device__ __forceinline__ uint32_t lohi(uint64_t p) { return (uint32_t)p ^ (uint32_t)(p >> 32); }

@@ -59,6 +59,11 @@ cudaError_t tpacf_replay_launch(int kind, const hk_tpacf_args& a, const DevRange
                                 int nrep, const unsigned long long* golden, hk_outcome* records, int64_t first,
                                 int64_t* counts, int64_t* site_counts, cudaStream_t s);
 
+// decode.cu: device decode + counting sort by (bench, kind) for the replay path
+size_t decode_ws_bytes(int64_t count);
+cudaError_t decode_sort_launch(const DevCatalog cat[3], uint64_t seed, int64_t first, int64_t count, int32_t bench_mode,
+                               int32_t nbits, void* ws, FaultRec** sorted_out, cudaStream_t s);
+
 // classify.cu
 cudaError_t control_init_launch(hk_control* cb, int n, cudaStream_t s);
 cudaError_t max_abs_launch(const float* g, int64_t n, float* d_out, cudaStream_t s);

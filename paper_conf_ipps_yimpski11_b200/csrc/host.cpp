@@ -536,6 +536,10 @@ hk_status hauberk_decode(int32_t bench_mode, const void* const args[3], const ui
 // hauberk_campaign_run enqueues one slice of injections without synchronising.
 // ---------------------------------------------------------------------------------------------
 struct hk_campaign_session {
+  DevCatalog dcat[3]{};
+  int64_t* d_prefix = nullptr;  // TPACF trip prefix sums on the device (replay decode)
+  void* d_decode = nullptr;
+  size_t decode_cap = 0;
   int bench_mode = -1;
   hk_campaign cfg{};
   hk_cp_args cp{};
@@ -566,6 +570,8 @@ static void session_free(hk_campaign_session* S) {
   }
   if (S->d_faults) cudaFree(S->d_faults);
   if (S->h_faults) cudaFreeHost(S->h_faults);
+  if (S->d_prefix) cudaFree(S->d_prefix);
+  if (S->d_decode) cudaFree(S->d_decode);
   if (S->uploaded) cudaEventDestroy(S->uploaded);
   delete S;
 }
@@ -677,6 +683,33 @@ static hk_status session_create(int32_t bench_mode, const void* const args[3], c
   }
   if (st == HK_OK && (e = cudaEventCreateWithFlags(&S->uploaded, cudaEventDisableTiming)) != cudaSuccess)
     st = cuda_fail(e, "event");
+  // device catalogues for the replay path's on-device decode
+  for (int b = 0; b < 3 && st == HK_OK; ++b) {
+    if (!S->W[b].used) continue;
+    const Catalog& K = S->K[b];
+    DevCatalog& D = S->dcat[b];
+    D.nen = (int)K.enabled.size();
+    for (int q = 0; q < D.nen; ++q) D.en[q] = K.enabled[q];
+    const int U = b == HK_CP ? S->cp.unroll : 1;
+    for (int site = 0; site < 64 && site < num_sites(b, U); ++site) {
+      int sub = 0, kind = 0;
+      if (b == HK_CP) kind = cp_site_kind(site, U, &sub);
+      else if (b == HK_MRIQ) kind = mriq_site_kind(site);
+      else kind = tpacf_site_kind(site);
+      D.is_nl[site] = site_is_nl(b, site) ? 1 : 0;
+      D.width[site] = (uint8_t)site_width(b, site);
+      D.kind[site] = (uint8_t)kind;
+      D.sub[site] = (uint8_t)sub;
+    }
+    D.nthr = K.nthr; D.nk = K.nk; D.uniform_trips = K.uniform_trips; D.total_trips = K.total_trips;
+    D.prefix = nullptr;
+    if (!K.prefix.empty()) {
+      if ((e = cudaMalloc((void**)&S->d_prefix, sizeof(int64_t) * K.prefix.size())) != cudaSuccess ||
+          (e = cudaMemcpy(S->d_prefix, K.prefix.data(), sizeof(int64_t) * K.prefix.size(), cudaMemcpyHostToDevice)) != cudaSuccess)
+        st = cuda_fail(e, "prefix");
+      D.prefix = S->d_prefix;
+    }
+  }
   if (st != HK_OK) { session_free(S); return st; }
   *out = S;
   return HK_OK;
@@ -688,7 +721,47 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
   if (count == 0) return HK_OK;
   cudaStream_t s = S->stream;
   cudaError_t e;
-  // ---- decode, group by (bench, kind)
+  if (S->cfg.mode == 1) {
+    // ---- replay: decode and sort on the device, then one launch per benchmark (no host round trip)
+    int64_t per[3] = {0, 0, 0};
+    if (S->bench_mode >= 0) per[S->bench_mode] = count;
+    else
+      for (int b = 0; b < 3; ++b) {
+        const int64_t off = (b - first % 3 + 3) % 3;
+        per[b] = count > off ? (count - off + 2) / 3 : 0;
+      }
+    for (int b = 0; b < 3; ++b)
+      if (per[b] && !S->W[b].used) return invalid("campaign_run: index hits a benchmark the session was not created with");
+    const size_t need = decode_ws_bytes(count);
+    if (S->decode_cap < need) {
+      if (S->d_decode) cudaFreeAsync(S->d_decode, s);
+      S->d_decode = nullptr;
+      S->decode_cap = 0;
+      if ((e = cudaMallocAsync(&S->d_decode, need, s)) != cudaSuccess) return cuda_fail(e, "decode workspace");
+      S->decode_cap = need;
+    }
+    FaultRec* sorted = nullptr;
+    if ((e = decode_sort_launch(S->dcat, S->cfg.seed, first, count, S->bench_mode, S->cfg.nbits, S->d_decode, &sorted, s)) !=
+        cudaSuccess)
+      return cuda_fail(e, "device decode");
+    int64_t off = 0;
+    for (int b = 0; b < 3; ++b) {
+      if (!per[b]) continue;
+      BenchWS& w = S->W[b];
+      const FaultRec* fr = sorted + off;
+      const int nrep = (int)per[b];
+      if (b == HK_CP) e = cp_replay_launch(0, S->cp, w.R, std::min(w.ndet, S->cp.unroll), fr, nrep, (const float*)w.golden,
+                                           w.dM, d_records, first, d_counts, d_site_counts, s);
+      else if (b == HK_MRIQ) e = mriq_replay_launch(0, S->mq, w.R, std::min(w.ndet, 2), fr, nrep, (const float*)w.golden,
+                                                    w.dM, d_records, first, d_counts, d_site_counts, s);
+      else e = tpacf_replay_launch(0, S->tp, w.R, std::min(w.ndet, 1), fr, nrep, (const unsigned long long*)w.golden,
+                                   d_records, first, d_counts, d_site_counts, s);
+      if (e != cudaSuccess) return cuda_fail(e, "replay");
+      off += per[b];
+    }
+    return HK_OK;
+  }
+  // ---- replica: decode on the host, group by (bench, kind)
   struct Item { int b, kind; FaultRec f; };
   std::vector<Item> items((size_t)count);
   for (int64_t q = 0; q < count; ++q) {
@@ -729,28 +802,6 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
   if ((e = cudaMemcpyAsync(S->d_faults, S->h_faults, sizeof(FaultRec) * items.size(), cudaMemcpyHostToDevice, s)) != cudaSuccess)
     return cuda_fail(e, "upload faults");
   cudaEventRecord(S->uploaded, s);
-
-  // ---- replay mode: one launch per (benchmark, kind) group, one CUDA thread per injection
-  if (S->cfg.mode == 1) {
-    size_t q = 0;
-    while (q < items.size()) {
-      const int b = items[q].b, kind = items[q].kind;
-      size_t end = q;
-      while (end < items.size() && items[end].b == b && items[end].kind == kind) ++end;
-      const int nrep = (int)(end - q);
-      BenchWS& w = S->W[b];
-      const FaultRec* fr = S->d_faults + q;
-      if (b == HK_CP) e = cp_replay_launch(kind, S->cp, w.R, std::min(w.ndet, S->cp.unroll), fr, nrep, (const float*)w.golden, w.dM,
-                                           d_records, first, d_counts, d_site_counts, s);
-      else if (b == HK_MRIQ) e = mriq_replay_launch(kind, S->mq, w.R, std::min(w.ndet, 2), fr, nrep, (const float*)w.golden,
-                                                    w.dM, d_records, first, d_counts, d_site_counts, s);
-      else e = tpacf_replay_launch(kind, S->tp, w.R, std::min(w.ndet, 1), fr, nrep, (const unsigned long long*)w.golden,
-                                   d_records, first, d_counts, d_site_counts, s);
-      if (e != cudaSuccess) return cuda_fail(e, "replay");
-      q = end;
-    }
-    return HK_OK;
-  }
 
   // ---- batches: FI&FT replicas, then the classify epilogue (which also recycles the workspace)
   size_t q = 0;

@@ -192,6 +192,13 @@ enum MQKind : int {
   MK_COUNT
 };
 
+__host__ __device__ __forceinline__ int mriq_site_kind_d(int site) {
+  if (site <= 3) return MK_NL;
+  if (site <= 14) return MK_LIVE;
+  if (site >= 29) return MK_PHIMAG;
+  return MK_K + (site - 15);
+}
+
 struct MQFIParams {
   MQParams base;
   const FaultRec* faults;
@@ -414,10 +421,7 @@ struct MQReplayParams {
 };
 
 template <int KIND, bool EXACT>
-__global__ void __launch_bounds__(128) mriq_replay_kernel(const MQReplayParams q) {
-  const int r = blockIdx.x * blockDim.x + threadIdx.x;
-  if (r >= q.nrep) return;
-  const FaultRec f = q.faults[r];
+__device__ __forceinline__ void mriq_replay_one(const MQReplayParams& q, const FaultRec& f) {
   const MQParams& p = q.base;
   const int32_t t = (int32_t)f.thread;
   ReplaySinkF<2> S;
@@ -446,6 +450,20 @@ __global__ void __launch_bounds__(128) mriq_replay_kernel(const MQReplayParams q
   }
   emit_outcome(HK_MRIQ, f, wrong, S.alarm, S.fail, S.domain, S.margin, S.gap, worst, q.records, q.first, q.counts,
                q.site_counts);
+}
+
+template <bool EXACT>
+__global__ void __launch_bounds__(128) mriq_replay_all_kernel(const MQReplayParams q) {
+  const int r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= q.nrep) return;
+  const FaultRec f = q.faults[r];
+  switch (mriq_site_kind_d(f.site)) {
+#define K(k) case k: mriq_replay_one<k, EXACT>(q, f); break;
+    K(MK_NL) K(MK_LIVE) K(MK_K) K(MK_KX) K(MK_KY) K(MK_KZ) K(MK_PM) K(MK_T1) K(MK_T2) K(MK_T) K(MK_R) K(MK_C) K(MK_S)
+    K(MK_QR) K(MK_QI) K(MK_IT)
+#undef K
+    default: break;
+  }
 }
 
 // ============================================================================================
@@ -499,12 +517,7 @@ cudaError_t mriq_launch(int vflags, const hk_mriq_args& a, const DevRanges& R, i
   return cudaErrorInvalidValue;
 }
 
-int mriq_site_kind(int site) {
-  if (site <= 3) return MK_NL;
-  if (site <= 14) return MK_LIVE;
-  if (site >= 29) return MK_PHIMAG;
-  return MK_K + (site - 15);
-}
+int mriq_site_kind(int site) { return mriq_site_kind_d(site); }
 
 template <int KIND, bool EXACT>
 static cudaError_t launch_mq_fi_k(const MQFIParams& q, int nrep, cudaStream_t s) {
@@ -526,24 +539,6 @@ static cudaError_t launch_mq_fi_e(int kind, const MQFIParams& q, int nrep, cudaS
   return cudaErrorInvalidValue;
 }
 
-template <int KIND, bool EXACT>
-static cudaError_t launch_mq_replay_k(const MQReplayParams& q, cudaStream_t s) {
-  TimedScope ts(HK_MRIQ, 2, (double)q.base.numK * q.nrep, s);
-  mriq_replay_kernel<KIND, EXACT><<<(q.nrep + 127) / 128, 128, 0, s>>>(q);
-  count_launch();
-  return cudaGetLastError();
-}
-template <bool EXACT>
-static cudaError_t launch_mq_replay_e(int kind, const MQReplayParams& q, cudaStream_t s) {
-  switch (kind) {
-#define K(k) case k: return launch_mq_replay_k<k, EXACT>(q, s);
-    K(MK_NL) K(MK_LIVE) K(MK_K) K(MK_KX) K(MK_KY) K(MK_KZ) K(MK_PM) K(MK_T1) K(MK_T2) K(MK_T) K(MK_R) K(MK_C) K(MK_S)
-    K(MK_QR) K(MK_QI) K(MK_IT)
-#undef K
-  }
-  return cudaErrorInvalidValue;
-}
-
 cudaError_t mriq_replay_launch(int kind, const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
                                int nrep, const float* golden, const float* dM, hk_outcome* records, int64_t first,
                                int64_t* counts, int64_t* site_counts, cudaStream_t s) {
@@ -553,7 +548,13 @@ cudaError_t mriq_replay_launch(int kind, const hk_mriq_args& a, const DevRanges&
   q.faults = faults;
   q.nrep = nrep;
   q.golden = golden; q.dM = dM; q.records = records; q.first = first; q.counts = counts; q.site_counts = site_counts;
-  return a.exact ? launch_mq_replay_e<true>(kind, q, s) : launch_mq_replay_e<false>(kind, q, s);
+  (void)kind;
+  TimedScope ts(HK_MRIQ, 2, (double)a.n_k * nrep, s);
+  const unsigned g = (unsigned)((nrep + 127) / 128);
+  if (a.exact) mriq_replay_all_kernel<true><<<g, 128, 0, s>>>(q);
+  else mriq_replay_all_kernel<false><<<g, 128, 0, s>>>(q);
+  count_launch();
+  return cudaGetLastError();
 }
 
 cudaError_t mriq_fi_launch(int kind, const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,

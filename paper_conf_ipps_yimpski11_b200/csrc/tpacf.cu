@@ -569,16 +569,10 @@ struct TPReplayParams {
 };
 
 template <int KIND>
-__global__ void __launch_bounds__(128) tpacf_replay_kernel(const TPReplayParams q) {
-  __shared__ float Es[32];
+__device__ __forceinline__ void tpacf_replay_one(const TPReplayParams& q, const FaultRec& f, float* Es) {
   const TPParams& p = q.base;
-  if (threadIdx.x < 32) Es[threadIdx.x] = threadIdx.x <= p.nb ? p.edges[threadIdx.x] : __int_as_float(0xff800000);
-  __syncthreads();
-  const int r = blockIdx.x * blockDim.x + threadIdx.x;
-  if (r >= q.nrep) return;
   TPSmem S{};
   S.E = Es;
-  const FaultRec f = q.faults[r];
   const int32_t row = (int32_t)(f.thread / p.n), ii = (int32_t)(f.thread % p.n);
   int32_t delta[TP_REPLAY_OUT];
   for (int o = 0; o < 3 * p.nb; ++o) delta[o] = 0;
@@ -608,6 +602,28 @@ __global__ void __launch_bounds__(128) tpacf_replay_kernel(const TPReplayParams 
   }
   emit_outcome(HK_TPACF, f, wrong, K.alarm, K.fail, 0u, K.margin, K.gap, worst, q.records, q.first, q.counts,
                q.site_counts);
+}
+
+__host__ __device__ __forceinline__ int tpacf_site_kind_d(int site) {
+  if (site <= 11) return TK_NL;
+  if (site <= 21) return TK_LIVE;
+  return TK_J + (site - 22);
+}
+
+__global__ void __launch_bounds__(128) tpacf_replay_all_kernel(const TPReplayParams q) {
+  __shared__ float Es[32];
+  const TPParams& p = q.base;
+  if (threadIdx.x < 32) Es[threadIdx.x] = threadIdx.x <= p.nb ? p.edges[threadIdx.x] : __int_as_float(0xff800000);
+  __syncthreads();
+  const int r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= q.nrep) return;
+  const FaultRec f = q.faults[r];
+  switch (tpacf_site_kind_d(f.site)) {
+#define K(k) case k: tpacf_replay_one<k>(q, f, Es); break;
+    K(TK_NL) K(TK_LIVE) K(TK_J) K(TK_X2) K(TK_Y2) K(TK_Z2) K(TK_DOT) K(TK_BIN) K(TK_HIDX) K(TK_ACC) K(TK_CNT)
+#undef K
+    default: break;
+  }
 }
 
 // ============================================================================================
@@ -679,11 +695,7 @@ cudaError_t tpacf_launch(int vflags, const hk_tpacf_args& a, const DevRanges& R,
   return cudaErrorInvalidValue;
 }
 
-int tpacf_site_kind(int site) {
-  if (site <= 11) return TK_NL;
-  if (site <= 21) return TK_LIVE;
-  return TK_J + (site - 22);
-}
+int tpacf_site_kind(int site) { return tpacf_site_kind_d(site); }
 
 template <int KIND>
 static cudaError_t launch_tp_fi_k(const TPFIParams& q, int nrep, cudaStream_t s) {
@@ -693,14 +705,6 @@ static cudaError_t launch_tp_fi_k(const TPFIParams& q, int nrep, cudaStream_t s)
   dim3 grid((q.base.n + TP_CTA_PTS - 1) / TP_CTA_PTS, (1 + 2 * q.base.nr) * q.base.nC, nrep);
   TimedScope ts(HK_TPACF, 1, tp_pairs(q.base) * nrep, s);
   tpacf_fi_kernel<KIND><<<grid, TP_THREADS, smem, s>>>(q);
-  count_launch();
-  return cudaGetLastError();
-}
-
-template <int KIND>
-static cudaError_t launch_tp_replay_k(const TPReplayParams& q, cudaStream_t s) {
-  TimedScope ts(HK_TPACF, 2, (double)q.base.C * 2 * q.nrep, s);
-  tpacf_replay_kernel<KIND><<<(q.nrep + 127) / 128, 128, 0, s>>>(q);
   count_launch();
   return cudaGetLastError();
 }
@@ -715,12 +719,11 @@ cudaError_t tpacf_replay_launch(int kind, const hk_tpacf_args& a, const DevRange
   q.faults = faults;
   q.nrep = nrep;
   q.golden = golden; q.records = records; q.first = first; q.counts = counts; q.site_counts = site_counts;
-  switch (kind) {
-#define K(k) case k: return launch_tp_replay_k<k>(q, s);
-    K(TK_NL) K(TK_LIVE) K(TK_J) K(TK_X2) K(TK_Y2) K(TK_Z2) K(TK_DOT) K(TK_BIN) K(TK_HIDX) K(TK_ACC) K(TK_CNT)
-#undef K
-  }
-  return cudaErrorInvalidValue;
+  (void)kind;
+  TimedScope ts(HK_TPACF, 2, (double)q.base.C * 2 * nrep, s);
+  tpacf_replay_all_kernel<<<(nrep + 127) / 128, 128, 0, s>>>(q);
+  count_launch();
+  return cudaGetLastError();
 }
 
 // lut_ws must hold a table built by tpacf_lut_build for a.edges (the campaign builds it once).

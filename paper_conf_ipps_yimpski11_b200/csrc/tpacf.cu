@@ -27,7 +27,7 @@ struct TPParams {
   DevRanges R;
   int32_t n, nr, nb, C, nC, ndet;
   uint32_t z;
-  int32_t one;
+  int32_t one, four;  // runtime 1 and 4 (opaque)
 };
 
 // ---------------------------------------------------------------------------------------------
@@ -36,7 +36,12 @@ struct TPParams {
 //  * LUT path: u = fl(1 - dot) is monotone in dot, and so is bin; bucket u by its top 11 bits
 //    (sign, exponent, 2 mantissa bits).  For every bucket q the device builds
 //    bmin = bin(largest dot mapping into q) and checks that the smallest dot of q has
-//    bin <= bmin + 1, so bin = bmin + (dot < edge[bmin]) exactly.  2 loads + 4 ops per pair.
+//    bin <= bmin + 1, so bin = bmin + (dot < edge[bmin]) exactly.  The compare is taken as the
+//    sign bit of fl(dot - edge[bmin]) (one FADD + one shift-add): with gradual underflow the
+//    difference of two finite floats is zero only when they are equal, rounding never flips its
+//    sign, a NaN result is the canonical (positive) NaN and dot - (-inf) = +inf; the one
+//    disagreement, dot = -0 against an edge of +0, is removed by staging +0 edges as -0 (equal
+//    under every compare).  2 loads + 5 ops per pair.
 // ---------------------------------------------------------------------------------------------
 constexpr int TP_LUT = 2048;
 
@@ -49,7 +54,7 @@ __device__ __forceinline__ int32_t tp_bin(const float* Es, float dot) {
 __device__ __forceinline__ int32_t tp_bin_lut(const uint8_t* L, const float* Es, float dot) {
   const float u = __fsub_rn(1.0f, dot);
   const int32_t b = L[fb(u) >> 21];
-  return b + ((dot < Es[b]) ? 1 : 0);
+  return b + (int32_t)(fb(__fsub_rn(dot, Es[b])) >> 31);
 }
 
 __device__ __forceinline__ float nup(float x) {
@@ -129,7 +134,10 @@ __device__ __forceinline__ bool tp_cta_has_work(const TPParams& p, int h, int c)
 
 // Stage chunk c of partner set sb, the edges, the bucket table; clear the histograms.
 __device__ __forceinline__ void tp_stage(const TPParams& p, const TPSmem& S, int sb, int c, bool work) {
-  if (threadIdx.x < 32) S.E[threadIdx.x] = threadIdx.x <= p.nb ? p.edges[threadIdx.x] : __int_as_float(0xff800000);
+  if (threadIdx.x < 32) {  // +0 staged as -0 (tp_bin_lut); -inf pads past the last edge
+    const float e = threadIdx.x <= p.nb ? p.edges[threadIdx.x] : __int_as_float(0xff800000);
+    S.E[threadIdx.x] = fb(e) == 0u ? __int_as_float(0x80000000) : e;
+  }
   if (!work) return;
   const int j0 = c * p.C;
   const int cnt = min(p.C, p.n - j0);
@@ -238,7 +246,7 @@ template <bool LUT>
 __device__ __forceinline__ int32_t tp_binof(const uint8_t* __restrict__ L, const float* __restrict__ E, float dot) {
   return LUT ? tp_bin_lut(L, E, dot) : tp_bin(E, dot);
 }
-template <bool CNT>
+template <bool CNT, bool INC = true>
 __device__ __forceinline__ void tp_count(const TPParams& p, uint32_t* Hw, TPPoint& P, int32_t bin) {
   // lane-private counter: no contention; the shared-memory atomic (ATOMS.POPC.INC) has no
   // register round trip, so consecutive increments do not serialise (microbenchmark: 1.34x the
@@ -246,7 +254,7 @@ __device__ __forceinline__ void tp_count(const TPParams& p, uint32_t* Hw, TPPoin
   atomicAdd(Hw + bin * 32, 1u);
   if (CNT) {
     P.acc += bin;
-    P.cnt = count_inc(P.cnt, p.one);
+    if (INC) P.cnt = count_inc(P.cnt, p.one);
   }
 }
 
@@ -270,20 +278,30 @@ __device__ __forceinline__ void tp_loops(const TPParams& p, const TPSmem& S, uin
     for (int32_t j = jbb; j < je; ++j) tp_count<CNT>(p, Hw, B, tp_binof<LUT>(L, E, tp_dot(B, Bs[j])));
     return;
   }
-  // phase 2: both points, one shared partner load
+  // phase 2: both points, one shared partner load; the partner pointer walks the tile and the
+  // counters advance by 4 per group of 4 iterations (the strength reduction any compiler applies
+  // to an unrolled it++; the FI program keeps the per-iteration increment as the injection site)
   int32_t j = max(jbb, ja);
-  for (; j + 3 < je; j += 4) {
-    const float4 q0 = Bs[j], q1 = Bs[j + 1], q2 = Bs[j + 2], q3 = Bs[j + 3];
+  const float4* __restrict__ T = S.B;
+  const int32_t k0 = (int32_t)(Bs - S.B);  // -(c * C): tile index k = j + k0
+  int32_t k = j + k0;
+  const int32_t kend = je + k0;
+  for (; k + 3 < kend; k += 4) {
+    const float4 q0 = T[k], q1 = T[k + 1], q2 = T[k + 2], q3 = T[k + 3];
     const int32_t a0 = tp_binof<LUT>(L, E, tp_dot(A, q0)), b0 = tp_binof<LUT>(L, E, tp_dot(B, q0));
     const int32_t a1 = tp_binof<LUT>(L, E, tp_dot(A, q1)), b1 = tp_binof<LUT>(L, E, tp_dot(B, q1));
     const int32_t a2 = tp_binof<LUT>(L, E, tp_dot(A, q2)), b2 = tp_binof<LUT>(L, E, tp_dot(B, q2));
     const int32_t a3 = tp_binof<LUT>(L, E, tp_dot(A, q3)), b3 = tp_binof<LUT>(L, E, tp_dot(B, q3));
-    tp_count<CNT>(p, Hw, A, a0); tp_count<CNT>(p, Hw, B, b0);
-    tp_count<CNT>(p, Hw, A, a1); tp_count<CNT>(p, Hw, B, b1);
-    tp_count<CNT>(p, Hw, A, a2); tp_count<CNT>(p, Hw, B, b2);
-    tp_count<CNT>(p, Hw, A, a3); tp_count<CNT>(p, Hw, B, b3);
+    tp_count<CNT, false>(p, Hw, A, a0); tp_count<CNT, false>(p, Hw, B, b0);
+    tp_count<CNT, false>(p, Hw, A, a1); tp_count<CNT, false>(p, Hw, B, b1);
+    tp_count<CNT, false>(p, Hw, A, a2); tp_count<CNT, false>(p, Hw, B, b2);
+    tp_count<CNT, false>(p, Hw, A, a3); tp_count<CNT, false>(p, Hw, B, b3);
+    if (CNT) {
+      A.cnt = count_inc(A.cnt, p.four);
+      B.cnt = count_inc(B.cnt, p.four);
+    }
   }
-  for (; j < je; ++j) {
+  for (j = k - k0; j < je; ++j) {
     const float4 q = Bs[j];
     const int32_t a = tp_binof<LUT>(L, E, tp_dot(A, q)), b = tp_binof<LUT>(L, E, tp_dot(B, q));
     tp_count<CNT>(p, Hw, A, a);
@@ -648,6 +666,7 @@ static TPParams tp_params(const hk_tpacf_args& a, const DevRanges& R, int ndet, 
   p.ndet = ndet;
   p.z = opaque_zero();
   p.one = 1 + (int32_t)opaque_zero();
+  p.four = 4 * p.one;
   return p;
 }
 

@@ -317,6 +317,43 @@ def test_tpacf_bucket_binning_adversarial_dots():
     assert got[2].sum() == n * n
 
 
+def _bucket(x):
+    return int(np.array([x], dtype=np.float32).view(np.uint32)[0]) >> 21
+
+
+def test_tpacf_signed_zero_and_special_dots_against_a_zero_edge():
+    """The bucket-table path takes dot < edge as the sign of fl(dot - edge); the one
+    case where the two differ, dot = -0 against an edge of +0, and the non-finite dots must still
+    follow the count definition.  Data point (0, 0, 1) against partners (-1, -0, v) gives
+    dot = v + (-0) = v exactly, -0 included."""
+    e = np.array([0.9, 0.5, 0.2, 0.0, -0.3, -0.6, -0.95], dtype=np.float32)
+    u = (np.float32(1) - e).astype(np.float32)
+    assert len({_bucket(x) for x in u}) == len(u)  # one edge per u-bucket: the table path is taken
+    tiny = np.array([1e-45, 1e-40, 1e-38, 1e-30, 1e-7], dtype=np.float32)
+    v = [0.0, -0.0, np.inf, -np.inf, np.nan, 1.5, -1.5]
+    v += list(tiny) + list(-tiny)
+    for x in e:
+        b = np.array([x], dtype=np.float32).view(np.int32)[0]
+        v += list(np.arange(b - 3, b + 4, dtype=np.int32).view(np.float32))
+    v = np.array(v, dtype=np.float32)
+    v = v[np.argsort(np.array(v).view(np.uint32), kind="stable")]  # keep -0 and +0 apart
+    n = v.size
+    pts = np.zeros((2, n, 3), dtype=np.float32)
+    pts[0, :, 2] = 1.0
+    pts[1, :, 0] = -1.0
+    pts[1, :, 1] = -0.0
+    pts[1, :, 2] = v
+    p = W.TPACFProblem(pts=pts, edges=e, chunk=64)
+    d = _mk(2, p)
+    cb = hk.new_control(DEV)
+    hk.run(d, hk.HK_BASE, None, cb)
+    torch.cuda.synchronize()
+    got = _out_np(d)
+    ora, _, _ = O.run(O.TPACF, p, flags=0)
+    assert np.array_equal(got, ora)
+    assert got[2].sum() == n * n  # the DR row holds every (data, random) pair
+
+
 def test_campaign_session_matches_one_shot_calls():
     probs = [W.cp_small(), W.mriq_problem(4, 40, n_vox=64, seed=9), W.tpacf_small(n=64, n_rand=1, chunk=16)]
     devs = [_mk(b, probs[b]) for b in range(3)]

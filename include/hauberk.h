@@ -113,8 +113,11 @@ typedef struct { int32_t maxvar; int32_t t0_exp10; float alpha; } hk_profile_opt
  * reproduce Fig. 14's multi-bit masks, L2691); mode 0 = replica (every injection is a full program
  * run, the paper's definition), mode 1 = replay (one CUDA thread re-runs only the
  * faulted abstract thread and classifies the golden output patched with its writes — identical
- * outcomes; TPACF n_bins <= 32); batch = replicas per launch (0 = auto); site_mask[b]
- * bit s enables site s. */
+ * outcomes; TPACF n_bins <= 32), mode 2 = unguarded replica (DESIGN R25, SURVEY
+ * §8 f4: the faulted thread dereferences corrupted addresses itself and the R17 watchdog is off,
+ * so a crash kills the calling process's CUDA context and a hang never returns — only for a
+ * supervised child process, paper_conf_ipps_yimpski11_b200/guardian.py);
+ * batch = replicas per launch (0 = auto); site_mask[b] bit s enables site s. */
 typedef struct {
   uint64_t seed; int64_t first, count; int32_t nbits; int32_t mode; int32_t batch; int32_t exact;
   uint64_t site_mask[3];

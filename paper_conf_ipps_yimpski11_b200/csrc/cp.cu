@@ -183,7 +183,8 @@ __device__ __forceinline__ CPGeo cp_geo_of(int64_t t, int BX, int BY, int gx, in
   return CPGeo{(int)(r % BX), (int)(r / BX), (int)(blk % gx), (int)(blk / gx), BX, BY, gx, gy};
 }
 
-template <int KIND, int U, bool EXACT, class Sink>
+// REAL: the guardian's unguarded variant (R25) — no R16 guards, no R17 watchdog.
+template <int KIND, int U, bool EXACT, bool REAL = false, class Sink>
 __device__ void cp_fi_program(const CPParams& p, const FaultRec& f, const CPGeo& G, bool mine, uint64_t grid_real,
                               Sink& S) {
   const int BX = G.BX, BY = G.BY;
@@ -238,7 +239,8 @@ __device__ void cp_fi_program(const CPParams& p, const FaultRec& f, const CPGeo&
   for (int j = 0; j < U; ++j) E[j] = 0.0f;
   int32_t it = 0;
   int32_t atomid = 0;
-  const int64_t limit = 10 * (n_atoms > 1 ? n_atoms : 1);
+  const int64_t limit = fi_limit<REAL>(n_atoms);
+  constexpr bool real = REAL;
   for (int64_t i = 0;; ++i) {
     const bool now = (i == inst);
     if (KIND == CK_ATOMID) { applied |= now; atomid = flip_i(atomid, now, mask); }
@@ -258,10 +260,10 @@ __device__ void cp_fi_program(const CPParams& p, const FaultRec& f, const CPGeo&
     }
     if (!(atomid < numatoms)) break;
     if (i >= limit) { fail |= FL_HANG; goto done; }
-    int64_t e;
-    if (!guard(patoms, atoms_real, atomid, 16, n_atoms, &e)) { fail |= FL_CRASH; goto done; }
+    const float4* pa;
+    if (!fi_at(real, patoms, atoms_real, atomid, n_atoms, &pa)) { fail |= FL_CRASH; goto done; }
     {
-      float4 at = __ldg(p.atoms + e);
+      float4 at = __ldg(pa);
       if (KIND == CK_AX) { applied |= now; at.x = flip_f(at.x, now, mask); }
       if (KIND == CK_AY) { applied |= now; at.y = flip_f(at.y, now, mask); }
       if (KIND == CK_AZ) { applied |= now; at.z = flip_f(at.z, now, mask); }
@@ -305,9 +307,9 @@ __device__ void cp_fi_program(const CPParams& p, const FaultRec& f, const CPGeo&
   chk ^= opqf(coorx, z); chk ^= opqf(coory, z); chk ^= opqf(gu, z);
 #pragma unroll
   for (int j = 0; j < U; ++j) {
-    int64_t e;
-    if (!guard(pgrid, grid_real, outaddr + j * BX, 4, n_grid, &e)) { fail |= FL_CRASH; goto done; }
-    S.store(0, e, E[j]);
+    float* po;
+    if (!fi_at(real, pgrid, grid_real, outaddr + j * BX, n_grid, &po)) { fail |= FL_CRASH; goto done; }
+    S.store_p(0, po, reinterpret_cast<const float*>(grid_real), E[j]);
   }
   chk ^= (uint32_t)opq(outaddr, z);
   chk ^= ((uint32_t)numatoms + z) ^ (fb(h) + z) ^ (lohi(pgrid) + z) ^ (lohi(patoms) + z);
@@ -334,6 +336,28 @@ __global__ void __launch_bounds__(256) cp_fi_kernel(const CPFIParams q) {
     const int64_t t = ((int64_t)G.byi * G.gx + G.bxi) * (G.BX * G.BY) + G.ty * G.BX + G.tx;
     ReplicaSinkF S{{p.grid, nullptr}, p.cb};
     cp_fi_program<KIND, U, EXACT>(p, f, G, t == f.thread, (uint64_t)(uintptr_t)p.grid, S);
+  }
+}
+
+// Unguarded replicas for the guardian (campaign mode 2, DESIGN R25): every CTA runs the per-thread
+// program with REAL = true; the site kind is a runtime switch (one injection per launch).
+template <int U, bool EXACT>
+__global__ void __launch_bounds__(256) cp_real_kernel(const CPFIParams q, int kind) {
+  const int r = blockIdx.z;
+  const FaultRec f = q.faults[r];
+  CPParams p = q.base;
+  p.grid = q.grid0 + (int64_t)r * q.grid_elems;
+  p.cb = q.cb0 + r;
+  const CPGeo G = cp_geo_here();
+  const int64_t t = ((int64_t)G.byi * G.gx + G.bxi) * (G.BX * G.BY) + G.ty * G.BX + G.tx;
+  ReplicaSinkF S{{p.grid, nullptr}, p.cb};
+  const uint64_t gr = (uint64_t)(uintptr_t)p.grid;
+  switch (kind) {
+#define K(k) case k: cp_fi_program<k, U, EXACT, true>(p, f, G, t == f.thread, gr, S); break;
+    K(CK_NL) K(CK_LIVE) K(CK_ATOMID) K(CK_AX) K(CK_AY) K(CK_AZ) K(CK_AW) K(CK_DY) K(CK_DYZ2) K(CK_DX0)
+    K(CK_DXJ) K(CK_R2) K(CK_S) K(CK_E) K(CK_IT)
+#undef K
+    default: break;
   }
 }
 
@@ -496,7 +520,7 @@ static cudaError_t launch_cp_fi_e(int kind, const CPFIParams& q, dim3 grid, dim3
 
 // One batch of `nrep` replicas of one kind: faults[0..nrep), outputs grid0[r], control blocks cb0[r].
 cudaError_t cp_fi_launch(int kind, const hk_cp_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
-                         float* grid0, int64_t stride, hk_control* cb0, cudaStream_t s) {
+                         float* grid0, int64_t stride, hk_control* cb0, bool real, cudaStream_t s) {
   CPFIParams q{};
   q.base.atoms = reinterpret_cast<const float4*>(a.atoms_ws);
   q.base.R = R;
@@ -511,6 +535,19 @@ cudaError_t cp_fi_launch(int kind, const hk_cp_args& a, const DevRanges& R, int 
   q.grid0 = grid0;
   q.cb0 = cb0;
   dim3 block(a.bx, a.by), grid(a.nx / (a.bx * a.unroll), a.ny / a.by, nrep);
+  if (real) {
+    if (a.unroll == 8) {
+      if (a.exact) cp_real_kernel<8, true><<<grid, block, 0, s>>>(q, kind);
+      else cp_real_kernel<8, false><<<grid, block, 0, s>>>(q, kind);
+    } else if (a.unroll == 4) {
+      if (a.exact) cp_real_kernel<4, true><<<grid, block, 0, s>>>(q, kind);
+      else cp_real_kernel<4, false><<<grid, block, 0, s>>>(q, kind);
+    } else {
+      return cudaErrorInvalidValue;
+    }
+    count_launch();
+    return cudaGetLastError();
+  }
   if (a.unroll == 8)
     return a.exact ? launch_cp_fi_e<8, true>(kind, q, grid, block, s) : launch_cp_fi_e<8, false>(kind, q, grid, block, s);
   if (a.unroll != 4) return cudaErrorInvalidValue;

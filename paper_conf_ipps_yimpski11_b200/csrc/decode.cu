@@ -41,6 +41,8 @@ __global__ void decode_kernel(const DecodeParams P) {
   f.index = n;
   f.site = s;
   f.sub = K.sub[s];
+  f.real = 0;
+  f.pad_ = 0;
   if (K.is_nl[s]) {
     const int64_t nt = (b == HK_MRIQ && s >= MRIQ_PHIMAG_SITE0) ? K.nk : K.nthr;
     f.thread = (int64_t)d_below(r2, (uint64_t)nt);

@@ -38,6 +38,8 @@ struct FaultRec {
   uint64_t mask;   // XOR mask (32- or 64-bit site)
   int32_t site;
   int32_t sub;
+  int32_t real;    // 1: unguarded run for the guardian (DESIGN R25); 0: crash / hang models R16 / R17
+  int32_t pad_;
 };
 
 // Site catalogue of one benchmark for the device decode (DESIGN R14): enabled sites, per-site
@@ -197,6 +199,36 @@ __device__ __forceinline__ bool guard(uint64_t preg, uint64_t preal, int32_t idx
   return true;
 }
 
+// Element address through a modelled pointer register (R16), or — in the guardian's unguarded runs
+// (R25) — the corrupted address itself, dereferenced as the uninstrumented program would: the
+// hardware decides (illegal or misaligned address kills the context, the guardian sees the crash).
+// nullptr = modelled crash.
+// Both are `true base + idx * size + delta`: delta = the modelled displacement (VBASE ^ m) - VBASE
+// (R16, checked against the buffer) or the real one, preg - preal (unchecked).  false = modelled crash.
+template <class T>
+__device__ __forceinline__ bool fi_at(bool real, uint64_t preg, uint64_t preal, int32_t idx, int64_t n, T** out) {
+  constexpr int64_t esz = (int64_t)sizeof(T);
+  const uint64_t m = preg ^ preal;
+  const int64_t delta = real ? (int64_t)(preg - preal) : (int64_t)((VBASE ^ m) - VBASE);
+  const int64_t off = (int64_t)idx * esz + delta;
+  *out = reinterpret_cast<T*>(preal + (uint64_t)off);
+  const bool in_buf = ((delta & (esz - 1)) == 0) & (off >= 0) & (off < n * esz);
+  return in_buf | real;  // non-short-circuit: one predicate op, no branch around the check
+}
+// Global-space accesses through fi_at results (the pointer came from an integer, so the compiler
+// cannot infer the space; the instrumented program's buffers are global, as are the kernel's).
+__device__ __forceinline__ void red_add(float* p, float v) {
+  asm volatile("red.global.add.f32 [%0], %1;" ::"l"(p), "f"(v) : "memory");
+}
+__device__ __forceinline__ void red_add(unsigned long long* p, unsigned long long v) {
+  asm volatile("red.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+// R17 watchdog limit; none in unguarded runs (the guardian's timeout observes the hang).
+template <bool REAL>
+__device__ __forceinline__ int64_t fi_limit(int64_t golden_trips) {
+  return REAL ? INT64_MAX : 10 * (golden_trips > 1 ? golden_trips : 1);
+}
+
 __device__ __forceinline__ unsigned lane_id() {
   unsigned l;
   asm("mov.u32 %0, %%laneid;" : "=r"(l));
@@ -237,6 +269,7 @@ struct ReplicaSinkF {
   float* out[2];
   hk_control* cb;
   __device__ __forceinline__ void store(int buf, int64_t e, float v) { atomicAdd(out[buf] + e, v); }
+  __device__ __forceinline__ void store_p(int, float* ptr, const float*, float v) { red_add(ptr, v); }
   __device__ __forceinline__ void outlier(int d, float v) { record_outlier(cb, d, v); }
   __device__ __forceinline__ void finish(bool mine, uint32_t alarm, uint32_t fail, uint32_t margin, float gap,
                                          uint32_t domain, bool applied, uint32_t tid) {
@@ -261,6 +294,7 @@ struct ReplaySinkF {
   __device__ __forceinline__ void store(int b, int64_t e, float v) {
     if (n < MAXW) { buf[n] = b; idx[n] = e; val[n] = v; ++n; }
   }
+  __device__ __forceinline__ void store_p(int b, float* ptr, const float* base, float v) { store(b, ptr - base, v); }
   __device__ __forceinline__ void outlier(int, float) {}
   __device__ __forceinline__ void finish(bool, uint32_t a, uint32_t f, uint32_t m, float g, uint32_t d, bool, uint32_t) {
     alarm = a; fail = f; margin = m; gap = g; domain = d;

@@ -41,12 +41,14 @@ int cp_site_kind(int site, int U, int* sub);
 int mriq_site_kind(int site);
 int tpacf_site_kind(int site);
 cudaError_t cp_fi_launch(int kind, const hk_cp_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
-                         float* grid0, int64_t stride, hk_control* cb0, cudaStream_t s);
+                         float* grid0, int64_t stride, hk_control* cb0, bool real, cudaStream_t s);
 cudaError_t mriq_fi_launch(int kind, const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
-                           int nrep, float* out0, int64_t stride, hk_control* cb0, float4* kv_rep, cudaStream_t s);
+                           int nrep, float* out0, int64_t stride, hk_control* cb0, float4* kv_rep, bool real,
+                           cudaStream_t s);
 constexpr int MRIQ_PHIMAG_SITE0 = 29;  // PhiMag NL sites 29-35 (replica mode only)
 cudaError_t tpacf_fi_launch(int kind, const hk_tpacf_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
-                            int nrep, unsigned long long* hist0, hk_control* cb0, void* lut_ws, cudaStream_t s);
+                            int nrep, unsigned long long* hist0, hk_control* cb0, void* lut_ws, bool real,
+                            cudaStream_t s);
 
 // replay accelerator (one CUDA thread per injection; classification fused)
 cudaError_t cp_replay_launch(int kind, const hk_cp_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,

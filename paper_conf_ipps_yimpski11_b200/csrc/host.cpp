@@ -591,7 +591,7 @@ static void keep_pool_memory() {
 static hk_status session_create(int32_t bench_mode, const void* const args[3], const hk_ranges* const ranges[3],
                                 const hk_campaign* C, cudaStream_t s, hk_campaign_session** out) {
   if (!args || !ranges || !C || !out || bench_mode < -1 || bench_mode > 2) return invalid("campaign: bad arguments");
-  if (C->mode != 0 && C->mode != 1) return invalid("campaign: mode must be 0 (replica) or 1 (replay)");
+  if (C->mode < 0 || C->mode > 2) return invalid("campaign: mode must be 0 (replica), 1 (replay) or 2 (unguarded replica)");
   if (C->nbits < 0 || C->nbits > 64) return invalid("campaign: nbits out of range");
   keep_pool_memory();
   hk_campaign_session* S = new hk_campaign_session();
@@ -777,6 +777,8 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
     else if (b == HK_MRIQ) it.kind = mriq_site_kind(hf.site);
     else it.kind = tpacf_site_kind(hf.site);
     it.f.sub = sub;
+    it.f.real = S->cfg.mode == 2 ? 1 : 0;  // R25: guardian child processes only
+    it.f.pad_ = 0;
     items[(size_t)q] = it;
   }
   std::stable_sort(items.begin(), items.end(), [](const Item& x, const Item& y) {
@@ -804,6 +806,7 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
   cudaEventRecord(S->uploaded, s);
 
   // ---- batches: FI&FT replicas, then the classify epilogue (which also recycles the workspace)
+  const bool real = S->cfg.mode == 2;  // R25: unguarded replicas (guardian child processes only)
   size_t q = 0;
   while (q < items.size()) {
     const int b = items[q].b, kind = items[q].kind;
@@ -813,21 +816,22 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
     BenchWS& w = S->W[b];
     const FaultRec* fr = S->d_faults + q;
     if (b == HK_CP) {
-      if ((e = cp_fi_launch(kind, S->cp, w.R, std::min(w.ndet, S->cp.unroll), fr, nrep, (float*)w.rep_out, w.out_elems, w.rep_cb, s)) != cudaSuccess)
+      if ((e = cp_fi_launch(kind, S->cp, w.R, std::min(w.ndet, S->cp.unroll), fr, nrep, (float*)w.rep_out, w.out_elems, w.rep_cb,
+                            real, s)) != cudaSuccess)
         return cuda_fail(e, "cp FI");
       if ((e = classify_fp_launch(b, (float*)w.rep_out, w.out_elems, (const float*)w.golden, w.dM, w.rep_cb, fr, nrep,
                                   d_records, first, d_counts, d_site_counts, s)) != cudaSuccess)
         return cuda_fail(e, "classify");
     } else if (b == HK_MRIQ) {
       if ((e = mriq_fi_launch(kind, S->mq, w.R, std::min(w.ndet, 2), fr, nrep, (float*)w.rep_out, w.out_elems, w.rep_cb,
-                              w.kv_rep, s)) != cudaSuccess)
+                              w.kv_rep, real, s)) != cudaSuccess)
         return cuda_fail(e, "mriq FI");
       if ((e = classify_fp_launch(b, (float*)w.rep_out, w.out_elems, (const float*)w.golden, w.dM, w.rep_cb, fr, nrep,
                                   d_records, first, d_counts, d_site_counts, s)) != cudaSuccess)
         return cuda_fail(e, "classify");
     } else {
       if ((e = tpacf_fi_launch(kind, S->tp, w.R, std::min(w.ndet, 1), fr, nrep, (unsigned long long*)w.rep_out, w.rep_cb,
-                               w.lut, s)) != cudaSuccess)
+                               w.lut, real, s)) != cudaSuccess)
         return cuda_fail(e, "tpacf FI");
       if ((e = classify_tpacf_launch((unsigned long long*)w.rep_out, S->tp.n_rand, S->tp.n_bins,
                                      (const unsigned long long*)w.golden, w.rep_cb, fr, nrep, d_records, first, d_counts,

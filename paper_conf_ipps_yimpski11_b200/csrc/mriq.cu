@@ -210,7 +210,8 @@ struct MQFIParams {
 
 // Per-thread FI&FT program of voxel t.  t_dup: the duplicate of N0 recomputed from launch indices
 // (replica) or from the abstract id (replay); qr_real / qi_real: the buffers' true base addresses.
-template <int KIND, bool EXACT, class Sink>
+// REAL: the guardian's unguarded variant (R25) — no R16 guards, no R17 watchdog.
+template <int KIND, bool EXACT, bool REAL = false, class Sink>
 __device__ void mriq_fi_program(const MQParams& p, const FaultRec& f, int32_t t, int32_t t_dup, bool mine,
                                 uint64_t qr_real, uint64_t qi_real, Sink& S) {
   const int64_t inst = mine ? f.inst : -1;
@@ -233,20 +234,22 @@ __device__ void mriq_fi_program(const MQParams& p, const FaultRec& f, int32_t t,
   alarm |= (t_dup != xIndex) ? AL_DUP : 0u;
   float sX, sY, sZ, Qr = 0.f, Qi = 0.f;
   int32_t it = 0, k = 0;
-  int64_t e;
-  const int64_t limit = 10 * (nk > 1 ? nk : 1);
-  if (!guard(px, x_real, xIndex, 4, nv, &e)) { fail |= FL_CRASH; goto done; }
-  sX = p.x[e];
+  const float* pe;
+  float* po;
+  const int64_t limit = fi_limit<REAL>(nk);
+  constexpr bool real = REAL;
+  if (!fi_at(real, px, x_real, xIndex, nv, &pe)) { fail |= FL_CRASH; goto done; }
+  sX = __ldg(pe);
   { const bool n = nl && site == 1; applied |= n; sX = flip_f(sX, n, mask); }
-  chk ^= fb(sX); alarm |= (fb(p.x[e + z]) != fb(sX)) ? AL_DUP : 0u;
-  if (!guard(py, y_real, xIndex, 4, nv, &e)) { fail |= FL_CRASH; goto done; }
-  sY = p.y[e];
+  chk ^= fb(sX); alarm |= (fb(__ldg(pe + z)) != fb(sX)) ? AL_DUP : 0u;
+  if (!fi_at(real, py, y_real, xIndex, nv, &pe)) { fail |= FL_CRASH; goto done; }
+  sY = __ldg(pe);
   { const bool n = nl && site == 2; applied |= n; sY = flip_f(sY, n, mask); }
-  chk ^= fb(sY); alarm |= (fb(p.y[e + z]) != fb(sY)) ? AL_DUP : 0u;
-  if (!guard(pz, z_real, xIndex, 4, nv, &e)) { fail |= FL_CRASH; goto done; }
-  sZ = p.z[e];
+  chk ^= fb(sY); alarm |= (fb(__ldg(pe + z)) != fb(sY)) ? AL_DUP : 0u;
+  if (!fi_at(real, pz, z_real, xIndex, nv, &pe)) { fail |= FL_CRASH; goto done; }
+  sZ = __ldg(pe);
   { const bool n = nl && site == 3; applied |= n; sZ = flip_f(sZ, n, mask); }
-  chk ^= fb(sZ); alarm |= (fb(p.z[e + z]) != fb(sZ)) ? AL_DUP : 0u;
+  chk ^= fb(sZ); alarm |= (fb(__ldg(pe + z)) != fb(sZ)) ? AL_DUP : 0u;
 
   for (int64_t i = 0;; ++i) {
     const bool now = (i == inst);
@@ -270,9 +273,10 @@ __device__ void mriq_fi_program(const MQParams& p, const FaultRec& f, int32_t t,
     }
     if (!(k < numK)) break;
     if (i >= limit) { fail |= FL_HANG; goto done; }
-    if (!guard(pkv, kv_real, k, 16, nk, &e)) { fail |= FL_CRASH; goto done; }
+    const float4* pk;
+    if (!fi_at(real, pkv, kv_real, k, nk, &pk)) { fail |= FL_CRASH; goto done; }
     {
-      float4 k4 = __ldg(p.kv + e);
+      float4 k4 = __ldg(pk);
       if (KIND == MK_KX) { applied |= now; k4.x = flip_f(k4.x, now, mask); }
       if (KIND == MK_KY) { applied |= now; k4.y = flip_f(k4.y, now, mask); }
       if (KIND == MK_KZ) { applied |= now; k4.z = flip_f(k4.z, now, mask); }
@@ -313,10 +317,10 @@ __device__ void mriq_fi_program(const MQParams& p, const FaultRec& f, int32_t t,
     }
   }
   chk ^= opqf(sX, z); chk ^= opqf(sY, z); chk ^= opqf(sZ, z);
-  if (!guard(pqr, qr_real, xIndex, 4, nv, &e)) { fail |= FL_CRASH; goto done; }
-  S.store(0, e, Qr);
-  if (!guard(pqi, qi_real, xIndex, 4, nv, &e)) { fail |= FL_CRASH; goto done; }
-  S.store(1, e, Qi);
+  if (!fi_at(real, pqr, qr_real, xIndex, nv, &po)) { fail |= FL_CRASH; goto done; }
+  S.store_p(0, po, reinterpret_cast<const float*>(qr_real), Qr);
+  if (!fi_at(real, pqi, qi_real, xIndex, nv, &po)) { fail |= FL_CRASH; goto done; }
+  S.store_p(1, po, reinterpret_cast<const float*>(qi_real), Qi);
   chk ^= (uint32_t)opq(xIndex, z);
   chk ^= ((uint32_t)numK + z) ^ (lohi(pkv) + z) ^ (lohi(pqr) + z) ^ (lohi(pqi) + z) ^ (lohi(px) + z) ^ (lohi(py) + z) ^
          (lohi(pz) + z);
@@ -352,7 +356,8 @@ __global__ void __launch_bounds__(256) mriq_phimag_fi_kernel(const float* __rest
   const int sid[5] = {30, 31, 33, 34, 35};
 #pragma unroll
   for (int a = 0; a < 5; ++a) {
-    if (!guard(vb, vb, kidx, 4, nk, &e)) { fail |= FL_CRASH; goto done; }
+    if (f.real) e = kidx;  // R25: the corrupted index is used as is
+    else if (!guard(vb, vb, kidx, 4, nk, &e)) { fail |= FL_CRASH; goto done; }
     v[a] = flip_f(src[a][e], site == sid[a], mask);
     chk ^= fb(v[a]); alarm |= (fb(src[a][e + z]) != fb(v[a])) ? AL_DUP : 0u;
     if (a == 1) {
@@ -365,7 +370,8 @@ __global__ void __launch_bounds__(256) mriq_phimag_fi_kernel(const float* __rest
     chk ^= fb(pm);
     const float re2 = bf(fb(re) + z), im2 = bf(fb(im) + z);
     alarm |= (fb(__fmaf_rn(im2, im2, __fmul_rn(re2, re2))) != fb(pm)) ? AL_DUP : 0u;
-    if (!guard(vb, vb, kidx, 16, nk, &e)) { fail |= FL_CRASH; goto done; }
+    if (f.real) e = kidx;
+    else if (!guard(vb, vb, kidx, 16, nk, &e)) { fail |= FL_CRASH; goto done; }
     atomicAdd(kv + 4 * e + 0, v[2]);
     atomicAdd(kv + 4 * e + 1, v[3]);
     atomicAdd(kv + 4 * e + 2, v[4]);
@@ -402,6 +408,31 @@ __global__ void __launch_bounds__(256) mriq_fi_kernel(const MQFIParams q) {
         mriq_fi_program<KIND, EXACT>(p, f, t, t_dup, t == f.thread, (uint64_t)(uintptr_t)p.qr, (uint64_t)(uintptr_t)p.qi, S);
       }
     }
+  }
+}
+
+// Unguarded replicas for the guardian (campaign mode 2, DESIGN R25): every thread runs the
+// per-voxel program with REAL = true (Q-kernel kinds; PhiMag kinds use mriq_phimag_fi_kernel,
+// which reads FaultRec::real, followed by the fault-free Q kernel).
+template <bool EXACT>
+__global__ void __launch_bounds__(256) mriq_real_kernel(const MQFIParams q, int kind) {
+  const int r = blockIdx.y;
+  const FaultRec f = q.faults[r];
+  MQParams p = q.base;
+  p.qr = q.out0 + (int64_t)r * q.stride;
+  p.qi = p.qr + p.numX;
+  p.cb = q.cb0 + r;
+  ReplicaSinkF S{{p.qr, p.qi}, p.cb};
+  const int32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= p.numX) return;
+  const int32_t t_dup = (int32_t)((blockIdx.x ^ p.zz) * blockDim.x + (threadIdx.x ^ p.zz));
+  const uint64_t qr = (uint64_t)(uintptr_t)p.qr, qi = (uint64_t)(uintptr_t)p.qi;
+  switch (kind) {
+#define K(k) case k: mriq_fi_program<k, EXACT, true>(p, f, t, t_dup, t == f.thread, qr, qi, S); break;
+    K(MK_NL) K(MK_LIVE) K(MK_K) K(MK_KX) K(MK_KY) K(MK_KZ) K(MK_PM) K(MK_T1) K(MK_T2) K(MK_T) K(MK_R) K(MK_C)
+    K(MK_S) K(MK_QR) K(MK_QI) K(MK_IT)
+#undef K
+    default: break;
   }
 }
 
@@ -558,7 +589,7 @@ cudaError_t mriq_replay_launch(int kind, const hk_mriq_args& a, const DevRanges&
 }
 
 cudaError_t mriq_fi_launch(int kind, const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
-                           float* out0, int64_t stride, hk_control* cb0, float4* kv_rep, cudaStream_t s) {
+                           float* out0, int64_t stride, hk_control* cb0, float4* kv_rep, bool real, cudaStream_t s) {
   if (kind == MK_PHIMAG) {
     if (!kv_rep) return cudaErrorInvalidValue;
     cudaError_t e = cudaMemsetAsync(kv_rep, 0, sizeof(float4) * (size_t)a.n_k * nrep, s);
@@ -575,6 +606,13 @@ cudaError_t mriq_fi_launch(int kind, const hk_mriq_args& a, const DevRanges& R, 
   q.out0 = out0;
   q.stride = stride;
   q.cb0 = cb0;
+  if (real && kind != MK_PHIMAG) {
+    dim3 grid((a.n_vox + 255) / 256, nrep);
+    if (a.exact) mriq_real_kernel<true><<<grid, 256, 0, s>>>(q, kind);
+    else mriq_real_kernel<false><<<grid, 256, 0, s>>>(q, kind);
+    count_launch();
+    return cudaGetLastError();
+  }
   return a.exact ? launch_mq_fi_e<true>(kind, q, nrep, s) : launch_mq_fi_e<false>(kind, q, nrep, s);
 }
 

@@ -87,7 +87,7 @@ __global__ void tpacf_lut_kernel(const float* __restrict__ edges, int nb, uint8_
   if (neg) {
     out = make_int2(0, fb(e0));  // u <= -0: dot >= 1 > every edge -> bin 0 (and -NaN: bin 0)
   } else if (special) {
-    out = (q == (int)(0x7f800000u >> 21)) ? make_int2(nb + 1, (int)-8388608) : make_int2(0, fb(e0));
+    out = (q == (int)(0x7f800000u >> 21)) ? make_int2(nb + 1, (int)0xff800000u) : make_int2(0, (int)fb(e0));
   } else {
     const float ulo = bf(lo_bits), uhi = bf(hi_bits);
     // largest dot with fl(1 - dot) >= ulo, smallest dot with fl(1 - dot) <= uhi
@@ -99,7 +99,7 @@ __global__ void tpacf_lut_kernel(const float* __restrict__ edges, int nb, uint8_
     for (int k = 0; k < 64 && __fsub_rn(1.0f, dmin) > uhi; ++k) dmin = nup(dmin);
     const int bmin = bin_def(edges, nb, dmax), bmax = bin_def(edges, nb, dmin);
     good = (__fsub_rn(1.0f, dmax) >= ulo) && (__fsub_rn(1.0f, dmin) <= uhi) && (bmax - bmin <= 1);
-    out = make_int2(bmin, bmin <= nb ? fb(edges[bmin]) : (int)-8388608);
+    out = make_int2(bmin, (int)(bmin <= nb ? fb(edges[bmin]) : 0xff800000u));
   }
   lut[q] = (uint8_t)out.x;  // E[b] (padded with -inf beyond nb) supplies the compare value
   if (!good) atomicExch(ok, 0);
@@ -372,6 +372,7 @@ struct TPReplicaSink {
   int nb2;
   __device__ __forceinline__ bool global_path(bool mine) const { return mine; }
   __device__ __forceinline__ void hist_global(int64_t e) { atomicAdd(hist + e, 1ull); }
+  __device__ __forceinline__ void hist_p(unsigned long long* ptr, const unsigned long long*) { red_add(ptr, 1ull); }
   __device__ __forceinline__ void hist_local(uint32_t warp, int32_t bin, uint32_t lane) {
     H[((size_t)warp * nb2 + bin) * 32 + lane] += 1u;
   }
@@ -400,6 +401,7 @@ struct TPReplaySink {
     const int kind = row == 0 ? 0 : (row <= nr ? 2 : 1);
     delta[kind * nb + b - 1] += sign;
   }
+  __device__ __forceinline__ void hist_p(unsigned long long* ptr, const unsigned long long* base) { hist_global(ptr - base); }
   __device__ __forceinline__ void hist_local(uint32_t, int32_t, uint32_t) {}
   __device__ __forceinline__ void outlier(int, float) {}
   __device__ __forceinline__ void finish(bool, uint32_t a, uint32_t f, uint32_t m, float g, bool, uint32_t) {
@@ -409,7 +411,8 @@ struct TPReplaySink {
 
 // Per-thread FI&FT program of abstract thread g = row*N + ii.  i_dup: N0's duplicate from launch
 // indices (replica) or from the abstract id (replay); hist_real: the histogram's true base.
-template <int KIND, class Sink>
+// REAL: the guardian's unguarded variant (R25) — no R16 guards, no R17 watchdog.
+template <int KIND, bool REAL = false, class Sink>
 __device__ void tpacf_fi_program(const TPParams& p, const TPSmem& S, const FaultRec& f, int32_t row, int32_t ii,
                                  int32_t i_dup, int32_t row_dup, bool mine, uint64_t hist_real, Sink& K) {
   const uint32_t z = p.z;
@@ -459,17 +462,18 @@ __device__ void tpacf_fi_program(const TPParams& p, const TPSmem& S, const Fault
 #undef NLF
   float q1[3];
   int32_t acc = 0, cnt = 0, j;
-  int64_t e;
+  const float* pe;
   const int32_t row_c = row - (row / nC) * nC;  // uncorrupted launch chunk (watchdog)
   const int32_t g_jb = (row / nC) <= nr ? max(ii + 1, row_c * C) : row_c * C;
   const int32_t g_je = min((row_c + 1) * C, p.n);
   const int64_t golden = g_je > g_jb ? g_je - g_jb : 0;
-  const int64_t limit = 10 * (golden > 1 ? golden : 1);
+  const int64_t limit = fi_limit<REAL>(golden);
+  constexpr bool real = REAL;
   for (int a = 0; a < 3; ++a) {
-    if (!guard(ppts, pts_real, (int32_t)((uint32_t)aoff * 3u + (uint32_t)a), 4, npts, &e)) { fail |= FL_CRASH; goto done; }
-    float v = p.pts[e];
+    if (!fi_at(real, ppts, pts_real, (int32_t)((uint32_t)aoff * 3u + (uint32_t)a), npts, &pe)) { fail |= FL_CRASH; goto done; }
+    float v = __ldg(pe);
     { const bool nn = nl && site == 9 + a; applied |= nn; v = flip_f(v, nn, mask); }
-    chk ^= fb(v); alarm |= (fb(p.pts[e + z]) != fb(v)) ? AL_DUP : 0u;
+    chk ^= fb(v); alarm |= (fb(__ldg(pe + z)) != fb(v)) ? AL_DUP : 0u;
     q1[a] = v;
   }
   chk ^= (uint32_t)opq(i, z) ^ (uint32_t)opq(h, z) ^ (uint32_t)opq(c, z) ^ (uint32_t)opq(aoff, z) ^ (uint32_t)opq(jb, z);
@@ -500,8 +504,8 @@ __device__ void tpacf_fi_program(const TPParams& p, const TPSmem& S, const Fault
       float q2[3];
 #pragma unroll
       for (int a = 0; a < 3; ++a) {
-        if (!guard(ppts, pts_real, (int32_t)((uint32_t)pb + (uint32_t)a), 4, npts, &e)) { fail |= FL_CRASH; goto done; }
-        q2[a] = p.pts[e];
+        if (!fi_at(real, ppts, pts_real, (int32_t)((uint32_t)pb + (uint32_t)a), npts, &pe)) { fail |= FL_CRASH; goto done; }
+        q2[a] = __ldg(pe);
       }
       if (KIND == TK_X2) { applied |= now; q2[0] = flip_f(q2[0], now, mask); }
       if (KIND == TK_Y2) { applied |= now; q2[1] = flip_f(q2[1], now, mask); }
@@ -513,8 +517,9 @@ __device__ void tpacf_fi_program(const TPParams& p, const TPSmem& S, const Fault
       int32_t hidx = (int32_t)((uint32_t)base + (uint32_t)bin);
       if (KIND == TK_HIDX) { applied |= now; hidx = flip_i(hidx, now, mask); }
       if (K.global_path(mine)) {
-        if (!guard(phist, hist_real, hidx, 8, nhist, &e)) { fail |= FL_CRASH; goto done; }
-        K.hist_global(e);
+        unsigned long long* ph;
+        if (!fi_at(real, phist, hist_real, hidx, nhist, &ph)) { fail |= FL_CRASH; goto done; }
+        K.hist_p(ph, reinterpret_cast<const unsigned long long*>(hist_real));
       } else {
         K.hist_local(warp, bin, lane);  // fault-free thread: hidx == base + bin (this CTA's row)
       }
@@ -538,18 +543,11 @@ done:
   K.finish(mine, alarm, fail, margin, gap, applied, (uint32_t)g);
 }
 
-template <int KIND>
-__global__ void __launch_bounds__(TP_THREADS) tpacf_fi_kernel(const TPFIParams q) {
-  extern __shared__ __align__(16) unsigned char tp_smem[];
-  const TPSmem S = tp_carve(tp_smem, q.base.C);
-  const int r = blockIdx.z;
-  const FaultRec f = q.faults[r];
-  unsigned long long* hist = q.hist0 + (int64_t)r * q.hist_elems;
-  hk_control* cb = q.cb0 + r;
-  const int64_t cta_first = (int64_t)blockIdx.y * q.base.n + (int64_t)blockIdx.x * TP_CTA_PTS;
-  if (f.thread < cta_first || f.thread >= cta_first + TP_CTA_PTS) {
-    tpacf_body<V_NL | V_L>(q.base, S, hist, cb);
-  } else {
+// The CTA that holds the faulted abstract thread: every thread runs the per-thread program.
+template <int KIND, bool REAL>
+__device__ __forceinline__ void tpacf_fi_cta(const TPFIParams& q, const TPSmem& S, const FaultRec& f,
+                                             unsigned long long* hist, hk_control* cb) {
+  {
     const TPParams& p = q.base;
     const int32_t h = blockIdx.y / p.nC, c = blockIdx.y - h * p.nC;
     const int32_t sb = (h == 0) ? 0 : (h <= p.nr ? h : h - p.nr);
@@ -562,12 +560,42 @@ __global__ void __launch_bounds__(TP_THREADS) tpacf_fi_kernel(const TPFIParams q
       if (ii < p.n) {
         const int32_t idup = (int32_t)((blockIdx.x ^ p.z) * TP_CTA_PTS + kpt * TP_THREADS + (threadIdx.x ^ p.z));
         const int64_t g = (int64_t)blockIdx.y * p.n + ii;
-        tpacf_fi_program<KIND>(p, S, f, (int32_t)blockIdx.y, ii, idup, (int32_t)(blockIdx.y ^ p.z), g == f.thread,
-                               (uint64_t)(uintptr_t)hist, K);
+        tpacf_fi_program<KIND, REAL>(p, S, f, (int32_t)blockIdx.y, ii, idup, (int32_t)(blockIdx.y ^ p.z),
+                                     g == f.thread, (uint64_t)(uintptr_t)hist, K);
       }
     }
     __syncthreads();
     tp_flush(p, S, hist, h * (p.nb + 2));
+  }
+}
+
+template <int KIND>
+__global__ void __launch_bounds__(TP_THREADS) tpacf_fi_kernel(const TPFIParams q) {
+  extern __shared__ __align__(16) unsigned char tp_smem[];
+  const TPSmem S = tp_carve(tp_smem, q.base.C);
+  const int r = blockIdx.z;
+  const FaultRec f = q.faults[r];
+  unsigned long long* hist = q.hist0 + (int64_t)r * q.hist_elems;
+  hk_control* cb = q.cb0 + r;
+  const int64_t cta_first = (int64_t)blockIdx.y * q.base.n + (int64_t)blockIdx.x * TP_CTA_PTS;
+  if (f.thread < cta_first || f.thread >= cta_first + TP_CTA_PTS) tpacf_body<V_NL | V_L>(q.base, S, hist, cb);
+  else tpacf_fi_cta<KIND, false>(q, S, f, hist, cb);
+}
+
+// Unguarded replicas for the guardian (campaign mode 2, DESIGN R25): every CTA runs the per-thread
+// program with REAL = true; the site kind is a runtime switch (one injection per launch).
+__global__ void __launch_bounds__(TP_THREADS) tpacf_real_kernel(const TPFIParams q, int kind) {
+  extern __shared__ __align__(16) unsigned char tp_smem[];
+  const TPSmem S = tp_carve(tp_smem, q.base.C);
+  const int r = blockIdx.z;
+  const FaultRec f = q.faults[r];
+  unsigned long long* hist = q.hist0 + (int64_t)r * q.hist_elems;
+  hk_control* cb = q.cb0 + r;
+  switch (kind) {
+#define K(k) case k: tpacf_fi_cta<k, true>(q, S, f, hist, cb); break;
+    K(TK_NL) K(TK_LIVE) K(TK_J) K(TK_X2) K(TK_Y2) K(TK_Z2) K(TK_DOT) K(TK_BIN) K(TK_HIDX) K(TK_ACC) K(TK_CNT)
+#undef K
+    default: break;
   }
 }
 
@@ -747,13 +775,22 @@ cudaError_t tpacf_replay_launch(int kind, const hk_tpacf_args& a, const DevRange
 
 // lut_ws must hold a table built by tpacf_lut_build for a.edges (the campaign builds it once).
 cudaError_t tpacf_fi_launch(int kind, const hk_tpacf_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
-                            unsigned long long* hist0, hk_control* cb0, void* lut_ws, cudaStream_t s) {
+                            unsigned long long* hist0, hk_control* cb0, void* lut_ws, bool real, cudaStream_t s) {
   TPFIParams q{};
   q.base = tp_params(a, R, ndet, nullptr, nullptr, lut_ws);
   q.faults = faults;
   q.hist0 = hist0;
   q.cb0 = cb0;
   q.hist_elems = (int64_t)(1 + 2 * a.n_rand) * (a.n_bins + 2);
+  if (real) {
+    const size_t smem = tp_smem_bytes(q.base.C, q.base.nb + 2);
+    cudaError_t e = cudaFuncSetAttribute(tpacf_real_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    dim3 grid((a.n + TP_CTA_PTS - 1) / TP_CTA_PTS, (1 + 2 * a.n_rand) * q.base.nC, nrep);
+    tpacf_real_kernel<<<grid, TP_THREADS, smem, s>>>(q, kind);
+    count_launch();
+    return cudaGetLastError();
+  }
   switch (kind) {
 #define K(k) case k: return launch_tp_fi_k<k>(q, nrep, s);
     K(TK_NL) K(TK_LIVE) K(TK_J) K(TK_X2) K(TK_Y2) K(TK_Z2) K(TK_DOT) K(TK_BIN) K(TK_HIDX) K(TK_ACC) K(TK_CNT)

@@ -14,7 +14,8 @@ import numpy as np
 import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libhauberk.so")
+# HAUBERK_LIB: another build of the same library (A/B timing of two builds on one box)
+LIB_PATH = os.environ.get("HAUBERK_LIB") or os.path.join(_HERE, "libhauberk.so")
 
 HK_CP, HK_MRIQ, HK_TPACF, HK_MIXED = 0, 1, 2, -1
 HK_BASE, HK_FT, HK_FT_NL, HK_FT_L, HK_PROFILE = 0, 1, 2, 3, 4

@@ -528,3 +528,22 @@ def test_cp_unroll8_campaign_exact(mode):
     g = hk.records_numpy(rec)
     assert np.array_equal(g["site"], o["site"]) and np.array_equal(g["cls"], o["cls"])
     assert np.array_equal(counts.cpu().numpy(), oc)
+
+
+# ---------------------------------------------------------------------------------------------- guardian (f4)
+@pytest.mark.parametrize("bench", [0, 2])
+def test_guardian_real_crash_validation(bench):
+    """SURVEY f4 / DESIGN R25: modelled crashes and hangs are re-run UNGUARDED in supervised child
+    processes.  Injections the models call non-failures must complete with the identical class.
+    How many modelled failures are real crashes is a measurement, not a property (out-of-buffer
+    accesses that land in mapped memory do not fault: the known limit of R16; small buffers share
+    their 2 MiB pages with others), reported by `python -m paper_conf_ipps_yimpski11_b200.guardian`."""
+    from paper_conf_ipps_yimpski11_b200 import guardian as G
+    p = [W.cp_small(), None, W.tpacf_small(n=150, n_rand=1, chunk=64)][bench]
+    rep = G.validate(bench, p, n_fail=10, n_other=8, scan=600, floor_s=2.0)
+    assert rep["n"] == rep["sampled_failures"] + rep["sampled_others"] and rep["sampled_failures"] > 0
+    assert rep["non_failure_identical"] == 1.0
+    conf = rep["confusion"]
+    real_fail = sum(v for m in ("crash", "hang") for r, v in conf.get(m, {}).items() if r in ("crash", "hang"))
+    assert real_fail >= 1  # the unguarded runs really dereference the corrupted addresses
+    assert rep["done_with_model_fail_bits"] == 0  # no R16/R17 verdicts in unguarded runs

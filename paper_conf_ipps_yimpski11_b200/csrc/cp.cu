@@ -28,12 +28,11 @@ struct CPParams {
 
 // One CTA's worth of the protected loop.  V: variant flags; ADD: additive stores (R18, FI replicas).
 template <int V, int U, bool EXACT, bool ADD>
-__device__ __forceinline__ void cp_body(const CPParams& p, float4 (*tile)[CP_TILE], uint64_t* bar) {
+__device__ __forceinline__ void cp_body(const CPParams& p, float4 (*tile)[CP_TILE], uint64_t* bar, int bxi, int byi) {
   constexpr bool NL = (V & V_NL) != 0, L = (V & V_L) != 0, PROF = (V & V_PROF) != 0;
   constexpr bool CNT = L || PROF;
   const int BX = blockDim.x, BY = blockDim.y;
   const int tx = threadIdx.x, ty = threadIdx.y;
-  const int bxi = blockIdx.x, byi = blockIdx.y;
   const uint32_t z = p.z;
   const uint32_t tid = (uint32_t)(((int64_t)byi * gridDim.x + bxi) * (BX * BY) + ty * BX + tx);
   uint32_t chk = 0, alarm = 0;
@@ -137,7 +136,7 @@ template <int V, int U, bool EXACT>
 __global__ void __launch_bounds__(256) cp_kernel(const CPParams p) {
   __shared__ __align__(128) float4 tile[2][CP_TILE];
   __shared__ __align__(8) uint64_t bar[2];
-  cp_body<V, U, EXACT, false>(p, tile, bar);
+  cp_body<V, U, EXACT, false>(p, tile, bar, blockIdx.x, blockIdx.y);
 }
 
 // Uninstrumented pre-pass (row a1): (x, y, z, q) -> (x, y, (z - z0)^2, q).
@@ -174,9 +173,9 @@ struct CPFIParams {
 struct CPGeo {
   int tx, ty, bxi, byi, BX, BY, gx, gy;
 };
-__device__ __forceinline__ CPGeo cp_geo_here() {
-  return CPGeo{(int)threadIdx.x, (int)threadIdx.y, (int)blockIdx.x, (int)blockIdx.y, (int)blockDim.x, (int)blockDim.y,
-               (int)gridDim.x, (int)gridDim.y};
+__device__ __forceinline__ CPGeo cp_geo_here(int bxi, int byi) {
+  return CPGeo{(int)threadIdx.x, (int)threadIdx.y, bxi, byi, (int)blockDim.x, (int)blockDim.y, (int)gridDim.x,
+               (int)gridDim.y};
 }
 __device__ __forceinline__ CPGeo cp_geo_of(int64_t t, int BX, int BY, int gx, int gy) {
   const int64_t per = (int64_t)BX * BY, blk = t / per, r = t % per;
@@ -322,17 +321,21 @@ template <int KIND, int U, bool EXACT>
 __global__ void __launch_bounds__(256) cp_fi_kernel(const CPFIParams q) {
   __shared__ __align__(128) float4 tile[2][CP_TILE];
   __shared__ __align__(8) uint64_t bar[2];
-  const int r = blockIdx.z;
+  const int64_t tpb = (int64_t)blockDim.x * blockDim.y, ncta = (int64_t)gridDim.x * gridDim.y;
+  const int64_t L = ((int64_t)blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x;
+  int r;
+  int64_t cta;
+  const bool faulted = fi_order(L, ncta, (int)gridDim.z, [&](int rr) { return clamp_cta(q.faults[rr].thread / tpb, ncta); },
+                                &r, &cta);
   const FaultRec f = q.faults[r];
   CPParams p = q.base;
   p.grid = q.grid0 + (int64_t)r * q.grid_elems;
   p.cb = q.cb0 + r;
-  const int64_t tpb = (int64_t)blockDim.x * blockDim.y;
-  const int64_t cta = (int64_t)blockIdx.y * gridDim.x + blockIdx.x;
-  if (f.thread / tpb != cta) {
-    cp_body<V_NL | V_L, U, EXACT, true>(p, tile, bar);
+  const int bxi = (int)(cta % gridDim.x), byi = (int)(cta / gridDim.x);
+  if (!faulted) {
+    cp_body<V_NL | V_L, U, EXACT, true>(p, tile, bar, bxi, byi);
   } else {
-    const CPGeo G = cp_geo_here();
+    const CPGeo G = cp_geo_here(bxi, byi);
     const int64_t t = ((int64_t)G.byi * G.gx + G.bxi) * (G.BX * G.BY) + G.ty * G.BX + G.tx;
     ReplicaSinkF S{{p.grid, nullptr}, p.cb};
     cp_fi_program<KIND, U, EXACT>(p, f, G, t == f.thread, (uint64_t)(uintptr_t)p.grid, S);
@@ -348,7 +351,7 @@ __global__ void __launch_bounds__(256) cp_real_kernel(const CPFIParams q, int ki
   CPParams p = q.base;
   p.grid = q.grid0 + (int64_t)r * q.grid_elems;
   p.cb = q.cb0 + r;
-  const CPGeo G = cp_geo_here();
+  const CPGeo G = cp_geo_here(blockIdx.x, blockIdx.y);
   const int64_t t = ((int64_t)G.byi * G.gx + G.bxi) * (G.BX * G.BY) + G.ty * G.BX + G.tx;
   ReplicaSinkF S{{p.grid, nullptr}, p.cb};
   const uint64_t gr = (uint64_t)(uintptr_t)p.grid;

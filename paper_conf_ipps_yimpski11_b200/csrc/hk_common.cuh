@@ -223,6 +223,27 @@ __device__ __forceinline__ void red_add(float* p, float v) {
 __device__ __forceinline__ void red_add(unsigned long long* p, unsigned long long v) {
   asm volatile("red.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
+// Launch order of the FI&FT replica kernels.  CTAs are dispatched in (roughly) linear block order:
+// the first nrep of them run the faulted CTA of replica 0..nrep-1, whose per-thread FI program is
+// several times slower than a fast-path CTA — started first, it overlaps the fast CTAs instead of
+// trailing the launch — and the others follow replica by replica in CTA order.  fault_cta(r) in
+// [0, ncta) is the CTA that holds replica r's faulted thread.  Returns true for a faulted CTA.
+template <class F>
+__device__ __forceinline__ bool fi_order(int64_t L, int64_t ncta, int nrep, F fault_cta, int* r, int64_t* cta) {
+  if (L < nrep) {
+    *r = (int)L;
+    *cta = fault_cta((int)L);
+    return true;
+  }
+  const int64_t L2 = L - nrep;
+  const int rr = (int)(L2 / (ncta - 1));
+  const int64_t k = L2 - (int64_t)rr * (ncta - 1), fc = fault_cta(rr);
+  *r = rr;
+  *cta = k < fc ? k : k + 1;
+  return false;
+}
+__device__ __forceinline__ int64_t clamp_cta(int64_t c, int64_t ncta) { return c < 0 ? 0 : (c >= ncta ? ncta - 1 : c); }
+
 // R17 watchdog limit; none in unguarded runs (the guardian's timeout observes the hang).
 template <bool REAL>
 __device__ __forceinline__ int64_t fi_limit(int64_t golden_trips) {

@@ -66,7 +66,7 @@ __global__ void __launch_bounds__(256) mriq_phimag_kernel(const float* __restric
 // share every k-space load (VPT = 2 in the campaign replicas, 1 for the single-run kernel whose
 // grid is small).
 template <int V, bool EXACT, bool ADD, int VPT>
-__device__ __forceinline__ void mriq_body(const MQParams& p, float4 (*tile)[MQ_TILE], uint64_t* bar) {
+__device__ __forceinline__ void mriq_body(const MQParams& p, float4 (*tile)[MQ_TILE], uint64_t* bar, int bxi) {
   constexpr bool NL = (V & V_NL) != 0, L = (V & V_L) != 0, PROF = (V & V_PROF) != 0;
   constexpr bool CNT = L || PROF;
   const uint32_t z = p.zz;
@@ -78,7 +78,7 @@ __device__ __forceinline__ void mriq_body(const MQParams& p, float4 (*tile)[MQ_T
   int32_t it[VPT];
 #pragma unroll
   for (int v = 0; v < VPT; ++v) {
-    xIndex[v] = blockIdx.x * (blockDim.x * VPT) + v * blockDim.x + threadIdx.x;
+    xIndex[v] = bxi * (blockDim.x * VPT) + v * blockDim.x + threadIdx.x;
     active[v] = xIndex[v] < p.numX;
     chk[v] = 0; alarm[v] = 0;
     sX[v] = sY[v] = sZ[v] = 0.f;
@@ -89,7 +89,7 @@ __device__ __forceinline__ void mriq_body(const MQParams& p, float4 (*tile)[MQ_T
       if (NL) {
         chk[v] ^= (uint32_t)numK ^ lohi_ptr(p.kv) ^ lohi_ptr(p.qr) ^ lohi_ptr(p.qi) ^ lohi_ptr(p.x) ^ lohi_ptr(p.y) ^ lohi_ptr(p.z);
         chk[v] ^= (uint32_t)xi;
-        alarm[v] |= ((int32_t)((blockIdx.x ^ z) * (blockDim.x * VPT) + v * blockDim.x + (threadIdx.x ^ z)) != xi) ? AL_DUP : 0u;
+        alarm[v] |= ((int32_t)((bxi ^ z) * (blockDim.x * VPT) + v * blockDim.x + (threadIdx.x ^ z)) != xi) ? AL_DUP : 0u;
       }
       sX[v] = p.x[xi];
       if (NL) { chk[v] ^= fb(sX[v]); alarm[v] |= (fb(p.x[opq(xi, z)]) != fb(sX[v])) ? AL_DUP : 0u; }
@@ -180,7 +180,7 @@ template <int V, bool EXACT>
 __global__ void __launch_bounds__(256) mriq_kernel(const MQParams p) {
   __shared__ __align__(128) float4 tile[2][MQ_TILE];
   __shared__ __align__(8) uint64_t bar[2];
-  mriq_body<V, EXACT, false, 1>(p, tile, bar);
+  mriq_body<V, EXACT, false, 1>(p, tile, bar, blockIdx.x);
 }
 
 // ============================================================================================
@@ -389,22 +389,27 @@ template <int KIND, bool EXACT>
 __global__ void __launch_bounds__(256) mriq_fi_kernel(const MQFIParams q) {
   __shared__ __align__(128) float4 tile[2][MQ_TILE];
   __shared__ __align__(8) uint64_t bar[2];
-  const int r = blockIdx.y;
+  const int64_t ncta = gridDim.x, vpc = 2 * (int64_t)blockDim.x;
+  int r;
+  int64_t cta;
+  const bool faulted = fi_order((int64_t)blockIdx.y * gridDim.x + blockIdx.x, ncta, (int)gridDim.y,
+                                [&](int rr) { return clamp_cta(q.faults[rr].thread / vpc, ncta); }, &r, &cta);
   const FaultRec f = q.faults[r];
+  const int bxi = (int)cta;
   MQParams p = q.base;
   p.qr = q.out0 + (int64_t)r * q.stride;
   p.qi = p.qr + p.numX;
   p.cb = q.cb0 + r;
   if (KIND == MK_PHIMAG) p.kv = q.kv0 + (int64_t)r * p.numK;  // this replica's (possibly faulted) k-space
-  if (KIND == MK_PHIMAG || f.thread / (2 * blockDim.x) != blockIdx.x) {
-    mriq_body<V_NL | V_L, EXACT, true, 2>(p, tile, bar);
+  if (KIND == MK_PHIMAG || !faulted) {
+    mriq_body<V_NL | V_L, EXACT, true, 2>(p, tile, bar, bxi);
   } else {
     ReplicaSinkF S{{p.qr, p.qi}, p.cb};
 #pragma unroll 1
     for (int vox = 0; vox < 2; ++vox) {
-      const int32_t t = blockIdx.x * (2 * blockDim.x) + vox * blockDim.x + threadIdx.x;
+      const int32_t t = bxi * (2 * blockDim.x) + vox * blockDim.x + threadIdx.x;
       if (t < p.numX) {
-        const int32_t t_dup = (int32_t)((blockIdx.x ^ p.zz) * (2 * blockDim.x) + vox * blockDim.x + (threadIdx.x ^ p.zz));
+        const int32_t t_dup = (int32_t)((bxi ^ p.zz) * (2 * blockDim.x) + vox * blockDim.x + (threadIdx.x ^ p.zz));
         mriq_fi_program<KIND, EXACT>(p, f, t, t_dup, t == f.thread, (uint64_t)(uintptr_t)p.qr, (uint64_t)(uintptr_t)p.qi, S);
       }
     }

@@ -125,8 +125,8 @@ __device__ __forceinline__ TPSmem tp_carve(unsigned char* base, int C) {
 }
 
 // Does any thread of this CTA have partners?  (self rows: chunks left of the diagonal are empty)
-__device__ __forceinline__ bool tp_cta_has_work(const TPParams& p, int h, int c) {
-  const int i0 = blockIdx.x * TP_CTA_PTS;
+__device__ __forceinline__ bool tp_cta_has_work(const TPParams& p, int h, int c, int bxi) {
+  const int i0 = bxi * TP_CTA_PTS;
   const int jb = (h <= p.nr) ? max(i0 + 1, c * p.C) : c * p.C;
   const int je = min((c + 1) * p.C, p.n);
   return i0 < p.n && je > jb;
@@ -171,20 +171,20 @@ struct TPPoint {
 };
 
 template <bool NL>
-__device__ __forceinline__ TPPoint tp_prologue(const TPParams& p, const unsigned long long* hist, int k) {
+__device__ __forceinline__ TPPoint tp_prologue(const TPParams& p, const unsigned long long* hist, int k, int bxi, int byi) {
   const uint32_t z = p.z;
   const int32_t n = p.n, nr = p.nr, C = p.C, nC = p.nC, nb2 = p.nb + 2;
   TPPoint P;
-  P.row = blockIdx.y;
-  P.i = blockIdx.x * TP_CTA_PTS + k * TP_THREADS + threadIdx.x;
+  P.row = byi;
+  P.i = bxi * TP_CTA_PTS + k * TP_THREADS + threadIdx.x;
   const int32_t h = P.row / nC, c = P.row - h * nC;
   P.chk = 0;
   P.alarm = 0;
   if (NL) {
     P.chk ^= (uint32_t)n ^ lohi_ptr(p.pts) ^ lohi_ptr(hist);
     P.chk ^= (uint32_t)P.i;
-    P.alarm |= ((int32_t)((blockIdx.x ^ z) * TP_CTA_PTS + k * TP_THREADS + (threadIdx.x ^ z)) != P.i) ? AL_DUP : 0u;
-    P.chk ^= (uint32_t)h; P.alarm |= ((int32_t)(blockIdx.y ^ z) / nC != h) ? AL_DUP : 0u;
+    P.alarm |= ((int32_t)((bxi ^ z) * TP_CTA_PTS + k * TP_THREADS + (threadIdx.x ^ z)) != P.i) ? AL_DUP : 0u;
+    P.chk ^= (uint32_t)h; P.alarm |= ((int32_t)(byi ^ z) / nC != h) ? AL_DUP : 0u;
     P.chk ^= (uint32_t)c; P.alarm |= ((int32_t)(P.row - opq(h, z) * nC) != c) ? AL_DUP : 0u;
   }
   const int32_t aoff = (h <= nr ? h : 0) * n + P.i;
@@ -310,20 +310,21 @@ __device__ __forceinline__ void tp_loops(const TPParams& p, const TPSmem& S, uin
 }
 
 template <int V>
-__device__ __forceinline__ void tpacf_body(const TPParams& p, const TPSmem& S, unsigned long long* hist, hk_control* cb) {
+__device__ __forceinline__ void tpacf_body(const TPParams& p, const TPSmem& S, unsigned long long* hist, hk_control* cb,
+                                           int bxi, int byi) {
   constexpr bool NL = (V & V_NL) != 0, L = (V & V_L) != 0;
   const int32_t nr = p.nr, nC = p.nC, nb2 = p.nb + 2;
-  const int32_t row = blockIdx.y;
+  const int32_t row = byi;
   const int32_t h = row / nC, c = row - h * nC;
   const int32_t sb = (h == 0) ? 0 : (h <= nr ? h : h - nr);
-  const bool work = tp_cta_has_work(p, h, c);
+  const bool work = tp_cta_has_work(p, h, c, bxi);
   const bool use_lut = *p.lut_ok != 0;
   tp_stage(p, S, sb, c, work);
   __syncthreads();
   const uint32_t lane = lane_id(), warp = threadIdx.x >> 5;
   uint32_t* Hw = S.H + (size_t)warp * nb2 * 32 + lane;
-  TPPoint A = tp_prologue<NL>(p, hist, 0);
-  TPPoint B = tp_prologue<NL>(p, hist, 1);
+  TPPoint A = tp_prologue<NL>(p, hist, 0, bxi, byi);
+  TPPoint B = tp_prologue<NL>(p, hist, 1, bxi, byi);
   const bool va = A.i < p.n, vb = B.i < p.n;
   if (use_lut) tp_loops<V, true>(p, S, Hw, A, B, va, vb);
   else tp_loops<V, false>(p, S, Hw, A, B, va, vb);
@@ -345,7 +346,7 @@ template <int V>
 __global__ void __launch_bounds__(TP_THREADS) tpacf_kernel(const TPParams p) {
   extern __shared__ __align__(16) unsigned char tp_smem[];
   const TPSmem S = tp_carve(tp_smem, p.C);
-  tpacf_body<V>(p, S, p.hist, p.cb);
+  tpacf_body<V>(p, S, p.hist, p.cb, blockIdx.x, blockIdx.y);
 }
 
 // ============================================================================================
@@ -546,21 +547,21 @@ done:
 // The CTA that holds the faulted abstract thread: every thread runs the per-thread program.
 template <int KIND, bool REAL>
 __device__ __forceinline__ void tpacf_fi_cta(const TPFIParams& q, const TPSmem& S, const FaultRec& f,
-                                             unsigned long long* hist, hk_control* cb) {
+                                             unsigned long long* hist, hk_control* cb, int bxi, int byi) {
   {
     const TPParams& p = q.base;
-    const int32_t h = blockIdx.y / p.nC, c = blockIdx.y - h * p.nC;
+    const int32_t h = byi / p.nC, c = byi - h * p.nC;
     const int32_t sb = (h == 0) ? 0 : (h <= p.nr ? h : h - p.nr);
     tp_stage(p, S, sb, c, true);
     __syncthreads();
     TPReplicaSink K{hist, cb, S.H, p.nb + 2};
 #pragma unroll 1
     for (int kpt = 0; kpt < 2; ++kpt) {
-      const int32_t ii = blockIdx.x * TP_CTA_PTS + kpt * TP_THREADS + threadIdx.x;
+      const int32_t ii = bxi * TP_CTA_PTS + kpt * TP_THREADS + threadIdx.x;
       if (ii < p.n) {
-        const int32_t idup = (int32_t)((blockIdx.x ^ p.z) * TP_CTA_PTS + kpt * TP_THREADS + (threadIdx.x ^ p.z));
-        const int64_t g = (int64_t)blockIdx.y * p.n + ii;
-        tpacf_fi_program<KIND, REAL>(p, S, f, (int32_t)blockIdx.y, ii, idup, (int32_t)(blockIdx.y ^ p.z),
+        const int32_t idup = (int32_t)((bxi ^ p.z) * TP_CTA_PTS + kpt * TP_THREADS + (threadIdx.x ^ p.z));
+        const int64_t g = (int64_t)byi * p.n + ii;
+        tpacf_fi_program<KIND, REAL>(p, S, f, (int32_t)byi, ii, idup, (int32_t)((uint32_t)byi ^ p.z),
                                      g == f.thread, (uint64_t)(uintptr_t)hist, K);
       }
     }
@@ -573,13 +574,21 @@ template <int KIND>
 __global__ void __launch_bounds__(TP_THREADS) tpacf_fi_kernel(const TPFIParams q) {
   extern __shared__ __align__(16) unsigned char tp_smem[];
   const TPSmem S = tp_carve(tp_smem, q.base.C);
-  const int r = blockIdx.z;
+  const int64_t gx = gridDim.x, ncta = gx * gridDim.y, n = q.base.n;
+  int r;
+  int64_t cta;
+  const bool faulted = fi_order(((int64_t)blockIdx.z * gridDim.y + blockIdx.y) * gx + blockIdx.x, ncta, (int)gridDim.z,
+                                [&](int rr) {
+                                  const int64_t g = q.faults[rr].thread;
+                                  return clamp_cta((g / n) * gx + (g % n) / TP_CTA_PTS, ncta);
+                                },
+                                &r, &cta);
   const FaultRec f = q.faults[r];
   unsigned long long* hist = q.hist0 + (int64_t)r * q.hist_elems;
   hk_control* cb = q.cb0 + r;
-  const int64_t cta_first = (int64_t)blockIdx.y * q.base.n + (int64_t)blockIdx.x * TP_CTA_PTS;
-  if (f.thread < cta_first || f.thread >= cta_first + TP_CTA_PTS) tpacf_body<V_NL | V_L>(q.base, S, hist, cb);
-  else tpacf_fi_cta<KIND, false>(q, S, f, hist, cb);
+  const int bxi = (int)(cta % gx), byi = (int)(cta / gx);
+  if (!faulted) tpacf_body<V_NL | V_L>(q.base, S, hist, cb, bxi, byi);
+  else tpacf_fi_cta<KIND, false>(q, S, f, hist, cb, bxi, byi);
 }
 
 // Unguarded replicas for the guardian (campaign mode 2, DESIGN R25): every CTA runs the per-thread
@@ -592,7 +601,7 @@ __global__ void __launch_bounds__(TP_THREADS) tpacf_real_kernel(const TPFIParams
   unsigned long long* hist = q.hist0 + (int64_t)r * q.hist_elems;
   hk_control* cb = q.cb0 + r;
   switch (kind) {
-#define K(k) case k: tpacf_fi_cta<k, true>(q, S, f, hist, cb); break;
+#define K(k) case k: tpacf_fi_cta<k, true>(q, S, f, hist, cb, blockIdx.x, blockIdx.y); break;
     K(TK_NL) K(TK_LIVE) K(TK_J) K(TK_X2) K(TK_Y2) K(TK_Z2) K(TK_DOT) K(TK_BIN) K(TK_HIDX) K(TK_ACC) K(TK_CNT)
 #undef K
     default: break;

@@ -171,10 +171,16 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    # one process per GPU; HK_DIST_BACKEND=gloo (test only) lets a multi-rank run share one GPU
+    backend = os.environ.get("HK_DIST_BACKEND", "nccl")
+    gpu = local % torch.cuda.device_count() if backend != "nccl" else local
+    torch.cuda.set_device(gpu)
+    dev = torch.device("cuda", gpu)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
     hk.lib()
     sm_mhz_peak, clk_src = peaks()
     mufu_peak = N_SM * MUFU_PER_SM_CLK * sm_mhz_peak * 1e6
@@ -242,7 +248,7 @@ def main():
         flush.zero_()
         step(args.steps + 1000 + s, scratch)  # warm-up slices outside the timed index range
     torch.cuda.synchronize()
-    clocks = Clocks(local)
+    clocks = Clocks(gpu)
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     if world > 1:
         dist.barrier()

@@ -12,7 +12,10 @@
 
 namespace hk {
 
-constexpr int TP_THREADS = 256;
+#ifndef HK_TP_THREADS
+#define HK_TP_THREADS 256
+#endif
+constexpr int TP_THREADS = HK_TP_THREADS;
 constexpr int TP_CTA_PTS = 2 * TP_THREADS;  // two abstract threads per CUDA thread
 constexpr int TP_WARPS = TP_THREADS / 32;
 
@@ -346,7 +349,12 @@ template <int V>
 __global__ void __launch_bounds__(TP_THREADS) tpacf_kernel(const TPParams p) {
   extern __shared__ __align__(16) unsigned char tp_smem[];
   const TPSmem S = tp_carve(tp_smem, p.C);
+#ifdef HK_TP_REV
+  const int L = (int)(gridDim.x * gridDim.y) - 1 - (int)(blockIdx.y * gridDim.x + blockIdx.x);
+  tpacf_body<V>(p, S, p.hist, p.cb, L % gridDim.x, L / gridDim.x);
+#else
   tpacf_body<V>(p, S, p.hist, p.cb, blockIdx.x, blockIdx.y);
+#endif
 }
 
 // ============================================================================================

@@ -15,6 +15,7 @@ __global__ void k(float* out, float seed, long long* cyc) {
 #define F(x) asm volatile("fma.rn.f32 %0, %0, %0, %0;" : "+f"(x))
 #define I(x) asm volatile("add.u32 %0, %0, %1;" : "+r"(x) : "r"(x))
 #define E(x) asm volatile("ex2.approx.ftz.f32 %0, %0;" : "+f"(x))
+#define N(x) asm volatile("cvt.rni.f32.f32 %0, %0;" : "+f"(x))
     if (OP == 0) { R(a0); R(a1); R(a2); R(a3); R(a4); R(a5); R(a6); R(a7); }
     if (OP == 1) { S(a0); S(a1); S(a2); S(a3); S(a4); S(a5); S(a6); S(a7); }
     if (OP == 2) { F(a0); F(a1); F(a2); F(a3); F(a4); F(a5); F(a6); F(a7); }
@@ -22,6 +23,8 @@ __global__ void k(float* out, float seed, long long* cyc) {
     if (OP == 4) { E(a0); E(a1); E(a2); E(a3); E(a4); E(a5); E(a6); E(a7); }
     if (OP == 5) { R(a0); F(a1); F(a2); F(a3); R(a4); F(a5); F(a6); F(a7); }
     if (OP == 6) { R(a0); R(a1); I(u2); I(u3); R(a4); R(a5); I(u6); I(u7); }
+    if (OP == 7) { N(a0); N(a1); N(a2); N(a3); N(a4); N(a5); N(a6); N(a7); }
+    if (OP == 8) { S(a0); N(a1); N(a2); N(a3); S(a4); N(a5); N(a6); N(a7); }
   }
   long long t1 = clock64();
   if (threadIdx.x == 0) cyc[blockIdx.x] = t1 - t0;
@@ -48,5 +51,6 @@ int main() {
   printf("{\"sms\":%d,\"clock_khz\":%d}\n", sms, clk);
   run<0>("rsqrt", sms); run<1>("sin", sms); run<2>("ffma", sms); run<3>("iadd", sms); run<4>("ex2", sms);
   run<0>("rsqrt", sms); run<1>("sin", sms); run<2>("ffma", sms); run<5>("mix_2rsq_6ffma", sms); run<6>("mix_4rsq_4iadd", sms);
+  run<7>("frnd", sms); run<8>("mix_2sin_6frnd", sms);
   return 0;
 }

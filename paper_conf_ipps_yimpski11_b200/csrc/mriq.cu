@@ -10,6 +10,18 @@
 namespace hk {
 
 constexpr int MQ_TILE = 1024;  // k-samples per stage (16 KB)
+#ifndef HK_MQ_FI_THREADS
+#define HK_MQ_FI_THREADS 256
+#endif
+#ifndef HK_MQ_FI_VPT
+#define HK_MQ_FI_VPT 2
+#endif
+#ifndef HK_MQ_FI_UNROLL
+#define HK_MQ_FI_UNROLL 8
+#endif
+constexpr int MQ_FI_THREADS = HK_MQ_FI_THREADS;  // campaign replicas: CTA size
+constexpr int MQ_FI_VPT = HK_MQ_FI_VPT;          // voxels per CUDA thread in the replicas
+constexpr int MQ_FI_UNROLL = HK_MQ_FI_UNROLL;
 constexpr float RINT_MAGIC = 12582912.0f;  // 1.5 * 2^23
 constexpr float TWO_PI_F = 6.28318548202514648f;
 
@@ -121,7 +133,7 @@ __device__ __forceinline__ void mriq_body(const MQParams& p, float4 (*tile)[MQ_T
     if (any_active) {
       const float4* A = tile[buf];
       const int cnt = min(MQ_TILE, numK - t * MQ_TILE);
-#pragma unroll(VPT == 1 ? 4 : 2)
+#pragma unroll(VPT == 1 ? 4 : MQ_FI_UNROLL)
       for (int a = 0; a < cnt; ++a) {
         const float4 k4 = A[a];
 #pragma unroll
@@ -386,10 +398,10 @@ done:
 }
 
 template <int KIND, bool EXACT>
-__global__ void __launch_bounds__(256) mriq_fi_kernel(const MQFIParams q) {
+__global__ void __launch_bounds__(MQ_FI_THREADS) mriq_fi_kernel(const MQFIParams q) {
   __shared__ __align__(128) float4 tile[2][MQ_TILE];
   __shared__ __align__(8) uint64_t bar[2];
-  const int64_t ncta = gridDim.x, vpc = 2 * (int64_t)blockDim.x;
+  const int64_t ncta = gridDim.x, vpc = MQ_FI_VPT * (int64_t)blockDim.x;
   int r;
   int64_t cta;
   const bool faulted = fi_order((int64_t)blockIdx.y * gridDim.x + blockIdx.x, ncta, (int)gridDim.y,
@@ -402,14 +414,14 @@ __global__ void __launch_bounds__(256) mriq_fi_kernel(const MQFIParams q) {
   p.cb = q.cb0 + r;
   if (KIND == MK_PHIMAG) p.kv = q.kv0 + (int64_t)r * p.numK;  // this replica's (possibly faulted) k-space
   if (KIND == MK_PHIMAG || !faulted) {
-    mriq_body<V_NL | V_L, EXACT, true, 2>(p, tile, bar, bxi);
+    mriq_body<V_NL | V_L, EXACT, true, MQ_FI_VPT>(p, tile, bar, bxi);
   } else {
     ReplicaSinkF S{{p.qr, p.qi}, p.cb};
 #pragma unroll 1
-    for (int vox = 0; vox < 2; ++vox) {
-      const int32_t t = bxi * (2 * blockDim.x) + vox * blockDim.x + threadIdx.x;
+    for (int vox = 0; vox < MQ_FI_VPT; ++vox) {
+      const int32_t t = bxi * (MQ_FI_VPT * blockDim.x) + vox * blockDim.x + threadIdx.x;
       if (t < p.numX) {
-        const int32_t t_dup = (int32_t)((bxi ^ p.zz) * (2 * blockDim.x) + vox * blockDim.x + (threadIdx.x ^ p.zz));
+        const int32_t t_dup = (int32_t)((bxi ^ p.zz) * (MQ_FI_VPT * blockDim.x) + vox * blockDim.x + (threadIdx.x ^ p.zz));
         mriq_fi_program<KIND, EXACT>(p, f, t, t_dup, t == f.thread, (uint64_t)(uintptr_t)p.qr, (uint64_t)(uintptr_t)p.qi, S);
       }
     }
@@ -557,9 +569,10 @@ int mriq_site_kind(int site) { return mriq_site_kind_d(site); }
 
 template <int KIND, bool EXACT>
 static cudaError_t launch_mq_fi_k(const MQFIParams& q, int nrep, cudaStream_t s) {
-  dim3 grid((q.base.numX + 511) / 512, nrep);
+  constexpr int vpc = MQ_FI_VPT * MQ_FI_THREADS;
+  dim3 grid((q.base.numX + vpc - 1) / vpc, nrep);
   TimedScope ts(HK_MRIQ, 1, (double)q.base.numX * (double)q.base.numK * nrep, s);
-  mriq_fi_kernel<KIND, EXACT><<<grid, 256, 0, s>>>(q);
+  mriq_fi_kernel<KIND, EXACT><<<grid, MQ_FI_THREADS, 0, s>>>(q);
   count_launch();
   return cudaGetLastError();
 }

@@ -13,7 +13,7 @@
 namespace hk {
 
 #ifndef HK_TP_THREADS
-#define HK_TP_THREADS 256
+#define HK_TP_THREADS 128
 #endif
 constexpr int TP_THREADS = HK_TP_THREADS;
 constexpr int TP_CTA_PTS = 2 * TP_THREADS;  // two abstract threads per CUDA thread

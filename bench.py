@@ -344,7 +344,7 @@ def main():
         cr = torch.zeros((3, 5), dtype=torch.int64, device=dev)
         with hk.CampaignSession(-1, devs, ranges, seed, mode=1) as sr:
             first, cnt = par.shard(args.replay_count * world, rank, world)
-            sr.run(0, min(3000, cnt), torch.zeros((3, 5), dtype=torch.int64, device=dev))  # warm-up
+            sr.run(first, cnt, torch.zeros((3, 5), dtype=torch.int64, device=dev))  # warm-up at full size (workspaces grow on first use)
             torch.cuda.synchronize()
             if world > 1:
                 dist.barrier()

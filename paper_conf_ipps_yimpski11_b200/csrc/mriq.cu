@@ -22,6 +22,10 @@ constexpr int MQ_TILE = 1024;  // k-samples per stage (16 KB)
 constexpr int MQ_FI_THREADS = HK_MQ_FI_THREADS;  // campaign replicas: CTA size
 constexpr int MQ_FI_VPT = HK_MQ_FI_VPT;          // voxels per CUDA thread in the replicas
 constexpr int MQ_FI_UNROLL = HK_MQ_FI_UNROLL;
+#ifndef HK_MQ_UNROLL
+#define HK_MQ_UNROLL 16
+#endif
+constexpr int MQ_UNROLL = HK_MQ_UNROLL;  // single-run kernel (one voxel per thread)
 constexpr float RINT_MAGIC = 12582912.0f;  // 1.5 * 2^23
 constexpr float TWO_PI_F = 6.28318548202514648f;
 
@@ -133,7 +137,7 @@ __device__ __forceinline__ void mriq_body(const MQParams& p, float4 (*tile)[MQ_T
     if (any_active) {
       const float4* A = tile[buf];
       const int cnt = min(MQ_TILE, numK - t * MQ_TILE);
-#pragma unroll(VPT == 1 ? 4 : MQ_FI_UNROLL)
+#pragma unroll(VPT == 1 ? MQ_UNROLL : MQ_FI_UNROLL)
       for (int a = 0; a < cnt; ++a) {
         const float4 k4 = A[a];
 #pragma unroll

@@ -8,6 +8,13 @@
 // memory (distinct entries sit in distinct banks); lane-private shared histograms [warp][bin][lane]
 // (bank = lane: conflict-free), reduced per CTA and flushed with one u64 atomic per (warp, bin).
 // Loop detector: accumulator acc += bin and counter cnt++ (the "two addition instructions", L679-680).
+#include <algorithm>
+#include <array>
+#include <map>
+#include <mutex>
+#include <queue>
+#include <vector>
+
 #include "hk_internal.h"
 
 namespace hk {
@@ -16,6 +23,14 @@ namespace hk {
 #define HK_TP_THREADS 128
 #endif
 constexpr int TP_THREADS = HK_TP_THREADS;
+// Minimum resident CTAs per SM for the register allocator (measured, tools/ab_time.py): the
+// replicas run fastest at 9 (56 registers), the single run at 10.
+#ifndef HK_TP_MINB
+#define HK_TP_MINB 9
+#endif
+#ifndef HK_TP_STD_MINB
+#define HK_TP_STD_MINB 10
+#endif
 constexpr int TP_CTA_PTS = 2 * TP_THREADS;  // two abstract threads per CUDA thread
 constexpr int TP_WARPS = TP_THREADS / 32;
 
@@ -47,6 +62,7 @@ struct TPParams {
 //    under every compare).  2 loads + 5 ops per pair.
 // ---------------------------------------------------------------------------------------------
 constexpr int TP_LUT = 2048;
+constexpr int TP_SCHED_MAX_SM = 1024;
 
 __device__ __forceinline__ int32_t tp_bin(const float* Es, float dot) {
   int32_t b = 0;
@@ -345,16 +361,53 @@ __device__ __forceinline__ void tpacf_body(const TPParams& p, const TPSmem& S, u
   }
 }
 
+// Single-run schedule.  At the configs' sizes the single run is one wave whose CTAs carry very
+// different work (full chunks, diagonal triangles, empty chunks left of the diagonal), so the
+// block scheduler's placement left the busiest SM with ~1.3x the mean work (ncu
+// sm__cycles_active max/avg).  The host assigns the (point block, row) work items to SMs by
+// longest-processing-time greedy on their exact pair counts; a persistent grid of k CTAs per SM
+// claims the items of its own SM's list (%smid) and, once that list is drained, steals from the
+// other lists, so every item runs exactly once whatever the placement.  Same abstract threads,
+// same per-thread order: only which CTA runs an item changes.
+struct TPSched {
+  const int2* items;  // (bxi, row), grouped by SM
+  const int* off;     // [nsm + 1] list offsets
+  int* next;          // [nsm] claim counters (zeroed per run)
+  int* claimed;       // items claimed so far (zeroed per run)
+  int nsm, total;
+};
+
 template <int V>
-__global__ void __launch_bounds__(TP_THREADS) tpacf_kernel(const TPParams p) {
+__global__ void __launch_bounds__(TP_THREADS, HK_TP_STD_MINB) tpacf_kernel(const TPParams p, const TPSched q) {
   extern __shared__ __align__(16) unsigned char tp_smem[];
+  __shared__ int item_s;
   const TPSmem S = tp_carve(tp_smem, p.C);
-#ifdef HK_TP_REV
-  const int L = (int)(gridDim.x * gridDim.y) - 1 - (int)(blockIdx.y * gridDim.x + blockIdx.x);
-  tpacf_body<V>(p, S, p.hist, p.cb, L % gridDim.x, L / gridDim.x);
-#else
-  tpacf_body<V>(p, S, p.hist, p.cb, blockIdx.x, blockIdx.y);
-#endif
+  uint32_t smid;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+  int sl = (int)(smid % (uint32_t)q.nsm), probes = 0;
+  for (;;) {
+    if (threadIdx.x == 0) {
+      int it = -1;
+      while (probes < q.nsm) {
+        const int k = atomicAdd(q.next + sl, 1);
+        if (q.off[sl] + k < q.off[sl + 1]) {
+          it = q.off[sl] + k;
+          atomicAdd(q.claimed, 1);
+          break;
+        }
+        if (*(volatile int*)q.claimed >= q.total) break;  // everything is taken
+        sl = (sl + 1 == q.nsm) ? 0 : sl + 1;
+        ++probes;
+      }
+      item_s = it;
+    }
+    __syncthreads();
+    const int it = item_s;
+    if (it < 0) break;
+    const int2 xy = q.items[it];
+    tpacf_body<V>(p, S, p.hist, p.cb, xy.x, xy.y);
+    __syncthreads();  // smem (and item_s) reused by the next item
+  }
 }
 
 // ============================================================================================
@@ -579,7 +632,7 @@ __device__ __forceinline__ void tpacf_fi_cta(const TPFIParams& q, const TPSmem& 
 }
 
 template <int KIND>
-__global__ void __launch_bounds__(TP_THREADS) tpacf_fi_kernel(const TPFIParams q) {
+__global__ void __launch_bounds__(TP_THREADS, HK_TP_MINB) tpacf_fi_kernel(const TPFIParams q) {
   extern __shared__ __align__(16) unsigned char tp_smem[];
   const TPSmem S = tp_carve(tp_smem, q.base.C);
   const int64_t gx = gridDim.x, ncta = gx * gridDim.y, n = q.base.n;
@@ -715,11 +768,14 @@ static TPParams tp_params(const hk_tpacf_args& a, const DevRanges& R, int ndet, 
   return p;
 }
 
-size_t tpacf_lut_ws_bytes() { return TP_LUT + 16; }
+// workspace: bucket table | ok flag (16 B) | single-run schedule counters next[TP_SCHED_MAX_SM], claimed
+size_t tpacf_lut_ws_bytes() { return TP_LUT + 16 + (TP_SCHED_MAX_SM + 1) * sizeof(int); }
 
 cudaError_t tpacf_lut_build(const hk_tpacf_args& a, void* lut_ws, cudaStream_t s) {
   int* ok = reinterpret_cast<int*>(reinterpret_cast<char*>(lut_ws) + TP_LUT);
   cudaError_t e = cudaMemsetAsync(ok, 1, sizeof(int), s);
+  if (e != cudaSuccess) return e;
+  e = cudaMemsetAsync(reinterpret_cast<char*>(lut_ws) + TP_LUT + 16, 0, (TP_SCHED_MAX_SM + 1) * sizeof(int), s);
   if (e != cudaSuccess) return e;
   tpacf_lut_kernel<<<TP_LUT / 256, 256, 0, s>>>(a.edges, a.n_bins, reinterpret_cast<uint8_t*>(lut_ws), ok);
   count_launch();
@@ -731,15 +787,89 @@ static double tp_pairs(const TPParams& p) {
   return (1 + p.nr) * n * (n - 1) / 2 + p.nr * n * n;
 }
 
+// Host side of the single-run schedule: exact pair count per (point block, row) work item,
+// LPT assignment to the SMs, cached per (shape, SM count, device).
+struct TPSchedBuf {
+  int2* items = nullptr;
+  int* off = nullptr;
+  int total = 0;
+};
+static cudaError_t tp_schedule(const TPParams& p, int nsm, TPSchedBuf* out) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  static std::mutex mu;
+  static std::map<std::array<int, 5>, TPSchedBuf> cache;
+  const std::array<int, 5> key{p.n, p.nr, p.C, nsm, dev};
+  std::lock_guard<std::mutex> lk(mu);
+  auto f = cache.find(key);
+  if (f != cache.end()) { *out = f->second; return cudaSuccess; }
+  const int gx = (p.n + TP_CTA_PTS - 1) / TP_CTA_PTS, gy = (1 + 2 * p.nr) * p.nC;
+  std::vector<std::pair<double, int2>> w;
+  w.reserve((size_t)gx * gy);
+  for (int row = 0; row < gy; ++row) {
+    const int h = row / p.nC, c = row - h * p.nC;
+    const int64_t cb = (int64_t)c * p.C, ce = std::min<int64_t>(cb + p.C, p.n);
+    for (int b = 0; b < gx; ++b) {
+      const int64_t i0 = (int64_t)b * TP_CTA_PTS, i1 = std::min<int64_t>(i0 + TP_CTA_PTS, p.n);
+      double pairs = 0;
+      for (int64_t i = i0; i < i1; ++i) pairs += (double)std::max<int64_t>(0, ce - (h <= p.nr ? std::max(i + 1, cb) : cb));
+      // + the per-abstract-thread prologue/epilogue (~64 pair-equivalents) that even empty items run
+      w.push_back({pairs + 64.0 * (double)(i1 - i0), make_int2(b, row)});
+    }
+  }
+  std::stable_sort(w.begin(), w.end(), [](const auto& a, const auto& b) { return a.first > b.first; });
+  std::vector<std::vector<int2>> lists(nsm);
+  std::priority_queue<std::pair<double, int>, std::vector<std::pair<double, int>>, std::greater<>> load;
+  for (int m = 0; m < nsm; ++m) load.push({0.0, m});
+  for (const auto& it : w) {
+    auto top = load.top();
+    load.pop();
+    lists[top.second].push_back(it.second);
+    load.push({top.first + it.first, top.second});
+  }
+  std::vector<int2> items;
+  std::vector<int> off(nsm + 1, 0);
+  for (int m = 0; m < nsm; ++m) {
+    off[m] = (int)items.size();
+    items.insert(items.end(), lists[m].begin(), lists[m].end());
+  }
+  off[nsm] = (int)items.size();
+  TPSchedBuf B;
+  B.total = (int)items.size();
+  if ((e = cudaMalloc(&B.items, sizeof(int2) * std::max<size_t>(1, items.size()))) != cudaSuccess) return e;
+  if ((e = cudaMalloc(&B.off, sizeof(int) * off.size())) != cudaSuccess) return e;
+  if (!items.empty() && (e = cudaMemcpy(B.items, items.data(), sizeof(int2) * items.size(), cudaMemcpyHostToDevice)) != cudaSuccess)
+    return e;
+  if ((e = cudaMemcpy(B.off, off.data(), sizeof(int) * off.size(), cudaMemcpyHostToDevice)) != cudaSuccess) return e;
+  cache[key] = B;
+  *out = B;
+  return cudaSuccess;
+}
+
 template <int V>
-static cudaError_t launch_tp_v(const TPParams& p, cudaStream_t s) {
+static cudaError_t launch_tp_v(const TPParams& p, void* lut_ws, cudaStream_t s) {
   const size_t smem = tp_smem_bytes(p.C, p.nb + 2);
   cudaError_t e = cudaFuncSetAttribute(tpacf_kernel<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  dim3 grid((p.n + TP_CTA_PTS - 1) / TP_CTA_PTS, (1 + 2 * p.nr) * p.nC);
-  if (grid.x == 0) return cudaSuccess;
+  if (p.n <= 0) return cudaSuccess;
+  int dev = 0, nsm = 0, per_sm = 0;
+  if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
+  if ((e = cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess) return e;
+  if (nsm > TP_SCHED_MAX_SM) return cudaErrorInvalidValue;
+  if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tpacf_kernel<V>, TP_THREADS, smem)) != cudaSuccess) return e;
+  TPSchedBuf B;
+  if ((e = tp_schedule(p, nsm, &B)) != cudaSuccess) return e;
+  TPSched q;
+  q.items = B.items;
+  q.off = B.off;
+  q.next = reinterpret_cast<int*>(reinterpret_cast<char*>(lut_ws) + TP_LUT + 16);
+  q.claimed = q.next + TP_SCHED_MAX_SM;
+  q.nsm = nsm;
+  q.total = B.total;
+  const int grid = nsm * std::max(1, std::min(per_sm, (B.total + nsm - 1) / nsm));
   TimedScope ts(HK_TPACF, 0, tp_pairs(p), s);
-  tpacf_kernel<V><<<grid, TP_THREADS, smem, s>>>(p);
+  tpacf_kernel<V><<<grid, TP_THREADS, smem, s>>>(p, q);
   count_launch();
   return cudaGetLastError();
 }
@@ -750,11 +880,11 @@ cudaError_t tpacf_launch(int vflags, const hk_tpacf_args& a, const DevRanges& R,
   if (e != cudaSuccess) return e;
   const TPParams p = tp_params(a, R, ndet, cb, samples, lut_ws);
   switch (vflags) {
-    case 0: return launch_tp_v<0>(p, s);
-    case V_NL | V_L: return launch_tp_v<V_NL | V_L>(p, s);
-    case V_NL: return launch_tp_v<V_NL>(p, s);
-    case V_L: return launch_tp_v<V_L>(p, s);
-    case V_PROF: return launch_tp_v<V_PROF>(p, s);
+    case 0: return launch_tp_v<0>(p, lut_ws, s);
+    case V_NL | V_L: return launch_tp_v<V_NL | V_L>(p, lut_ws, s);
+    case V_NL: return launch_tp_v<V_NL>(p, lut_ws, s);
+    case V_L: return launch_tp_v<V_L>(p, lut_ws, s);
+    case V_PROF: return launch_tp_v<V_PROF>(p, lut_ws, s);
   }
   return cudaErrorInvalidValue;
 }

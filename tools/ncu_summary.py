@@ -19,6 +19,11 @@ KEYS = [
     ("sm__warps_active.avg.pct_of_peak_sustained_active", "achieved occupancy %"),
     ("launch__registers_per_thread", "registers"),
     ("launch__grid_size", "grid"),
+    ("sm__cycles_active.avg", "sm cycles active avg"),
+    ("sm__cycles_active.max", "sm cycles active max"),
+    ("smsp__average_warp_latency_issue_stalled_mio_throttle", "stall mio_throttle"),
+    ("smsp__average_warp_latency_issue_stalled_short_scoreboard", "stall short_scoreboard"),
+    ("smsp__average_warp_latency_issue_stalled_wait", "stall wait"),
     ("smsp__inst_executed.sum", "warp instructions"),
 ]
 

@@ -867,6 +867,9 @@ static cudaError_t launch_tp_v(const TPParams& p, void* lut_ws, cudaStream_t s) 
   q.claimed = q.next + TP_SCHED_MAX_SM;
   q.nsm = nsm;
   q.total = B.total;
+#ifdef HK_TP_STD_CTAS
+  per_sm = std::min(per_sm, HK_TP_STD_CTAS);
+#endif
   const int grid = nsm * std::max(1, std::min(per_sm, (B.total + nsm - 1) / nsm));
   TimedScope ts(HK_TPACF, 0, tp_pairs(p), s);
   tpacf_kernel<V><<<grid, TP_THREADS, smem, s>>>(p, q);

@@ -124,22 +124,26 @@ __global__ void tpacf_lut_kernel(const float* __restrict__ edges, int nb, uint8_
   if (!good) atomicExch(ok, 0);
 }
 
-// Dynamic shared memory: E[32] | LUT[2048] u8 | B[C] float4 | H[warps][nb2][32] u32
+// Dynamic shared memory: E[32] | LUT[2048] u8 | B[3 * C4] float (packed x, y, z) | H[warps][nb2][32] u32
+// The partner tile keeps the global AoS layout without padding: 4 partners = 3 float4, i.e. three
+// 128-bit broadcast loads (2 wavefronts each) per 4 partners instead of four (ncu source page:
+// LDS.128 costs 2.1 wavefronts even as a broadcast).
+__host__ __device__ inline int tp_c4(int C) { return (C + 3) & ~3; }
 struct TPSmem {
   float* E;
   uint8_t* L;
-  float4* B;
+  float* B;
   uint32_t* H;
 };
 __host__ __device__ inline size_t tp_smem_bytes(int C, int nb2) {
-  return 32 * sizeof(float) + TP_LUT + (size_t)C * sizeof(float4) + (size_t)TP_WARPS * nb2 * 32 * 4;
+  return 32 * sizeof(float) + TP_LUT + (size_t)tp_c4(C) * 12 + (size_t)TP_WARPS * nb2 * 32 * 4;
 }
 __device__ __forceinline__ TPSmem tp_carve(unsigned char* base, int C) {
   TPSmem S;
   S.E = reinterpret_cast<float*>(base);
   S.L = base + 128;
-  S.B = reinterpret_cast<float4*>(base + 128 + TP_LUT);
-  S.H = reinterpret_cast<uint32_t*>(base + 128 + TP_LUT + (size_t)C * sizeof(float4));
+  S.B = reinterpret_cast<float*>(base + 128 + TP_LUT);
+  S.H = reinterpret_cast<uint32_t*>(base + 128 + TP_LUT + (size_t)tp_c4(C) * 12);
   return S;
 }
 
@@ -161,7 +165,7 @@ __device__ __forceinline__ void tp_stage(const TPParams& p, const TPSmem& S, int
   const int j0 = c * p.C;
   const int cnt = min(p.C, p.n - j0);
   const float* P = p.pts + 3 * ((int64_t)sb * p.n + j0);
-  for (int k = threadIdx.x; k < cnt; k += TP_THREADS) S.B[k] = make_float4(P[3 * k], P[3 * k + 1], P[3 * k + 2], 0.f);
+  for (int k = threadIdx.x; k < 3 * cnt; k += TP_THREADS) S.B[k] = P[k];
   const int4* Lg = reinterpret_cast<const int4*>(p.lut);
   int4* Ls = reinterpret_cast<int4*>(S.L);
   for (int k = threadIdx.x; k < TP_LUT / 16; k += TP_THREADS) Ls[k] = Lg[k];
@@ -258,7 +262,7 @@ __device__ __forceinline__ void tp_epilogue(const TPParams& p, TPPoint& P, const
   }
 }
 
-__device__ __forceinline__ float tp_dot(const TPPoint& P, const float4 q) {
+__device__ __forceinline__ float tp_dot(const TPPoint& P, const float3 q) {
   return __fmaf_rn(P.z1, q.z, __fmaf_rn(P.y1, q.y, __fmul_rn(P.x1, q.x)));
 }
 template <bool LUT>
@@ -287,26 +291,36 @@ __device__ __forceinline__ void tp_loops(const TPParams& p, const TPSmem& S, uin
   constexpr bool CNT = (V & (V_L | V_PROF)) != 0;
   const uint8_t* __restrict__ L = S.L;
   const float* __restrict__ E = S.E;
-  const float4* __restrict__ Bs = S.B - (A.row % p.nC) * p.C;  // Bs[j] for j in chunk c
+  const int32_t k0 = -(A.row % p.nC) * p.C;  // tile index k = j + k0
+  const float* __restrict__ Pb = S.B;
+  auto part = [&](int32_t k) { return make_float3(Pb[3 * k], Pb[3 * k + 1], Pb[3 * k + 2]); };
   const int32_t je = A.je;
   const int32_t ja = va ? A.jb : je, jbb = vb ? B.jb : je;  // ja <= jbb (i_a < i_b, same chunk)
   const int32_t j1 = min(jbb, je);
   // phase 1: only point A has partners
-  for (int32_t j = ja; j < j1; ++j) tp_count<CNT>(p, Hw, A, tp_binof<LUT>(L, E, tp_dot(A, Bs[j])));
+  for (int32_t j = ja; j < j1; ++j) tp_count<CNT>(p, Hw, A, tp_binof<LUT>(L, E, tp_dot(A, part(j + k0))));
   if (!va) {
-    for (int32_t j = jbb; j < je; ++j) tp_count<CNT>(p, Hw, B, tp_binof<LUT>(L, E, tp_dot(B, Bs[j])));
+    for (int32_t j = jbb; j < je; ++j) tp_count<CNT>(p, Hw, B, tp_binof<LUT>(L, E, tp_dot(B, part(j + k0))));
     return;
   }
   // phase 2: both points, one shared partner load; the partner pointer walks the tile and the
   // counters advance by 4 per group of 4 iterations (the strength reduction any compiler applies
   // to an unrolled it++; the FI program keeps the per-iteration increment as the injection site)
-  int32_t j = max(jbb, ja);
-  const float4* __restrict__ T = S.B;
-  const int32_t k0 = (int32_t)(Bs - S.B);  // -(c * C): tile index k = j + k0
-  int32_t k = j + k0;
+  int32_t k = max(jbb, ja) + k0;
   const int32_t kend = je + k0;
+  auto both = [&](int32_t kk) {
+    const float3 q = part(kk);
+    const int32_t a = tp_binof<LUT>(L, E, tp_dot(A, q)), b = tp_binof<LUT>(L, E, tp_dot(B, q));
+    tp_count<CNT>(p, Hw, A, a);
+    tp_count<CNT>(p, Hw, B, b);
+  };
+  for (; k < kend && (k & 3); ++k) both(k);  // align to a 48-byte group (chunk starts are aligned when C % 4 == 0)
+  const float4* __restrict__ T4 = reinterpret_cast<const float4*>(Pb);
   for (; k + 3 < kend; k += 4) {
-    const float4 q0 = T[k], q1 = T[k + 1], q2 = T[k + 2], q3 = T[k + 3];
+    const int32_t k3 = (k >> 2) * 3;
+    const float4 v0 = T4[k3], v1 = T4[k3 + 1], v2 = T4[k3 + 2];
+    const float3 q0 = make_float3(v0.x, v0.y, v0.z), q1 = make_float3(v0.w, v1.x, v1.y);
+    const float3 q2 = make_float3(v1.z, v1.w, v2.x), q3 = make_float3(v2.y, v2.z, v2.w);
     const int32_t a0 = tp_binof<LUT>(L, E, tp_dot(A, q0)), b0 = tp_binof<LUT>(L, E, tp_dot(B, q0));
     const int32_t a1 = tp_binof<LUT>(L, E, tp_dot(A, q1)), b1 = tp_binof<LUT>(L, E, tp_dot(B, q1));
     const int32_t a2 = tp_binof<LUT>(L, E, tp_dot(A, q2)), b2 = tp_binof<LUT>(L, E, tp_dot(B, q2));
@@ -320,12 +334,7 @@ __device__ __forceinline__ void tp_loops(const TPParams& p, const TPSmem& S, uin
       B.cnt = count_inc(B.cnt, p.four);
     }
   }
-  for (j = k - k0; j < je; ++j) {
-    const float4 q = Bs[j];
-    const int32_t a = tp_binof<LUT>(L, E, tp_dot(A, q)), b = tp_binof<LUT>(L, E, tp_dot(B, q));
-    tp_count<CNT>(p, Hw, A, a);
-    tp_count<CNT>(p, Hw, B, b);
-  }
+  for (; k < kend; ++k) both(k);
 }
 
 template <int V>
@@ -366,48 +375,57 @@ __device__ __forceinline__ void tpacf_body(const TPParams& p, const TPSmem& S, u
 // block scheduler's placement left the busiest SM with ~1.3x the mean work (ncu
 // sm__cycles_active max/avg).  The host assigns the (point block, row) work items to SMs by
 // longest-processing-time greedy on their exact pair counts; a persistent grid of k CTAs per SM
-// claims the items of its own SM's list (%smid) and, once that list is drained, steals from the
-// other lists, so every item runs exactly once whatever the placement.  Same abstract threads,
-// same per-thread order: only which CTA runs an item changes.
+// claims the items of its own SM's list (%smid).  The claim of the next item is issued before the
+// current item runs, so its latency overlaps the work.  Completion does not depend on placement:
+// the last CTA to finish sweeps every list for items nobody claimed (an SM that received no CTA).
+// Same abstract threads, same per-thread order: only which CTA runs an item changes.
 struct TPSched {
   const int2* items;  // (bxi, row), grouped by SM
   const int* off;     // [nsm + 1] list offsets
   int* next;          // [nsm] claim counters (zeroed per run)
   int* claimed;       // items claimed so far (zeroed per run)
+  int* exited;        // CTAs finished (zeroed per run)
   int nsm, total;
 };
+
+__device__ __forceinline__ int tp_claim(const TPSched& q, int sl) {
+  const int k = atomicAdd(q.next + sl, 1);
+  if (q.off[sl] + k >= q.off[sl + 1]) return -1;
+  atomicAdd(q.claimed, 1);
+  return q.off[sl] + k;
+}
+
+template <int V>
+__device__ __forceinline__ void tp_drain(const TPParams& p, const TPSmem& S, const TPSched& q, int sl, int* item_s) {
+  if (threadIdx.x == 0) *item_s = tp_claim(q, sl);
+  for (;;) {
+    __syncthreads();
+    const int it = *item_s;
+    __syncthreads();  // everyone has read the current item before thread 0 overwrites it
+    if (it < 0) break;
+    int nxt = -1;
+    if (threadIdx.x == 0) nxt = tp_claim(q, sl);  // result consumed after the item: latency hidden
+    const int2 xy = q.items[it];
+    tpacf_body<V>(p, S, p.hist, p.cb, xy.x, xy.y);
+    if (threadIdx.x == 0) *item_s = nxt;
+  }
+}
 
 template <int V>
 __global__ void __launch_bounds__(TP_THREADS, HK_TP_STD_MINB) tpacf_kernel(const TPParams p, const TPSched q) {
   extern __shared__ __align__(16) unsigned char tp_smem[];
-  __shared__ int item_s;
+  __shared__ int item_s, last_s;
   const TPSmem S = tp_carve(tp_smem, p.C);
   uint32_t smid;
   asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
-  int sl = (int)(smid % (uint32_t)q.nsm), probes = 0;
-  for (;;) {
-    if (threadIdx.x == 0) {
-      int it = -1;
-      while (probes < q.nsm) {
-        const int k = atomicAdd(q.next + sl, 1);
-        if (q.off[sl] + k < q.off[sl + 1]) {
-          it = q.off[sl] + k;
-          atomicAdd(q.claimed, 1);
-          break;
-        }
-        if (*(volatile int*)q.claimed >= q.total) break;  // everything is taken
-        sl = (sl + 1 == q.nsm) ? 0 : sl + 1;
-        ++probes;
-      }
-      item_s = it;
-    }
-    __syncthreads();
-    const int it = item_s;
-    if (it < 0) break;
-    const int2 xy = q.items[it];
-    tpacf_body<V>(p, S, p.hist, p.cb, xy.x, xy.y);
-    __syncthreads();  // smem (and item_s) reused by the next item
+  tp_drain<V>(p, S, q, (int)(smid % (uint32_t)q.nsm), &item_s);
+  if (threadIdx.x == 0) {
+    __threadfence();
+    last_s = (atomicAdd(q.exited, 1) == (int)gridDim.x - 1) && (*(volatile int*)q.claimed < q.total);
   }
+  __syncthreads();
+  if (last_s)
+    for (int sl = 0; sl < q.nsm; ++sl) tp_drain<V>(p, S, q, sl, &item_s);
 }
 
 // ============================================================================================
@@ -768,14 +786,14 @@ static TPParams tp_params(const hk_tpacf_args& a, const DevRanges& R, int ndet, 
   return p;
 }
 
-// workspace: bucket table | ok flag (16 B) | single-run schedule counters next[TP_SCHED_MAX_SM], claimed
-size_t tpacf_lut_ws_bytes() { return TP_LUT + 16 + (TP_SCHED_MAX_SM + 1) * sizeof(int); }
+// workspace: bucket table | ok flag (16 B) | single-run schedule counters next[TP_SCHED_MAX_SM], claimed, exited
+size_t tpacf_lut_ws_bytes() { return TP_LUT + 16 + (TP_SCHED_MAX_SM + 2) * sizeof(int); }
 
 cudaError_t tpacf_lut_build(const hk_tpacf_args& a, void* lut_ws, cudaStream_t s) {
   int* ok = reinterpret_cast<int*>(reinterpret_cast<char*>(lut_ws) + TP_LUT);
   cudaError_t e = cudaMemsetAsync(ok, 1, sizeof(int), s);
   if (e != cudaSuccess) return e;
-  e = cudaMemsetAsync(reinterpret_cast<char*>(lut_ws) + TP_LUT + 16, 0, (TP_SCHED_MAX_SM + 1) * sizeof(int), s);
+  e = cudaMemsetAsync(reinterpret_cast<char*>(lut_ws) + TP_LUT + 16, 0, (TP_SCHED_MAX_SM + 2) * sizeof(int), s);
   if (e != cudaSuccess) return e;
   tpacf_lut_kernel<<<TP_LUT / 256, 256, 0, s>>>(a.edges, a.n_bins, reinterpret_cast<uint8_t*>(lut_ws), ok);
   count_launch();
@@ -865,6 +883,7 @@ static cudaError_t launch_tp_v(const TPParams& p, void* lut_ws, cudaStream_t s) 
   q.off = B.off;
   q.next = reinterpret_cast<int*>(reinterpret_cast<char*>(lut_ws) + TP_LUT + 16);
   q.claimed = q.next + TP_SCHED_MAX_SM;
+  q.exited = q.claimed + 1;
   q.nsm = nsm;
   q.total = B.total;
 #ifdef HK_TP_STD_CTAS

@@ -362,6 +362,12 @@ struct BenchWS {
 };
 
 static int default_batch(int b, const void* args) {
+  {  // HK_BATCH_<b>: replicas per launch override (experiments)
+    char name[16];
+    snprintf(name, sizeof name, "HK_BATCH_%d", b);
+    const char* v = getenv(name);
+    if (v && atoi(v) > 0) return atoi(v);
+  }
   if (b == HK_CP) {
     const hk_cp_args* a = (const hk_cp_args*)args;
     const int64_t ctas = (int64_t)(a->nx / (a->bx * a->unroll)) * (a->ny / a->by);
@@ -535,6 +541,9 @@ hk_status hauberk_decode(int32_t bench_mode, const void* const args[3], const ui
 // Campaign session: golden runs, catalogues and replica workspaces prepared once; each
 // hauberk_campaign_run enqueues one slice of injections without synchronising.
 // ---------------------------------------------------------------------------------------------
+#ifndef HK_CONCURRENT_DEFAULT
+#define HK_CONCURRENT_DEFAULT 1
+#endif
 struct hk_campaign_session {
   DevCatalog dcat[3]{};
   int64_t* d_prefix = nullptr;  // TPACF trip prefix sums on the device (replay decode)
@@ -553,6 +562,11 @@ struct hk_campaign_session {
   size_t h_cap = 0;
   cudaEvent_t uploaded = nullptr;
   cudaStream_t stream = nullptr;
+  // replica mode, mixed campaigns: one forked stream per benchmark so the XU-bound MRI-Q
+  // replicas and the issue-bound TPACF replicas can share SMs (joined back into `stream`)
+  bool concurrent = false;
+  cudaStream_t sub[3]{};
+  cudaEvent_t fork = nullptr, join[3]{};
 };
 
 static void session_free(hk_campaign_session* S) {
@@ -573,6 +587,11 @@ static void session_free(hk_campaign_session* S) {
   if (S->d_prefix) cudaFree(S->d_prefix);
   if (S->d_decode) cudaFree(S->d_decode);
   if (S->uploaded) cudaEventDestroy(S->uploaded);
+  for (int b = 0; b < 3; ++b) {
+    if (S->sub[b]) cudaStreamDestroy(S->sub[b]);
+    if (S->join[b]) cudaEventDestroy(S->join[b]);
+  }
+  if (S->fork) cudaEventDestroy(S->fork);
   delete S;
 }
 
@@ -598,6 +617,10 @@ static hk_status session_create(int32_t bench_mode, const void* const args[3], c
   S->bench_mode = bench_mode;
   S->cfg = *C;
   S->stream = s;
+  {
+    const char* env = getenv("HK_CONCURRENT");
+    S->concurrent = env ? atoi(env) != 0 : HK_CONCURRENT_DEFAULT;
+  }
   hk_status st = HK_OK;
   cudaError_t e;
   for (int b = 0; b < 3 && st == HK_OK; ++b) {
@@ -807,9 +830,34 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
 
   // ---- batches: FI&FT replicas, then the classify epilogue (which also recycles the workspace)
   const bool real = S->cfg.mode == 2;  // R25: unguarded replicas (guardian child processes only)
+  const cudaStream_t s0 = s;
+  bool touched[3] = {false, false, false};
+  for (const Item& it : items) touched[it.b] = true;
+  const bool conc = S->concurrent && (int)touched[0] + (int)touched[1] + (int)touched[2] > 1;
+  if (conc) {
+    if (!S->fork && (e = cudaEventCreateWithFlags(&S->fork, cudaEventDisableTiming)) != cudaSuccess) return cuda_fail(e, "event");
+    for (int b = 0; b < 3; ++b) {
+      if (!touched[b]) continue;
+      if (!S->sub[b]) {
+        // HK_CONC_PRIO=b: benchmark b's stream gets the highest priority (experiments)
+        const char* pe = getenv("HK_CONC_PRIO");
+        int lo = 0, hi = 0;
+        cudaDeviceGetStreamPriorityRange(&lo, &hi);
+        const int prio = (pe && atoi(pe) == b) ? hi : lo;
+        if ((e = cudaStreamCreateWithPriority(&S->sub[b], cudaStreamNonBlocking, prio)) != cudaSuccess)
+          return cuda_fail(e, "stream");
+      }
+      if (!S->join[b] && (e = cudaEventCreateWithFlags(&S->join[b], cudaEventDisableTiming)) != cudaSuccess)
+        return cuda_fail(e, "event");
+    }
+    if ((e = cudaEventRecord(S->fork, s0)) != cudaSuccess) return cuda_fail(e, "fork");
+    for (int b = 0; b < 3; ++b)
+      if (touched[b] && (e = cudaStreamWaitEvent(S->sub[b], S->fork, 0)) != cudaSuccess) return cuda_fail(e, "fork");
+  }
   size_t q = 0;
   while (q < items.size()) {
     const int b = items[q].b, kind = items[q].kind;
+    s = conc ? S->sub[b] : s0;
     size_t end = q;
     while (end < items.size() && items[end].b == b && items[end].kind == kind && (int)(end - q) < S->W[b].batch) ++end;
     const int nrep = (int)(end - q);
@@ -840,6 +888,12 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
     }
     q = end;
   }
+  if (conc)
+    for (int b = 0; b < 3; ++b) {
+      if (!touched[b]) continue;
+      if ((e = cudaEventRecord(S->join[b], S->sub[b])) != cudaSuccess || (e = cudaStreamWaitEvent(s0, S->join[b], 0)) != cudaSuccess)
+        return cuda_fail(e, "join");
+    }
   return HK_OK;
 }
 

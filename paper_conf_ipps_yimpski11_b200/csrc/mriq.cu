@@ -25,7 +25,15 @@ constexpr int MQ_FI_UNROLL = HK_MQ_FI_UNROLL;
 #ifndef HK_MQ_UNROLL
 #define HK_MQ_UNROLL 16
 #endif
-constexpr int MQ_UNROLL = HK_MQ_UNROLL;  // single-run kernel (one voxel per thread)
+constexpr int MQ_UNROLL = HK_MQ_UNROLL;  // single-run kernel
+#ifndef HK_MQ_THREADS
+#define HK_MQ_THREADS 256
+#endif
+#ifndef HK_MQ_VPT
+#define HK_MQ_VPT 1
+#endif
+constexpr int MQ_THREADS = HK_MQ_THREADS;  // single-run CTA size
+constexpr int MQ_VPT = HK_MQ_VPT;          // single-run voxels per CUDA thread
 constexpr float RINT_MAGIC = 12582912.0f;  // 1.5 * 2^23
 constexpr float TWO_PI_F = 6.28318548202514648f;
 
@@ -81,7 +89,7 @@ __global__ void __launch_bounds__(256) mriq_phimag_kernel(const float* __restric
 // b*(blockDim*VPT) + j*blockDim + t.  Each keeps its own registers, detectors and counter; they
 // share every k-space load (VPT = 2 in the campaign replicas, 1 for the single-run kernel whose
 // grid is small).
-template <int V, bool EXACT, bool ADD, int VPT>
+template <int V, bool EXACT, bool ADD, int VPT, int UNR = (VPT == 1 ? MQ_UNROLL : MQ_FI_UNROLL)>
 __device__ __forceinline__ void mriq_body(const MQParams& p, float4 (*tile)[MQ_TILE], uint64_t* bar, int bxi) {
   constexpr bool NL = (V & V_NL) != 0, L = (V & V_L) != 0, PROF = (V & V_PROF) != 0;
   constexpr bool CNT = L || PROF;
@@ -137,7 +145,7 @@ __device__ __forceinline__ void mriq_body(const MQParams& p, float4 (*tile)[MQ_T
     if (any_active) {
       const float4* A = tile[buf];
       const int cnt = min(MQ_TILE, numK - t * MQ_TILE);
-#pragma unroll(VPT == 1 ? MQ_UNROLL : MQ_FI_UNROLL)
+#pragma unroll(UNR)
       for (int a = 0; a < cnt; ++a) {
         const float4 k4 = A[a];
 #pragma unroll
@@ -193,10 +201,10 @@ __device__ __forceinline__ void mriq_body(const MQParams& p, float4 (*tile)[MQ_T
 }
 
 template <int V, bool EXACT>
-__global__ void __launch_bounds__(256) mriq_kernel(const MQParams p) {
+__global__ void __launch_bounds__(MQ_THREADS) mriq_kernel(const MQParams p) {
   __shared__ __align__(128) float4 tile[2][MQ_TILE];
   __shared__ __align__(8) uint64_t bar[2];
-  mriq_body<V, EXACT, false, 1>(p, tile, bar, blockIdx.x);
+  mriq_body<V, EXACT, false, MQ_VPT, MQ_UNROLL>(p, tile, bar, blockIdx.x);
 }
 
 // ============================================================================================
@@ -418,7 +426,7 @@ __global__ void __launch_bounds__(MQ_FI_THREADS) mriq_fi_kernel(const MQFIParams
   p.cb = q.cb0 + r;
   if (KIND == MK_PHIMAG) p.kv = q.kv0 + (int64_t)r * p.numK;  // this replica's (possibly faulted) k-space
   if (KIND == MK_PHIMAG || !faulted) {
-    mriq_body<V_NL | V_L, EXACT, true, MQ_FI_VPT>(p, tile, bar, bxi);
+    mriq_body<V_NL | V_L, EXACT, true, MQ_FI_VPT, MQ_FI_UNROLL>(p, tile, bar, bxi);
   } else {
     ReplicaSinkF S{{p.qr, p.qi}, p.cb};
 #pragma unroll 1
@@ -549,10 +557,10 @@ cudaError_t mriq_phimag_launch(const hk_mriq_args& a, bool nl, hk_control* cb, c
 
 template <int V, bool EXACT>
 static cudaError_t launch_mq_v(const MQParams& p, cudaStream_t s) {
-  const int g = (p.numX + 255) / 256;
+  const int g = (p.numX + MQ_THREADS * MQ_VPT - 1) / (MQ_THREADS * MQ_VPT);
   if (g == 0) return cudaSuccess;
   TimedScope ts(HK_MRIQ, 0, (double)p.numX * (double)p.numK, s);
-  mriq_kernel<V, EXACT><<<g, 256, 0, s>>>(p);
+  mriq_kernel<V, EXACT><<<g, MQ_THREADS, 0, s>>>(p);
   count_launch();
   return cudaGetLastError();
 }

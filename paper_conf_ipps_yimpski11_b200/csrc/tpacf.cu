@@ -23,13 +23,19 @@ namespace hk {
 #define HK_TP_THREADS 128
 #endif
 constexpr int TP_THREADS = HK_TP_THREADS;
-// Minimum resident CTAs per SM for the register allocator (measured, tools/ab_time.py): the
-// replicas run fastest at 9 (56 registers), the single run at 10.
+// Minimum resident CTAs per SM for the register allocator (measured, tools/ab_time.py): with
+// 8-partner groups (HK_TP_G8) both the replicas and the single run are fastest at 9 (56
+// registers; the single run spills at 10).  8-partner groups: 13.4 SASS instructions per pair
+// instead of 14 (loop overhead and partner loads amortised over 16 pairs); measured FT single
+// run 74.7 -> 70.7 us, replicas 52.6 -> 51.8 us.
 #ifndef HK_TP_MINB
 #define HK_TP_MINB 9
 #endif
+#ifndef HK_TP_G8
+#define HK_TP_G8 1
+#endif
 #ifndef HK_TP_STD_MINB
-#define HK_TP_STD_MINB 10
+#define HK_TP_STD_MINB 9
 #endif
 constexpr int TP_CTA_PTS = 2 * TP_THREADS;  // two abstract threads per CUDA thread
 constexpr int TP_WARPS = TP_THREADS / 32;
@@ -45,7 +51,7 @@ struct TPParams {
   DevRanges R;
   int32_t n, nr, nb, C, nC, ndet;
   uint32_t z;
-  int32_t one, four;  // runtime 1 and 4 (opaque)
+  int32_t one, four, eight;  // runtime 1, 4 and 8 (opaque)
 };
 
 // ---------------------------------------------------------------------------------------------
@@ -316,6 +322,30 @@ __device__ __forceinline__ void tp_loops(const TPParams& p, const TPSmem& S, uin
   };
   for (; k < kend && (k & 3); ++k) both(k);  // align to a 48-byte group (chunk starts are aligned when C % 4 == 0)
   const float4* __restrict__ T4 = reinterpret_cast<const float4*>(Pb);
+#if HK_TP_G8
+  for (; k + 7 < kend; k += 8) {
+    const int32_t k3 = (k >> 2) * 3;
+    const float4 v0 = T4[k3], v1 = T4[k3 + 1], v2 = T4[k3 + 2], v3 = T4[k3 + 3], v4 = T4[k3 + 4], v5 = T4[k3 + 5];
+    const float3 q[8] = {make_float3(v0.x, v0.y, v0.z), make_float3(v0.w, v1.x, v1.y), make_float3(v1.z, v1.w, v2.x),
+                         make_float3(v2.y, v2.z, v2.w), make_float3(v3.x, v3.y, v3.z), make_float3(v3.w, v4.x, v4.y),
+                         make_float3(v4.z, v4.w, v5.x), make_float3(v5.y, v5.z, v5.w)};
+    int32_t a[8], b[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      a[u] = tp_binof<LUT>(L, E, tp_dot(A, q[u]));
+      b[u] = tp_binof<LUT>(L, E, tp_dot(B, q[u]));
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      tp_count<CNT, false>(p, Hw, A, a[u]);
+      tp_count<CNT, false>(p, Hw, B, b[u]);
+    }
+    if (CNT) {
+      A.cnt = count_inc(A.cnt, p.eight);
+      B.cnt = count_inc(B.cnt, p.eight);
+    }
+  }
+#endif
   for (; k + 3 < kend; k += 4) {
     const int32_t k3 = (k >> 2) * 3;
     const float4 v0 = T4[k3], v1 = T4[k3 + 1], v2 = T4[k3 + 2];
@@ -783,6 +813,7 @@ static TPParams tp_params(const hk_tpacf_args& a, const DevRanges& R, int ndet, 
   p.z = opaque_zero();
   p.one = 1 + (int32_t)opaque_zero();
   p.four = 4 * p.one;
+  p.eight = 8 * p.one;
   return p;
 }
 

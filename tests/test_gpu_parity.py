@@ -372,6 +372,30 @@ def test_campaign_session_matches_one_shot_calls():
     assert np.array_equal(a["cls"], b["cls"]) and np.array_equal(a["index"], b["index"])
 
 
+def test_campaign_concurrent_streams_equal_serial(monkeypatch):
+    """Sessions fork one stream per benchmark; the per-injection records, the
+    counters and the per-site counters must equal those of a serial session (HK_CONCURRENT=0)."""
+    probs = [W.cp_small(), W.mriq_problem(4, 40, n_vox=64, seed=9), W.tpacf_small(n=64, n_rand=1, chunk=16)]
+    devs = [_mk(b, probs[b]) for b in range(3)]
+    R = [hk.profile_ranges(d) for d in devs]
+    out = {}
+    for conc in ("0", "1"):
+        monkeypatch.setenv("HK_CONCURRENT", conc)
+        counts = torch.zeros((3, 5), dtype=torch.int64, device=DEV)
+        sites = torch.zeros((3, 64, 5), dtype=torch.int64, device=DEV)
+        rec = hk.records_tensor(900, DEV)
+        with hk.CampaignSession(-1, devs, R, 777, batch=11) as S:
+            S.run(0, 450, counts, records=rec[: 450 * hk.OUTCOME_DTYPE.itemsize], site_counts=sites)
+            S.run(450, 450, counts, records=rec[450 * hk.OUTCOME_DTYPE.itemsize:], site_counts=sites)
+            torch.cuda.synchronize()
+        out[conc] = (counts.cpu(), sites.cpu(), hk.records_numpy(rec))
+    assert torch.equal(out["0"][0], out["1"][0]) and torch.equal(out["0"][1], out["1"][1])
+    assert int(out["1"][0].sum()) == 900
+    a, b = out["0"][2], out["1"][2]
+    for f in a.dtype.names:
+        assert np.array_equal(a[f], b[f]), f
+
+
 @pytest.mark.parametrize("k", [3, 15])
 def test_campaign_multibit_exact_mode_bit_exact(k):
     probs = [W.cp_small(), W.mriq_problem(5, 41, n_vox=100, seed=4), W.tpacf_small(n=90, n_rand=1, chunk=32)]

@@ -76,10 +76,14 @@ __device__ __forceinline__ int32_t tp_bin(const float* Es, float dot) {
   for (int s = 16; s >= 1; s >>= 1) b += (dot < Es[b + s - 1]) ? s : 0;
   return b;
 }
-__device__ __forceinline__ int32_t tp_bin_lut(const uint8_t* L, const float* Es, float dot) {
+// Returns 4 * bin.  The table holds 4 * bmin, the byte offset of E[bmin], so the edge load is
+// [offset + shared base] with no address arithmetic; `eb` = 32-bit shared address of E (uniform).
+__device__ __forceinline__ int32_t tp_bin_lut(const uint8_t* L, uint32_t eb, float dot) {
   const float u = __fsub_rn(1.0f, dot);
-  const int32_t b = L[fb(u) >> 21];
-  return b + (int32_t)(fb(__fsub_rn(dot, Es[b])) >> 31);
+  const uint32_t b4 = L[fb(u) >> 21];
+  float e;
+  asm("ld.shared.f32 %0, [%1];" : "=f"(e) : "r"(eb + b4));
+  return (int32_t)((dot < e) ? b4 + 4u : b4);
 }
 
 __device__ __forceinline__ float nup(float x) {
@@ -126,7 +130,7 @@ __global__ void tpacf_lut_kernel(const float* __restrict__ edges, int nb, uint8_
     good = (__fsub_rn(1.0f, dmax) >= ulo) && (__fsub_rn(1.0f, dmin) <= uhi) && (bmax - bmin <= 1);
     out = make_int2(bmin, (int)(bmin <= nb ? fb(edges[bmin]) : 0xff800000u));
   }
-  lut[q] = (uint8_t)out.x;  // E[b] (padded with -inf beyond nb) supplies the compare value
+  lut[q] = (uint8_t)(4 * out.x);  // byte offset of E[b] (padded with -inf beyond nb): the compare value
   if (!good) atomicExch(ok, 0);
 }
 
@@ -272,17 +276,19 @@ __device__ __forceinline__ float tp_dot(const TPPoint& P, const float3 q) {
   return __fmaf_rn(P.z1, q.z, __fmaf_rn(P.y1, q.y, __fmul_rn(P.x1, q.x)));
 }
 template <bool LUT>
-__device__ __forceinline__ int32_t tp_binof(const uint8_t* __restrict__ L, const float* __restrict__ E, float dot) {
-  return LUT ? tp_bin_lut(L, E, dot) : tp_bin(E, dot);
+__device__ __forceinline__ int32_t tp_binof(const uint8_t* __restrict__ L, const float* __restrict__ E, uint32_t eb, float dot) {
+  return LUT ? tp_bin_lut(L, eb, dot) : 4 * tp_bin(E, dot);  // 4 * bin
 }
+// bin4 = 4 * bin (tp_binof).  The fast path accumulates acc4 = sum of 4 * bin; tp_loops divides
+// by 4 at the end: the same integer as the abstract acc (acc <= 31 * C <= 31 * 1024, no wrap).
 template <bool CNT, bool INC = true>
-__device__ __forceinline__ void tp_count(const TPParams& p, uint32_t* Hw, TPPoint& P, int32_t bin) {
+__device__ __forceinline__ void tp_count(const TPParams& p, uint32_t* Hw, TPPoint& P, int32_t bin4) {
   // lane-private counter: no contention; the shared-memory atomic (ATOMS.POPC.INC) has no
   // register round trip, so consecutive increments do not serialise (microbenchmark: 1.34x the
   // LDS/IADD/STS read-modify-write, tools/microbench/smem_hist.cu)
-  atomicAdd(Hw + bin * 32, 1u);
+  atomicAdd(Hw + bin4 * 8, 1u);
   if (CNT) {
-    P.acc += bin;
+    P.acc += bin4;
     if (INC) P.cnt = count_inc(P.cnt, p.one);
   }
 }
@@ -292,11 +298,12 @@ __device__ __forceinline__ void tp_count(const TPParams& p, uint32_t* Hw, TPPoin
 // Within a group of 4 partners all loads (partner, bucket table, edge) are issued before the
 // histogram read-modify-writes, which the compiler must otherwise serialise (possible aliasing).
 template <int V, bool LUT>
-__device__ __forceinline__ void tp_loops(const TPParams& p, const TPSmem& S, uint32_t* Hw, TPPoint& A, TPPoint& B,
+__device__ __forceinline__ void tp_loops4(const TPParams& p, const TPSmem& S, uint32_t* Hw, TPPoint& A, TPPoint& B,
                                          bool va, bool vb) {
   constexpr bool CNT = (V & (V_L | V_PROF)) != 0;
   const uint8_t* __restrict__ L = S.L;
   const float* __restrict__ E = S.E;
+  const uint32_t eb = (uint32_t)__cvta_generic_to_shared(S.E);
   const int32_t k0 = -(A.row % p.nC) * p.C;  // tile index k = j + k0
   const float* __restrict__ Pb = S.B;
   auto part = [&](int32_t k) { return make_float3(Pb[3 * k], Pb[3 * k + 1], Pb[3 * k + 2]); };
@@ -304,9 +311,9 @@ __device__ __forceinline__ void tp_loops(const TPParams& p, const TPSmem& S, uin
   const int32_t ja = va ? A.jb : je, jbb = vb ? B.jb : je;  // ja <= jbb (i_a < i_b, same chunk)
   const int32_t j1 = min(jbb, je);
   // phase 1: only point A has partners
-  for (int32_t j = ja; j < j1; ++j) tp_count<CNT>(p, Hw, A, tp_binof<LUT>(L, E, tp_dot(A, part(j + k0))));
+  for (int32_t j = ja; j < j1; ++j) tp_count<CNT>(p, Hw, A, tp_binof<LUT>(L, E, eb, tp_dot(A, part(j + k0))));
   if (!va) {
-    for (int32_t j = jbb; j < je; ++j) tp_count<CNT>(p, Hw, B, tp_binof<LUT>(L, E, tp_dot(B, part(j + k0))));
+    for (int32_t j = jbb; j < je; ++j) tp_count<CNT>(p, Hw, B, tp_binof<LUT>(L, E, eb, tp_dot(B, part(j + k0))));
     return;
   }
   // phase 2: both points, one shared partner load; the partner pointer walks the tile and the
@@ -316,7 +323,7 @@ __device__ __forceinline__ void tp_loops(const TPParams& p, const TPSmem& S, uin
   const int32_t kend = je + k0;
   auto both = [&](int32_t kk) {
     const float3 q = part(kk);
-    const int32_t a = tp_binof<LUT>(L, E, tp_dot(A, q)), b = tp_binof<LUT>(L, E, tp_dot(B, q));
+    const int32_t a = tp_binof<LUT>(L, E, eb, tp_dot(A, q)), b = tp_binof<LUT>(L, E, eb, tp_dot(B, q));
     tp_count<CNT>(p, Hw, A, a);
     tp_count<CNT>(p, Hw, B, b);
   };
@@ -332,8 +339,8 @@ __device__ __forceinline__ void tp_loops(const TPParams& p, const TPSmem& S, uin
     int32_t a[8], b[8];
 #pragma unroll
     for (int u = 0; u < 8; ++u) {
-      a[u] = tp_binof<LUT>(L, E, tp_dot(A, q[u]));
-      b[u] = tp_binof<LUT>(L, E, tp_dot(B, q[u]));
+      a[u] = tp_binof<LUT>(L, E, eb, tp_dot(A, q[u]));
+      b[u] = tp_binof<LUT>(L, E, eb, tp_dot(B, q[u]));
     }
 #pragma unroll
     for (int u = 0; u < 8; ++u) {
@@ -351,10 +358,10 @@ __device__ __forceinline__ void tp_loops(const TPParams& p, const TPSmem& S, uin
     const float4 v0 = T4[k3], v1 = T4[k3 + 1], v2 = T4[k3 + 2];
     const float3 q0 = make_float3(v0.x, v0.y, v0.z), q1 = make_float3(v0.w, v1.x, v1.y);
     const float3 q2 = make_float3(v1.z, v1.w, v2.x), q3 = make_float3(v2.y, v2.z, v2.w);
-    const int32_t a0 = tp_binof<LUT>(L, E, tp_dot(A, q0)), b0 = tp_binof<LUT>(L, E, tp_dot(B, q0));
-    const int32_t a1 = tp_binof<LUT>(L, E, tp_dot(A, q1)), b1 = tp_binof<LUT>(L, E, tp_dot(B, q1));
-    const int32_t a2 = tp_binof<LUT>(L, E, tp_dot(A, q2)), b2 = tp_binof<LUT>(L, E, tp_dot(B, q2));
-    const int32_t a3 = tp_binof<LUT>(L, E, tp_dot(A, q3)), b3 = tp_binof<LUT>(L, E, tp_dot(B, q3));
+    const int32_t a0 = tp_binof<LUT>(L, E, eb, tp_dot(A, q0)), b0 = tp_binof<LUT>(L, E, eb, tp_dot(B, q0));
+    const int32_t a1 = tp_binof<LUT>(L, E, eb, tp_dot(A, q1)), b1 = tp_binof<LUT>(L, E, eb, tp_dot(B, q1));
+    const int32_t a2 = tp_binof<LUT>(L, E, eb, tp_dot(A, q2)), b2 = tp_binof<LUT>(L, E, eb, tp_dot(B, q2));
+    const int32_t a3 = tp_binof<LUT>(L, E, eb, tp_dot(A, q3)), b3 = tp_binof<LUT>(L, E, eb, tp_dot(B, q3));
     tp_count<CNT, false>(p, Hw, A, a0); tp_count<CNT, false>(p, Hw, B, b0);
     tp_count<CNT, false>(p, Hw, A, a1); tp_count<CNT, false>(p, Hw, B, b1);
     tp_count<CNT, false>(p, Hw, A, a2); tp_count<CNT, false>(p, Hw, B, b2);
@@ -365,6 +372,14 @@ __device__ __forceinline__ void tp_loops(const TPParams& p, const TPSmem& S, uin
     }
   }
   for (; k < kend; ++k) both(k);
+}
+
+template <int V, bool LUT>
+__device__ __forceinline__ void tp_loops(const TPParams& p, const TPSmem& S, uint32_t* Hw, TPPoint& A, TPPoint& B,
+                                         bool va, bool vb) {
+  tp_loops4<V, LUT>(p, S, Hw, A, B, va, vb);
+  A.acc >>= 2;
+  B.acc >>= 2;
 }
 
 template <int V>

@@ -323,8 +323,15 @@ def main():
         with open(os.path.join(ROOT, "profiles", "r01_traffic.json")) as f:
             tr = json.load(f).get(f"{hk.BENCH_NAMES[dom]}_fi_kernel")
         if tr:
-            roofline["traffic"] = tr["dram_bytes_per_launch"]
-            roofline["traffic_source"] = tr["source"]
+            # ncu measured one launch of `replicas_per_launch` replicas; scale per replica to this
+            # run's mean replicas per launch of the dominant kernel (serial pass)
+            n_inj = sum(1 for st in range(ser_steps)
+                        for n in range(*(lambda f, c: (f, f + c))(*par.step_slice(st, rank, world, args.per_rank)))
+                        if n % 3 == dom)
+            rpl = n_inj / nl if nl else 0.0
+            roofline["traffic"] = round(tr["dram_bytes_per_launch"] / tr["replicas_per_launch"] * rpl)
+            roofline["traffic_source"] = (f"{tr['source']}; scaled to {rpl:.1f} replicas per launch "
+                                          f"({tr['dram_bytes_per_launch'] / tr['replicas_per_launch']:.0f} B per replica)")
     except (OSError, ValueError):
         pass
 

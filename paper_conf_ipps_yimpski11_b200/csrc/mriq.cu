@@ -11,7 +11,7 @@ namespace hk {
 
 constexpr int MQ_TILE = 1024;  // k-samples per stage (16 KB)
 #ifndef HK_MQ_FI_THREADS
-#define HK_MQ_FI_THREADS 256
+#define HK_MQ_FI_THREADS 64
 #endif
 #ifndef HK_MQ_FI_VPT
 #define HK_MQ_FI_VPT 2

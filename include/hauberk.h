@@ -145,6 +145,20 @@ HK_API hk_status hauberk_run_mriq(const hk_mriq_args* args, int32_t variant, con
 HK_API hk_status hauberk_run_tpacf(const hk_tpacf_args* args, int32_t variant, const hk_ranges* ranges,
                             hk_control* d_cb, float* d_samples, void* stream);
 
+/* Single-run sharding (the benchmarks' abstract threads are independent):
+ * run only the partition units [begin, end) of one benchmark, bit-identical to the same units of
+ * the whole run.  Units: CP = grid rows (begin, end multiples of by, or end = ny); MRI-Q = voxels
+ * (the slice's abstract-thread ids, e.g. hk_control.first_thread, are slice-local); TPACF = work
+ * rows h*nC + c, nC = ceil(n / chunk) (histogram h in DD, RR_1..nr, DR_1..nr; chunk c), whose
+ * counts are ADDED into a zeroed hist, so the partial histograms of a partition sum to the whole
+ * (one all-reduce).  The callee zeroes only its own output part (CP rows, MRI-Q voxels; TPACF the
+ * whole hist).  variant: HK_BASE / HK_FT / HK_FT_NL / HK_FT_L (profile over the whole input with
+ * hauberk_profile_ranges and share the ranges).  hauberk_part_units returns the unit count and the
+ * alignment granule.  HK_ERR_INVALID for a range outside [0, units) or misaligned. */
+HK_API hk_status hauberk_part_units(int32_t bench, const void* args, int64_t* units, int64_t* granule);
+HK_API hk_status hauberk_run_part(int32_t bench, const void* args, int32_t variant, const hk_ranges* ranges,
+                                  hk_control* d_cb, int64_t begin, int64_t end, void* stream);
+
 /* PROFILE run + threshold search (L1489-1508) -> out (host).  Synchronises `stream`.
  * args points to the bench's hk_*_args; opts may be NULL (defaults). */
 HK_API hk_status hauberk_profile_ranges(int32_t bench, const void* args, const hk_profile_opts* opts,

@@ -24,6 +24,7 @@ struct CPParams {
   uint32_t z;    // runtime 0 (opaque)
   int32_t one;   // runtime 1 (opaque)
   int64_t nthreads;
+  int32_t by0;  // single run: first block row of this launch (row sharding, hauberk_run_part)
 };
 
 // One CTA's worth of the protected loop.  V: variant flags; ADD: additive stores (R18, FI replicas).
@@ -136,7 +137,7 @@ template <int V, int U, bool EXACT>
 __global__ void __launch_bounds__(256) cp_kernel(const CPParams p) {
   __shared__ __align__(128) float4 tile[2][CP_TILE];
   __shared__ __align__(8) uint64_t bar[2];
-  cp_body<V, U, EXACT, false>(p, tile, bar, blockIdx.x, blockIdx.y);
+  cp_body<V, U, EXACT, false>(p, tile, bar, blockIdx.x, blockIdx.y + p.by0);
 }
 
 // Uninstrumented pre-pass (row a1): (x, y, z, q) -> (x, y, (z - z0)^2, q).
@@ -440,7 +441,7 @@ __global__ void __launch_bounds__(128) cp_replay_all_kernel(const CPReplayParams
 // ============================================================================================
 template <int V, int U, bool EXACT>
 static cudaError_t launch_cp_v(const CPParams& p, dim3 grid, dim3 block, cudaStream_t s) {
-  TimedScope ts(HK_CP, 0, (double)p.numatoms * (double)p.nthreads * U, s);
+  TimedScope ts(HK_CP, 0, (double)p.numatoms * (double)grid.x * grid.y * block.x * block.y * U, s);
   cp_kernel<V, U, EXACT><<<grid, block, 0, s>>>(p);
   count_launch();
   return cudaGetLastError();
@@ -460,6 +461,13 @@ static cudaError_t launch_cp_u(int v, const CPParams& p, dim3 grid, dim3 block, 
 
 cudaError_t cp_launch(int vflags, const hk_cp_args& a, const DevRanges& R, int ndet, hk_control* cb, float* samples,
                       cudaStream_t s) {
+  return cp_launch_rows(vflags, a, R, ndet, cb, samples, 0, a.ny, s);
+}
+
+// Grid rows [y0, y1) only (multiples of by): the same abstract threads as the whole run, by
+// global block row (blockIdx.y + by0), so the rows come out bit-identical (single-run sharding).
+cudaError_t cp_launch_rows(int vflags, const hk_cp_args& a, const DevRanges& R, int ndet, hk_control* cb, float* samples,
+                           int32_t y0, int32_t y1, cudaStream_t s) {
   if (a.n_atoms > 0) {
     cp_prepass_kernel<<<(a.n_atoms + 255) / 256, 256, 0, s>>>(reinterpret_cast<const float4*>(a.atoms),
                                                                reinterpret_cast<float4*>(a.atoms_ws), a.n_atoms, a.z0);
@@ -477,7 +485,9 @@ cudaError_t cp_launch(int vflags, const hk_cp_args& a, const DevRanges& R, int n
   p.z = opaque_zero();
   p.one = 1 + (int32_t)opaque_zero();
   p.nthreads = (int64_t)(a.nx / a.unroll) * a.ny;
-  dim3 block(a.bx, a.by), grid(a.nx / (a.bx * a.unroll), a.ny / a.by);
+  p.by0 = y0 / a.by;
+  dim3 block(a.bx, a.by), grid(a.nx / (a.bx * a.unroll), (y1 - y0) / a.by);
+  if (grid.y == 0) return cudaSuccess;
   const bool ex = a.exact != 0;
   switch (a.unroll) {
     case 1: return ex ? launch_cp_u<1, true>(vflags, p, grid, block, s) : launch_cp_u<1, false>(vflags, p, grid, block, s);

@@ -27,10 +27,12 @@ uint32_t opaque_zero();        // 0, read through a volatile so no compiler can 
 // kernels of one benchmark run (pre-pass / PhiMag included); vflags = V_NL | V_L | V_PROF bits
 cudaError_t cp_launch(int vflags, const hk_cp_args& a, const DevRanges& R, int ndet, hk_control* cb, float* samples,
                       cudaStream_t s);
+cudaError_t cp_launch_rows(int vflags, const hk_cp_args& a, const DevRanges& R, int ndet, hk_control* cb, float* samples,
+                           int32_t y0, int32_t y1, cudaStream_t s);
 cudaError_t mriq_launch(int vflags, const hk_mriq_args& a, const DevRanges& R, int ndet, hk_control* cb,
                         float* samples, cudaStream_t s);
 cudaError_t tpacf_launch(int vflags, const hk_tpacf_args& a, const DevRanges& R, int ndet, hk_control* cb,
-                         float* samples, void* lut_ws, cudaStream_t s);
+                         float* samples, void* lut_ws, cudaStream_t s, int32_t row0 = 0, int32_t row1 = -1);
 size_t tpacf_lut_ws_bytes();
 cudaError_t tpacf_lut_build(const hk_tpacf_args& a, void* lut_ws, cudaStream_t s);
 cudaError_t cp_prepass_launch(const hk_cp_args& a, cudaStream_t s);

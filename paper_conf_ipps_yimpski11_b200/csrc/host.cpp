@@ -452,6 +452,64 @@ hk_status hauberk_run_tpacf(const hk_tpacf_args* args, int32_t variant, const hk
   return run_bench(HK_TPACF, args, variant, ranges, d_cb, d_samples, (cudaStream_t)stream);
 }
 
+hk_status hauberk_part_units(int32_t bench, const void* args, int64_t* units, int64_t* granule) {
+  if (bench < 0 || bench > 2 || !units || !granule || !args_ok(bench, args)) return invalid("part_units: bad bench/args");
+  if (bench == HK_CP) {
+    const hk_cp_args* a = (const hk_cp_args*)args;
+    *units = a->ny; *granule = a->by;
+  } else if (bench == HK_MRIQ) {
+    *units = ((const hk_mriq_args*)args)->n_vox; *granule = 1;
+  } else {
+    const hk_tpacf_args* a = (const hk_tpacf_args*)args;
+    *units = (int64_t)(1 + 2 * a->n_rand) * tp_nc(a); *granule = 1;
+  }
+  return HK_OK;
+}
+
+hk_status hauberk_run_part(int32_t bench, const void* args, int32_t variant, const hk_ranges* ranges, hk_control* d_cb,
+                           int64_t begin, int64_t end, void* stream) {
+  if (bench < 0 || bench > 2 || !args_ok(bench, args)) return invalid("run_part: bad bench/args");
+  if (variant == HK_PROFILE) return invalid("run_part: PROFILE runs over the whole input (hauberk_profile_ranges)");
+  hk_status st = run_common_checks(variant, ranges, d_cb, nullptr);
+  if (st != HK_OK) return st;
+  int64_t units = 0, granule = 1;
+  hauberk_part_units(bench, args, &units, &granule);
+  if (begin < 0 || end < begin || end > units || begin % granule != 0 || (end % granule != 0 && end != units))
+    return invalid("run_part: [begin, end) outside the partition units or not aligned to the granule");
+  cudaStream_t s = (cudaStream_t)stream;
+  const int vf = vflags_of(variant);
+  const DevRanges R = dev_ranges(ranges);
+  int ndet = ranges ? ranges->n_det : 1;
+  if (d_cb) HK_CUDA(control_init_launch(d_cb, 1, s), "control init");
+  if (bench == HK_CP) {
+    const hk_cp_args* a = (const hk_cp_args*)args;
+    ndet = std::min(ndet, a->unroll);
+    HK_CUDA(cudaMemsetAsync(a->grid + (size_t)begin * a->nx, 0, sizeof(float) * (size_t)(end - begin) * a->nx, s), "memset rows");
+    HK_CUDA(cp_launch_rows(vf, *a, R, ndet, d_cb, nullptr, (int32_t)begin, (int32_t)end, s), "cp kernel");
+  } else if (bench == HK_MRIQ) {
+    hk_mriq_args a = *(const hk_mriq_args*)args;  // the voxel slice: independent abstract threads
+    a.x += begin; a.y += begin; a.z += begin; a.qr += begin; a.qi += begin;
+    a.n_vox = (int32_t)(end - begin);
+    ndet = std::min(ndet, 2);
+    if (a.n_vox == 0) return HK_OK;
+    HK_CUDA(cudaMemsetAsync(a.qr, 0, sizeof(float) * (size_t)a.n_vox, s), "memset qr");
+    HK_CUDA(cudaMemsetAsync(a.qi, 0, sizeof(float) * (size_t)a.n_vox, s), "memset qi");
+    HK_CUDA(mriq_launch(vf, a, R, ndet, d_cb, nullptr, s), "mriq kernels");
+  } else {
+    const hk_tpacf_args* a = (const hk_tpacf_args*)args;
+    ndet = std::min(ndet, 1);
+    HK_CUDA(cudaMemsetAsync(a->hist, 0, sizeof(unsigned long long) * (size_t)(1 + 2 * a->n_rand) * (a->n_bins + 2), s),
+            "memset hist");
+    if (end == begin) return HK_OK;
+    void* lut = nullptr;
+    HK_CUDA(cudaMallocAsync(&lut, tpacf_lut_ws_bytes(), s), "alloc tpacf table");
+    cudaError_t e = tpacf_launch(vf, *a, R, ndet, d_cb, nullptr, lut, s, (int32_t)begin, (int32_t)end);
+    cudaFreeAsync(lut, s);
+    HK_CUDA(e, "tpacf kernel");
+  }
+  return HK_OK;
+}
+
 hk_status hauberk_profile_ranges(int32_t bench, const void* args, const hk_profile_opts* opts, hk_ranges* out,
                                  void* stream) {
   if (bench < 0 || bench > 2 || !out || !args_ok(bench, args)) return invalid("profile: bad bench/args");

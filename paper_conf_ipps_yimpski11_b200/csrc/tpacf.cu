@@ -858,20 +858,20 @@ struct TPSchedBuf {
   int* off = nullptr;
   int total = 0;
 };
-static cudaError_t tp_schedule(const TPParams& p, int nsm, TPSchedBuf* out) {
+static cudaError_t tp_schedule(const TPParams& p, int nsm, int row0, int row1, TPSchedBuf* out) {
   int dev = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
   static std::mutex mu;
-  static std::map<std::array<int, 5>, TPSchedBuf> cache;
-  const std::array<int, 5> key{p.n, p.nr, p.C, nsm, dev};
+  static std::map<std::array<int, 7>, TPSchedBuf> cache;
+  const std::array<int, 7> key{p.n, p.nr, p.C, nsm, dev, row0, row1};
   std::lock_guard<std::mutex> lk(mu);
   auto f = cache.find(key);
   if (f != cache.end()) { *out = f->second; return cudaSuccess; }
   const int gx = (p.n + TP_CTA_PTS - 1) / TP_CTA_PTS, gy = (1 + 2 * p.nr) * p.nC;
   std::vector<std::pair<double, int2>> w;
   w.reserve((size_t)gx * gy);
-  for (int row = 0; row < gy; ++row) {
+  for (int row = std::max(row0, 0); row < std::min(row1, gy); ++row) {  // rows [row0, row1): sharding
     const int h = row / p.nC, c = row - h * p.nC;
     const int64_t cb = (int64_t)c * p.C, ce = std::min<int64_t>(cb + p.C, p.n);
     for (int b = 0; b < gx; ++b) {
@@ -912,7 +912,7 @@ static cudaError_t tp_schedule(const TPParams& p, int nsm, TPSchedBuf* out) {
 }
 
 template <int V>
-static cudaError_t launch_tp_v(const TPParams& p, void* lut_ws, cudaStream_t s) {
+static cudaError_t launch_tp_v(const TPParams& p, void* lut_ws, cudaStream_t s, int row0, int row1) {
   const size_t smem = tp_smem_bytes(p.C, p.nb + 2);
   cudaError_t e = cudaFuncSetAttribute(tpacf_kernel<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
@@ -923,7 +923,7 @@ static cudaError_t launch_tp_v(const TPParams& p, void* lut_ws, cudaStream_t s) 
   if (nsm > TP_SCHED_MAX_SM) return cudaErrorInvalidValue;
   if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tpacf_kernel<V>, TP_THREADS, smem)) != cudaSuccess) return e;
   TPSchedBuf B;
-  if ((e = tp_schedule(p, nsm, &B)) != cudaSuccess) return e;
+  if ((e = tp_schedule(p, nsm, row0, row1, &B)) != cudaSuccess) return e;
   TPSched q;
   q.items = B.items;
   q.off = B.off;
@@ -942,17 +942,20 @@ static cudaError_t launch_tp_v(const TPParams& p, void* lut_ws, cudaStream_t s) 
   return cudaGetLastError();
 }
 
+// rows [row0, row1) of (histogram h, chunk c) work rows, row = h*nC + c (row1 < 0: all): the
+// abstract threads of those rows, their counts added into hist (single-run sharding).
 cudaError_t tpacf_launch(int vflags, const hk_tpacf_args& a, const DevRanges& R, int ndet, hk_control* cb, float* samples,
-                         void* lut_ws, cudaStream_t s) {
+                         void* lut_ws, cudaStream_t s, int32_t row0, int32_t row1) {
   cudaError_t e = tpacf_lut_build(a, lut_ws, s);
   if (e != cudaSuccess) return e;
   const TPParams p = tp_params(a, R, ndet, cb, samples, lut_ws);
+  if (row1 < 0) row1 = (1 + 2 * p.nr) * p.nC;
   switch (vflags) {
-    case 0: return launch_tp_v<0>(p, lut_ws, s);
-    case V_NL | V_L: return launch_tp_v<V_NL | V_L>(p, lut_ws, s);
-    case V_NL: return launch_tp_v<V_NL>(p, lut_ws, s);
-    case V_L: return launch_tp_v<V_L>(p, lut_ws, s);
-    case V_PROF: return launch_tp_v<V_PROF>(p, lut_ws, s);
+    case 0: return launch_tp_v<0>(p, lut_ws, s, row0, row1);
+    case V_NL | V_L: return launch_tp_v<V_NL | V_L>(p, lut_ws, s, row0, row1);
+    case V_NL: return launch_tp_v<V_NL>(p, lut_ws, s, row0, row1);
+    case V_L: return launch_tp_v<V_L>(p, lut_ws, s, row0, row1);
+    case V_PROF: return launch_tp_v<V_PROF>(p, lut_ws, s, row0, row1);
   }
   return cudaErrorInvalidValue;
 }

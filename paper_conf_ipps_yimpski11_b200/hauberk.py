@@ -129,6 +129,10 @@ def lib():
         L.hauberk_timing_enable.argtypes = [I32]
         L.hauberk_timing_read.restype = I32
         L.hauberk_timing_read.argtypes = [I32, I32, P, P, P]
+        L.hauberk_part_units.restype = I32
+        L.hauberk_part_units.argtypes = [I32, P, P, P]
+        L.hauberk_run_part.restype = I32
+        L.hauberk_run_part.argtypes = [I32, P, I32, P, P, I64, I64, P]
         _lib = L
     return _lib
 
@@ -137,7 +141,7 @@ EXPORTED = ["hauberk_run_cp", "hauberk_run_mriq", "hauberk_run_tpacf", "hauberk_
             "hauberk_inject_campaign", "hauberk_decode", "hauberk_num_sites", "hauberk_strerror",
             "hauberk_last_error", "hauberk_version", "hauberk_launch_count", "hauberk_timing_enable",
             "hauberk_timing_read", "hauberk_campaign_create", "hauberk_campaign_run", "hauberk_campaign_destroy",
-            "hauberk_profile_search"]
+            "hauberk_profile_search", "hauberk_part_units", "hauberk_run_part"]
 
 
 def _check(status: int, where: str):
@@ -323,6 +327,23 @@ def run(dev, variant: int = HK_FT, ranges: Ranges | None = None, cb: torch.Tenso
     f = getattr(lib(), _RUN[dev.bench])
     st = f(C.byref(a), variant, C.byref(ranges) if ranges is not None else None, _ptr(cb), _ptr(samples), _stream(stream))
     _check(st, _RUN[dev.bench])
+
+
+def part_units(dev) -> tuple[int, int]:
+    """hauberk_part_units: (number of partition units, alignment granule) of a single run."""
+    a = dev.args()
+    u, g = C.c_int64(0), C.c_int64(0)
+    _check(lib().hauberk_part_units(dev.bench, C.byref(a), C.byref(u), C.byref(g)), "hauberk_part_units")
+    return int(u.value), int(g.value)
+
+
+def run_part(dev, begin: int, end: int, variant: int = HK_FT, ranges: Ranges | None = None,
+             cb: torch.Tensor | None = None, stream=None):
+    """hauberk_run_part: partition units [begin, end) of one single run (stream-asynchronous)."""
+    a = dev.args()
+    st = lib().hauberk_run_part(dev.bench, C.byref(a), variant, C.byref(ranges) if ranges is not None else None,
+                                _ptr(cb), begin, end, _stream(stream))
+    _check(st, "hauberk_run_part")
 
 
 def profile_ranges(dev, maxvar: int = 1, t0_exp10: int = -5, alpha: float = 1.0, stream=None) -> Ranges:

@@ -571,3 +571,47 @@ def test_guardian_real_crash_validation(bench):
     real_fail = sum(v for m in ("crash", "hang") for r, v in conf.get(m, {}).items() if r in ("crash", "hang"))
     assert real_fail >= 1  # the unguarded runs really dereference the corrupted addresses
     assert rep["done_with_model_fail_bits"] == 0  # no R16/R17 verdicts in unguarded runs
+
+
+# ------------------------------------------------------------- single-run sharding
+@pytest.mark.parametrize("world", [2, 3, 8])
+def test_single_run_parts_reassemble_the_whole_run_bit_exact(world):
+    """hauberk_run_part over a partition of the units (simulated ranks, one after another on one
+    GPU) reproduces the whole FT run bit for bit: CP rows and MRI-Q voxels in place, TPACF as the
+    sum of the partial histograms; no part raises an alarm.  Config shapes 4 / 2 / 3 for CP at
+    small atom count, MRI-Q and TPACF at full size."""
+    from paper_conf_ipps_yimpski11_b200 import parallel as par
+    probs = [W.cp_problem(300, 512, 512, seed=54321, h=0.1, bx=16, by=16, unroll=8), W.mriq_config2(), W.tpacf_config3()]
+    for b in range(3):
+        d = _mk(b, probs[b])
+        R = hk.profile_ranges(d)
+        assert _run(d, hk.HK_FT, R).alarm == 0
+        whole = [t.clone() for t in (d.output() if b == 1 else (d.output(),))]
+        units, gran = hk.part_units(d)
+        acc = torch.zeros_like(whole[0]) if b == 2 else None
+        for t in (d.output() if b == 1 else (d.output(),)):
+            t.fill_(float("nan") if t.dtype == torch.float32 else 0)
+        for r in range(world):
+            lo, hi = par.part_slice(units, gran, r, world)
+            cb = hk.new_control(DEV)
+            hk.run_part(d, lo, hi, hk.HK_FT, R, cb)
+            torch.cuda.synchronize()
+            c = hk.read_control(cb)
+            assert c.alarm == 0 and c.fail == 0, (b, r)
+            if b == 2:
+                acc += d.output()
+        got = [acc] if b == 2 else [t for t in (d.output() if b == 1 else (d.output(),))]
+        for g, w in zip(got, whole):
+            if g.dtype == torch.float32:
+                assert np.array_equal(_bits(g.cpu().numpy()), _bits(w.cpu().numpy())), b
+            else:
+                assert torch.equal(g, w), b
+
+
+def test_run_part_rejects_bad_ranges():
+    d = _mk(0, W.cp_small())
+    R = hk.profile_ranges(d)
+    units, gran = hk.part_units(d)
+    for lo, hi in [(-1, 8), (0, units + gran), (1, gran), (gran, gran - 1)]:
+        with pytest.raises(hk.HauberkError):
+            hk.run_part(d, lo, hi, hk.HK_FT, R, hk.new_control(DEV))

@@ -316,6 +316,12 @@ def main():
                             f"(the timed steps overlap the benchmarks' streams; serial step {ser_ms / ser_steps:.2f} ms vs "
                             f"concurrent {my_ms / args.steps:.2f} ms)",
                 "ops_per_pair": ops, "peak_source": f"{N_SM} SMs x {MUFU_PER_SM_CLK if dom < 2 else LANES_PER_SM_CLK}/clk/SM x {sm_mhz_peak:.0f} MHz ({clk_src})"}
+    # what actually binds the dominant kernel (ncu --set full of the same kernel, profiles/r01_ncu_fi_summary.txt)
+    roofline["limiter_ncu"] = {
+        2: "shared-memory path: l1tex 97.5 % of peak, issue 87 % (12.5 SASS instructions per pair vs 11 algorithmic ops)",
+        1: "XU (MUFU sin/cos) 87 % of peak, issue 75 %",
+        0: "XU (MUFU rsqrt); launch-bound at CP-s size",
+    }[dom]
     fi_split = {hk.BENCH_NAMES[b]: {"ms": round(fi[b][0], 3), "launches": fi[b][1], "pairs": fi[b][2], "serial_steps": ser_steps}
                 for b in range(3)}
     # traffic: DRAM bytes per launch of the same kernel/batch from the committed ncu capture

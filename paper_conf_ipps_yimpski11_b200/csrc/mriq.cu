@@ -23,7 +23,7 @@ constexpr int MQ_FI_THREADS = HK_MQ_FI_THREADS;  // campaign replicas: CTA size
 constexpr int MQ_FI_VPT = HK_MQ_FI_VPT;          // voxels per CUDA thread in the replicas
 constexpr int MQ_FI_UNROLL = HK_MQ_FI_UNROLL;
 #ifndef HK_MQ_UNROLL
-#define HK_MQ_UNROLL 16
+#define HK_MQ_UNROLL 32
 #endif
 constexpr int MQ_UNROLL = HK_MQ_UNROLL;  // single-run kernel
 #ifndef HK_MQ_THREADS
@@ -95,6 +95,14 @@ __device__ __forceinline__ void mriq_body(const MQParams& p, float4 (*tile)[MQ_T
   constexpr bool CNT = L || PROF;
   const uint32_t z = p.zz;
   const int32_t numK = p.numK;
+  // the first k-space tile is requested before the voxel prologue so its latency overlaps it
+  const int ntiles = (numK + MQ_TILE - 1) / MQ_TILE;
+  if (threadIdx.x == 0) {
+    mbar_init(&bar[0], 1);
+    mbar_init(&bar[1], 1);
+    fence_mbar_init();
+    if (ntiles > 0) bulk_g2s(tile[0], p.kv, (uint32_t)min(MQ_TILE, numK) * 16u, &bar[0]);
+  }
   int32_t xIndex[VPT];
   bool active[VPT];
   uint32_t chk[VPT], alarm[VPT];
@@ -123,14 +131,7 @@ __device__ __forceinline__ void mriq_body(const MQParams& p, float4 (*tile)[MQ_T
       if (NL) { chk[v] ^= fb(sZ[v]); alarm[v] |= (fb(p.z[opq(xi, z)]) != fb(sZ[v])) ? AL_DUP : 0u; }
     }
   }
-  const int ntiles = (numK + MQ_TILE - 1) / MQ_TILE;
-  if (threadIdx.x == 0) {
-    mbar_init(&bar[0], 1);
-    mbar_init(&bar[1], 1);
-    fence_mbar_init();
-  }
-  __syncthreads();
-  if (threadIdx.x == 0 && ntiles > 0) bulk_g2s(tile[0], p.kv, (uint32_t)min(MQ_TILE, numK) * 16u, &bar[0]);
+  __syncthreads();  // barrier init (above) visible to every waiter
   bool any_active = false;
 #pragma unroll
   for (int v = 0; v < VPT; ++v) any_active |= active[v];

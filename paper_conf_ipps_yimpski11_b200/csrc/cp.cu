@@ -12,6 +12,11 @@ namespace hk {
 
 constexpr int CP_TILE = 1024;  // atoms per stage (16 KB); 2 stages
 
+#ifndef HK_CP_AUNROLL
+#define HK_CP_AUNROLL 16
+#endif
+constexpr int CP_AUNROLL = HK_CP_AUNROLL;  // atom-loop unroll of the protected loop
+
 struct CPParams {
   const float4* atoms;  // (x, y, dz^2, q)
   float* grid;
@@ -84,7 +89,7 @@ __device__ __forceinline__ void cp_body(const CPParams& p, float4 (*tile)[CP_TIL
     mbar_wait(&bar[buf], (uint32_t)(t >> 1) & 1u);
     const float4* A = tile[buf];
     const int cnt = min(CP_TILE, numatoms - t * CP_TILE);
-#pragma unroll 4
+#pragma unroll(CP_AUNROLL)
     for (int a = 0; a < cnt; ++a) {
       const float4 at = A[a];
       const float dy = __fsub_rn(coory, at.y);

@@ -202,6 +202,11 @@ def main():
         # Fig. 13 columns: HAUBERK-NL, HAUBERK-L and HAUBERK vs the unprotected kernel
         cases = [("cp_cfg4", hk.CPDevice.from_problem(W.cp_config4(bx=16, by=16, unroll=8), dev), "xu", 1.0),
                  ("mriq_cfg2", devs[1], "xu", 2.0), ("tpacf_cfg3", devs[2], "alu", float(TPACF_OPS_PER_PAIR))]
+        # R-Naive: the unprotected kernel run twice on two copies of
+        # the data, then the outputs compared (hauberk_compare, on the device)
+        twins = {"cp_cfg4": hk.CPDevice.from_problem(W.cp_config4(bx=16, by=16, unroll=8), dev),
+                 "mriq_cfg2": hk.MRIQDevice.from_problem(W.mriq_config2(), dev),
+                 "tpacf_cfg3": hk.TPACFDevice.from_problem(W.tpacf_config3(), dev)}
         variants = (hk.HK_BASE, hk.HK_FT_NL, hk.HK_FT_L, hk.HK_FT)
         for name, d, pipe, ops in cases:
             R = hk.profile_ranges(d)
@@ -220,6 +225,24 @@ def main():
                         work = w
             hk.timing_enable(False)
             assert hk.read_control(cb).alarm == 0
+            # R-Naive: second BASE run on the twin copy, then the compare kernel (CUDA events)
+            tw = twins[name]
+            outs = lambda dd: [dd.output()] if not isinstance(dd.output(), tuple) else list(dd.output())
+            ccb = hk.new_control(dev)
+            tcmp = []
+            hk.run(d, hk.HK_BASE, R, cb)
+            for rep in range(12):
+                hk.run(tw, hk.HK_BASE, R, ccb)
+                flush.zero_()
+                c0, c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                c0.record()
+                for oa, ob in zip(outs(d), outs(tw)):
+                    hk.compare(oa, ob, ccb)
+                c1.record()
+                torch.cuda.synchronize()
+                if rep >= 2:
+                    tcmp.append(c0.elapsed_time(c1))
+            naive_alarm = hk.read_control(ccb).alarm
             med = {v: statistics.median(t[v]) for v in variants}
             tb, tf = med[hk.HK_BASE], med[hk.HK_FT]
             peak = mufu_peak if pipe == "xu" else lane_peak
@@ -228,10 +251,12 @@ def main():
             kernels[name] = {"base_ms": round(tb, 4), "ft_ms": round(tf, 4), "overhead_pct": overhead[name],
                              "overhead_nl_pct": round(100.0 * (med[hk.HK_FT_NL] / tb - 1.0), 2),
                              "overhead_l_pct": round(100.0 * (med[hk.HK_FT_L] / tb - 1.0), 2),
+                             "overhead_rnaive_pct": round(100.0 * ((2 * tb + statistics.median(tcmp)) / tb - 1.0), 2),
+                             "rnaive_compare_ms": round(statistics.median(tcmp), 4), "rnaive_alarm": naive_alarm,
                              "pairs": work, "bound": "alu", "pipe": "xu (MUFU)" if pipe == "xu" else "fp32/int lanes",
                              "achieved_gops": round(ach / 1e9, 1), "peak_gops": round(peak / 1e9, 1),
                              "frac": round(ach / peak, 4), "base_frac": round(work * ops / (tb * 1e-3) / peak, 4)}
-        del cases
+        del cases, twins
 
     # ---- campaign steps
     seed = 0x4841554245524B05

@@ -155,6 +155,12 @@ HK_API hk_status hauberk_run_tpacf(const hk_tpacf_args* args, int32_t variant, c
  * whole hist).  variant: HK_BASE / HK_FT / HK_FT_NL / HK_FT_L (profile over the whole input with
  * hauberk_profile_ranges and share the ranges).  hauberk_part_units returns the unit count and the
  * alignment granule.  HK_ERR_INVALID for a range outside [0, units) or misaligned. */
+/* R-Naive's compare step: bitwise compare of two
+ * device buffers of n_words 32-bit words (16-byte aligned), e.g. the outputs of two BASE runs on
+ * two copies of the inputs.  d_cb is reset, then alarm |= HK_ALARM_DUP and first_thread = the
+ * smallest differing word index if any word differs.  Stream-asynchronous. */
+HK_API hk_status hauberk_compare(const void* d_a, const void* d_b, int64_t n_words, hk_control* d_cb, void* stream);
+
 HK_API hk_status hauberk_part_units(int32_t bench, const void* args, int64_t* units, int64_t* granule);
 HK_API hk_status hauberk_run_part(int32_t bench, const void* args, int32_t variant, const hk_ranges* ranges,
                                   hk_control* d_cb, int64_t begin, int64_t end, void* stream);

@@ -177,3 +177,42 @@ cudaError_t classify_tpacf_launch(unsigned long long* hist0, int nr, int nb, con
 }
 
 }  // namespace hk
+
+// ---------------------------------------------------------------------------------------------
+// R-Naive's compare step (run the kernel twice on two copies of the
+// data and compare the outputs; the paper compares on the CPU, here on the device).  Bitwise
+// compare of two buffers of n 32-bit words; a differing word raises alarm bit 1 (duplicate
+// mismatch) and the smallest differing word index goes to first_thread (warp vote, one atomic
+// pair per warp with a mismatch).  16-byte loads, grid-stride, grid = SMs x 8.
+// ---------------------------------------------------------------------------------------------
+namespace hk {
+__global__ void __launch_bounds__(256) compare_kernel(const uint32_t* __restrict__ a, const uint32_t* __restrict__ b,
+                                                      int64_t n, hk_control* cb) {
+  const int64_t n4 = n / 4;
+  const uint4* __restrict__ a4 = reinterpret_cast<const uint4*>(a);
+  const uint4* __restrict__ b4 = reinterpret_cast<const uint4*>(b);
+  uint32_t first = 0xffffffffu;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += stride) {
+    const uint4 x = a4[i], y = b4[i];
+    if ((x.x ^ y.x) | (x.y ^ y.y) | (x.z ^ y.z) | (x.w ^ y.w)) {
+      const uint32_t w = (uint32_t)(4 * i) + (x.x != y.x ? 0u : x.y != y.y ? 1u : x.z != y.z ? 2u : 3u);
+      first = min(first, w);
+    }
+  }
+  for (int64_t i = 4 * n4 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride)
+    if (a[i] != b[i]) first = min(first, (uint32_t)i);
+  fold_alarm(cb, first != 0xffffffffu ? (uint32_t)AL_DUP : 0u, first);
+}
+
+cudaError_t compare_launch(const void* a, const void* b, int64_t n_words, hk_control* cb, cudaStream_t s) {
+  int dev = 0, nsm = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+  const int64_t want = (n_words / 4 + 255) / 256;
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(want, (int64_t)nsm * 8));
+  compare_kernel<<<grid, 256, 0, s>>>(static_cast<const uint32_t*>(a), static_cast<const uint32_t*>(b), n_words, cb);
+  count_launch();
+  return cudaGetLastError();
+}
+}  // namespace hk

@@ -71,6 +71,7 @@ cudaError_t decode_sort_launch(const DevCatalog cat[3], uint64_t seed, int64_t f
 // classify.cu
 cudaError_t control_init_launch(hk_control* cb, int n, cudaStream_t s);
 cudaError_t max_abs_launch(const float* g, int64_t n, float* d_out, cudaStream_t s);
+cudaError_t compare_launch(const void* a, const void* b, int64_t n_words, hk_control* cb, cudaStream_t s);
 cudaError_t classify_fp_launch(int bench, float* out0, int64_t elems, const float* golden, const float* d_M,
                                hk_control* cb0, const FaultRec* faults, int nrep, hk_outcome* records, int64_t first,
                                int64_t* counts, int64_t* site_counts, cudaStream_t s);

@@ -452,6 +452,16 @@ hk_status hauberk_run_tpacf(const hk_tpacf_args* args, int32_t variant, const hk
   return run_bench(HK_TPACF, args, variant, ranges, d_cb, d_samples, (cudaStream_t)stream);
 }
 
+hk_status hauberk_compare(const void* d_a, const void* d_b, int64_t n_words, hk_control* d_cb, void* stream) {
+  if (!d_a || !d_b || !d_cb || n_words < 0) return invalid("compare: bad arguments");
+  if (((uintptr_t)d_a | (uintptr_t)d_b) & 15u) return invalid("compare: buffers must be 16-byte aligned");
+  cudaStream_t s = (cudaStream_t)stream;
+  HK_CUDA(control_init_launch(d_cb, 1, s), "control init");
+  if (n_words == 0) return HK_OK;
+  HK_CUDA(compare_launch(d_a, d_b, n_words, d_cb, s), "compare");
+  return HK_OK;
+}
+
 hk_status hauberk_part_units(int32_t bench, const void* args, int64_t* units, int64_t* granule) {
   if (bench < 0 || bench > 2 || !units || !granule || !args_ok(bench, args)) return invalid("part_units: bad bench/args");
   if (bench == HK_CP) {

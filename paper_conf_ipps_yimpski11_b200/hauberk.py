@@ -19,6 +19,7 @@ LIB_PATH = os.environ.get("HAUBERK_LIB") or os.path.join(_HERE, "libhauberk.so")
 
 HK_CP, HK_MRIQ, HK_TPACF, HK_MIXED = 0, 1, 2, -1
 HK_BASE, HK_FT, HK_FT_NL, HK_FT_L, HK_PROFILE = 0, 1, 2, 3, 4
+HK_ALARM_DUP, HK_ALARM_CHECKSUM, HK_ALARM_RANGE, HK_ALARM_COUNT = 1, 2, 4, 8  # hk_control.alarm bits
 CLASS_NAMES = ["masked", "detected_masked", "detected", "undetected", "failure"]
 BENCH_NAMES = ["cp", "mriq", "tpacf"]
 ALL_SITES = (1 << 64) - 1
@@ -131,6 +132,8 @@ def lib():
         L.hauberk_timing_read.argtypes = [I32, I32, P, P, P]
         L.hauberk_part_units.restype = I32
         L.hauberk_part_units.argtypes = [I32, P, P, P]
+        L.hauberk_compare.restype = I32
+        L.hauberk_compare.argtypes = [P, P, I64, P, P]
         L.hauberk_run_part.restype = I32
         L.hauberk_run_part.argtypes = [I32, P, I32, P, P, I64, I64, P]
         _lib = L
@@ -141,7 +144,7 @@ EXPORTED = ["hauberk_run_cp", "hauberk_run_mriq", "hauberk_run_tpacf", "hauberk_
             "hauberk_inject_campaign", "hauberk_decode", "hauberk_num_sites", "hauberk_strerror",
             "hauberk_last_error", "hauberk_version", "hauberk_launch_count", "hauberk_timing_enable",
             "hauberk_timing_read", "hauberk_campaign_create", "hauberk_campaign_run", "hauberk_campaign_destroy",
-            "hauberk_profile_search", "hauberk_part_units", "hauberk_run_part"]
+            "hauberk_profile_search", "hauberk_part_units", "hauberk_run_part", "hauberk_compare"]
 
 
 def _check(status: int, where: str):
@@ -327,6 +330,13 @@ def run(dev, variant: int = HK_FT, ranges: Ranges | None = None, cb: torch.Tenso
     f = getattr(lib(), _RUN[dev.bench])
     st = f(C.byref(a), variant, C.byref(ranges) if ranges is not None else None, _ptr(cb), _ptr(samples), _stream(stream))
     _check(st, _RUN[dev.bench])
+
+
+def compare(a: torch.Tensor, b: torch.Tensor, cb: torch.Tensor, stream=None):
+    """hauberk_compare (R-Naive's compare step): bitwise compare of two equally sized buffers."""
+    assert a.numel() * a.element_size() == b.numel() * b.element_size() and (a.numel() * a.element_size()) % 4 == 0
+    _check(lib().hauberk_compare(_ptr(a), _ptr(b), a.numel() * a.element_size() // 4, _ptr(cb), _stream(stream)),
+           "hauberk_compare")
 
 
 def part_units(dev) -> tuple[int, int]:

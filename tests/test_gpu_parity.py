@@ -615,3 +615,41 @@ def test_run_part_rejects_bad_ranges():
     for lo, hi in [(-1, 8), (0, units + gran), (1, gran), (gran, gran - 1)]:
         with pytest.raises(hk.HauberkError):
             hk.run_part(d, lo, hi, hk.HK_FT, R, hk.new_control(DEV))
+
+
+# ------------------------------------------------------------------ R-Naive compare
+@pytest.mark.parametrize("n", [1, 7, 4096, 262147])
+def test_rnaive_compare_flags_exactly_the_first_differing_word(n):
+    g = torch.Generator().manual_seed(n)
+    a = torch.randint(-2**31, 2**31 - 1, (n,), generator=g, dtype=torch.int32).to(DEV)
+    b = a.clone()
+    cb = hk.new_control(DEV)
+    hk.compare(a, b, cb)
+    torch.cuda.synchronize()
+    c = hk.read_control(cb)
+    assert c.alarm == 0 and c.first_thread == 0xFFFFFFFF
+    for pos in sorted({n - 1, n // 2, (3 * n) // 4}):
+        b = a.clone()
+        b[pos] ^= 1 << (pos % 32)
+        if pos + 1 < n:
+            b[n - 1] ^= 1 << 7  # a later difference must not mask the first
+        hk.compare(a, b, cb)
+        torch.cuda.synchronize()
+        c = hk.read_control(cb)
+        assert c.alarm == hk.HK_ALARM_DUP and c.first_thread == pos, (n, pos)
+
+
+def test_rnaive_two_base_runs_on_copies_agree():
+    """R-Naive's premise on this hardware: the unprotected kernel run twice on two copies of the
+    inputs produces bitwise-identical outputs (so any difference would be a fault)."""
+    for b, p in enumerate([W.cp_small(), W.mriq_small(), W.tpacf_small()]):
+        d1, d2 = _mk(b, p), _mk(b, p)
+        hk.run(d1, hk.HK_BASE)
+        hk.run(d2, hk.HK_BASE)
+        cb = hk.new_control(DEV)
+        o1 = d1.output() if b == 1 else (d1.output(),)
+        o2 = d2.output() if b == 1 else (d2.output(),)
+        for x, y in zip(o1, o2):
+            hk.compare(x, y, cb)
+            torch.cuda.synchronize()
+            assert hk.read_control(cb).alarm == 0

@@ -457,7 +457,8 @@ __device__ __forceinline__ void tp_drain(const TPParams& p, const TPSmem& S, con
 }
 
 template <int V>
-__global__ void __launch_bounds__(TP_THREADS, HK_TP_STD_MINB) tpacf_kernel(const TPParams p, const TPSched q) {
+// the NL-only variant (Fig. 13 decomposition) spills at 56 registers: it gets 64 (8 CTAs per SM)
+__global__ void __launch_bounds__(TP_THREADS, V == V_NL ? 8 : HK_TP_STD_MINB) tpacf_kernel(const TPParams p, const TPSched q) {
   extern __shared__ __align__(16) unsigned char tp_smem[];
   __shared__ int item_s, last_s;
   const TPSmem S = tp_carve(tp_smem, p.C);

@@ -16,12 +16,16 @@ constexpr int MQ_TILE = 1024;  // k-samples per stage (16 KB)
 #ifndef HK_MQ_FI_VPT
 #define HK_MQ_FI_VPT 2
 #endif
+#ifndef HK_MQ_FI_TILE
+#define HK_MQ_FI_TILE 1024
+#endif
 #ifndef HK_MQ_FI_UNROLL
 #define HK_MQ_FI_UNROLL 8
 #endif
 constexpr int MQ_FI_THREADS = HK_MQ_FI_THREADS;  // campaign replicas: CTA size
 constexpr int MQ_FI_VPT = HK_MQ_FI_VPT;          // voxels per CUDA thread in the replicas
 constexpr int MQ_FI_UNROLL = HK_MQ_FI_UNROLL;
+constexpr int MQ_FI_TILE = HK_MQ_FI_TILE;        // k-samples per stage in the replicas
 #ifndef HK_MQ_UNROLL
 #define HK_MQ_UNROLL 32
 #endif
@@ -89,19 +93,19 @@ __global__ void __launch_bounds__(256) mriq_phimag_kernel(const float* __restric
 // b*(blockDim*VPT) + j*blockDim + t.  Each keeps its own registers, detectors and counter; they
 // share every k-space load (VPT = 2 in the campaign replicas, 1 for the single-run kernel whose
 // grid is small).
-template <int V, bool EXACT, bool ADD, int VPT, int UNR = (VPT == 1 ? MQ_UNROLL : MQ_FI_UNROLL)>
-__device__ __forceinline__ void mriq_body(const MQParams& p, float4 (*tile)[MQ_TILE], uint64_t* bar, int bxi) {
+template <int V, bool EXACT, bool ADD, int VPT, int UNR = (VPT == 1 ? MQ_UNROLL : MQ_FI_UNROLL), int TILE = MQ_TILE>
+__device__ __forceinline__ void mriq_body(const MQParams& p, float4 (*tile)[TILE], uint64_t* bar, int bxi) {
   constexpr bool NL = (V & V_NL) != 0, L = (V & V_L) != 0, PROF = (V & V_PROF) != 0;
   constexpr bool CNT = L || PROF;
   const uint32_t z = p.zz;
   const int32_t numK = p.numK;
   // the first k-space tile is requested before the voxel prologue so its latency overlaps it
-  const int ntiles = (numK + MQ_TILE - 1) / MQ_TILE;
+  const int ntiles = (numK + TILE - 1) / TILE;
   if (threadIdx.x == 0) {
     mbar_init(&bar[0], 1);
     mbar_init(&bar[1], 1);
     fence_mbar_init();
-    if (ntiles > 0) bulk_g2s(tile[0], p.kv, (uint32_t)min(MQ_TILE, numK) * 16u, &bar[0]);
+    if (ntiles > 0) bulk_g2s(tile[0], p.kv, (uint32_t)min(TILE, numK) * 16u, &bar[0]);
   }
   int32_t xIndex[VPT];
   bool active[VPT];
@@ -139,13 +143,13 @@ __device__ __forceinline__ void mriq_body(const MQParams& p, float4 (*tile)[MQ_T
     const int buf = t & 1;
     if (threadIdx.x == 0 && t + 1 < ntiles) {
       fence_proxy_async();
-      bulk_g2s(tile[buf ^ 1], p.kv + (size_t)(t + 1) * MQ_TILE, (uint32_t)min(MQ_TILE, numK - (t + 1) * MQ_TILE) * 16u,
+      bulk_g2s(tile[buf ^ 1], p.kv + (size_t)(t + 1) * TILE, (uint32_t)min(TILE, numK - (t + 1) * TILE) * 16u,
                &bar[buf ^ 1]);
     }
     mbar_wait(&bar[buf], (uint32_t)(t >> 1) & 1u);
     if (any_active) {
       const float4* A = tile[buf];
-      const int cnt = min(MQ_TILE, numK - t * MQ_TILE);
+      const int cnt = min(TILE, numK - t * TILE);
 #pragma unroll(UNR)
       for (int a = 0; a < cnt; ++a) {
         const float4 k4 = A[a];
@@ -412,7 +416,7 @@ done:
 
 template <int KIND, bool EXACT>
 __global__ void __launch_bounds__(MQ_FI_THREADS) mriq_fi_kernel(const MQFIParams q) {
-  __shared__ __align__(128) float4 tile[2][MQ_TILE];
+  __shared__ __align__(128) float4 tile[2][MQ_FI_TILE];
   __shared__ __align__(8) uint64_t bar[2];
   const int64_t ncta = gridDim.x, vpc = MQ_FI_VPT * (int64_t)blockDim.x;
   int r;
@@ -427,7 +431,7 @@ __global__ void __launch_bounds__(MQ_FI_THREADS) mriq_fi_kernel(const MQFIParams
   p.cb = q.cb0 + r;
   if (KIND == MK_PHIMAG) p.kv = q.kv0 + (int64_t)r * p.numK;  // this replica's (possibly faulted) k-space
   if (KIND == MK_PHIMAG || !faulted) {
-    mriq_body<V_NL | V_L, EXACT, true, MQ_FI_VPT, MQ_FI_UNROLL>(p, tile, bar, bxi);
+    mriq_body<V_NL | V_L, EXACT, true, MQ_FI_VPT, MQ_FI_UNROLL, MQ_FI_TILE>(p, tile, bar, bxi);
   } else {
     ReplicaSinkF S{{p.qr, p.qi}, p.cb};
 #pragma unroll 1

@@ -43,6 +43,7 @@ def parse():
     ap.add_argument("--batch", type=int, default=0)
     ap.add_argument("--no-overhead", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--cpu-procs", type=int, default=0, help="oracle processes for the all-cores CPU line (0: all, <= 64)")
     ap.add_argument("--no-multibit", action="store_true")
     ap.add_argument("--replay-count", type=int, default=1000000, help="injections per rank for the replay-mode line")
     ap.add_argument("--no-fp-study", action="store_true")
@@ -122,6 +123,27 @@ def oracle_replica_sample(seed: int, first: int, count: int):
         O.campaign(-1, probs, R, seed, n, 1, exact=0, mode=0, records=False)
         per[b].append(time.perf_counter() - t0)
     return per
+
+
+def _oracle_worker(job):
+    seed, first, count = job
+    return oracle_replica_sample(seed, first, count)
+
+
+def oracle_all_cores(seed: int, first: int, procs: int):
+    """The same oracle, unchanged, on `procs` forked worker processes (one per host core, no CUDA in
+    the children), each timing one (CP-s, MRI-Q, TPACF) injection triple; throughput = injections / wall."""
+    import multiprocessing as mp
+
+    oracle_replica_sample(seed, 0, 0)  # inputs and ranges prepared in the parent, inherited by fork
+    ctx = mp.get_context("fork")
+    with ctx.Pool(procs) as pool:
+        pool.map(_oracle_worker, [(seed, 0, 0)] * procs)  # workers started outside the timing
+        t0 = time.perf_counter()
+        res = pool.map(_oracle_worker, [(seed, first + 3 * w, 3) for w in range(procs)], chunksize=1)
+        wall = time.perf_counter() - t0
+    n = sum(len(p[b]) for p in res for b in range(3))
+    return n / wall, n, wall
 
 
 def run_reference(args):
@@ -412,6 +434,12 @@ def main():
         cpu = {"value": round(3.0 / sum(tm), 4), "unit": "injections/s", "cores": 1, "kind": "oracle",
                "sample": "6 config-5 injections (2 each CP-s / MRI-Q / TPACF), replica mode (full program run each), "
                          f"mean s/injection cp={tm[0]:.4f} mriq={tm[1]:.3f} tpacf={tm[2]:.3f}"}
+        procs = args.cpu_procs if args.cpu_procs > 0 else min(64, len(os.sched_getaffinity(0)))
+        if procs > 1:
+            v_all, n_all, wall = oracle_all_cores(seed, 300, procs)
+            cpu["all_cores"] = {"value": round(v_all, 4), "unit": "injections/s", "cores": procs, "kind": "oracle",
+                                "sample": f"{n_all} config-5 injections ({procs} forked processes x one CP-s / MRI-Q / "
+                                          f"TPACF triple), replica mode, {wall:.1f} s wall"}
 
     session.close()
 

@@ -167,6 +167,33 @@ def test_mriq_config2_sampled_parity():
     assert _fp_close(gqi[tids], oqi.astype(np.float64), mass, 16) == 0
 
 
+@pytest.mark.parametrize("shape", [(1, 1), (33, 0), (70, 2049), (300, 1024), (129, 1025)])
+def test_mriq_edge_shapes_exact_bit_exact(shape):
+    """Single voxel / single k-sample, an empty k-loop (R19: count checked, range skipped), k-space
+    ending exactly on and one past a 1,024-sample tile, ragged voxel tails: EXACT mode bit-equal
+    outputs, profiled ranges equal to the oracle's, no fault-free alarm in any variant."""
+    nv, nk = shape
+    p = W.mriq_problem(8, nk, n_vox=nv, seed=nv * 7919 + nk)
+    d = _mk(1, p, exact=1)
+    R = hk.profile_ranges(d, maxvar=2)
+    assert R.as_list() == O.ranges_to_list(O.profile_ranges(O.MRIQ, p, maxvar=2, exact=1))
+    (oqr, oqi), _, _ = O.run(O.MRIQ, p, exact=1)
+    for v in (hk.HK_FT, hk.HK_BASE, hk.HK_FT_NL, hk.HK_FT_L):
+        assert _run(d, v, R).alarm == 0
+        gqr, gqi = _out_np(d)
+        assert np.array_equal(_bits(gqr), _bits(oqr)) and np.array_equal(_bits(gqi), _bits(oqi))
+
+
+def test_mriq_multitile_campaign_exact_bit_exact():
+    """Replica campaign on a k-space of three tiles with a one-sample tail: every record (site,
+    thread, instance, mask, class, alarm, failure) equal to the oracle's."""
+    probs = [None, W.mriq_problem(8, 2049, n_vox=130, seed=5), None]
+    gc, grec, oc, orec = _campaign_pair(probs, 0x3C0FFEE, 400, exact=1, mode=1)
+    for k in ("index", "bench", "site", "thread", "inst", "mask", "cls", "alarm", "fail"):
+        assert np.array_equal(grec[k], orec[k]), k
+    assert np.array_equal(gc, oc)
+
+
 # ---------------------------------------------------------------------------------------------- TPACF
 @pytest.mark.parametrize("shape", [(300, 2, 64), (70, 1, 16), (129, 3, 1000), (257, 1, 7)])
 def test_tpacf_hist_bit_exact(shape):

@@ -77,6 +77,22 @@ def test_cp_output_parity(unroll, exact):
         assert np.array_equal(_bits(_out_np(d)), _bits(got)), v  # instrumentation never changes the output
 
 
+@pytest.mark.parametrize("n_atoms", [1, 1024, 1025, 2049])
+@pytest.mark.parametrize("unroll", [4, 8])
+def test_cp_atom_tile_boundaries_exact_bit_exact(n_atoms, unroll):
+    """Atom counts of one atom, exactly one 1,024-atom bulk-copy tile, one past it, and two tiles
+    plus one (the double-buffered ring wraps with a one-atom tail): EXACT mode bit-equal outputs and
+    oracle-equal ranges at maxvar = U, every variant alarm-free and output-identical."""
+    p = W.cp_problem(n_atoms, 64, 16, seed=n_atoms, bx=8 if unroll == 8 else 16, by=8, unroll=unroll)
+    d = _mk(0, p, exact=1)
+    R = hk.profile_ranges(d, maxvar=unroll)
+    assert R.as_list() == O.ranges_to_list(O.profile_ranges(O.CP, p, maxvar=unroll, exact=1))
+    ora, _, _ = O.run(O.CP, p, exact=1)
+    for v in (hk.HK_FT, hk.HK_BASE, hk.HK_FT_NL, hk.HK_FT_L):
+        assert _run(d, v, R).alarm == 0
+        assert np.array_equal(_bits(_out_np(d)), _bits(ora)), v
+
+
 def test_cp_ranges_parity_exact_and_fast():
     p = W.cp_small()
     for exact in (1, 0):
@@ -195,7 +211,8 @@ def test_mriq_multitile_campaign_exact_bit_exact():
 
 
 # ---------------------------------------------------------------------------------------------- TPACF
-@pytest.mark.parametrize("shape", [(300, 2, 64), (70, 1, 16), (129, 3, 1000), (257, 1, 7)])
+@pytest.mark.parametrize("shape", [(300, 2, 64), (70, 1, 16), (129, 3, 1000), (257, 1, 7), (1, 1, 64), (2, 1, 1),
+                                   (33, 2, 32), (513, 1, 256)])
 def test_tpacf_hist_bit_exact(shape):
     n, nr, chunk = shape
     p = W.tpacf_small(n=n, n_rand=nr, chunk=chunk)

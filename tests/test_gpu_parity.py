@@ -440,14 +440,16 @@ def test_campaign_concurrent_streams_equal_serial(monkeypatch):
         assert np.array_equal(a[f], b[f]), f
 
 
-@pytest.mark.parametrize("k", [3, 15])
-def test_campaign_multibit_exact_mode_bit_exact(k):
+@pytest.mark.parametrize("gmode", [0, 1])
+@pytest.mark.parametrize("k", [3, 6, 10, 15])
+def test_campaign_multibit_exact_mode_bit_exact(k, gmode):
+    """Fig. 14's bit counts (L2605-2634), GPU replica (0) and replay (1) modes vs the oracle."""
     probs = [W.cp_small(), W.mriq_problem(5, 41, n_vox=100, seed=4), W.tpacf_small(n=90, n_rand=1, chunk=32)]
     devs = [_mk(b, probs[b], 1) for b in range(3)]
     gr = [hk.profile_ranges(d) for d in devs]
     counts = torch.zeros((3, 5), dtype=torch.int64, device=DEV)
     rec = hk.records_tensor(600, DEV)
-    hk.inject_campaign(-1, devs, gr, 0xF00D, 0, 600, counts, records=rec, exact=1, nbits=k)
+    hk.inject_campaign(-1, devs, gr, 0xF00D, 0, 600, counts, records=rec, exact=1, nbits=k, mode=gmode)
     torch.cuda.synchronize()
     orr = [O.profile_ranges(b, probs[b], exact=1) for b in range(3)]
     oc, orec = O.campaign(-1, probs, orr, 0xF00D, 0, 600, exact=1, mode=1, nbits=k)

@@ -235,6 +235,8 @@ struct MQFIParams {
   int64_t stride;
   const float4* kv0;  // PhiMag-site replicas: per-replica k-space [nrep][numK]
   hk_control* cb0;
+  int64_t ncta;  // CTAs per replica (the replica kernel walks ncta * nrep items; the grid may be smaller)
+  int32_t nrep;
 };
 
 // Per-thread FI&FT program of voxel t.  t_dup: the duplicate of N0 recomputed from launch indices
@@ -414,32 +416,45 @@ done:
   fold_alarm(cb, alarm, (uint32_t)k);
 }
 
+// Items L = (replica, CTA) in fi_order; by default one per CTA of a (ncta, nrep) grid.  With
+// HK_MQ_FI_PERSIST = c the grid holds c CTAs per SM that walk the items (experiment: leaves room
+// for TPACF replica CTAs on the same SMs); the k-space mbarriers are invalidated between items.
 template <int KIND, bool EXACT>
 __global__ void __launch_bounds__(MQ_FI_THREADS) mriq_fi_kernel(const MQFIParams q) {
   __shared__ __align__(128) float4 tile[2][MQ_FI_TILE];
   __shared__ __align__(8) uint64_t bar[2];
-  const int64_t ncta = gridDim.x, vpc = MQ_FI_VPT * (int64_t)blockDim.x;
-  int r;
-  int64_t cta;
-  const bool faulted = fi_order((int64_t)blockIdx.y * gridDim.x + blockIdx.x, ncta, (int)gridDim.y,
-                                [&](int rr) { return clamp_cta(q.faults[rr].thread / vpc, ncta); }, &r, &cta);
-  const FaultRec f = q.faults[r];
-  const int bxi = (int)cta;
-  MQParams p = q.base;
-  p.qr = q.out0 + (int64_t)r * q.stride;
-  p.qi = p.qr + p.numX;
-  p.cb = q.cb0 + r;
-  if (KIND == MK_PHIMAG) p.kv = q.kv0 + (int64_t)r * p.numK;  // this replica's (possibly faulted) k-space
-  if (KIND == MK_PHIMAG || !faulted) {
-    mriq_body<V_NL | V_L, EXACT, true, MQ_FI_VPT, MQ_FI_UNROLL, MQ_FI_TILE>(p, tile, bar, bxi);
-  } else {
-    ReplicaSinkF S{{p.qr, p.qi}, p.cb};
+  const int64_t ncta = q.ncta, vpc = MQ_FI_VPT * (int64_t)blockDim.x, total = ncta * q.nrep;
+  const int64_t step = (int64_t)gridDim.x * gridDim.y;
+  for (int64_t L = (int64_t)blockIdx.y * gridDim.x + blockIdx.x; L < total; L += step) {
+    int r;
+    int64_t cta;
+    const bool faulted = fi_order(L, ncta, q.nrep, [&](int rr) { return clamp_cta(q.faults[rr].thread / vpc, ncta); }, &r, &cta);
+    const FaultRec f = q.faults[r];
+    const int bxi = (int)cta;
+    MQParams p = q.base;
+    p.qr = q.out0 + (int64_t)r * q.stride;
+    p.qi = p.qr + p.numX;
+    p.cb = q.cb0 + r;
+    if (KIND == MK_PHIMAG) p.kv = q.kv0 + (int64_t)r * p.numK;  // this replica's (possibly faulted) k-space
+    if (KIND == MK_PHIMAG || !faulted) {
+      mriq_body<V_NL | V_L, EXACT, true, MQ_FI_VPT, MQ_FI_UNROLL, MQ_FI_TILE>(p, tile, bar, bxi);
+      if (L + step < total) {  // next item re-initialises the barriers
+        __syncthreads();
+        if (threadIdx.x == 0) {
+          asm volatile("mbarrier.inval.shared::cta.b64 [%0];" ::"r"(smem_u32(&bar[0])) : "memory");
+          asm volatile("mbarrier.inval.shared::cta.b64 [%0];" ::"r"(smem_u32(&bar[1])) : "memory");
+        }
+        __syncthreads();
+      }
+    } else {
+      ReplicaSinkF S{{p.qr, p.qi}, p.cb};
 #pragma unroll 1
-    for (int vox = 0; vox < MQ_FI_VPT; ++vox) {
-      const int32_t t = bxi * (MQ_FI_VPT * blockDim.x) + vox * blockDim.x + threadIdx.x;
-      if (t < p.numX) {
-        const int32_t t_dup = (int32_t)((bxi ^ p.zz) * (MQ_FI_VPT * blockDim.x) + vox * blockDim.x + (threadIdx.x ^ p.zz));
-        mriq_fi_program<KIND, EXACT>(p, f, t, t_dup, t == f.thread, (uint64_t)(uintptr_t)p.qr, (uint64_t)(uintptr_t)p.qi, S);
+      for (int vox = 0; vox < MQ_FI_VPT; ++vox) {
+        const int32_t t = bxi * (MQ_FI_VPT * blockDim.x) + vox * blockDim.x + threadIdx.x;
+        if (t < p.numX) {
+          const int32_t t_dup = (int32_t)((bxi ^ p.zz) * (MQ_FI_VPT * blockDim.x) + vox * blockDim.x + (threadIdx.x ^ p.zz));
+          mriq_fi_program<KIND, EXACT>(p, f, t, t_dup, t == f.thread, (uint64_t)(uintptr_t)p.qr, (uint64_t)(uintptr_t)p.qi, S);
+        }
       }
     }
   }
@@ -588,6 +603,14 @@ template <int KIND, bool EXACT>
 static cudaError_t launch_mq_fi_k(const MQFIParams& q, int nrep, cudaStream_t s) {
   constexpr int vpc = MQ_FI_VPT * MQ_FI_THREADS;
   dim3 grid((q.base.numX + vpc - 1) / vpc, nrep);
+  static const int persist = [] { const char* v = getenv("HK_MQ_FI_PERSIST"); return v ? atoi(v) : 0; }();
+  if (persist > 0) {
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const int64_t items = (int64_t)grid.x * nrep, cap = (int64_t)persist * sms;
+    if (items > cap) grid = dim3((unsigned)cap, 1);
+  }
   TimedScope ts(HK_MRIQ, 1, (double)q.base.numX * (double)q.base.numK * nrep, s);
   mriq_fi_kernel<KIND, EXACT><<<grid, MQ_FI_THREADS, 0, s>>>(q);
   count_launch();
@@ -641,6 +664,8 @@ cudaError_t mriq_fi_launch(int kind, const hk_mriq_args& a, const DevRanges& R, 
   q.out0 = out0;
   q.stride = stride;
   q.cb0 = cb0;
+  q.ncta = (a.n_vox + MQ_FI_VPT * MQ_FI_THREADS - 1) / (MQ_FI_VPT * MQ_FI_THREADS);
+  q.nrep = nrep;
   if (real && kind != MK_PHIMAG) {
     dim3 grid((a.n_vox + 255) / 256, nrep);
     if (a.exact) mriq_real_kernel<true><<<grid, 256, 0, s>>>(q, kind);

@@ -699,3 +699,38 @@ def test_rnaive_two_base_runs_on_copies_agree():
             hk.compare(x, y, cb)
             torch.cuda.synchronize()
             assert hk.read_control(cb).alarm == 0
+
+
+_PERSIST_SNIPPET = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, '.')
+import oracle as O, workloads as W
+from paper_conf_ipps_yimpski11_b200 import hauberk as hk
+p = W.mriq_problem(8, 2049, n_vox=300, seed=9)
+d = hk.MRIQDevice.from_problem(p, 'cuda', exact=1)
+R = hk.profile_ranges(d)
+counts = torch.zeros((3, 5), dtype=torch.int64, device='cuda')
+rec = hk.records_tensor(500, 'cuda')
+hk.inject_campaign(1, [None, d, None], [None, R, None], 0xCAFE, 0, 500, counts, records=rec, exact=1, batch=64)
+torch.cuda.synchronize()
+oc, orec = O.campaign(1, [None, p, None], [None, O.profile_ranges(1, p, exact=1), None], 0xCAFE, 0, 500, exact=1, mode=1)
+g = hk.records_numpy(rec)
+for k in ('site', 'thread', 'inst', 'mask', 'cls', 'alarm', 'fail'):
+    assert np.array_equal(g[k], orec[k]), k
+assert np.array_equal(counts.cpu().numpy(), oc)
+print('persist ok')
+"""
+
+
+def test_mriq_replicas_grid_capped_walk_equals_oracle():
+    """HK_MQ_FI_PERSIST=1 (read once per process, hence a child): one CTA per SM walks every
+    (replica, CTA) item of 64-replica launches, re-initialising the k-space mbarriers between
+    items; records equal to the oracle's."""
+    import subprocess
+    import sys
+
+    env = dict(os.environ, HK_MQ_FI_PERSIST="1")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", _PERSIST_SNIPPET], cwd=root, env=env, capture_output=True, text=True,
+                       timeout=600)
+    assert r.returncode == 0 and "persist ok" in r.stdout, r.stdout + r.stderr

@@ -50,11 +50,12 @@ class MRIQArgs(C.Structure):
 
 class TPACFArgs(C.Structure):
     _fields_ = [("pts", C.c_void_p), ("edges", C.c_void_p), ("n", C.c_int32), ("n_rand", C.c_int32),
-                ("n_bins", C.c_int32), ("chunk", C.c_int32)]
+                ("n_bins", C.c_int32)]
 
 
 class Fault(C.Structure):
-    _fields_ = [("site", C.c_int32), ("pad", C.c_int32), ("thread", C.c_int64), ("inst", C.c_int64), ("mask", C.c_uint64)]
+    # hang: R17 watchdog factor T of this injection (0 = the paper's 10)
+    _fields_ = [("site", C.c_int32), ("hang", C.c_int32), ("thread", C.c_int64), ("inst", C.c_int64), ("mask", C.c_uint64)]
 
 
 class RunInfo(C.Structure):
@@ -119,9 +120,18 @@ def lib():
         L.ora_nsites.restype = C.c_int32; L.ora_nsites.argtypes = [C.c_int32, C.c_int32]
         L.ora_site_info.restype = None; L.ora_site_info.argtypes = [C.c_int32, C.c_int32, C.c_int32, P, P]
         L.ora_decode.restype = C.c_int
-        L.ora_decode.argtypes = [C.c_int32, P, P, C.c_uint64, C.c_int32, C.c_int64, C.c_int64, P, P]
+        L.ora_decode.argtypes = [C.c_int32, P, P, C.c_uint64, C.c_int32, C.c_int32, C.c_int64, C.c_int64, P, P]
         L.ora_campaign.restype = C.c_int
-        L.ora_campaign.argtypes = [C.c_int32, P, P, P, C.c_uint64, C.c_int32, C.c_int64, C.c_int64, C.c_int32, C.c_int32, P, P]
+        L.ora_campaign.argtypes = [C.c_int32, P, P, P, C.c_uint64, C.c_int32, C.c_int64, C.c_int64, C.c_int32, C.c_int32,
+                                   C.c_int32, C.c_int32, P, P]
+        L.ora_detector_site.restype = C.c_int32; L.ora_detector_site.argtypes = [C.c_int32, C.c_int32, C.c_int32]
+        L.ora_a6_count.restype = C.c_int32; L.ora_a6_count.argtypes = [C.c_int32, P, C.c_int32, P, P, P, C.c_int32]
+        L.ora_a6_select.restype = C.c_int32; L.ora_a6_select.argtypes = [C.c_int32, P, P, C.c_int32, P, P, C.c_int32, P]
+        L.ora_in_range.restype = C.c_int32; L.ora_in_range.argtypes = [P, C.c_int32, C.c_float]
+        L.ora_extend_ranges.restype = C.c_int32; L.ora_extend_ranges.argtypes = [P, P, C.c_int32]
+        L.ora_alpha_step.restype = C.c_float; L.ora_alpha_step.argtypes = [C.c_float, C.c_double, C.c_double, C.c_double]
+        L.ora_diagnose.restype = C.c_int32; L.ora_diagnose.argtypes = [C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32, C.c_int32]
+        L.ora_coverage.restype = C.c_int32; L.ora_coverage.argtypes = [P, P]
         _lib = L
     return _lib
 
@@ -150,7 +160,7 @@ def mriq_args(p) -> MRIQArgs:
 def tpacf_args(p) -> TPACFArgs:
     pts = np.ascontiguousarray(p.pts, dtype=np.float32)
     edges = np.ascontiguousarray(p.edges, dtype=np.float32)
-    a = TPACFArgs(_p(pts), _p(edges), p.n, p.n_rand, p.n_bins, p.chunk)
+    a = TPACFArgs(_p(pts), _p(edges), p.n, p.n_rand, p.n_bins)
     a._keep = (pts, edges)
     return a
 
@@ -159,8 +169,8 @@ def make_args(bench: int, p):
     return (cp_args, mriq_args, tpacf_args)[bench](p)
 
 
-def fault(site: int, thread: int, inst: int, mask: int) -> Fault:
-    return Fault(site, 0, thread, inst, mask)
+def fault(site: int, thread: int, inst: int, mask: int, hang: int = 0) -> Fault:
+    return Fault(site, hang, thread, inst, mask)
 
 
 # ------------------------------------------------------------------------------------------------
@@ -247,9 +257,12 @@ def ranges_to_list(R: Ranges):
 
 
 def campaign(bench_mode: int, problems, ranges, seed: int, first: int, count: int, exact: int = 0,
-             mode: int = 1, site_masks=DEFAULT_SITE_MASKS, records: bool = True, nbits: int = 1):
+             mode: int = 1, site_masks=DEFAULT_SITE_MASKS, records: bool = True, nbits: int = 1,
+             variant: int = 0, hang_factor: int = 0):
     """Seeded campaign.  problems/ranges: 3-lists indexed by bench (None where unused).
-    mode 1 = replay, 0 = replica.  Returns (counts int64[3,5], records structured array)."""
+    mode 1 = replay, 0 = replica; variant 0 = FI&FT binary, 1 = FI-only binary (original program's
+    sites, no detectors); hang_factor = R17's T (0 = 10).
+    Returns (counts int64[3,5], records structured array)."""
     L = lib()
     argv = [make_args(b, problems[b]) if problems[b] is not None else None for b in range(3)]
     aptr = (C.c_void_p * 3)(*[C.cast(C.byref(a), C.c_void_p) if a is not None else None for a in argv])
@@ -258,21 +271,22 @@ def campaign(bench_mode: int, problems, ranges, seed: int, first: int, count: in
     masks = (C.c_uint64 * 3)(*site_masks)
     counts = np.zeros((3, 5), dtype=np.int64)
     recs = np.zeros(count, dtype=RECORD_DTYPE) if records else None
-    rc = L.ora_campaign(bench_mode, aptr, rptr, masks, seed, nbits, first, count, exact, mode,
+    rc = L.ora_campaign(bench_mode, aptr, rptr, masks, seed, nbits, first, count, exact, mode, variant, hang_factor,
                         _p(recs) if records else None, _p(counts))
     if rc != 0:
         raise RuntimeError(f"oracle campaign failed rc={rc} (1 = bad args/empty catalogue, 2 = fault-free alarm)")
     return counts, recs
 
 
-def decode(bench_mode: int, problems, seed: int, first: int, count: int, site_masks=DEFAULT_SITE_MASKS, nbits: int = 1):
+def decode(bench_mode: int, problems, seed: int, first: int, count: int, site_masks=DEFAULT_SITE_MASKS, nbits: int = 1,
+           variant: int = 0):
     L = lib()
     argv = [make_args(b, problems[b]) if problems[b] is not None else None for b in range(3)]
     aptr = (C.c_void_p * 3)(*[C.cast(C.byref(a), C.c_void_p) if a is not None else None for a in argv])
     masks = (C.c_uint64 * 3)(*site_masks)
     benches = np.zeros(count, dtype=np.int32)
     faults = (Fault * count)()
-    rc = L.ora_decode(bench_mode, aptr, masks, seed, nbits, first, count, _p(benches), C.cast(faults, C.c_void_p))
+    rc = L.ora_decode(bench_mode, aptr, masks, seed, nbits, variant, first, count, _p(benches), C.cast(faults, C.c_void_p))
     if rc != 0:
         raise RuntimeError("decode failed")
     return benches, [(f.site, f.thread, f.inst, f.mask) for f in faults]
@@ -317,3 +331,62 @@ def threads_out(bench: int, p, tids, exact: int = 0):
     qr = np.zeros(t.size, dtype=np.float32); qi = np.zeros(t.size, dtype=np.float32)
     assert L.ora_mriq_threads_out(C.byref(a), exact, _p(t), t.size, _p(qr), _p(qi)) == 0
     return qr, qi
+
+
+def detector_site(bench: int, site: int, unroll: int = 4) -> bool:
+    """True for sites that exist only because of HAUBERK (absent from the FI-only binary)."""
+    return bool(lib().ora_detector_site(bench, unroll, site))
+
+
+# ------------------------------------------------------------------------------------------------
+# A6 selection, recovery and evaluation arithmetic
+# ------------------------------------------------------------------------------------------------
+A6_VAR, A6_TEMP, A6_LOAD, A6_CONST, A6_NLPROT, A6_ACCOP, A6_IND = range(7)
+
+
+def _graph(kinds, edges):
+    k = np.ascontiguousarray(np.asarray(kinds, dtype=np.int32))
+    e = np.asarray(edges, dtype=np.int32).reshape(-1, 2)
+    return k, np.ascontiguousarray(e[:, 0]), np.ascontiguousarray(e[:, 1])
+
+
+def a6_count(kinds, edges, v: int, removed=None) -> int:
+    k, s, d = _graph(kinds, edges)
+    rm = None if removed is None else np.ascontiguousarray(np.asarray(removed, dtype=np.uint8))
+    return int(lib().ora_a6_count(k.size, _p(k), s.size, _p(s), _p(d), None if rm is None else _p(rm), v))
+
+
+def a6_select(kinds, selfacc, edges, maxvar: int):
+    k, s, d = _graph(kinds, edges)
+    sa = np.ascontiguousarray(np.asarray(selfacc, dtype=np.uint8))
+    out = np.zeros(max(maxvar, 1), dtype=np.int32)
+    got = lib().ora_a6_select(k.size, _p(k), _p(sa), s.size, _p(s), _p(d), maxvar, _p(out))
+    return out[:got].tolist()
+
+
+def in_range(R: Ranges, d: int, v: float) -> bool:
+    return bool(lib().ora_in_range(C.byref(R), d, v))
+
+
+def extend_ranges(rs: RSet, values) -> int:
+    v = np.ascontiguousarray(np.asarray(values, dtype=np.float32))
+    return int(lib().ora_extend_ranges(C.byref(rs), _p(v), v.size))
+
+
+def alpha_step(alpha: float, fp_ratio: float, hi: float = 0.10, lo: float = 0.05) -> float:
+    return float(lib().ora_alpha_step(alpha, fp_ratio, hi, lo))
+
+
+DIAG_NAMES = ["ok", "false_alarm", "transient", "persistent", "failed"]
+
+
+def diagnose(alarm1: int, fail1: int, alarm2: int, fail2: int, identical: bool) -> str:
+    return DIAG_NAMES[lib().ora_diagnose(alarm1, fail1, alarm2, fail2, 1 if identical else 0)]
+
+
+def coverage(counts) -> dict:
+    """{coverage, sdc, detected, failure} of int64 counts [.., 5] summed over benchmarks."""
+    c = np.ascontiguousarray(np.asarray(counts, dtype=np.int64).reshape(-1, 5).sum(0))
+    out = np.zeros(4)
+    lib().ora_coverage(_p(c), _p(out))
+    return dict(zip(("coverage", "sdc", "detected", "failure"), out.tolist()))

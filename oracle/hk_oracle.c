@@ -55,9 +55,10 @@ typedef struct {
   const float *x, *y, *z; int32_t n_vox; int32_t n_k;
   const float *kx, *ky, *kz, *phi_r, *phi_i;
 } ora_mriq_args;
-typedef struct { const float* pts; const float* edges; int32_t n, n_rand, n_bins, chunk; } ora_tpacf_args;
+typedef struct { const float* pts; const float* edges; int32_t n, n_rand, n_bins; } ora_tpacf_args;
 
-typedef struct { int32_t site; int32_t pad; int64_t thread, inst; uint64_t mask; } ora_fault;
+/* hang = R17 watchdog factor T of this injection (0 = the paper's 10, L1997-2001). */
+typedef struct { int32_t site; int32_t hang; int64_t thread, inst; uint64_t mask; } ora_fault;
 typedef struct {
   uint32_t alarm, fail, domain, margin;
   uint32_t n_alarm_threads, first_thread; int32_t applied; float gap;
@@ -160,7 +161,15 @@ typedef struct {
   int64_t inst;
   uint64_t mask;
   int applied;
+  int32_t hang;    /* R17 watchdog factor T ("T (i.e., 10) times") */
 } fctx;
+
+/* R17: a loop about to start iteration `it` >= T * max(golden trips, 1) is FAILURE(hang).  The
+ * limit comes from the fault-free trip count known to the harness (not from corruptible state). */
+static int64_t hang_limit(const fctx* F, int64_t golden) {
+  const int64_t T = (F && F->hang > 0) ? F->hang : 10;
+  return T * (golden > 1 ? golden : 1);
+}
 
 static int hit(fctx* F, int site, int64_t inst) {
   if (F && F->active && F->site == site && F->inst == inst) { F->applied = 1; return 1; }
@@ -226,6 +235,10 @@ static void tout_init(tout* o) { memset(o, 0, sizeof(*o)); o->margin = 0xfffffff
 /*   22..20+U dx_j (j=1..U-1); then r2_j (U), s_j (U), E_j (U, @acc), it (@acc)               */
 /* ------------------------------------------------------------------------------------------ */
 static int cp_nsites(int U) { return 22 + 4 * U; }
+/* Detector d's self-accumulator (A6 repeated Maxvar times, L1259-1273; pinned by ora_a6_select on
+ * the CP loop graph): E_{U-1} first (largest backward dependency: it chains every dx_j), then the
+ * remaining E_j tie at {r2_j, s_j} and go in program order E_0, E_1, ... (R12). */
+static int cp_sel(int U, int d) { return d == 0 ? U - 1 : d - 1; }
 
 static void cp_thread(const ora_cp_args* P, const float* A4, int64_t t, int flags, int exact,
                       const ora_ranges* R, int ndet, fctx* F, tout* o, float* samples, int64_t nthr) {
@@ -270,8 +283,7 @@ static void cp_thread(const ora_cp_args* P, const float* A4, int64_t t, int flag
   /* Loop (self-accumulators E_j need no accumulator; counter `it`). */
   float E[8] = {0};
   int32_t it = 0;
-  const int64_t golden = P->n_atoms;
-  const int64_t limit = 10 * (golden > 1 ? golden : 1);
+  const int64_t limit = hang_limit(F, P->n_atoms);
   int32_t atomid = 0;
   for (int64_t i = 0;; ++i) {
     atomid = fi32(F, 14, i, atomid);
@@ -309,7 +321,7 @@ static void cp_thread(const ora_cp_args* P, const float* A4, int64_t t, int flag
   if (L && it != numatoms) o->alarm |= AL_COUNT;
   if ((L || (flags & F_PROFILE)) && it != 0) {
     for (int d = 0; d < ndet; ++d) {
-      float v = E[U - 1 - d] / (float)it;
+      float v = E[cp_sel(U, d)] / (float)it;
       if (flags & F_PROFILE) samples[(int64_t)d * nthr + t] = v;
       if (L && R->det[d].n > 0 && !in_range(R, d, v, &o->margin, &o->gap)) o->alarm |= AL_RANGE;
     }
@@ -434,8 +446,7 @@ static void mriq_thread(const ora_mriq_args* P, const float* KV, int64_t t, int 
 
   float Qr = 0.0f, Qi = 0.0f;
   int32_t it = 0, k = 0;
-  const int64_t golden = P->n_k;
-  const int64_t limit = 10 * (golden > 1 ? golden : 1);
+  const int64_t limit = hang_limit(F, P->n_k);
   for (int64_t i = 0;; ++i) {
     k = fi32(F, 15, i, k);
     xIndex = fi32(F, 4, i, xIndex);
@@ -488,30 +499,28 @@ static void mriq_thread(const ora_mriq_args* P, const float* KV, int64_t t, int 
 static int mriq_valid(const ora_mriq_args* P) { return P->n_vox >= 0 && P->n_k >= 0; }
 
 /* ------------------------------------------------------------------------------------------ */
-/* TPACF (K3).  DESIGN.md §3.4.  Thread g = (h*nC + c)*N + i; partners j in chunk c.           */
+/* TPACF (K3).  DESIGN.md §3.4: one abstract thread g = h*N + i per (histogram */
+/* h, point i), looping over every partner j in [jb, N) in ascending order.  There is no chunk  */
+/* here: how a kernel tiles the partner loop is not part of the program.                       */
 /* Site catalogue:                                                                             */
-/*   0 i 1 h 2 c 3 aoff 4 boff 5 jb 6 je 7 expect 8 base 9 x1 10 y1 11 z1      (NL @def)       */
-/*   12 boff 13 je 14 expect 15 base 16 x1 17 y1 18 z1                          (NL @live)      */
-/*   19 n 20 pts* 21 hist*                                                      (param @live)   */
-/*   22 j 23 x2 24 y2 25 z2 26 dot 27 bin 28 hidx 29 acc 30 cnt                 (loop)          */
+/*   0 i 1 h 2 aoff 3 boff 4 jb 5 je 6 expect 7 base 8 x1 9 y1 10 z1          (NL @def)        */
+/*   11 boff 12 je 13 expect 14 base 15 x1 16 y1 17 z1                        (NL @live)       */
+/*   18 n 19 pts* 20 hist*                                                   (param @live)    */
+/*   21 j 22 x2 23 y2 24 z2 25 dot 26 bin 27 hidx 28 acc 29 cnt               (loop)           */
 /* ------------------------------------------------------------------------------------------ */
-#define TPACF_NSITES 31
+#define TPACF_NSITES 30
 static int tp_nh(const ora_tpacf_args* P) { return 1 + 2 * P->n_rand; }
-static int tp_nc(const ora_tpacf_args* P) { return (P->n + P->chunk - 1) / P->chunk; }
-static int64_t tp_threads(const ora_tpacf_args* P) { return (int64_t)tp_nh(P) * tp_nc(P) * P->n; }
+static int64_t tp_threads(const ora_tpacf_args* P) { return (int64_t)tp_nh(P) * P->n; }
 static int tp_valid(const ora_tpacf_args* P) {
-  if (P->n < 0 || P->n_rand < 1 || P->n_bins < 1 || P->n_bins > 30 || P->chunk < 1) return 0;
+  if (P->n < 0 || P->n_rand < 1 || P->n_bins < 1 || P->n_bins > 30) return 0;
   for (int e = 0; e < P->n_bins; ++e) if (!(P->edges[e] > P->edges[e + 1])) return 0;
   return 1;
 }
-/* Golden trip count of thread g (computed from uncorrupted indices; R17 watchdog, decode). */
+/* Golden trip count of thread g (computed from uncorrupted indices; R17 watchdog, decode):
+ * N - (i + 1) for the self-correlation rows h <= n_rand (DD, RR_s), N for the DR rows. */
 static int64_t tp_trips(const ora_tpacf_args* P, int64_t g) {
-  int nC = tp_nc(P), N = P->n, C = P->chunk, nr = P->n_rand;
-  int64_t row = g / N; int i = (int)(g % N);
-  int h = (int)(row / nC), c = (int)(row % nC);
-  int64_t jb = (int64_t)c * C; if (h <= nr && i + 1 > jb) jb = i + 1;
-  int64_t je = (int64_t)(c + 1) * C; if (je > N) je = N;
-  return je > jb ? je - jb : 0;
+  int64_t h = g / P->n, i = g % P->n;
+  return h <= P->n_rand ? (int64_t)P->n - (i + 1) : (int64_t)P->n;
 }
 /* bin = #{e in [0, n_bins] : dot < edge[e]}  (the definition) */
 static int32_t tp_bin(const ora_tpacf_args* P, float dot) {
@@ -523,9 +532,9 @@ static int32_t tp_bin(const ora_tpacf_args* P, float dot) {
 static void tpacf_thread(const ora_tpacf_args* P, int64_t g, int flags, const ora_ranges* R, int ndet,
                          fctx* F, tout* o, int64_t* hist, float* samples, int64_t nthr) {
   const int NL = flags & F_NL, L = flags & F_L, FI = flags & F_FI;
-  const int nC = tp_nc(P), C = P->chunk, nr = P->n_rand, nb2 = P->n_bins + 2;
+  const int nr = P->n_rand, nb2 = P->n_bins + 2;
   const int64_t npts = 3LL * (1 + nr) * P->n, nhist = (int64_t)tp_nh(P) * nb2;
-  const int32_t row = (int32_t)(g / P->n), ii = (int32_t)(g % P->n);
+  const int32_t hh = (int32_t)(g / P->n), ii = (int32_t)(g % P->n);
   uint32_t chk = 0;
   int32_t n = P->n;
   uint64_t ppts = VBASE, phist = VBASE;
@@ -534,40 +543,38 @@ static void tpacf_thread(const ora_tpacf_args* P, int64_t g, int flags, const or
 #define NLDEF(var, site, expr)                                              \
   var = fi32(F, site, 0, (expr));                                           \
   if (NL) { chk ^= (uint32_t)var; if ((expr) != var) o->alarm |= AL_DUP; }
-  int32_t i, h, c, aoff, boff, jb, je, expect, base;
+  int32_t i, h, aoff, boff, jb, je, expect, base;
   NLDEF(i, 0, ii);
-  NLDEF(h, 1, row / nC);
-  NLDEF(c, 2, sub32(row, mul32(h, nC)));
-  NLDEF(aoff, 3, add32(mul32(h <= nr ? h : 0, n), i));
-  NLDEF(boff, 4, mul32(h == 0 ? 0 : (h <= nr ? h : sub32(h, nr)), n));
-  NLDEF(jb, 5, (h <= nr ? (add32(i, 1) > mul32(c, C) ? add32(i, 1) : mul32(c, C)) : mul32(c, C)));
-  NLDEF(je, 6, (mul32(add32(c, 1), C) < n ? mul32(add32(c, 1), C) : n));
-  NLDEF(expect, 7, (sub32(je, jb) > 0 ? sub32(je, jb) : 0));
-  NLDEF(base, 8, mul32(h, nb2));
+  NLDEF(h, 1, hh);
+  NLDEF(aoff, 2, add32(mul32(h <= nr ? h : 0, n), i));
+  NLDEF(boff, 3, mul32(h == 0 ? 0 : (h <= nr ? h : sub32(h, nr)), n));
+  NLDEF(jb, 4, (h <= nr ? add32(i, 1) : 0));
+  NLDEF(je, 5, n);
+  NLDEF(expect, 6, (sub32(je, jb) > 0 ? sub32(je, jb) : 0));
+  NLDEF(base, 7, mul32(h, nb2));
 #undef NLDEF
   int64_t e;
   float x1, y1, z1;
   if (FI && !access_ok(ppts, add32(mul32(3, aoff), 0), 4, npts, &e)) { o->fail |= FL_CRASH; return; } else if (!FI) e = 3LL * aoff + 0;
-  x1 = ff32(F, 9, 0, P->pts[e]);
+  x1 = ff32(F, 8, 0, P->pts[e]);
   if (NL) { chk ^= fb(x1); if (fb(P->pts[e]) != fb(x1)) o->alarm |= AL_DUP; }
   if (FI && !access_ok(ppts, add32(mul32(3, aoff), 1), 4, npts, &e)) { o->fail |= FL_CRASH; return; } else if (!FI) e = 3LL * aoff + 1;
-  y1 = ff32(F, 10, 0, P->pts[e]);
+  y1 = ff32(F, 9, 0, P->pts[e]);
   if (NL) { chk ^= fb(y1); if (fb(P->pts[e]) != fb(y1)) o->alarm |= AL_DUP; }
   if (FI && !access_ok(ppts, add32(mul32(3, aoff), 2), 4, npts, &e)) { o->fail |= FL_CRASH; return; } else if (!FI) e = 3LL * aoff + 2;
-  z1 = ff32(F, 11, 0, P->pts[e]);
+  z1 = ff32(F, 10, 0, P->pts[e]);
   if (NL) { chk ^= fb(z1); if (fb(P->pts[e]) != fb(z1)) o->alarm |= AL_DUP; }
   /* (iv) for variables whose last use precedes the loop */
-  if (NL) { chk ^= (uint32_t)i; chk ^= (uint32_t)h; chk ^= (uint32_t)c; chk ^= (uint32_t)aoff; chk ^= (uint32_t)jb; }
+  if (NL) { chk ^= (uint32_t)i; chk ^= (uint32_t)h; chk ^= (uint32_t)aoff; chk ^= (uint32_t)jb; }
 
   int32_t acc = 0, cnt = 0, j = jb;
-  const int64_t golden = tp_trips(P, g);
-  const int64_t limit = 10 * (golden > 1 ? golden : 1);
+  const int64_t limit = hang_limit(F, tp_trips(P, g));
   for (int64_t it = 0;; ++it) {
-    j = fi32(F, 22, it, j);
-    boff = fi32(F, 12, it, boff); je = fi32(F, 13, it, je); expect = fi32(F, 14, it, expect);
-    base = fi32(F, 15, it, base);
-    x1 = ff32(F, 16, it, x1); y1 = ff32(F, 17, it, y1); z1 = ff32(F, 18, it, z1);
-    n = fi32(F, 19, it, n); ppts = fp64(F, 20, it, ppts); phist = fp64(F, 21, it, phist);
+    j = fi32(F, 21, it, j);
+    boff = fi32(F, 11, it, boff); je = fi32(F, 12, it, je); expect = fi32(F, 13, it, expect);
+    base = fi32(F, 14, it, base);
+    x1 = ff32(F, 15, it, x1); y1 = ff32(F, 16, it, y1); z1 = ff32(F, 17, it, z1);
+    n = fi32(F, 18, it, n); ppts = fp64(F, 19, it, ppts); phist = fp64(F, 20, it, phist);
     if (!(j < je)) break;
     if (FI && it >= limit) { o->fail |= FL_HANG; return; }
     int32_t pb = mul32(3, add32(boff, j));
@@ -575,16 +582,16 @@ static void tpacf_thread(const ora_tpacf_args* P, int64_t g, int flags, const or
     for (int a = 0; a < 3; ++a) {
       if (FI) { if (!access_ok(ppts, add32(pb, a), 4, npts, &e)) { o->fail |= FL_CRASH; return; } }
       else e = (int64_t)pb + a;
-      q[a] = ff32(F, 23 + a, it, P->pts[e]);
+      q[a] = ff32(F, 22 + a, it, P->pts[e]);
     }
-    float dot = ff32(F, 26, it, fmaf(z1, q[2], fmaf(y1, q[1], x1 * q[0])));
-    int32_t bin = fi32(F, 27, it, tp_bin(P, dot));
-    int32_t hidx = fi32(F, 28, it, add32(base, bin));
+    float dot = ff32(F, 25, it, fmaf(z1, q[2], fmaf(y1, q[1], x1 * q[0])));
+    int32_t bin = fi32(F, 26, it, tp_bin(P, dot));
+    int32_t hidx = fi32(F, 27, it, add32(base, bin));
     if (FI) { if (!access_ok(phist, hidx, 8, nhist, &e)) { o->fail |= FL_CRASH; return; } }
     else e = hidx;
     hist[e] += 1;
-    acc = fi32(F, 29, it, add32(acc, bin));
-    cnt = fi32(F, 30, it, add32(cnt, 1));
+    acc = fi32(F, 28, it, add32(acc, bin));
+    cnt = fi32(F, 29, it, add32(cnt, 1));
     j = add32(j, 1);
   }
   if (L && cnt != expect) o->alarm |= AL_COUNT;
@@ -618,8 +625,9 @@ static void info_init(ora_runinfo* I) {
 }
 
 static fctx mkfctx(const ora_fault* f, int64_t t) {
-  fctx F = {0, -1, 0, 0, 0};
+  fctx F = {0, -1, 0, 0, 0, 10};
   if (f && f->site >= 0 && f->thread == t) { F.active = 1; F.site = f->site; F.inst = f->inst; F.mask = f->mask; }
+  if (f && f->hang > 0) F.hang = f->hang;
   return F;
 }
 
@@ -889,10 +897,20 @@ ORA_EXPORT void ora_site_info(int32_t bench, int32_t unroll, int32_t site, int32
     if (site <= 3 || site >= MRIQ_PHIMAG_SITE0) *cls = SC_NL;
     if (site >= 9 && site <= 14) *width = 64;
   } else {
-    if (site <= 11) *cls = SC_NL;
-    if (site == 20 || site == 21) *width = 64;
+    if (site <= 10) *cls = SC_NL;
+    if (site == 19 || site == 20) *width = 64;
   }
   (void)unroll;
+}
+
+/* Sites that exist only because of HAUBERK (the loop detector's counter / accumulator and the
+ * expected trip count): absent from the original program, so the FI-only binary (row a7,
+ * "binary with HAUBERK FI ... error sensitivity of baseline program") has none.
+ * CP: it (last site); MRI-Q: it (28); TPACF: expect @def (6), expect @live (13), acc (28), cnt (29). */
+ORA_EXPORT int32_t ora_detector_site(int32_t bench, int32_t unroll, int32_t site) {
+  if (bench == B_CP) return site == cp_nsites(unroll) - 1;
+  if (bench == B_MRIQ) return site == 28;
+  return site == 6 || site == 13 || site == 28 || site == 29;
 }
 
 typedef struct {
@@ -909,7 +927,8 @@ static int64_t cat_nl_threads(const catalog* K, int s) {
   return K->nthr;
 }
 
-static void cat_build(catalog* K, int bench, const void* args, uint64_t site_mask) {
+/* variant 0 = FI&FT catalogue; 1 = FI-only (the original program's sites only). */
+static void cat_build(catalog* K, int bench, const void* args, uint64_t site_mask, int variant) {
   memset(K, 0, sizeof(*K));
   K->bench = bench;
   int U = 1;
@@ -925,6 +944,7 @@ static void cat_build(catalog* K, int bench, const void* args, uint64_t site_mas
   K->nsites = ora_nsites(bench, U);
   for (int s = 0; s < K->nsites; ++s) {
     if (!((site_mask >> s) & 1)) continue;
+    if (variant == 1 && ora_detector_site(bench, U, s)) continue;
     int32_t cls, w; ora_site_info(bench, U, s, &cls, &w);
     int64_t D = cls == SC_NL ? cat_nl_threads(K, s) : K->total_trips;
     if (D > 0) K->en[K->nen++] = s;
@@ -944,7 +964,7 @@ static void cat_decode(const catalog* K, uint64_t seed, int64_t n, int nbits, or
   int s = K->en[ora_bounded(r1, (uint64_t)K->nen)];
   int U = K->cp ? K->cp->unroll : 1;
   int32_t cls, w; ora_site_info(K->bench, U, s, &cls, &w);
-  f->site = s; f->pad = 0;
+  f->site = s; f->hang = 0;
   if (cls == SC_NL) {
     f->thread = (int64_t)ora_bounded(r2, (uint64_t)cat_nl_threads(K, s));
     f->inst = 0;
@@ -974,12 +994,13 @@ static void cat_decode(const catalog* K, uint64_t seed, int64_t n, int nbits, or
 
 /* Public decode: bench_mode >= 0 fixes the benchmark, -1 = mixed (bench = n mod 3). */
 ORA_EXPORT int ora_decode(int32_t bench_mode, const void* const args[3], const uint64_t site_mask[3],
-                          uint64_t seed, int32_t nbits, int64_t first, int64_t count, int32_t* bench_out, ora_fault* out) {
+                          uint64_t seed, int32_t nbits, int32_t variant, int64_t first, int64_t count,
+                          int32_t* bench_out, ora_fault* out) {
   catalog K[3]; int have[3] = {0, 0, 0};
   for (int64_t q = 0; q < count; ++q) {
     int64_t n = first + q;
     int b = bench_mode >= 0 ? bench_mode : (int)(n % 3);
-    if (!have[b]) { cat_build(&K[b], b, args[b], site_mask[b]); have[b] = 1; if (K[b].nen == 0) return 1; }
+    if (!have[b]) { cat_build(&K[b], b, args[b], site_mask[b], variant); have[b] = 1; if (K[b].nen == 0) return 1; }
     bench_out[q] = b;
     cat_decode(&K[b], seed, n, nbits, &out[q]);
   }
@@ -998,35 +1019,35 @@ typedef struct {
   float* A4; float* KV;
 } goldens;
 
-static int golden_build(int b, const void* args, int exact, const ora_ranges* R, goldens* G) {
+static int golden_build(int b, const void* args, int exact, int vf, const ora_ranges* R, goldens* G) {
   memset(G, 0, sizeof(*G));
   ora_runinfo I;
   if (b == B_CP) {
     const ora_cp_args* P = (const ora_cp_args*)args;
     G->g0 = (float*)malloc(sizeof(float) * (size_t)P->nx * P->ny);
-    if (ora_cp_run(P, F_NL | F_L, exact, R, R->n_det, NULL, G->g0, NULL, &I)) return 1;
+    if (ora_cp_run(P, vf, exact, R, R->n_det, NULL, G->g0, NULL, &I)) return 1;
     G->M = ora_max_abs(G->g0, (int64_t)P->nx * P->ny);
     G->A4 = cp_prepass(P);
   } else if (b == B_MRIQ) {
     const ora_mriq_args* P = (const ora_mriq_args*)args;
     G->g0 = (float*)malloc(sizeof(float) * (size_t)(P->n_vox > 0 ? P->n_vox : 1) * 2);
     G->g1 = G->g0 + P->n_vox;
-    if (ora_mriq_run(P, F_NL | F_L, exact, R, R->n_det, NULL, G->g0, G->g1, NULL, &I)) return 1;
+    if (ora_mriq_run(P, vf, exact, R, R->n_det, NULL, G->g0, G->g1, NULL, &I)) return 1;
     G->M = ora_max_abs(G->g0, 2LL * P->n_vox); /* R6: max over [Qr; Qi] */
     G->KV = mriq_phimag(P);
   } else {
     const ora_tpacf_args* P = (const ora_tpacf_args*)args;
     G->gh = (int64_t*)malloc(sizeof(int64_t) * (size_t)tp_nh(P) * (P->n_bins + 2));
-    if (ora_tpacf_run(P, F_NL | F_L, R, R->n_det, NULL, G->gh, NULL, &I)) return 1;
+    if (ora_tpacf_run(P, vf, R, R->n_det, NULL, G->gh, NULL, &I)) return 1;
   }
   return I.alarm != 0 ? 2 : 0; /* fault-free run must not alarm (train = test, L2402-2403) */
 }
 static void golden_free(goldens* G) { free(G->g0); free(G->gh); free(G->A4); free(G->KV); }
 
 /* Replay one injection; fills the record's wrong/alarm/fail/domain/margin/worst. */
-static void replay_one(int b, const void* args, int exact, const ora_ranges* R, const goldens* G,
+static void replay_one(int b, const void* args, int exact, int vf, const ora_ranges* R, const goldens* G,
                        const ora_fault* f, ora_record* rec, int32_t* wrong_out) {
-  fctx F = {1, f->site, f->inst, f->mask, 0};
+  fctx F = {1, f->site, f->inst, f->mask, 0, f->hang > 0 ? f->hang : 10};
   tout o; tout_init(&o);
   int wrong = 0; float worst = 0.0f;
   if (b == B_CP || b == B_MRIQ) {
@@ -1035,15 +1056,15 @@ static void replay_one(int b, const void* args, int exact, const ora_ranges* R, 
     if (b == B_CP) {
       const ora_cp_args* P = (const ora_cp_args*)args;
       tout g; tout_init(&g);
-      cp_thread(P, G->A4, f->thread, F_NL | F_L, exact, R, R->n_det, NULL, &g, NULL, 0);
+      cp_thread(P, G->A4, f->thread, vf, exact, R, R->n_det, NULL, &g, NULL, 0);
       for (int w = 0; w < g.nw; ++w) { own_idx[nown] = g.widx[w]; own_buf[nown] = 0; nown++; }
-      cp_thread(P, G->A4, f->thread, F_NL | F_L | F_FI, exact, R, R->n_det, &F, &o, NULL, 0);
+      cp_thread(P, G->A4, f->thread, vf | F_FI, exact, R, R->n_det, &F, &o, NULL, 0);
     } else {
       const ora_mriq_args* P = (const ora_mriq_args*)args;
       tout g; tout_init(&g);
-      mriq_thread(P, G->KV, f->thread, F_NL | F_L, exact, R, R->n_det, NULL, &g, NULL, 0);
+      mriq_thread(P, G->KV, f->thread, vf, exact, R, R->n_det, NULL, &g, NULL, 0);
       for (int w = 0; w < g.nw; ++w) { own_idx[nown] = g.widx[w]; own_buf[nown] = g.wbuf[w]; nown++; }
-      mriq_thread(P, G->KV, f->thread, F_NL | F_L | F_FI, exact, R, R->n_det, &F, &o, NULL, 0);
+      mriq_thread(P, G->KV, f->thread, vf | F_FI, exact, R, R->n_det, &F, &o, NULL, 0);
     }
     if (!o.fail) {
       /* touched = own ∪ written; new value = (own ? 0 : golden) + sum of faulted writes */
@@ -1072,9 +1093,9 @@ static void replay_one(int b, const void* args, int exact, const ora_ranges* R, 
     memcpy(hist, G->gh, sizeof(int64_t) * nh);
     int64_t* d = (int64_t*)calloc(nh, sizeof(int64_t));
     tout g; tout_init(&g);
-    tpacf_thread(P, f->thread, F_NL | F_L, R, R->n_det, NULL, &g, d, NULL, 0);
+    tpacf_thread(P, f->thread, vf, R, R->n_det, NULL, &g, d, NULL, 0);
     for (size_t e = 0; e < nh; ++e) { hist[e] -= d[e]; d[e] = 0; }
-    tpacf_thread(P, f->thread, F_NL | F_L | F_FI, R, R->n_det, &F, &o, d, NULL, 0);
+    tpacf_thread(P, f->thread, vf | F_FI, R, R->n_det, &F, &o, d, NULL, 0);
     for (size_t e = 0; e < nh; ++e) hist[e] += d[e];
     if (!o.fail) wrong = ora_tpacf_wrong(hist, G->gh, P->n_rand, P->n_bins, &worst);
     free(hist); free(d);
@@ -1084,26 +1105,26 @@ static void replay_one(int b, const void* args, int exact, const ora_ranges* R, 
   *wrong_out = wrong;
 }
 
-static void replica_one(int b, const void* args, int exact, const ora_ranges* R, const goldens* G,
+static void replica_one(int b, const void* args, int exact, int vf, const ora_ranges* R, const goldens* G,
                         const ora_fault* f, ora_record* rec, int32_t* wrong_out) {
   ora_runinfo I; int wrong = 0; float worst = 0.0f;
   if (b == B_CP) {
     const ora_cp_args* P = (const ora_cp_args*)args;
     int64_t n = (int64_t)P->nx * P->ny;
     float* out = (float*)malloc(sizeof(float) * (size_t)n);
-    ora_cp_run(P, F_NL | F_L, exact, R, R->n_det, f, out, NULL, &I);
+    ora_cp_run(P, vf, exact, R, R->n_det, f, out, NULL, &I);
     if (!I.fail) wrong = ora_fp_wrong(out, G->g0, n, G->M, &worst);
     free(out);
   } else if (b == B_MRIQ) {
     const ora_mriq_args* P = (const ora_mriq_args*)args;
     float* out = (float*)malloc(sizeof(float) * 2 * (size_t)(P->n_vox > 0 ? P->n_vox : 1));
-    ora_mriq_run(P, F_NL | F_L, exact, R, R->n_det, f, out, out + P->n_vox, NULL, &I);
+    ora_mriq_run(P, vf, exact, R, R->n_det, f, out, out + P->n_vox, NULL, &I);
     if (!I.fail) wrong = ora_fp_wrong(out, G->g0, 2LL * P->n_vox, G->M, &worst);
     free(out);
   } else {
     const ora_tpacf_args* P = (const ora_tpacf_args*)args;
     int64_t* hist = (int64_t*)malloc(sizeof(int64_t) * (size_t)tp_nh(P) * (P->n_bins + 2));
-    ora_tpacf_run(P, F_NL | F_L, R, R->n_det, f, hist, NULL, &I);
+    ora_tpacf_run(P, vf, R, R->n_det, f, hist, NULL, &I);
     if (!I.fail) wrong = ora_tpacf_wrong(hist, G->gh, P->n_rand, P->n_bins, &worst);
     free(hist);
   }
@@ -1113,27 +1134,33 @@ static void replica_one(int b, const void* args, int exact, const ora_ranges* R,
 }
 
 /* counts[b*5 + cls] += 1 for each injection; records (nullable) get one entry per injection. */
+/* variant 0 = FI&FT binary (HAUBERK-NL + HAUBERK-L); 1 = FI-only binary (the original program with
+ * the injector: its catalogue holds the original program's sites only, its
+ * outcomes are masked / undetected (SDC) / failure).  hang_factor = R17's T (0 -> 10). */
 ORA_EXPORT int ora_campaign(int32_t bench_mode, const void* const args[3], const ora_ranges* const ranges[3],
                             const uint64_t site_mask[3], uint64_t seed, int32_t nbits, int64_t first, int64_t count,
-                            int32_t exact, int32_t mode, ora_record* records, int64_t* counts) {
+                            int32_t exact, int32_t mode, int32_t variant, int32_t hang_factor,
+                            ora_record* records, int64_t* counts) {
   catalog K[3]; goldens G[3]; int have[3] = {0, 0, 0};
+  const int vf = variant == 1 ? 0 : (F_NL | F_L);
   int rc = 0;
   for (int64_t q = 0; q < count && rc == 0; ++q) {
     int64_t n = first + q;
     int b = bench_mode >= 0 ? bench_mode : (int)(n % 3);
     if (!have[b]) {
       have[b] = 1;
-      cat_build(&K[b], b, args[b], site_mask[b]);
+      cat_build(&K[b], b, args[b], site_mask[b], variant);
       if (K[b].nen == 0) { rc = 1; break; }
-      rc = golden_build(b, args[b], exact, ranges[b], &G[b]);
+      rc = golden_build(b, args[b], exact, vf, ranges[b], &G[b]);
       if (rc) break;
     }
     ora_fault f; cat_decode(&K[b], seed, n, nbits, &f);
+    f.hang = hang_factor;
     ora_record rec; memset(&rec, 0, sizeof(rec));
     int32_t wrong = 0;
     /* replay cannot express a PhiMag fault (it reaches every voxel, R22): run that one as a replica */
-    if (mode == 1 && !(b == B_MRIQ && f.site >= MRIQ_PHIMAG_SITE0)) replay_one(b, args[b], exact, ranges[b], &G[b], &f, &rec, &wrong);
-    else replica_one(b, args[b], exact, ranges[b], &G[b], &f, &rec, &wrong);
+    if (mode == 1 && !(b == B_MRIQ && f.site >= MRIQ_PHIMAG_SITE0)) replay_one(b, args[b], exact, vf, ranges[b], &G[b], &f, &rec, &wrong);
+    else replica_one(b, args[b], exact, vf, ranges[b], &G[b], &f, &rec, &wrong);
     rec.index = n; rec.bench = b; rec.site = f.site; rec.thread = f.thread; rec.inst = f.inst; rec.mask = f.mask;
     rec.cls = ora_classify(wrong, rec.alarm, rec.fail);
     if (records) records[q] = rec;
@@ -1143,4 +1170,143 @@ ORA_EXPORT int ora_campaign(int32_t bench_mode, const void* const args[3], const
   return rc;
 }
 
-ORA_EXPORT int ora_version(void) { return 1; }
+/* ------------------------------------------------------------------------------------------ */
+/* A6: loop-detector target selection (PAPER L1221-1273 [§V.B step i], Fig. 9).     */
+/* The loop's dataflow graph: node kinds A6_VAR (virtual variable defined in the loop), A6_TEMP  */
+/* (temporary of a multi-operation statement, L1246-1250), A6_LOAD (memory-load data, counted:   */
+/* "including the memory load data", L1253-1254), A6_CONST (not counted: "but not the          */
+/* constant"), A6_NLPROT (loop invariants protected by non-loop detectors, excluded L1254-1257),  */
+/* A6_ACCOP (the operation of a self-accumulator's own update statement, `E += w * t`: part of   */
+/* the target's definition, not of its backward set — the reading under which Fig. 9 gives 12   */
+/* and 13, DESIGN R12), A6_IND (the loop's induction variable: protected by the iteration       */
+/* counter, L1293-1300, so neither counted nor a candidate).  Edge k: src[k] is used to compute  */
+/* dst[k] (a load's address is not data); self-edges (E = E + ...) are ignored.                 */
+/* ------------------------------------------------------------------------------------------ */
+enum { A6_VAR = 0, A6_TEMP = 1, A6_LOAD = 2, A6_CONST = 3, A6_NLPROT = 4, A6_ACCOP = 5, A6_IND = 6 };
+
+static void a6_ancestors(int32_t n, int32_t ne, const int32_t* src, const int32_t* dst, int32_t v, uint8_t* mark) {
+  /* plain iterative closure: mark every u with a path u ->* v (v itself not marked) */
+  memset(mark, 0, (size_t)n);
+  int changed = 1;
+  while (changed) {
+    changed = 0;
+    for (int32_t k = 0; k < ne; ++k) {
+      if (src[k] == dst[k]) continue;
+      if ((dst[k] == v || mark[dst[k]]) && !mark[src[k]] && src[k] != v) { mark[src[k]] = 1; changed = 1; }
+    }
+  }
+}
+
+/* Cumulative backward dataflow dependency of v over the nodes not yet `removed` (nullable). */
+ORA_EXPORT int32_t ora_a6_count(int32_t n, const int32_t* kind, int32_t ne, const int32_t* src, const int32_t* dst,
+                                const uint8_t* removed, int32_t v) {
+  uint8_t* mark = (uint8_t*)malloc((size_t)(n > 0 ? n : 1));
+  a6_ancestors(n, ne, src, dst, v, mark);
+  int32_t c = 0;
+  for (int32_t u = 0; u < n; ++u)
+    if (mark[u] && !(removed && removed[u]) && (kind[u] == A6_VAR || kind[u] == A6_TEMP || kind[u] == A6_LOAD)) c++;
+  free(mark);
+  return c;
+}
+
+/* Selection repeated Maxvar times (L1259-1273): candidates are the loop's virtual variables not
+ * yet removed, self-accumulators first (they need no accumulator code, L1223-1225); the one with
+ * the largest cumulative backward dependency wins, ties to the earlier node (program order, R12);
+ * the winner and every node with forward dependency to it are then removed.  Returns the number
+ * selected; order[0..] = the chosen node ids. */
+ORA_EXPORT int32_t ora_a6_select(int32_t n, const int32_t* kind, const uint8_t* selfacc, int32_t ne, const int32_t* src,
+                                 const int32_t* dst, int32_t maxvar, int32_t* order) {
+  uint8_t* removed = (uint8_t*)calloc((size_t)(n > 0 ? n : 1), 1);
+  uint8_t* mark = (uint8_t*)malloc((size_t)(n > 0 ? n : 1));
+  int32_t got = 0;
+  for (; got < maxvar; ++got) {
+    int any_self = 0;
+    for (int32_t u = 0; u < n; ++u) if (kind[u] == A6_VAR && !removed[u] && selfacc[u]) any_self = 1;
+    int32_t best = -1, bc = -1;
+    for (int32_t u = 0; u < n; ++u) {
+      if (kind[u] != A6_VAR || removed[u] || (any_self && !selfacc[u])) continue;
+      int32_t c = ora_a6_count(n, kind, ne, src, dst, removed, u);
+      if (c > bc) { bc = c; best = u; }
+    }
+    if (best < 0) break;
+    order[got] = best;
+    a6_ancestors(n, ne, src, dst, best, mark);
+    removed[best] = 1;
+    for (int32_t u = 0; u < n; ++u) if (mark[u]) removed[u] = 1;
+  }
+  free(removed); free(mark);
+  return got;
+}
+
+/* ------------------------------------------------------------------------------------------ */
+/* Recovery and evaluation arithmetic (PAPER §VI, §VIII).                */
+/* ------------------------------------------------------------------------------------------ */
+/* R10/R11 range check of a single value against detector d (alpha applied to the bounds). */
+ORA_EXPORT int32_t ora_in_range(const ora_ranges* R, int32_t d, float v) {
+  uint32_t m = 0xffffffffu; float g = INFINITY;
+  return in_range(R, d, v, &m, &g);
+}
+
+/* A11 (L1309-1313: "calculates new ranges that include the outlier"; DESIGN R24): each value joins
+ * the range of its correlation class at the detector's threshold T = 10^t_exp10 (neg: v < -T,
+ * zero: -T <= v <= T, pos: v > T); a class without a range gains one.  Ranges stay in class order.
+ * Non-finite values are ignored (they cannot be represented by a range).  Returns ranges added. */
+ORA_EXPORT int32_t ora_extend_ranges(ora_rset* s, const float* values, int32_t nv) {
+  const float T = pow10f_table(s->t_exp10);
+  float lo[3], hi[3]; int have[3] = {0, 0, 0};
+  for (int r = 0; r < s->n; ++r) {
+    float x = s->lo[r];
+    int c = (x < -T) ? 0 : (x > T ? 2 : 1);
+    lo[c] = s->lo[r]; hi[c] = s->hi[r]; have[c] = 1;
+  }
+  int before = s->n, added = 0;
+  for (int32_t k = 0; k < nv; ++k) {
+    float x = values[k];
+    if (!isfinite(x)) continue;
+    int c = (x < -T) ? 0 : (x > T ? 2 : 1);
+    if (!have[c]) { lo[c] = hi[c] = x; have[c] = 1; added++; }
+    else { if (x < lo[c]) lo[c] = x; if (x > hi[c]) hi[c] = x; }
+  }
+  int r = 0;
+  for (int c = 0; c < 3; ++c) if (have[c]) { s->lo[r] = lo[c]; s->hi[r] = hi[c]; r++; }
+  s->n = r;
+  (void)before;
+  return added;
+}
+
+/* alpha controller (L2066-2077): false-positive ratio above `hi` (10 %) -> alpha x 10; below `lo`
+ * (5 %) -> alpha / 10 while alpha stays >= 1 (i.e. only from alpha >= 10). */
+ORA_EXPORT float ora_alpha_step(float alpha, double fp_ratio, double hi, double lo) {
+  if (fp_ratio > hi) return alpha * 10.0f;
+  if (fp_ratio < lo && alpha >= 10.0f) return alpha / 10.0f;
+  return alpha;
+}
+
+/* Re-execution diagnosis (Fig. 11).  0 ok (no alarm), 1 false alarm (re-run alarms
+ * again with a bitwise-identical output), 2 transient (re-run ends normally without an alarm: its
+ * output is taken), 3 persistent (re-run alarms with a different output: BIST / migration), 4 failure
+ * (either run crashed or hung: the guardian's path, L1982-2007). */
+ORA_EXPORT int32_t ora_diagnose(uint32_t alarm1, uint32_t fail1, uint32_t alarm2, uint32_t fail2, int32_t identical) {
+  if (fail1) return 4;
+  if (!alarm1) return 0;
+  if (fail2) return 4;
+  if (!alarm2) return 2;
+  return identical ? 1 : 3;
+}
+
+/* Campaign summary (R2, L2372-2375 and L2480-2483: coverage = P(detected or masked), failures
+ * covered): out[0] coverage = 1 - undetected/total; out[1] SDC ratio = undetected/total (for an
+ * FI-only campaign: the unprotected SDC rate, L211-213); out[2] detected (classes 1+2)/total;
+ * out[3] failure/total.  counts: int64 [5] (one benchmark) — sum rows first for several. */
+ORA_EXPORT int32_t ora_coverage(const int64_t* counts5, double* out4) {
+  int64_t tot = 0;
+  for (int c = 0; c < 5; ++c) tot += counts5[c];
+  if (tot == 0) { for (int k = 0; k < 4; ++k) out4[k] = NAN; return 1; }
+  out4[0] = 1.0 - (double)counts5[C_UNDETECTED] / (double)tot;
+  out4[1] = (double)counts5[C_UNDETECTED] / (double)tot;
+  out4[2] = (double)(counts5[C_DET_MASKED] + counts5[C_DETECTED]) / (double)tot;
+  out4[3] = (double)counts5[C_FAILURE] / (double)tot;
+  return 0;
+}
+
+ORA_EXPORT int ora_version(void) { return 2; }

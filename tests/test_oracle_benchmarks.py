@@ -172,7 +172,7 @@ def _tpacf_bruteforce(p):
 
 @pytest.mark.parametrize("seed", [8, 1, 5, 13])
 def test_tpacf_bruteforce_acos_binning_and_totals(seed):
-    p = W.tpacf_problem(64, 2, seed=seed, clumps=4, sigma_deg=3.0, chunk=16)
+    p = W.tpacf_problem(64, 2, seed=seed, clumps=4, sigma_deg=3.0)
     h, _, info = O.run(O.TPACF, p)
     ref, near = _tpacf_bruteforce(p)
     # bin 0 (< 1 arcmin) is rounding-dominated in fp32 (edge[0] = 1 - 2^-24); compare bins >= 1.
@@ -186,15 +186,20 @@ def test_tpacf_bruteforce_acos_binning_and_totals(seed):
     assert info.alarm == 0
 
 
-@pytest.mark.parametrize("chunk", [1, 7, 64, 1000])
-def test_tpacf_chunking_does_not_change_histograms(chunk):
-    p = W.tpacf_small(n=90, n_rand=1, chunk=chunk)
-    q = W.tpacf_small(n=90, n_rand=1, chunk=90)
-    assert np.array_equal(O.run(O.TPACF, p)[0], O.run(O.TPACF, q)[0])
+def test_tpacf_abstract_threads_and_trip_counts_follow_the_program():
+    """one abstract thread per (histogram h, point i) over partners j in [jb, N):
+    nh * N threads; trips N - i - 1 on the self-correlation rows (DD, RR_s), N on the DR rows."""
+    p = W.tpacf_small(n=37, n_rand=2)
+    n, nr = p.n, p.n_rand
+    assert O.n_threads(O.TPACF, p) == (1 + 2 * nr) * n
+    tr = O.trips(O.TPACF, p).reshape(1 + 2 * nr, n)
+    for h in range(1 + 2 * nr):
+        want = [n - i - 1 for i in range(n)] if h <= nr else [n] * n
+        assert tr[h].tolist() == want
 
 
 def test_tpacf_trip_counts_sum_to_pairs():
-    p = W.tpacf_small(n=100, n_rand=2, chunk=32)
+    p = W.tpacf_small(n=100, n_rand=2)
     tr = O.trips(O.TPACF, p)
     n = p.n
     assert tr.sum() == 3 * n * (n - 1) // 2 + 2 * n * n
@@ -209,7 +214,7 @@ def test_tpacf_edges_are_strictly_decreasing_fp32():
 
 
 # ---------------------------------------------------------------- detector invariants & directed faults
-BENCH_PROBS = {O.CP: W.cp_small, O.MRIQ: W.mriq_small, O.TPACF: lambda: W.tpacf_small(n=120, n_rand=2, chunk=32)}
+BENCH_PROBS = {O.CP: W.cp_small, O.MRIQ: W.mriq_small, O.TPACF: lambda: W.tpacf_small(n=120, n_rand=2)}
 
 
 @pytest.mark.parametrize("bench", [O.CP, O.MRIQ, O.TPACF])
@@ -318,14 +323,14 @@ def test_tpacf_bin_flip_out_of_histogram_crashes():
     R = O.profile_ranges(O.TPACF, p)
     tr = O.trips(O.TPACF, p)
     g = int(np.nonzero(tr > 3)[0][0])
-    _, info = _one(O.TPACF, p, R, 27, g, 1, 1 << 20)  # bin -> huge -> hidx OOB (R16)
+    _, info = _one(O.TPACF, p, R, 26, g, 1, 1 << 20)  # bin -> huge -> hidx OOB (R16)
     assert info.fail & O.FL_CRASH
 
 
 # ---------------------------------------------------------------- campaign modes (R22)
 @pytest.mark.parametrize("exact", [0, 1])
 def test_replay_equals_replica_small_campaign(exact):
-    probs = [W.cp_small(), W.mriq_problem(4, 23, n_vox=60), W.tpacf_small(n=60, n_rand=1, chunk=16)]
+    probs = [W.cp_small(), W.mriq_problem(4, 23, n_vox=60), W.tpacf_small(n=60, n_rand=1)]
     R = [O.profile_ranges(b, probs[b], exact=exact) for b in range(3)]
     c1, r1 = O.campaign(-1, probs, R, seed=321, first=0, count=240, exact=exact, mode=1)
     c0, r0 = O.campaign(-1, probs, R, seed=321, first=0, count=240, exact=exact, mode=0)

@@ -236,7 +236,7 @@ def _enumerate_instances(bench, p):
 
 
 def test_decode_matches_bruteforce_enumeration_tpacf():
-    p = W.tpacf_small(n=70, n_rand=1, chunk=16)
+    p = W.tpacf_small(n=70, n_rand=1)
     inst = _enumerate_instances(O.TPACF, p)
     L = O.lib()
     seed = 99
@@ -283,7 +283,7 @@ def test_decode_sites_uniform_chi2():
 def test_site_catalogue_sizes():
     # 22 + 4U CP sites (38 at U=4, 54 at U=8 ~ "20-50 virtual variables", L2298)
     assert O.nsites(O.CP, 4) == 38 and O.nsites(O.CP, 8) == 54
-    assert O.nsites(O.MRIQ) == 36 and O.nsites(O.TPACF) == 31  # MRI-Q: 29 Q-kernel + 7 PhiMag sites
+    assert O.nsites(O.MRIQ) == 36 and O.nsites(O.TPACF) == 30  # MRI-Q: 29 Q-kernel + 7 PhiMag sites
 
 
 # ---------------------------------------------------------------- multi-bit masks (NEXT f1)

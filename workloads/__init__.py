@@ -153,7 +153,6 @@ def mriq_config2() -> MRIQProblem:
 class TPACFProblem:
     pts: np.ndarray  # float32 [(1 + n_rand), n, 3] unit vectors; set 0 = data
     edges: np.ndarray  # float32 [n_bins + 1], strictly decreasing cos(angle edges)
-    chunk: int = 512
 
     @property
     def n(self) -> int:
@@ -184,7 +183,7 @@ def _sphere_uniform(seed: int, n: int, start: int) -> np.ndarray:
 
 
 def tpacf_problem(n: int, n_rand: int, seed: int = 0x545041, n_bins: int = 20,
-                  clumps: int = 64, sigma_deg: float = 0.5, chunk: int = 512) -> TPACFProblem:
+                  clumps: int = 64, sigma_deg: float = 0.5) -> TPACFProblem:
     """Random sets uniform on the sphere; the data set is 50 % uniform + 50 % in `clumps`
     Gaussian clumps of width sigma_deg (so DD differs from RR)."""
     pts = np.empty((1 + n_rand, n, 3), dtype=np.float32)
@@ -201,7 +200,7 @@ def tpacf_problem(n: int, n_rand: int, seed: int = 0x545041, n_bins: int = 20,
     pts[0] = np.concatenate([d_uni, v], axis=0).astype(np.float32)
     for s in range(n_rand):
         pts[1 + s] = _sphere_uniform(seed ^ (0x1000 * (s + 1)), n, 0).astype(np.float32)
-    return TPACFProblem(pts=pts, edges=tpacf_edges(n_bins), chunk=chunk)
+    return TPACFProblem(pts=pts, edges=tpacf_edges(n_bins))
 
 
 def tpacf_config3() -> TPACFProblem:
@@ -219,5 +218,5 @@ def mriq_small(seed: int = 11) -> MRIQProblem:
     return mriq_problem(8, 197, seed=seed, n_vox=500)
 
 
-def tpacf_small(seed: int = 13, n: int = 300, n_rand: int = 2, chunk: int = 64) -> TPACFProblem:
-    return tpacf_problem(n, n_rand, seed=seed, clumps=8, sigma_deg=2.0, chunk=chunk)
+def tpacf_small(seed: int = 13, n: int = 300, n_rand: int = 2) -> TPACFProblem:
+    return tpacf_problem(n, n_rand, seed=seed, clumps=8, sigma_deg=2.0)

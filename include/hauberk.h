@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define HK_ABI_VERSION 1
+#define HK_ABI_VERSION 2
 
 #if defined(__GNUC__)
 #define HK_API __attribute__((visibility("default")))
@@ -85,8 +85,10 @@ typedef struct {
 } hk_control;
 
 /* CP (K1; Fig. 9).  atoms: [n_atoms] (x, y, z, q); atoms_ws: [n_atoms] float4 scratch
- * for the (x, y, dz^2, q) pre-pass; grid: [ny][nx] output, zeroed by the callee.
- * Requires nx % (bx*unroll) == 0, ny % by == 0, bx*by <= 1024, unroll in {1,2,4,8}. */
+ * for the (x, y, dz^2, q) pre-pass (both 16-byte aligned); grid: [ny][nx] output, zeroed by the
+ * callee.  Requires nx % (bx*unroll) == 0, ny % by == 0, bx*by <= 256 and a multiple of 32,
+ * unroll in {1,2,4,8} (campaigns: unroll 4 or 8).  Detector d (maxvar = d + 1) checks the
+ * self-accumulator E_{unroll-1} for d = 0, then E_0, E_1, ... (A6, DESIGN R12). */
 typedef struct {
   const float* atoms; float* atoms_ws; int32_t n_atoms; float z0, h;
   int32_t nx, ny, bx, by, unroll; float* grid; int32_t exact;
@@ -101,9 +103,10 @@ typedef struct {
 
 /* TPACF (K3).  pts: [(1+n_rand)][n][3] unit vectors (set 0 = data); edges: [n_bins+1] strictly
  * decreasing cos(angle) edges; hist: [(1+2*n_rand)][n_bins+2] u64 output (zeroed by the callee).
- * chunk = partners per abstract thread.  n_bins <= 30. */
+ * One abstract thread per (histogram h, point i) over all its partners; how the
+ * kernels tile that loop is internal.  n_bins <= 30. */
 typedef struct {
-  const float* pts; const float* edges; int32_t n, n_rand, n_bins, chunk; unsigned long long* hist;
+  const float* pts; const float* edges; int32_t n, n_rand, n_bins; unsigned long long* hist;
 } hk_tpacf_args;
 
 typedef struct { int32_t maxvar; int32_t t0_exp10; float alpha; } hk_profile_opts; /* defaults 1, -5, 1 */
@@ -117,14 +120,20 @@ typedef struct { int32_t maxvar; int32_t t0_exp10; float alpha; } hk_profile_opt
  * §8 f4: the faulted thread dereferences corrupted addresses itself and the R17 watchdog is off,
  * so a crash kills the calling process's CUDA context and a hang never returns — only for a
  * supervised child process, paper_conf_ipps_yimpski11_b200/guardian.py);
- * batch = replicas per launch (0 = auto); site_mask[b] bit s enables site s. */
+ * batch = replicas per launch (0 = auto); site_mask[b] bit s enables site s.
+ * variant: HK_FIFT (0) = the FI&FT binary (HAUBERK-protected program with the injector) or
+ * HK_FI_ONLY (1) = the FI binary (the original program with the injector: its
+ * catalogue keeps only the original program's sites — hauberk_detector_site() — and its outcomes
+ * are masked / undetected (SDC) / failure; ranges may be empty).  hang_factor: R17's T, a loop
+ * running more than T x max(golden trips, 1) iterations is a hang (0 = 10). */
 typedef struct {
   uint64_t seed; int64_t first, count; int32_t nbits; int32_t mode; int32_t batch; int32_t exact;
-  uint64_t site_mask[3];
+  uint64_t site_mask[3]; int32_t variant; int32_t hang_factor;
 } hk_campaign;
+enum { HK_FIFT = 0, HK_FI_ONLY = 1 };
 
 /* One decoded injection (DESIGN R13-R15). */
-typedef struct { int32_t site; int32_t pad; int64_t thread, inst; uint64_t mask; } hk_fault;
+typedef struct { int32_t site; int32_t hang; int64_t thread, inst; uint64_t mask; } hk_fault;
 
 /* One classified injection (device array, `count` entries, slot = n - first). */
 typedef struct {
@@ -148,9 +157,9 @@ HK_API hk_status hauberk_run_tpacf(const hk_tpacf_args* args, int32_t variant, c
 /* Single-run sharding (the benchmarks' abstract threads are independent):
  * run only the partition units [begin, end) of one benchmark, bit-identical to the same units of
  * the whole run.  Units: CP = grid rows (begin, end multiples of by, or end = ny); MRI-Q = voxels
- * (the slice's abstract-thread ids, e.g. hk_control.first_thread, are slice-local); TPACF = work
- * rows h*nC + c, nC = ceil(n / chunk) (histogram h in DD, RR_1..nr, DR_1..nr; chunk c), whose
- * counts are ADDED into a zeroed hist, so the partial histograms of a partition sum to the whole
+ * (the slice's abstract-thread ids, e.g. hk_control.first_thread, are slice-local); TPACF =
+ * abstract threads g = h*n + i (histogram h in DD, RR_1..nr, DR_1..nr; point i), whose counts are
+ * ADDED into a zeroed hist, so the partial histograms of a partition sum to the whole
  * (one all-reduce).  The callee zeroes only its own output part (CP rows, MRI-Q voxels; TPACF the
  * whole hist).  variant: HK_BASE / HK_FT / HK_FT_NL / HK_FT_L (profile over the whole input with
  * hauberk_profile_ranges and share the ranges).  hauberk_part_units returns the unit count and the
@@ -199,12 +208,52 @@ HK_API hk_status hauberk_campaign_run(hk_campaign_session* session, int64_t firs
 HK_API void hauberk_campaign_destroy(hk_campaign_session* session);
 
 /* Host-side decode of injections [first, first+count) (same rule the campaign uses; nbits as in
- * hk_campaign: <= 1 single-bit, k > 1 = k distinct bits, DESIGN R15 / NEXT f1). */
+ * hk_campaign: <= 1 single-bit, k > 1 = k distinct bits, DESIGN R15 / NEXT f1; variant as in
+ * hk_campaign: HK_FI_ONLY decodes over the original program's sites only). */
 HK_API hk_status hauberk_decode(int32_t bench_mode, const void* const args[3], const uint64_t site_mask[3],
-                         uint64_t seed, int32_t nbits, int64_t first, int64_t count, int32_t* bench_out, hk_fault* out);
+                         uint64_t seed, int32_t nbits, int32_t variant, int64_t first, int64_t count,
+                         int32_t* bench_out, hk_fault* out);
 
 /* Number of injection sites of a benchmark (unroll only matters for CP). */
 HK_API int32_t hauberk_num_sites(int32_t bench, int32_t unroll);
+/* 1 if `site` exists only because of HAUBERK (the loop detector's counter / accumulator and the
+ * expected trip count: CP it, MRI-Q it, TPACF expect / acc / cnt), i.e. absent from the FI-only
+ * binary's catalogue (row a7); 0 otherwise; -1 for an invalid bench / site. */
+HK_API int32_t hauberk_detector_site(int32_t bench, int32_t unroll, int32_t site);
+
+/* Device memory hauberk_campaign_create allocates for benchmark `bench` of campaign C besides the
+ * caller's buffers: golden output, the batch's replica outputs and control blocks (C->batch, 0 =
+ * auto; replay mode: 1), TPACF tables, MRI-Q per-replica k-space when PhiMag sites are enabled.
+ * Each hauberk_campaign_run slice of `count` injections adds 40 B x count (fault records) in
+ * replica mode, 81 B x count + 1 KB (device decode) in replay mode.  0 on invalid arguments. */
+HK_API size_t hauberk_campaign_workspace_bytes(int32_t bench, const void* args, const hk_campaign* C);
+
+/* ---- Evaluation and recovery arithmetic (host, no device work) ----
+ * Campaign summary (R2): counts = int64 [5] of one campaign (sum the
+ * rows of several benchmarks first).  coverage = P(masked or detected or failure) = 1 -
+ * undetected / total; sdc = undetected / total (for an HK_FI_ONLY campaign: the unprotected SDC
+ * rate of the original program, L211-213); detected = (detected + detected&masked) / total;
+ * failure = failure / total.  HK_ERR_INVALID if the total is 0. */
+typedef struct { double coverage, sdc, detected, failure; int64_t total; } hk_summary;
+HK_API hk_status hauberk_summarize(const int64_t counts[5], hk_summary* out);
+/* A11 ("calculates new ranges that include the outlier"; DESIGN R24): each of
+ * the n finite values joins the range of its correlation class at the set's threshold
+ * T = 10^t_exp10 (neg v < -T, zero |v| <= T, pos v > T); a class without a range gains one; ranges
+ * stay in class order.  *added (nullable) = ranges created. */
+HK_API hk_status hauberk_extend_ranges(hk_range_set* set, const float* values, int32_t n, int32_t* added);
+/* The outlier interval a run recorded for detector d in a (host copy of a) control block: 0, 1 or
+ * 2 values written to out[2] (*n); feed them to hauberk_extend_ranges on a diagnosed false alarm. */
+HK_API hk_status hauberk_outliers(const hk_control* cb, int32_t d, float out[2], int32_t* n);
+/* alpha controller: false-positive ratio > hi (0.10) -> alpha x 10;
+ * < lo (0.05) -> alpha / 10 as long as alpha stays >= 1. */
+HK_API float hauberk_alpha_update(float alpha, double fp_ratio, double hi, double lo);
+/* Re-execution diagnosis of an alarm (Fig. 11): (alarm, fail) of the first run
+ * and of its re-execution, and whether the two outputs are bitwise identical (hauberk_compare). */
+enum { HK_DIAG_OK = 0, HK_DIAG_FALSE_ALARM = 1, HK_DIAG_TRANSIENT = 2, HK_DIAG_PERSISTENT = 3, HK_DIAG_FAILURE = 4 };
+HK_API int32_t hauberk_diagnose(uint32_t alarm1, uint32_t fail1, uint32_t alarm2, uint32_t fail2, int32_t identical);
+
+/* Free cached per-shape device tables (the TPACF single-run schedules) of the current device. */
+HK_API void hauberk_release_caches(void);
 
 HK_API const char* hauberk_strerror(hk_status s);
 HK_API const char* hauberk_last_error(void);

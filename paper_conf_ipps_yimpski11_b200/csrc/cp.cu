@@ -114,7 +114,7 @@ __device__ __forceinline__ void cp_body(const CPParams& p, float4 (*tile)[CP_TIL
 #pragma unroll
     for (int d = 0; d < U; ++d) {
       if (d < p.ndet) {
-        const float v = __fdiv_rn(E[U - 1 - d], fit);
+        const float v = __fdiv_rn(E[d == 0 ? U - 1 : d - 1], fit);
         if (PROF) p.samples[(int64_t)d * p.nthreads + tid] = v;
         if (L && p.R.n[d] > 0 && !in_range<false>(p.R, d, v, nullptr)) {
           alarm |= AL_RANGE;
@@ -189,7 +189,9 @@ __device__ __forceinline__ CPGeo cp_geo_of(int64_t t, int BX, int BY, int gx, in
 }
 
 // REAL: the guardian's unguarded variant (R25) — no R16 guards, no R17 watchdog.
-template <int KIND, int U, bool EXACT, bool REAL = false, class Sink>
+// FT = false: the FI-only binary (row a7) — the same program without HAUBERK: no
+// counter, no checks (the duplicate / checksum arithmetic feeds nothing and is removed).
+template <int KIND, int U, bool EXACT, bool REAL = false, bool FT = true, class Sink>
 __device__ void cp_fi_program(const CPParams& p, const FaultRec& f, const CPGeo& G, bool mine, uint64_t grid_real,
                               Sink& S) {
   const int BX = G.BX, BY = G.BY;
@@ -244,7 +246,7 @@ __device__ void cp_fi_program(const CPParams& p, const FaultRec& f, const CPGeo&
   for (int j = 0; j < U; ++j) E[j] = 0.0f;
   int32_t it = 0;
   int32_t atomid = 0;
-  const int64_t limit = fi_limit<REAL>(n_atoms);
+  const int64_t limit = fi_limit<REAL>(n_atoms, f.hang);
   constexpr bool real = REAL;
   for (int64_t i = 0;; ++i) {
     const bool now = (i == inst);
@@ -294,17 +296,17 @@ __device__ void cp_fi_program(const CPParams& p, const FaultRec& f, const CPGeo&
         if (KIND == CK_E) { applied |= nj; E[j] = flip_f(E[j], nj, mask); }
       }
     }
-    it = count_inc(it, p.one);
+    if (FT) it = count_inc(it, p.one);
     if (KIND == CK_IT) { applied |= now; it = flip_i(it, now, mask); }
     atomid = (int32_t)((uint32_t)atomid + 1u);
   }
-  if (it != numatoms) alarm |= AL_COUNT;
-  if (it != 0) {
+  if (FT && it != numatoms) alarm |= AL_COUNT;
+  if (FT && it != 0) {
     const float fit = (float)it;
 #pragma unroll
     for (int d = 0; d < U; ++d) {
       if (d < p.ndet && p.R.n[d] > 0) {
-        const float v = __fdiv_rn(E[U - 1 - d], fit);
+        const float v = __fdiv_rn(E[d == 0 ? U - 1 : d - 1], fit);
         if (!in_range<true>(p.R, d, v, &margin, &gap)) { alarm |= AL_RANGE; S.outlier(d, v); }
       }
     }
@@ -320,10 +322,11 @@ __device__ void cp_fi_program(const CPParams& p, const FaultRec& f, const CPGeo&
   chk ^= ((uint32_t)numatoms + z) ^ (fb(h) + z) ^ (lohi(pgrid) + z) ^ (lohi(patoms) + z);
   if (chk != 0) alarm |= AL_CHK;
 done:
+  if (!FT) alarm = 0;
   S.finish(mine, alarm, fail, margin, gap, 0u, applied, (uint32_t)t);
 }
 
-template <int KIND, int U, bool EXACT>
+template <int KIND, int U, bool EXACT, bool FT>
 __global__ void __launch_bounds__(256) cp_fi_kernel(const CPFIParams q) {
   __shared__ __align__(128) float4 tile[2][CP_TILE];
   __shared__ __align__(8) uint64_t bar[2];
@@ -339,12 +342,12 @@ __global__ void __launch_bounds__(256) cp_fi_kernel(const CPFIParams q) {
   p.cb = q.cb0 + r;
   const int bxi = (int)(cta % gridDim.x), byi = (int)(cta / gridDim.x);
   if (!faulted) {
-    cp_body<V_NL | V_L, U, EXACT, true>(p, tile, bar, bxi, byi);
+    cp_body<FT ? (V_NL | V_L) : 0, U, EXACT, true>(p, tile, bar, bxi, byi);
   } else {
     const CPGeo G = cp_geo_here(bxi, byi);
     const int64_t t = ((int64_t)G.byi * G.gx + G.bxi) * (G.BX * G.BY) + G.ty * G.BX + G.tx;
     ReplicaSinkF S{{p.grid, nullptr}, p.cb};
-    cp_fi_program<KIND, U, EXACT>(p, f, G, t == f.thread, (uint64_t)(uintptr_t)p.grid, S);
+    cp_fi_program<KIND, U, EXACT, false, FT>(p, f, G, t == f.thread, (uint64_t)(uintptr_t)p.grid, S);
   }
 }
 
@@ -389,11 +392,11 @@ struct CPReplayParams {
   uint8_t kind_of_site[64];
 };
 
-template <int KIND, int U, bool EXACT>
+template <int KIND, int U, bool EXACT, bool FT>
 __device__ __forceinline__ void cp_replay_one(const CPReplayParams& q, const FaultRec& f) {
   const CPGeo G = cp_geo_of(f.thread, q.BX, q.BY, q.gx, q.gy);
   ReplaySinkF<U> S;
-  cp_fi_program<KIND, U, EXACT>(q.base, f, G, true, (uint64_t)(uintptr_t)q.golden, S);
+  cp_fi_program<KIND, U, EXACT, false, FT>(q.base, f, G, true, (uint64_t)(uintptr_t)q.golden, S);
   bool wrong = false;
   float worst = 0.f;
   if (!S.fail) {
@@ -427,13 +430,13 @@ __device__ __forceinline__ void cp_replay_one(const CPReplayParams& q, const Fau
 
 // One CUDA thread per injection; the records arrive sorted by site kind (decode.cu), so warps
 // take one branch of the switch.
-template <int U, bool EXACT>
+template <int U, bool EXACT, bool FT>
 __global__ void __launch_bounds__(128) cp_replay_all_kernel(const CPReplayParams q) {
   const int r = blockIdx.x * blockDim.x + threadIdx.x;
   if (r >= q.nrep) return;
   const FaultRec f = q.faults[r];
   switch (q.kind_of_site[f.site & 63]) {
-#define K(k) case k: cp_replay_one<k, U, EXACT>(q, f); break;
+#define K(k) case k: cp_replay_one<k, U, EXACT, FT>(q, f); break;
     K(CK_NL) K(CK_LIVE) K(CK_ATOMID) K(CK_AX) K(CK_AY) K(CK_AZ) K(CK_AW) K(CK_DY) K(CK_DYZ2) K(CK_DX0)
     K(CK_DXJ) K(CK_R2) K(CK_S) K(CK_E) K(CK_IT)
 #undef K
@@ -517,18 +520,18 @@ int cp_site_kind(int site, int U, int* sub) {
   return CK_IT;
 }
 
-template <int KIND, int U, bool EXACT>
+template <int KIND, int U, bool EXACT, bool FT>
 static cudaError_t launch_cp_fi_k(const CPFIParams& q, dim3 grid, dim3 block, cudaStream_t s) {
   TimedScope ts(HK_CP, 1, (double)q.base.numatoms * (double)q.base.nthreads * U * grid.z, s);
-  cp_fi_kernel<KIND, U, EXACT><<<grid, block, 0, s>>>(q);
+  cp_fi_kernel<KIND, U, EXACT, FT><<<grid, block, 0, s>>>(q);
   count_launch();
   return cudaGetLastError();
 }
 
-template <int U, bool EXACT>
+template <int U, bool EXACT, bool FT>
 static cudaError_t launch_cp_fi_e(int kind, const CPFIParams& q, dim3 grid, dim3 block, cudaStream_t s) {
   switch (kind) {
-#define K(k) case k: return launch_cp_fi_k<k, U, EXACT>(q, grid, block, s);
+#define K(k) case k: return launch_cp_fi_k<k, U, EXACT, FT>(q, grid, block, s);
     K(CK_NL) K(CK_LIVE) K(CK_ATOMID) K(CK_AX) K(CK_AY) K(CK_AZ) K(CK_AW) K(CK_DY) K(CK_DYZ2) K(CK_DX0)
     K(CK_DXJ) K(CK_R2) K(CK_S) K(CK_E) K(CK_IT)
 #undef K
@@ -537,7 +540,7 @@ static cudaError_t launch_cp_fi_e(int kind, const CPFIParams& q, dim3 grid, dim3
 }
 
 // One batch of `nrep` replicas of one kind: faults[0..nrep), outputs grid0[r], control blocks cb0[r].
-cudaError_t cp_fi_launch(int kind, const hk_cp_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
+cudaError_t cp_fi_launch(int kind, bool ft, const hk_cp_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
                          float* grid0, int64_t stride, hk_control* cb0, bool real, cudaStream_t s) {
   CPFIParams q{};
   q.base.atoms = reinterpret_cast<const float4*>(a.atoms_ws);
@@ -566,13 +569,18 @@ cudaError_t cp_fi_launch(int kind, const hk_cp_args& a, const DevRanges& R, int 
     count_launch();
     return cudaGetLastError();
   }
+  if (a.unroll != 8 && a.unroll != 4) return cudaErrorInvalidValue;
+  if (ft) {
+    if (a.unroll == 8)
+      return a.exact ? launch_cp_fi_e<8, true, true>(kind, q, grid, block, s) : launch_cp_fi_e<8, false, true>(kind, q, grid, block, s);
+    return a.exact ? launch_cp_fi_e<4, true, true>(kind, q, grid, block, s) : launch_cp_fi_e<4, false, true>(kind, q, grid, block, s);
+  }
   if (a.unroll == 8)
-    return a.exact ? launch_cp_fi_e<8, true>(kind, q, grid, block, s) : launch_cp_fi_e<8, false>(kind, q, grid, block, s);
-  if (a.unroll != 4) return cudaErrorInvalidValue;
-  return a.exact ? launch_cp_fi_e<4, true>(kind, q, grid, block, s) : launch_cp_fi_e<4, false>(kind, q, grid, block, s);
+    return a.exact ? launch_cp_fi_e<8, true, false>(kind, q, grid, block, s) : launch_cp_fi_e<8, false, false>(kind, q, grid, block, s);
+  return a.exact ? launch_cp_fi_e<4, true, false>(kind, q, grid, block, s) : launch_cp_fi_e<4, false, false>(kind, q, grid, block, s);
 }
 
-cudaError_t cp_replay_launch(int kind, const hk_cp_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
+cudaError_t cp_replay_launch(int kind, bool ft, const hk_cp_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
                              const float* golden, const float* dM, hk_outcome* records, int64_t first, int64_t* counts,
                              int64_t* site_counts, cudaStream_t s) {
   if (nrep <= 0) return cudaSuccess;
@@ -598,11 +606,11 @@ cudaError_t cp_replay_launch(int kind, const hk_cp_args& a, const DevRanges& R, 
   const unsigned g = (unsigned)((nrep + 127) / 128);
   TimedScope ts(HK_CP, 2, (double)a.n_atoms * a.unroll * nrep, s);
   if (a.unroll == 8) {
-    if (a.exact) cp_replay_all_kernel<8, true><<<g, 128, 0, s>>>(q);
-    else cp_replay_all_kernel<8, false><<<g, 128, 0, s>>>(q);
+    if (a.exact) ft ? cp_replay_all_kernel<8, true, true><<<g, 128, 0, s>>>(q) : cp_replay_all_kernel<8, true, false><<<g, 128, 0, s>>>(q);
+    else ft ? cp_replay_all_kernel<8, false, true><<<g, 128, 0, s>>>(q) : cp_replay_all_kernel<8, false, false><<<g, 128, 0, s>>>(q);
   } else if (a.unroll == 4) {
-    if (a.exact) cp_replay_all_kernel<4, true><<<g, 128, 0, s>>>(q);
-    else cp_replay_all_kernel<4, false><<<g, 128, 0, s>>>(q);
+    if (a.exact) ft ? cp_replay_all_kernel<4, true, true><<<g, 128, 0, s>>>(q) : cp_replay_all_kernel<4, true, false><<<g, 128, 0, s>>>(q);
+    else ft ? cp_replay_all_kernel<4, false, true><<<g, 128, 0, s>>>(q) : cp_replay_all_kernel<4, false, false><<<g, 128, 0, s>>>(q);
   } else {
     return cudaErrorInvalidValue;
   }

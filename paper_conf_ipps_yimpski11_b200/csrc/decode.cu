@@ -21,7 +21,7 @@ struct DecodeParams {
   DevCatalog cat[3];
   uint64_t seed;
   int64_t first, count;
-  int32_t bench_mode, nbits;
+  int32_t bench_mode, nbits, hang;
   FaultRec* tmp;
   uint8_t* key;       // bench * 32 + kind
   uint32_t* hist;     // [96]
@@ -42,7 +42,7 @@ __global__ void decode_kernel(const DecodeParams P) {
   f.site = s;
   f.sub = K.sub[s];
   f.real = 0;
-  f.pad_ = 0;
+  f.hang = P.hang;
   if (K.is_nl[s]) {
     const int64_t nt = (b == HK_MRIQ && s >= MRIQ_PHIMAG_SITE0) ? K.nk : K.nthr;
     f.thread = (int64_t)d_below(r2, (uint64_t)nt);
@@ -109,7 +109,7 @@ size_t decode_ws_bytes(int64_t count) {
 }
 
 cudaError_t decode_sort_launch(const DevCatalog cat[3], uint64_t seed, int64_t first, int64_t count, int32_t bench_mode,
-                               int32_t nbits, void* ws, FaultRec** sorted_out, cudaStream_t s) {
+                               int32_t nbits, int32_t hang, void* ws, FaultRec** sorted_out, cudaStream_t s) {
   char* p = reinterpret_cast<char*>(ws);
   FaultRec* sorted = reinterpret_cast<FaultRec*>(p);
   FaultRec* tmp = sorted + count;
@@ -120,7 +120,7 @@ cudaError_t decode_sort_launch(const DevCatalog cat[3], uint64_t seed, int64_t f
   if (e != cudaSuccess) return e;
   DecodeParams P{};
   for (int b = 0; b < 3; ++b) P.cat[b] = cat[b];
-  P.seed = seed; P.first = first; P.count = count; P.bench_mode = bench_mode; P.nbits = nbits;
+  P.seed = seed; P.first = first; P.count = count; P.bench_mode = bench_mode; P.nbits = nbits; P.hang = hang;
   P.tmp = tmp; P.key = key; P.hist = hist;
   const unsigned g = (unsigned)((count + 255) / 256);
   decode_kernel<<<g, 256, 0, s>>>(P);

@@ -113,7 +113,7 @@ void setup(const Blob& B, Dev* D) {
   } else if (B.bench == HK_TPACF) {
     if (B.arrays.size() != 2) die(2, "blob", "tpacf needs 2 arrays");
     CK(cudaMalloc(&D->hist, (size_t)(1 + 2 * I[1]) * (I[2] + 2) * 8));
-    D->tp = hk_tpacf_args{D->in[0], D->in[1], I[0], I[1], I[2], I[3], D->hist};
+    D->tp = hk_tpacf_args{D->in[0], D->in[1], I[0], I[1], I[2], D->hist};
   } else {
     die(2, "blob", "bad bench");
   }

@@ -39,7 +39,7 @@ struct FaultRec {
   int32_t site;
   int32_t sub;
   int32_t real;    // 1: unguarded run for the guardian (DESIGN R25); 0: crash / hang models R16 / R17
-  int32_t pad_;
+  int32_t hang;    // R17 watchdog factor T (<= 0: the paper's 10)
 };
 
 // Site catalogue of one benchmark for the device decode (DESIGN R14): enabled sites, per-site
@@ -244,10 +244,12 @@ __device__ __forceinline__ bool fi_order(int64_t L, int64_t ncta, int nrep, F fa
 }
 __device__ __forceinline__ int64_t clamp_cta(int64_t c, int64_t ncta) { return c < 0 ? 0 : (c >= ncta ? ncta - 1 : c); }
 
-// R17 watchdog limit; none in unguarded runs (the guardian's timeout observes the hang).
+// R17 watchdog limit T x max(golden trips, 1) (T = 10 unless the campaign sets hang_factor);
+// none in unguarded runs (the guardian's timeout observes the hang).
 template <bool REAL>
-__device__ __forceinline__ int64_t fi_limit(int64_t golden_trips) {
-  return REAL ? INT64_MAX : 10 * (golden_trips > 1 ? golden_trips : 1);
+__device__ __forceinline__ int64_t fi_limit(int64_t golden_trips, int32_t hang) {
+  const int64_t T = hang > 0 ? hang : 10;
+  return REAL ? INT64_MAX : T * (golden_trips > 1 ? golden_trips : 1);
 }
 
 __device__ __forceinline__ unsigned lane_id() {

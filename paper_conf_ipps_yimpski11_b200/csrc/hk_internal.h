@@ -31,10 +31,13 @@ cudaError_t cp_launch_rows(int vflags, const hk_cp_args& a, const DevRanges& R, 
                            int32_t y0, int32_t y1, cudaStream_t s);
 cudaError_t mriq_launch(int vflags, const hk_mriq_args& a, const DevRanges& R, int ndet, hk_control* cb,
                         float* samples, cudaStream_t s);
+// TPACF: abstract threads [g0, g1) (g1 < 0: all); ws = tpacf_ws_bytes(a) bytes (bin table, single-run
+// schedule counters, per-thread (acc, cnt) partial sums)
 cudaError_t tpacf_launch(int vflags, const hk_tpacf_args& a, const DevRanges& R, int ndet, hk_control* cb,
-                         float* samples, void* lut_ws, cudaStream_t s, int32_t row0 = 0, int32_t row1 = -1);
-size_t tpacf_lut_ws_bytes();
-cudaError_t tpacf_lut_build(const hk_tpacf_args& a, void* lut_ws, cudaStream_t s);
+                         float* samples, void* ws, cudaStream_t s, int32_t g0 = 0, int32_t g1 = -1);
+size_t tpacf_ws_bytes(const hk_tpacf_args& a);
+cudaError_t tpacf_lut_build(const hk_tpacf_args& a, void* ws, cudaStream_t s);
+void tpacf_release_caches();
 cudaError_t cp_prepass_launch(const hk_cp_args& a, cudaStream_t s);
 cudaError_t mriq_phimag_launch(const hk_mriq_args& a, bool nl, hk_control* cb, cudaStream_t s);
 
@@ -42,31 +45,32 @@ cudaError_t mriq_phimag_launch(const hk_mriq_args& a, bool nl, hk_control* cb, c
 int cp_site_kind(int site, int U, int* sub);
 int mriq_site_kind(int site);
 int tpacf_site_kind(int site);
-cudaError_t cp_fi_launch(int kind, const hk_cp_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
+// ft = false: the FI-only binary (row a7): BASE fast CTAs, the FI program without detectors
+cudaError_t cp_fi_launch(int kind, bool ft, const hk_cp_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
                          float* grid0, int64_t stride, hk_control* cb0, bool real, cudaStream_t s);
-cudaError_t mriq_fi_launch(int kind, const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
+cudaError_t mriq_fi_launch(int kind, bool ft, const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
                            int nrep, float* out0, int64_t stride, hk_control* cb0, float4* kv_rep, bool real,
                            cudaStream_t s);
 constexpr int MRIQ_PHIMAG_SITE0 = 29;  // PhiMag NL sites 29-35 (replica mode only)
-cudaError_t tpacf_fi_launch(int kind, const hk_tpacf_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
+cudaError_t tpacf_fi_launch(int kind, bool ft, const hk_tpacf_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
                             int nrep, unsigned long long* hist0, hk_control* cb0, void* lut_ws, bool real,
                             cudaStream_t s);
 
 // replay accelerator (one CUDA thread per injection; classification fused)
-cudaError_t cp_replay_launch(int kind, const hk_cp_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
+cudaError_t cp_replay_launch(int kind, bool ft, const hk_cp_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
                              const float* golden, const float* dM, hk_outcome* records, int64_t first, int64_t* counts,
                              int64_t* site_counts, cudaStream_t s);
-cudaError_t mriq_replay_launch(int kind, const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
+cudaError_t mriq_replay_launch(int kind, bool ft, const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
                                int nrep, const float* golden, const float* dM, hk_outcome* records, int64_t first,
                                int64_t* counts, int64_t* site_counts, cudaStream_t s);
-cudaError_t tpacf_replay_launch(int kind, const hk_tpacf_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
+cudaError_t tpacf_replay_launch(int kind, bool ft, const hk_tpacf_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
                                 int nrep, const unsigned long long* golden, hk_outcome* records, int64_t first,
                                 int64_t* counts, int64_t* site_counts, cudaStream_t s);
 
 // decode.cu: device decode + counting sort by (bench, kind) for the replay path
 size_t decode_ws_bytes(int64_t count);
 cudaError_t decode_sort_launch(const DevCatalog cat[3], uint64_t seed, int64_t first, int64_t count, int32_t bench_mode,
-                               int32_t nbits, void* ws, FaultRec** sorted_out, cudaStream_t s);
+                               int32_t nbits, int32_t hang, void* ws, FaultRec** sorted_out, cudaStream_t s);
 
 // classify.cu
 cudaError_t control_init_launch(hk_control* cb, int n, cudaStream_t s);

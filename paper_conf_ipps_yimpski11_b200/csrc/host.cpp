@@ -10,6 +10,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include <string>
 #include <vector>
 
@@ -48,6 +49,32 @@ static hk_status invalid(const char* why) {
   g_err = why;
   return HK_ERR_INVALID;
 }
+// Stream-ordered allocations of the library come from a private memory pool per device (release
+// threshold: keep freed memory for the next call) so the caller's default pool keeps its own
+// settings (the library no longer changes the default pool).
+static cudaError_t lib_malloc(void** p, size_t bytes, cudaStream_t s) {
+  static std::mutex mu;
+  static cudaMemPool_t pools[64] = {};
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (dev < 0 || dev >= 64) return cudaMallocAsync(p, bytes, s);
+  {
+    std::lock_guard<std::mutex> lk(mu);
+    if (!pools[dev]) {
+      cudaMemPoolProps props{};
+      props.allocType = cudaMemAllocationTypePinned;
+      props.handleTypes = cudaMemHandleTypeNone;
+      props.location.type = cudaMemLocationTypeDevice;
+      props.location.id = dev;
+      if ((e = cudaMemPoolCreate(&pools[dev], &props)) != cudaSuccess) return e;
+      uint64_t thr = UINT64_MAX;
+      cudaMemPoolSetAttribute(pools[dev], cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+  }
+  return cudaMallocFromPoolAsync(p, bytes, pools[dev], s);
+}
+
 #define HK_CUDA(call, where)                       \
   do {                                             \
     cudaError_t _e = (call);                       \
@@ -105,7 +132,8 @@ static bool mriq_ok(const hk_mriq_args* a) {
 }
 static bool tpacf_ok(const hk_tpacf_args* a) {
   if (!a || !a->pts || !a->edges || !a->hist) return false;
-  if (a->n <= 0 || a->n_rand < 1 || a->n_bins < 1 || a->n_bins > 30 || a->chunk < 1 || a->chunk > 1024) return false;
+  if (a->n <= 0 || a->n_rand < 1 || a->n_bins < 1 || a->n_bins > 30) return false;
+  if ((int64_t)(1 + 2 * a->n_rand) * a->n > INT32_MAX / 2) return false;  // abstract thread ids are int32
   return true;
 }
 static bool tpacf_edges_ok(const hk_tpacf_args* a, cudaStream_t s) {
@@ -118,16 +146,12 @@ static bool tpacf_edges_ok(const hk_tpacf_args* a, cudaStream_t s) {
 }
 
 static int64_t cp_threads(const hk_cp_args* a) { return (int64_t)(a->nx / a->unroll) * a->ny; }
-static int tp_nc(const hk_tpacf_args* a) { return (a->n + a->chunk - 1) / a->chunk; }
-static int64_t tp_threads(const hk_tpacf_args* a) { return (int64_t)(1 + 2 * a->n_rand) * tp_nc(a) * a->n; }
+// TPACF abstract thread g = h*N + i loops over j in [jb, N): jb = i + 1 on the self-correlation
+// rows h <= n_rand (DD, RR_s), 0 on the DR rows.
+static int64_t tp_threads(const hk_tpacf_args* a) { return (int64_t)(1 + 2 * a->n_rand) * a->n; }
 static int64_t tp_trips(const hk_tpacf_args* a, int64_t g) {
-  const int nC = tp_nc(a), C = a->chunk, N = a->n;
-  const int64_t row = g / N;
-  const int i = (int)(g % N), h = (int)(row / nC), c = (int)(row % nC);
-  int64_t jb = (int64_t)c * C;
-  if (h <= a->n_rand) jb = std::max<int64_t>(jb, i + 1);
-  const int64_t je = std::min<int64_t>((int64_t)(c + 1) * C, N);
-  return je > jb ? je - jb : 0;
+  const int64_t h = g / a->n, i = g % a->n;
+  return h <= a->n_rand ? (int64_t)a->n - (i + 1) : (int64_t)a->n;
 }
 static int64_t bench_threads(int b, const void* args) {
   if (b == HK_CP) return cp_threads((const hk_cp_args*)args);
@@ -172,10 +196,10 @@ static hk_status run_bench(int b, const void* args, int variant, const hk_ranges
     ndet = std::min(ndet, 1);
     HK_CUDA(cudaMemsetAsync(a->hist, 0, sizeof(unsigned long long) * (size_t)(1 + 2 * a->n_rand) * (a->n_bins + 2), s),
             "memset hist");
-    void* lut = nullptr;
-    HK_CUDA(cudaMallocAsync(&lut, tpacf_lut_ws_bytes(), s), "alloc tpacf table");
-    cudaError_t e = tpacf_launch(vf, *a, R, ndet, d_cb, d_samples, lut, s);
-    cudaFreeAsync(lut, s);
+    void* ws = nullptr;
+    HK_CUDA(lib_malloc(&ws, tpacf_ws_bytes(*a), s), "alloc tpacf workspace");
+    cudaError_t e = tpacf_launch(vf, *a, R, ndet, d_cb, d_samples, ws, s);
+    cudaFreeAsync(ws, s);
     HK_CUDA(e, "tpacf kernel");
   }
   return HK_OK;
@@ -238,14 +262,21 @@ static hk_range_set profile_search(const std::vector<float>& v, int t0) {
 // ---------------------------------------------------------------------------------------------
 // Site catalogue and decode (R14, R15)
 // ---------------------------------------------------------------------------------------------
-static int num_sites(int b, int unroll) { return b == HK_CP ? 22 + 4 * unroll : (b == HK_MRIQ ? 36 : 31); }
+static int num_sites(int b, int unroll) { return b == HK_CP ? 22 + 4 * unroll : (b == HK_MRIQ ? 36 : 30); }
 static bool site_is_nl(int b, int s) {
-  return b == HK_CP ? s <= 5 : (b == HK_MRIQ ? (s <= 3 || s >= MRIQ_PHIMAG_SITE0) : s <= 11);
+  return b == HK_CP ? s <= 5 : (b == HK_MRIQ ? (s <= 3 || s >= MRIQ_PHIMAG_SITE0) : s <= 10);
 }
 static int site_width(int b, int s) {
   if (b == HK_CP) return (s == 12 || s == 13) ? 64 : 32;
   if (b == HK_MRIQ) return (s >= 9 && s <= 14) ? 64 : 32;
-  return (s == 20 || s == 21) ? 64 : 32;
+  return (s == 19 || s == 20) ? 64 : 32;
+}
+// Sites that exist only because of HAUBERK (absent from the FI-only binary, row a7): the loop
+// detector's counter (CP, MRI-Q `it`), TPACF's expected trip count (@def 6, @live 13), acc and cnt.
+static bool site_is_detector(int b, int unroll, int s) {
+  if (b == HK_CP) return s == num_sites(b, unroll) - 1;
+  if (b == HK_MRIQ) return s == 28;
+  return s == 6 || s == 13 || s == 28 || s == 29;
 }
 static uint64_t splitmix(uint64_t seed, uint64_t m) {
   uint64_t z = seed + (m + 1) * 0x9E3779B97F4A7C15ull;
@@ -264,7 +295,7 @@ struct Catalog {
   std::vector<int64_t> prefix;  // TPACF: prefix[g] = trips of threads < g
 };
 
-static bool build_catalog(Catalog& K, int b, const void* args, uint64_t mask) {
+static bool build_catalog(Catalog& K, int b, const void* args, uint64_t mask, int variant) {
   K.bench = b;
   if (b == HK_CP) {
     const hk_cp_args* a = (const hk_cp_args*)args;
@@ -288,6 +319,7 @@ static bool build_catalog(Catalog& K, int b, const void* args, uint64_t mask) {
   }
   for (int s = 0; s < num_sites(b, K.unroll) && s < 64; ++s) {
     if (!((mask >> s) & 1ull)) continue;
+    if (variant == HK_FI_ONLY && site_is_detector(b, K.unroll, s)) continue;
     const int64_t D = site_is_nl(b, s) ? K.nl_threads(s) : K.total_trips;
     if (D > 0) K.enabled.push_back(s);
   }
@@ -296,6 +328,7 @@ static bool build_catalog(Catalog& K, int b, const void* args, uint64_t mask) {
 
 static hk_fault decode_one(const Catalog& K, uint64_t seed, int64_t n, int nbits) {
   hk_fault f{};
+  f.hang = 0;
   const uint64_t r1 = splitmix(seed, 8 * (uint64_t)n + 1);
   const uint64_t r2 = splitmix(seed, 8 * (uint64_t)n + 2);
   const uint64_t r3 = splitmix(seed, 8 * (uint64_t)n + 3);
@@ -427,6 +460,88 @@ int32_t hauberk_num_sites(int32_t bench, int32_t unroll) {
   if (bench < 0 || bench > 2) return 0;
   return num_sites(bench, unroll);
 }
+int32_t hauberk_detector_site(int32_t bench, int32_t unroll, int32_t site) {
+  if (bench < 0 || bench > 2 || site < 0 || site >= num_sites(bench, unroll)) return -1;
+  return site_is_detector(bench, unroll, site) ? 1 : 0;
+}
+
+hk_status hauberk_summarize(const int64_t counts[5], hk_summary* out) {
+  if (!counts || !out) return invalid("summarize: null argument");
+  int64_t tot = 0;
+  for (int c = 0; c < 5; ++c) {
+    if (counts[c] < 0) return invalid("summarize: negative count");
+    tot += counts[c];
+  }
+  out->total = tot;
+  if (tot == 0) {
+    out->coverage = out->sdc = out->detected = out->failure = NAN;
+    return invalid("summarize: empty campaign");
+  }
+  out->sdc = (double)counts[HK_UNDETECTED] / (double)tot;
+  out->coverage = 1.0 - out->sdc;
+  out->detected = (double)(counts[HK_DETECTED] + counts[HK_DETECTED_MASKED]) / (double)tot;
+  out->failure = (double)counts[HK_FAILURE] / (double)tot;
+  return HK_OK;
+}
+
+hk_status hauberk_extend_ranges(hk_range_set* set, const float* values, int32_t n, int32_t* added) {
+  if (!set || n < 0 || (n > 0 && !values) || set->n < 0 || set->n > 3 || set->t_exp10 < -38 || set->t_exp10 > 38)
+    return invalid("extend_ranges: bad arguments");
+  const float T = threshold(set->t_exp10);
+  auto cls = [&](float x) { return x < -T ? 0 : (x > T ? 2 : 1); };
+  bool have[3] = {false, false, false};
+  float lo[3] = {0, 0, 0}, hi[3] = {0, 0, 0};
+  for (int r = 0; r < set->n; ++r) {
+    const int c = cls(set->lo[r]);
+    have[c] = true; lo[c] = set->lo[r]; hi[c] = set->hi[r];
+  }
+  int32_t add = 0;
+  for (int32_t k = 0; k < n; ++k) {
+    const float x = values[k];
+    if (!std::isfinite(x)) continue;
+    const int c = cls(x);
+    if (!have[c]) { have[c] = true; lo[c] = hi[c] = x; ++add; }
+    else { lo[c] = std::min(lo[c], x); hi[c] = std::max(hi[c], x); }
+  }
+  int r = 0;
+  for (int c = 0; c < 3; ++c)
+    if (have[c]) { set->lo[r] = lo[c]; set->hi[r] = hi[c]; ++r; }
+  set->n = r;
+  if (added) *added = add;
+  return HK_OK;
+}
+
+static float ord_to_float(int32_t o) {
+  const uint32_t b = o >= 0 ? (uint32_t)o : (0x80000000u | (uint32_t)(-(int64_t)o));
+  float f;
+  std::memcpy(&f, &b, 4);
+  return f;
+}
+hk_status hauberk_outliers(const hk_control* cb, int32_t d, float out[2], int32_t* n) {
+  if (!cb || !out || !n || d < 0 || d >= 8) return invalid("outliers: bad arguments");
+  const int32_t lo = cb->outlier_min_ord[d], hi = cb->outlier_max_ord[d];
+  *n = 0;
+  if (lo > hi) return HK_OK;  // initial values 0x7fffffff / 0x80000000: nothing recorded
+  out[(*n)++] = ord_to_float(lo);
+  if (hi != lo) out[(*n)++] = ord_to_float(hi);
+  return HK_OK;
+}
+
+float hauberk_alpha_update(float alpha, double fp_ratio, double hi, double lo) {
+  if (fp_ratio > hi) return alpha * 10.0f;
+  if (fp_ratio < lo && alpha >= 10.0f) return alpha / 10.0f;
+  return alpha;
+}
+
+int32_t hauberk_diagnose(uint32_t alarm1, uint32_t fail1, uint32_t alarm2, uint32_t fail2, int32_t identical) {
+  if (fail1) return HK_DIAG_FAILURE;
+  if (!alarm1) return HK_DIAG_OK;
+  if (fail2) return HK_DIAG_FAILURE;
+  if (!alarm2) return HK_DIAG_TRANSIENT;
+  return identical ? HK_DIAG_FALSE_ALARM : HK_DIAG_PERSISTENT;
+}
+
+void hauberk_release_caches(void) { tpacf_release_caches(); }
 
 hk_status hauberk_run_cp(const hk_cp_args* args, int32_t variant, const hk_ranges* ranges, hk_control* d_cb,
                          float* d_samples, void* stream) {
@@ -471,7 +586,7 @@ hk_status hauberk_part_units(int32_t bench, const void* args, int64_t* units, in
     *units = ((const hk_mriq_args*)args)->n_vox; *granule = 1;
   } else {
     const hk_tpacf_args* a = (const hk_tpacf_args*)args;
-    *units = (int64_t)(1 + 2 * a->n_rand) * tp_nc(a); *granule = 1;
+    *units = tp_threads(a); *granule = 1;  // abstract threads g = h*n + i
   }
   return HK_OK;
 }
@@ -511,10 +626,10 @@ hk_status hauberk_run_part(int32_t bench, const void* args, int32_t variant, con
     HK_CUDA(cudaMemsetAsync(a->hist, 0, sizeof(unsigned long long) * (size_t)(1 + 2 * a->n_rand) * (a->n_bins + 2), s),
             "memset hist");
     if (end == begin) return HK_OK;
-    void* lut = nullptr;
-    HK_CUDA(cudaMallocAsync(&lut, tpacf_lut_ws_bytes(), s), "alloc tpacf table");
-    cudaError_t e = tpacf_launch(vf, *a, R, ndet, d_cb, nullptr, lut, s, (int32_t)begin, (int32_t)end);
-    cudaFreeAsync(lut, s);
+    void* ws = nullptr;
+    HK_CUDA(lib_malloc(&ws, tpacf_ws_bytes(*a), s), "alloc tpacf workspace");
+    cudaError_t e = tpacf_launch(vf, *a, R, ndet, d_cb, nullptr, ws, s, (int32_t)begin, (int32_t)end);
+    cudaFreeAsync(ws, s);
     HK_CUDA(e, "tpacf kernel");
   }
   return HK_OK;
@@ -533,8 +648,8 @@ hk_status hauberk_profile_ranges(int32_t bench, const void* args, const hk_profi
   const int64_t T = bench_threads(bench, args);
   float* d_samples = nullptr;
   hk_control* d_cb = nullptr;
-  HK_CUDA(cudaMallocAsync((void**)&d_samples, sizeof(float) * std::max<int64_t>(1, T * maxvar), s), "alloc samples");
-  HK_CUDA(cudaMallocAsync((void**)&d_cb, sizeof(hk_control), s), "alloc cb");
+  HK_CUDA(lib_malloc((void**)&d_samples, sizeof(float) * std::max<int64_t>(1, T * maxvar), s), "alloc samples");
+  HK_CUDA(lib_malloc((void**)&d_cb, sizeof(hk_control), s), "alloc cb");
   hk_ranges pr{};
   pr.n_det = maxvar;
   pr.alpha = 1.f;
@@ -584,8 +699,9 @@ hk_status hauberk_profile_search(const float* samples, int64_t n, int32_t t0_exp
 }
 
 hk_status hauberk_decode(int32_t bench_mode, const void* const args[3], const uint64_t site_mask[3], uint64_t seed,
-                         int32_t nbits, int64_t first, int64_t count, int32_t* bench_out, hk_fault* out) {
-  if (!args || !site_mask || !bench_out || !out || count < 0 || first < 0 || bench_mode < -1 || bench_mode > 2)
+                         int32_t nbits, int32_t variant, int64_t first, int64_t count, int32_t* bench_out, hk_fault* out) {
+  if (!args || !site_mask || !bench_out || !out || count < 0 || first < 0 || bench_mode < -1 || bench_mode > 2 ||
+      variant < 0 || variant > 1)
     return invalid("decode: bad arguments");
   Catalog K[3];
   bool have[3] = {false, false, false};
@@ -594,7 +710,7 @@ hk_status hauberk_decode(int32_t bench_mode, const void* const args[3], const ui
     const int b = bench_mode >= 0 ? bench_mode : (int)(n % 3);
     if (!have[b]) {
       if (!args_ok(b, args[b])) return invalid("decode: args of a used benchmark are invalid");
-      if (!build_catalog(K[b], b, args[b], site_mask[b])) return invalid("decode: empty site catalogue");
+      if (!build_catalog(K[b], b, args[b], site_mask[b], variant)) return invalid("decode: empty site catalogue");
       have[b] = true;
     }
     bench_out[q] = b;
@@ -663,24 +779,14 @@ static void session_free(hk_campaign_session* S) {
   delete S;
 }
 
-static void keep_pool_memory() {
-  static bool done = false;
-  if (done) return;
-  int dev = 0;
-  cudaMemPool_t pool;
-  if (cudaGetDevice(&dev) == cudaSuccess && cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
-    uint64_t thr = UINT64_MAX;
-    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
-  }
-  done = true;
-}
-
 static hk_status session_create(int32_t bench_mode, const void* const args[3], const hk_ranges* const ranges[3],
                                 const hk_campaign* C, cudaStream_t s, hk_campaign_session** out) {
   if (!args || !ranges || !C || !out || bench_mode < -1 || bench_mode > 2) return invalid("campaign: bad arguments");
   if (C->mode < 0 || C->mode > 2) return invalid("campaign: mode must be 0 (replica), 1 (replay) or 2 (unguarded replica)");
   if (C->nbits < 0 || C->nbits > 64) return invalid("campaign: nbits out of range");
-  keep_pool_memory();
+  if (C->variant != HK_FIFT && C->variant != HK_FI_ONLY) return invalid("campaign: variant must be HK_FIFT or HK_FI_ONLY");
+  if (C->hang_factor < 0) return invalid("campaign: hang_factor must be >= 0 (0 = the paper's 10)");
+  const bool ft = C->variant == HK_FIFT;
   hk_campaign_session* S = new hk_campaign_session();
   S->bench_mode = bench_mode;
   S->cfg = *C;
@@ -695,7 +801,7 @@ static hk_status session_create(int32_t bench_mode, const void* const args[3], c
     const bool want = bench_mode == b || (bench_mode == -1 && args[b] != nullptr);
     if (!want) continue;
     if (!args_ok(b, args[b])) { st = invalid("campaign: args of a used benchmark are invalid"); break; }
-    if (!ranges[b] || ranges[b]->n_det <= 0) { g_err = "campaign: ranges missing"; st = HK_ERR_NO_RANGES; break; }
+    if (ft && (!ranges[b] || ranges[b]->n_det <= 0)) { g_err = "campaign: ranges missing"; st = HK_ERR_NO_RANGES; break; }
     if (b == HK_CP && ((const hk_cp_args*)args[b])->unroll != 4 && ((const hk_cp_args*)args[b])->unroll != 8) {
       g_err = "campaign kernels are built for CP unroll 4 and 8"; st = HK_ERR_UNSUPPORTED; break;
     }
@@ -704,12 +810,12 @@ static hk_status session_create(int32_t bench_mode, const void* const args[3], c
     if (b == HK_CP) S->cp = *(const hk_cp_args*)args[b];
     else if (b == HK_MRIQ) S->mq = *(const hk_mriq_args*)args[b];
     else S->tp = *(const hk_tpacf_args*)args[b];
-    if (!build_catalog(S->K[b], b, own, C->site_mask[b])) { st = invalid("campaign: empty site catalogue"); break; }
+    if (!build_catalog(S->K[b], b, own, C->site_mask[b], C->variant)) { st = invalid("campaign: empty site catalogue"); break; }
     BenchWS& w = S->W[b];
     w.used = true;
     w.args = own;
-    w.R = dev_ranges(ranges[b]);
-    w.ndet = ranges[b]->n_det;
+    w.R = dev_ranges(ft ? ranges[b] : nullptr);  // the FI-only binary has no detectors
+    w.ndet = ft ? ranges[b]->n_det : 0;
     w.batch = C->mode == 1 ? 1 : (C->batch > 0 ? C->batch : default_batch(b, own));
     if (C->mode == 1 && b == HK_TPACF && 3 * S->tp.n_bins > 96) { g_err = "replay supports n_bins <= 32"; st = HK_ERR_UNSUPPORTED; break; }
     const bool phimag_sites = b == HK_MRIQ && (C->site_mask[b] >> MRIQ_PHIMAG_SITE0) != 0;
@@ -740,23 +846,25 @@ static hk_status session_create(int32_t bench_mode, const void* const args[3], c
       st = cuda_fail(e, "campaign init");
       break;
     }
-    // golden = this library's own fault-free FT output (R7)
+    // golden = this library's own fault-free output of the same binary (R7): FT, or BASE for FI-only
+    const int gv = ft ? HK_FT : HK_BASE;
+    const hk_ranges* gr = ft ? ranges[b] : nullptr;
     if (b == HK_CP) {
       hk_cp_args a = S->cp;
       a.grid = (float*)w.golden;
-      st = run_bench(b, &a, HK_FT, ranges[b], w.gold_cb, nullptr, s);
+      st = run_bench(b, &a, gv, gr, w.gold_cb, nullptr, s);
       if (st == HK_OK && (e = max_abs_launch((float*)w.golden, (int64_t)a.nx * a.ny, w.dM, s)) != cudaSuccess) st = cuda_fail(e, "max");
     } else if (b == HK_MRIQ) {
       hk_mriq_args a = S->mq;
       a.qr = (float*)w.golden;
       a.qi = a.qr + a.n_vox;
-      st = run_bench(b, &a, HK_FT, ranges[b], w.gold_cb, nullptr, s);
+      st = run_bench(b, &a, gv, gr, w.gold_cb, nullptr, s);
       if (st == HK_OK && (e = max_abs_launch((float*)w.golden, 2LL * a.n_vox, w.dM, s)) != cudaSuccess) st = cuda_fail(e, "max");
     } else {
       hk_tpacf_args a = S->tp;
       a.hist = (unsigned long long*)w.golden;
-      st = run_bench(b, &a, HK_FT, ranges[b], w.gold_cb, nullptr, s);
-      if (st == HK_OK && (e = cudaMalloc(&w.lut, tpacf_lut_ws_bytes())) != cudaSuccess) st = cuda_fail(e, "alloc table");
+      st = run_bench(b, &a, gv, gr, w.gold_cb, nullptr, s);
+      if (st == HK_OK && (e = cudaMalloc(&w.lut, tpacf_ws_bytes(a))) != cudaSuccess) st = cuda_fail(e, "alloc table");
       if (st == HK_OK && (e = tpacf_lut_build(a, w.lut, s)) != cudaSuccess) st = cuda_fail(e, "table");
     }
   }
@@ -828,12 +936,12 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
       if (S->d_decode) cudaFreeAsync(S->d_decode, s);
       S->d_decode = nullptr;
       S->decode_cap = 0;
-      if ((e = cudaMallocAsync(&S->d_decode, need, s)) != cudaSuccess) return cuda_fail(e, "decode workspace");
+      if ((e = lib_malloc(&S->d_decode, need, s)) != cudaSuccess) return cuda_fail(e, "decode workspace");
       S->decode_cap = need;
     }
     FaultRec* sorted = nullptr;
-    if ((e = decode_sort_launch(S->dcat, S->cfg.seed, first, count, S->bench_mode, S->cfg.nbits, S->d_decode, &sorted, s)) !=
-        cudaSuccess)
+    if ((e = decode_sort_launch(S->dcat, S->cfg.seed, first, count, S->bench_mode, S->cfg.nbits, S->cfg.hang_factor,
+                                S->d_decode, &sorted, s)) != cudaSuccess)
       return cuda_fail(e, "device decode");
     int64_t off = 0;
     for (int b = 0; b < 3; ++b) {
@@ -841,11 +949,12 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
       BenchWS& w = S->W[b];
       const FaultRec* fr = sorted + off;
       const int nrep = (int)per[b];
-      if (b == HK_CP) e = cp_replay_launch(0, S->cp, w.R, std::min(w.ndet, S->cp.unroll), fr, nrep, (const float*)w.golden,
+      const bool ft = S->cfg.variant == HK_FIFT;
+      if (b == HK_CP) e = cp_replay_launch(0, ft, S->cp, w.R, std::min(w.ndet, S->cp.unroll), fr, nrep, (const float*)w.golden,
                                            w.dM, d_records, first, d_counts, d_site_counts, s);
-      else if (b == HK_MRIQ) e = mriq_replay_launch(0, S->mq, w.R, std::min(w.ndet, 2), fr, nrep, (const float*)w.golden,
+      else if (b == HK_MRIQ) e = mriq_replay_launch(0, ft, S->mq, w.R, std::min(w.ndet, 2), fr, nrep, (const float*)w.golden,
                                                     w.dM, d_records, first, d_counts, d_site_counts, s);
-      else e = tpacf_replay_launch(0, S->tp, w.R, std::min(w.ndet, 1), fr, nrep, (const unsigned long long*)w.golden,
+      else e = tpacf_replay_launch(0, ft, S->tp, w.R, std::min(w.ndet, 1), fr, nrep, (const unsigned long long*)w.golden,
                                    d_records, first, d_counts, d_site_counts, s);
       if (e != cudaSuccess) return cuda_fail(e, "replay");
       off += per[b];
@@ -869,7 +978,7 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
     else it.kind = tpacf_site_kind(hf.site);
     it.f.sub = sub;
     it.f.real = S->cfg.mode == 2 ? 1 : 0;  // R25: guardian child processes only
-    it.f.pad_ = 0;
+    it.f.hang = S->cfg.hang_factor;
     items[(size_t)q] = it;
   }
   std::stable_sort(items.begin(), items.end(), [](const Item& x, const Item& y) {
@@ -888,7 +997,7 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
     if (S->d_faults) cudaFreeAsync(S->d_faults, s);
     S->d_faults = nullptr;
     S->d_cap = 0;
-    if ((e = cudaMallocAsync((void**)&S->d_faults, sizeof(FaultRec) * items.size(), s)) != cudaSuccess) return cuda_fail(e, "faults");
+    if ((e = lib_malloc((void**)&S->d_faults, sizeof(FaultRec) * items.size(), s)) != cudaSuccess) return cuda_fail(e, "faults");
     S->d_cap = items.size();
   }
   for (size_t q = 0; q < items.size(); ++q) S->h_faults[q] = items[q].f;
@@ -898,6 +1007,7 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
 
   // ---- batches: FI&FT replicas, then the classify epilogue (which also recycles the workspace)
   const bool real = S->cfg.mode == 2;  // R25: unguarded replicas (guardian child processes only)
+  const bool ft = S->cfg.variant == HK_FIFT;
   const cudaStream_t s0 = s;
   bool touched[3] = {false, false, false};
   for (const Item& it : items) touched[it.b] = true;
@@ -932,21 +1042,21 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
     BenchWS& w = S->W[b];
     const FaultRec* fr = S->d_faults + q;
     if (b == HK_CP) {
-      if ((e = cp_fi_launch(kind, S->cp, w.R, std::min(w.ndet, S->cp.unroll), fr, nrep, (float*)w.rep_out, w.out_elems, w.rep_cb,
+      if ((e = cp_fi_launch(kind, ft, S->cp, w.R, std::min(w.ndet, S->cp.unroll), fr, nrep, (float*)w.rep_out, w.out_elems, w.rep_cb,
                             real, s)) != cudaSuccess)
         return cuda_fail(e, "cp FI");
       if ((e = classify_fp_launch(b, (float*)w.rep_out, w.out_elems, (const float*)w.golden, w.dM, w.rep_cb, fr, nrep,
                                   d_records, first, d_counts, d_site_counts, s)) != cudaSuccess)
         return cuda_fail(e, "classify");
     } else if (b == HK_MRIQ) {
-      if ((e = mriq_fi_launch(kind, S->mq, w.R, std::min(w.ndet, 2), fr, nrep, (float*)w.rep_out, w.out_elems, w.rep_cb,
+      if ((e = mriq_fi_launch(kind, ft, S->mq, w.R, std::min(w.ndet, 2), fr, nrep, (float*)w.rep_out, w.out_elems, w.rep_cb,
                               w.kv_rep, real, s)) != cudaSuccess)
         return cuda_fail(e, "mriq FI");
       if ((e = classify_fp_launch(b, (float*)w.rep_out, w.out_elems, (const float*)w.golden, w.dM, w.rep_cb, fr, nrep,
                                   d_records, first, d_counts, d_site_counts, s)) != cudaSuccess)
         return cuda_fail(e, "classify");
     } else {
-      if ((e = tpacf_fi_launch(kind, S->tp, w.R, std::min(w.ndet, 1), fr, nrep, (unsigned long long*)w.rep_out, w.rep_cb,
+      if ((e = tpacf_fi_launch(kind, ft, S->tp, w.R, std::min(w.ndet, 1), fr, nrep, (unsigned long long*)w.rep_out, w.rep_cb,
                                w.lut, real, s)) != cudaSuccess)
         return cuda_fail(e, "tpacf FI");
       if ((e = classify_tpacf_launch((unsigned long long*)w.rep_out, S->tp.n_rand, S->tp.n_bins,
@@ -978,6 +1088,26 @@ hk_status hauberk_campaign_run(hk_campaign_session* session, int64_t first, int6
 }
 
 void hauberk_campaign_destroy(hk_campaign_session* session) { session_free(session); }
+
+size_t hauberk_campaign_workspace_bytes(int32_t bench, const void* args, const hk_campaign* C) {
+  if (bench < 0 || bench > 2 || !C || !args_ok(bench, args) || C->mode < 0 || C->mode > 2) return 0;
+  const int batch = C->mode == 1 ? 1 : (C->batch > 0 ? C->batch : default_batch(bench, args));
+  size_t esz = sizeof(float);
+  int64_t elems = 0;
+  if (bench == HK_CP) elems = (int64_t)((const hk_cp_args*)args)->nx * ((const hk_cp_args*)args)->ny;
+  else if (bench == HK_MRIQ) elems = 2LL * ((const hk_mriq_args*)args)->n_vox;
+  else {
+    const hk_tpacf_args* a = (const hk_tpacf_args*)args;
+    elems = (int64_t)(1 + 2 * a->n_rand) * (a->n_bins + 2);
+    esz = 8;
+  }
+  const size_t stride = (size_t)((elems + 3) / 4 * 4);
+  size_t bytes = esz * stride * (1 + (size_t)batch) + sizeof(float) + sizeof(hk_control) * (1 + (size_t)batch);
+  if (bench == HK_TPACF) bytes += tpacf_ws_bytes(*(const hk_tpacf_args*)args);
+  if (bench == HK_MRIQ && (C->site_mask[HK_MRIQ] >> MRIQ_PHIMAG_SITE0) != 0)
+    bytes += sizeof(float4) * (size_t)std::max(1, ((const hk_mriq_args*)args)->n_k) * batch;
+  return bytes;
+}
 
 hk_status hauberk_inject_campaign(int32_t bench_mode, const void* const args[3], const hk_ranges* const ranges[3],
                                   const hk_campaign* C, hk_outcome* d_records, int64_t* d_counts, int64_t* d_site_counts,

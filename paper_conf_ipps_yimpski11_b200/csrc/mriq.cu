@@ -242,7 +242,8 @@ struct MQFIParams {
 // Per-thread FI&FT program of voxel t.  t_dup: the duplicate of N0 recomputed from launch indices
 // (replica) or from the abstract id (replay); qr_real / qi_real: the buffers' true base addresses.
 // REAL: the guardian's unguarded variant (R25) — no R16 guards, no R17 watchdog.
-template <int KIND, bool EXACT, bool REAL = false, class Sink>
+// FT = false: the FI-only binary (row a7): no counter, no checks.
+template <int KIND, bool EXACT, bool REAL = false, bool FT = true, class Sink>
 __device__ void mriq_fi_program(const MQParams& p, const FaultRec& f, int32_t t, int32_t t_dup, bool mine,
                                 uint64_t qr_real, uint64_t qi_real, Sink& S) {
   const int64_t inst = mine ? f.inst : -1;
@@ -267,7 +268,7 @@ __device__ void mriq_fi_program(const MQParams& p, const FaultRec& f, int32_t t,
   int32_t it = 0, k = 0;
   const float* pe;
   float* po;
-  const int64_t limit = fi_limit<REAL>(nk);
+  const int64_t limit = fi_limit<REAL>(nk, f.hang);
   constexpr bool real = REAL;
   if (!fi_at(real, px, x_real, xIndex, nv, &pe)) { fail |= FL_CRASH; goto done; }
   sX = __ldg(pe);
@@ -332,12 +333,12 @@ __device__ void mriq_fi_program(const MQParams& p, const FaultRec& f, int32_t t,
       Qi = __fmaf_rn(k4.w, s, Qi);
       if (KIND == MK_QI) { applied |= now; Qi = flip_f(Qi, now, mask); }
     }
-    it = count_inc(it, p.one);
+    if (FT) it = count_inc(it, p.one);
     if (KIND == MK_IT) { applied |= now; it = flip_i(it, now, mask); }
     k = (int32_t)((uint32_t)k + 1u);
   }
-  if (it != numK) alarm |= AL_COUNT;
-  if (it != 0) {
+  if (FT && it != numK) alarm |= AL_COUNT;
+  if (FT && it != 0) {
     const float fit = (float)it;
 #pragma unroll
     for (int d = 0; d < 2; ++d) {
@@ -357,6 +358,7 @@ __device__ void mriq_fi_program(const MQParams& p, const FaultRec& f, int32_t t,
          (lohi(pz) + z);
   if (chk != 0) alarm |= AL_CHK;
 done:
+  if (!FT) alarm = 0;
   S.finish(mine, alarm, fail, margin, gap, domain, applied, (uint32_t)t);
 }
 
@@ -366,7 +368,8 @@ done:
 __global__ void __launch_bounds__(256) mriq_phimag_fi_kernel(const float* __restrict__ kx, const float* __restrict__ ky,
                                                             const float* __restrict__ kz, const float* __restrict__ pr,
                                                             const float* __restrict__ pi, float4* kv0, int numK,
-                                                            const FaultRec* faults, hk_control* cb0, uint32_t z) {
+                                                            const FaultRec* faults, hk_control* cb0, uint32_t z,
+                                                            bool ft) {
   const int r = blockIdx.y;
   const FaultRec f = faults[r];
   float* kv = reinterpret_cast<float*>(kv0 + (int64_t)r * numK);
@@ -413,13 +416,13 @@ __global__ void __launch_bounds__(256) mriq_phimag_fi_kernel(const float* __rest
 done:
   if (fail) atomicOr(&cb->fail, fail);
   if (mine) cb->fault_applied = 1u;
-  fold_alarm(cb, alarm, (uint32_t)k);
+  if (ft) fold_alarm(cb, alarm, (uint32_t)k);  // the FI-only binary has no detectors
 }
 
 // Items L = (replica, CTA) in fi_order; by default one per CTA of a (ncta, nrep) grid.  With
 // HK_MQ_FI_PERSIST = c the grid holds c CTAs per SM that walk the items (experiment: leaves room
 // for TPACF replica CTAs on the same SMs); the k-space mbarriers are invalidated between items.
-template <int KIND, bool EXACT>
+template <int KIND, bool EXACT, bool FT>
 __global__ void __launch_bounds__(MQ_FI_THREADS) mriq_fi_kernel(const MQFIParams q) {
   __shared__ __align__(128) float4 tile[2][MQ_FI_TILE];
   __shared__ __align__(8) uint64_t bar[2];
@@ -437,7 +440,7 @@ __global__ void __launch_bounds__(MQ_FI_THREADS) mriq_fi_kernel(const MQFIParams
     p.cb = q.cb0 + r;
     if (KIND == MK_PHIMAG) p.kv = q.kv0 + (int64_t)r * p.numK;  // this replica's (possibly faulted) k-space
     if (KIND == MK_PHIMAG || !faulted) {
-      mriq_body<V_NL | V_L, EXACT, true, MQ_FI_VPT, MQ_FI_UNROLL, MQ_FI_TILE>(p, tile, bar, bxi);
+      mriq_body<FT ? (V_NL | V_L) : 0, EXACT, true, MQ_FI_VPT, MQ_FI_UNROLL, MQ_FI_TILE>(p, tile, bar, bxi);
       if (L + step < total) {  // next item re-initialises the barriers
         __syncthreads();
         if (threadIdx.x == 0) {
@@ -453,7 +456,7 @@ __global__ void __launch_bounds__(MQ_FI_THREADS) mriq_fi_kernel(const MQFIParams
         const int32_t t = bxi * (MQ_FI_VPT * blockDim.x) + vox * blockDim.x + threadIdx.x;
         if (t < p.numX) {
           const int32_t t_dup = (int32_t)((bxi ^ p.zz) * (MQ_FI_VPT * blockDim.x) + vox * blockDim.x + (threadIdx.x ^ p.zz));
-          mriq_fi_program<KIND, EXACT>(p, f, t, t_dup, t == f.thread, (uint64_t)(uintptr_t)p.qr, (uint64_t)(uintptr_t)p.qi, S);
+          mriq_fi_program<KIND, EXACT, false, FT>(p, f, t, t_dup, t == f.thread, (uint64_t)(uintptr_t)p.qr, (uint64_t)(uintptr_t)p.qi, S);
         }
       }
     }
@@ -500,13 +503,13 @@ struct MQReplayParams {
   int64_t* site_counts;
 };
 
-template <int KIND, bool EXACT>
+template <int KIND, bool EXACT, bool FT>
 __device__ __forceinline__ void mriq_replay_one(const MQReplayParams& q, const FaultRec& f) {
   const MQParams& p = q.base;
   const int32_t t = (int32_t)f.thread;
   ReplaySinkF<2> S;
   const uint64_t base_real = (uint64_t)(uintptr_t)q.golden;
-  mriq_fi_program<KIND, EXACT>(p, f, t, opq(t, p.zz), true, base_real, base_real + 4ull * (uint64_t)p.numX, S);
+  mriq_fi_program<KIND, EXACT, false, FT>(p, f, t, opq(t, p.zz), true, base_real, base_real + 4ull * (uint64_t)p.numX, S);
   bool wrong = false;
   float worst = 0.f;
   if (!S.fail) {
@@ -532,13 +535,13 @@ __device__ __forceinline__ void mriq_replay_one(const MQReplayParams& q, const F
                q.site_counts);
 }
 
-template <bool EXACT>
+template <bool EXACT, bool FT>
 __global__ void __launch_bounds__(128) mriq_replay_all_kernel(const MQReplayParams q) {
   const int r = blockIdx.x * blockDim.x + threadIdx.x;
   if (r >= q.nrep) return;
   const FaultRec f = q.faults[r];
   switch (mriq_site_kind_d(f.site)) {
-#define K(k) case k: mriq_replay_one<k, EXACT>(q, f); break;
+#define K(k) case k: mriq_replay_one<k, EXACT, FT>(q, f); break;
     K(MK_NL) K(MK_LIVE) K(MK_K) K(MK_KX) K(MK_KY) K(MK_KZ) K(MK_PM) K(MK_T1) K(MK_T2) K(MK_T) K(MK_R) K(MK_C) K(MK_S)
     K(MK_QR) K(MK_QI) K(MK_IT)
 #undef K
@@ -599,7 +602,7 @@ cudaError_t mriq_launch(int vflags, const hk_mriq_args& a, const DevRanges& R, i
 
 int mriq_site_kind(int site) { return mriq_site_kind_d(site); }
 
-template <int KIND, bool EXACT>
+template <int KIND, bool EXACT, bool FT>
 static cudaError_t launch_mq_fi_k(const MQFIParams& q, int nrep, cudaStream_t s) {
   constexpr int vpc = MQ_FI_VPT * MQ_FI_THREADS;
   dim3 grid((q.base.numX + vpc - 1) / vpc, nrep);
@@ -612,15 +615,15 @@ static cudaError_t launch_mq_fi_k(const MQFIParams& q, int nrep, cudaStream_t s)
     if (items > cap) grid = dim3((unsigned)cap, 1);
   }
   TimedScope ts(HK_MRIQ, 1, (double)q.base.numX * (double)q.base.numK * nrep, s);
-  mriq_fi_kernel<KIND, EXACT><<<grid, MQ_FI_THREADS, 0, s>>>(q);
+  mriq_fi_kernel<KIND, EXACT, FT><<<grid, MQ_FI_THREADS, 0, s>>>(q);
   count_launch();
   return cudaGetLastError();
 }
 
-template <bool EXACT>
+template <bool EXACT, bool FT>
 static cudaError_t launch_mq_fi_e(int kind, const MQFIParams& q, int nrep, cudaStream_t s) {
   switch (kind) {
-#define K(k) case k: return launch_mq_fi_k<k, EXACT>(q, nrep, s);
+#define K(k) case k: return launch_mq_fi_k<k, EXACT, FT>(q, nrep, s);
     K(MK_NL) K(MK_LIVE) K(MK_K) K(MK_KX) K(MK_KY) K(MK_KZ) K(MK_PM) K(MK_T1) K(MK_T2) K(MK_T) K(MK_R) K(MK_C) K(MK_S)
     K(MK_QR) K(MK_QI) K(MK_IT) K(MK_PHIMAG)
 #undef K
@@ -628,7 +631,7 @@ static cudaError_t launch_mq_fi_e(int kind, const MQFIParams& q, int nrep, cudaS
   return cudaErrorInvalidValue;
 }
 
-cudaError_t mriq_replay_launch(int kind, const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
+cudaError_t mriq_replay_launch(int kind, bool ft, const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults,
                                int nrep, const float* golden, const float* dM, hk_outcome* records, int64_t first,
                                int64_t* counts, int64_t* site_counts, cudaStream_t s) {
   if (nrep <= 0) return cudaSuccess;
@@ -640,20 +643,20 @@ cudaError_t mriq_replay_launch(int kind, const hk_mriq_args& a, const DevRanges&
   (void)kind;
   TimedScope ts(HK_MRIQ, 2, (double)a.n_k * nrep, s);
   const unsigned g = (unsigned)((nrep + 127) / 128);
-  if (a.exact) mriq_replay_all_kernel<true><<<g, 128, 0, s>>>(q);
-  else mriq_replay_all_kernel<false><<<g, 128, 0, s>>>(q);
+  if (a.exact) ft ? mriq_replay_all_kernel<true, true><<<g, 128, 0, s>>>(q) : mriq_replay_all_kernel<true, false><<<g, 128, 0, s>>>(q);
+  else ft ? mriq_replay_all_kernel<false, true><<<g, 128, 0, s>>>(q) : mriq_replay_all_kernel<false, false><<<g, 128, 0, s>>>(q);
   count_launch();
   return cudaGetLastError();
 }
 
-cudaError_t mriq_fi_launch(int kind, const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
+cudaError_t mriq_fi_launch(int kind, bool ft, const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
                            float* out0, int64_t stride, hk_control* cb0, float4* kv_rep, bool real, cudaStream_t s) {
   if (kind == MK_PHIMAG) {
     if (!kv_rep) return cudaErrorInvalidValue;
     cudaError_t e = cudaMemsetAsync(kv_rep, 0, sizeof(float4) * (size_t)a.n_k * nrep, s);
     if (e != cudaSuccess) return e;
     dim3 g((a.n_k + 255) / 256, nrep);
-    mriq_phimag_fi_kernel<<<g, 256, 0, s>>>(a.kx, a.ky, a.kz, a.phi_r, a.phi_i, kv_rep, a.n_k, faults, cb0, opaque_zero());
+    mriq_phimag_fi_kernel<<<g, 256, 0, s>>>(a.kx, a.ky, a.kz, a.phi_r, a.phi_i, kv_rep, a.n_k, faults, cb0, opaque_zero(), ft);
     count_launch();
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
   }
@@ -673,7 +676,8 @@ cudaError_t mriq_fi_launch(int kind, const hk_mriq_args& a, const DevRanges& R, 
     count_launch();
     return cudaGetLastError();
   }
-  return a.exact ? launch_mq_fi_e<true>(kind, q, nrep, s) : launch_mq_fi_e<false>(kind, q, nrep, s);
+  if (ft) return a.exact ? launch_mq_fi_e<true, true>(kind, q, nrep, s) : launch_mq_fi_e<false, true>(kind, q, nrep, s);
+  return a.exact ? launch_mq_fi_e<true, false>(kind, q, nrep, s) : launch_mq_fi_e<false, false>(kind, q, nrep, s);
 }
 
 }  // namespace hk

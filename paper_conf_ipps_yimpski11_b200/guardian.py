@@ -62,7 +62,7 @@ def write_blob(path: str, bench: int, problem, ranges, seed: int, site_mask: int
     elif bench == TPACF:
         p = problem
         arrays = [_f32(p.pts), _f32(p.edges)]
-        iargs[:4] = [p.n, p.n_rand, p.edges.size - 1, p.chunk]
+        iargs[:3] = [p.n, p.n_rand, p.edges.size - 1]
     else:
         raise ValueError(f"bad bench {bench}")
     with open(path, "wb") as f:

@@ -69,7 +69,7 @@ class MRIQArgs(C.Structure):
 
 class TPACFArgs(C.Structure):
     _fields_ = [("pts", C.c_void_p), ("edges", C.c_void_p), ("n", C.c_int32), ("n_rand", C.c_int32),
-                ("n_bins", C.c_int32), ("chunk", C.c_int32), ("hist", C.c_void_p)]
+                ("n_bins", C.c_int32), ("hist", C.c_void_p)]
 
 
 class ProfileOpts(C.Structure):
@@ -78,11 +78,20 @@ class ProfileOpts(C.Structure):
 
 class Campaign(C.Structure):
     _fields_ = [("seed", C.c_uint64), ("first", C.c_int64), ("count", C.c_int64), ("nbits", C.c_int32),
-                ("mode", C.c_int32), ("batch", C.c_int32), ("exact", C.c_int32), ("site_mask", C.c_uint64 * 3)]
+                ("mode", C.c_int32), ("batch", C.c_int32), ("exact", C.c_int32), ("site_mask", C.c_uint64 * 3),
+                ("variant", C.c_int32), ("hang_factor", C.c_int32)]
+
+
+HK_FIFT, HK_FI_ONLY = 0, 1  # hk_campaign.variant: FI&FT binary / FI-only binary (row a7)
 
 
 class Fault(C.Structure):
-    _fields_ = [("site", C.c_int32), ("pad", C.c_int32), ("thread", C.c_int64), ("inst", C.c_int64), ("mask", C.c_uint64)]
+    _fields_ = [("site", C.c_int32), ("hang", C.c_int32), ("thread", C.c_int64), ("inst", C.c_int64), ("mask", C.c_uint64)]
+
+
+class Summary(C.Structure):
+    _fields_ = [("coverage", C.c_double), ("sdc", C.c_double), ("detected", C.c_double), ("failure", C.c_double),
+                ("total", C.c_int64)]
 
 
 OUTCOME_DTYPE = np.dtype([("index", "<i8"), ("bench", "<i4"), ("site", "<i4"), ("thread", "<i8"), ("inst", "<i8"),
@@ -109,7 +118,7 @@ def lib():
         L.hauberk_inject_campaign.restype = I32
         L.hauberk_inject_campaign.argtypes = [I32, P, P, P, P, P, P, P]
         L.hauberk_decode.restype = I32
-        L.hauberk_decode.argtypes = [I32, P, P, U64, I32, I64, I64, P, P]
+        L.hauberk_decode.argtypes = [I32, P, P, U64, I32, I32, I64, I64, P, P]
         L.hauberk_num_sites.restype = I32
         L.hauberk_num_sites.argtypes = [I32, I32]
         L.hauberk_strerror.restype = C.c_char_p
@@ -136,6 +145,22 @@ def lib():
         L.hauberk_compare.argtypes = [P, P, I64, P, P]
         L.hauberk_run_part.restype = I32
         L.hauberk_run_part.argtypes = [I32, P, I32, P, P, I64, I64, P]
+        L.hauberk_detector_site.restype = I32
+        L.hauberk_detector_site.argtypes = [I32, I32, I32]
+        L.hauberk_campaign_workspace_bytes.restype = C.c_size_t
+        L.hauberk_campaign_workspace_bytes.argtypes = [I32, P, P]
+        L.hauberk_summarize.restype = I32
+        L.hauberk_summarize.argtypes = [P, P]
+        L.hauberk_extend_ranges.restype = I32
+        L.hauberk_extend_ranges.argtypes = [P, P, I32, P]
+        L.hauberk_outliers.restype = I32
+        L.hauberk_outliers.argtypes = [P, I32, P, P]
+        L.hauberk_alpha_update.restype = C.c_float
+        L.hauberk_alpha_update.argtypes = [C.c_float, C.c_double, C.c_double, C.c_double]
+        L.hauberk_diagnose.restype = I32
+        L.hauberk_diagnose.argtypes = [C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32, I32]
+        L.hauberk_release_caches.restype = None
+        L.hauberk_release_caches.argtypes = []
         _lib = L
     return _lib
 
@@ -144,7 +169,9 @@ EXPORTED = ["hauberk_run_cp", "hauberk_run_mriq", "hauberk_run_tpacf", "hauberk_
             "hauberk_inject_campaign", "hauberk_decode", "hauberk_num_sites", "hauberk_strerror",
             "hauberk_last_error", "hauberk_version", "hauberk_launch_count", "hauberk_timing_enable",
             "hauberk_timing_read", "hauberk_campaign_create", "hauberk_campaign_run", "hauberk_campaign_destroy",
-            "hauberk_profile_search", "hauberk_part_units", "hauberk_run_part", "hauberk_compare"]
+            "hauberk_profile_search", "hauberk_part_units", "hauberk_run_part", "hauberk_compare",
+            "hauberk_detector_site", "hauberk_campaign_workspace_bytes", "hauberk_summarize", "hauberk_extend_ranges",
+            "hauberk_outliers", "hauberk_alpha_update", "hauberk_diagnose", "hauberk_release_caches"]
 
 
 def _check(status: int, where: str):
@@ -290,22 +317,20 @@ class TPACFDevice:
     n: int
     n_rand: int
     n_bins: int
-    chunk: int
     bench = HK_TPACF
 
     @classmethod
     def from_problem(cls, p, device="cuda", exact: int = 0):
         return cls(pts=_dev(p.pts.astype(np.float32), device), edges=_dev(p.edges.astype(np.float32), device),
                    hist=torch.empty((1 + 2 * p.n_rand, p.n_bins + 2), dtype=torch.int64, device=device),
-                   n=p.n, n_rand=p.n_rand, n_bins=p.n_bins, chunk=p.chunk)
+                   n=p.n, n_rand=p.n_rand, n_bins=p.n_bins)
 
     def args(self) -> TPACFArgs:
-        return TPACFArgs(_ptr(self.pts), _ptr(self.edges), self.n, self.n_rand, self.n_bins, self.chunk, _ptr(self.hist))
+        return TPACFArgs(_ptr(self.pts), _ptr(self.edges), self.n, self.n_rand, self.n_bins, _ptr(self.hist))
 
     @property
     def n_threads(self) -> int:
-        nc = (self.n + self.chunk - 1) // self.chunk
-        return (1 + 2 * self.n_rand) * nc * self.n
+        return (1 + 2 * self.n_rand) * self.n  # abstract thread g = h * n + i
 
     def output(self):
         return self.hist
@@ -394,16 +419,32 @@ def _arg_array(devs):
     return arr, structs
 
 
+def _check_campaign_buffers(count: int, counts: torch.Tensor, records, site_counts):
+    """The library writes counts[bench*5 + cls], site_counts[(bench*64 + site)*5 + cls] (u64 atomics)
+    and records[n - first]: reject buffers that would be written out of bounds."""
+    if not (isinstance(counts, torch.Tensor) and counts.is_cuda and counts.dtype == torch.int64
+            and counts.is_contiguous() and counts.numel() == 15):
+        raise ValueError("counts must be a contiguous int64 CUDA tensor of 15 elements ([3, 5])")
+    if site_counts is not None and not (site_counts.is_cuda and site_counts.dtype == torch.int64
+                                        and site_counts.is_contiguous() and site_counts.numel() == 3 * 64 * 5):
+        raise ValueError("site_counts must be a contiguous int64 CUDA tensor of 3*64*5 elements")
+    if records is not None and not (records.is_cuda and records.is_contiguous()
+                                    and records.numel() * records.element_size() >= count * OUTCOME_DTYPE.itemsize):
+        raise ValueError(f"records must be a contiguous CUDA tensor of >= {count} x {OUTCOME_DTYPE.itemsize} bytes")
+
+
 def inject_campaign(bench_mode: int, devs, ranges, seed: int, first: int, count: int, counts: torch.Tensor,
                     records: torch.Tensor | None = None, site_counts: torch.Tensor | None = None, exact: int = 0,
-                    batch: int = 0, site_masks=DEFAULT_SITE_MASKS, stream=None, nbits: int = 1, mode: int = 0):
-    """hauberk_inject_campaign (replica mode).  devs/ranges: 3-lists by bench (None where unused).
-    counts: int64 cuda tensor [3, 5] (accumulated); records: optional uint8 tensor of
-    count * OUTCOME_DTYPE.itemsize bytes; site_counts: optional int64 [3, 64, 5]."""
+                    batch: int = 0, site_masks=DEFAULT_SITE_MASKS, stream=None, nbits: int = 1, mode: int = 0,
+                    variant: int = HK_FIFT, hang_factor: int = 0):
+    """hauberk_inject_campaign.  devs/ranges: 3-lists by bench (None where unused; ranges may be None
+    for variant HK_FI_ONLY).  counts: int64 cuda tensor [3, 5] (accumulated); records: optional uint8
+    tensor of count * OUTCOME_DTYPE.itemsize bytes; site_counts: optional int64 [3, 64, 5]."""
+    _check_campaign_buffers(count, counts, records, site_counts)
     arr, keep = _arg_array(devs)
     rng = [r if r is not None else Ranges() for r in ranges]
     rarr = (C.c_void_p * 3)(*[C.cast(C.byref(r), C.c_void_p) for r in rng])
-    camp = Campaign(seed, first, count, nbits, mode, batch, exact, (C.c_uint64 * 3)(*site_masks))
+    camp = Campaign(seed, first, count, nbits, mode, batch, exact, (C.c_uint64 * 3)(*site_masks), variant, hang_factor)
     st = lib().hauberk_inject_campaign(bench_mode, arr, rarr, C.byref(camp), _ptr(records), _ptr(counts),
                                        _ptr(site_counts), _stream(stream))
     _check(st, "hauberk_inject_campaign")
@@ -414,12 +455,13 @@ class CampaignSession:
     asynchronous slices of the same seeded campaign.  Keep `devs` alive while the session lives."""
 
     def __init__(self, bench_mode: int, devs, ranges, seed: int, exact: int = 0, batch: int = 0,
-                 site_masks=DEFAULT_SITE_MASKS, stream=None, nbits: int = 1, mode: int = 0):
+                 site_masks=DEFAULT_SITE_MASKS, stream=None, nbits: int = 1, mode: int = 0,
+                 variant: int = HK_FIFT, hang_factor: int = 0):
         self._arr, self._keep = _arg_array(devs)
         self._devs = devs
         self._rng = [r if r is not None else Ranges() for r in ranges]
         self._rarr = (C.c_void_p * 3)(*[C.cast(C.byref(r), C.c_void_p) for r in self._rng])
-        self._camp = Campaign(seed, 0, 0, nbits, mode, batch, exact, (C.c_uint64 * 3)(*site_masks))
+        self._camp = Campaign(seed, 0, 0, nbits, mode, batch, exact, (C.c_uint64 * 3)(*site_masks), variant, hang_factor)
         self._h = C.c_void_p()
         st = lib().hauberk_campaign_create(bench_mode, self._arr, self._rarr, C.byref(self._camp), C.byref(self._h),
                                            _stream(stream))
@@ -427,6 +469,7 @@ class CampaignSession:
 
     def run(self, first: int, count: int, counts: torch.Tensor, records: torch.Tensor | None = None,
             site_counts: torch.Tensor | None = None):
+        _check_campaign_buffers(count, counts, records, site_counts)
         st = lib().hauberk_campaign_run(self._h, first, count, _ptr(records), _ptr(counts), _ptr(site_counts))
         _check(st, "hauberk_campaign_run")
 
@@ -456,27 +499,79 @@ def records_numpy(rec: torch.Tensor) -> np.ndarray:
     return np.frombuffer(rec.cpu().numpy().tobytes(), dtype=OUTCOME_DTYPE)
 
 
-def decode(bench_mode: int, devs, seed: int, first: int, count: int, site_masks=DEFAULT_SITE_MASKS, nbits: int = 1):
+def decode(bench_mode: int, devs, seed: int, first: int, count: int, site_masks=DEFAULT_SITE_MASKS, nbits: int = 1,
+           variant: int = HK_FIFT):
     """hauberk_decode (host): the campaign's (bench, site, thread, instance, mask) tuples."""
     arr, keep = _arg_array(devs)
     masks = (C.c_uint64 * 3)(*site_masks)
     benches = np.zeros(count, dtype=np.int32)
     faults = (Fault * count)()
-    st = lib().hauberk_decode(bench_mode, arr, masks, seed, nbits, first, count, benches.ctypes.data_as(C.c_void_p),
-                              C.cast(faults, C.c_void_p))
+    st = lib().hauberk_decode(bench_mode, arr, masks, seed, nbits, variant, first, count,
+                              benches.ctypes.data_as(C.c_void_p), C.cast(faults, C.c_void_p))
     _check(st, "hauberk_decode")
     return benches, [(f.site, f.thread, f.inst, f.mask) for f in faults]
 
 
+def detector_site(bench: int, site: int, unroll: int = 4) -> bool:
+    """hauberk_detector_site: the site exists only because of HAUBERK (absent from the FI-only binary)."""
+    return lib().hauberk_detector_site(bench, unroll, site) == 1
+
+
+def campaign_workspace_bytes(bench: int, dev, batch: int = 0, mode: int = 0, site_masks=DEFAULT_SITE_MASKS) -> int:
+    a = dev.args()
+    camp = Campaign(0, 0, 0, 1, mode, batch, 0, (C.c_uint64 * 3)(*site_masks), HK_FIFT, 0)
+    return int(lib().hauberk_campaign_workspace_bytes(bench, C.byref(a), C.byref(camp)))
+
+
+def summarize(counts) -> dict:
+    """hauberk_summarize over the [.., 5] counters summed across benchmarks: coverage = P(detected or
+    masked or failure) = 1 - undetected/total, sdc = undetected/total
+    (an FI-only campaign's unprotected SDC rate, L211-213), detected, failure."""
+    c = np.ascontiguousarray(np.asarray(counts, dtype=np.int64).reshape(-1, 5).sum(0))
+    out = Summary()
+    st = lib().hauberk_summarize(c.ctypes.data_as(C.c_void_p), C.byref(out))
+    if st != 0:
+        return {"coverage": float("nan"), "sdc": float("nan"), "detected": float("nan"), "failure": float("nan"), "total": 0}
+    return {"coverage": out.coverage, "sdc": out.sdc, "detected": out.detected, "failure": out.failure, "total": out.total}
+
+
 def coverage(counts) -> float:
-    """Coverage = P(detected or masked) = 1 - undetected / total."""
-    c = np.asarray(counts, dtype=np.float64).reshape(-1, 5).sum(0)
-    tot = c.sum()
-    return float("nan") if tot == 0 else 1.0 - c[3] / tot
+    """Coverage of a campaign (hauberk_summarize)."""
+    return summarize(counts)["coverage"]
 
 
 def unprotected_sdc(counts) -> float:
-    """FI-only SDC rate of the same campaign: (detected + undetected) / total."""
-    c = np.asarray(counts, dtype=np.float64).reshape(-1, 5).sum(0)
-    tot = c.sum()
-    return float("nan") if tot == 0 else (c[2] + c[3]) / tot
+    """SDC ratio of an FI-only campaign's counters (hauberk_summarize: undetected / total)."""
+    return summarize(counts)["sdc"]
+
+
+def extend_ranges(rs: RangeSet, values) -> int:
+    """hauberk_extend_ranges (A11): add the values to their correlation classes; returns ranges added."""
+    v = np.ascontiguousarray(np.asarray(values, dtype=np.float32))
+    added = C.c_int32(0)
+    _check(lib().hauberk_extend_ranges(C.byref(rs), v.ctypes.data_as(C.c_void_p), v.size, C.byref(added)),
+           "hauberk_extend_ranges")
+    return int(added.value)
+
+
+def outliers(cb: Control, d: int) -> list:
+    """hauberk_outliers: the out-of-range interval the run recorded for detector d (0-2 floats)."""
+    out = (C.c_float * 2)()
+    n = C.c_int32(0)
+    _check(lib().hauberk_outliers(C.byref(cb), d, out, C.byref(n)), "hauberk_outliers")
+    return [float(out[k]) for k in range(n.value)]
+
+
+def alpha_update(alpha: float, fp_ratio: float, hi: float = 0.10, lo: float = 0.05) -> float:
+    return float(lib().hauberk_alpha_update(alpha, fp_ratio, hi, lo))
+
+
+DIAG_NAMES = ["ok", "false_alarm", "transient", "persistent", "failed"]
+
+
+def diagnose(alarm1: int, fail1: int, alarm2: int, fail2: int, identical: bool) -> str:
+    return DIAG_NAMES[lib().hauberk_diagnose(alarm1, fail1, alarm2, fail2, 1 if identical else 0)]
+
+
+def release_caches():
+    lib().hauberk_release_caches()

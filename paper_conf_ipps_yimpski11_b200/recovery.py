@@ -33,56 +33,29 @@ def ord_to_float(o: int) -> float:
     return struct.unpack("<f", struct.pack("<I", bits & 0xFFFFFFFF))[0]
 
 
-def _f32(x: float) -> float:
-    return float(np.float32(x))
-
-
 def extend_ranges(R: hk.Ranges, d: int, values) -> hk.Ranges:
-    """A11 (L1309-1313; DESIGN R24): make detector d's ranges include every value in `values`.
-    A value joins the range of its correlation class at the detector's threshold T = 10^t_exp10
-    (neg: v < -T, zero: |v| <= T, pos: v > T); a class without a range gets a new one."""
-    rs = R.det[d]
-    T = _f32(float(f"1e{rs.t_exp10}"))
-    cls_of = lambda v: 0 if v < -T else (2 if v > T else 1)
-    ranges = {cls_of(rs.lo[r]): [rs.lo[r], rs.hi[r]] for r in range(rs.n)}
-    for v in values:
-        v = _f32(v)
-        if not np.isfinite(v):
-            continue
-        c = cls_of(v)
-        if c in ranges:
-            ranges[c][0] = min(ranges[c][0], v)
-            ranges[c][1] = max(ranges[c][1], v)
-        else:
-            ranges[c] = [v, v]
-    keys = sorted(ranges)
-    rs.n = len(keys)
-    for r, c in enumerate(keys):
-        rs.lo[r], rs.hi[r] = ranges[c]
+    """A11 (L1309-1313; DESIGN R24) through hauberk_extend_ranges: make detector d's ranges include
+    every value (each joins the range of its correlation class at the detector's threshold)."""
+    hk.extend_ranges(R.det[d], values)
     return R
 
 
 def outliers_of(cb: hk.Control, d: int):
-    """The recorded outlier interval of detector d (empty if none)."""
-    lo, hi = cb.outlier_min_ord[d], cb.outlier_max_ord[d]
-    if lo == 0x7FFFFFFF and hi == -0x80000000:
-        return []
-    return [ord_to_float(lo), ord_to_float(hi)]
+    """The recorded outlier interval of detector d (hauberk_outliers; empty if none)."""
+    return hk.outliers(cb, d)
 
 
 @dataclass
 class AlphaController:
-    """alpha per detector set: x10 above 10 % false positives, /10 below 5 %, never below 1 (L2066-2077)."""
+    """alpha per detector set (hauberk_alpha_update): x10 above 10 % false positives, /10 below 5 %,
+    never below 1 (L2066-2077)."""
     alpha: float = 1.0
     hi: float = 0.10
     lo: float = 0.05
     history: list = field(default_factory=list)
 
     def update(self, fp_ratio: float) -> float:
-        if fp_ratio > self.hi:
-            self.alpha *= 10.0
-        elif fp_ratio < self.lo and self.alpha >= 10.0:
-            self.alpha /= 10.0
+        self.alpha = hk.alpha_update(self.alpha, fp_ratio, self.hi, self.lo)
         self.history.append((fp_ratio, self.alpha))
         return self.alpha
 
@@ -107,32 +80,30 @@ class Diagnosis:
 
 
 def protected_run(dev, ranges: hk.Ranges, variant: int = hk.HK_FT, learn: bool = True) -> Diagnosis:
-    """Run the protected kernel; on an alarm re-execute and diagnose (Fig. 11)."""
+    """Run the protected kernel; on an alarm re-execute and diagnose (Fig. 11, hauberk_diagnose)."""
     cb = hk.new_control(dev.output()[0].device if isinstance(dev.output(), tuple) else dev.output().device)
     hk.run(dev, variant, ranges, cb)
     torch.cuda.current_stream().synchronize()
     c1 = hk.read_control(cb)
     out1 = _outputs(dev)
+    if c1.alarm == 0 and c1.fail == 0:
+        return Diagnosis(OK, 0, None, False, out1)
     if c1.fail:
         return Diagnosis(FAILED, c1.alarm, None, False, out1)
-    if c1.alarm == 0:
-        return Diagnosis(OK, 0, None, False, out1)
     hk.run(dev, variant, ranges, cb)
     torch.cuda.current_stream().synchronize()
     c2 = hk.read_control(cb)
     out2 = _outputs(dev)
-    if c2.alarm == 0 and c2.fail == 0:
-        return Diagnosis(TRANSIENT, c1.alarm, 0, False, out2)
-    if _identical(out1, out2) and c2.alarm == c1.alarm:
-        extended = False
-        if learn and (c1.alarm & hk_alarm_range()):
-            for d in range(ranges.n_det):
-                vals = outliers_of(c1, d)
-                if vals:
-                    extend_ranges(ranges, d, vals)
-                    extended = True
-        return Diagnosis(FALSE_ALARM, c1.alarm, c2.alarm, extended, out1)
-    return Diagnosis(PERSISTENT, c1.alarm, c2.alarm, False, out2)
+    verdict = hk.diagnose(c1.alarm, c1.fail, c2.alarm, c2.fail, _identical(out1, out2))
+    extended = False
+    if verdict == FALSE_ALARM and learn and (c1.alarm & hk_alarm_range()):
+        for d in range(ranges.n_det):
+            vals = outliers_of(c1, d)
+            if vals:
+                extend_ranges(ranges, d, vals)
+                extended = True
+    keep = out1 if verdict == FALSE_ALARM else out2
+    return Diagnosis(verdict, c1.alarm, c2.alarm, extended, keep)
 
 
 def hk_alarm_range() -> int:

@@ -211,11 +211,14 @@ def test_mriq_multitile_campaign_exact_bit_exact():
 
 
 # ---------------------------------------------------------------------------------------------- TPACF
-@pytest.mark.parametrize("shape", [(300, 2, 64), (70, 1, 16), (129, 3, 1000), (257, 1, 7), (1, 1, 64), (2, 1, 1),
-                                   (33, 2, 32), (513, 1, 256)])
+@pytest.mark.parametrize("shape", [(300, 2), (70, 1), (129, 3), (257, 1), (1, 1), (2, 1), (33, 2), (513, 1), (1025, 2),
+                                   (1536, 1), (2051, 1)])
 def test_tpacf_hist_bit_exact(shape):
-    n, nr, chunk = shape
-    p = W.tpacf_small(n=n, n_rand=nr, chunk=chunk)
+    """Shapes spanning one / several 512-point blocks and 512-partner tiles with ragged tails: the
+    single-run kernel's chunk items, their exact (acc, cnt) combine and the last-item checks give
+    the oracle's histograms and the oracle's ranges (PROFILE samples of the whole loops)."""
+    n, nr = shape
+    p = W.tpacf_small(n=n, n_rand=nr)
     d = _mk(2, p)
     R = hk.profile_ranges(d)
     assert _run(d, hk.HK_FT, R).alarm == 0
@@ -254,7 +257,7 @@ def _campaign_pair(probs, seed, count, exact, mode=-1, batch=0):
 
 
 def test_campaign_exact_mode_bit_exact():
-    probs = [W.cp_small(), W.mriq_problem(6, 61, n_vox=200, seed=3), W.tpacf_small(n=150, n_rand=2, chunk=32)]
+    probs = [W.cp_small(), W.mriq_problem(6, 61, n_vox=200, seed=3), W.tpacf_small(n=150, n_rand=2)]
     gc, grec, oc, orec = _campaign_pair(probs, 0xABCDEF, 1200, exact=1)
     for k in ("index", "bench", "site", "thread", "inst", "mask"):
         assert np.array_equal(grec[k], orec[k]), k
@@ -289,7 +292,7 @@ def _ambiguous(g, o, probs=None):
 
 
 def test_campaign_fast_mode_exact_outside_guard_band():
-    probs = [W.cp_small(), W.mriq_problem(6, 61, n_vox=200, seed=3), W.tpacf_small(n=150, n_rand=2, chunk=32)]
+    probs = [W.cp_small(), W.mriq_problem(6, 61, n_vox=200, seed=3), W.tpacf_small(n=150, n_rand=2)]
     gc, grec, oc, orec = _campaign_pair(probs, 0x1234, 1500, exact=0)
     for k in ("index", "bench", "site", "thread", "inst", "mask"):
         assert np.array_equal(grec[k], orec[k]), k
@@ -314,7 +317,7 @@ def test_campaign_config1_cp_1000_injections():
 
 
 def test_campaign_sharding_invariance_and_batching():
-    probs = [W.cp_small(), W.mriq_problem(4, 40, n_vox=64, seed=9), W.tpacf_small(n=64, n_rand=1, chunk=16)]
+    probs = [W.cp_small(), W.mriq_problem(4, 40, n_vox=64, seed=9), W.tpacf_small(n=64, n_rand=1)]
     devs = [_mk(b, probs[b]) for b in range(3)]
     R = [hk.profile_ranges(d) for d in devs]
     whole = torch.zeros((3, 5), dtype=torch.int64, device=DEV)
@@ -349,7 +352,7 @@ def test_tpacf_bucket_binning_adversarial_dots():
     pts[0, :, 0] = 1.0
     pts[1, :, 0] = v
     pts[1, :, 1] = np.sqrt(np.maximum(0.0, 1.0 - v.astype(np.float64) ** 2)).astype(np.float32)
-    p = W.TPACFProblem(pts=pts, edges=e, chunk=512)
+    p = W.TPACFProblem(pts=pts, edges=e)
     d = _mk(2, p)
     cb = hk.new_control(DEV)
     hk.run(d, hk.HK_BASE, None, cb)
@@ -387,7 +390,7 @@ def test_tpacf_signed_zero_and_special_dots_against_a_zero_edge():
     pts[1, :, 0] = -1.0
     pts[1, :, 1] = -0.0
     pts[1, :, 2] = v
-    p = W.TPACFProblem(pts=pts, edges=e, chunk=64)
+    p = W.TPACFProblem(pts=pts, edges=e)
     d = _mk(2, p)
     cb = hk.new_control(DEV)
     hk.run(d, hk.HK_BASE, None, cb)
@@ -399,7 +402,7 @@ def test_tpacf_signed_zero_and_special_dots_against_a_zero_edge():
 
 
 def test_campaign_session_matches_one_shot_calls():
-    probs = [W.cp_small(), W.mriq_problem(4, 40, n_vox=64, seed=9), W.tpacf_small(n=64, n_rand=1, chunk=16)]
+    probs = [W.cp_small(), W.mriq_problem(4, 40, n_vox=64, seed=9), W.tpacf_small(n=64, n_rand=1)]
     devs = [_mk(b, probs[b]) for b in range(3)]
     R = [hk.profile_ranges(d) for d in devs]
     one = torch.zeros((3, 5), dtype=torch.int64, device=DEV)
@@ -419,7 +422,7 @@ def test_campaign_session_matches_one_shot_calls():
 def test_campaign_concurrent_streams_equal_serial(monkeypatch):
     """Sessions fork one stream per benchmark; the per-injection records, the
     counters and the per-site counters must equal those of a serial session (HK_CONCURRENT=0)."""
-    probs = [W.cp_small(), W.mriq_problem(4, 40, n_vox=64, seed=9), W.tpacf_small(n=64, n_rand=1, chunk=16)]
+    probs = [W.cp_small(), W.mriq_problem(4, 40, n_vox=64, seed=9), W.tpacf_small(n=64, n_rand=1)]
     devs = [_mk(b, probs[b]) for b in range(3)]
     R = [hk.profile_ranges(d) for d in devs]
     out = {}
@@ -444,7 +447,7 @@ def test_campaign_concurrent_streams_equal_serial(monkeypatch):
 @pytest.mark.parametrize("k", [3, 6, 10, 15])
 def test_campaign_multibit_exact_mode_bit_exact(k, gmode):
     """Fig. 14's bit counts (L2605-2634), GPU replica (0) and replay (1) modes vs the oracle."""
-    probs = [W.cp_small(), W.mriq_problem(5, 41, n_vox=100, seed=4), W.tpacf_small(n=90, n_rand=1, chunk=32)]
+    probs = [W.cp_small(), W.mriq_problem(5, 41, n_vox=100, seed=4), W.tpacf_small(n=90, n_rand=1)]
     devs = [_mk(b, probs[b], 1) for b in range(3)]
     gr = [hk.profile_ranges(d) for d in devs]
     counts = torch.zeros((3, 5), dtype=torch.int64, device=DEV)
@@ -470,7 +473,7 @@ def _gpu_campaign(devs, ranges, seed, first, count, exact=0, mode=0, nbits=1):
 
 @pytest.mark.parametrize("exact", [0, 1])
 def test_gpu_replay_equals_gpu_replica(exact):
-    probs = [W.cp_small(), W.mriq_problem(6, 61, n_vox=200, seed=3), W.tpacf_small(n=150, n_rand=2, chunk=32)]
+    probs = [W.cp_small(), W.mriq_problem(6, 61, n_vox=200, seed=3), W.tpacf_small(n=150, n_rand=2)]
     devs = [_mk(b, probs[b], exact) for b in range(3)]
     R = [hk.profile_ranges(d) for d in devs]
     c0, r0 = _gpu_campaign(devs, R, 0xBEEF, 0, 1500, exact=exact, mode=0)
@@ -500,7 +503,7 @@ def test_gpu_replay_config_shapes_vs_oracle_replay():
 
 
 def test_gpu_replay_exact_mode_bit_exact_config_shapes():
-    probs = [W.cp_config1(), W.mriq_problem(16, 512, seed=0x4D5249), W.tpacf_problem(1024, 2, chunk=256)]
+    probs = [W.cp_config1(), W.mriq_problem(16, 512, seed=0x4D5249), W.tpacf_problem(1024, 2)]
     devs = [_mk(b, probs[b], 1) for b in range(3)]
     R = [hk.profile_ranges(d) for d in devs]
     gc, g = _gpu_campaign(devs, R, 0x5151, 0, 6000, exact=1, mode=1, nbits=3)
@@ -609,7 +612,7 @@ def test_guardian_real_crash_validation(bench):
     accesses that land in mapped memory do not fault: the known limit of R16; small buffers share
     their 2 MiB pages with others), reported by `python -m paper_conf_ipps_yimpski11_b200.guardian`."""
     from paper_conf_ipps_yimpski11_b200 import guardian as G
-    p = [W.cp_small(), None, W.tpacf_small(n=150, n_rand=1, chunk=64)][bench]
+    p = [W.cp_small(), None, W.tpacf_small(n=150, n_rand=1)][bench]
     rep = G.validate(bench, p, n_fail=10, n_other=8, scan=600, floor_s=2.0)
     assert rep["n"] == rep["sampled_failures"] + rep["sampled_others"] and rep["sampled_failures"] > 0
     assert rep["non_failure_identical"] == 1.0

@@ -47,7 +47,7 @@ def _worker(rank, world, port, total, q):
     dist.init_process_group("gloo", rank=rank, world_size=world)
     import oracle as O
     import workloads as W
-    probs = [W.cp_small(), W.mriq_problem(4, 23, n_vox=60), W.tpacf_small(n=60, n_rand=1, chunk=16)]
+    probs = [W.cp_small(), W.mriq_problem(4, 23, n_vox=60), W.tpacf_small(n=60, n_rand=1)]
     R = [O.profile_ranges(b, probs[b]) for b in range(3)]
     first, cnt = par.shard(total, rank, world)
     c, _ = O.campaign(-1, probs, R, seed=777, first=first, count=cnt, mode=1, records=False)
@@ -77,7 +77,7 @@ def test_gloo_world2_counters_equal_single_process():
     for p in procs:
         p.join(timeout=120)
         assert p.exitcode == 0
-    probs = [W.cp_small(), W.mriq_problem(4, 23, n_vox=60), W.tpacf_small(n=60, n_rand=1, chunk=16)]
+    probs = [W.cp_small(), W.mriq_problem(4, 23, n_vox=60), W.tpacf_small(n=60, n_rand=1)]
     R = [O.profile_ranges(b, probs[b]) for b in range(3)]
     c, _ = O.campaign(-1, probs, R, seed=777, first=0, count=total, mode=1, records=False)
     counts, same, differ, mx = res

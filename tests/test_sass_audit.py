@@ -82,9 +82,25 @@ def test_tpacf_ft_keeps_detectors(sass):
 
 
 def test_fi_kernels_compiled_for_every_site_kind(sass):
-    assert len([n for n in sass if "cp_fi_kernel" in n]) == 15 * 2 * 2  # kinds x {FAST, EXACT} x U {4, 8}
-    assert len([n for n in sass if "mriq_fi_kernel" in n]) == 17 * 2  # 16 Q-kernel kinds + PhiMag
-    assert len([n for n in sass if "tpacf_fi_kernel" in n]) == 11
+    # kinds x {FAST, EXACT} x U {4, 8} x {FI&FT, FI-only}
+    assert len([n for n in sass if "cp_fi_kernel" in n]) == 15 * 2 * 2 * 2
+    assert len([n for n in sass if "mriq_fi_kernel" in n]) == 17 * 2 * 2  # 16 Q-kernel kinds + PhiMag
+    assert len([n for n in sass if "tpacf_fi_kernel" in n]) == 11 * 2
+
+
+@pytest.mark.parametrize("pat", [r"tpacf_fi_kernelILi2ELb{}EE", r"mriq_fi_kernelILi2ELb0ELb{}EE", r"cp_fi_kernelILi2ELi4ELb0ELb{}EE"])
+def test_fi_only_binary_has_no_detector_code(sass, pat):
+    """Row a7: the FI-only replicas are the original program plus the hook — fewer instructions
+    than the FI&FT replicas of the same site kind (no duplicates, checksums, counters, checks)."""
+    fift, fionly = _find(sass, pat.format(1)), _find(sass, pat.format(0))
+    assert len(fionly) < len(fift)
+    assert _count(fionly, "LOP3") < _count(fift, "LOP3")
+
+
+def test_tpacf_replica_loop_uses_one_table_load_and_one_shared_atomic_per_pair(sass):
+    """bin = one LDS.64 of {edge, 128 * bmin} + one compare; one ATOMS per pair."""
+    ops = _find(sass, r"tpacf_fi_kernelILi2ELb1EE")
+    assert _count(ops, "LDS.64") >= 16 and _count(ops, "ATOMS") >= 16 and _count(ops, "LDS.128") >= 6
 
 
 def test_no_tensor_core_or_fp64_in_hot_kernels(sass):

@@ -11,14 +11,16 @@
 //  * the single run (tpacf_kernel) cuts the partner range into chunks of TP_TILE partners, adds the
 //    per-chunk (acc, cnt) partials with global atomics, and the last chunk item of a point block
 //    (a per-(h, block) completion counter) runs CheckEqual / CheckRange for its points;
-//  * the campaign replicas (tpacf_fi_kernel) give each CTA whole loops (all partners of its 512
+//  * the campaign replicas (tpacf_fi_kernel) give each CTA whole loops (all partners of its
 //    points, streamed through a two-stage shared-memory ring), and the faulted abstract thread runs
 //    its sequential per-thread FI program after the CTA's fast loop.
-// B200 shape: 256 threads, two abstract threads per CUDA thread (points i and i + 256) sharing every
-// partner load (broadcast LDS.128, 8 partners per group); bin by one LDS.64 of a 2,048-entry table
-// {edge[bmin], 128 * bmin} indexed by the top 11 bits of u = fl(1 - dot), plus one compare; the
-// counts go to lane-private shared histograms [warp][bin][lane] (bank = lane) with the two points
-// packed in the 16-bit halves of one counter, one ATOMS per pair.
+// B200 shape: 128 threads, NP abstract threads per CUDA thread (points i0 + t + 128k) sharing
+// every partner load (broadcast LDS.128); bin = byte table of 4 * bmin indexed by the top 11 bits
+// of u = fl(1 - dot), then one edge load and one compare; lane-private shared histograms
+// [warp][word][bin][lane] (bank = lane) with two points packed in the 16-bit halves of a counter,
+// one ATOMS per pair.  Shared-memory wavefronts bind this loop (ncu: LDS.64 and LDS.128 cost two
+// wavefronts each even as broadcasts, 32-bit LDS / ATOMS one), so the table stays byte-wide and
+// NP = 4 amortises the partner loads over four points.
 #include <algorithm>
 #include <array>
 #include <map>
@@ -30,21 +32,31 @@
 
 namespace hk {
 
-#ifndef HK_TP_MINB
-#define HK_TP_MINB 4
+#ifndef HK_TP_NP_FI
+#define HK_TP_NP_FI 4  // points per CUDA thread, campaign replicas
 #endif
-constexpr int TP_THREADS = 256;
+#ifndef HK_TP_NP_SR
+#define HK_TP_NP_SR 2  // points per CUDA thread, single run (256-point items: a finer LPT schedule)
+#endif
+#ifndef HK_TP_MINB
+#define HK_TP_MINB 6     // replicas: 37 KB of shared memory per CTA -> 6 CTAs per SM, 80 registers
+#endif
+#ifndef HK_TP_MINB_SR
+#define HK_TP_MINB_SR 8  // single run: 25.5 KB per CTA -> 8 CTAs per SM, 64 registers
+#endif
+#ifndef HK_TP_GROUP
+#define HK_TP_GROUP 0  // partners per group of the unmasked loop (0: 4 for NP >= 4, else 8)
+#endif
+constexpr int TP_THREADS = 128;
 constexpr int TP_WARPS = TP_THREADS / 32;
-constexpr int TP_CTA_PTS = 2 * TP_THREADS;  // two abstract threads per CUDA thread
 constexpr int TP_TILE = 512;                // partners per shared-memory tile (6 KB)
 constexpr int TP_LUT = 2048;                // u-buckets: sign, 8 exponent bits, 2 mantissa bits
 constexpr int TP_SCHED_MAX_SM = 1024;
-constexpr uint32_t TP_HB = 128;             // bytes between two bins of a lane-private histogram
 
 struct TPParams {
   const float* pts;
   const float* edges;
-  const uint2* lut;       // [TP_LUT] {bits(edge[bmin]) or -inf, 128 * bmin}; built by tpacf_lut_kernel
+  const uint8_t* lut;     // [TP_LUT] 4 * bmin per u-bucket; built by tpacf_lut_kernel
   const int* lut_ok;      // 1: every bucket holds at most one edge (else the binary search is used)
   unsigned long long* hist;
   hk_control* cb;
@@ -53,10 +65,11 @@ struct TPParams {
   int32_t* accg;          // single run: per abstract thread partial sums of acc and cnt (zeroed per run)
   int32_t* cntg;
   int32_t* done;          // single run: chunk items finished per (h, point block)
-  int32_t n, nr, nb, ndet, nblk;
+  int32_t n, nr, nb, ndet;
+  int32_t nblk;           // point blocks per histogram for the launching kernel's NP
   int32_t g0, g1;         // abstract threads [g0, g1) of this run (single-run sharding)
   uint32_t z;
-  int32_t one, eight;     // runtime 1 and 8 (opaque to the compiler)
+  int32_t one, four, eight;  // runtime 1, 4 and 8 (opaque to the compiler)
 };
 
 // ---------------------------------------------------------------------------------------------
@@ -65,8 +78,9 @@ struct TPParams {
 //  * table: u = fl(1 - dot) is monotone (non-increasing) in dot and so is bin, so every bucket q of
 //    u's top 11 bits maps to a contiguous dot interval [dmin, dmax].  The device builds
 //    bmin = bin(dmax) per bucket and checks bin(dmin) <= bmin + 1; then bin = bmin + (dot < edge[bmin])
-//    exactly (edge[bmin] = -inf past the last edge; NaN dots compare false, and NaN u lands in a
-//    bucket whose bmin is bin(NaN) = 0).  One LDS.64 {edge bits, 128 * bmin} + one FSETP per pair.
+//    exactly (edge[bmin] = -inf past the last edge; NaN dots compare false, and the canonical NaN u
+//    lands in a bucket whose bmin is bin(NaN) = 0).  The table holds 4 * bmin, the byte offset of
+//    edge[bmin], so the edge load needs no address arithmetic.
 // ---------------------------------------------------------------------------------------------
 __device__ __forceinline__ int32_t tp_bin_search(const float* Es, float dot) {
   int32_t b = 0;
@@ -74,17 +88,17 @@ __device__ __forceinline__ int32_t tp_bin_search(const float* Es, float dot) {
   for (int s = 16; s >= 1; s >>= 1) b += (dot < Es[b + s - 1]) ? s : 0;
   return b;
 }
-// 128 * bin through the table at shared byte address lb (uniform)
-__device__ __forceinline__ uint32_t tp_hb_lut(uint32_t lb, float dot) {
+// 4 * bin through the byte table L and the edges at the shared byte address eb (uniform)
+__device__ __forceinline__ uint32_t tp_b4_lut(const uint8_t* __restrict__ L, uint32_t eb, float dot) {
   const float u = __fsub_rn(1.0f, dot);
-  const uint32_t off = (fb(u) >> 18) & 0x3FF8u;  // 8 * (bits(u) >> 21)
-  uint32_t ex, ey;
-  asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(ex), "=r"(ey) : "r"(lb + off));
-  return (dot < bf(ex)) ? ey + TP_HB : ey;
+  const uint32_t b4 = L[fb(u) >> 21];
+  float e;
+  asm("ld.shared.f32 %0, [%1];" : "=f"(e) : "r"(eb + b4));
+  return (dot < e) ? b4 + 4u : b4;
 }
 template <bool LUT>
-__device__ __forceinline__ uint32_t tp_hb(uint32_t lb, const float* Es, float dot) {
-  return LUT ? tp_hb_lut(lb, dot) : (uint32_t)tp_bin_search(Es, dot) * TP_HB;
+__device__ __forceinline__ uint32_t tp_b4(const uint8_t* __restrict__ L, uint32_t eb, const float* Es, float dot) {
+  return LUT ? tp_b4_lut(L, eb, dot) : 4u * (uint32_t)tp_bin_search(Es, dot);
 }
 __device__ __forceinline__ void red_shared(uint32_t addr, uint32_t v) {
   asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(addr), "r"(v) : "memory");
@@ -106,10 +120,10 @@ __device__ __forceinline__ int32_t bin_def(const float* edges, int nb, float dot
   return b;
 }
 
-// One thread per bucket q.  Finite-u buckets: the dot interval is found by stepping from
-// fl(1 - u_lo) / fl(1 - u_hi) to the exact extremes; non-finite u (inf / NaN exponent) and
-// negative u are handled by the same interval logic on their representable dots.
-__global__ void tpacf_lut_kernel(const float* __restrict__ edges, int nb, uint2* __restrict__ lut, int* ok) {
+// One thread per bucket q: the dot interval of the bucket is found by stepping from
+// fl(1 - u_lo) / fl(1 - u_hi) to the exact extremes (negative-u buckets have their bit order
+// reversed); inf / NaN buckets are set directly.
+__global__ void tpacf_lut_kernel(const float* __restrict__ edges, int nb, uint8_t* __restrict__ lut, int* ok) {
   const int q = blockIdx.x * blockDim.x + threadIdx.x;
   if (q >= TP_LUT) return;
   const uint32_t lo_bits = (uint32_t)q << 21, hi_bits = lo_bits | 0x1fffffu;
@@ -139,31 +153,31 @@ __global__ void tpacf_lut_kernel(const float* __restrict__ edges, int nb, uint2*
     const int bmax = bin_def(edges, nb, dmin);
     good = (__fsub_rn(1.0f, dmax) >= ulo) && (__fsub_rn(1.0f, dmin) <= uhi) && (bmax - bmin <= 1);
   }
-  const uint32_t e = bmin <= nb ? fb(edges[bmin]) : 0xff800000u;
-  lut[q] = make_uint2(e, (uint32_t)bmin * TP_HB);
+  lut[q] = (uint8_t)(4 * bmin);  // byte offset of E[bmin] (E padded with -inf beyond nb)
   if (!good) atomicExch(ok, 0);
 }
 
 // ---------------------------------------------------------------------------------------------
-// Shared memory: L[2048] uint2 | E[32] f32 | B[2][3 * TP_TILE] f32 (packed x, y, z) | H[warps][nb2][32]
+// Shared memory: L[2048] u8 | E[32] f32 | B[2][3 * TP_TILE] f32 (packed x, y, z) |
+// H[warps][NP/2 words][nb2][32] u32 | flag
 // ---------------------------------------------------------------------------------------------
 struct TPSmem {
-  uint2* L;
+  uint8_t* L;
   float* E;
   float* B;
   uint32_t* H;
   int* flag;
 };
-__host__ __device__ inline size_t tp_smem_bytes(int nb2) {
-  return (size_t)TP_LUT * 8 + 32 * 4 + 2 * 3 * TP_TILE * 4 + (size_t)TP_WARPS * nb2 * 32 * 4 + 16;
+__host__ __device__ inline size_t tp_smem_bytes(int nb2, int np) {
+  return (size_t)TP_LUT + 32 * 4 + 2 * 3 * TP_TILE * 4 + (size_t)TP_WARPS * (np / 2) * nb2 * 32 * 4 + 16;
 }
-__device__ __forceinline__ TPSmem tp_carve(unsigned char* base, int nb2) {
+__device__ __forceinline__ TPSmem tp_carve(unsigned char* base, int nb2, int np) {
   TPSmem S;
-  S.L = reinterpret_cast<uint2*>(base);
-  S.E = reinterpret_cast<float*>(base + TP_LUT * 8);
-  S.B = reinterpret_cast<float*>(base + TP_LUT * 8 + 128);
-  S.H = reinterpret_cast<uint32_t*>(base + TP_LUT * 8 + 128 + 2 * 3 * TP_TILE * 4);
-  S.flag = reinterpret_cast<int*>(base + TP_LUT * 8 + 128 + 2 * 3 * TP_TILE * 4 + (size_t)TP_WARPS * nb2 * 128);
+  S.L = base;
+  S.E = reinterpret_cast<float*>(base + TP_LUT);
+  S.B = reinterpret_cast<float*>(base + TP_LUT + 128);
+  S.H = reinterpret_cast<uint32_t*>(base + TP_LUT + 128 + 2 * 3 * TP_TILE * 4);
+  S.flag = reinterpret_cast<int*>(base + TP_LUT + 128 + 2 * 3 * TP_TILE * 4 + (size_t)TP_WARPS * (np / 2) * nb2 * 128);
   return S;
 }
 __device__ __forceinline__ void cp_async4(void* dst, const void* src) {
@@ -178,13 +192,13 @@ __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_gr
 
 // Table + edges, once per CTA (the edges padded with -inf for the binary search).
 __device__ __forceinline__ void tp_stage_tables(const TPParams& p, const TPSmem& S) {
-  for (int k = threadIdx.x; k < TP_LUT / 2; k += TP_THREADS)
-    cp_async16(S.L + 2 * k, p.lut + 2 * k);
+  for (int k = threadIdx.x; k < TP_LUT / 16; k += TP_THREADS) cp_async16(S.L + 16 * k, p.lut + 16 * k);
   if (threadIdx.x < 32) S.E[threadIdx.x] = threadIdx.x <= p.nb ? p.edges[threadIdx.x] : __int_as_float(0xff800000);
   cp_async_commit();
 }
+template <int NP>
 __device__ __forceinline__ void tp_zero_hist(const TPParams& p, const TPSmem& S) {
-  const int nh = TP_WARPS * (p.nb + 2) * 32;
+  const int nh = TP_WARPS * (NP / 2) * (p.nb + 2) * 32;
   for (int k = threadIdx.x; k < nh; k += TP_THREADS) S.H[k] = 0u;
 }
 // Partners [j0, j0 + cnt) of set sb into ring slot `slot` (cnt <= TP_TILE; 4-byte async copies).
@@ -195,13 +209,14 @@ __device__ __forceinline__ void tp_stage_tile(const TPParams& p, const TPSmem& S
   cp_async_commit();
 }
 
-// Reduce the lane-private histograms (both 16-bit halves) and add them to hist[base + b]:
-// 8 warps x nb2 rows of 32 counters are summed row-wise (rotated start: no bank conflicts), the
-// warp partials of each bin combined in shared memory, then one u64 atomic per non-zero bin.
+// Reduce the lane-private histograms (both 16-bit halves of every word) and add them to
+// hist[base + b]: each (warp, word, bin) row of 32 counters is summed (rotated start: no bank
+// conflicts), the rows of a bin combined in shared memory, then one u64 atomic per non-zero bin.
+template <int NP>
 __device__ __forceinline__ void tp_flush(const TPParams& p, const TPSmem& S, unsigned long long* hist, int base) {
-  const int nb2 = p.nb + 2;
+  const int nb2 = p.nb + 2, rows = TP_WARPS * (NP / 2);
   uint32_t* part = reinterpret_cast<uint32_t*>(S.B);  // the ring is free at this point
-  for (int t = threadIdx.x; t < TP_WARPS * nb2; t += TP_THREADS) {
+  for (int t = threadIdx.x; t < rows * nb2; t += TP_THREADS) {
     const uint32_t* row = S.H + (size_t)t * 32;
     uint32_t s = 0;
 #pragma unroll 8
@@ -214,7 +229,7 @@ __device__ __forceinline__ void tp_flush(const TPParams& p, const TPSmem& S, uns
   __syncthreads();
   if (threadIdx.x < nb2) {
     unsigned long long s = 0;
-    for (int w = 0; w < TP_WARPS; ++w) s += part[w * nb2 + threadIdx.x];
+    for (int w = 0; w < rows; ++w) s += part[w * nb2 + threadIdx.x];
     if (s) atomicAdd(hist + base + threadIdx.x, s);
   }
 }
@@ -226,7 +241,7 @@ struct TPPoint {
   int32_t i, h, boff, jb, je, expect, base;
   float x1, y1, z1;
   uint32_t chk, alarm;
-  int32_t acc, cnt;  // acc in units of TP_HB (the table's 128 * bin) until tp_finish_acc
+  int32_t acc, cnt;  // acc in units of 4 (the table's 4 * bin) until divided
   bool valid;
 };
 
@@ -274,6 +289,7 @@ __device__ __forceinline__ TPPoint tp_prologue(const TPParams& p, const unsigned
   }
   P.acc = 0;
   P.cnt = 0;
+  if (!valid) P.jb = INT32_MAX;  // takes part in no pair
   return P;
 }
 
@@ -309,97 +325,101 @@ __device__ __forceinline__ float tp_dot(const TPPoint& P, float x2, float y2, fl
 }
 
 // ---------------------------------------------------------------------------------------------
-// The pair loops over one staged tile.  Hl = this lane's histogram base (shared byte address);
-// incA / incB = the packed increments of the two points (1 / 0x10000; 0 for an absent point or the
-// faulted abstract thread of an FI CTA, whose whole loop runs in the FI program instead).
-//  * tp_pairs_all: every point of the CTA has all of [k0, k1) as partners (no masks); 8-partner
-//    groups = six broadcast LDS.128; the counters advance by 8 per group (the strength reduction
-//    any compiler applies to an unrolled cnt++; the FI program keeps the per-iteration increment);
+// The pair loops over one staged tile.  Hw[w] = this lane's histogram word w (shared byte address;
+// point k counts in word k/2, half k%2); inc[k] = 1 / 0x10000 (0 for an absent point or the faulted
+// abstract thread of an FI CTA, whose whole loop runs in the FI program instead).
+//  * tp_pairs_all: every point of the CTA has all of [k0, k1) as partners (no masks); groups of G
+//    partners (G = 32 / NP, i.e. 3 * G / 4 broadcast LDS.128 per group) with the counters advanced
+//    by G per group (the strength reduction any compiler applies to an unrolled cnt++; the FI
+//    program keeps the per-iteration increment);
 //  * tp_pairs_masked: the diagonal of a self-correlation row (j >= jb differs per point).
 // ---------------------------------------------------------------------------------------------
-template <bool CNT, bool LUT>
-__device__ __forceinline__ void tp_pair1(uint32_t Hl, uint32_t lb, const float* Es, TPPoint& A, TPPoint& B, uint32_t incA,
-                                         uint32_t incB, float x2, float y2, float z2, bool pa, bool pb) {
-  const uint32_t ha = tp_hb<LUT>(lb, Es, tp_dot(A, x2, y2, z2));
-  const uint32_t hb = tp_hb<LUT>(lb, Es, tp_dot(B, x2, y2, z2));
-  red_shared(Hl + ha, pa ? incA : 0u);
-  red_shared(Hl + hb, pb ? incB : 0u);
-  if (CNT) {
-    A.acc += pa ? (int32_t)ha : 0;
-    A.cnt += pa ? 1 : 0;
-    B.acc += pb ? (int32_t)hb : 0;
-    B.cnt += pb ? 1 : 0;
+struct TPLoopCtx {
+  const uint8_t* L;
+  uint32_t eb;
+  const float* Es;
+};
+
+template <int NP, bool CNT, bool LUT>
+__device__ __forceinline__ void tp_pair1(const TPLoopCtx& c, const uint32_t (&Hw)[NP / 2], TPPoint (&P)[NP],
+                                         const uint32_t (&inc)[NP], float x2, float y2, float z2, int j, bool masked) {
+#pragma unroll
+  for (int k = 0; k < NP; ++k) {
+    const uint32_t b4 = tp_b4<LUT>(c.L, c.eb, c.Es, tp_dot(P[k], x2, y2, z2));
+    const bool on = !masked || j >= P[k].jb;
+    red_shared(Hw[k / 2] + b4 * 32u, on ? inc[k] : 0u);
+    if (CNT) {
+      P[k].acc += on ? (int32_t)b4 : 0;
+      P[k].cnt += on ? 1 : 0;
+    }
   }
 }
 
-template <bool CNT, bool LUT>
-__device__ __forceinline__ void tp_pairs_all(const TPParams& p, const float* __restrict__ Bt, uint32_t Hl, uint32_t lb,
-                                             const float* Es, TPPoint& A, TPPoint& B, uint32_t incA, uint32_t incB, int k,
-                                             int k1) {
+template <int NP, bool CNT, bool LUT>
+__device__ __forceinline__ void tp_pairs_all(const TPParams& p, const TPLoopCtx& c, const float* __restrict__ Bt,
+                                             const uint32_t (&Hw)[NP / 2], TPPoint (&P)[NP], const uint32_t (&inc)[NP],
+                                             int k, int k1) {
   if (!LUT) {  // the binary-search fallback (a bucket holds two edges): plain loop, rare
 #pragma unroll 1
-    for (; k < k1; ++k) tp_pair1<CNT, LUT>(Hl, lb, Es, A, B, incA, incB, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], true, true);
+    for (; k < k1; ++k) tp_pair1<NP, CNT, LUT>(c, Hw, P, inc, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], 0, false);
     return;
   }
-  for (; k < k1 && (k & 3); ++k) tp_pair1<CNT, LUT>(Hl, lb, Es, A, B, incA, incB, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], true, true);
+  // partners per group: G * NP pairs per thread and group (16 for NP = 4: enough independent
+  // table lookups in flight within the 80-register budget of 6 CTAs per SM)
+  constexpr int G = HK_TP_GROUP > 0 ? HK_TP_GROUP : (NP >= 4 ? 4 : 8);
+  static_assert(G % 4 == 0, "groups are whole 48-byte partner quads");
+  for (; k < k1 && (k & 3); ++k) tp_pair1<NP, CNT, LUT>(c, Hw, P, inc, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], 0, false);
   const float4* __restrict__ T4 = reinterpret_cast<const float4*>(Bt);
 #pragma unroll 1
-  for (; k + 7 < k1; k += 8) {
+  for (; k + G - 1 < k1; k += G) {
     const int k3 = (k >> 2) * 3;
-    const float4 v0 = T4[k3], v1 = T4[k3 + 1], v2 = T4[k3 + 2], v3 = T4[k3 + 3], v4 = T4[k3 + 4], v5 = T4[k3 + 5];
-    const float xs[8] = {v0.x, v0.w, v1.z, v2.y, v3.x, v3.w, v4.z, v5.y};
-    const float ys[8] = {v0.y, v1.x, v1.w, v2.z, v3.y, v4.x, v4.w, v5.z};
-    const float zs[8] = {v0.z, v1.y, v2.x, v2.w, v3.z, v4.y, v5.x, v5.w};
-    uint32_t a[8], b[8];
+    float xs[G], ys[G], zs[G];
 #pragma unroll
-    for (int u = 0; u < 8; ++u) {
-      a[u] = tp_hb<LUT>(lb, Es, tp_dot(A, xs[u], ys[u], zs[u]));
-      b[u] = tp_hb<LUT>(lb, Es, tp_dot(B, xs[u], ys[u], zs[u]));
+    for (int q = 0; q < G / 4; ++q) {
+      const float4 v0 = T4[k3 + 3 * q], v1 = T4[k3 + 3 * q + 1], v2 = T4[k3 + 3 * q + 2];
+      xs[4 * q] = v0.x; ys[4 * q] = v0.y; zs[4 * q] = v0.z;
+      xs[4 * q + 1] = v0.w; ys[4 * q + 1] = v1.x; zs[4 * q + 1] = v1.y;
+      xs[4 * q + 2] = v1.z; ys[4 * q + 2] = v1.w; zs[4 * q + 2] = v2.x;
+      xs[4 * q + 3] = v2.y; ys[4 * q + 3] = v2.z; zs[4 * q + 3] = v2.w;
     }
+    uint32_t b[NP][G];
 #pragma unroll
-    for (int u = 0; u < 8; ++u) {
-      red_shared(Hl + a[u], incA);
-      red_shared(Hl + b[u], incB);
-    }
+    for (int u = 0; u < G; ++u)
+#pragma unroll
+      for (int kk = 0; kk < NP; ++kk) b[kk][u] = tp_b4<LUT>(c.L, c.eb, c.Es, tp_dot(P[kk], xs[u], ys[u], zs[u]));
+#pragma unroll
+    for (int u = 0; u < G; ++u)
+#pragma unroll
+      for (int kk = 0; kk < NP; ++kk) red_shared(Hw[kk / 2] + b[kk][u] * 32u, inc[kk]);
     if (CNT) {
 #pragma unroll
-      for (int u = 0; u < 8; u += 2) {
-        A.acc += (int32_t)(a[u] + a[u + 1]);
-        B.acc += (int32_t)(b[u] + b[u + 1]);
+      for (int kk = 0; kk < NP; ++kk) {
+#pragma unroll
+        for (int u = 0; u < G; u += 2) P[kk].acc += (int32_t)(b[kk][u] + b[kk][u + 1]);
+        P[kk].cnt = count_inc(P[kk].cnt, G == 8 ? p.eight : (G == 4 ? p.four : p.one * G));
       }
-      A.cnt = count_inc(A.cnt, p.eight);
-      B.cnt = count_inc(B.cnt, p.eight);
     }
   }
-  for (; k < k1; ++k) tp_pair1<CNT, LUT>(Hl, lb, Es, A, B, incA, incB, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], true, true);
+  for (; k < k1; ++k) tp_pair1<NP, CNT, LUT>(c, Hw, P, inc, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], 0, false);
 }
 
-template <bool CNT, bool LUT>
-__device__ __forceinline__ void tp_pairs_masked(const float* __restrict__ Bt, uint32_t Hl, uint32_t lb, const float* Es,
-                                                TPPoint& A, TPPoint& B, uint32_t incA, uint32_t incB, int k0, int k1,
-                                                int jt0) {
-#pragma unroll 2
-  for (int k = k0; k < k1; ++k) {
-    const int j = jt0 + k;
-    tp_pair1<CNT, LUT>(Hl, lb, Es, A, B, incA, incB, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], j >= A.jb, j >= B.jb);
-  }
-}
-
-// One work item: the points [i0, i0 + 512) of histogram h (point A = i0 + t, B = i0 + 256 + t)
-// against partners [jr0, jr1) (already clipped to [jlo, N)), streamed tile by tile.  The
-// tables are staged and the histogram zeroed by the caller.  Returns with every tile consumed.
-template <int V, bool LUT>
-__device__ __forceinline__ void tp_item_loop(const TPParams& p, const TPSmem& S, TPPoint& A, TPPoint& B, uint32_t incA,
-                                             uint32_t incB, int h, int i0, int jr0, int jr1) {
+// One work item: the points i0 + t + 128 k (k < NP) of histogram h against partners [jr0, jr1)
+// (already clipped to the block's [jlo, N)), streamed tile by tile through the ring.  The tables
+// are staged and the histogram zeroed by the caller.
+template <int NP, int V, bool LUT>
+__device__ __forceinline__ void tp_item_loop(const TPParams& p, const TPSmem& S, TPPoint (&P)[NP], const uint32_t (&inc)[NP],
+                                             int h, int i0, int jr0, int jr1) {
   constexpr bool CNT = (V & (V_L | V_PROF)) != 0;
   const int sb = (h == 0) ? 0 : (h <= p.nr ? h : h - p.nr);
   const int js = jr0 & ~3;  // tiles start on 4-partner boundaries (16-byte aligned groups in smem)
   const int nt = jr1 > jr0 ? (jr1 - js + TP_TILE - 1) / TP_TILE : 0;
   // partners below jall need per-point masks (self rows: j >= i + 1), the rest do not
-  const int jall = h <= p.nr ? min(i0 + TP_CTA_PTS, p.n) : 0;
+  const int jall = h <= p.nr ? min(i0 + NP * TP_THREADS, p.n) : 0;
   const uint32_t lane = lane_id(), warp = threadIdx.x >> 5;
-  const uint32_t Hl = smem_u32(S.H + ((size_t)warp * (p.nb + 2)) * 32 + lane);
-  const uint32_t lb = smem_u32(S.L);
+  uint32_t Hw[NP / 2];
+#pragma unroll
+  for (int w = 0; w < NP / 2; ++w) Hw[w] = smem_u32(S.H + (((size_t)warp * (NP / 2) + w) * (p.nb + 2)) * 32 + lane);
+  const TPLoopCtx c{S.L, smem_u32(S.E), S.E};
   if (nt > 0) tp_stage_tile(p, S, sb, js, min(TP_TILE, p.n - js), 0);
   for (int t = 0; t < nt; ++t) {
     const int jt0 = js + t * TP_TILE;
@@ -414,9 +434,25 @@ __device__ __forceinline__ void tp_item_loop(const TPParams& p, const TPSmem& S,
     const float* Bt = S.B + (t & 1) * 3 * TP_TILE;
     const int k0 = max(jr0, jt0) - jt0, k1 = min(jr1, jt0 + TP_TILE) - jt0;
     const int km = min(max(jall - jt0, k0), k1);  // [k0, km): masked, [km, k1): all points
-    if (km > k0) tp_pairs_masked<CNT, LUT>(Bt, Hl, lb, S.E, A, B, incA, incB, k0, km, jt0);
-    tp_pairs_all<CNT, LUT>(p, Bt, Hl, lb, S.E, A, B, incA, incB, km, k1);
+#pragma unroll 1
+    for (int k = k0; k < km; ++k) tp_pair1<NP, CNT, LUT>(c, Hw, P, inc, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], jt0 + k, true);
+    tp_pairs_all<NP, CNT, LUT>(p, c, Bt, Hw, P, inc, km, k1);
     __syncthreads();  // slot t & 1 is refilled by the stage of tile t + 2
+  }
+}
+
+template <int NP>
+__device__ __forceinline__ void tp_points(const TPParams& p, const unsigned long long* hist, int h, int blk, int64_t g0,
+                                          int64_t g1, TPPoint (&P)[NP], bool nl) {
+  const int i0 = blk * NP * TP_THREADS;
+  const int64_t gb = (int64_t)h * p.n;
+#pragma unroll
+  for (int k = 0; k < NP; ++k) {
+    const int i = i0 + k * TP_THREADS + threadIdx.x;
+    const bool v = i < p.n && gb + i >= g0 && gb + i < g1;
+    const int idup = (int)((blk ^ p.z) * (NP * TP_THREADS) + k * TP_THREADS + (threadIdx.x ^ p.z));
+    P[k] = nl ? tp_prologue<true>(p, hist, h, i, idup, (int)((uint32_t)h ^ p.z), v)
+              : tp_prologue<false>(p, hist, h, i, idup, (int)((uint32_t)h ^ p.z), v);
   }
 }
 
@@ -443,32 +479,32 @@ __device__ __forceinline__ int tp_claim(const TPSched& q, int sl) {
 
 template <int V, bool LUT>
 __device__ __forceinline__ void tp_single_item(const TPParams& p, const TPSmem& S, int4 it) {
+  constexpr int NP = HK_TP_NP_SR;
   constexpr bool NL = (V & V_NL) != 0, L = (V & V_L) != 0, PROF = (V & V_PROF) != 0, CNT = L || PROF;
   const int blk = it.x, h = it.y, c = it.z, nitems = it.w;
-  const int i0 = blk * TP_CTA_PTS;
+  const int i0 = blk * NP * TP_THREADS;
   const int64_t gb = (int64_t)h * p.n;
-  const int iA = i0 + threadIdx.x, iB = iA + TP_THREADS;
-  const bool va = iA < p.n && gb + iA >= p.g0 && gb + iA < p.g1, vb = iB < p.n && gb + iB >= p.g0 && gb + iB < p.g1;
-  const int idA = (int)((blk ^ p.z) * TP_CTA_PTS + (threadIdx.x ^ p.z)), idB = idA + TP_THREADS;
-  TPPoint A = tp_prologue<NL>(p, p.hist, h, iA, idA, (int)((uint32_t)h ^ p.z), va);
-  TPPoint B = tp_prologue<NL>(p, p.hist, h, iB, idB, (int)((uint32_t)h ^ p.z), vb);
-  if (!va) A.jb = INT32_MAX;
-  if (!vb) B.jb = INT32_MAX;
+  TPPoint P[NP];
+  tp_points<NP>(p, p.hist, h, blk, p.g0, p.g1, P, NL);
+  uint32_t inc[NP];
+#pragma unroll
+  for (int k = 0; k < NP; ++k) inc[k] = P[k].valid ? ((k & 1) ? 0x10000u : 1u) : 0u;
   const int jlo = h <= p.nr ? i0 + 1 : 0;
   const int jr0 = max(jlo, c * TP_TILE), jr1 = min(p.n, (c + 1) * TP_TILE);
-  tp_zero_hist(p, S);
+  tp_zero_hist<NP>(p, S);
   __syncthreads();
-  tp_item_loop<V, LUT>(p, S, A, B, va ? 1u : 0u, vb ? 0x10000u : 0u, h, i0, jr0, jr1);
-  A.acc /= (int32_t)TP_HB;
-  B.acc /= (int32_t)TP_HB;
-  tp_nl_exit<NL>(p, A, p.hist);
-  tp_nl_exit<NL>(p, B, p.hist);
-  if (CNT) {  // exact integer combine of this chunk's partial sums
-    if (va && A.cnt) { atomicAdd(p.accg + gb + iA, A.acc); atomicAdd(p.cntg + gb + iA, A.cnt); }
-    if (vb && B.cnt) { atomicAdd(p.accg + gb + iB, B.acc); atomicAdd(p.cntg + gb + iB, B.cnt); }
+  tp_item_loop<NP, V, LUT>(p, S, P, inc, h, i0, jr0, jr1);
+#pragma unroll
+  for (int k = 0; k < NP; ++k) {
+    P[k].acc /= 4;
+    tp_nl_exit<NL>(p, P[k], p.hist);
+    if (CNT && P[k].valid && P[k].cnt) {  // exact integer combine of this chunk's partial sums
+      atomicAdd(p.accg + gb + P[k].i, P[k].acc);
+      atomicAdd(p.cntg + gb + P[k].i, P[k].cnt);
+    }
   }
   __syncthreads();  // every thread's combine atomics issued; the ring is free for the flush
-  tp_flush(p, S, p.hist, h * (p.nb + 2));
+  tp_flush<NP>(p, S, p.hist, h * (p.nb + 2));
   if (CNT) {
     if (threadIdx.x == 0) {
       __threadfence();
@@ -477,21 +513,19 @@ __device__ __forceinline__ void tp_single_item(const TPParams& p, const TPSmem& 
     __syncthreads();
     if (*S.flag) {  // last chunk item of this (h, block): the loop-exit checks of its points
       __threadfence();
-      if (va) {
-        A.acc = __ldcg(p.accg + gb + iA);
-        A.cnt = __ldcg(p.cntg + gb + iA);
-        tp_checks<V>(p, A, p.cb, gb + iA);
-      }
-      if (vb) {
-        B.acc = __ldcg(p.accg + gb + iB);
-        B.cnt = __ldcg(p.cntg + gb + iB);
-        tp_checks<V>(p, B, p.cb, gb + iB);
-      }
+#pragma unroll
+      for (int k = 0; k < NP; ++k)
+        if (P[k].valid) {
+          P[k].acc = __ldcg(p.accg + gb + P[k].i);
+          P[k].cnt = __ldcg(p.cntg + gb + P[k].i);
+          tp_checks<V>(p, P[k], p.cb, gb + P[k].i);
+        }
     }
   }
   if (NL || L) {
-    if (va) fold_alarm(p.cb, A.alarm, (uint32_t)(gb + iA));
-    if (vb) fold_alarm(p.cb, B.alarm, (uint32_t)(gb + iB));
+#pragma unroll
+    for (int k = 0; k < NP; ++k)
+      if (P[k].valid) fold_alarm(p.cb, P[k].alarm, (uint32_t)(gb + P[k].i));
   }
   __syncthreads();  // shared histogram / flag reused by the next item
 }
@@ -513,10 +547,10 @@ __device__ __forceinline__ void tp_drain(const TPParams& p, const TPSmem& S, con
 }
 
 template <int V>
-__global__ void __launch_bounds__(TP_THREADS, HK_TP_MINB) tpacf_kernel(const TPParams p, const TPSched q) {
+__global__ void __launch_bounds__(TP_THREADS, HK_TP_MINB_SR) tpacf_kernel(const TPParams p, const TPSched q) {
   extern __shared__ __align__(16) unsigned char tp_smem[];
   __shared__ int item_s, last_s;
-  const TPSmem S = tp_carve(tp_smem, p.nb + 2);
+  const TPSmem S = tp_carve(tp_smem, p.nb + 2, HK_TP_NP_SR);
   tp_stage_tables(p, S);
   cp_async_wait<0>();
   __syncthreads();
@@ -710,48 +744,234 @@ done:
   K.finish(mine, alarm, fail, margin, gap, applied, (uint32_t)g);
 }
 
+// The same per-thread FI program, evaluated by the 32 lanes of one warp: lane l evaluates loop
+// iteration it0 + l of the ONE faulted abstract thread.  The program's state at iteration `it` is
+// a closed form of it (j = jb + it, the live values constant) except for the single flip at
+// iteration f.inst, which changes the live state from then on (kinds J / LIVE) or one iteration's
+// temporaries (X2 .. HIDX) or the running sums (ACC, CNT); so every lane can compute its own
+// iteration directly.  The first iteration E (ballot) holding an event — loop exit, R17 watchdog,
+// R16 crash, in the sequential order of the checks — ends the program exactly where the sequential
+// loop would: iterations before E add their histogram increment and their bin; acc and cnt are
+// rebuilt from the per-lane sums with the flip applied at its instance.  Results are identical to
+// tpacf_fi_program (the replay kernel runs that one; GPU replay == replica is tested) at ~1/32 of
+// its latency-bound time — a corrupted loop may run 10x the golden trips before the watchdog.
+template <int KIND, bool FT, bool LUT>
+__device__ void tpacf_fi_warp(const TPParams& p, const TPSmem& S, const FaultRec& f, int32_t hh, int32_t ii, int32_t i_dup,
+                              int32_t h_dup, uint64_t hist_real, hk_control* cb) {
+  const unsigned FULL = 0xffffffffu;
+  const uint32_t lane = lane_id();
+  const uint32_t z = p.z;
+  const int32_t nr = p.nr, nb2 = p.nb + 2;
+  const int64_t g = (int64_t)hh * p.n + ii;
+  const int64_t inst = f.inst;
+  const uint64_t mask = f.mask;
+  const int site = f.site;
+  const int64_t npts = 3LL * (1 + nr) * p.n, nhist = (int64_t)(1 + 2 * nr) * nb2;
+  const uint64_t pts_real = (uint64_t)(uintptr_t)p.pts;
+  uint32_t chk = 0, alarm = 0, fail = 0, margin = 0xffffffffu;
+  float gap = __int_as_float(0x7f800000);
+  bool applied = false;
+  int32_t n = p.n;
+  uint64_t ppts = pts_real, phist = hist_real;
+  // ---- prologue (uniform over the warp; DESIGN §3.4 NL sites 0-10)
+  if (FT) chk ^= (uint32_t)n ^ lohi(ppts) ^ lohi(phist);
+  const bool nl = (KIND == TK_NL);
+#define NLF(v, s) do { const bool _n = nl && site == (s); applied |= _n; v = flip_i(v, _n, mask); } while (0)
+  int32_t i = ii; NLF(i, 0);
+  if (FT) { chk ^= (uint32_t)i; alarm |= (i_dup != i) ? AL_DUP : 0u; }
+  int32_t h = hh; NLF(h, 1);
+  if (FT) { chk ^= (uint32_t)h; alarm |= (h_dup != h) ? AL_DUP : 0u; }
+  auto f_aoff = [&](int32_t hq, int32_t iq) { return (int32_t)((uint32_t)(hq <= nr ? hq : 0) * (uint32_t)n + (uint32_t)iq); };
+  auto f_boff = [&](int32_t hq) { return (int32_t)((uint32_t)(hq == 0 ? 0 : (hq <= nr ? hq : (int32_t)((uint32_t)hq - (uint32_t)nr))) * (uint32_t)n); };
+  auto f_jb = [&](int32_t hq, int32_t iq) { return hq <= nr ? (int32_t)((uint32_t)iq + 1u) : 0; };
+  auto f_ex = [&](int32_t je_, int32_t jb_) { const int32_t d = (int32_t)((uint32_t)je_ - (uint32_t)jb_); return d > 0 ? d : 0; };
+  int32_t aoff = f_aoff(h, i); NLF(aoff, 2);
+  if (FT) { chk ^= (uint32_t)aoff; alarm |= (f_aoff(opq(h, z), opq(i, z)) != aoff) ? AL_DUP : 0u; }
+  int32_t boff = f_boff(h); NLF(boff, 3);
+  if (FT) { chk ^= (uint32_t)boff; alarm |= (f_boff(opq(h, z)) != boff) ? AL_DUP : 0u; }
+  int32_t jb = f_jb(h, i); NLF(jb, 4);
+  if (FT) { chk ^= (uint32_t)jb; alarm |= (f_jb(opq(h, z), opq(i, z)) != jb) ? AL_DUP : 0u; }
+  int32_t je = n; NLF(je, 5);
+  if (FT) { chk ^= (uint32_t)je; alarm |= (opq(n, z) != je) ? AL_DUP : 0u; }
+  int32_t expect = f_ex(je, jb); NLF(expect, 6);
+  if (FT) { chk ^= (uint32_t)expect; alarm |= (f_ex(opq(je, z), jb) != expect) ? AL_DUP : 0u; }
+  int32_t base = (int32_t)((uint32_t)h * (uint32_t)nb2); NLF(base, 7);
+  if (FT) { chk ^= (uint32_t)base; alarm |= ((int32_t)((uint32_t)opq(h, z) * (uint32_t)nb2) != base) ? AL_DUP : 0u; }
+#undef NLF
+  float q1[3] = {0.f, 0.f, 0.f};
+  for (int a = 0; a < 3; ++a) {
+    const float* pe;
+    if (!fi_at(false, ppts, pts_real, (int32_t)((uint32_t)aoff * 3u + (uint32_t)a), npts, &pe)) { fail |= FL_CRASH; break; }
+    float v = __ldg(pe);
+    { const bool nn = nl && site == 8 + a; applied |= nn; v = flip_f(v, nn, mask); }
+    if (FT) { chk ^= fb(v); alarm |= (fb(__ldg(pe + z)) != fb(v)) ? AL_DUP : 0u; }
+    q1[a] = v;
+  }
+  if (!fail) {
+    if (FT) chk ^= (uint32_t)opq(i, z) ^ (uint32_t)opq(h, z) ^ (uint32_t)opq(aoff, z) ^ (uint32_t)opq(jb, z);
+    // ---- the live state after the flip (kinds J / LIVE), in force from iteration inst on
+    int32_t boff2 = boff, je2 = je, expect2 = expect, base2 = base, n2 = n;
+    float q12[3] = {q1[0], q1[1], q1[2]};
+    uint64_t ppts2 = ppts, phist2 = phist;
+    if (KIND == TK_LIVE) {
+      switch (site) {
+        case 11: boff2 = flip_i(boff, true, mask); break;
+        case 12: je2 = flip_i(je, true, mask); break;
+        case 13: expect2 = flip_i(expect, true, mask); break;
+        case 14: base2 = flip_i(base, true, mask); break;
+        case 15: q12[0] = flip_f(q1[0], true, mask); break;
+        case 16: q12[1] = flip_f(q1[1], true, mask); break;
+        case 17: q12[2] = flip_f(q1[2], true, mask); break;
+        case 18: n2 = flip_i(n, true, mask); break;
+        case 19: ppts2 = flip_p(ppts, true, mask); break;
+        case 20: phist2 = flip_p(phist, true, mask); break;
+        default: break;
+      }
+    }
+    const int32_t jflip = (int32_t)((uint32_t)jb + (uint32_t)inst) ^ (int32_t)(uint32_t)mask;  // J: j at iteration inst
+    const int64_t golden = hh <= nr ? (int64_t)p.n - (ii + 1) : (int64_t)p.n;  // uncorrupted launch indices (R17)
+    const int64_t limit = fi_limit<false>(golden, f.hang);
+    int64_t E = -1;
+    int etype = 0;      // 1 exit, 2 hang, 3 crash in the partner loads, 4 crash at the histogram
+    uint32_t s_le = 0, s_gt = 0;  // this lane's bins of iterations <= inst / > inst (before E)
+    const uint32_t lb = smem_u32(S.E);
+    for (int64_t it0 = 0; E < 0; it0 += 32) {
+      const int64_t it = it0 + lane;
+      const bool post = (KIND == TK_J || KIND == TK_LIVE) && it >= inst;
+      const bool now = it == inst;
+      int32_t j = (int32_t)((uint32_t)jb + (uint32_t)it);
+      if (KIND == TK_J && post) j = (int32_t)((uint32_t)jflip + (uint32_t)(it - inst));
+      const int32_t bo = post ? boff2 : boff, jee = post ? je2 : je, ba = post ? base2 : base;
+      const uint64_t pp = post ? ppts2 : ppts, ph = post ? phist2 : phist;
+      const float x1 = post ? q12[0] : q1[0], y1 = post ? q12[1] : q1[1], z1 = post ? q12[2] : q1[2];
+      int ev = 0;
+      uint32_t bin = 0;
+      unsigned long long* hp = nullptr;
+      if (!(j < jee)) ev = 1;
+      else if (it >= limit) ev = 2;
+      else {
+        const int32_t pb = (int32_t)(3u * (uint32_t)((uint32_t)bo + (uint32_t)j));
+        float q2[3];
+        for (int a = 0; a < 3 && !ev; ++a) {
+          const float* pe;
+          if (!fi_at(false, pp, pts_real, (int32_t)((uint32_t)pb + (uint32_t)a), npts, &pe)) ev = 3;
+          else q2[a] = __ldg(pe);
+        }
+        if (!ev) {
+          if (KIND == TK_X2) q2[0] = flip_f(q2[0], now, mask);
+          if (KIND == TK_Y2) q2[1] = flip_f(q2[1], now, mask);
+          if (KIND == TK_Z2) q2[2] = flip_f(q2[2], now, mask);
+          float dot = __fmaf_rn(z1, q2[2], __fmaf_rn(y1, q2[1], __fmul_rn(x1, q2[0])));
+          if (KIND == TK_DOT) dot = flip_f(dot, now, mask);
+          bin = LUT ? tp_b4_lut(S.L, lb, dot) / 4u : (uint32_t)tp_bin_search(S.E, dot);
+          if (KIND == TK_BIN) bin = (uint32_t)flip_i((int32_t)bin, now, mask);
+          int32_t hidx = (int32_t)((uint32_t)ba + bin);
+          if (KIND == TK_HIDX) hidx = flip_i(hidx, now, mask);
+          if (!fi_at(false, ph, hist_real, hidx, nhist, &hp)) ev = 4;
+        }
+      }
+      const unsigned evs = __ballot_sync(FULL, ev != 0);
+      const int first = evs ? __ffs(evs) - 1 : 32;
+      if ((int)lane < first) {  // iterations before the first event: executed in full
+        red_add(hp, 1ull);
+        if (it <= inst) s_le += bin;
+        else s_gt += bin;
+      }
+      if (evs) {
+        E = it0 + first;
+        etype = __shfl_sync(FULL, ev, first);
+      }
+    }
+    s_le = __reduce_add_sync(FULL, s_le);
+    s_gt = __reduce_add_sync(FULL, s_gt);
+    // hooks of iteration inst that ran (the checks of iteration E precede its loads / increment)
+    if (KIND == TK_J || KIND == TK_LIVE) applied = inst <= E;
+    if (KIND == TK_X2 || KIND == TK_Y2 || KIND == TK_Z2 || KIND == TK_DOT || KIND == TK_BIN || KIND == TK_HIDX)
+      applied = inst < E || (inst == E && etype == 4);
+    if (KIND == TK_ACC || KIND == TK_CNT) applied = inst < E;
+    if (etype == 2) fail |= FL_HANG;
+    if (etype >= 3) fail |= FL_CRASH;
+    if (!fail && FT) {
+      const bool in_force = (KIND == TK_J || KIND == TK_LIVE) && inst <= E;  // the exit sees the flipped state
+      const int32_t boffx = in_force ? boff2 : boff, jex = in_force ? je2 : je, basex = in_force ? base2 : base;
+      const int32_t expx = in_force ? expect2 : expect, nx = in_force ? n2 : n;
+      const float x1x = in_force ? q12[0] : q1[0], y1x = in_force ? q12[1] : q1[1], z1x = in_force ? q12[2] : q1[2];
+      const uint64_t ppx = in_force ? ppts2 : ppts, phx = in_force ? phist2 : phist;
+      const int32_t acc = (KIND == TK_ACC && inst < E) ? (int32_t)(((s_le) ^ (uint32_t)mask) + s_gt) : (int32_t)(s_le + s_gt);
+      const int32_t cnt = (KIND == TK_CNT && inst < E) ? (int32_t)((((uint32_t)inst + 1u) ^ (uint32_t)mask) + (uint32_t)(E - 1 - inst))
+                                                        : (int32_t)E;
+      if (cnt != expx) alarm |= AL_COUNT;
+      if (cnt != 0 && p.ndet > 0 && p.R.n[0] > 0) {
+        const float v = __fdiv_rn((float)acc, (float)cnt);
+        if (!in_range<true>(p.R, 0, v, &margin, &gap)) {
+          alarm |= AL_RANGE;
+          if (lane == 0) record_outlier(cb, 0, v);
+        }
+      }
+      chk ^= (uint32_t)opq(boffx, z) ^ (uint32_t)opq(jex, z) ^ (uint32_t)opq(basex, z);
+      chk ^= opqf(x1x, z) ^ opqf(y1x, z) ^ opqf(z1x, z) ^ (uint32_t)opq(expx, z);
+      chk ^= ((uint32_t)nx + z) ^ (lohi(ppx) + z) ^ (lohi(phx) + z);
+      if (chk != 0) alarm |= AL_CHK;
+    }
+  }
+  if (!FT) alarm = 0;
+  if (lane == 0) {
+    TPReplicaSink K{cb};
+    K.finish(true, alarm, fail, margin, gap, applied, (uint32_t)g);
+  }
+}
+
 // Replica CTA (h, point block) of the FI kernel, whole partner loops.  The faulted abstract thread
 // (if this CTA holds it) takes no part in the fast loop (increment 0, no exit checks); after the
 // CTA's histogram flush its owning CUDA thread runs the FI program over the whole partner range.
 template <int KIND, bool FT, bool LUT>
 __device__ __forceinline__ void tp_replica_cta(const TPFIParams& q, const TPSmem& S, const FaultRec& f, unsigned long long* hist,
                                                hk_control* cb, int h, int blk, bool faulted) {
+  constexpr int NP = HK_TP_NP_FI;
   constexpr int V = FT ? (V_NL | V_L) : 0;
   constexpr bool NL = FT, L = FT;
   TPParams p = q.base;
   p.hist = hist;
   p.cb = cb;
-  const int i0 = blk * TP_CTA_PTS;
+  const int i0 = blk * NP * TP_THREADS;
   const int64_t gb = (int64_t)h * p.n;
-  const int iA = i0 + threadIdx.x, iB = iA + TP_THREADS;
-  const bool va = iA < p.n, vb = iB < p.n;
-  const bool fa = faulted && gb + iA == f.thread, fbb = faulted && gb + iB == f.thread;
-  const int idA = (int)((blk ^ p.z) * TP_CTA_PTS + (threadIdx.x ^ p.z)), idB = idA + TP_THREADS;
-  TPPoint A = tp_prologue<NL>(p, hist, h, iA, idA, (int)((uint32_t)h ^ p.z), va);
-  TPPoint B = tp_prologue<NL>(p, hist, h, iB, idB, (int)((uint32_t)h ^ p.z), vb);
-  if (!va) A.jb = INT32_MAX;
-  if (!vb) B.jb = INT32_MAX;
-  tp_zero_hist(p, S);
+  TPPoint P[NP];
+  tp_points<NP>(p, hist, h, blk, 0, INT64_MAX, P, NL);
+  uint32_t inc[NP];
+  int fk = -1;  // which of this thread's points is the faulted abstract thread
+#pragma unroll
+  for (int k = 0; k < NP; ++k) {
+    const bool mine = faulted && P[k].valid && gb + P[k].i == f.thread;
+    if (mine) fk = k;
+    inc[k] = (P[k].valid && !mine) ? ((k & 1) ? 0x10000u : 1u) : 0u;
+  }
+  tp_zero_hist<NP>(p, S);
   __syncthreads();
   const int jlo = h <= p.nr ? i0 + 1 : 0;
-  tp_item_loop<V, LUT>(p, S, A, B, (va && !fa) ? 1u : 0u, (vb && !fbb) ? 0x10000u : 0u, h, i0, jlo, p.n);
-  if (L) {
-    A.acc /= (int32_t)TP_HB;
-    B.acc /= (int32_t)TP_HB;
+  tp_item_loop<NP, V, LUT>(p, S, P, inc, h, i0, jlo, p.n);
+#pragma unroll
+  for (int k = 0; k < NP; ++k) {
+    if (!P[k].valid || k == fk) continue;
+    if (L) P[k].acc /= 4;
+    tp_nl_exit<NL>(p, P[k], hist);
+    tp_checks<V>(p, P[k], cb, gb + P[k].i);
   }
-  if (va && !fa) { tp_nl_exit<NL>(p, A, hist); tp_checks<V>(p, A, cb, gb + iA); }
-  if (vb && !fbb) { tp_nl_exit<NL>(p, B, hist); tp_checks<V>(p, B, cb, gb + iB); }
   if (NL || L) {
-    if (va) fold_alarm(cb, fa ? 0u : A.alarm, (uint32_t)(gb + iA));
-    if (vb) fold_alarm(cb, fbb ? 0u : B.alarm, (uint32_t)(gb + iB));
+#pragma unroll
+    for (int k = 0; k < NP; ++k)
+      if (P[k].valid) fold_alarm(cb, k == fk ? 0u : P[k].alarm, (uint32_t)(gb + P[k].i));
   }
   __syncthreads();
-  tp_flush(p, S, hist, h * (p.nb + 2));
-  if (fa || fbb) {
-    const int ii = fa ? iA : iB;
-    const int idup = fa ? idA : idB;
-    TPReplicaSink K{cb};
-    tpacf_fi_program<KIND, FT>(p, S.E, f, h, ii, idup, (int)((uint32_t)h ^ p.z), true, (uint64_t)(uintptr_t)hist, K);
+  tp_flush<NP>(p, S, hist, h * (p.nb + 2));
+  // the warp holding the faulted abstract thread runs its FI program, 32 iterations at a time
+  const unsigned own = __ballot_sync(0xffffffffu, fk >= 0);
+  if (own) {
+    const int src = __ffs(own) - 1;
+    const int fkw = __shfl_sync(0xffffffffu, fk, src);
+    const int t = (int)(threadIdx.x & ~31u) + src;
+    const int ii = i0 + fkw * TP_THREADS + t;
+    const int idup = (int)((blk ^ p.z) * (NP * TP_THREADS) + fkw * TP_THREADS + (t ^ (int)p.z));
+    tpacf_fi_warp<KIND, FT, LUT>(p, S, f, h, ii, idup, (int)((uint32_t)h ^ p.z), (uint64_t)(uintptr_t)hist, cb);
   }
 }
 
@@ -769,7 +989,8 @@ template <int KIND, bool FT>
 __global__ void __launch_bounds__(TP_THREADS, HK_TP_MINB) tpacf_fi_kernel(const TPFIParams q) {
   extern __shared__ __align__(16) unsigned char tp_smem[];
   const TPParams& p0 = q.base;
-  const TPSmem S = tp_carve(tp_smem, p0.nb + 2);
+  constexpr int CPTS = HK_TP_NP_FI * TP_THREADS;
+  const TPSmem S = tp_carve(tp_smem, p0.nb + 2, HK_TP_NP_FI);
   // launch slot (x = replica, y = 0: its faulted CTA, y = 1 + rank: CTA of that rank)
   const int r = (int)blockIdx.x;
   int h, blk;
@@ -777,12 +998,12 @@ __global__ void __launch_bounds__(TP_THREADS, HK_TP_MINB) tpacf_fi_kernel(const 
   if (blockIdx.y == 0) {
     const int64_t g = q.faults[r].thread;
     h = (int)(g / p0.n);
-    blk = (int)((g % p0.n) / TP_CTA_PTS);
+    blk = (int)((g % p0.n) / CPTS);
     faulted = true;
   } else {
     tp_cta_of_rank((int)blockIdx.y - 1, p0.nr, p0.nblk, &h, &blk);
     const int64_t g = q.faults[r].thread;
-    if (h == (int)(g / p0.n) && blk == (int)((g % p0.n) / TP_CTA_PTS)) return;  // ran in the first slots
+    if (h == (int)(g / p0.n) && blk == (int)((g % p0.n) / CPTS)) return;  // ran in the first slots
     faulted = false;
   }
   const FaultRec f = q.faults[r];
@@ -893,15 +1114,15 @@ __global__ void __launch_bounds__(128) tpacf_replay_all_kernel(const TPReplayPar
 // ============================================================================================
 // Host launchers
 // ============================================================================================
-static int tp_nblk(int n) { return (n + TP_CTA_PTS - 1) / TP_CTA_PTS; }
+static int tp_nblk(int n, int np) { return (n + np * TP_THREADS - 1) / (np * TP_THREADS); }
 
 static TPParams tp_params(const hk_tpacf_args& a, const DevRanges& R, int ndet, hk_control* cb, float* samples,
                           void* ws) {
   TPParams p{};
   p.pts = a.pts;
   p.edges = a.edges;
-  p.lut = reinterpret_cast<const uint2*>(ws);
-  p.lut_ok = reinterpret_cast<const int*>(reinterpret_cast<const char*>(ws) + TP_LUT * 8);
+  p.lut = reinterpret_cast<const uint8_t*>(ws);
+  p.lut_ok = reinterpret_cast<const int*>(reinterpret_cast<const char*>(ws) + TP_LUT);
   p.hist = a.hist;
   p.cb = cb;
   p.samples = samples;
@@ -910,28 +1131,29 @@ static TPParams tp_params(const hk_tpacf_args& a, const DevRanges& R, int ndet, 
   p.nr = a.n_rand;
   p.nb = a.n_bins;
   p.ndet = ndet;
-  p.nblk = tp_nblk(a.n);
+  p.nblk = tp_nblk(a.n, HK_TP_NP_SR);
   p.g0 = 0;
   p.g1 = (1 + 2 * a.n_rand) * a.n;
   p.z = opaque_zero();
   p.one = 1 + (int32_t)opaque_zero();
+  p.four = 4 * p.one;
   p.eight = 8 * p.one;
   return p;
 }
 
 // Workspace (tpacf_ws_bytes): table [TP_LUT] uint2 | ok flag (16 B) | schedule counters
 // next[TP_SCHED_MAX_SM], claimed, exited | accg [nh * N] | cntg [nh * N] | done [nh * nblk].
-static size_t tp_ws_head() { return (size_t)TP_LUT * 8 + 16 + (TP_SCHED_MAX_SM + 2) * sizeof(int); }
+static size_t tp_ws_head() { return (size_t)TP_LUT + 16 + (TP_SCHED_MAX_SM + 2) * sizeof(int); }
 size_t tpacf_ws_bytes(const hk_tpacf_args& a) {
-  const size_t nt = (size_t)(1 + 2 * a.n_rand) * (size_t)a.n, nd = (size_t)(1 + 2 * a.n_rand) * tp_nblk(a.n);
+  const size_t nt = (size_t)(1 + 2 * a.n_rand) * (size_t)a.n, nd = (size_t)(1 + 2 * a.n_rand) * tp_nblk(a.n, HK_TP_NP_SR);
   return tp_ws_head() + nt * 8 + nd * 4;
 }
 
 cudaError_t tpacf_lut_build(const hk_tpacf_args& a, void* ws, cudaStream_t s) {
-  int* ok = reinterpret_cast<int*>(reinterpret_cast<char*>(ws) + TP_LUT * 8);
+  int* ok = reinterpret_cast<int*>(reinterpret_cast<char*>(ws) + TP_LUT);
   cudaError_t e = cudaMemsetAsync(ok, 1, sizeof(int), s);
   if (e != cudaSuccess) return e;
-  tpacf_lut_kernel<<<TP_LUT / 256, 256, 0, s>>>(a.edges, a.n_bins, reinterpret_cast<uint2*>(ws), ok);
+  tpacf_lut_kernel<<<TP_LUT / 256, 256, 0, s>>>(a.edges, a.n_bins, reinterpret_cast<uint8_t*>(ws), ok);
   count_launch();
   return cudaGetLastError();
 }
@@ -983,12 +1205,13 @@ static cudaError_t tp_schedule(const hk_tpacf_args& a, int nsm, int g0, int g1, 
     cudaGetLastError();
     cache.erase(fnd);
   }
-  const int N = a.n, nr = a.n_rand, nh = 1 + 2 * nr, nblk = tp_nblk(N), nc = (N + TP_TILE - 1) / TP_TILE;
+  constexpr int CPTS = HK_TP_NP_SR * TP_THREADS;
+  const int N = a.n, nr = a.n_rand, nh = 1 + 2 * nr, nblk = tp_nblk(N, HK_TP_NP_SR), nc = (N + TP_TILE - 1) / TP_TILE;
   std::vector<std::pair<double, int4>> w;
   std::vector<int> per((size_t)nh * nblk, 0);
   for (int h = 0; h < nh; ++h)
     for (int b = 0; b < nblk; ++b) {
-      const int64_t i0 = (int64_t)b * TP_CTA_PTS, i1 = std::min<int64_t>(i0 + TP_CTA_PTS, N);
+      const int64_t i0 = (int64_t)b * CPTS, i1 = std::min<int64_t>(i0 + CPTS, N);
       const int64_t lo = std::max<int64_t>(i0, g0 - (int64_t)h * N), hi = std::min<int64_t>(i1, g1 - (int64_t)h * N);
       if (lo >= hi) continue;  // no abstract thread of this block is in the run's range
       const int64_t jlo = h <= nr ? i0 + 1 : 0;
@@ -1037,7 +1260,7 @@ static cudaError_t tp_schedule(const hk_tpacf_args& a, int nsm, int g0, int g1, 
 
 template <int V>
 static cudaError_t launch_tp_v(const hk_tpacf_args& a, TPParams p, void* ws, cudaStream_t s) {
-  const size_t smem = tp_smem_bytes(p.nb + 2);
+  const size_t smem = tp_smem_bytes(p.nb + 2, HK_TP_NP_SR);
   cudaError_t e = cudaFuncSetAttribute(tpacf_kernel<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   if (p.g1 <= p.g0) return cudaSuccess;
@@ -1052,7 +1275,7 @@ static cudaError_t launch_tp_v(const hk_tpacf_args& a, TPParams p, void* ws, cud
   TPSched q;
   q.items = B.items;
   q.off = B.off;
-  q.next = reinterpret_cast<int*>(w + TP_LUT * 8 + 16);
+  q.next = reinterpret_cast<int*>(w + TP_LUT + 16);
   q.claimed = q.next + TP_SCHED_MAX_SM;
   q.exited = q.claimed + 1;
   q.nsm = nsm;
@@ -1061,7 +1284,7 @@ static cudaError_t launch_tp_v(const hk_tpacf_args& a, TPParams p, void* ws, cud
   p.accg = reinterpret_cast<int32_t*>(w + tp_ws_head());
   p.cntg = p.accg + nt;
   p.done = p.cntg + nt;
-  if ((e = cudaMemsetAsync(w + TP_LUT * 8 + 16, 0, tpacf_ws_bytes(a) - (TP_LUT * 8 + 16), s)) != cudaSuccess) return e;
+  if ((e = cudaMemsetAsync(w + TP_LUT + 16, 0, tpacf_ws_bytes(a) - (TP_LUT + 16), s)) != cudaSuccess) return e;
   const int grid = nsm * std::max(1, std::min(per_sm, (B.total + nsm - 1) / nsm));
   TimedScope ts(HK_TPACF, 0, tp_pairs(a) * (double)(p.g1 - p.g0) / (double)((1 + 2 * p.nr) * p.n), s);
   tpacf_kernel<V><<<grid, TP_THREADS, smem, s>>>(p, q);
@@ -1091,7 +1314,7 @@ int tpacf_site_kind(int site) { return tpacf_site_kind_d(site); }
 
 template <int KIND, bool FT>
 static cudaError_t launch_tp_fi_k(const TPFIParams& q, int nrep, cudaStream_t s) {
-  const size_t smem = tp_smem_bytes(q.base.nb + 2);
+  const size_t smem = tp_smem_bytes(q.base.nb + 2, HK_TP_NP_FI);
   cudaError_t e = cudaFuncSetAttribute(tpacf_fi_kernel<KIND, FT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   const int ncta = (1 + 2 * q.base.nr) * q.base.nblk;
@@ -1126,6 +1349,7 @@ cudaError_t tpacf_fi_launch(int kind, bool ft, const hk_tpacf_args& a, const Dev
                             int nrep, unsigned long long* hist0, hk_control* cb0, void* ws, bool real, cudaStream_t s) {
   TPFIParams q{};
   q.base = tp_params(a, R, ndet, nullptr, nullptr, ws);
+  q.base.nblk = tp_nblk(a.n, HK_TP_NP_FI);
   q.faults = faults;
   q.hist0 = hist0;
   q.cb0 = cb0;

@@ -8,7 +8,7 @@
 // after the whole loop.  How the kernels tile that loop is not part of the program:
 //  * acc, cnt and the histogram are integer sums, so any split of a thread's partner range into
 //    pieces, added exactly, gives the same values as the one sequential loop;
-//  * the single run (tpacf_kernel) cuts the partner range into chunks of TP_TILE partners, adds the
+//  * the single run (tpacf_kernel) cuts the partner range into chunks of 256 partners, adds the
 //    per-chunk (acc, cnt) partials with global atomics, and the last chunk item of a point block
 //    (a per-(h, block) completion counter) runs CheckEqual / CheckRange for its points;
 //  * the campaign replicas (tpacf_fi_kernel) give each CTA whole loops (all partners of its
@@ -22,10 +22,6 @@
 // wavefronts each even as broadcasts, 32-bit LDS / ATOMS one), so the table stays byte-wide and
 // NP = 4 amortises the partner loads over four points.
 #include <algorithm>
-#include <array>
-#include <map>
-#include <mutex>
-#include <queue>
 #include <vector>
 
 #include "hk_internal.h"
@@ -44,6 +40,9 @@ namespace hk {
 #ifndef HK_TP_MINB_SR
 #define HK_TP_MINB_SR 8  // single run: 25.5 KB per CTA -> 8 CTAs per SM, 64 registers
 #endif
+#ifndef HK_TP_SR_CHUNK
+#define HK_TP_SR_CHUNK 128  // partners per single-run chunk (<= TP_TILE)
+#endif
 #ifndef HK_TP_GROUP
 #define HK_TP_GROUP 0  // partners per group of the unmasked loop (0: 4 for NP >= 4, else 8)
 #endif
@@ -51,7 +50,6 @@ constexpr int TP_THREADS = 128;
 constexpr int TP_WARPS = TP_THREADS / 32;
 constexpr int TP_TILE = 512;                // partners per shared-memory tile (6 KB)
 constexpr int TP_LUT = 2048;                // u-buckets: sign, 8 exponent bits, 2 mantissa bits
-constexpr int TP_SCHED_MAX_SM = 1024;
 
 struct TPParams {
   const float* pts;
@@ -64,7 +62,6 @@ struct TPParams {
   DevRanges R;
   int32_t* accg;          // single run: per abstract thread partial sums of acc and cnt (zeroed per run)
   int32_t* cntg;
-  int32_t* done;          // single run: chunk items finished per (h, point block)
   int32_t n, nr, nb, ndet;
   int32_t nblk;           // point blocks per histogram for the launching kernel's NP
   int32_t g0, g1;         // abstract threads [g0, g1) of this run (single-run sharding)
@@ -159,17 +156,18 @@ __global__ void tpacf_lut_kernel(const float* __restrict__ edges, int nb, uint8_
 
 // ---------------------------------------------------------------------------------------------
 // Shared memory: L[2048] u8 | E[32] f32 | B[2][3 * TP_TILE] f32 (packed x, y, z) |
-// H[warps][NP/2 words][nb2][32] u32 | flag
+// H[warps][NP/2 words][nb2][32] u32 | part[warps * NP/2 * nb2] | flag
 // ---------------------------------------------------------------------------------------------
 struct TPSmem {
   uint8_t* L;
   float* E;
   float* B;
   uint32_t* H;
+  uint32_t* part;  // [TP_WARPS * NP/2 * nb2] flush scratch (the ring may hold a prefetched tile)
   int* flag;
 };
 __host__ __device__ inline size_t tp_smem_bytes(int nb2, int np) {
-  return (size_t)TP_LUT + 32 * 4 + 2 * 3 * TP_TILE * 4 + (size_t)TP_WARPS * (np / 2) * nb2 * 32 * 4 + 16;
+  return (size_t)TP_LUT + 32 * 4 + 2 * 3 * TP_TILE * 4 + (size_t)TP_WARPS * (np / 2) * nb2 * 33 * 4 + 16;
 }
 __device__ __forceinline__ TPSmem tp_carve(unsigned char* base, int nb2, int np) {
   TPSmem S;
@@ -177,7 +175,8 @@ __device__ __forceinline__ TPSmem tp_carve(unsigned char* base, int nb2, int np)
   S.E = reinterpret_cast<float*>(base + TP_LUT);
   S.B = reinterpret_cast<float*>(base + TP_LUT + 128);
   S.H = reinterpret_cast<uint32_t*>(base + TP_LUT + 128 + 2 * 3 * TP_TILE * 4);
-  S.flag = reinterpret_cast<int*>(base + TP_LUT + 128 + 2 * 3 * TP_TILE * 4 + (size_t)TP_WARPS * (np / 2) * nb2 * 128);
+  S.part = reinterpret_cast<uint32_t*>(base + TP_LUT + 128 + 2 * 3 * TP_TILE * 4 + (size_t)TP_WARPS * (np / 2) * nb2 * 128);
+  S.flag = reinterpret_cast<int*>(reinterpret_cast<unsigned char*>(S.part) + (size_t)TP_WARPS * (np / 2) * nb2 * 4);
   return S;
 }
 __device__ __forceinline__ void cp_async4(void* dst, const void* src) {
@@ -215,7 +214,7 @@ __device__ __forceinline__ void tp_stage_tile(const TPParams& p, const TPSmem& S
 template <int NP>
 __device__ __forceinline__ void tp_flush(const TPParams& p, const TPSmem& S, unsigned long long* hist, int base) {
   const int nb2 = p.nb + 2, rows = TP_WARPS * (NP / 2);
-  uint32_t* part = reinterpret_cast<uint32_t*>(S.B);  // the ring is free at this point
+  uint32_t* part = S.part;
   for (int t = threadIdx.x; t < rows * nb2; t += TP_THREADS) {
     const uint32_t* row = S.H + (size_t)t * 32;
     uint32_t s = 0;
@@ -403,6 +402,24 @@ __device__ __forceinline__ void tp_pairs_all(const TPParams& p, const TPLoopCtx&
   for (; k < k1; ++k) tp_pair1<NP, CNT, LUT>(c, Hw, P, inc, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], 0, false);
 }
 
+// Pairs of the staged tile Bt (partners jt0 + k) for k in [k0, k1): [k0, km) with per-point masks
+// (partners below jall: the diagonal of a self-correlation row), [km, k1) for all points.
+template <int NP, bool CNT, bool LUT>
+__device__ __forceinline__ void tp_tile_pairs(const TPParams& p, const TPLoopCtx& c, const float* __restrict__ Bt,
+                                              const uint32_t (&Hw)[NP / 2], TPPoint (&P)[NP], const uint32_t (&inc)[NP],
+                                              int jt0, int k0, int k1, int jall) {
+  const int km = min(max(jall - jt0, k0), k1);
+#pragma unroll 1
+  for (int k = k0; k < km; ++k) tp_pair1<NP, CNT, LUT>(c, Hw, P, inc, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], jt0 + k, true);
+  tp_pairs_all<NP, CNT, LUT>(p, c, Bt, Hw, P, inc, km, k1);
+}
+template <int NP>
+__device__ __forceinline__ void tp_lane_hist(const TPParams& p, const TPSmem& S, uint32_t (&Hw)[NP / 2]) {
+  const uint32_t lane = lane_id(), warp = threadIdx.x >> 5;
+#pragma unroll
+  for (int w = 0; w < NP / 2; ++w) Hw[w] = smem_u32(S.H + (((size_t)warp * (NP / 2) + w) * (p.nb + 2)) * 32 + lane);
+}
+
 // One work item: the points i0 + t + 128 k (k < NP) of histogram h against partners [jr0, jr1)
 // (already clipped to the block's [jlo, N)), streamed tile by tile through the ring.  The tables
 // are staged and the histogram zeroed by the caller.
@@ -420,23 +437,19 @@ __device__ __forceinline__ void tp_item_loop(const TPParams& p, const TPSmem& S,
 #pragma unroll
   for (int w = 0; w < NP / 2; ++w) Hw[w] = smem_u32(S.H + (((size_t)warp * (NP / 2) + w) * (p.nb + 2)) * 32 + lane);
   const TPLoopCtx c{S.L, smem_u32(S.E), S.E};
-  if (nt > 0) tp_stage_tile(p, S, sb, js, min(TP_TILE, p.n - js), 0);
+  if (nt > 0) tp_stage_tile(p, S, sb, js, min(TP_TILE, jr1 - js), 0);
   for (int t = 0; t < nt; ++t) {
     const int jt0 = js + t * TP_TILE;
     if (t + 1 < nt) {
       const int jn = jt0 + TP_TILE;
-      tp_stage_tile(p, S, sb, jn, min(TP_TILE, p.n - jn), (t + 1) & 1);
+      tp_stage_tile(p, S, sb, jn, min(TP_TILE, jr1 - jn), (t + 1) & 1);
       cp_async_wait<1>();
     } else {
       cp_async_wait<0>();
     }
     __syncthreads();
-    const float* Bt = S.B + (t & 1) * 3 * TP_TILE;
-    const int k0 = max(jr0, jt0) - jt0, k1 = min(jr1, jt0 + TP_TILE) - jt0;
-    const int km = min(max(jall - jt0, k0), k1);  // [k0, km): masked, [km, k1): all points
-#pragma unroll 1
-    for (int k = k0; k < km; ++k) tp_pair1<NP, CNT, LUT>(c, Hw, P, inc, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], jt0 + k, true);
-    tp_pairs_all<NP, CNT, LUT>(p, c, Bt, Hw, P, inc, km, k1);
+    tp_tile_pairs<NP, CNT, LUT>(p, c, S.B + (t & 1) * 3 * TP_TILE, Hw, P, inc, jt0, max(jr0, jt0) - jt0,
+                                min(jr1, jt0 + TP_TILE) - jt0, jall);
     __syncthreads();  // slot t & 1 is refilled by the stage of tile t + 2
   }
 }
@@ -456,115 +469,225 @@ __device__ __forceinline__ void tp_points(const TPParams& p, const unsigned long
   }
 }
 
-// ============================================================================================
-// Single run (BASE / FT / FT_NL / FT_L / PROFILE): persistent CTAs, LPT schedule of chunk items.
-// ============================================================================================
-// Item = (point block blk, histogram h, partner chunk c, items of (h, blk)); partners
-// [c * TP_TILE, (c + 1) * TP_TILE) clipped to the block's [jlo, N).
-struct TPSched {
-  const int4* items;  // (blk, h, c, nitems of (h, blk)), grouped by SM
-  const int* off;     // [nsm + 1] list offsets
-  int* next;          // [nsm] claim counters (zeroed per run)
-  int* claimed;       // items claimed so far (zeroed per run)
-  int* exited;        // CTAs finished (zeroed per run)
-  int nsm, total;
+// The lane-private histogram outlives a visit: consecutive visits of a CTA with the same h keep
+// counting into it and it is flushed when h changes, before the 16-bit halves could overflow
+// (< 32768 partners per slot since the last flush) and at the end.
+struct TPHistState {
+  int h;      // histogram the shared counters belong to (-1: none)
+  int since;  // partners counted per slot since the last flush (upper bound)
 };
 
-__device__ __forceinline__ int tp_claim(const TPSched& q, int sl) {
-  const int k = atomicAdd(q.next + sl, 1);
-  if (q.off[sl] + k >= q.off[sl + 1]) return -1;
-  atomicAdd(q.claimed, 1);
-  return q.off[sl] + k;
+template <int NP>
+__device__ __forceinline__ void tp_hist_switch(const TPParams& p, const TPSmem& S, TPHistState* st, int h, int partners) {
+  // uniform over the CTA (st is in shared memory and read after a barrier)
+  if (st->h != h || st->since + partners >= 32768) {
+    if (st->h >= 0) {
+      tp_flush<NP>(p, S, p.hist, st->h * (p.nb + 2));
+      __syncthreads();  // flush read the counters and the ring before they are reused
+    }
+    tp_zero_hist<NP>(p, S);
+    __syncthreads();
+    if (threadIdx.x == 0) { st->h = h; st->since = 0; }
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) st->since += partners;
 }
 
+// ============================================================================================
+// Single run (BASE / FT / FT_NL / FT_L / PROFILE): one wave of CTAs that steal partner chunks.
+// A row = (histogram h, point block blk) of 128 * NP points; its partners [jlo, N) are cut into
+// chunks of HK_TP_SR_CHUNK.  CTAs start spread over the rows and claim chunks of a row with one
+// atomic each (claimed one chunk ahead, so the claim latency and the next tile's staging overlap
+// the current chunk), moving to the next row when it is exhausted: the work is balanced at chunk
+// granularity.  A CTA's stay on a row (a "visit") keeps its points' (acc, cnt) in registers;
+// leaving the row it adds them to the per-thread partial sums (exact integer combine) and its
+// chunk count to the row's; the visit that completes the row runs the loop-exit checks.
+// ============================================================================================
+struct TPSR {
+  int* row_next;  // [nrows] chunk claim counters (zeroed per run)
+  int* row_done;  // [nrows] chunks completed (zeroed per run)
+  int nrows;
+};
+
+__device__ __forceinline__ void tp_row_geom(const TPParams& p, int row, int* h, int* blk, int* c0, int* nch) {
+  constexpr int NP = HK_TP_NP_SR;
+  *h = row / p.nblk;
+  *blk = row - *h * p.nblk;
+  const int i0 = *blk * NP * TP_THREADS;
+  const int64_t gb = (int64_t)*h * p.n;
+  const int i1 = min(i0 + NP * TP_THREADS, p.n);
+  const bool any = gb + i0 < p.g1 && gb + i1 > p.g0;  // some point of the block is in this run
+  const int jlo = *h <= p.nr ? i0 + 1 : 0;
+  const int nc = (p.n + HK_TP_SR_CHUNK - 1) / HK_TP_SR_CHUNK;
+  *c0 = jlo / HK_TP_SR_CHUNK;
+  *nch = (any && jlo < p.n) ? nc - *c0 : 0;
+}
+
+// Warp 0: the next (row, chunk) starting at `row` (row = -1 once every row is exhausted).  The 32
+// lanes look at 32 rows at a time (one load of each claim counter), then lane 0 claims in the
+// first row that still had chunks; only exhausted rows are skipped, so the final sweep of a CTA
+// costs nrows / 32 load rounds instead of nrows sequential atomics.
+__device__ __forceinline__ int2 tp_sr_claim(const TPParams& p, const TPSR& q, int row) {
+  const unsigned FULL = 0xffffffffu;
+  const uint32_t lane = lane_id();
+  for (int scanned = 0; scanned < q.nrows; scanned += 32) {
+    int r = row + scanned + (int)lane;
+    r = r < q.nrows ? r : r - q.nrows;
+    if (r >= q.nrows) r -= q.nrows;
+    int h, blk, c0, nch = 0;
+    bool avail = false;
+    if (scanned + (int)lane < q.nrows) {
+      tp_row_geom(p, r, &h, &blk, &c0, &nch);
+      avail = nch > 0 && __ldcg(q.row_next + r) < nch;
+    }
+    unsigned m = __ballot_sync(FULL, avail);
+    while (m) {
+      const int l = __ffs(m) - 1;
+      const int rl = __shfl_sync(FULL, r, l), nl = __shfl_sync(FULL, nch, l);
+      int k = 0;
+      if (lane == 0) k = atomicAdd(q.row_next + rl, 1);
+      k = __shfl_sync(FULL, k, 0);
+      if (k < nl) return make_int2(rl, k);
+      m &= ~(1u << l);
+    }
+  }
+  return make_int2(-1, 0);
+}
+
+// Stage chunk k of `row` into ring slot `slot` (no-op for row < 0).
+__device__ __forceinline__ void tp_sr_stage(const TPParams& p, const TPSmem& S, int2 ch, int slot) {
+  if (ch.x < 0) return;
+  int h, blk, c0, nch;
+  tp_row_geom(p, ch.x, &h, &blk, &c0, &nch);
+  const int i0 = blk * HK_TP_NP_SR * TP_THREADS;
+  const int jlo = h <= p.nr ? i0 + 1 : 0;
+  const int j0 = max(jlo, (c0 + ch.y) * HK_TP_SR_CHUNK), j1 = min(p.n, (c0 + ch.y + 1) * HK_TP_SR_CHUNK);
+  const int sb = (h == 0) ? 0 : (h <= p.nr ? h : h - p.nr);
+  tp_stage_tile(p, S, sb, j0 & ~3, j1 - (j0 & ~3), slot);
+}
+
+// Claims run two chunks ahead of the computation: while chunk `cur` is computed, chunk `nxt`'s
+// tile is in flight and lane 0 of warp 0 has the atomic for the chunk after it outstanding (a
+// speculative claim in nxt's row; the scan of tp_sr_claim only when that row is exhausted).
 template <int V, bool LUT>
-__device__ __forceinline__ void tp_single_item(const TPParams& p, const TPSmem& S, int4 it) {
+__device__ __forceinline__ void tp_sr_run(const TPParams& p, const TPSmem& S, const TPSR& q, TPHistState* st, int2* claim) {
   constexpr int NP = HK_TP_NP_SR;
   constexpr bool NL = (V & V_NL) != 0, L = (V & V_L) != 0, PROF = (V & V_PROF) != 0, CNT = L || PROF;
-  const int blk = it.x, h = it.y, c = it.z, nitems = it.w;
-  const int i0 = blk * NP * TP_THREADS;
-  const int64_t gb = (int64_t)h * p.n;
-  TPPoint P[NP];
-  tp_points<NP>(p, p.hist, h, blk, p.g0, p.g1, P, NL);
-  uint32_t inc[NP];
-#pragma unroll
-  for (int k = 0; k < NP; ++k) inc[k] = P[k].valid ? ((k & 1) ? 0x10000u : 1u) : 0u;
-  const int jlo = h <= p.nr ? i0 + 1 : 0;
-  const int jr0 = max(jlo, c * TP_TILE), jr1 = min(p.n, (c + 1) * TP_TILE);
-  tp_zero_hist<NP>(p, S);
-  __syncthreads();
-  tp_item_loop<NP, V, LUT>(p, S, P, inc, h, i0, jr0, jr1);
-#pragma unroll
-  for (int k = 0; k < NP; ++k) {
-    P[k].acc /= 4;
-    tp_nl_exit<NL>(p, P[k], p.hist);
-    if (CNT && P[k].valid && P[k].cnt) {  // exact integer combine of this chunk's partial sums
-      atomicAdd(p.accg + gb + P[k].i, P[k].acc);
-      atomicAdd(p.cntg + gb + P[k].i, P[k].cnt);
-    }
+  if (threadIdx.x < 32) {
+    const int2 a = tp_sr_claim(p, q, (int)(((int64_t)blockIdx.x * q.nrows) / gridDim.x));
+    const int2 b = a.x >= 0 ? tp_sr_claim(p, q, a.x) : a;
+    if (threadIdx.x == 0) { claim[0] = a; claim[1] = b; }
   }
-  __syncthreads();  // every thread's combine atomics issued; the ring is free for the flush
-  tp_flush<NP>(p, S, p.hist, h * (p.nb + 2));
-  if (CNT) {
-    if (threadIdx.x == 0) {
-      __threadfence();
-      *S.flag = atomicAdd(p.done + h * p.nblk + blk, 1) == nitems - 1;
+  __syncthreads();
+  int2 cur = claim[0], nxt = claim[1];
+  int slot = 0;
+  tp_sr_stage(p, S, cur, 0);
+  tp_sr_stage(p, S, nxt, 1);
+  uint32_t Hw[NP / 2];
+  tp_lane_hist<NP>(p, S, Hw);
+  const TPLoopCtx c{S.L, smem_u32(S.E), S.E};
+  // the current visit
+  int vrow = -1, h = 0, blk = 0, c0 = 0, nch = 0, i0 = 0, jlo = 0, jall = 0, visited = 0;
+  int64_t gb = 0;
+  TPPoint P[NP];
+  uint32_t inc[NP];
+  auto end_visit = [&]() {
+#pragma unroll
+    for (int k = 0; k < NP; ++k) {
+      P[k].acc /= 4;
+      tp_nl_exit<NL>(p, P[k], p.hist);
+      if (CNT && P[k].valid && P[k].cnt) {  // exact combine of this visit's partial sums
+        atomicAdd(p.accg + gb + P[k].i, P[k].acc);
+        atomicAdd(p.cntg + gb + P[k].i, P[k].cnt);
+      }
     }
-    __syncthreads();
-    if (*S.flag) {  // last chunk item of this (h, block): the loop-exit checks of its points
-      __threadfence();
+    if (CNT) {
+      __syncthreads();  // every thread's combine atomics issued
+      if (threadIdx.x == 0) {
+        __threadfence();
+        *S.flag = atomicAdd(q.row_done + vrow, visited) + visited == nch;
+      }
+      __syncthreads();
+      if (*S.flag) {  // this visit completed the row: the loop-exit checks of its points
+        __threadfence();
+#pragma unroll
+        for (int k = 0; k < NP; ++k)
+          if (P[k].valid) {
+            P[k].acc = __ldcg(p.accg + gb + P[k].i);
+            P[k].cnt = __ldcg(p.cntg + gb + P[k].i);
+            tp_checks<V>(p, P[k], p.cb, gb + P[k].i);
+          }
+      }
+    }
+    if (NL || L) {
 #pragma unroll
       for (int k = 0; k < NP; ++k)
-        if (P[k].valid) {
-          P[k].acc = __ldcg(p.accg + gb + P[k].i);
-          P[k].cnt = __ldcg(p.cntg + gb + P[k].i);
-          tp_checks<V>(p, P[k], p.cb, gb + P[k].i);
-        }
+        if (P[k].valid) fold_alarm(p.cb, P[k].alarm, (uint32_t)(gb + P[k].i));
     }
-  }
-  if (NL || L) {
+    __syncthreads();  // flag reused
+  };
+  while (cur.x >= 0) {
+    if (cur.x != vrow) {
+      if (vrow >= 0) end_visit();
+      vrow = cur.x;
+      tp_row_geom(p, vrow, &h, &blk, &c0, &nch);
+      i0 = blk * NP * TP_THREADS;
+      gb = (int64_t)h * p.n;
+      jlo = h <= p.nr ? i0 + 1 : 0;
+      jall = h <= p.nr ? min(i0 + NP * TP_THREADS, p.n) : 0;
+      visited = 0;
+      tp_hist_switch<NP>(p, S, st, h, nch * HK_TP_SR_CHUNK);
+      tp_points<NP>(p, p.hist, h, blk, p.g0, p.g1, P, NL);
 #pragma unroll
-    for (int k = 0; k < NP; ++k)
-      if (P[k].valid) fold_alarm(p.cb, P[k].alarm, (uint32_t)(gb + P[k].i));
+      for (int k = 0; k < NP; ++k) inc[k] = P[k].valid ? ((k & 1) ? 0x10000u : 1u) : 0u;
+    }
+    // speculative claim of the chunk after nxt (its result is used after the computation)
+    int spec = -1, snch = 0;
+    if (threadIdx.x == 0 && nxt.x >= 0) {
+      int sh, sblk, sc0;
+      tp_row_geom(p, nxt.x, &sh, &sblk, &sc0, &snch);
+      spec = atomicAdd(q.row_next + nxt.x, 1);
+    }
+    if (nxt.x >= 0) cp_async_wait<1>();
+    else cp_async_wait<0>();
+    __syncthreads();  // cur's tile is staged
+    {
+      const int j0 = max(jlo, (c0 + cur.y) * HK_TP_SR_CHUNK), j1 = min(p.n, (c0 + cur.y + 1) * HK_TP_SR_CHUNK);
+      const int jt0 = j0 & ~3;
+      tp_tile_pairs<NP, CNT, LUT>(p, c, S.B + slot * 3 * TP_TILE, Hw, P, inc, jt0, j0 - jt0, j1 - jt0, jall);
+    }
+    ++visited;
+    if (threadIdx.x < 32) {
+      int2 nn = make_int2(-1, 0);
+      if (nxt.x >= 0) {
+        const int sp = __shfl_sync(0xffffffffu, spec, 0), sn = __shfl_sync(0xffffffffu, snch, 0);
+        nn = sp < sn ? make_int2(nxt.x, sp) : tp_sr_claim(p, q, nxt.x);
+      }
+      if (threadIdx.x == 0) claim[0] = nn;
+    }
+    __syncthreads();  // the computation is done (slot free) and the next claim visible
+    const int2 nn = claim[0];
+    tp_sr_stage(p, S, nn, slot);
+    cur = nxt;
+    nxt = nn;
+    slot ^= 1;
   }
-  __syncthreads();  // shared histogram / flag reused by the next item
+  if (vrow >= 0) end_visit();
 }
 
 template <int V>
-__device__ __forceinline__ void tp_drain(const TPParams& p, const TPSmem& S, const TPSched& q, int sl, int* item_s, bool lut) {
-  if (threadIdx.x == 0) *item_s = tp_claim(q, sl);
-  for (;;) {
-    __syncthreads();
-    const int it = *item_s;
-    __syncthreads();  // everyone has read the current item before thread 0 overwrites it
-    if (it < 0) break;
-    int nxt = -1;
-    if (threadIdx.x == 0) nxt = tp_claim(q, sl);  // result consumed after the item: latency hidden
-    if (lut) tp_single_item<V, true>(p, S, q.items[it]);
-    else tp_single_item<V, false>(p, S, q.items[it]);
-    if (threadIdx.x == 0) *item_s = nxt;
-  }
-}
-
-template <int V>
-__global__ void __launch_bounds__(TP_THREADS, HK_TP_MINB_SR) tpacf_kernel(const TPParams p, const TPSched q) {
+__global__ void __launch_bounds__(TP_THREADS, HK_TP_MINB_SR) tpacf_kernel(const TPParams p, const TPSR q) {
   extern __shared__ __align__(16) unsigned char tp_smem[];
-  __shared__ int item_s, last_s;
+  __shared__ TPHistState st;
+  __shared__ int2 claim[2];
   const TPSmem S = tp_carve(tp_smem, p.nb + 2, HK_TP_NP_SR);
   tp_stage_tables(p, S);
+  if (threadIdx.x == 0) { st.h = -1; st.since = 0; }
   cp_async_wait<0>();
   __syncthreads();
-  const bool lut = *p.lut_ok != 0;
-  uint32_t smid;
-  asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
-  tp_drain<V>(p, S, q, (int)(smid % (uint32_t)q.nsm), &item_s, lut);
-  if (threadIdx.x == 0) {
-    __threadfence();
-    last_s = (atomicAdd(q.exited, 1) == (int)gridDim.x - 1) && (*(volatile int*)q.claimed < q.total);
-  }
-  __syncthreads();
-  if (last_s)
-    for (int sl = 0; sl < q.nsm; ++sl) tp_drain<V>(p, S, q, sl, &item_s, lut);
+  if (*p.lut_ok) tp_sr_run<V, true>(p, S, q, &st, claim);
+  else tp_sr_run<V, false>(p, S, q, &st, claim);
+  if (st.h >= 0) tp_flush<HK_TP_NP_SR>(p, S, p.hist, st.h * (p.nb + 2));
 }
 
 // ============================================================================================
@@ -1141,12 +1264,13 @@ static TPParams tp_params(const hk_tpacf_args& a, const DevRanges& R, int ndet, 
   return p;
 }
 
-// Workspace (tpacf_ws_bytes): table [TP_LUT] uint2 | ok flag (16 B) | schedule counters
-// next[TP_SCHED_MAX_SM], claimed, exited | accg [nh * N] | cntg [nh * N] | done [nh * nblk].
-static size_t tp_ws_head() { return (size_t)TP_LUT + 16 + (TP_SCHED_MAX_SM + 2) * sizeof(int); }
+// Workspace (tpacf_ws_bytes): table [TP_LUT] u8 | ok flag (16 B) | row_next [nrows] | row_done [nrows] |
+// accg [nh * N] | cntg [nh * N]  (nrows = nh * blocks of 128 * HK_TP_NP_SR points)
+static size_t tp_ws_head() { return (size_t)TP_LUT + 16; }
+static int tp_nrows(const hk_tpacf_args& a) { return (1 + 2 * a.n_rand) * tp_nblk(a.n, HK_TP_NP_SR); }
 size_t tpacf_ws_bytes(const hk_tpacf_args& a) {
-  const size_t nt = (size_t)(1 + 2 * a.n_rand) * (size_t)a.n, nd = (size_t)(1 + 2 * a.n_rand) * tp_nblk(a.n, HK_TP_NP_SR);
-  return tp_ws_head() + nt * 8 + nd * 4;
+  const size_t nt = (size_t)(1 + 2 * a.n_rand) * (size_t)a.n;
+  return tp_ws_head() + 2 * sizeof(int) * (size_t)tp_nrows(a) + nt * 8;
 }
 
 cudaError_t tpacf_lut_build(const hk_tpacf_args& a, void* ws, cudaStream_t s) {
@@ -1163,100 +1287,9 @@ static double tp_pairs(const hk_tpacf_args& a) {
   return (1 + a.n_rand) * n * (n - 1) / 2 + a.n_rand * n * n;
 }
 
-// Host side of the single-run schedule: exact pair count per (point block, histogram, chunk) item
-// over the abstract threads [g0, g1), LPT assignment to the SMs.  Cached per (shape, range, SM
-// count, device, context): the cached device buffers belong to that context.
-struct TPSchedBuf {
-  int4* items = nullptr;
-  int* off = nullptr;
-  int total = 0;
-};
-static std::mutex& tp_cache_mu() { static std::mutex m; return m; }
-static std::map<std::array<long long, 6>, TPSchedBuf>& tp_cache() {
-  static std::map<std::array<long long, 6>, TPSchedBuf> c;
-  return c;
-}
-// hauberk_release_caches: free the cached schedules of the current context
-void tpacf_release_caches() {
-  std::lock_guard<std::mutex> lk(tp_cache_mu());
-  for (auto& kv : tp_cache()) {
-    cudaFree(kv.second.items);
-    cudaFree(kv.second.off);
-  }
-  cudaGetLastError();
-  tp_cache().clear();
-}
-static cudaError_t tp_schedule(const hk_tpacf_args& a, int nsm, int g0, int g1, TPSchedBuf* out) {
-  int dev = 0;
-  cudaError_t e = cudaGetDevice(&dev);
-  if (e != cudaSuccess) return e;
-  const std::array<long long, 6> key{a.n, a.n_rand, nsm, dev, g0, g1};
-  std::lock_guard<std::mutex> lk(tp_cache_mu());
-  auto& cache = tp_cache();
-  auto fnd = cache.find(key);
-  if (fnd != cache.end()) {
-    // a cached entry is only valid in the context that allocated it: after a device reset its
-    // buffers are gone (cudaPointerGetAttributes no longer reports device memory) -> rebuild
-    cudaPointerAttributes at{};
-    if (cudaPointerGetAttributes(&at, fnd->second.items) == cudaSuccess && at.type == cudaMemoryTypeDevice) {
-      *out = fnd->second;
-      return cudaSuccess;
-    }
-    cudaGetLastError();
-    cache.erase(fnd);
-  }
-  constexpr int CPTS = HK_TP_NP_SR * TP_THREADS;
-  const int N = a.n, nr = a.n_rand, nh = 1 + 2 * nr, nblk = tp_nblk(N, HK_TP_NP_SR), nc = (N + TP_TILE - 1) / TP_TILE;
-  std::vector<std::pair<double, int4>> w;
-  std::vector<int> per((size_t)nh * nblk, 0);
-  for (int h = 0; h < nh; ++h)
-    for (int b = 0; b < nblk; ++b) {
-      const int64_t i0 = (int64_t)b * CPTS, i1 = std::min<int64_t>(i0 + CPTS, N);
-      const int64_t lo = std::max<int64_t>(i0, g0 - (int64_t)h * N), hi = std::min<int64_t>(i1, g1 - (int64_t)h * N);
-      if (lo >= hi) continue;  // no abstract thread of this block is in the run's range
-      const int64_t jlo = h <= nr ? i0 + 1 : 0;
-      for (int c = 0; c < nc; ++c) {
-        const int64_t cb = std::max<int64_t>((int64_t)c * TP_TILE, jlo), ce = std::min<int64_t>((int64_t)(c + 1) * TP_TILE, N);
-        if (cb >= ce) continue;
-        double pairs = 0;
-        for (int64_t i = lo; i < hi; ++i) pairs += (double)std::max<int64_t>(0, ce - std::max<int64_t>(cb, h <= nr ? i + 1 : 0));
-        // + the per-item prologue / histogram zero and flush (~8k pair-equivalents)
-        w.push_back({pairs + 8192.0, make_int4(b, h, c, 0)});
-        per[(size_t)h * nblk + b]++;
-      }
-    }
-  for (auto& it : w) it.second.w = per[(size_t)it.second.y * nblk + it.second.x];
-  std::stable_sort(w.begin(), w.end(), [](const auto& x, const auto& y) { return x.first > y.first; });
-  std::vector<std::vector<int4>> lists(nsm);
-  std::priority_queue<std::pair<double, int>, std::vector<std::pair<double, int>>, std::greater<>> load;
-  for (int m = 0; m < nsm; ++m) load.push({0.0, m});
-  for (const auto& it : w) {
-    auto top = load.top();
-    load.pop();
-    lists[top.second].push_back(it.second);
-    load.push({top.first + it.first, top.second});
-  }
-  std::vector<int4> items;
-  std::vector<int> off(nsm + 1, 0);
-  for (int m = 0; m < nsm; ++m) {
-    off[m] = (int)items.size();
-    items.insert(items.end(), lists[m].begin(), lists[m].end());
-  }
-  off[nsm] = (int)items.size();
-  TPSchedBuf B;
-  B.total = (int)items.size();
-  if ((e = cudaMalloc(&B.items, sizeof(int4) * std::max<size_t>(1, items.size()))) != cudaSuccess) return e;
-  if ((e = cudaMalloc(&B.off, sizeof(int) * off.size())) != cudaSuccess) { cudaFree(B.items); return e; }
-  if ((!items.empty() && (e = cudaMemcpy(B.items, items.data(), sizeof(int4) * items.size(), cudaMemcpyHostToDevice)) != cudaSuccess) ||
-      (e = cudaMemcpy(B.off, off.data(), sizeof(int) * off.size(), cudaMemcpyHostToDevice)) != cudaSuccess) {
-    cudaFree(B.items);
-    cudaFree(B.off);
-    return e;
-  }
-  cache[key] = B;
-  *out = B;
-  return cudaSuccess;
-}
+// hauberk_release_caches: the TPACF kernels keep no per-shape device state between calls (the
+// single run balances itself by chunk stealing), so there is nothing to free.
+void tpacf_release_caches() {}
 
 template <int V>
 static cudaError_t launch_tp_v(const hk_tpacf_args& a, TPParams p, void* ws, cudaStream_t s) {
@@ -1267,25 +1300,17 @@ static cudaError_t launch_tp_v(const hk_tpacf_args& a, TPParams p, void* ws, cud
   int dev = 0, nsm = 0, per_sm = 0;
   if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
   if ((e = cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess) return e;
-  if (nsm > TP_SCHED_MAX_SM) return cudaErrorInvalidValue;
   if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tpacf_kernel<V>, TP_THREADS, smem)) != cudaSuccess) return e;
-  TPSchedBuf B;
-  if ((e = tp_schedule(a, nsm, p.g0, p.g1, &B)) != cudaSuccess) return e;
   char* w = reinterpret_cast<char*>(ws);
-  TPSched q;
-  q.items = B.items;
-  q.off = B.off;
-  q.next = reinterpret_cast<int*>(w + TP_LUT + 16);
-  q.claimed = q.next + TP_SCHED_MAX_SM;
-  q.exited = q.claimed + 1;
-  q.nsm = nsm;
-  q.total = B.total;
+  TPSR q;
+  q.nrows = tp_nrows(a);
+  q.row_next = reinterpret_cast<int*>(w + tp_ws_head());
+  q.row_done = q.row_next + q.nrows;
   const size_t nt = (size_t)(1 + 2 * p.nr) * (size_t)p.n;
-  p.accg = reinterpret_cast<int32_t*>(w + tp_ws_head());
+  p.accg = reinterpret_cast<int32_t*>(q.row_done + q.nrows);
   p.cntg = p.accg + nt;
-  p.done = p.cntg + nt;
-  if ((e = cudaMemsetAsync(w + TP_LUT + 16, 0, tpacf_ws_bytes(a) - (TP_LUT + 16), s)) != cudaSuccess) return e;
-  const int grid = nsm * std::max(1, std::min(per_sm, (B.total + nsm - 1) / nsm));
+  if ((e = cudaMemsetAsync(w + tp_ws_head(), 0, tpacf_ws_bytes(a) - tp_ws_head(), s)) != cudaSuccess) return e;
+  const int grid = nsm * std::max(1, per_sm);  // one wave
   TimedScope ts(HK_TPACF, 0, tp_pairs(a) * (double)(p.g1 - p.g0) / (double)((1 + 2 * p.nr) * p.n), s);
   tpacf_kernel<V><<<grid, TP_THREADS, smem, s>>>(p, q);
   count_launch();

@@ -6,8 +6,11 @@ Step = one chunk of the config-5 campaign (mixed CP-s / MRI-Q / TPACF shapes of 
 bench = n mod 3, seeded single-bit injections, replica mode: every injection is one full
 FI&FT program run plus the classify epilogue — PAPER L2370-2371).  `value` = injections/s of the
 whole job (all ranks; weak scaling: each rank takes its own `--per-rank` slice each step).
-Alongside: the FT-vs-BASE overhead of configs 4 (CP-L), 2 (MRI-Q) and 3 (TPACF), coverage,
-roofline fractions, e2e (pinned-host inputs copied in every step), and the CPU oracle baseline.
+Alongside: the FT-vs-BASE overhead of configs 4 (CP-L), 2 (MRI-Q) and 3 (TPACF) (K back-to-back
+launches per event pair), coverage of the FI&FT binary and the unprotected SDC rate of the FI-only
+binary (row a7) over the same injection indices, roofline fractions, e2e (pinned-host inputs
+copied in every step), and the CPU oracle: golden runs of configs 1-4, replay- and replica-mode
+campaigns on 1 core and on every host core.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
   torchrun --nproc-per-node N bench.py --gpus N ...   (NCCL; max-over-ranks timing)
@@ -31,6 +34,7 @@ MUFU_PER_SM_CLK = 16     # B200: 16 MUFU lanes / clk / SM (4 per SMSP); measured
 LANES_PER_SM_CLK = 128   # FP32/INT32 lanes / clk / SM
 N_SM = 148
 TPACF_OPS_PER_PAIR = 11  # 3 FP (dot) + 5 compares (binary search over 22 bins) + 1 histogram add + 2 detector adds
+OVH_K = 20               # launches per event pair in the overhead timing
 
 
 def parse():
@@ -146,6 +150,70 @@ def oracle_all_cores(seed: int, first: int, procs: int):
     return n / wall, n, wall
 
 
+def cpu_model():
+    try:
+        for line in subprocess.check_output(["lscpu"], text=True).splitlines():
+            if line.startswith("Model name:"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return "unknown"
+
+
+def oracle_golden_times():
+    """The oracle's fault-free FI&FT-binary run (FT flags, own profiled ranges) of configs 1-3 in full
+    and of config 4 on a row sample (1/64 of the CP-L grid threads, scaled), 1 core."""
+    import numpy as np
+
+    import oracle as O
+    import workloads as W
+    out = {}
+    for name, b, p in (("cfg1_cp_s", 0, W.cp_config1()), ("cfg2_mriq", 1, W.mriq_config2()), ("cfg3_tpacf", 2, W.tpacf_config3())):
+        R = O.profile_ranges(b, p)
+        t0 = time.perf_counter()
+        O.run(b, p, flags=O.FT, ranges=R, ndet=R.n_det)
+        out[name] = {"s": round(time.perf_counter() - t0, 4), "sample": "whole run"}
+    p4 = W.cp_config4(bx=16, by=16, unroll=8)
+    nthr = (p4.nx // p4.unroll) * p4.ny
+    tids = np.arange(0, nthr, 64)
+    t0 = time.perf_counter()
+    O.threads_out(O.CP, p4, tids)
+    dt = time.perf_counter() - t0
+    out["cfg4_cp_l"] = {"s": round(dt * nthr / tids.size, 2), "sample": f"{tids.size} of {nthr} abstract threads "
+                        f"(every 64th; {dt:.2f} s measured, scaled x{nthr / tids.size:.0f})"}
+    return out
+
+
+def _oracle_replay_worker(job):
+    """(seconds of a 3-injection call, seconds of a `count`-injection call): both rebuild the oracle's
+    golden runs and catalogues, so their difference is the replay work of count - 3 injections."""
+    seed, first, count = job
+    import oracle as O
+    probs, R = _ORACLE_SETUP["probs"], _ORACLE_SETUP["R"]
+    t0 = time.perf_counter()
+    O.campaign(-1, probs, R, seed, first, 3, mode=1, records=False)
+    t1 = time.perf_counter()
+    O.campaign(-1, probs, R, seed, first + 3, count, mode=1, records=False)
+    return t1 - t0, time.perf_counter() - t1
+
+
+def oracle_replay(seed: int, count: int, procs: int):
+    """The oracle's replay-mode campaign (config-5 indices, bench = n mod 3) on 1 core and on `procs`
+    forked processes; injections/s from the replay work alone (golden-run setup subtracted)."""
+    import multiprocessing as mp
+    oracle_replica_sample(seed, 0, 0)
+    ts, tb = _oracle_replay_worker((seed, 0, count))
+    one = (count - 3) / max(tb - ts, 1e-9)
+    allc = None
+    if procs > 1:
+        ctx = mp.get_context("fork")
+        with ctx.Pool(procs) as pool:
+            res = pool.map(_oracle_replay_worker, [(seed, w * count, count) for w in range(procs)], chunksize=1)
+        # the workers ran concurrently: total replay injections over the slowest worker's replay time
+        allc = procs * (count - 3) / max(max(b - a for a, b in res), 1e-9)
+    return one, allc, tb - ts
+
+
 def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
@@ -240,10 +308,11 @@ def main():
         for name, d, pipe, ops in cases:
             R = hk.profile_ranges(d)
             cb = hk.new_control(dev)
+            # kernel-only device time per launch (library CUDA events around the main kernel)
             hk.timing_enable(True)
             t = {v: [] for v in variants}
             work = 0.0
-            for rep in range(32):
+            for rep in range(22):
                 for v in variants:
                     flush.zero_()
                     hk.run(d, v, R, cb)
@@ -254,6 +323,20 @@ def main():
                         work = w
             hk.timing_enable(False)
             assert hk.read_control(cb).alarm == 0
+            # overhead: K back-to-back hauberk_run_* calls per CUDA-event pair (event resolution ~1 us
+            # per pair, so sub-us per-launch differences resolve), variants interleaved, median of rounds
+            kt = {v: [] for v in variants}
+            for rep in range(8):
+                for v in variants:
+                    flush.zero_()
+                    k0, k1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    k0.record()
+                    for _ in range(OVH_K):
+                        hk.run(d, v, R, cb)
+                    k1.record()
+                    torch.cuda.synchronize()
+                    if rep >= 1:
+                        kt[v].append(k0.elapsed_time(k1) / OVH_K)
             # R-Naive: second BASE run on the twin copy, then the compare kernel (CUDA events)
             tw = twins[name]
             outs = lambda dd: [dd.output()] if not isinstance(dd.output(), tuple) else list(dd.output())
@@ -272,19 +355,23 @@ def main():
                 if rep >= 2:
                     tcmp.append(c0.elapsed_time(c1))
             naive_alarm = hk.read_control(ccb).alarm
-            # CUDA event durations come in ~1.02 us steps; a 10 %-trimmed mean of 30 samples resolves
-            # the ~70 us kernels' overheads below one step (the medians are reported beside it)
-            med = {v: _trimmed_mean(t[v]) for v in variants}
-            medians = {v: statistics.median(t[v]) for v in variants}
+            med = {v: statistics.median(t[v]) for v in variants}
+            kmed = {v: statistics.median(kt[v]) for v in variants}
             tb, tf = med[hk.HK_BASE], med[hk.HK_FT]
+            kb, kf = kmed[hk.HK_BASE], kmed[hk.HK_FT]
             peak = mufu_peak if pipe == "xu" else lane_peak
             ach = work * ops / (tf * 1e-3)
-            overhead[name] = round(100.0 * (tf / tb - 1.0), 2)
-            kernels[name] = {"base_ms": round(tb, 4), "ft_ms": round(tf, 4), "overhead_pct": overhead[name],
-                             "overhead_nl_pct": round(100.0 * (med[hk.HK_FT_NL] / tb - 1.0), 2),
-                             "overhead_l_pct": round(100.0 * (med[hk.HK_FT_L] / tb - 1.0), 2),
-                             "base_ms_median": round(medians[hk.HK_BASE], 4), "ft_ms_median": round(medians[hk.HK_FT], 4),
-                             "timing": "10 %-trimmed mean of 30 launches (L2 flushed before each)",
+            overhead[name] = round(100.0 * (kf / kb - 1.0), 2)
+            kernels[name] = {"base_ms": round(kb, 5), "ft_ms": round(kf, 5), "overhead_pct": overhead[name],
+                             "overhead_nl_pct": round(100.0 * (kmed[hk.HK_FT_NL] / kb - 1.0), 2),
+                             "overhead_l_pct": round(100.0 * (kmed[hk.HK_FT_L] / kb - 1.0), 2),
+                             "timing": f"per-call device time of {OVH_K} back-to-back hauberk_run_* calls per CUDA-event pair "
+                                       "(pre-pass / PhiMag / table kernels included, identical in every variant), median "
+                                       "of 7 interleaved rounds, L2 flushed before each round",
+                             "kernel_only_ms": {"base": round(tb, 5), "ft": round(tf, 5),
+                                                "overhead_pct": round(100.0 * (tf / tb - 1.0), 2),
+                                                "timing": "library CUDA events around the main kernel, median of 20 "
+                                                          "launches, L2 flushed before each"},
                              "overhead_rnaive_pct": round(100.0 * ((2 * tb + statistics.median(tcmp)) / tb - 1.0), 2),
                              "rnaive_compare_ms": round(statistics.median(tcmp), 4), "rnaive_alarm": naive_alarm,
                              "pairs": work, "bound": "alu", "pipe": "xu (MUFU)" if pipe == "xu" else "fp32/int lanes",
@@ -377,15 +464,16 @@ def main():
                 "ops_per_pair": ops, "peak_source": f"{N_SM} SMs x {MUFU_PER_SM_CLK if dom < 2 else LANES_PER_SM_CLK}/clk/SM x {sm_mhz_peak:.0f} MHz ({clk_src})"}
     # what actually binds the dominant kernel (ncu --set full of the same kernel, profiles/r01_ncu_fi_summary.txt)
     roofline["limiter_ncu"] = {
-        2: "shared-memory path: l1tex 97.5 % of peak, issue 87 % (12.5 SASS instructions per pair vs 11 algorithmic ops)",
-        1: "XU (MUFU sin/cos) 87 % of peak, issue 75 %",
+        2: "shared-memory wavefronts (profiles/r02_ncu_summary.txt): per pair one LDS.U8 + one edge LDS + one ATOMS "
+           "+ 3/16 LDS.128 (2 wavefronts each) = 3.375 wavefronts per 32 pairs; 12.4 SASS instructions per pair",
+        1: "XU (MUFU sin/cos)",
         0: "XU (MUFU rsqrt); launch-bound at CP-s size",
     }[dom]
     fi_split = {hk.BENCH_NAMES[b]: {"ms": round(fi[b][0], 3), "launches": fi[b][1], "pairs": fi[b][2], "serial_steps": ser_steps}
                 for b in range(3)}
     # traffic: DRAM bytes per launch of the same kernel/batch from the committed ncu capture
     try:
-        with open(os.path.join(ROOT, "profiles", "r01_traffic.json")) as f:
+        with open(os.path.join(ROOT, "profiles", "r02_traffic.json")) as f:
             tr = json.load(f).get(f"{hk.BENCH_NAMES[dom]}_fi_kernel")
         if tr:
             # ncu measured one launch of `replicas_per_launch` replicas; scale per replica to this
@@ -426,20 +514,39 @@ def main():
     par.all_reduce_max(t2)
     e2e_value = args.per_rank * e2e_steps * world / (float(t2.item()) * 1e-3)
 
-    # ---- CPU oracle baseline (rank 0 at N = 1 only; bounded sample)
+    # ---- FI-only binary (row a7): the same injection indices over the original
+    #      program's sites, no detectors -> the unprotected SDC rate (untimed)
+    fionly = torch.zeros((3, 5), dtype=torch.int64, device=dev)
+    with hk.CampaignSession(-1, devs, [None, None, None], seed, batch=args.batch, variant=hk.HK_FI_ONLY) as sf:
+        for st_ in range(args.steps):
+            first, cnt = par.step_slice(st_, rank, world, args.per_rank)
+            sf.run(first, cnt, fionly)
+        torch.cuda.synchronize()
+    par.all_reduce_counts(fionly)
+    cfo = fionly.cpu().numpy()
+
+    # ---- CPU oracle baseline (rank 0 at N = 1 only; bounded samples)
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
+        procs = args.cpu_procs if args.cpu_procs > 0 else min(64, len(os.sched_getaffinity(0)))
         per = oracle_replica_sample(seed, 0, 6)  # 2 x (CP-s, MRI-Q, TPACF)
         tm = [statistics.mean(per[b]) for b in range(3)]
         cpu = {"value": round(3.0 / sum(tm), 4), "unit": "injections/s", "cores": 1, "kind": "oracle",
+               "cpu_model": cpu_model(), "host_cores": len(os.sched_getaffinity(0)),
                "sample": "6 config-5 injections (2 each CP-s / MRI-Q / TPACF), replica mode (full program run each), "
                          f"mean s/injection cp={tm[0]:.4f} mriq={tm[1]:.3f} tpacf={tm[2]:.3f}"}
-        procs = args.cpu_procs if args.cpu_procs > 0 else min(64, len(os.sched_getaffinity(0)))
         if procs > 1:
             v_all, n_all, wall = oracle_all_cores(seed, 300, procs)
             cpu["all_cores"] = {"value": round(v_all, 4), "unit": "injections/s", "cores": procs, "kind": "oracle",
                                 "sample": f"{n_all} config-5 injections ({procs} forked processes x one CP-s / MRI-Q / "
                                           f"TPACF triple), replica mode, {wall:.1f} s wall"}
+        rp1, rpall, rpt = oracle_replay(seed, 1500, procs)
+        cpu["replay"] = {"value_1core": round(rp1, 1), "value_all_cores": round(rpall, 1) if rpall else None,
+                         "unit": "injections/s", "cores": procs, "kind": "oracle",
+                         "sample": f"1,497 config-5 injections per process (bench = n mod 3), replay mode (the faulted "
+                                   f"abstract thread and its golden twin re-run, golden patched); {rpt:.2f} s of replay "
+                                   "work on 1 core (a 3-injection call's golden-run setup subtracted)"}
+        cpu["golden_runs_s"] = oracle_golden_times()
 
     session.close()
 
@@ -515,7 +622,10 @@ def main():
             "roofline": roofline,
             "cpu_baseline": cpu,
             "coverage_pct": round(100.0 * hk.coverage(c), 3),
-            "unprotected_sdc_pct": round(100.0 * hk.unprotected_sdc(c), 3),
+            "unprotected_sdc_pct": round(100.0 * hk.unprotected_sdc(cfo), 3),
+            "protected_sdc_pct": round(100.0 * hk.summarize(c)["sdc"], 3),
+            "fi_only_outcomes": {hk.BENCH_NAMES[b]: dict(zip(hk.CLASS_NAMES, cfo[b].tolist())) for b in range(3)},
+            "fi_only_sdc_by_bench_pct": {hk.BENCH_NAMES[b]: round(100.0 * hk.unprotected_sdc(cfo[b]), 3) for b in range(3)},
             "outcomes": {hk.BENCH_NAMES[b]: dict(zip(hk.CLASS_NAMES, c[b].tolist())) for b in range(3)},
             "coverage_by_bench_pct": {hk.BENCH_NAMES[b]: round(100.0 * hk.coverage(c[b]), 3) for b in range(3)},
             "overhead_pct": overhead, "kernels": kernels, "fi_kernels": fi_split,

@@ -268,27 +268,13 @@ def test_campaign_exact_mode_bit_exact():
     assert np.array_equal(gc, oc)
 
 
-def _taus(probs):
-    """R22(a) absolute half-width per benchmark: the R21 output bound of one thread's accumulation
-    divided by its trip count (CP c=4 with the largest per-point mass; MRI-Q c=16 with sum |phi|^2)."""
-    t = [0.0, 0.0, 0.0]
-    if probs[0] is not None and probs[0].n_atoms:
-        _, mass = O.reference_f64(O.CP, probs[0])
-        t[0] = 4 * 2.0**-23 * float(mass.max()) / probs[0].n_atoms
-    if probs[1] is not None and probs[1].n_k:
-        pm = probs[1].phi_r.astype(np.float64) ** 2 + probs[1].phi_i.astype(np.float64) ** 2
-        t[1] = 16 * 2.0**-23 * float(pm.sum()) / probs[1].n_k
-    return np.array(t)
-
-
 def _ambiguous(g, o, probs=None):
-    band = (g["margin"] <= 1024) | (o["margin"] <= 1024)
-    if probs is not None:
-        tau = _taus(probs)[g["bench"]]
-        band |= (g["gap"] <= tau) | (o["gap"] <= tau)
-    band |= ((g["worst"] >= 0.98) & (g["worst"] <= 1.02)) | ((o["worst"] >= 0.98) & (o["worst"] <= 1.02))
-    band |= (g["domain"] != 0) | (o["domain"] != 0)
-    return band
+    """R22 guard band with half-widths derived from R21 (tests/test_gpu_r02.band_halfwidths)."""
+    from test_gpu_r02 import ambiguous
+    if probs is None:
+        probs = [None, None, None]
+    band = ambiguous(g, o, probs)
+    return band["a"] | band["b"] | band["c"]
 
 
 def test_campaign_fast_mode_exact_outside_guard_band():
@@ -298,7 +284,6 @@ def test_campaign_fast_mode_exact_outside_guard_band():
         assert np.array_equal(grec[k], orec[k]), k
     amb = _ambiguous(grec, orec, probs)
     tp = grec["bench"] == 2
-    assert not amb[tp].any() or True
     mism = np.nonzero((grec["cls"] != orec["cls"]) & ~amb)[0]
     assert mism.size == 0, [(grec[i], orec[i]) for i in mism[:5]]
     assert np.array_equal(grec["cls"][tp], orec["cls"][tp])  # TPACF: no band needed
@@ -499,7 +484,7 @@ def test_gpu_replay_config_shapes_vs_oracle_replay():
     assert not mism.any(), [(g[i], o[i]) for i in np.nonzero(mism)[0][:5]]
     tp = g["bench"] == 2
     assert np.array_equal(g["cls"][tp], o["cls"][tp])
-    assert amb.mean() < 0.01
+    assert amb.mean() < 0.02  # R21-derived band (b) is +-3.8 % of tol for MRI-Q at config 2 (test_gpu_r02)
 
 
 def test_gpu_replay_exact_mode_bit_exact_config_shapes():
@@ -554,7 +539,7 @@ def test_full_config5_campaign_1M_gpu_replay_vs_oracle():
     assert not mism.any(), detail
     tp = g["bench"] == 2
     assert np.array_equal(g["cls"][tp], o["cls"][tp])
-    assert amb.mean() < 0.01
+    assert amb.mean() < 0.02  # R21-derived band (b) is +-3.8 % of tol for MRI-Q at config 2 (test_gpu_r02)
     assert gc.sum() == N
 
 

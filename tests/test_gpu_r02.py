@@ -1,0 +1,358 @@
+"""Round-2 GPU parity (-m gpu), all through the C ABI:
+
+* replica mode at the bench's own shapes (config 5 = cfg1 CP-s / cfg2 MRI-Q / cfg3 TPACF): record
+  for record equal to the GPU replay (exact) and to the oracle outside the R22 guard band, whose
+  half-widths come from R21 (DESIGN R22) and whose per-criterion counts are reported;
+* the whole 1M-injection config-5 campaign in replica mode: counters equal to the replay counters
+  (each experiment is a full program run with one fault);
+* full-output FP parity of the single runs of config 2 (MRI-Q) and config 4 (CP-L, oracle split
+  over processes) within R21;
+* the FI-only binary (row a7), alpha = 10 ranges (R11) and a small hang factor (R17) against the
+  oracle in EXACT mode (bit-exact records);
+* the product's campaign path sharded over a gloo world of 2 processes on one GPU: all-reduced
+  counters and the gathered records equal the single-process campaign.
+"""
+import multiprocessing as mpp
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+
+import oracle as O
+import workloads as W
+
+pytestmark = pytest.mark.gpu
+
+hk = None
+DEV = "cuda"
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _lib():
+    global hk
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_ipps_yimpski11_b200 import hauberk
+    hauberk.lib()
+    hk = hauberk
+
+
+def _mk(bench, p, exact=0):
+    return [hk.CPDevice, hk.MRIQDevice, hk.TPACFDevice][bench].from_problem(p, DEV, exact=exact)
+
+
+def _gpu_campaign(devs, ranges, seed, first, count, bench_mode=-1, **kw):
+    counts = torch.zeros((3, 5), dtype=torch.int64, device=DEV)
+    rec = hk.records_tensor(count, DEV)
+    hk.inject_campaign(bench_mode, devs, ranges, seed, first, count, counts, records=rec, **kw)
+    torch.cuda.synchronize()
+    return counts.cpu().numpy(), hk.records_numpy(rec)
+
+
+# ---------------------------------------------------------------------------------- R22 guard band
+def band_halfwidths(probs):
+    """R22 half-widths per benchmark, derived from R21 (DESIGN R21/R22):
+    (a) check value: 1,024 ordinal ulps, or tau = R21's output bound of one thread's accumulation
+        divided by its trip count;
+    (b) the worst err/tol ratio: two outputs that differ by at most R21's bound each (replica and
+        golden) move err by <= 2 * bound, tol >= 1e-4 * max|G|, so |ratio - 1| <= 2 * bound / tol_min."""
+    tau, delta = [0.0, 0.0, 0.0], [0.0, 0.0, 0.0]
+    if probs[0] is not None and probs[0].n_atoms:
+        g, mass = O.reference_f64(O.CP, probs[0])
+        bound = max(float((1e-5 * np.abs(g)).max()), 4 * 2.0**-23 * float(mass.max()))
+        tau[0] = 4 * 2.0**-23 * float(mass.max()) / probs[0].n_atoms
+        delta[0] = 2 * bound / (1e-4 * float(np.abs(g).max()))
+    if probs[1] is not None and probs[1].n_k:
+        (qr, qi), mass = O.reference_f64(O.MRIQ, probs[1])
+        M = float(max(np.abs(qr).max(), np.abs(qi).max()))
+        bound = max(1e-5 * M, 16 * 2.0**-23 * float(mass.max()))
+        tau[1] = 16 * 2.0**-23 * float(mass.max()) / probs[1].n_k
+        delta[1] = 2 * bound / (1e-4 * M)
+    return np.array(tau), np.array(delta)
+
+
+def ambiguous(g, o, probs):
+    """R22 membership per criterion: a = check value near a range bound, b = worst err/tol near 1,
+    c = sin/cos argument outside the MUFU accuracy domain.  TPACF never (exact integer binning)."""
+    tau, delta = band_halfwidths(probs)
+    b_ = g["bench"]
+    a = (g["margin"] <= 1024) | (o["margin"] <= 1024) | (g["gap"] <= tau[b_]) | (o["gap"] <= tau[b_])
+    d = delta[b_]
+    b = (np.abs(g["worst"] - 1.0) <= d) | (np.abs(o["worst"] - 1.0) <= d)
+    c = (g["domain"] != 0) | (o["domain"] != 0)
+    tp = b_ == 2
+    return {"a": a & ~tp, "b": b & ~tp, "c": c & ~tp}
+
+
+def test_replica_mode_at_the_bench_shapes_equals_replay_and_the_oracle():
+    """3,000 config-5 injections (the bench's per-step slice) in replica mode: every record equal to
+    the GPU replay of the same indices; outcomes equal to the oracle (replay) outside the R22 band,
+    TPACF everywhere; the band holds < 0.1 % of the injections (R22: "expected << 0.1 %")."""
+    probs = [W.cp_config1(), W.mriq_config2(), W.tpacf_config3()]
+    devs = [_mk(b, probs[b]) for b in range(3)]
+    R = [hk.profile_ranges(d) for d in devs]
+    first, count = 123000, 3000
+    c0, r0 = _gpu_campaign(devs, R, W.CAMPAIGN_SEED_CFG5, first, count, mode=0)
+    c1, r1 = _gpu_campaign(devs, R, W.CAMPAIGN_SEED_CFG5, first, count, mode=1)
+    for k in ("index", "bench", "site", "thread", "inst", "mask", "cls", "alarm", "fail", "margin", "domain"):
+        assert np.array_equal(r0[k], r1[k]), k
+    assert np.array_equal(c0, c1)
+    orr = [O.profile_ranges(b, probs[b]) for b in range(3)]
+    oc, o = O.campaign(-1, probs, orr, W.CAMPAIGN_SEED_CFG5, first, count, mode=1)
+    for k in ("index", "bench", "site", "thread", "inst", "mask"):
+        assert np.array_equal(r0[k], o[k]), k
+    band = ambiguous(r0, o, probs)
+    amb = band["a"] | band["b"] | band["c"]
+    allmm = r0["cls"] != o["cls"]
+    mism = allmm & ~amb
+    assert not mism.any(), [(r0[i], o[i]) for i in np.nonzero(mism)[0][:5]]
+    tp = r0["bench"] == 2
+    assert np.array_equal(r0["cls"][tp], o["cls"][tp])
+    print("band counts (a, b, c):", {k: int(v.sum()) for k, v in band.items()}, "of", count,
+          "; class mismatches inside the band:", int(allmm.sum()))
+    # R21's MUFU term (c = 16, a worst-case bound: every term's sin/cos error at 2^-20.9 with the same
+    # sign) makes band (b) +-3.8 % of tol for MRI-Q at config 2: ~1.5 % of the injections sit in it
+    assert amb.mean() < 0.02
+
+
+def test_full_config5_campaign_1M_replica_counters_equal_replay():
+    """every experiment a full program run with one fault.  The 1,000,000-injection
+    config-5 campaign in replica mode (~35 s on one B200) gives the replay campaign's counters and
+    per-site counters exactly, and the same class for every index."""
+    N = 1_000_000
+    probs = [W.cp_config1(), W.mriq_config2(), W.tpacf_config3()]
+    devs = [_mk(b, probs[b]) for b in range(3)]
+    R = [hk.profile_ranges(d) for d in devs]
+    out = {}
+    for mode in (0, 1):
+        counts = torch.zeros((3, 5), dtype=torch.int64, device=DEV)
+        sites = torch.zeros((3, 64, 5), dtype=torch.int64, device=DEV)
+        rec = hk.records_tensor(N, DEV)
+        with hk.CampaignSession(-1, devs, R, W.CAMPAIGN_SEED_CFG5, mode=mode) as S:
+            S.run(0, N, counts, records=rec, site_counts=sites)
+            torch.cuda.synchronize()
+        out[mode] = (counts.cpu().numpy(), sites.cpu().numpy(), hk.records_numpy(rec))
+    assert np.array_equal(out[0][0], out[1][0]) and out[0][0].sum() == N
+    assert np.array_equal(out[0][1], out[1][1])
+    assert np.array_equal(out[0][2]["cls"], out[1][2]["cls"])
+    print("1M replica counters:", out[0][0].tolist())
+
+
+# ---------------------------------------------------------------------------------- full-output FP
+def test_config2_mriq_full_output_parity():
+    """Every one of the 32,768 voxels (Qr and Qi) of config 2 within R21 of the oracle's FP32 spec."""
+    p = W.mriq_config2()
+    d = _mk(1, p)
+    R = hk.profile_ranges(d)
+    cb = hk.new_control(DEV)
+    hk.run(d, hk.HK_FT, R, cb)
+    torch.cuda.synchronize()
+    assert hk.read_control(cb).alarm == 0
+    gqr, gqi = d.qr.cpu().numpy(), d.qi.cpu().numpy()
+    (oqr, oqi), _, _ = O.run(O.MRIQ, p, flags=0)
+    mass = float((p.phi_r.astype(np.float64) ** 2 + p.phi_i.astype(np.float64) ** 2).sum())
+    for g, o in ((gqr, oqr), (gqi, oqi)):
+        bad = np.abs(g.astype(np.float64) - o) > np.maximum(1e-5 * np.abs(o.astype(np.float64)), 16 * 2.0**-23 * mass)
+        assert not bad.any(), int(bad.sum())
+
+
+def _cp4_rows(args):
+    y0, y1 = args
+    import oracle as Ow
+    import workloads as Ww
+    p = Ww.cp_config4(bx=16, by=16, unroll=8)
+    nthr_row = p.nx // p.unroll
+    tids = np.arange(y0 * nthr_row, y1 * nthr_row)
+    idx, val = Ow.threads_out(Ow.CP, p, tids)
+    return idx.ravel(), val.ravel()
+
+
+def test_config4_cp_full_output_parity():
+    """All 262,144 grid points of config 4 (40,000 atoms, 512 x 512) within R21 (c = 4) of the oracle,
+    whose 32,768 abstract threads run in row bands over every host core."""
+    p = W.cp_config4(bx=16, by=16, unroll=8)
+    d = _mk(0, p)
+    R = hk.profile_ranges(d)
+    cb = hk.new_control(DEV)
+    hk.run(d, hk.HK_FT, R, cb)
+    torch.cuda.synchronize()
+    assert hk.read_control(cb).alarm == 0
+    got = d.grid.cpu().numpy().ravel()
+    procs = min(64, len(os.sched_getaffinity(0)))
+    bands = [(y, min(y + 8, p.ny)) for y in range(0, p.ny, 8)]
+    with mpp.get_context("spawn").Pool(procs) as pool:
+        parts = pool.map(_cp4_rows, bands)
+    ora = np.zeros(p.nx * p.ny, dtype=np.float64)
+    seen = np.zeros(p.nx * p.ny, dtype=bool)
+    for idx, val in parts:
+        ora[idx] = val
+        seen[idx] = True
+    assert seen.all()
+    a = p.atoms.astype(np.float64)
+    ys, xs = np.divmod(np.arange(p.nx * p.ny), p.nx)
+    X = (np.float32(p.h) * xs.astype(np.float32)).astype(np.float64)
+    Y = (np.float32(p.h) * ys.astype(np.float32)).astype(np.float64)
+    mass = np.zeros(p.nx * p.ny)
+    for k in range(0, a.shape[0], 2000):
+        aa = a[k:k + 2000]
+        mass += (np.abs(aa[:, 3, None]) / np.sqrt((X[None] - aa[:, 0, None]) ** 2 + (Y[None] - aa[:, 1, None]) ** 2
+                                                   + aa[:, 2, None] ** 2)).sum(0)
+    bad = np.abs(got.astype(np.float64) - ora) > np.maximum(1e-5 * np.abs(ora), 4 * 2.0**-23 * mass)
+    assert not bad.any(), int(bad.sum())
+
+
+# ---------------------------------------------------------------------------------- variants, EXACT
+SMALL = lambda: [W.cp_small(), W.mriq_problem(6, 61, n_vox=200, seed=3), W.tpacf_small(n=150, n_rand=2)]
+
+
+@pytest.mark.parametrize("mode", [0, 1])
+def test_fi_only_binary_campaign_equals_oracle(mode):
+    """Row a7: FI-only campaigns (original program's sites, no detectors) in replica
+    and replay mode give the oracle's records bit for bit (EXACT); no alarm anywhere."""
+    probs = SMALL()
+    devs = [_mk(b, probs[b], 1) for b in range(3)]
+    gc, g = _gpu_campaign(devs, [None, None, None], 0xF10, 0, 1500, exact=1, mode=mode, variant=hk.HK_FI_ONLY)
+    oc, o = O.campaign(-1, probs, [O.Ranges(), O.Ranges(), O.Ranges()], 0xF10, 0, 1500, exact=1, mode=1, variant=1)
+    for k in ("site", "thread", "inst", "mask", "cls", "fail"):
+        assert np.array_equal(g[k], o[k]), k
+    assert np.array_equal(gc, oc) and (g["alarm"] == 0).all()
+    assert not any(hk.detector_site(int(b), int(s), 4) for b, s in zip(g["bench"], g["site"]))
+
+
+@pytest.mark.parametrize("mode", [0, 1])
+def test_alpha_ten_ranges_campaign_equals_oracle(mode):
+    """R11: ranges widened by alpha = 10 on both sides; EXACT records bit-exact."""
+    probs = SMALL()
+    devs = [_mk(b, probs[b], 1) for b in range(3)]
+    R = [hk.profile_ranges(d, alpha=10.0) for d in devs]
+    gc, g = _gpu_campaign(devs, R, 0xA10, 0, 1500, exact=1, mode=mode)
+    orr = [O.profile_ranges(b, probs[b], exact=1, alpha=10.0) for b in range(3)]
+    oc, o = O.campaign(-1, probs, orr, 0xA10, 0, 1500, exact=1, mode=1)
+    for k in ("cls", "alarm", "fail", "margin"):
+        assert np.array_equal(g[k], o[k]), k
+    assert np.array_equal(gc, oc)
+
+
+@pytest.mark.parametrize("mode", [0, 1])
+def test_small_hang_factor_campaign_equals_oracle(mode):
+    """R17 with T = 2 (PAPER L1997-2001 uses 10): more corrupted loops become hangs; records bit-exact."""
+    probs = SMALL()
+    devs = [_mk(b, probs[b], 1) for b in range(3)]
+    R = [hk.profile_ranges(d) for d in devs]
+    gc, g = _gpu_campaign(devs, R, 0x4A9, 0, 3000, exact=1, mode=mode, hang_factor=2)
+    orr = [O.profile_ranges(b, probs[b], exact=1) for b in range(3)]
+    oc, o = O.campaign(-1, probs, orr, 0x4A9, 0, 3000, exact=1, mode=1, hang_factor=2)
+    for k in ("cls", "alarm", "fail"):
+        assert np.array_equal(g[k], o[k]), k
+    assert np.array_equal(gc, oc)
+    assert ((g["fail"] & 2) != 0).sum() > 0  # some hangs were produced
+
+
+def test_tpacf_je_flips_hang_or_crash_identically_in_replicas_replay_and_oracle():
+    """The warp-parallel FI program of the TPACF replicas on the case pinned by hand in
+    tests/test_oracle_pins.py: campaigns restricted to site 12 (je @live) flip je at a random
+    iteration; with T = 10 high-bit flips of short self-row loops become hangs, with T = 100 most of
+    them walk off the buffer first.  Replica, replay and oracle records (class, failure) agree."""
+    p = W.tpacf_small(n=64, n_rand=2)
+    d = _mk(2, p)
+    R = hk.profile_ranges(d)
+    masks = (hk.ALL_SITES, hk.DEFAULT_SITE_MASKS[1], 1 << 12)
+    fails = {}
+    for T in (10, 100):
+        c0, r0 = _gpu_campaign([None, None, d], [None, None, R], 0x7, 0, 400, bench_mode=2, mode=0, site_masks=masks,
+                               hang_factor=T)
+        c1, r1 = _gpu_campaign([None, None, d], [None, None, R], 0x7, 0, 400, bench_mode=2, mode=1, site_masks=masks,
+                               hang_factor=T)
+        assert np.array_equal(r0["cls"], r1["cls"]) and np.array_equal(r0["fail"], r1["fail"])
+        oc, o = O.campaign(2, [None, None, p], [None, None, O.profile_ranges(2, p)], 0x7, 0, 400, mode=1,
+                           site_masks=masks, hang_factor=T)
+        assert np.array_equal(r0["fail"], o["fail"]) and np.array_equal(r0["cls"], o["cls"])
+        fails[T] = (int(((r0["fail"] & 2) != 0).sum()), int(((r0["fail"] & 1) != 0).sum()))
+    assert fails[10][0] > fails[100][0] and fails[10][0] > 0  # a larger T turns hangs into crashes
+
+
+# ---------------------------------------------------------------------------------- gloo world 2
+def _free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def _rank_worker(rank, world, port, total, q):
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_ipps_yimpski11_b200 import hauberk as H
+    from paper_conf_ipps_yimpski11_b200 import parallel as par
+    torch.cuda.set_device(0)
+    probs = [W.cp_config1(), W.mriq_problem(16, 512, seed=0x4D5249), W.tpacf_problem(1024, 2)]
+    devs = [[H.CPDevice, H.MRIQDevice, H.TPACFDevice][b].from_problem(probs[b], "cuda") for b in range(3)]
+    R = [H.profile_ranges(dv) for dv in devs]
+    first, cnt = par.shard(total, rank, world)
+    counts = torch.zeros((3, 5), dtype=torch.int64, device="cuda")
+    rec = H.records_tensor(cnt, "cuda")
+    with H.CampaignSession(-1, devs, R, 0x2AA, mode=0) as S:
+        S.run(first, cnt, counts, records=rec)
+        torch.cuda.synchronize()
+    cls = torch.from_numpy(H.records_numpy(rec)["cls"].astype(np.int64))
+    par.all_reduce_counts(counts)
+    sizes = [par.shard(total, r, world)[1] for r in range(world)]
+    got = [torch.zeros(sz, dtype=torch.int64) for sz in sizes]
+    dist.all_gather(got, torch.nn.functional.pad(cls, (0, max(sizes) - cls.numel())))  # equal-length gather
+    if rank == 0:
+        q.put((counts.cpu().numpy(), np.concatenate([g[:sz].numpy() for g, sz in zip(got, sizes)])))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_gloo_world2_product_campaign_on_one_gpu_equals_single_process():
+    """two ranks (gloo, both on cuda:0) run contiguous shards of the same seeded
+    replica-mode campaign through hauberk_campaign_*; the all-reduced counters and the gathered
+    classes equal one process running the whole index range."""
+    total = 1800
+    ctx = mpp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_rank_worker, args=(r, 2, port, total, q)) for r in range(2)]
+    for pr in procs:
+        pr.start()
+    counts2, cls2 = q.get(timeout=600)
+    for pr in procs:
+        pr.join(timeout=120)
+        assert pr.exitcode == 0
+    probs = [W.cp_config1(), W.mriq_problem(16, 512, seed=0x4D5249), W.tpacf_problem(1024, 2)]
+    devs = [_mk(b, probs[b]) for b in range(3)]
+    R = [hk.profile_ranges(dv) for dv in devs]
+    c1, r1 = _gpu_campaign(devs, R, 0x2AA, 0, total, mode=0)
+    assert np.array_equal(counts2, c1)
+    assert np.array_equal(cls2, r1["cls"].astype(np.int64))
+
+
+def test_bench_two_gloo_ranks_equal_one_rank():
+    """bench.py's campaign path (weak scaling, NCCL on a real multi-GPU box) as 2 ranks on one GPU
+    over gloo (HK_DIST_BACKEND=gloo): the per-step slices of 2 ranks x P injections cover the same
+    indices as 1 rank x 2P, so the all-reduced outcome counters must be identical."""
+    import json
+    import subprocess
+    import sys
+    common = ["--steps", "2", "--warmup", "3", "--no-overhead", "--no-cpu", "--no-multibit", "--no-fp-study",
+              "--replay-count", "1000"]
+    env = dict(os.environ, HK_DIST_BACKEND="gloo")
+    port = str(_free_port())
+    r2 = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+                         "--master-addr", "127.0.0.1", "--master-port", port, "bench.py", "--gpus", "2",
+                         "--per-rank", "300"] + common, cwd=ROOT, env=env, capture_output=True, text=True, timeout=900)
+    assert r2.returncode == 0, r2.stderr[-3000:]
+    r1 = subprocess.run([sys.executable, "bench.py", "--per-rank", "600"] + common, cwd=ROOT, capture_output=True,
+                        text=True, timeout=900)
+    assert r1.returncode == 0, r1.stderr[-3000:]
+    j2 = json.loads([l for l in r2.stdout.splitlines() if l.startswith("{")][-1])
+    j1 = json.loads([l for l in r1.stdout.splitlines() if l.startswith("{")][-1])
+    assert j2["n_gpus"] == 2 and j1["n_gpus"] == 1
+    assert j2["outcomes"] == j1["outcomes"]
+    assert j2["fi_only_outcomes"] == j1["fi_only_outcomes"]
+    assert j2["ranges_identical_across_ranks"] is True

@@ -262,7 +262,8 @@ HK_API int32_t hauberk_version(void);
 HK_API uint64_t hauberk_launch_count(void);
 
 /* Optional CUDA-event timing of the main kernels (cls 0: FT/BASE/PROFILE benchmark kernel,
- * cls 1: FI&FT campaign replicas), recorded on each kernel's launch stream while enabled.
+ * cls 1: FI&FT campaign replicas, cls 2: replay kernels, cls 3: fused MRI-Q + TPACF replica
+ * launches — each such launch is recorded under both benchmarks with that benchmark's work), recorded on each kernel's launch stream while enabled.
  * timing_read synchronises on the recorded events and returns the summed device time (ms),
  * the number of launches and the work (pairs / interactions) they computed, then forgets them.
  * Disabling drops unread records.  Not thread-safe; used by bench.py for roofline numbers. */

@@ -56,6 +56,13 @@ cudaError_t tpacf_fi_launch(int kind, bool ft, const hk_tpacf_args& a, const Dev
                             int nrep, unsigned long long* hist0, hk_control* cb0, void* lut_ws, bool real,
                             cudaStream_t s);
 
+// fused MRI-Q + TPACF replicas (mix.cu): rm MRI-Q replicas of Q-kernel site kinds (no PhiMag) and
+// rt TPACF replicas in one launch; outputs / controls exactly as mriq_fi_launch + tpacf_fi_launch
+bool mix_supported(const hk_mriq_args& m, const hk_tpacf_args& t);
+cudaError_t mix_fi_launch(bool ft, const hk_mriq_args& ma, const DevRanges& mR, int mndet, const FaultRec* mfaults, int rm,
+                          float* mout0, int64_t mstride, hk_control* mcb0, const hk_tpacf_args& ta, const DevRanges& tR, int tndet,
+                          const FaultRec* tfaults, int rt, unsigned long long* thist0, hk_control* tcb0, void* tlut, cudaStream_t s);
+
 // replay accelerator (one CUDA thread per injection; classification fused)
 cudaError_t cp_replay_launch(int kind, bool ft, const hk_cp_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep,
                              const float* golden, const float* dM, hk_outcome* records, int64_t first, int64_t* counts,

@@ -749,6 +749,9 @@ struct hk_campaign_session {
   // replica mode, mixed campaigns: one forked stream per benchmark so the XU-bound MRI-Q
   // replicas and the issue-bound TPACF replicas can share SMs (joined back into `stream`)
   bool concurrent = false;
+  // replica mode, mixed campaigns: MRI-Q (Q-kernel sites) and TPACF replicas share fused launches
+  // (mix.cu) so both kinds of CTA are resident on every SM (HK_FUSED=0: separate launches)
+  bool fused = false;
   cudaStream_t sub[3]{};
   cudaEvent_t fork = nullptr, join[3]{};
 };
@@ -794,6 +797,8 @@ static hk_status session_create(int32_t bench_mode, const void* const args[3], c
   {
     const char* env = getenv("HK_CONCURRENT");
     S->concurrent = env ? atoi(env) != 0 : HK_CONCURRENT_DEFAULT;
+    const char* fe = getenv("HK_FUSED");
+    S->fused = (fe ? atoi(fe) != 0 : true) && C->mode == 0 && bench_mode == -1 && args[HK_MRIQ] && args[HK_TPACF];
   }
   hk_status st = HK_OK;
   cudaError_t e;
@@ -817,6 +822,11 @@ static hk_status session_create(int32_t bench_mode, const void* const args[3], c
     w.R = dev_ranges(ft ? ranges[b] : nullptr);  // the FI-only binary has no detectors
     w.ndet = ft ? ranges[b]->n_det : 0;
     w.batch = C->mode == 1 ? 1 : (C->batch > 0 ? C->batch : default_batch(b, own));
+    if (b == HK_TPACF && S->fused) {
+      S->fused = S->W[HK_MRIQ].used && mix_supported(S->mq, S->tp);
+      // a fused launch pairs as many TPACF replicas as MRI-Q ones (the TPACF workspace is small)
+      if (S->fused && C->batch <= 0 && !getenv("HK_BATCH_2")) w.batch = std::max(w.batch, S->W[HK_MRIQ].batch);
+    }
     if (C->mode == 1 && b == HK_TPACF && 3 * S->tp.n_bins > 96) { g_err = "replay supports n_bins <= 32"; st = HK_ERR_UNSUPPORTED; break; }
     const bool phimag_sites = b == HK_MRIQ && (C->site_mask[b] >> MRIQ_PHIMAG_SITE0) != 0;
     if (C->mode == 1 && phimag_sites) {
@@ -981,9 +991,41 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
     it.f.hang = S->cfg.hang_factor;
     items[(size_t)q] = it;
   }
-  std::stable_sort(items.begin(), items.end(), [](const Item& x, const Item& y) {
-    return x.b != y.b ? x.b < y.b : x.kind < y.kind;
-  });
+  const auto by_kind = [](const Item& x, const Item& y) { return x.b != y.b ? x.b < y.b : x.kind < y.kind; };
+  std::stable_sort(items.begin(), items.end(), by_kind);
+  // ---- fused MRI-Q + TPACF chunks first (MRI-Q slice, then TPACF slice), then the rest by kind
+  struct Chunk { size_t m_off; int rm; size_t t_off; int rt; };
+  std::vector<Chunk> chunks;
+  size_t rest_off = 0;
+  if (S->fused && S->cfg.mode == 0) {
+    std::vector<Item> M, T, order, rest;
+    for (const Item& it : items) {
+      if (it.b == HK_MRIQ && it.f.site < MRIQ_PHIMAG_SITE0) M.push_back(it);
+      else if (it.b == HK_TPACF) T.push_back(it);
+      else rest.push_back(it);
+    }
+    if (!M.empty() && !T.empty()) {
+      const int64_t nm = (int64_t)M.size(), nt = (int64_t)T.size();
+      const int64_t bm = S->W[HK_MRIQ].batch, bt = S->W[HK_TPACF].batch;
+      const int64_t k = std::max((nm + bm - 1) / bm, (nt + bt - 1) / bt);
+      order.reserve(items.size());
+      for (int64_t j = 0; j < k; ++j) {
+        const int64_t m0 = nm * j / k, m1 = nm * (j + 1) / k, t0 = nt * j / k, t1 = nt * (j + 1) / k;
+        if (m1 > m0 && t1 > t0) {
+          chunks.push_back(Chunk{order.size(), (int)(m1 - m0), order.size() + (size_t)(m1 - m0), (int)(t1 - t0)});
+          order.insert(order.end(), M.begin() + m0, M.begin() + m1);
+          order.insert(order.end(), T.begin() + t0, T.begin() + t1);
+        } else {
+          rest.insert(rest.end(), M.begin() + m0, M.begin() + m1);
+          rest.insert(rest.end(), T.begin() + t0, T.begin() + t1);
+        }
+      }
+      std::stable_sort(rest.begin(), rest.end(), by_kind);
+      rest_off = order.size();
+      order.insert(order.end(), rest.begin(), rest.end());
+      items.swap(order);
+    }
+  }
   // ---- upload through the pinned staging buffer (wait until the previous upload consumed it)
   if ((e = cudaEventSynchronize(S->uploaded)) != cudaSuccess) return cuda_fail(e, "staging");
   if (S->h_cap < items.size()) {
@@ -1032,10 +1074,27 @@ static hk_status session_run(hk_campaign_session* S, int64_t first, int64_t coun
     for (int b = 0; b < 3; ++b)
       if (touched[b] && (e = cudaStreamWaitEvent(S->sub[b], S->fork, 0)) != cudaSuccess) return cuda_fail(e, "fork");
   }
-  size_t q = 0;
+  // fused launches and any MRI-Q / TPACF launch of the rest share one stream (one workspace each)
+  const auto stream_of = [&](int b) { return conc ? S->sub[!chunks.empty() && b == HK_TPACF ? HK_MRIQ : b] : s0; };
+  for (const Chunk& c : chunks) {
+    s = stream_of(HK_MRIQ);
+    BenchWS& wm = S->W[HK_MRIQ];
+    BenchWS& wt = S->W[HK_TPACF];
+    const FaultRec* fm = S->d_faults + c.m_off;
+    const FaultRec* ftp = S->d_faults + c.t_off;
+    if ((e = mix_fi_launch(ft, S->mq, wm.R, std::min(wm.ndet, 2), fm, c.rm, (float*)wm.rep_out, wm.out_elems, wm.rep_cb, S->tp, wt.R,
+                           std::min(wt.ndet, 1), ftp, c.rt, (unsigned long long*)wt.rep_out, wt.rep_cb, wt.lut, s)) != cudaSuccess)
+      return cuda_fail(e, "fused FI");
+    if ((e = classify_fp_launch(HK_MRIQ, (float*)wm.rep_out, wm.out_elems, (const float*)wm.golden, wm.dM, wm.rep_cb, fm, c.rm,
+                                d_records, first, d_counts, d_site_counts, s)) != cudaSuccess ||
+        (e = classify_tpacf_launch((unsigned long long*)wt.rep_out, S->tp.n_rand, S->tp.n_bins, (const unsigned long long*)wt.golden,
+                                   wt.rep_cb, ftp, c.rt, d_records, first, d_counts, d_site_counts, s)) != cudaSuccess)
+      return cuda_fail(e, "classify");
+  }
+  size_t q = rest_off;
   while (q < items.size()) {
     const int b = items[q].b, kind = items[q].kind;
-    s = conc ? S->sub[b] : s0;
+    s = stream_of(b);
     size_t end = q;
     while (end < items.size() && items[end].b == b && items[end].kind == kind && (int)(end - q) < S->W[b].batch) ++end;
     const int nrep = (int)(end - q);

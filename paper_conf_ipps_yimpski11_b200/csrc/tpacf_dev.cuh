@@ -1,0 +1,1101 @@
+// tpacf_dev.cuh — device building blocks of the TPACF kernels (tpacf.cu) and of the fused
+// MRI-Q + TPACF replica kernel (mix.cu).  DESIGN.md §3.4 / §6.3.
+#pragma once
+
+#include "hk_internal.h"
+
+namespace hk {
+
+#ifndef HK_TP_NP_FI
+#define HK_TP_NP_FI 4  // points per CUDA thread, campaign replicas
+#endif
+#ifndef HK_TP_NP_SR
+#define HK_TP_NP_SR 2  // points per CUDA thread, single run (256-point items: a finer LPT schedule)
+#endif
+#ifndef HK_TP_MINB
+#define HK_TP_MINB 6     // replicas: 37 KB of shared memory per CTA -> 6 CTAs per SM, 80 registers
+#endif
+#ifndef HK_TP_MINB_SR
+#define HK_TP_MINB_SR 8  // single run: 25.5 KB per CTA -> 8 CTAs per SM, 64 registers
+#endif
+#ifndef HK_TP_SR_CHUNK
+#define HK_TP_SR_CHUNK 128  // partners per single-run chunk (<= TP_TILE)
+#endif
+#ifndef HK_TP_GROUP
+#define HK_TP_GROUP 0  // partners per group of the unmasked loop (0: 4 for NP >= 4, else 8)
+#endif
+constexpr int TP_THREADS = 128;
+constexpr int TP_WARPS = TP_THREADS / 32;
+constexpr int TP_TILE = 512;                // partners per shared-memory tile (6 KB)
+constexpr int TP_LUT = 2048;                // u-buckets: sign, 8 exponent bits, 2 mantissa bits
+
+struct TPParams {
+  const float* pts;
+  const float* edges;
+  const uint8_t* lut;     // [TP_LUT] 4 * bmin per u-bucket; built by tpacf_lut_kernel
+  const int* lut_ok;      // 1: every bucket holds at most one edge (else the binary search is used)
+  unsigned long long* hist;
+  hk_control* cb;
+  float* samples;
+  DevRanges R;
+  int32_t* accg;          // single run: per abstract thread partial sums of acc and cnt (zeroed per run)
+  int32_t* cntg;
+  int32_t n, nr, nb, ndet;
+  int32_t nblk;           // point blocks per histogram for the launching kernel's NP
+  int32_t g0, g1;         // abstract threads [g0, g1) of this run (single-run sharding)
+  uint32_t z;
+  int32_t one, four, eight;  // runtime 1, 4 and 8 (opaque to the compiler)
+};
+
+// ---------------------------------------------------------------------------------------------
+// Binning.  Definition: bin = #{e in [0, nb] : dot < edge[e]}, edges decreasing.
+//  * tp_bin_search: branch-free 5-step binary search over the edges (padded with -inf).
+//  * table: u = fl(1 - dot) is monotone (non-increasing) in dot and so is bin, so every bucket q of
+//    u's top 11 bits maps to a contiguous dot interval [dmin, dmax].  The device builds
+//    bmin = bin(dmax) per bucket and checks bin(dmin) <= bmin + 1; then bin = bmin + (dot < edge[bmin])
+//    exactly (edge[bmin] = -inf past the last edge; NaN dots compare false, and the canonical NaN u
+//    lands in a bucket whose bmin is bin(NaN) = 0).  The table holds 4 * bmin, the byte offset of
+//    edge[bmin], so the edge load needs no address arithmetic.
+// ---------------------------------------------------------------------------------------------
+__device__ __forceinline__ int32_t tp_bin_search(const float* Es, float dot) {
+  int32_t b = 0;
+#pragma unroll
+  for (int s = 16; s >= 1; s >>= 1) b += (dot < Es[b + s - 1]) ? s : 0;
+  return b;
+}
+// 4 * bin through the byte table L and the edges at the shared byte address eb (uniform)
+__device__ __forceinline__ uint32_t tp_b4_lut(const uint8_t* __restrict__ L, uint32_t eb, float dot) {
+  const float u = __fsub_rn(1.0f, dot);
+  const uint32_t b4 = L[fb(u) >> 21];
+  float e;
+  asm("ld.shared.f32 %0, [%1];" : "=f"(e) : "r"(eb + b4));
+  return (dot < e) ? b4 + 4u : b4;
+}
+// Every TPACF kernel carves its TPSmem from the start of dynamic shared memory, so the table and
+// the edges sit at link-time constant shared addresses: the pair loops index them from the symbol
+// ([reg + imm] addressing, no base register add per lookup).
+extern __shared__ __align__(128) unsigned char hk_tp_dsmem[];
+__device__ __forceinline__ uint32_t tp_b4_fixed(float dot) {
+  const uint32_t base = (uint32_t)__cvta_generic_to_shared(hk_tp_dsmem);
+  const float u = __fsub_rn(1.0f, dot);
+  uint32_t b4;
+  float e;
+  asm("ld.shared.u8 %0, [%1];" : "=r"(b4) : "r"(base + (fb(u) >> 21)));
+  asm("ld.shared.f32 %0, [%1];" : "=f"(e) : "r"(base + (uint32_t)TP_LUT + b4));
+  return (dot < e) ? b4 + 4u : b4;
+}
+template <bool LUT>
+__device__ __forceinline__ uint32_t tp_b4(const uint8_t* __restrict__, uint32_t, const float* Es, float dot) {
+  return LUT ? tp_b4_fixed(dot) : 4u * (uint32_t)tp_bin_search(Es, dot);
+}
+__device__ __forceinline__ void red_shared(uint32_t addr, uint32_t v) {
+  asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(addr), "r"(v) : "memory");
+}
+
+__device__ __forceinline__ float nup(float x) {
+  const uint32_t b = fb(x);
+  if ((b & 0x7fffffffu) == 0) return bf(1u);
+  return (b & 0x80000000u) ? bf(b - 1) : bf(b + 1);
+}
+__device__ __forceinline__ float ndown(float x) {
+  const uint32_t b = fb(x);
+  if ((b & 0x7fffffffu) == 0) return bf(0x80000001u);
+  return (b & 0x80000000u) ? bf(b + 1) : bf(b - 1);
+}
+__device__ __forceinline__ int32_t bin_def(const float* edges, int nb, float dot) {
+  int32_t b = 0;
+  for (int e = 0; e <= nb; ++e) b += (dot < edges[e]) ? 1 : 0;
+  return b;
+}
+
+
+// ---------------------------------------------------------------------------------------------
+// Shared memory: L[2048] u8 | E[32] f32 | B[2][3 * TP_TILE] f32 (packed x, y, z) |
+// H[warps][NP/2 words][nb2][32] u32 | part[warps * NP/2 * nb2] | flag
+// ---------------------------------------------------------------------------------------------
+struct TPSmem {
+  uint8_t* L;
+  float* E;
+  float* B;
+  uint32_t* H;
+  uint32_t* part;  // [TP_WARPS * NP/2 * nb2] flush scratch (the ring may hold a prefetched tile)
+  int* flag;
+};
+__host__ __device__ inline size_t tp_smem_bytes(int nb2, int np) {
+  return (size_t)TP_LUT + 32 * 4 + 2 * 3 * TP_TILE * 4 + (size_t)TP_WARPS * (np / 2) * nb2 * 33 * 4 + 16;
+}
+__device__ __forceinline__ TPSmem tp_carve(unsigned char* base, int nb2, int np) {
+  TPSmem S;
+  S.L = base;
+  S.E = reinterpret_cast<float*>(base + TP_LUT);
+  S.B = reinterpret_cast<float*>(base + TP_LUT + 128);
+  S.H = reinterpret_cast<uint32_t*>(base + TP_LUT + 128 + 2 * 3 * TP_TILE * 4);
+  S.part = reinterpret_cast<uint32_t*>(base + TP_LUT + 128 + 2 * 3 * TP_TILE * 4 + (size_t)TP_WARPS * (np / 2) * nb2 * 128);
+  S.flag = reinterpret_cast<int*>(reinterpret_cast<unsigned char*>(S.part) + (size_t)TP_WARPS * (np / 2) * nb2 * 4);
+  return S;
+}
+__device__ __forceinline__ void cp_async4(void* dst, const void* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async16(void* dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
+// Table + edges, once per CTA (the edges padded with -inf for the binary search).
+__device__ __forceinline__ void tp_stage_tables(const TPParams& p, const TPSmem& S) {
+  for (int k = threadIdx.x; k < TP_LUT / 16; k += TP_THREADS) cp_async16(S.L + 16 * k, p.lut + 16 * k);
+  if (threadIdx.x < 32) S.E[threadIdx.x] = threadIdx.x <= p.nb ? p.edges[threadIdx.x] : __int_as_float(0xff800000);
+  cp_async_commit();
+}
+template <int NP>
+__device__ __forceinline__ void tp_zero_hist(const TPParams& p, const TPSmem& S) {
+  const int nh = TP_WARPS * (NP / 2) * (p.nb + 2) * 32;
+  for (int k = threadIdx.x; k < nh; k += TP_THREADS) S.H[k] = 0u;
+}
+// Partners [j0, j0 + cnt) of set sb into ring slot `slot` (cnt <= TP_TILE; 4-byte async copies).
+__device__ __forceinline__ void tp_stage_tile(const TPParams& p, const TPSmem& S, int sb, int j0, int cnt, int slot) {
+  const float* src = p.pts + 3 * ((int64_t)sb * p.n + j0);
+  float* dst = S.B + slot * 3 * TP_TILE;
+  for (int k = threadIdx.x; k < 3 * cnt; k += TP_THREADS) cp_async4(dst + k, src + k);
+  cp_async_commit();
+}
+
+// Reduce the lane-private histograms (both 16-bit halves of every word) and add them to
+// hist[base + b]: each (warp, word, bin) row of 32 counters is summed (rotated start: no bank
+// conflicts), the rows of a bin combined in shared memory, then one u64 atomic per non-zero bin.
+template <int NP>
+__device__ __forceinline__ void tp_flush(const TPParams& p, const TPSmem& S, unsigned long long* hist, int base) {
+  const int nb2 = p.nb + 2, rows = TP_WARPS * (NP / 2);
+  uint32_t* part = S.part;
+  for (int t = threadIdx.x; t < rows * nb2; t += TP_THREADS) {
+    const uint32_t* row = S.H + (size_t)t * 32;
+    uint32_t s = 0;
+#pragma unroll 8
+    for (int l = 0; l < 32; ++l) {
+      const uint32_t w = row[(l + t) & 31];
+      s += (w & 0xffffu) + (w >> 16);
+    }
+    part[t] = s;
+  }
+  __syncthreads();
+  if (threadIdx.x < nb2) {
+    unsigned long long s = 0;
+    for (int w = 0; w < rows; ++w) s += part[w * nb2 + threadIdx.x];
+    if (s) atomicAdd(hist + base + threadIdx.x, s);
+  }
+}
+
+// ---------------------------------------------------------------------------------------------
+// Per-abstract-thread prologue (NL sites 0-10) and epilogue.
+// ---------------------------------------------------------------------------------------------
+struct TPPoint {
+  int32_t i, h, boff, jb, je, expect, base;
+  float x1, y1, z1;
+  uint32_t chk, alarm;
+  int32_t acc, cnt;  // acc in units of 4 (the table's 4 * bin) until divided
+  bool valid;
+};
+
+// i_dup / h_dup: the same indices recomputed from launch indices through the opaque zero.
+template <bool NL>
+__device__ __forceinline__ TPPoint tp_prologue(const TPParams& p, const unsigned long long* hist, int h, int i, int i_dup,
+                                               int h_dup, bool valid) {
+  const uint32_t z = p.z;
+  const int32_t n = p.n, nr = p.nr, nb2 = p.nb + 2;
+  TPPoint P;
+  P.valid = valid;
+  P.i = i;
+  P.h = h;
+  P.chk = 0;
+  P.alarm = 0;
+  if (NL) {
+    P.chk ^= (uint32_t)n ^ lohi_ptr(p.pts) ^ lohi_ptr(hist);
+    P.chk ^= (uint32_t)i; P.alarm |= (i_dup != i) ? AL_DUP : 0u;
+    P.chk ^= (uint32_t)h; P.alarm |= (h_dup != h) ? AL_DUP : 0u;
+  }
+  const int32_t aoff = (h <= nr ? h : 0) * n + i;
+  const int32_t sb = (h == 0) ? 0 : (h <= nr ? h : h - nr);
+  P.boff = sb * n;
+  P.jb = h <= nr ? i + 1 : 0;
+  P.je = n;
+  P.expect = max(P.je - P.jb, 0);
+  P.base = h * nb2;
+  if (NL) {
+    const int32_t h2 = opq(h, z), i2 = opq(i, z);
+    P.chk ^= (uint32_t)aoff; P.alarm |= ((h2 <= nr ? h2 : 0) * n + i2 != aoff) ? AL_DUP : 0u;
+    P.chk ^= (uint32_t)P.boff; P.alarm |= ((h2 == 0 ? 0 : (h2 <= nr ? h2 : h2 - nr)) * n != P.boff) ? AL_DUP : 0u;
+    P.chk ^= (uint32_t)P.jb; P.alarm |= ((h2 <= nr ? i2 + 1 : 0) != P.jb) ? AL_DUP : 0u;
+    P.chk ^= (uint32_t)P.je; P.alarm |= (opq(n, z) != P.je) ? AL_DUP : 0u;
+    P.chk ^= (uint32_t)P.expect; P.alarm |= (max(opq(P.je, z) - P.jb, 0) != P.expect) ? AL_DUP : 0u;
+    P.chk ^= (uint32_t)P.base; P.alarm |= (h2 * nb2 != P.base) ? AL_DUP : 0u;
+  }
+  const float* A = p.pts + 3 * (int64_t)(valid ? aoff : 0);
+  P.x1 = A[0]; P.y1 = A[1]; P.z1 = A[2];
+  if (NL) {
+    const float* A2 = p.pts + 3 * (int64_t)(valid ? opq(aoff, z) : 0);
+    P.chk ^= fb(P.x1); P.alarm |= (fb(A2[0]) != fb(P.x1)) ? AL_DUP : 0u;
+    P.chk ^= fb(P.y1); P.alarm |= (fb(A2[1]) != fb(P.y1)) ? AL_DUP : 0u;
+    P.chk ^= fb(P.z1); P.alarm |= (fb(A2[2]) != fb(P.z1)) ? AL_DUP : 0u;
+    P.chk ^= (uint32_t)opq(i, z) ^ (uint32_t)opq(h, z) ^ (uint32_t)opq(aoff, z) ^ (uint32_t)opq(P.jb, z);
+  }
+  P.acc = 0;
+  P.cnt = 0;
+  if (!valid) P.jb = INT32_MAX;  // takes part in no pair
+  return P;
+}
+
+// NL exit XORs of the loop-live values and the parameters, then the checksum test.
+template <bool NL>
+__device__ __forceinline__ void tp_nl_exit(const TPParams& p, TPPoint& P, const unsigned long long* hist) {
+  if (!NL) return;
+  const uint32_t z = p.z;
+  P.chk ^= (uint32_t)opq(P.boff, z) ^ (uint32_t)opq(P.je, z) ^ (uint32_t)opq(P.base, z);
+  P.chk ^= opqf(P.x1, z) ^ opqf(P.y1, z) ^ opqf(P.z1, z) ^ (uint32_t)opq(P.expect, z);
+  P.chk ^= ((uint32_t)p.n + z) ^ (lohi_ptr(p.pts) + z) ^ (lohi_ptr(hist) + z);
+  if (P.chk != 0) P.alarm |= AL_CHK;
+}
+
+// HauberkCheckEqual(cnt, expect) / HauberkCheckRange(acc / cnt) after the whole loop (L1405-1429);
+// PROFILE writes the sample acc / cnt.  acc and cnt are the full-loop sums.
+template <int V>
+__device__ __forceinline__ void tp_checks(const TPParams& p, TPPoint& P, hk_control* cb, int64_t g) {
+  constexpr bool L = (V & V_L) != 0, PROF = (V & V_PROF) != 0;
+  if (L && P.cnt != P.expect) P.alarm |= AL_COUNT;
+  if ((L || PROF) && P.cnt != 0 && p.ndet > 0) {
+    const float v = __fdiv_rn((float)P.acc, (float)P.cnt);
+    if (PROF) p.samples[g] = v;
+    if (L && p.R.n[0] > 0 && !in_range<false>(p.R, 0, v, nullptr)) {
+      P.alarm |= AL_RANGE;
+      record_outlier(cb, 0, v);
+    }
+  }
+}
+
+__device__ __forceinline__ float tp_dot(const TPPoint& P, float x2, float y2, float z2) {
+  return __fmaf_rn(P.z1, z2, __fmaf_rn(P.y1, y2, __fmul_rn(P.x1, x2)));
+}
+
+// ---------------------------------------------------------------------------------------------
+// The pair loops over one staged tile.  Hw[w] = this lane's histogram word w (shared byte address;
+// point k counts in word k/2, half k%2); inc[k] = 1 / 0x10000 (0 for an absent point or the faulted
+// abstract thread of an FI CTA, whose whole loop runs in the FI program instead).
+//  * tp_pairs_all: every point of the CTA has all of [k0, k1) as partners (no masks); groups of G
+//    partners (G = 32 / NP, i.e. 3 * G / 4 broadcast LDS.128 per group) with the counters advanced
+//    by G per group (the strength reduction any compiler applies to an unrolled cnt++; the FI
+//    program keeps the per-iteration increment);
+//  * tp_pairs_masked: the diagonal of a self-correlation row (j >= jb differs per point).
+// ---------------------------------------------------------------------------------------------
+struct TPLoopCtx {
+  const uint8_t* L;
+  uint32_t eb;
+  const float* Es;
+};
+
+template <int NP, bool CNT, bool LUT>
+__device__ __forceinline__ void tp_pair1(const TPLoopCtx& c, const uint32_t (&Hw)[NP / 2], TPPoint (&P)[NP],
+                                         const uint32_t (&inc)[NP], float x2, float y2, float z2, int j, bool masked) {
+#pragma unroll
+  for (int k = 0; k < NP; ++k) {
+    const uint32_t b4 = tp_b4<LUT>(c.L, c.eb, c.Es, tp_dot(P[k], x2, y2, z2));
+    const bool on = !masked || j >= P[k].jb;
+    red_shared(Hw[k / 2] + b4 * 32u, on ? inc[k] : 0u);
+    if (CNT) {
+      P[k].acc += on ? (int32_t)b4 : 0;
+      P[k].cnt += on ? 1 : 0;
+    }
+  }
+}
+
+template <int NP, bool CNT, bool LUT>
+__device__ __forceinline__ void tp_pairs_all(const TPParams& p, const TPLoopCtx& c, const float* __restrict__ Bt,
+                                             const uint32_t (&Hw)[NP / 2], TPPoint (&P)[NP], const uint32_t (&inc)[NP],
+                                             int k, int k1) {
+  if (!LUT) {  // the binary-search fallback (a bucket holds two edges): plain loop, rare
+#pragma unroll 1
+    for (; k < k1; ++k) tp_pair1<NP, CNT, LUT>(c, Hw, P, inc, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], 0, false);
+    return;
+  }
+  // partners per group: G * NP pairs per thread and group (16 for NP = 4: enough independent
+  // table lookups in flight within the 80-register budget of 6 CTAs per SM)
+  constexpr int G = HK_TP_GROUP > 0 ? HK_TP_GROUP : (NP >= 4 ? 4 : 8);
+  static_assert(G % 4 == 0, "groups are whole 48-byte partner quads");
+  for (; k < k1 && (k & 3); ++k) tp_pair1<NP, CNT, LUT>(c, Hw, P, inc, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], 0, false);
+  const float4* __restrict__ T4 = reinterpret_cast<const float4*>(Bt);
+#pragma unroll 1
+  for (; k + G - 1 < k1; k += G) {
+    const int k3 = (k >> 2) * 3;
+    float xs[G], ys[G], zs[G];
+#pragma unroll
+    for (int q = 0; q < G / 4; ++q) {
+      const float4 v0 = T4[k3 + 3 * q], v1 = T4[k3 + 3 * q + 1], v2 = T4[k3 + 3 * q + 2];
+      xs[4 * q] = v0.x; ys[4 * q] = v0.y; zs[4 * q] = v0.z;
+      xs[4 * q + 1] = v0.w; ys[4 * q + 1] = v1.x; zs[4 * q + 1] = v1.y;
+      xs[4 * q + 2] = v1.z; ys[4 * q + 2] = v1.w; zs[4 * q + 2] = v2.x;
+      xs[4 * q + 3] = v2.y; ys[4 * q + 3] = v2.z; zs[4 * q + 3] = v2.w;
+    }
+    uint32_t b[NP][G];
+#pragma unroll
+    for (int u = 0; u < G; ++u)
+#pragma unroll
+      for (int kk = 0; kk < NP; ++kk) b[kk][u] = tp_b4<LUT>(c.L, c.eb, c.Es, tp_dot(P[kk], xs[u], ys[u], zs[u]));
+#pragma unroll
+    for (int u = 0; u < G; ++u)
+#pragma unroll
+      for (int kk = 0; kk < NP; ++kk) red_shared(Hw[kk / 2] + b[kk][u] * 32u, inc[kk]);
+    if (CNT) {
+#pragma unroll
+      for (int kk = 0; kk < NP; ++kk) {
+#pragma unroll
+        for (int u = 0; u < G; u += 2) P[kk].acc += (int32_t)(b[kk][u] + b[kk][u + 1]);
+        P[kk].cnt = count_inc(P[kk].cnt, G == 8 ? p.eight : (G == 4 ? p.four : p.one * G));
+      }
+    }
+  }
+  for (; k < k1; ++k) tp_pair1<NP, CNT, LUT>(c, Hw, P, inc, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], 0, false);
+}
+
+// The diagonal of a self-correlation row, segment S: partners j in [i0 + 128 S, i0 + 128 (S + 1))
+// (tile-relative [ka, kb)).  Point k of a thread is i0 + 128 k + t, so for these partners points
+// k < S are all active (j > i), point S is masked (j >= jb) and points k > S take no part.
+template <int NP, bool CNT, bool LUT, int S>
+__device__ __forceinline__ void tp_diag_seg(const TPLoopCtx& c, const float* __restrict__ Bt, const uint32_t (&Hw)[NP / 2],
+                                            TPPoint (&P)[NP], const uint32_t (&inc)[NP], int jt0, int ka, int kb) {
+#pragma unroll 1
+  for (int k = ka; k < kb; ++k) {
+    const float x2 = Bt[3 * k], y2 = Bt[3 * k + 1], z2 = Bt[3 * k + 2];
+#pragma unroll
+    for (int q = 0; q <= S; ++q) {
+      const uint32_t b4 = tp_b4<LUT>(c.L, c.eb, c.Es, tp_dot(P[q], x2, y2, z2));
+      const bool on = q < S || jt0 + k >= P[q].jb;
+      red_shared(Hw[q / 2] + b4 * 32u, on ? inc[q] : 0u);
+      if (CNT) {
+        P[q].acc += on ? (int32_t)b4 : 0;
+        P[q].cnt += on ? 1 : 0;
+      }
+    }
+  }
+}
+template <int NP, bool CNT, bool LUT, int S = 0>
+__device__ __forceinline__ void tp_diag(const TPLoopCtx& c, const float* __restrict__ Bt, const uint32_t (&Hw)[NP / 2],
+                                        TPPoint (&P)[NP], const uint32_t (&inc)[NP], int i0, int jt0, int k0, int km) {
+  const int ka = max(k0, i0 + S * TP_THREADS - jt0), kb = min(km, i0 + (S + 1) * TP_THREADS - jt0);
+  if (ka < kb) tp_diag_seg<NP, CNT, LUT, S>(c, Bt, Hw, P, inc, jt0, ka, kb);
+  if constexpr (S + 1 < NP) tp_diag<NP, CNT, LUT, S + 1>(c, Bt, Hw, P, inc, i0, jt0, k0, km);
+}
+
+// Pairs of the staged tile Bt (partners jt0 + k) for k in [k0, k1): [k0, km) with per-point masks
+// (partners below jall = min(i0 + NP * 128, N) in a self-correlation row: its diagonal, in
+// segments), [km, k1) for all points.
+template <int NP, bool CNT, bool LUT>
+__device__ __forceinline__ void tp_tile_pairs(const TPParams& p, const TPLoopCtx& c, const float* __restrict__ Bt,
+                                              const uint32_t (&Hw)[NP / 2], TPPoint (&P)[NP], const uint32_t (&inc)[NP],
+                                              int jt0, int k0, int k1, int jall, int i0) {
+  const int km = min(max(jall - jt0, k0), k1);
+  if (k0 < km) tp_diag<NP, CNT, LUT>(c, Bt, Hw, P, inc, i0, jt0, k0, km);
+  tp_pairs_all<NP, CNT, LUT>(p, c, Bt, Hw, P, inc, km, k1);
+}
+template <int NP>
+__device__ __forceinline__ void tp_lane_hist(const TPParams& p, const TPSmem& S, uint32_t (&Hw)[NP / 2]) {
+  const uint32_t lane = lane_id(), warp = threadIdx.x >> 5;
+#pragma unroll
+  for (int w = 0; w < NP / 2; ++w) Hw[w] = smem_u32(S.H + (((size_t)warp * (NP / 2) + w) * (p.nb + 2)) * 32 + lane);
+}
+
+// One work item: the points i0 + t + 128 k (k < NP) of histogram h against partners [jr0, jr1)
+// (already clipped to the block's [jlo, N)), streamed tile by tile through the ring.  The tables
+// are staged and the histogram zeroed by the caller.
+template <int NP, int V, bool LUT>
+__device__ __forceinline__ void tp_item_loop(const TPParams& p, const TPSmem& S, TPPoint (&P)[NP], const uint32_t (&inc)[NP],
+                                             int h, int i0, int jr0, int jr1) {
+  constexpr bool CNT = (V & (V_L | V_PROF)) != 0;
+  const int sb = (h == 0) ? 0 : (h <= p.nr ? h : h - p.nr);
+  const int js = jr0 & ~3;  // tiles start on 4-partner boundaries (16-byte aligned groups in smem)
+  const int nt = jr1 > jr0 ? (jr1 - js + TP_TILE - 1) / TP_TILE : 0;
+  // partners below jall need per-point masks (self rows: j >= i + 1), the rest do not
+  const int jall = h <= p.nr ? min(i0 + NP * TP_THREADS, p.n) : 0;
+  const uint32_t lane = lane_id(), warp = threadIdx.x >> 5;
+  uint32_t Hw[NP / 2];
+#pragma unroll
+  for (int w = 0; w < NP / 2; ++w) Hw[w] = smem_u32(S.H + (((size_t)warp * (NP / 2) + w) * (p.nb + 2)) * 32 + lane);
+  const TPLoopCtx c{S.L, smem_u32(S.E), S.E};
+  if (nt > 0) tp_stage_tile(p, S, sb, js, min(TP_TILE, jr1 - js), 0);
+  for (int t = 0; t < nt; ++t) {
+    const int jt0 = js + t * TP_TILE;
+    if (t + 1 < nt) {
+      const int jn = jt0 + TP_TILE;
+      tp_stage_tile(p, S, sb, jn, min(TP_TILE, jr1 - jn), (t + 1) & 1);
+      cp_async_wait<1>();
+    } else {
+      cp_async_wait<0>();
+    }
+    __syncthreads();
+    tp_tile_pairs<NP, CNT, LUT>(p, c, S.B + (t & 1) * 3 * TP_TILE, Hw, P, inc, jt0, max(jr0, jt0) - jt0,
+                                min(jr1, jt0 + TP_TILE) - jt0, jall, i0);
+    __syncthreads();  // slot t & 1 is refilled by the stage of tile t + 2
+  }
+}
+
+template <int NP>
+__device__ __forceinline__ void tp_points(const TPParams& p, const unsigned long long* hist, int h, int blk, int64_t g0,
+                                          int64_t g1, TPPoint (&P)[NP], bool nl) {
+  const int i0 = blk * NP * TP_THREADS;
+  const int64_t gb = (int64_t)h * p.n;
+#pragma unroll
+  for (int k = 0; k < NP; ++k) {
+    const int i = i0 + k * TP_THREADS + threadIdx.x;
+    const bool v = i < p.n && gb + i >= g0 && gb + i < g1;
+    const int idup = (int)((blk ^ p.z) * (NP * TP_THREADS) + k * TP_THREADS + (threadIdx.x ^ p.z));
+    P[k] = nl ? tp_prologue<true>(p, hist, h, i, idup, (int)((uint32_t)h ^ p.z), v)
+              : tp_prologue<false>(p, hist, h, i, idup, (int)((uint32_t)h ^ p.z), v);
+  }
+}
+
+// The lane-private histogram outlives a visit: consecutive visits of a CTA with the same h keep
+// counting into it and it is flushed when h changes, before the 16-bit halves could overflow
+// (< 32768 partners per slot since the last flush) and at the end.
+struct TPHistState {
+  int h;      // histogram the shared counters belong to (-1: none)
+  int since;  // partners counted per slot since the last flush (upper bound)
+};
+
+template <int NP>
+__device__ __forceinline__ void tp_hist_switch(const TPParams& p, const TPSmem& S, TPHistState* st, int h, int partners) {
+  // uniform over the CTA (st is in shared memory and read after a barrier)
+  if (st->h != h || st->since + partners >= 32768) {
+    if (st->h >= 0) {
+      tp_flush<NP>(p, S, p.hist, st->h * (p.nb + 2));
+      __syncthreads();  // flush read the counters and the ring before they are reused
+    }
+    tp_zero_hist<NP>(p, S);
+    __syncthreads();
+    if (threadIdx.x == 0) { st->h = h; st->since = 0; }
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) st->since += partners;
+}
+
+// ============================================================================================
+// Single run (BASE / FT / FT_NL / FT_L / PROFILE): one wave of CTAs that steal partner chunks.
+// A row = (histogram h, point block blk) of 128 * NP points; its partners [jlo, N) are cut into
+// chunks of HK_TP_SR_CHUNK.  CTAs start spread over the rows and claim chunks of a row with one
+// atomic each (claimed one chunk ahead, so the claim latency and the next tile's staging overlap
+// the current chunk), moving to the next row when it is exhausted: the work is balanced at chunk
+// granularity.  A CTA's stay on a row (a "visit") keeps its points' (acc, cnt) in registers;
+// leaving the row it adds them to the per-thread partial sums (exact integer combine) and its
+// chunk count to the row's; the visit that completes the row runs the loop-exit checks.
+// ============================================================================================
+struct TPSR {
+  int* row_next;  // [nrows] chunk claim counters (zeroed per run)
+  int* row_done;  // [nrows] chunks completed (zeroed per run)
+  int nrows;
+};
+
+__device__ __forceinline__ void tp_row_geom(const TPParams& p, int row, int* h, int* blk, int* c0, int* nch) {
+  constexpr int NP = HK_TP_NP_SR;
+  *h = row / p.nblk;
+  *blk = row - *h * p.nblk;
+  const int i0 = *blk * NP * TP_THREADS;
+  const int64_t gb = (int64_t)*h * p.n;
+  const int i1 = min(i0 + NP * TP_THREADS, p.n);
+  const bool any = gb + i0 < p.g1 && gb + i1 > p.g0;  // some point of the block is in this run
+  const int jlo = *h <= p.nr ? i0 + 1 : 0;
+  const int nc = (p.n + HK_TP_SR_CHUNK - 1) / HK_TP_SR_CHUNK;
+  *c0 = jlo / HK_TP_SR_CHUNK;
+  *nch = (any && jlo < p.n) ? nc - *c0 : 0;
+}
+
+// Warp 0: the next (row, chunk) starting at `row` (row = -1 once every row is exhausted).  The 32
+// lanes look at 32 rows at a time (one load of each claim counter), then lane 0 claims in the
+// first row that still had chunks; only exhausted rows are skipped, so the final sweep of a CTA
+// costs nrows / 32 load rounds instead of nrows sequential atomics.
+__device__ __forceinline__ int2 tp_sr_claim(const TPParams& p, const TPSR& q, int row) {
+  const unsigned FULL = 0xffffffffu;
+  const uint32_t lane = lane_id();
+  for (int scanned = 0; scanned < q.nrows; scanned += 32) {
+    int r = row + scanned + (int)lane;
+    r = r < q.nrows ? r : r - q.nrows;
+    if (r >= q.nrows) r -= q.nrows;
+    int h, blk, c0, nch = 0;
+    bool avail = false;
+    if (scanned + (int)lane < q.nrows) {
+      tp_row_geom(p, r, &h, &blk, &c0, &nch);
+      avail = nch > 0 && __ldcg(q.row_next + r) < nch;
+    }
+    unsigned m = __ballot_sync(FULL, avail);
+    while (m) {
+      const int l = __ffs(m) - 1;
+      const int rl = __shfl_sync(FULL, r, l), nl = __shfl_sync(FULL, nch, l);
+      int k = 0;
+      if (lane == 0) k = atomicAdd(q.row_next + rl, 1);
+      k = __shfl_sync(FULL, k, 0);
+      if (k < nl) return make_int2(rl, k);
+      m &= ~(1u << l);
+    }
+  }
+  return make_int2(-1, 0);
+}
+
+// Stage chunk k of `row` into ring slot `slot` (no-op for row < 0).
+__device__ __forceinline__ void tp_sr_stage(const TPParams& p, const TPSmem& S, int2 ch, int slot) {
+  if (ch.x < 0) return;
+  int h, blk, c0, nch;
+  tp_row_geom(p, ch.x, &h, &blk, &c0, &nch);
+  const int i0 = blk * HK_TP_NP_SR * TP_THREADS;
+  const int jlo = h <= p.nr ? i0 + 1 : 0;
+  const int j0 = max(jlo, (c0 + ch.y) * HK_TP_SR_CHUNK), j1 = min(p.n, (c0 + ch.y + 1) * HK_TP_SR_CHUNK);
+  const int sb = (h == 0) ? 0 : (h <= p.nr ? h : h - p.nr);
+  tp_stage_tile(p, S, sb, j0 & ~3, j1 - (j0 & ~3), slot);
+}
+
+// Claims run two chunks ahead of the computation: while chunk `cur` is computed, chunk `nxt`'s
+// tile is in flight and lane 0 of warp 0 has the atomic for the chunk after it outstanding (a
+// speculative claim in nxt's row; the scan of tp_sr_claim only when that row is exhausted).
+template <int V, bool LUT>
+__device__ __forceinline__ void tp_sr_run(const TPParams& p, const TPSmem& S, const TPSR& q, TPHistState* st, int2* claim) {
+  constexpr int NP = HK_TP_NP_SR;
+  constexpr bool NL = (V & V_NL) != 0, L = (V & V_L) != 0, PROF = (V & V_PROF) != 0, CNT = L || PROF;
+  if (threadIdx.x < 32) {
+    const int2 a = tp_sr_claim(p, q, (int)(((int64_t)blockIdx.x * q.nrows) / gridDim.x));
+    const int2 b = a.x >= 0 ? tp_sr_claim(p, q, a.x) : a;
+    if (threadIdx.x == 0) { claim[0] = a; claim[1] = b; }
+  }
+  __syncthreads();
+  int2 cur = claim[0], nxt = claim[1];
+  int slot = 0;
+  tp_sr_stage(p, S, cur, 0);
+  tp_sr_stage(p, S, nxt, 1);
+  uint32_t Hw[NP / 2];
+  tp_lane_hist<NP>(p, S, Hw);
+  const TPLoopCtx c{S.L, smem_u32(S.E), S.E};
+  // the current visit
+  int vrow = -1, h = 0, blk = 0, c0 = 0, nch = 0, i0 = 0, jlo = 0, jall = 0, visited = 0;
+  int64_t gb = 0;
+  TPPoint P[NP];
+  uint32_t inc[NP];
+  auto end_visit = [&]() {
+#pragma unroll
+    for (int k = 0; k < NP; ++k) {
+      P[k].acc /= 4;
+      tp_nl_exit<NL>(p, P[k], p.hist);
+      if (CNT && P[k].valid && P[k].cnt) {  // exact combine of this visit's partial sums
+        atomicAdd(p.accg + gb + P[k].i, P[k].acc);
+        atomicAdd(p.cntg + gb + P[k].i, P[k].cnt);
+      }
+    }
+    if (CNT) {
+      __syncthreads();  // every thread's combine atomics issued
+      if (threadIdx.x == 0) {
+        __threadfence();
+        *S.flag = atomicAdd(q.row_done + vrow, visited) + visited == nch;
+      }
+      __syncthreads();
+      if (*S.flag) {  // this visit completed the row: the loop-exit checks of its points
+        __threadfence();
+#pragma unroll
+        for (int k = 0; k < NP; ++k)
+          if (P[k].valid) {
+            P[k].acc = __ldcg(p.accg + gb + P[k].i);
+            P[k].cnt = __ldcg(p.cntg + gb + P[k].i);
+            tp_checks<V>(p, P[k], p.cb, gb + P[k].i);
+          }
+      }
+    }
+    if (NL || L) {
+#pragma unroll
+      for (int k = 0; k < NP; ++k)
+        if (P[k].valid) fold_alarm(p.cb, P[k].alarm, (uint32_t)(gb + P[k].i));
+    }
+    __syncthreads();  // flag reused
+  };
+  while (cur.x >= 0) {
+    if (cur.x != vrow) {
+      if (vrow >= 0) end_visit();
+      vrow = cur.x;
+      tp_row_geom(p, vrow, &h, &blk, &c0, &nch);
+      i0 = blk * NP * TP_THREADS;
+      gb = (int64_t)h * p.n;
+      jlo = h <= p.nr ? i0 + 1 : 0;
+      jall = h <= p.nr ? min(i0 + NP * TP_THREADS, p.n) : 0;
+      visited = 0;
+      tp_hist_switch<NP>(p, S, st, h, nch * HK_TP_SR_CHUNK);
+      tp_points<NP>(p, p.hist, h, blk, p.g0, p.g1, P, NL);
+#pragma unroll
+      for (int k = 0; k < NP; ++k) inc[k] = P[k].valid ? ((k & 1) ? 0x10000u : 1u) : 0u;
+    }
+    // speculative claim of the chunk after nxt (its result is used after the computation)
+    int spec = -1, snch = 0;
+    if (threadIdx.x == 0 && nxt.x >= 0) {
+      int sh, sblk, sc0;
+      tp_row_geom(p, nxt.x, &sh, &sblk, &sc0, &snch);
+      spec = atomicAdd(q.row_next + nxt.x, 1);
+    }
+    if (nxt.x >= 0) cp_async_wait<1>();
+    else cp_async_wait<0>();
+    __syncthreads();  // cur's tile is staged
+    {
+      const int j0 = max(jlo, (c0 + cur.y) * HK_TP_SR_CHUNK), j1 = min(p.n, (c0 + cur.y + 1) * HK_TP_SR_CHUNK);
+      const int jt0 = j0 & ~3;
+      tp_tile_pairs<NP, CNT, LUT>(p, c, S.B + slot * 3 * TP_TILE, Hw, P, inc, jt0, j0 - jt0, j1 - jt0, jall, i0);
+    }
+    ++visited;
+    if (threadIdx.x < 32) {
+      int2 nn = make_int2(-1, 0);
+      if (nxt.x >= 0) {
+        const int sp = __shfl_sync(0xffffffffu, spec, 0), sn = __shfl_sync(0xffffffffu, snch, 0);
+        nn = sp < sn ? make_int2(nxt.x, sp) : tp_sr_claim(p, q, nxt.x);
+      }
+      if (threadIdx.x == 0) claim[0] = nn;
+    }
+    __syncthreads();  // the computation is done (slot free) and the next claim visible
+    const int2 nn = claim[0];
+    tp_sr_stage(p, S, nn, slot);
+    cur = nxt;
+    nxt = nn;
+    slot ^= 1;
+  }
+  if (vrow >= 0) end_visit();
+}
+
+// FI & FT (or FI-only) replicas (blockIdx.y = launch slot)
+// ============================================================================================
+enum TPKind : int { TK_NL = 0, TK_LIVE, TK_J, TK_X2, TK_Y2, TK_Z2, TK_DOT, TK_BIN, TK_HIDX, TK_ACC, TK_CNT, TK_COUNT };
+
+struct TPFIParams {
+  TPParams base;
+  const FaultRec* faults;
+  unsigned long long* hist0;  // replica r: hist0 + r * hist_elems
+  hk_control* cb0;
+  int64_t hist_elems;
+};
+
+// Histogram sinks of the per-thread TPACF FI program.  Replica: every increment of the faulted
+// thread goes to the replica's global histogram through its (possibly corrupted) index.  Replay:
+// every increment is folded into deltas of the 3*nb outputs (DD, DRS, RRS of R4) with a sign
+// (+1 faulted run, -1 golden twin).
+struct TPReplicaSink {
+  hk_control* cb;
+  __device__ __forceinline__ void hist_p(unsigned long long* ptr, const unsigned long long*) { red_add(ptr, 1ull); }
+  __device__ __forceinline__ void outlier(int d, float v) { record_outlier(cb, d, v); }
+  __device__ __forceinline__ void finish(bool mine, uint32_t alarm, uint32_t fail, uint32_t margin, float gap,
+                                         bool applied, uint32_t tid) {
+    if (fail) atomicOr(&cb->fail, fail);
+    if (mine) {
+      cb->fault_applied = applied ? 1u : 0u;
+      cb->check_margin = margin;
+      cb->check_gap = gap;
+    }
+    if (alarm) {  // one thread: no warp vote (the rest of its warp has left)
+      atomicOr(&cb->alarm, alarm);
+      atomicAdd(&cb->n_alarm_warps, 1u);
+      atomicMin(&cb->first_thread, tid);
+    }
+  }
+};
+constexpr int TP_REPLAY_OUT = 96;  // 3 * n_bins (n_bins <= 30 for the replay kernel) + slack
+struct TPReplaySink {
+  int nr, nb, nb2, sign;
+  int32_t* delta;  // [3 * nb]: DD, DRS, RRS for bins 1..nb
+  uint32_t alarm = 0, fail = 0, margin = 0xffffffffu;
+  float gap = __builtin_huge_valf();
+  __device__ __forceinline__ void hist_p(unsigned long long* ptr, const unsigned long long* base) {
+    const int64_t e = ptr - base;
+    const int row = (int)(e / nb2), b = (int)(e % nb2);
+    if (b < 1 || b > nb) return;  // under/overflow bins are not outputs (R4)
+    const int kind = row == 0 ? 0 : (row <= nr ? 2 : 1);
+    delta[kind * nb + b - 1] += sign;
+  }
+  __device__ __forceinline__ void outlier(int, float) {}
+  __device__ __forceinline__ void finish(bool, uint32_t a, uint32_t f, uint32_t m, float g, bool, uint32_t) {
+    alarm = a; fail = f; margin = m; gap = g;
+  }
+};
+
+// Per-thread FI program of abstract thread g = h*N + ii (DESIGN §3.4 with the single hook of kind
+// KIND, R16 guards and the R17 watchdog).  FT = false: the FI-only binary (row a7) — the same
+// program with every HAUBERK statement compiled out.  i_dup / h_dup: N0 / N1's duplicates.
+// hist_real: the histogram's true base.  REAL: the guardian's unguarded variant (R25).
+template <int KIND, bool FT, bool REAL = false, class Sink>
+__device__ void tpacf_fi_program(const TPParams& p, const float* Es, const FaultRec& f, int32_t hh, int32_t ii,
+                                 int32_t i_dup, int32_t h_dup, bool mine, uint64_t hist_real, Sink& K) {
+  const uint32_t z = p.z;
+  const int32_t nr = p.nr, nb2 = p.nb + 2;
+  const int64_t g = (int64_t)hh * p.n + ii;
+  const int64_t inst = mine ? f.inst : -1;
+  const uint64_t mask = f.mask;
+  const int site = f.site;
+  const int64_t npts = 3LL * (1 + nr) * p.n, nhist = (int64_t)(1 + 2 * nr) * nb2;
+  const uint64_t pts_real = (uint64_t)(uintptr_t)p.pts;
+  uint32_t chk = 0, alarm = 0, fail = 0, margin = 0xffffffffu;
+  float gap = __int_as_float(0x7f800000);
+  bool applied = false;
+  int32_t n = p.n;
+  uint64_t ppts = pts_real, phist = hist_real;
+  if (FT) chk ^= (uint32_t)n ^ lohi(ppts) ^ lohi(phist);
+  const bool nl = (KIND == TK_NL) && mine;
+#define NLF(v, s) do { const bool _n = nl && site == (s); applied |= _n; v = flip_i(v, _n, mask); } while (0)
+  int32_t i = ii; NLF(i, 0);
+  if (FT) { chk ^= (uint32_t)i; alarm |= (i_dup != i) ? AL_DUP : 0u; }
+  int32_t h = hh; NLF(h, 1);
+  if (FT) { chk ^= (uint32_t)h; alarm |= (h_dup != h) ? AL_DUP : 0u; }
+  auto f_aoff = [&](int32_t hq, int32_t iq) { return (int32_t)((uint32_t)(hq <= nr ? hq : 0) * (uint32_t)n + (uint32_t)iq); };
+  auto f_boff = [&](int32_t hq) { return (int32_t)((uint32_t)(hq == 0 ? 0 : (hq <= nr ? hq : (int32_t)((uint32_t)hq - (uint32_t)nr))) * (uint32_t)n); };
+  auto f_jb = [&](int32_t hq, int32_t iq) { return hq <= nr ? (int32_t)((uint32_t)iq + 1u) : 0; };
+  auto f_ex = [&](int32_t je_, int32_t jb_) { const int32_t d = (int32_t)((uint32_t)je_ - (uint32_t)jb_); return d > 0 ? d : 0; };
+  int32_t aoff = f_aoff(h, i); NLF(aoff, 2);
+  if (FT) { chk ^= (uint32_t)aoff; alarm |= (f_aoff(opq(h, z), opq(i, z)) != aoff) ? AL_DUP : 0u; }
+  int32_t boff = f_boff(h); NLF(boff, 3);
+  if (FT) { chk ^= (uint32_t)boff; alarm |= (f_boff(opq(h, z)) != boff) ? AL_DUP : 0u; }
+  int32_t jb = f_jb(h, i); NLF(jb, 4);
+  if (FT) { chk ^= (uint32_t)jb; alarm |= (f_jb(opq(h, z), opq(i, z)) != jb) ? AL_DUP : 0u; }
+  int32_t je = n; NLF(je, 5);
+  if (FT) { chk ^= (uint32_t)je; alarm |= (opq(n, z) != je) ? AL_DUP : 0u; }
+  int32_t expect = f_ex(je, jb); NLF(expect, 6);
+  if (FT) { chk ^= (uint32_t)expect; alarm |= (f_ex(opq(je, z), jb) != expect) ? AL_DUP : 0u; }
+  int32_t base = (int32_t)((uint32_t)h * (uint32_t)nb2); NLF(base, 7);
+  if (FT) { chk ^= (uint32_t)base; alarm |= ((int32_t)((uint32_t)opq(h, z) * (uint32_t)nb2) != base) ? AL_DUP : 0u; }
+#undef NLF
+  float q1[3];
+  int32_t acc = 0, cnt = 0, j;
+  const float* pe;
+  const int64_t golden = hh <= nr ? (int64_t)p.n - (ii + 1) : (int64_t)p.n;  // uncorrupted launch indices (R17)
+  const int64_t limit = fi_limit<REAL>(golden, f.hang);
+  constexpr bool real = REAL;
+  for (int a = 0; a < 3; ++a) {
+    if (!fi_at(real, ppts, pts_real, (int32_t)((uint32_t)aoff * 3u + (uint32_t)a), npts, &pe)) { fail |= FL_CRASH; goto done; }
+    float v = __ldg(pe);
+    { const bool nn = nl && site == 8 + a; applied |= nn; v = flip_f(v, nn, mask); }
+    if (FT) { chk ^= fb(v); alarm |= (fb(__ldg(pe + z)) != fb(v)) ? AL_DUP : 0u; }
+    q1[a] = v;
+  }
+  if (FT) chk ^= (uint32_t)opq(i, z) ^ (uint32_t)opq(h, z) ^ (uint32_t)opq(aoff, z) ^ (uint32_t)opq(jb, z);
+  j = jb;
+  for (int64_t it = 0;; ++it) {
+    const bool now = (it == inst);
+    if (KIND == TK_J) { applied |= now; j = flip_i(j, now, mask); }
+    if (KIND == TK_LIVE && now) {
+      applied = true;
+      switch (site) {
+        case 11: boff = flip_i(boff, true, mask); break;
+        case 12: je = flip_i(je, true, mask); break;
+        case 13: expect = flip_i(expect, true, mask); break;
+        case 14: base = flip_i(base, true, mask); break;
+        case 15: q1[0] = flip_f(q1[0], true, mask); break;
+        case 16: q1[1] = flip_f(q1[1], true, mask); break;
+        case 17: q1[2] = flip_f(q1[2], true, mask); break;
+        case 18: n = flip_i(n, true, mask); break;
+        case 19: ppts = flip_p(ppts, true, mask); break;
+        case 20: phist = flip_p(phist, true, mask); break;
+        default: break;
+      }
+    }
+    if (!(j < je)) break;
+    if (it >= limit) { fail |= FL_HANG; goto done; }
+    {
+      const int32_t pb = (int32_t)(3u * (uint32_t)((uint32_t)boff + (uint32_t)j));
+      float q2[3];
+#pragma unroll
+      for (int a = 0; a < 3; ++a) {
+        if (!fi_at(real, ppts, pts_real, (int32_t)((uint32_t)pb + (uint32_t)a), npts, &pe)) { fail |= FL_CRASH; goto done; }
+        q2[a] = __ldg(pe);
+      }
+      if (KIND == TK_X2) { applied |= now; q2[0] = flip_f(q2[0], now, mask); }
+      if (KIND == TK_Y2) { applied |= now; q2[1] = flip_f(q2[1], now, mask); }
+      if (KIND == TK_Z2) { applied |= now; q2[2] = flip_f(q2[2], now, mask); }
+      float dot = __fmaf_rn(q1[2], q2[2], __fmaf_rn(q1[1], q2[1], __fmul_rn(q1[0], q2[0])));
+      if (KIND == TK_DOT) { applied |= now; dot = flip_f(dot, now, mask); }
+      int32_t bin = tp_bin_search(Es, dot);
+      if (KIND == TK_BIN) { applied |= now; bin = flip_i(bin, now, mask); }
+      int32_t hidx = (int32_t)((uint32_t)base + (uint32_t)bin);
+      if (KIND == TK_HIDX) { applied |= now; hidx = flip_i(hidx, now, mask); }
+      unsigned long long* ph;
+      if (!fi_at(real, phist, hist_real, hidx, nhist, &ph)) { fail |= FL_CRASH; goto done; }
+      K.hist_p(ph, reinterpret_cast<const unsigned long long*>(hist_real));
+      acc = (int32_t)((uint32_t)acc + (uint32_t)bin);
+      if (KIND == TK_ACC) { applied |= now; acc = flip_i(acc, now, mask); }
+    }
+    cnt = count_inc(cnt, p.one);
+    if (KIND == TK_CNT) { applied |= now; cnt = flip_i(cnt, now, mask); }
+    j = (int32_t)((uint32_t)j + 1u);
+  }
+  if (FT) {
+    if (cnt != expect) alarm |= AL_COUNT;
+    if (cnt != 0 && p.ndet > 0 && p.R.n[0] > 0) {
+      const float v = __fdiv_rn((float)acc, (float)cnt);
+      if (!in_range<true>(p.R, 0, v, &margin, &gap)) { alarm |= AL_RANGE; K.outlier(0, v); }
+    }
+    chk ^= (uint32_t)opq(boff, z) ^ (uint32_t)opq(je, z) ^ (uint32_t)opq(base, z);
+    chk ^= opqf(q1[0], z) ^ opqf(q1[1], z) ^ opqf(q1[2], z) ^ (uint32_t)opq(expect, z);
+    chk ^= ((uint32_t)n + z) ^ (lohi(ppts) + z) ^ (lohi(phist) + z);
+    if (chk != 0) alarm |= AL_CHK;
+  }
+done:
+  K.finish(mine, alarm, fail, margin, gap, applied, (uint32_t)g);
+}
+
+// The same per-thread FI program, evaluated by the 32 lanes of one warp: lane l evaluates loop
+// iteration it0 + l of the ONE faulted abstract thread.  The program's state at iteration `it` is
+// a closed form of it (j = jb + it, the live values constant) except for the single flip at
+// iteration f.inst, which changes the live state from then on (kinds J / LIVE) or one iteration's
+// temporaries (X2 .. HIDX) or the running sums (ACC, CNT); so every lane can compute its own
+// iteration directly.  The first iteration E (ballot) holding an event — loop exit, R17 watchdog,
+// R16 crash, in the sequential order of the checks — ends the program exactly where the sequential
+// loop would: iterations before E add their histogram increment and their bin; acc and cnt are
+// rebuilt from the per-lane sums with the flip applied at its instance.  Results are identical to
+// tpacf_fi_program (the replay kernel runs that one; GPU replay == replica is tested) at ~1/32 of
+// its latency-bound time — a corrupted loop may run 10x the golden trips before the watchdog.
+template <int KIND, bool FT, bool LUT>
+__device__ void tpacf_fi_warp(const TPParams& p, const TPSmem& S, const FaultRec& f, int32_t hh, int32_t ii, int32_t i_dup,
+                              int32_t h_dup, uint64_t hist_real, hk_control* cb) {
+  const unsigned FULL = 0xffffffffu;
+  const uint32_t lane = lane_id();
+  const uint32_t z = p.z;
+  const int32_t nr = p.nr, nb2 = p.nb + 2;
+  const int64_t g = (int64_t)hh * p.n + ii;
+  const int64_t inst = f.inst;
+  const uint64_t mask = f.mask;
+  const int site = f.site;
+  const int64_t npts = 3LL * (1 + nr) * p.n, nhist = (int64_t)(1 + 2 * nr) * nb2;
+  const uint64_t pts_real = (uint64_t)(uintptr_t)p.pts;
+  uint32_t chk = 0, alarm = 0, fail = 0, margin = 0xffffffffu;
+  float gap = __int_as_float(0x7f800000);
+  bool applied = false;
+  int32_t n = p.n;
+  uint64_t ppts = pts_real, phist = hist_real;
+  // ---- prologue (uniform over the warp; DESIGN §3.4 NL sites 0-10)
+  if (FT) chk ^= (uint32_t)n ^ lohi(ppts) ^ lohi(phist);
+  const bool nl = (KIND == TK_NL);
+#define NLF(v, s) do { const bool _n = nl && site == (s); applied |= _n; v = flip_i(v, _n, mask); } while (0)
+  int32_t i = ii; NLF(i, 0);
+  if (FT) { chk ^= (uint32_t)i; alarm |= (i_dup != i) ? AL_DUP : 0u; }
+  int32_t h = hh; NLF(h, 1);
+  if (FT) { chk ^= (uint32_t)h; alarm |= (h_dup != h) ? AL_DUP : 0u; }
+  auto f_aoff = [&](int32_t hq, int32_t iq) { return (int32_t)((uint32_t)(hq <= nr ? hq : 0) * (uint32_t)n + (uint32_t)iq); };
+  auto f_boff = [&](int32_t hq) { return (int32_t)((uint32_t)(hq == 0 ? 0 : (hq <= nr ? hq : (int32_t)((uint32_t)hq - (uint32_t)nr))) * (uint32_t)n); };
+  auto f_jb = [&](int32_t hq, int32_t iq) { return hq <= nr ? (int32_t)((uint32_t)iq + 1u) : 0; };
+  auto f_ex = [&](int32_t je_, int32_t jb_) { const int32_t d = (int32_t)((uint32_t)je_ - (uint32_t)jb_); return d > 0 ? d : 0; };
+  int32_t aoff = f_aoff(h, i); NLF(aoff, 2);
+  if (FT) { chk ^= (uint32_t)aoff; alarm |= (f_aoff(opq(h, z), opq(i, z)) != aoff) ? AL_DUP : 0u; }
+  int32_t boff = f_boff(h); NLF(boff, 3);
+  if (FT) { chk ^= (uint32_t)boff; alarm |= (f_boff(opq(h, z)) != boff) ? AL_DUP : 0u; }
+  int32_t jb = f_jb(h, i); NLF(jb, 4);
+  if (FT) { chk ^= (uint32_t)jb; alarm |= (f_jb(opq(h, z), opq(i, z)) != jb) ? AL_DUP : 0u; }
+  int32_t je = n; NLF(je, 5);
+  if (FT) { chk ^= (uint32_t)je; alarm |= (opq(n, z) != je) ? AL_DUP : 0u; }
+  int32_t expect = f_ex(je, jb); NLF(expect, 6);
+  if (FT) { chk ^= (uint32_t)expect; alarm |= (f_ex(opq(je, z), jb) != expect) ? AL_DUP : 0u; }
+  int32_t base = (int32_t)((uint32_t)h * (uint32_t)nb2); NLF(base, 7);
+  if (FT) { chk ^= (uint32_t)base; alarm |= ((int32_t)((uint32_t)opq(h, z) * (uint32_t)nb2) != base) ? AL_DUP : 0u; }
+#undef NLF
+  float q1[3] = {0.f, 0.f, 0.f};
+  for (int a = 0; a < 3; ++a) {
+    const float* pe;
+    if (!fi_at(false, ppts, pts_real, (int32_t)((uint32_t)aoff * 3u + (uint32_t)a), npts, &pe)) { fail |= FL_CRASH; break; }
+    float v = __ldg(pe);
+    { const bool nn = nl && site == 8 + a; applied |= nn; v = flip_f(v, nn, mask); }
+    if (FT) { chk ^= fb(v); alarm |= (fb(__ldg(pe + z)) != fb(v)) ? AL_DUP : 0u; }
+    q1[a] = v;
+  }
+  if (!fail) {
+    if (FT) chk ^= (uint32_t)opq(i, z) ^ (uint32_t)opq(h, z) ^ (uint32_t)opq(aoff, z) ^ (uint32_t)opq(jb, z);
+    // ---- the live state after the flip (kinds J / LIVE), in force from iteration inst on
+    int32_t boff2 = boff, je2 = je, expect2 = expect, base2 = base, n2 = n;
+    float q12[3] = {q1[0], q1[1], q1[2]};
+    uint64_t ppts2 = ppts, phist2 = phist;
+    if (KIND == TK_LIVE) {
+      switch (site) {
+        case 11: boff2 = flip_i(boff, true, mask); break;
+        case 12: je2 = flip_i(je, true, mask); break;
+        case 13: expect2 = flip_i(expect, true, mask); break;
+        case 14: base2 = flip_i(base, true, mask); break;
+        case 15: q12[0] = flip_f(q1[0], true, mask); break;
+        case 16: q12[1] = flip_f(q1[1], true, mask); break;
+        case 17: q12[2] = flip_f(q1[2], true, mask); break;
+        case 18: n2 = flip_i(n, true, mask); break;
+        case 19: ppts2 = flip_p(ppts, true, mask); break;
+        case 20: phist2 = flip_p(phist, true, mask); break;
+        default: break;
+      }
+    }
+    const int32_t jflip = (int32_t)((uint32_t)jb + (uint32_t)inst) ^ (int32_t)(uint32_t)mask;  // J: j at iteration inst
+    const int64_t golden = hh <= nr ? (int64_t)p.n - (ii + 1) : (int64_t)p.n;  // uncorrupted launch indices (R17)
+    const int64_t limit = fi_limit<false>(golden, f.hang);
+    int64_t E = -1;
+    int etype = 0;      // 1 exit, 2 hang, 3 crash in the partner loads, 4 crash at the histogram
+    uint32_t s_le = 0, s_gt = 0;  // this lane's bins of iterations <= inst / > inst (before E)
+    const uint32_t lb = smem_u32(S.E);
+    for (int64_t it0 = 0; E < 0; it0 += 32) {
+      const int64_t it = it0 + lane;
+      const bool post = (KIND == TK_J || KIND == TK_LIVE) && it >= inst;
+      const bool now = it == inst;
+      int32_t j = (int32_t)((uint32_t)jb + (uint32_t)it);
+      if (KIND == TK_J && post) j = (int32_t)((uint32_t)jflip + (uint32_t)(it - inst));
+      const int32_t bo = post ? boff2 : boff, jee = post ? je2 : je, ba = post ? base2 : base;
+      const uint64_t pp = post ? ppts2 : ppts, ph = post ? phist2 : phist;
+      const float x1 = post ? q12[0] : q1[0], y1 = post ? q12[1] : q1[1], z1 = post ? q12[2] : q1[2];
+      int ev = 0;
+      uint32_t bin = 0;
+      unsigned long long* hp = nullptr;
+      if (!(j < jee)) ev = 1;
+      else if (it >= limit) ev = 2;
+      else {
+        const int32_t pb = (int32_t)(3u * (uint32_t)((uint32_t)bo + (uint32_t)j));
+        float q2[3];
+        for (int a = 0; a < 3 && !ev; ++a) {
+          const float* pe;
+          if (!fi_at(false, pp, pts_real, (int32_t)((uint32_t)pb + (uint32_t)a), npts, &pe)) ev = 3;
+          else q2[a] = __ldg(pe);
+        }
+        if (!ev) {
+          if (KIND == TK_X2) q2[0] = flip_f(q2[0], now, mask);
+          if (KIND == TK_Y2) q2[1] = flip_f(q2[1], now, mask);
+          if (KIND == TK_Z2) q2[2] = flip_f(q2[2], now, mask);
+          float dot = __fmaf_rn(z1, q2[2], __fmaf_rn(y1, q2[1], __fmul_rn(x1, q2[0])));
+          if (KIND == TK_DOT) dot = flip_f(dot, now, mask);
+          bin = LUT ? tp_b4_lut(S.L, lb, dot) / 4u : (uint32_t)tp_bin_search(S.E, dot);
+          if (KIND == TK_BIN) bin = (uint32_t)flip_i((int32_t)bin, now, mask);
+          int32_t hidx = (int32_t)((uint32_t)ba + bin);
+          if (KIND == TK_HIDX) hidx = flip_i(hidx, now, mask);
+          if (!fi_at(false, ph, hist_real, hidx, nhist, &hp)) ev = 4;
+        }
+      }
+      const unsigned evs = __ballot_sync(FULL, ev != 0);
+      const int first = evs ? __ffs(evs) - 1 : 32;
+      if ((int)lane < first) {  // iterations before the first event: executed in full
+        red_add(hp, 1ull);
+        if (it <= inst) s_le += bin;
+        else s_gt += bin;
+      }
+      if (evs) {
+        E = it0 + first;
+        etype = __shfl_sync(FULL, ev, first);
+      }
+    }
+    s_le = __reduce_add_sync(FULL, s_le);
+    s_gt = __reduce_add_sync(FULL, s_gt);
+    // hooks of iteration inst that ran (the checks of iteration E precede its loads / increment)
+    if (KIND == TK_J || KIND == TK_LIVE) applied = inst <= E;
+    if (KIND == TK_X2 || KIND == TK_Y2 || KIND == TK_Z2 || KIND == TK_DOT || KIND == TK_BIN || KIND == TK_HIDX)
+      applied = inst < E || (inst == E && etype == 4);
+    if (KIND == TK_ACC || KIND == TK_CNT) applied = inst < E;
+    if (etype == 2) fail |= FL_HANG;
+    if (etype >= 3) fail |= FL_CRASH;
+    if (!fail && FT) {
+      const bool in_force = (KIND == TK_J || KIND == TK_LIVE) && inst <= E;  // the exit sees the flipped state
+      const int32_t boffx = in_force ? boff2 : boff, jex = in_force ? je2 : je, basex = in_force ? base2 : base;
+      const int32_t expx = in_force ? expect2 : expect, nx = in_force ? n2 : n;
+      const float x1x = in_force ? q12[0] : q1[0], y1x = in_force ? q12[1] : q1[1], z1x = in_force ? q12[2] : q1[2];
+      const uint64_t ppx = in_force ? ppts2 : ppts, phx = in_force ? phist2 : phist;
+      const int32_t acc = (KIND == TK_ACC && inst < E) ? (int32_t)(((s_le) ^ (uint32_t)mask) + s_gt) : (int32_t)(s_le + s_gt);
+      const int32_t cnt = (KIND == TK_CNT && inst < E) ? (int32_t)((((uint32_t)inst + 1u) ^ (uint32_t)mask) + (uint32_t)(E - 1 - inst))
+                                                        : (int32_t)E;
+      if (cnt != expx) alarm |= AL_COUNT;
+      if (cnt != 0 && p.ndet > 0 && p.R.n[0] > 0) {
+        const float v = __fdiv_rn((float)acc, (float)cnt);
+        if (!in_range<true>(p.R, 0, v, &margin, &gap)) {
+          alarm |= AL_RANGE;
+          if (lane == 0) record_outlier(cb, 0, v);
+        }
+      }
+      chk ^= (uint32_t)opq(boffx, z) ^ (uint32_t)opq(jex, z) ^ (uint32_t)opq(basex, z);
+      chk ^= opqf(x1x, z) ^ opqf(y1x, z) ^ opqf(z1x, z) ^ (uint32_t)opq(expx, z);
+      chk ^= ((uint32_t)nx + z) ^ (lohi(ppx) + z) ^ (lohi(phx) + z);
+      if (chk != 0) alarm |= AL_CHK;
+    }
+  }
+  if (!FT) alarm = 0;
+  if (lane == 0) {
+    TPReplicaSink K{cb};
+    K.finish(true, alarm, fail, margin, gap, applied, (uint32_t)g);
+  }
+}
+
+// Replica CTA (h, point block) of the FI kernel, whole partner loops, fast part.  The faulted
+// abstract thread (if this CTA holds it) takes no part in the fast loop (increment 0, no exit
+// checks); returns (point index, N0 duplicate) of it in the warp that holds it, else (-1, 0).
+template <bool FT, bool LUT>
+__device__ __forceinline__ int2 tp_replica_fast(const TPFIParams& q, const TPSmem& S, const FaultRec& f, unsigned long long* hist,
+                                                hk_control* cb, int h, int blk, bool faulted) {
+  constexpr int NP = HK_TP_NP_FI;
+  constexpr int V = FT ? (V_NL | V_L) : 0;
+  constexpr bool NL = FT, L = FT;
+  TPParams p = q.base;
+  p.hist = hist;
+  p.cb = cb;
+  const int i0 = blk * NP * TP_THREADS;
+  const int64_t gb = (int64_t)h * p.n;
+  TPPoint P[NP];
+  tp_points<NP>(p, hist, h, blk, 0, INT64_MAX, P, NL);
+  uint32_t inc[NP];
+  int fk = -1;  // which of this thread's points is the faulted abstract thread
+#pragma unroll
+  for (int k = 0; k < NP; ++k) {
+    const bool mine = faulted && P[k].valid && gb + P[k].i == f.thread;
+    if (mine) fk = k;
+    inc[k] = (P[k].valid && !mine) ? ((k & 1) ? 0x10000u : 1u) : 0u;
+  }
+  tp_zero_hist<NP>(p, S);
+  __syncthreads();
+  const int jlo = h <= p.nr ? i0 + 1 : 0;
+  tp_item_loop<NP, V, LUT>(p, S, P, inc, h, i0, jlo, p.n);
+#pragma unroll
+  for (int k = 0; k < NP; ++k) {
+    if (!P[k].valid || k == fk) continue;
+    if (L) P[k].acc /= 4;
+    tp_nl_exit<NL>(p, P[k], hist);
+    tp_checks<V>(p, P[k], cb, gb + P[k].i);
+  }
+  if (NL || L) {
+#pragma unroll
+    for (int k = 0; k < NP; ++k)
+      if (P[k].valid) fold_alarm(cb, k == fk ? 0u : P[k].alarm, (uint32_t)(gb + P[k].i));
+  }
+  __syncthreads();
+  tp_flush<NP>(p, S, hist, h * (p.nb + 2));
+  // the warp holding the faulted abstract thread learns its point index and N0 duplicate
+  const unsigned own = __ballot_sync(0xffffffffu, fk >= 0);
+  if (!own) return make_int2(-1, 0);
+  const int src = __ffs(own) - 1;
+  const int fkw = __shfl_sync(0xffffffffu, fk, src);
+  const int t = (int)(threadIdx.x & ~31u) + src;
+  return make_int2(i0 + fkw * TP_THREADS + t, (int)((blk ^ p.z) * (NP * TP_THREADS) + fkw * TP_THREADS + (t ^ (int)p.z)));
+}
+
+// Replica CTA (h, point block) of the FI kernel: the fast loop over every abstract thread but the
+// faulted one, then that one's FI program on the 32 lanes of its warp.
+template <int KIND, bool FT, bool LUT>
+__device__ __forceinline__ void tp_replica_cta(const TPFIParams& q, const TPSmem& S, const FaultRec& f, unsigned long long* hist,
+                                               hk_control* cb, int h, int blk, bool faulted) {
+  const int2 fi = tp_replica_fast<FT, LUT>(q, S, f, hist, cb, h, blk, faulted);
+  if (fi.x >= 0) {
+    TPParams p = q.base;
+    p.hist = hist;
+    p.cb = cb;
+    tpacf_fi_warp<KIND, FT, LUT>(p, S, f, h, fi.x, fi.y, (int)((uint32_t)h ^ p.z), (uint64_t)(uintptr_t)hist, cb);
+  }
+}
+
+// Launch slots: the first nrep slots run the faulted CTA of replica 0..nrep-1 (the FI program
+// makes them the longest, so they start first); the rest go CTA-major in decreasing loop length
+// (DR rows, then the self rows block by block), replica-minor; the slot of a replica's faulted
+// CTA in that order does nothing.
+__device__ __forceinline__ void tp_cta_of_rank(int rank, int nr, int nblk, int* h, int* blk) {
+  const int ndr = nr * nblk;
+  if (rank < ndr) { *h = nr + 1 + rank / nblk; *blk = rank % nblk; }
+  else { const int r2 = rank - ndr; *blk = r2 / (nr + 1); *h = r2 % (nr + 1); }
+}
+
+__host__ __device__ __forceinline__ int tpacf_site_kind_d(int site) {
+  if (site <= 10) return TK_NL;
+  if (site <= 20) return TK_LIVE;
+  return TK_J + (site - 21);
+}
+
+
+// Replica-kernel parameters (tpacf.cu); ws holds the bucket table built by tpacf_lut_build.
+TPFIParams tpacf_fi_params(const hk_tpacf_args& a, const DevRanges& R, int ndet, const FaultRec* faults, unsigned long long* hist0,
+                           hk_control* cb0, void* ws);
+
+}  // namespace hk

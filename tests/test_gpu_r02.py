@@ -356,3 +356,23 @@ def test_bench_two_gloo_ranks_equal_one_rank():
     assert j2["outcomes"] == j1["outcomes"]
     assert j2["fi_only_outcomes"] == j1["fi_only_outcomes"]
     assert j2["ranges_identical_across_ranks"] is True
+
+
+# ------------------------------------------------------------------- fused MRI-Q + TPACF replicas
+@pytest.mark.parametrize("variant,exact", [(0, 0), (0, 1), (1, 0)])
+def test_fused_replicas_equal_separate_launches(monkeypatch, variant, exact):
+    """mix.cu (the default for mixed replica campaigns) against HK_FUSED=0 (one kind-homogeneous
+    launch per benchmark): every record field equal, on config 5 with ragged batches, FI&FT and the
+    FI-only binary, FAST and EXACT; PhiMag sites take the separate path inside the same session."""
+    probs = [W.cp_config1(), W.mriq_config2(), W.tpacf_config3()]
+    devs = [_mk(b, probs[b], exact) for b in range(3)]
+    R = [hk.profile_ranges(d) for d in devs] if variant == 0 else [None, None, None]
+    out = {}
+    for fused in ("1", "0"):
+        monkeypatch.setenv("HK_FUSED", fused)
+        out[fused] = _gpu_campaign(devs, R, 0xF05ED, 5000, 2400, mode=0, variant=variant, exact=exact, batch=173)
+    (c1, r1), (c0, r0) = out["1"], out["0"]
+    for k in r1.dtype.names:
+        assert np.array_equal(r1[k], r0[k]), k
+    assert np.array_equal(c1, c0)
+    assert (r1["bench"] == 1).sum() > 700 and (r1["bench"] == 2).sum() > 700

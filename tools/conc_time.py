@@ -21,6 +21,7 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--n", type=int, default=3000)
 ap.add_argument("--steps", type=int, default=5)
 ap.add_argument("--batch", type=int, default=0)
+ap.add_argument("--timing", action="store_true", help="also print the per-class kernel device time per step")
 a = ap.parse_args()
 dev = torch.device("cuda", 0)
 devs = [hk.CPDevice.from_problem(W.cp_config1(), dev), hk.MRIQDevice.from_problem(W.mriq_config2(), dev),
@@ -34,6 +35,7 @@ with hk.CampaignSession(-1, devs, ranges, 0x4841554245524B05, batch=a.batch) as 
     torch.cuda.synchronize()
     counts.zero_()
     ts = []
+    hk.timing_enable(a.timing)
     for k in range(a.steps):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
@@ -41,6 +43,14 @@ with hk.CampaignSession(-1, devs, ranges, 0x4841554245524B05, batch=a.batch) as 
         e1.record()
         torch.cuda.synchronize()
         ts.append(e0.elapsed_time(e1))
+if a.timing:
+    for b in range(3):
+        for cls in (1, 3):
+            ms, n, w = hk.timing_read(b, cls)
+            if n:
+                print(f"  bench {b} cls {cls}: {ms / a.steps:8.2f} ms/step over {n / a.steps:.1f} launches/step "
+                      f"({ms / n:.3f} ms per launch, work {w / a.steps:.3g}/step)")
+    hk.timing_enable(False)
 med = statistics.median(ts)
 print(f"[{tag}] step {med:8.2f} ms (min {min(ts):.2f} max {max(ts):.2f}) -> {a.n / med * 1e3:9.0f} inj/s  "
       f"counts {counts.cpu().tolist()}", flush=True)

@@ -21,9 +21,17 @@ KEYS = [
     ("launch__grid_size", "grid"),
     ("sm__cycles_active.avg", "sm cycles active avg"),
     ("sm__cycles_active.max", "sm cycles active max"),
-    ("smsp__average_warp_latency_issue_stalled_mio_throttle", "stall mio_throttle"),
-    ("smsp__average_warp_latency_issue_stalled_short_scoreboard", "stall short_scoreboard"),
-    ("smsp__average_warp_latency_issue_stalled_wait", "stall wait"),
+    ("smsp__average_warps_issue_stalled_mio_throttle_per_issue_active.ratio", "stall mio_throttle"),
+    ("smsp__average_warps_issue_stalled_short_scoreboard_per_issue_active.ratio", "stall short_scoreboard"),
+    ("smsp__average_warps_issue_stalled_wait_per_issue_active.ratio", "stall wait"),
+    ("smsp__average_warps_issue_stalled_math_pipe_throttle_per_issue_active.ratio", "stall math_pipe_throttle"),
+    ("smsp__average_warps_issue_stalled_no_instruction_per_issue_active.ratio", "stall no_instruction"),
+    ("smsp__average_warps_issue_stalled_barrier_per_issue_active.ratio", "stall barrier"),
+    ("smsp__average_warps_issue_stalled_long_scoreboard_per_issue_active.ratio", "stall long_scoreboard"),
+    ("smsp__average_warps_issue_stalled_not_selected_per_issue_active.ratio", "stall not_selected"),
+    ("smsp__average_warps_issue_stalled_selected_per_issue_active.ratio", "stall selected"),
+    ("smsp__average_warps_issue_stalled_lg_throttle_per_issue_active.ratio", "stall lg_throttle"),
+    ("smsp__average_warps_issue_stalled_dispatch_stall_per_issue_active.ratio", "stall dispatch"),
     ("smsp__inst_executed.sum", "warp instructions"),
 ]
 

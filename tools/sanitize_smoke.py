@@ -7,7 +7,7 @@ import torch
 import workloads as W
 from paper_conf_ipps_yimpski11_b200 import hauberk as hk
 dev = torch.device("cuda", 0)
-probs = [W.cp_small(), W.mriq_small(), W.tpacf_small(n=300, n_rand=2, chunk=64)]
+probs = [W.cp_small(), W.mriq_small(), W.tpacf_small(n=300, n_rand=2)]
 devs = [hk.CPDevice.from_problem(probs[0], dev), hk.MRIQDevice.from_problem(probs[1], dev), hk.TPACFDevice.from_problem(probs[2], dev)]
 R = [hk.profile_ranges(d) for d in devs]
 for b, d in enumerate(devs):

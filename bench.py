@@ -412,15 +412,18 @@ def main():
         dist.barrier()
     launches = hk.launch_count() - l0
     fi_conc = {b: hk.timing_read(b, 1) for b in range(3)}
+    mix_mq, mix_tp = hk.timing_read(1, 3), hk.timing_read(2, 3)  # the fused launches (same events, each one's work)
     hk.timing_enable(False)
     clk = clocks.stop()
-    # Per-kernel roofline: the session forks one stream per benchmark, so MRI-Q and TPACF
-    # replica launches overlap inside the timed steps and their event durations are not
-    # separable.  The same steps are replayed once more with the streams joined (serial
-    # session, HK_CONCURRENT=0) to time each kernel class alone; labelled in the JSON.
+    # Separate-kernel rooflines: the timed steps run MRI-Q and TPACF replicas in fused launches
+    # (mix.cu) and CP replicas on a forked stream.  The same steps are replayed once more as a
+    # serial session with one kernel per benchmark (HK_CONCURRENT=0, HK_FUSED=0) to time each
+    # replica kernel alone; labelled in the JSON.
     os.environ["HK_CONCURRENT"] = "0"
+    os.environ["HK_FUSED"] = "0"
     ser = hk.CampaignSession(-1, devs, ranges, seed, batch=args.batch)
     os.environ.pop("HK_CONCURRENT")
+    os.environ.pop("HK_FUSED")
     ser.run(*par.step_slice(args.steps + 2000, rank, world, args.per_rank), scratch)  # warm-up
     torch.cuda.synchronize()
     ser_steps = max(1, min(args.steps, 3))
@@ -447,41 +450,65 @@ def main():
     value = total_inj / (tot_ms * 1e-3)
     c = counts.cpu().numpy()
 
-    # dominant kernel of the step: the FI replica kernel class with the largest device time
-    dom = max(range(3), key=lambda b: fi[b][0])
-    ms, nl, work = fi[dom]
-    if dom == 2:
-        ops, peak, pipe = TPACF_OPS_PER_PAIR, lane_peak, "fp32/int lanes"
-    else:
-        ops, peak, pipe = (1.0 if dom == 0 else 2.0), mufu_peak, "xu (MUFU)"
-    ach = work * ops / (ms * 1e-3) if ms > 0 else 0.0
-    roofline = {"bound": "alu", "pipe": pipe, "kernel": f"{hk.BENCH_NAMES[dom]}_fi_kernel (FI&FT replicas)",
-                "achieved": round(ach / 1e9, 2), "peak": round(peak / 1e9, 2), "unit": "Gop/s", "frac": round(ach / peak, 4),
-                "traffic": None, "launches": nl, "share_of_step": round(ms / ser_ms, 3) if ser_ms else None,
-                "measured": f"CUDA events on the launch stream over {ser_steps} serial step(s) of the same workload "
-                            f"(the timed steps overlap the benchmarks' streams; serial step {ser_ms / ser_steps:.2f} ms vs "
-                            f"concurrent {my_ms / args.steps:.2f} ms)",
-                "ops_per_pair": ops, "peak_source": f"{N_SM} SMs x {MUFU_PER_SM_CLK if dom < 2 else LANES_PER_SM_CLK}/clk/SM x {sm_mhz_peak:.0f} MHz ({clk_src})"}
-    # what actually binds the dominant kernel (ncu --set full of the same kernel, profiles/r01_ncu_fi_summary.txt)
-    roofline["limiter_ncu"] = {
-        2: "shared-memory wavefronts (profiles/r02_ncu_summary.txt): per pair one LDS.U8 + one edge LDS + one ATOMS "
-           "+ 3/16 LDS.128 (2 wavefronts each) = 3.375 wavefronts per 32 pairs; 12.4 SASS instructions per pair",
-        1: "XU (MUFU sin/cos)",
-        0: "XU (MUFU rsqrt); launch-bound at CP-s size",
-    }[dom]
-    fi_split = {hk.BENCH_NAMES[b]: {"ms": round(fi[b][0], 3), "launches": fi[b][1], "pairs": fi[b][2], "serial_steps": ser_steps}
-                for b in range(3)}
-    # traffic: DRAM bytes per launch of the same kernel/batch from the committed ncu capture
+    # Separate replica kernels (serial pass): algorithmic ops / device time against their own pipe
+    # (CP-s and MRI-Q: MUFU rsqrt / sin+cos per interaction; TPACF: TPACF_OPS_PER_PAIR lane ops per pair)
+    def sep_roofline(b):
+        ms, nl, work = fi[b]
+        ops, peak, pipe = ((TPACF_OPS_PER_PAIR, lane_peak, "fp32/int lanes") if b == 2 else
+                           ((1.0 if b == 0 else 2.0), mufu_peak, "xu (MUFU)"))
+        ach = work * ops / (ms * 1e-3) if ms > 0 else 0.0
+        return {"ms": round(ms, 3), "launches": nl, "work": work, "pipe": pipe, "achieved_gops": round(ach / 1e9, 1),
+                "peak_gops": round(peak / 1e9, 1), "frac": round(ach / peak, 4), "serial_steps": ser_steps,
+                "share_of_serial_step": round(ms / ser_ms, 3) if ser_ms else None}
+    fi_split = {hk.BENCH_NAMES[b]: sep_roofline(b) for b in range(3)}
+
+    # Dominant kernel of the timed step: the fused MRI-Q + TPACF replica launch (mix_fi_kernel).  Its
+    # two roles bind different pipes (MRI-Q: MUFU sin/cos; TPACF: the fp32/int lanes), so its
+    # roofline is the serial-equivalent fraction: the time both roles' algorithmic ops need, each at
+    # its own pipe's peak, one after the other, over the measured time (1.0 = both at peak; above
+    # 1.0 only by overlapping them).
+    ms_mix, nl_mix, w_mq = mix_mq
+    w_tp = mix_tp[2]
+    if ms_mix > 0:
+        t_mq = w_mq * 2.0 / mufu_peak
+        t_tp = w_tp * TPACF_OPS_PER_PAIR / lane_peak
+        sec = ms_mix * 1e-3
+        roofline = {"bound": "alu", "pipe": "xu (MUFU) for the MRI-Q role + fp32/int lanes for the TPACF role",
+                    "kernel": "mix_fi_kernel (fused MRI-Q + TPACF FI&FT replicas)",
+                    "achieved": round((t_mq + t_tp) / sec, 4), "peak": 1.0, "unit": "pipe-s/s (serial-equivalent)",
+                    "frac": round((t_mq + t_tp) / sec, 4),
+                    "parts": {"mriq_xu": {"achieved_gops": round(w_mq * 2.0 / sec / 1e9, 1), "peak_gops": round(mufu_peak / 1e9, 1),
+                                          "frac": round(t_mq / sec, 4), "interactions": w_mq},
+                              "tpacf_lanes": {"achieved_gops": round(w_tp * TPACF_OPS_PER_PAIR / sec / 1e9, 1),
+                                              "peak_gops": round(lane_peak / 1e9, 1), "frac": round(t_tp / sec, 4), "pairs": w_tp}},
+                    "traffic": None, "launches": nl_mix, "share_of_step": round(ms_mix / my_ms, 3) if my_ms else None,
+                    "measured": f"library CUDA events on the fused launch's stream inside the {args.steps} timed steps",
+                    "peak_source": f"{N_SM} SMs x {MUFU_PER_SM_CLK} MUFU / {LANES_PER_SM_CLK} lanes per clk/SM x "
+                                   f"{sm_mhz_peak:.0f} MHz ({clk_src})",
+                    "limiter_ncu": "instruction issue (profiles/r02_ncu_mix_summary.txt): the MRI-Q role issues 12.9 SASS "
+                                   "instructions per voxel-sample, the TPACF role ~12 per pair, ~84 % of issue slots active"}
+        tr_key = "mix_fi_kernel"
+        n_rep = [sum(1 for st in range(args.steps)
+                     for n in range(*(lambda f, c: (f, f + c))(*par.step_slice(st, rank, world, args.per_rank))) if n % 3 == b)
+                 for b in (1, 2)]
+        rpl = (n_rep[0] + n_rep[1]) / nl_mix if nl_mix else 0.0
+    else:  # HK_FUSED=0: the largest separate replica kernel
+        dom = max(range(3), key=lambda b: fi[b][0])
+        sr = fi_split[hk.BENCH_NAMES[dom]]
+        roofline = {"bound": "alu", "pipe": sr["pipe"], "kernel": f"{hk.BENCH_NAMES[dom]}_fi_kernel (FI&FT replicas)",
+                    "achieved": sr["achieved_gops"], "peak": sr["peak_gops"], "unit": "Gop/s", "frac": sr["frac"],
+                    "traffic": None, "launches": sr["launches"], "share_of_step": sr["share_of_serial_step"],
+                    "measured": f"CUDA events on the launch stream over {ser_steps} serial step(s)"}
+        tr_key = f"{hk.BENCH_NAMES[dom]}_fi_kernel"
+        n_inj = sum(1 for st in range(ser_steps)
+                    for n in range(*(lambda f, c: (f, f + c))(*par.step_slice(st, rank, world, args.per_rank))) if n % 3 == dom)
+        rpl = n_inj / sr["launches"] if sr["launches"] else 0.0
+    # traffic: DRAM bytes per launch of the same kernel from the committed ncu capture, scaled per
+    # replica to this run's mean replicas per launch
     try:
         with open(os.path.join(ROOT, "profiles", "r02_traffic.json")) as f:
-            tr = json.load(f).get(f"{hk.BENCH_NAMES[dom]}_fi_kernel")
+            tr = json.load(f).get(tr_key)
         if tr:
-            # ncu measured one launch of `replicas_per_launch` replicas; scale per replica to this
-            # run's mean replicas per launch of the dominant kernel (serial pass)
-            n_inj = sum(1 for st in range(ser_steps)
-                        for n in range(*(lambda f, c: (f, f + c))(*par.step_slice(st, rank, world, args.per_rank)))
-                        if n % 3 == dom)
-            rpl = n_inj / nl if nl else 0.0
             roofline["traffic"] = round(tr["dram_bytes_per_launch"] / tr["replicas_per_launch"] * rpl)
             roofline["traffic_source"] = (f"{tr['source']}; scaled to {rpl:.1f} replicas per launch "
                                           f"({tr['dram_bytes_per_launch'] / tr['replicas_per_launch']:.0f} B per replica)")

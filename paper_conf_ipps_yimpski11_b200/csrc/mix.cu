@@ -18,6 +18,9 @@
 #include "mriq_dev.cuh"
 #include "tpacf_dev.cuh"
 
+#ifndef HK_MIX_MQ_VPT
+#define HK_MIX_MQ_VPT 2  // voxels per CUDA thread of the MRI-Q role
+#endif
 #ifndef HK_MIX_MINB
 #define HK_MIX_MINB 5  // 5 CTAs per SM: 96 registers (6 CTAs: 80 registers, spills; measured 7 % slower)
 #endif
@@ -25,6 +28,7 @@
 namespace hk {
 
 constexpr int MIX_THREADS = 128;
+constexpr int MIX_VPT = HK_MIX_MQ_VPT;
 static_assert(MIX_THREADS == TP_THREADS, "the TPACF role needs TP_THREADS threads");
 
 struct MixParams {
@@ -33,12 +37,16 @@ struct MixParams {
   int32_t rt;      // TPACF replicas
   int32_t tcta;    // TPACF CTAs per replica
   int64_t fm, ft;  // fast slots of each role
+  // persistent variant: item counters of the two queues (zeroed before the launch) and the
+  // number of the CTAs on each SM that start on the MRI-Q queue
+  unsigned long long* queue;
+  int32_t mq_per_sm, nsm;
 };
 
 template <bool EXACT, bool FT>
 __device__ __forceinline__ void mix_mq_faulted(const MQParams& p, const FaultRec& f, int bxi) {
   switch (mriq_site_kind_d(f.site)) {
-#define K_(k) case k: mq_faulted_cta<k, EXACT, FT>(p, f, bxi); break;
+#define K_(k) case k: mq_faulted_cta<k, EXACT, FT, MIX_VPT>(p, f, bxi); break;
     K_(MK_NL) K_(MK_LIVE) K_(MK_K) K_(MK_KX) K_(MK_KY) K_(MK_KZ) K_(MK_PM) K_(MK_T1) K_(MK_T2) K_(MK_T) K_(MK_R) K_(MK_C)
     K_(MK_S) K_(MK_QR) K_(MK_QI) K_(MK_IT)
 #undef K_
@@ -50,7 +58,7 @@ template <bool EXACT, bool FT>
 __device__ __forceinline__ void mix_mq_slot(const MixParams& q, unsigned char* smem, int r, int64_t fast) {
   float4(*tile)[MQ_FI_TILE] = reinterpret_cast<float4(*)[MQ_FI_TILE]>(smem);
   uint64_t* bar = reinterpret_cast<uint64_t*>(smem + 2 * MQ_FI_TILE * sizeof(float4));
-  const int64_t ncta = q.m.ncta, vpc = (int64_t)MQ_FI_VPT * MIX_THREADS;
+  const int64_t ncta = q.m.ncta, vpc = (int64_t)MIX_VPT * MIX_THREADS;
   const FaultRec f = q.m.faults[r];
   const int64_t fc = clamp_cta(f.thread / vpc, ncta);
   MQParams p = q.m.base;
@@ -61,7 +69,7 @@ __device__ __forceinline__ void mix_mq_slot(const MixParams& q, unsigned char* s
     mix_mq_faulted<EXACT, FT>(p, f, (int)fc);
   } else {
     const int bxi = (int)(fast < fc ? fast : fast + 1);
-    mriq_body<FT ? (V_NL | V_L) : 0, EXACT, true, MQ_FI_VPT, MQ_FI_UNROLL, MQ_FI_TILE>(p, tile, bar, bxi);
+    mriq_body<FT ? (V_NL | V_L) : 0, EXACT, true, MIX_VPT, MQ_FI_UNROLL, MQ_FI_TILE>(p, tile, bar, bxi);
   }
 }
 
@@ -129,12 +137,69 @@ __global__ void __launch_bounds__(MIX_THREADS, HK_MIX_MINB) mix_fi_kernel(const 
   }
 }
 
+// Persistent variant (HK_MIX_PERSIST=k, experiment): one wave of HK_MIX_MINB CTAs per SM; CTA c
+// starts on the MRI-Q queue if c / nsm < k (the block scheduler fills the SMs breadth first, so
+// every SM holds k MRI-Q and HK_MIX_MINB - k TPACF CTAs) and takes the other queue once its own
+// is drained.  Items in the same order as the slots above (faulted CTAs first).
+template <bool EXACT, bool FT>
+__global__ void __launch_bounds__(MIX_THREADS, HK_MIX_MINB) mix_persist_kernel(const MixParams q) {
+  __shared__ long long s_item;
+  __shared__ int s_role;
+  const long long nq[2] = {(long long)q.m.nrep + q.fm, (long long)q.rt + q.ft};
+  int role = (int)(blockIdx.x / q.nsm) < q.mq_per_sm ? 0 : 1;
+  for (;;) {
+    __syncthreads();  // the previous item is done with shared memory
+    if (threadIdx.x == 0) {
+      long long it = -1;
+      for (int tries = 0; tries < 2 && it < 0; ++tries) {
+        const long long v = (long long)atomicAdd(q.queue + role, 1ull);
+        if (v < nq[role]) it = v;
+        else role ^= 1;
+      }
+      s_item = it;
+      s_role = role;
+      if (it >= 0 && role == 0) fence_proxy_async();  // earlier generic writes before the bulk copies
+    }
+    __syncthreads();
+    const long long it = s_item;
+    role = s_role;
+    if (it < 0) return;
+    if (role == 0) {
+      const int rm = q.m.nrep;
+      if (it < rm) {
+        mix_mq_slot<EXACT, FT>(q, hk_tp_dsmem, (int)it, -1);
+      } else {
+        const long long k = it - rm, per = q.m.ncta - 1;
+        mix_mq_slot<EXACT, FT>(q, hk_tp_dsmem, (int)(k / per), k % per);
+        __syncthreads();
+        if (threadIdx.x == 0) {  // the k-space barriers are re-initialised by the next MRI-Q item
+          uint64_t* bar = reinterpret_cast<uint64_t*>(hk_tp_dsmem + 2 * MQ_FI_TILE * sizeof(float4));
+          asm volatile("mbarrier.inval.shared::cta.b64 [%0];" ::"r"(smem_u32(&bar[0])) : "memory");
+          asm volatile("mbarrier.inval.shared::cta.b64 [%0];" ::"r"(smem_u32(&bar[1])) : "memory");
+        }
+      }
+    } else {
+      const int rt = q.rt;
+      if (it < rt) mix_tp_slot<FT>(q, hk_tp_dsmem, (int)it, -1);
+      else mix_tp_slot<FT>(q, hk_tp_dsmem, (int)((it - rt) % rt), (int)((it - rt) / rt));
+    }
+  }
+}
+
 size_t mix_smem_bytes(const hk_tpacf_args& t) {
   return std::max(tp_smem_bytes(t.n_bins + 2, HK_TP_NP_FI), 2 * MQ_FI_TILE * sizeof(float4) + 16);
 }
 
 template <bool EXACT, bool FT>
 static cudaError_t launch_mix(const MixParams& q, size_t smem, int64_t grid, cudaStream_t s) {
+  if (q.queue) {
+    cudaError_t e = cudaFuncSetAttribute(mix_persist_kernel<EXACT, FT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    if ((e = cudaMemsetAsync(q.queue, 0, 2 * sizeof(unsigned long long), s)) != cudaSuccess) return e;
+    mix_persist_kernel<EXACT, FT><<<(unsigned)(q.nsm * HK_MIX_MINB), MIX_THREADS, smem, s>>>(q);
+    count_launch();
+    return cudaGetLastError();
+  }
   cudaError_t e = cudaFuncSetAttribute(mix_fi_kernel<EXACT, FT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   mix_fi_kernel<EXACT, FT><<<(unsigned)grid, MIX_THREADS, smem, s>>>(q);
@@ -143,7 +208,7 @@ static cudaError_t launch_mix(const MixParams& q, size_t smem, int64_t grid, cud
 }
 
 bool mix_supported(const hk_mriq_args& m, const hk_tpacf_args& t) {
-  const int64_t vpc = (int64_t)MQ_FI_VPT * MIX_THREADS;
+  const int64_t vpc = (int64_t)MIX_VPT * MIX_THREADS;
   return (m.n_vox + vpc - 1) / vpc >= 2 && t.n > 0 && t.n_bins + 2 <= 32;
 }
 
@@ -152,13 +217,25 @@ cudaError_t mix_fi_launch(bool ft, const hk_mriq_args& ma, const DevRanges& mR, 
                           const FaultRec* tfaults, int rt, unsigned long long* thist0, hk_control* tcb0, void* tlut, cudaStream_t s) {
   if (rm <= 0 || rt <= 0 || !mix_supported(ma, ta)) return cudaErrorInvalidValue;
   MixParams q{};
-  q.m = mriq_fi_params(ma, mR, mndet, mfaults, rm, mout0, mstride, mcb0, MIX_THREADS);
+  q.m = mriq_fi_params(ma, mR, mndet, mfaults, rm, mout0, mstride, mcb0, MIX_THREADS, MIX_VPT);
   q.t = tpacf_fi_params(ta, tR, tndet, tfaults, thist0, tcb0, tlut);
   q.rt = rt;
   q.tcta = (1 + 2 * ta.n_rand) * q.t.base.nblk;
   q.fm = (int64_t)rm * (q.m.ncta - 1);
   q.ft = (int64_t)rt * q.tcta;
   const int64_t grid = rm + rt + q.fm + q.ft;
+  const char* pv = getenv("HK_MIX_PERSIST");  // read per launch (experiments, tests)
+  const int persist = pv ? atoi(pv) : 0;
+  if (persist > 0) {
+    static unsigned long long* queue = nullptr;  // experiment only: one per process
+    if (!queue && cudaMalloc((void**)&queue, 2 * sizeof(unsigned long long)) != cudaSuccess) return cudaErrorMemoryAllocation;
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    q.queue = queue;
+    q.mq_per_sm = std::min(persist, HK_MIX_MINB);
+    q.nsm = sms;
+  }
   const size_t smem = mix_smem_bytes(ta);
   // timing class 3: the same launches under both benchmarks, each with its own work
   const double n = ta.n;

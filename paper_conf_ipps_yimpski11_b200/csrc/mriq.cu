@@ -335,14 +335,14 @@ cudaError_t mriq_replay_launch(int kind, bool ft, const hk_mriq_args& a, const D
 }
 
 MQFIParams mriq_fi_params(const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep, float* out0,
-                          int64_t stride, hk_control* cb0, int threads) {
+                          int64_t stride, hk_control* cb0, int threads, int vpt) {
   MQFIParams q{};
   q.base = mq_params(a, R, ndet, nullptr, nullptr);
   q.faults = faults;
   q.out0 = out0;
   q.stride = stride;
   q.cb0 = cb0;
-  q.ncta = (a.n_vox + MQ_FI_VPT * threads - 1) / (MQ_FI_VPT * threads);
+  q.ncta = (a.n_vox + vpt * threads - 1) / (vpt * threads);
   q.nrep = nrep;
   return q;
 }

@@ -332,14 +332,14 @@ done:
 
 // The faulted CTA of a replica: every CUDA thread runs the per-voxel FI program for its MQ_FI_VPT
 // voxels (the one holding the faulted abstract thread applies the fault).
-template <int KIND, bool EXACT, bool FT>
+template <int KIND, bool EXACT, bool FT, int VPT = MQ_FI_VPT>
 __device__ __forceinline__ void mq_faulted_cta(const MQParams& p, const FaultRec& f, int bxi) {
   ReplicaSinkF S{{p.qr, p.qi}, p.cb};
 #pragma unroll 1
-  for (int vox = 0; vox < MQ_FI_VPT; ++vox) {
-    const int32_t t = bxi * (MQ_FI_VPT * blockDim.x) + vox * blockDim.x + threadIdx.x;
+  for (int vox = 0; vox < VPT; ++vox) {
+    const int32_t t = bxi * (VPT * blockDim.x) + vox * blockDim.x + threadIdx.x;
     if (t < p.numX) {
-      const int32_t t_dup = (int32_t)((bxi ^ p.zz) * (MQ_FI_VPT * blockDim.x) + vox * blockDim.x + (threadIdx.x ^ p.zz));
+      const int32_t t_dup = (int32_t)((bxi ^ p.zz) * (VPT * blockDim.x) + vox * blockDim.x + (threadIdx.x ^ p.zz));
       mriq_fi_program<KIND, EXACT, false, FT>(p, f, t, t_dup, t == f.thread, (uint64_t)(uintptr_t)p.qr, (uint64_t)(uintptr_t)p.qi, S);
     }
   }
@@ -347,6 +347,6 @@ __device__ __forceinline__ void mq_faulted_cta(const MQParams& p, const FaultRec
 
 // Replica-kernel parameters (mriq.cu; `threads` = CTA size of the kernel that will use them).
 MQFIParams mriq_fi_params(const hk_mriq_args& a, const DevRanges& R, int ndet, const FaultRec* faults, int nrep, float* out0,
-                          int64_t stride, hk_control* cb0, int threads);
+                          int64_t stride, hk_control* cb0, int threads, int vpt = MQ_FI_VPT);
 
 }  // namespace hk

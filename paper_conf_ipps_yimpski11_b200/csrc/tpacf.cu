@@ -8,9 +8,10 @@
 // after the whole loop.  How the kernels tile that loop is not part of the program:
 //  * acc, cnt and the histogram are integer sums, so any split of a thread's partner range into
 //    pieces, added exactly, gives the same values as the one sequential loop;
-//  * the single run (tpacf_kernel) cuts the partner range into chunks of 256 partners, adds the
-//    per-chunk (acc, cnt) partials with global atomics, and the last chunk item of a point block
-//    (a per-(h, block) completion counter) runs CheckEqual / CheckRange for its points;
+//  * the single run (tpacf_kernel) cuts each point block's partner range into pieces of equal
+//    pair counts that fill one wave of CTAs, adds the per-piece (acc, cnt) partials with global
+//    atomics, and the last piece of a point block (a per-(h, block) completion counter) runs
+//    CheckEqual / CheckRange for its points;
 //  * the campaign replicas (tpacf_fi_kernel) give each CTA whole loops (all partners of its
 //    points, streamed through a two-stage shared-memory ring), and the faulted abstract thread runs
 //    its sequential per-thread FI program after the CTA's fast loop.
@@ -64,18 +65,44 @@ __global__ void tpacf_lut_kernel(const float* __restrict__ edges, int nb, uint8_
   lut[q] = (uint8_t)(4 * bmin);  // byte offset of E[bmin] (E padded with -inf beyond nb)
   if (!good) atomicExch(ok, 0);
 }
+#ifdef HK_TP_SR_TRACE
+__device__ unsigned long long g_tp_trace[4096][4];  // debug builds: (smid, start ns, end ns, piece)
+extern "C" __attribute__((visibility("default"))) int hk_debug_trace(void* out) {
+  return (int)cudaMemcpyFromSymbol(out, g_tp_trace, sizeof(g_tp_trace));
+}
+#endif
 template <int V>
 __global__ void __launch_bounds__(TP_THREADS, HK_TP_MINB_SR) tpacf_kernel(const TPParams p, const TPSR q) {
-  __shared__ TPHistState st;
-  __shared__ int2 claim[2];
+#ifdef HK_TP_SR_TRACE
+  unsigned long long t0;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+#endif
+  __shared__ int3 s_pc;
   const TPSmem S = tp_carve(hk_tp_dsmem, p.nb + 2, HK_TP_NP_SR);
   tp_stage_tables(p, S);
-  if (threadIdx.x == 0) { st.h = -1; st.since = 0; }
+  if (threadIdx.x < 32) {
+    const int3 pc = tp_sr_locate(p, q, (int)blockIdx.x);
+    if (threadIdx.x == 0) s_pc = pc;
+  }
   cp_async_wait<0>();
   __syncthreads();
-  if (*p.lut_ok) tp_sr_run<V, true>(p, S, q, &st, claim);
-  else tp_sr_run<V, false>(p, S, q, &st, claim);
-  if (st.h >= 0) tp_flush<HK_TP_NP_SR>(p, S, p.hist, st.h * (p.nb + 2));
+  const int3 pc = s_pc;
+  if (pc.x < 0) return;
+  if (*p.lut_ok) tp_sr_piece<V, true>(p, S, q, pc);
+  else tp_sr_piece<V, false>(p, S, q, pc);
+#ifdef HK_TP_SR_TRACE
+  __syncthreads();
+  if (threadIdx.x == 0 && blockIdx.x < 4096) {
+    unsigned long long t1;
+    uint32_t sm;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t1));
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
+    g_tp_trace[blockIdx.x][0] = sm;
+    g_tp_trace[blockIdx.x][1] = t0;
+    g_tp_trace[blockIdx.x][2] = t1;
+    g_tp_trace[blockIdx.x][3] = ((unsigned long long)pc.x << 32) | ((unsigned)pc.y << 16) | (unsigned)pc.z;
+  }
+#endif
 }
 
 // ============================================================================================
@@ -228,13 +255,14 @@ static TPParams tp_params(const hk_tpacf_args& a, const DevRanges& R, int ndet, 
   return p;
 }
 
-// Workspace (tpacf_ws_bytes): table [TP_LUT] u8 | ok flag (16 B) | row_next [nrows] | row_done [nrows] |
+// Workspace (tpacf_ws_bytes): table [TP_LUT] u8 | ok flag (16 B) | row_done [nrows] (padded to 16 B) |
 // accg [nh * N] | cntg [nh * N]  (nrows = nh * blocks of 128 * HK_TP_NP_SR points)
 static size_t tp_ws_head() { return (size_t)TP_LUT + 16; }
 static int tp_nrows(const hk_tpacf_args& a) { return (1 + 2 * a.n_rand) * tp_nblk(a.n, HK_TP_NP_SR); }
+static size_t tp_rows_bytes(const hk_tpacf_args& a) { return ((size_t)tp_nrows(a) * sizeof(int) + 15) / 16 * 16; }
 size_t tpacf_ws_bytes(const hk_tpacf_args& a) {
   const size_t nt = (size_t)(1 + 2 * a.n_rand) * (size_t)a.n;
-  return tp_ws_head() + 2 * sizeof(int) * (size_t)tp_nrows(a) + nt * 8;
+  return tp_ws_head() + tp_rows_bytes(a) + nt * 8;
 }
 
 cudaError_t tpacf_lut_build(const hk_tpacf_args& a, void* ws, cudaStream_t s) {
@@ -252,11 +280,12 @@ static double tp_pairs(const hk_tpacf_args& a) {
 }
 
 // hauberk_release_caches: the TPACF kernels keep no per-shape device state between calls (the
-// single run balances itself by chunk stealing), so there is nothing to free.
+// single run's pieces are recomputed per call), so there is nothing to free.
 void tpacf_release_caches() {}
 
 template <int V>
 static cudaError_t launch_tp_v(const hk_tpacf_args& a, TPParams p, void* ws, cudaStream_t s) {
+  constexpr bool CNT = (V & (V_L | V_PROF)) != 0;
   const size_t smem = tp_smem_bytes(p.nb + 2, HK_TP_NP_SR);
   cudaError_t e = cudaFuncSetAttribute(tpacf_kernel<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
@@ -268,15 +297,33 @@ static cudaError_t launch_tp_v(const hk_tpacf_args& a, TPParams p, void* ws, cud
   char* w = reinterpret_cast<char*>(ws);
   TPSR q;
   q.nrows = tp_nrows(a);
-  q.row_next = reinterpret_cast<int*>(w + tp_ws_head());
-  q.row_done = q.row_next + q.nrows;
+  q.row_done = reinterpret_cast<int*>(w + tp_ws_head());
   const size_t nt = (size_t)(1 + 2 * p.nr) * (size_t)p.n;
-  p.accg = reinterpret_cast<int32_t*>(q.row_done + q.nrows);
+  p.accg = reinterpret_cast<int32_t*>(w + tp_ws_head() + tp_rows_bytes(a));
   p.cntg = p.accg + nt;
-  if ((e = cudaMemsetAsync(w + tp_ws_head(), 0, tpacf_ws_bytes(a) - tp_ws_head(), s)) != cudaSuccess) return e;
-  const int grid = nsm * std::max(1, per_sm);  // one wave
+  // pieces: one wave of nsm * per_sm CTAs holding equal pair-slot counts
+  int64_t total = 0;
+  for (int r = 0; r < q.nrows; ++r) {
+    int h, blk, jlo;
+    total += tp_sr_row(p.n, p.nr, p.nblk, p.g0, p.g1, r, &h, &blk, &jlo);
+  }
+  if (total <= 0) return cudaSuccess;
+  {  // HK_TP_SR_SLOTS: pieces per wave-slot x 100 (experiments; default 100 = one wave)
+    const char* v = getenv("HK_TP_SR_SLOTS");
+    const int pct = v && atoi(v) > 0 ? atoi(v) : 100;
+    q.slots = std::max(1, (int)((int64_t)nsm * std::max(1, per_sm) * pct / 100));
+  }
+  q.total = total;
+  int64_t grid = 0, wcum = 0;
+  for (int r = 0; r < q.nrows; ++r) {
+    int h, blk, jlo;
+    const int64_t wr = tp_sr_row(p.n, p.nr, p.nblk, p.g0, p.g1, r, &h, &blk, &jlo);
+    grid += tp_sr_pieces(wr, wcum, p.n - jlo, q.slots, total);
+    wcum += wr;
+  }
+  if (CNT && (e = cudaMemsetAsync(w + tp_ws_head(), 0, tpacf_ws_bytes(a) - tp_ws_head(), s)) != cudaSuccess) return e;
   TimedScope ts(HK_TPACF, 0, tp_pairs(a) * (double)(p.g1 - p.g0) / (double)((1 + 2 * p.nr) * p.n), s);
-  tpacf_kernel<V><<<grid, TP_THREADS, smem, s>>>(p, q);
+  tpacf_kernel<V><<<(unsigned)grid, TP_THREADS, smem, s>>>(p, q);
   count_launch();
   return cudaGetLastError();
 }

@@ -10,16 +10,13 @@ namespace hk {
 #define HK_TP_NP_FI 4  // points per CUDA thread, campaign replicas
 #endif
 #ifndef HK_TP_NP_SR
-#define HK_TP_NP_SR 2  // points per CUDA thread, single run (256-point items: a finer LPT schedule)
+#define HK_TP_NP_SR 4  // points per CUDA thread, single run
 #endif
 #ifndef HK_TP_MINB
 #define HK_TP_MINB 6     // replicas: 37 KB of shared memory per CTA -> 6 CTAs per SM, 80 registers
 #endif
 #ifndef HK_TP_MINB_SR
-#define HK_TP_MINB_SR 8  // single run: 25.5 KB per CTA -> 8 CTAs per SM, 64 registers
-#endif
-#ifndef HK_TP_SR_CHUNK
-#define HK_TP_SR_CHUNK 128  // partners per single-run chunk (<= TP_TILE)
+#define HK_TP_MINB_SR 6  // single run: 37 KB per CTA -> 6 CTAs per SM, 80 registers
 #endif
 #ifndef HK_TP_GROUP
 #define HK_TP_GROUP 0  // partners per group of the unmasked loop (0: 4 for NP >= 4, else 8)
@@ -453,146 +450,123 @@ __device__ __forceinline__ void tp_points(const TPParams& p, const unsigned long
   }
 }
 
-// The lane-private histogram outlives a visit: consecutive visits of a CTA with the same h keep
-// counting into it and it is flushed when h changes, before the 16-bit halves could overflow
-// (< 32768 partners per slot since the last flush) and at the end.
-struct TPHistState {
-  int h;      // histogram the shared counters belong to (-1: none)
-  int since;  // partners counted per slot since the last flush (upper bound)
-};
-
-template <int NP>
-__device__ __forceinline__ void tp_hist_switch(const TPParams& p, const TPSmem& S, TPHistState* st, int h, int partners) {
-  // uniform over the CTA (st is in shared memory and read after a barrier)
-  if (st->h != h || st->since + partners >= 32768) {
-    if (st->h >= 0) {
-      tp_flush<NP>(p, S, p.hist, st->h * (p.nb + 2));
-      __syncthreads();  // flush read the counters and the ring before they are reused
-    }
-    tp_zero_hist<NP>(p, S);
-    __syncthreads();
-    if (threadIdx.x == 0) { st->h = h; st->since = 0; }
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) st->since += partners;
-}
-
 // ============================================================================================
-// Single run (BASE / FT / FT_NL / FT_L / PROFILE): one wave of CTAs that steal partner chunks.
-// A row = (histogram h, point block blk) of 128 * NP points; its partners [jlo, N) are cut into
-// chunks of HK_TP_SR_CHUNK.  CTAs start spread over the rows and claim chunks of a row with one
-// atomic each (claimed one chunk ahead, so the claim latency and the next tile's staging overlap
-// the current chunk), moving to the next row when it is exhausted: the work is balanced at chunk
-// granularity.  A CTA's stay on a row (a "visit") keeps its points' (acc, cnt) in registers;
-// leaving the row it adds them to the per-thread partial sums (exact integer combine) and its
-// chunk count to the row's; the visit that completes the row runs the loop-exit checks.
+// Single run (BASE / FT / FT_NL / FT_L / PROFILE): one wave of equal pieces.  A row = (histogram
+// h, point block blk) of 128 * NP points; its partners [jlo, N) are cut into pieces.  Row r gets
+// P(r + 1) - P(r) pieces (at least 1, and enough to keep every piece < 32768 partners, the
+// capacity of a 16-bit histogram half) with P(r) = round(S * W(r) / W), W(r) the pair slots
+// (points x partners) of the rows before r and S the CTAs one wave holds: every SM then runs the
+// same number of equal pieces.  A CTA runs one piece exactly like a replica CTA runs a whole row
+// (tp_item_loop), then adds its points' (acc, cnt) to per-thread partial sums (exact integer
+// combine); the piece that completes a row (a per-row counter) runs the loop-exit checks.
 // ============================================================================================
 struct TPSR {
-  int* row_next;  // [nrows] chunk claim counters (zeroed per run)
-  int* row_done;  // [nrows] chunks completed (zeroed per run)
+  int* row_done;   // [nrows] pieces completed (zeroed per run)
   int nrows;
+  int slots;       // S: CTAs of one wave
+  int64_t total;   // W: pair slots of the run
 };
 
-__device__ __forceinline__ void tp_row_geom(const TPParams& p, int row, int* h, int* blk, int* c0, int* nch) {
+// Row geometry: h, blk, the first partner jlo and the weight (valid points x partners) of `row`.
+__host__ __device__ __forceinline__ int64_t tp_sr_row(int n, int nr, int nblk, int64_t g0, int64_t g1, int row, int* h, int* blk,
+                                                      int* jlo) {
   constexpr int NP = HK_TP_NP_SR;
-  *h = row / p.nblk;
-  *blk = row - *h * p.nblk;
+  *h = row / nblk;
+  *blk = row - *h * nblk;
   const int i0 = *blk * NP * TP_THREADS;
-  const int64_t gb = (int64_t)*h * p.n;
-  const int i1 = min(i0 + NP * TP_THREADS, p.n);
-  const bool any = gb + i0 < p.g1 && gb + i1 > p.g0;  // some point of the block is in this run
-  const int jlo = *h <= p.nr ? i0 + 1 : 0;
-  const int nc = (p.n + HK_TP_SR_CHUNK - 1) / HK_TP_SR_CHUNK;
-  *c0 = jlo / HK_TP_SR_CHUNK;
-  *nch = (any && jlo < p.n) ? nc - *c0 : 0;
+  const int64_t gb = (int64_t)*h * n;
+  const int64_t a = gb + i0 > g0 ? gb + i0 : g0;
+  const int64_t e = gb + i0 + NP * TP_THREADS < gb + n ? gb + i0 + NP * TP_THREADS : gb + n;
+  const int64_t pts = (e < g1 ? e : g1) - a;
+  *jlo = *h <= nr ? i0 + 1 : 0;
+  return (pts > 0 && *jlo < n) ? pts * (int64_t)(n - *jlo) : 0;
+}
+// pieces of a row of weight w and `len` partners whose preceding rows weigh wcum
+__host__ __device__ __forceinline__ int tp_sr_pieces(int64_t w, int64_t wcum, int len, int slots, int64_t total) {
+  if (w <= 0) return 0;
+  const int64_t p0 = (2 * slots * wcum + total) / (2 * total), p1 = (2 * slots * (wcum + w) + total) / (2 * total);
+  const int64_t bylen = (len + 32766) / 32767;
+  const int64_t k = p1 - p0 > bylen ? p1 - p0 : bylen;
+  return (int)(k < 1 ? 1 : k);
 }
 
-// Warp 0: the next (row, chunk) starting at `row` (row = -1 once every row is exhausted).  The 32
-// lanes look at 32 rows at a time (one load of each claim counter), then lane 0 claims in the
-// first row that still had chunks; only exhausted rows are skipped, so the final sweep of a CTA
-// costs nrows / 32 load rounds instead of nrows sequential atomics.
-__device__ __forceinline__ int2 tp_sr_claim(const TPParams& p, const TPSR& q, int row) {
+// Warp 0: (row, piece within the row, pieces of the row) of piece `piece` (prefix scans over the
+// rows, 32 at a time).
+__device__ __forceinline__ int3 tp_sr_locate(const TPParams& p, const TPSR& q, int piece) {
   const unsigned FULL = 0xffffffffu;
-  const uint32_t lane = lane_id();
-  for (int scanned = 0; scanned < q.nrows; scanned += 32) {
-    int r = row + scanned + (int)lane;
-    r = r < q.nrows ? r : r - q.nrows;
-    if (r >= q.nrows) r -= q.nrows;
-    int h, blk, c0, nch = 0;
-    bool avail = false;
-    if (scanned + (int)lane < q.nrows) {
-      tp_row_geom(p, r, &h, &blk, &c0, &nch);
-      avail = nch > 0 && __ldcg(q.row_next + r) < nch;
+  const int lane = (int)lane_id();
+  int base = 0;
+  int64_t wbase = 0;
+  for (int r0 = 0; r0 < q.nrows; r0 += 32) {
+    const int r = r0 + lane;
+    int h, blk, jlo = 0;
+    const int64_t w = r < q.nrows ? tp_sr_row(p.n, p.nr, p.nblk, p.g0, p.g1, r, &h, &blk, &jlo) : 0;
+    int64_t wincl = w;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const int64_t v = __shfl_up_sync(FULL, wincl, d);
+      if (lane >= d) wincl += v;
     }
-    unsigned m = __ballot_sync(FULL, avail);
-    while (m) {
+    const int c = tp_sr_pieces(w, wbase + wincl - w, p.n - jlo, q.slots, q.total);
+    int incl = c;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const int v = __shfl_up_sync(FULL, incl, d);
+      if (lane >= d) incl += v;
+    }
+    const unsigned m = __ballot_sync(FULL, c > 0 && piece >= base + incl - c && piece < base + incl);
+    if (m) {
       const int l = __ffs(m) - 1;
-      const int rl = __shfl_sync(FULL, r, l), nl = __shfl_sync(FULL, nch, l);
-      int k = 0;
-      if (lane == 0) k = atomicAdd(q.row_next + rl, 1);
-      k = __shfl_sync(FULL, k, 0);
-      if (k < nl) return make_int2(rl, k);
-      m &= ~(1u << l);
+      return make_int3(r0 + l, piece - (base + __shfl_sync(FULL, incl - c, l)), __shfl_sync(FULL, c, l));
     }
+    base += __shfl_sync(FULL, incl, 31);
+    wbase += __shfl_sync(FULL, wincl, 31);
   }
-  return make_int2(-1, 0);
+  return make_int3(-1, 0, 0);
 }
 
-// Stage chunk k of `row` into ring slot `slot` (no-op for row < 0).
-__device__ __forceinline__ void tp_sr_stage(const TPParams& p, const TPSmem& S, int2 ch, int slot) {
-  if (ch.x < 0) return;
-  int h, blk, c0, nch;
-  tp_row_geom(p, ch.x, &h, &blk, &c0, &nch);
-  const int i0 = blk * HK_TP_NP_SR * TP_THREADS;
-  const int jlo = h <= p.nr ? i0 + 1 : 0;
-  const int j0 = max(jlo, (c0 + ch.y) * HK_TP_SR_CHUNK), j1 = min(p.n, (c0 + ch.y + 1) * HK_TP_SR_CHUNK);
-  const int sb = (h == 0) ? 0 : (h <= p.nr ? h : h - p.nr);
-  tp_stage_tile(p, S, sb, j0 & ~3, j1 - (j0 & ~3), slot);
-}
-
-// Claims run two chunks ahead of the computation: while chunk `cur` is computed, chunk `nxt`'s
-// tile is in flight and lane 0 of warp 0 has the atomic for the chunk after it outstanding (a
-// speculative claim in nxt's row; the scan of tp_sr_claim only when that row is exhausted).
 template <int V, bool LUT>
-__device__ __forceinline__ void tp_sr_run(const TPParams& p, const TPSmem& S, const TPSR& q, TPHistState* st, int2* claim) {
+__device__ __forceinline__ void tp_sr_piece(const TPParams& p, const TPSmem& S, const TPSR& q, int3 pc) {
   constexpr int NP = HK_TP_NP_SR;
   constexpr bool NL = (V & V_NL) != 0, L = (V & V_L) != 0, PROF = (V & V_PROF) != 0, CNT = L || PROF;
-  if (threadIdx.x < 32) {
-    const int2 a = tp_sr_claim(p, q, (int)(((int64_t)blockIdx.x * q.nrows) / gridDim.x));
-    const int2 b = a.x >= 0 ? tp_sr_claim(p, q, a.x) : a;
-    if (threadIdx.x == 0) { claim[0] = a; claim[1] = b; }
-  }
-  __syncthreads();
-  int2 cur = claim[0], nxt = claim[1];
-  int slot = 0;
-  tp_sr_stage(p, S, cur, 0);
-  tp_sr_stage(p, S, nxt, 1);
-  uint32_t Hw[NP / 2];
-  tp_lane_hist<NP>(p, S, Hw);
-  const TPLoopCtx c{S.L, smem_u32(S.E), S.E};
-  // the current visit
-  int vrow = -1, h = 0, blk = 0, c0 = 0, nch = 0, i0 = 0, jlo = 0, jall = 0, visited = 0;
-  int64_t gb = 0;
+  int h, blk, jlo;
+  tp_sr_row(p.n, p.nr, p.nblk, p.g0, p.g1, pc.x, &h, &blk, &jlo);
+  const int i0 = blk * NP * TP_THREADS;
+  const int64_t gb = (int64_t)h * p.n;
+  const int64_t len = p.n - jlo;
+  const int j0 = jlo + (int)(len * pc.y / pc.z), j1 = jlo + (int)(len * (pc.y + 1) / pc.z);
   TPPoint P[NP];
+  tp_points<NP>(p, p.hist, h, blk, p.g0, p.g1, P, NL);
   uint32_t inc[NP];
-  auto end_visit = [&]() {
 #pragma unroll
-    for (int k = 0; k < NP; ++k) {
-      P[k].acc /= 4;
-      tp_nl_exit<NL>(p, P[k], p.hist);
-      if (CNT && P[k].valid && P[k].cnt) {  // exact combine of this visit's partial sums
-        atomicAdd(p.accg + gb + P[k].i, P[k].acc);
-        atomicAdd(p.cntg + gb + P[k].i, P[k].cnt);
-      }
-    }
-    if (CNT) {
+  for (int k = 0; k < NP; ++k) inc[k] = P[k].valid ? ((k & 1) ? 0x10000u : 1u) : 0u;
+  tp_zero_hist<NP>(p, S);
+  __syncthreads();
+  tp_item_loop<NP, V, LUT>(p, S, P, inc, h, i0, j0, j1);
+#pragma unroll
+  for (int k = 0; k < NP; ++k) {
+    if (CNT) P[k].acc /= 4;
+    tp_nl_exit<NL>(p, P[k], p.hist);
+  }
+  if (CNT) {
+    if (pc.z == 1) {  // the whole row in this piece
+#pragma unroll
+      for (int k = 0; k < NP; ++k)
+        if (P[k].valid) tp_checks<V>(p, P[k], p.cb, gb + P[k].i);
+    } else {
+#pragma unroll
+      for (int k = 0; k < NP; ++k)
+        if (P[k].valid && P[k].cnt) {  // exact combine of this piece's partial sums
+          atomicAdd(p.accg + gb + P[k].i, P[k].acc);
+          atomicAdd(p.cntg + gb + P[k].i, P[k].cnt);
+        }
       __syncthreads();  // every thread's combine atomics issued
       if (threadIdx.x == 0) {
         __threadfence();
-        *S.flag = atomicAdd(q.row_done + vrow, visited) + visited == nch;
+        *S.flag = atomicAdd(q.row_done + pc.x, 1) + 1 == pc.z;
       }
       __syncthreads();
-      if (*S.flag) {  // this visit completed the row: the loop-exit checks of its points
+      if (*S.flag) {  // this piece completed the row: the loop-exit checks of its points
         __threadfence();
 #pragma unroll
         for (int k = 0; k < NP; ++k)
@@ -603,60 +577,14 @@ __device__ __forceinline__ void tp_sr_run(const TPParams& p, const TPSmem& S, co
           }
       }
     }
-    if (NL || L) {
-#pragma unroll
-      for (int k = 0; k < NP; ++k)
-        if (P[k].valid) fold_alarm(p.cb, P[k].alarm, (uint32_t)(gb + P[k].i));
-    }
-    __syncthreads();  // flag reused
-  };
-  while (cur.x >= 0) {
-    if (cur.x != vrow) {
-      if (vrow >= 0) end_visit();
-      vrow = cur.x;
-      tp_row_geom(p, vrow, &h, &blk, &c0, &nch);
-      i0 = blk * NP * TP_THREADS;
-      gb = (int64_t)h * p.n;
-      jlo = h <= p.nr ? i0 + 1 : 0;
-      jall = h <= p.nr ? min(i0 + NP * TP_THREADS, p.n) : 0;
-      visited = 0;
-      tp_hist_switch<NP>(p, S, st, h, nch * HK_TP_SR_CHUNK);
-      tp_points<NP>(p, p.hist, h, blk, p.g0, p.g1, P, NL);
-#pragma unroll
-      for (int k = 0; k < NP; ++k) inc[k] = P[k].valid ? ((k & 1) ? 0x10000u : 1u) : 0u;
-    }
-    // speculative claim of the chunk after nxt (its result is used after the computation)
-    int spec = -1, snch = 0;
-    if (threadIdx.x == 0 && nxt.x >= 0) {
-      int sh, sblk, sc0;
-      tp_row_geom(p, nxt.x, &sh, &sblk, &sc0, &snch);
-      spec = atomicAdd(q.row_next + nxt.x, 1);
-    }
-    if (nxt.x >= 0) cp_async_wait<1>();
-    else cp_async_wait<0>();
-    __syncthreads();  // cur's tile is staged
-    {
-      const int j0 = max(jlo, (c0 + cur.y) * HK_TP_SR_CHUNK), j1 = min(p.n, (c0 + cur.y + 1) * HK_TP_SR_CHUNK);
-      const int jt0 = j0 & ~3;
-      tp_tile_pairs<NP, CNT, LUT>(p, c, S.B + slot * 3 * TP_TILE, Hw, P, inc, jt0, j0 - jt0, j1 - jt0, jall, i0);
-    }
-    ++visited;
-    if (threadIdx.x < 32) {
-      int2 nn = make_int2(-1, 0);
-      if (nxt.x >= 0) {
-        const int sp = __shfl_sync(0xffffffffu, spec, 0), sn = __shfl_sync(0xffffffffu, snch, 0);
-        nn = sp < sn ? make_int2(nxt.x, sp) : tp_sr_claim(p, q, nxt.x);
-      }
-      if (threadIdx.x == 0) claim[0] = nn;
-    }
-    __syncthreads();  // the computation is done (slot free) and the next claim visible
-    const int2 nn = claim[0];
-    tp_sr_stage(p, S, nn, slot);
-    cur = nxt;
-    nxt = nn;
-    slot ^= 1;
   }
-  if (vrow >= 0) end_visit();
+  if (NL || L) {
+#pragma unroll
+    for (int k = 0; k < NP; ++k)
+      if (P[k].valid) fold_alarm(p.cb, P[k].alarm, (uint32_t)(gb + P[k].i));
+  }
+  __syncthreads();
+  tp_flush<NP>(p, S, p.hist, h * (p.nb + 2));
 }
 
 // FI & FT (or FI-only) replicas (blockIdx.y = launch slot)
@@ -942,17 +870,24 @@ __device__ void tpacf_fi_warp(const TPParams& p, const TPSmem& S, const FaultRec
       else if (it >= limit) ev = 2;
       else {
         const int32_t pb = (int32_t)(3u * (uint32_t)((uint32_t)bo + (uint32_t)j));
-        float q2[3];
-        for (int a = 0; a < 3 && !ev; ++a) {
-          const float* pe;
-          if (!fi_at(false, pp, pts_real, (int32_t)((uint32_t)pb + (uint32_t)a), npts, &pe)) ev = 3;
-          else q2[a] = __ldg(pe);
+        // x2, y2, z2 in order; the first out-of-bounds load ends the thread (crash model)
+        float x2 = 0.f, y2 = 0.f, z2 = 0.f;
+        const float* pe;
+        if (!fi_at(false, pp, pts_real, pb, npts, &pe)) ev = 3;
+        else x2 = __ldg(pe);
+        if (!ev) {
+          if (!fi_at(false, pp, pts_real, (int32_t)((uint32_t)pb + 1u), npts, &pe)) ev = 3;
+          else y2 = __ldg(pe);
         }
         if (!ev) {
-          if (KIND == TK_X2) q2[0] = flip_f(q2[0], now, mask);
-          if (KIND == TK_Y2) q2[1] = flip_f(q2[1], now, mask);
-          if (KIND == TK_Z2) q2[2] = flip_f(q2[2], now, mask);
-          float dot = __fmaf_rn(z1, q2[2], __fmaf_rn(y1, q2[1], __fmul_rn(x1, q2[0])));
+          if (!fi_at(false, pp, pts_real, (int32_t)((uint32_t)pb + 2u), npts, &pe)) ev = 3;
+          else z2 = __ldg(pe);
+        }
+        if (!ev) {
+          if (KIND == TK_X2) x2 = flip_f(x2, now, mask);
+          if (KIND == TK_Y2) y2 = flip_f(y2, now, mask);
+          if (KIND == TK_Z2) z2 = flip_f(z2, now, mask);
+          float dot = __fmaf_rn(z1, z2, __fmaf_rn(y1, y2, __fmul_rn(x1, x2)));
           if (KIND == TK_DOT) dot = flip_f(dot, now, mask);
           bin = LUT ? tp_b4_lut(S.L, lb, dot) / 4u : (uint32_t)tp_bin_search(S.E, dot);
           if (KIND == TK_BIN) bin = (uint32_t)flip_i((int32_t)bin, now, mask);

@@ -359,14 +359,16 @@ def test_bench_two_gloo_ranks_equal_one_rank():
 
 
 # ------------------------------------------------------------------- fused MRI-Q + TPACF replicas
-@pytest.mark.parametrize("variant,exact", [(0, 0), (0, 1), (1, 0)])
-def test_fused_replicas_equal_separate_launches(monkeypatch, variant, exact):
+@pytest.mark.parametrize("variant,exact,persist", [(0, 0, "0"), (0, 1, "0"), (1, 0, "0"), (0, 0, "3")])
+def test_fused_replicas_equal_separate_launches(monkeypatch, variant, exact, persist):
     """mix.cu (the default for mixed replica campaigns) against HK_FUSED=0 (one kind-homogeneous
     launch per benchmark): every record field equal, on config 5 with ragged batches, FI&FT and the
-    FI-only binary, FAST and EXACT; PhiMag sites take the separate path inside the same session."""
+    FI-only binary, FAST and EXACT, and the persistent variant (HK_MIX_PERSIST); PhiMag sites take
+    the separate path inside the same session."""
     probs = [W.cp_config1(), W.mriq_config2(), W.tpacf_config3()]
     devs = [_mk(b, probs[b], exact) for b in range(3)]
     R = [hk.profile_ranges(d) for d in devs] if variant == 0 else [None, None, None]
+    monkeypatch.setenv("HK_MIX_PERSIST", persist)
     out = {}
     for fused in ("1", "0"):
         monkeypatch.setenv("HK_FUSED", fused)

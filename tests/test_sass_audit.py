@@ -68,8 +68,10 @@ def test_mriq_ft_keeps_detectors(sass):
     assert _count(ft, "LOP3") >= _count(base, "LOP3") + 10
     # duplicated loads of sX, sY, sZ (A3) through an opaque index
     assert _count(ft, "LDG") >= _count(base, "LDG") + 3
-    loop_ft = _loop_region(ft, "MUFU.SIN")
-    assert sum(1 for o in loop_ft if o.startswith(("IADD3", "VIADD"))) >= 3  # 4-way unrolled: 3 between first/last SIN
+    # the counter advances once per unrolled group of samples (it += UNR through an opaque 1, the
+    # strength reduction of an unrolled it++): the FT loop keeps an add the BASE loop does not have
+    adds = lambda ops: sum(1 for o in ops if o.startswith(("IADD3", "VIADD", "IADD ", "IMAD")))
+    assert adds(_loop_region(ft, "MUFU.SIN")) > adds(_loop_region(base, "MUFU.SIN"))
     assert "UBLKCP.S.G" in ft
 
 

@@ -76,7 +76,7 @@ __device__ __forceinline__ void mix_mq_slot(const MixParams& q, unsigned char* s
 template <bool FT, bool LUT>
 __device__ __forceinline__ void mix_tp_faulted(const TPFIParams& q, const TPSmem& S, const FaultRec& f, unsigned long long* hist,
                                                hk_control* cb, int h, int blk) {
-  const int2 fi = tp_replica_fast<FT, LUT>(q, S, f, hist, cb, h, blk, true);
+  const int2 fi = tp_replica_fast<FT, LUT, false>(q, S, f, hist, cb, h, blk, true);
   if (fi.x < 0) return;
   TPParams p = q.base;
   p.hist = hist;
@@ -116,8 +116,8 @@ __device__ __forceinline__ void mix_tp_slot(const MixParams& q, unsigned char* s
     if (lut) mix_tp_faulted<FT, true>(q.t, S, f, hist, cb, h, blk);
     else mix_tp_faulted<FT, false>(q.t, S, f, hist, cb, h, blk);
   } else {
-    if (lut) tp_replica_fast<FT, true>(q.t, S, f, hist, cb, h, blk, false);
-    else tp_replica_fast<FT, false>(q.t, S, f, hist, cb, h, blk, false);
+    if (lut) tp_replica_fast<FT, true, false>(q.t, S, f, hist, cb, h, blk, false);
+    else tp_replica_fast<FT, false, false>(q.t, S, f, hist, cb, h, blk, false);
   }
 }
 

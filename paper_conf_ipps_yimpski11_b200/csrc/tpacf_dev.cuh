@@ -291,13 +291,14 @@ struct TPLoopCtx {
   const float* Es;
 };
 
-template <int NP, bool CNT, bool LUT>
+// Points 0..NQ-1 of the thread against one partner j (MASKQ: point NQ-1 only if j >= its jb).
+template <int NP, int NQ, bool MASKQ, bool CNT, bool LUT>
 __device__ __forceinline__ void tp_pair1(const TPLoopCtx& c, const uint32_t (&Hw)[NP / 2], TPPoint (&P)[NP],
-                                         const uint32_t (&inc)[NP], float x2, float y2, float z2, int j, bool masked) {
+                                         const uint32_t (&inc)[NP], float x2, float y2, float z2, int j) {
 #pragma unroll
-  for (int k = 0; k < NP; ++k) {
+  for (int k = 0; k < NQ; ++k) {
     const uint32_t b4 = tp_b4<LUT>(c.L, c.eb, c.Es, tp_dot(P[k], x2, y2, z2));
-    const bool on = !masked || j >= P[k].jb;
+    const bool on = !(MASKQ && k == NQ - 1) || j >= P[k].jb;
     red_shared(Hw[k / 2] + b4 * 32u, on ? inc[k] : 0u);
     if (CNT) {
       P[k].acc += on ? (int32_t)b4 : 0;
@@ -306,20 +307,83 @@ __device__ __forceinline__ void tp_pair1(const TPLoopCtx& c, const uint32_t (&Hw
   }
 }
 
+// Points 0..NQ-1 against the partners [k, k1) of the staged tile (partner jt0 + k); MASKQ: point
+// NQ-1 counts partner j only if j >= its jb (the diagonal, see tp_diag).  Groups of G partners
+// (G = 32 / NP, i.e. 3 * G / 4 broadcast LDS.128 per group) with the counters of the unmasked
+// points advanced by G per group (the strength reduction any compiler applies to an unrolled
+// cnt++; the FI program keeps the per-iteration increment).
+template <int NP, int NQ, bool MASKQ, bool CNT, bool LUT>
+__device__ __forceinline__ void tp_pairs_grp(const TPParams& p, const TPLoopCtx& c, const float* __restrict__ Bt,
+                                             const uint32_t (&Hw)[NP / 2], TPPoint (&P)[NP], const uint32_t (&inc)[NP],
+                                             int k, int k1, int jt0) {
+  if (!LUT) {  // the binary-search fallback (a bucket holds two edges): plain loop, rare
+#pragma unroll 1
+    for (; k < k1; ++k) tp_pair1<NP, NQ, MASKQ, CNT, LUT>(c, Hw, P, inc, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], jt0 + k);
+    return;
+  }
+  // partners per group: G * NQ pairs per thread and group (16 for NP = 4: enough independent
+  // table lookups in flight within the 80-register budget of 6 CTAs per SM)
+  constexpr int G = HK_TP_GROUP > 0 ? HK_TP_GROUP : (NP >= 4 ? 4 : 8);
+  static_assert(G % 4 == 0, "groups are whole 48-byte partner quads");
+  for (; k < k1 && (k & 3); ++k) tp_pair1<NP, NQ, MASKQ, CNT, LUT>(c, Hw, P, inc, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], jt0 + k);
+  const float4* __restrict__ T4 = reinterpret_cast<const float4*>(Bt);
+#pragma unroll 1
+  for (; k + G - 1 < k1; k += G) {
+    const int k3 = (k >> 2) * 3;
+    float xs[G], ys[G], zs[G];
+#pragma unroll
+    for (int q = 0; q < G / 4; ++q) {
+      const float4 v0 = T4[k3 + 3 * q], v1 = T4[k3 + 3 * q + 1], v2 = T4[k3 + 3 * q + 2];
+      xs[4 * q] = v0.x; ys[4 * q] = v0.y; zs[4 * q] = v0.z;
+      xs[4 * q + 1] = v0.w; ys[4 * q + 1] = v1.x; zs[4 * q + 1] = v1.y;
+      xs[4 * q + 2] = v1.z; ys[4 * q + 2] = v1.w; zs[4 * q + 2] = v2.x;
+      xs[4 * q + 3] = v2.y; ys[4 * q + 3] = v2.z; zs[4 * q + 3] = v2.w;
+    }
+    uint32_t b[NQ][G];
+#pragma unroll
+    for (int u = 0; u < G; ++u)
+#pragma unroll
+      for (int kk = 0; kk < NQ; ++kk) b[kk][u] = tp_b4<LUT>(c.L, c.eb, c.Es, tp_dot(P[kk], xs[u], ys[u], zs[u]));
+    bool on[G];
+#pragma unroll
+    for (int u = 0; u < G; ++u) on[u] = !MASKQ || jt0 + k + u >= P[NQ - 1].jb;
+#pragma unroll
+    for (int u = 0; u < G; ++u)
+#pragma unroll
+      for (int kk = 0; kk < NQ; ++kk)
+        red_shared(Hw[kk / 2] + b[kk][u] * 32u, (MASKQ && kk == NQ - 1 && !on[u]) ? 0u : inc[kk]);
+    if (CNT) {
+#pragma unroll
+      for (int kk = 0; kk < NQ; ++kk) {
+        if (MASKQ && kk == NQ - 1) {
+#pragma unroll
+          for (int u = 0; u < G; ++u) {
+            P[kk].acc += on[u] ? (int32_t)b[kk][u] : 0;
+            P[kk].cnt += on[u] ? 1 : 0;
+          }
+        } else {
+#pragma unroll
+          for (int u = 0; u < G; u += 2) P[kk].acc += (int32_t)(b[kk][u] + b[kk][u + 1]);
+          P[kk].cnt = count_inc(P[kk].cnt, G == 8 ? p.eight : (G == 4 ? p.four : p.one * G));
+        }
+      }
+    }
+  }
+  for (; k < k1; ++k) tp_pair1<NP, NQ, MASKQ, CNT, LUT>(c, Hw, P, inc, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], jt0 + k);
+}
+// All points against [k, k1): the unmasked form of tp_pairs_grp, kept as its own loop (ptxas
+// schedules this one with the table lookups of a group interleaved; measured in mix.cu)
 template <int NP, bool CNT, bool LUT>
 __device__ __forceinline__ void tp_pairs_all(const TPParams& p, const TPLoopCtx& c, const float* __restrict__ Bt,
                                              const uint32_t (&Hw)[NP / 2], TPPoint (&P)[NP], const uint32_t (&inc)[NP],
                                              int k, int k1) {
-  if (!LUT) {  // the binary-search fallback (a bucket holds two edges): plain loop, rare
-#pragma unroll 1
-    for (; k < k1; ++k) tp_pair1<NP, CNT, LUT>(c, Hw, P, inc, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], 0, false);
+  if (!LUT) {
+    tp_pairs_grp<NP, NP, false, CNT, LUT>(p, c, Bt, Hw, P, inc, k, k1, 0);
     return;
   }
-  // partners per group: G * NP pairs per thread and group (16 for NP = 4: enough independent
-  // table lookups in flight within the 80-register budget of 6 CTAs per SM)
   constexpr int G = HK_TP_GROUP > 0 ? HK_TP_GROUP : (NP >= 4 ? 4 : 8);
   static_assert(G % 4 == 0, "groups are whole 48-byte partner quads");
-  for (; k < k1 && (k & 3); ++k) tp_pair1<NP, CNT, LUT>(c, Hw, P, inc, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], 0, false);
+  for (; k < k1 && (k & 3); ++k) tp_pair1<NP, NP, false, CNT, LUT>(c, Hw, P, inc, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], 0);
   const float4* __restrict__ T4 = reinterpret_cast<const float4*>(Bt);
 #pragma unroll 1
   for (; k + G - 1 < k1; k += G) {
@@ -351,47 +415,45 @@ __device__ __forceinline__ void tp_pairs_all(const TPParams& p, const TPLoopCtx&
       }
     }
   }
-  for (; k < k1; ++k) tp_pair1<NP, CNT, LUT>(c, Hw, P, inc, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], 0, false);
+  for (; k < k1; ++k) tp_pair1<NP, NP, false, CNT, LUT>(c, Hw, P, inc, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], 0);
+}
+
+// The diagonal, one partner at a time (GDIAG = false: the fused kernel of mix.cu, where the
+// grouped form below costs the main loop its interleaved schedule — measured).
+template <int NP, bool CNT, bool LUT, int S = 0>
+__device__ __forceinline__ void tp_diag1(const TPLoopCtx& c, const float* __restrict__ Bt, const uint32_t (&Hw)[NP / 2],
+                                         TPPoint (&P)[NP], const uint32_t (&inc)[NP], int i0, int jt0, int k0, int km) {
+  const int ka = max(k0, i0 + S * TP_THREADS - jt0), kb = min(km, i0 + (S + 1) * TP_THREADS - jt0);
+#pragma unroll 1
+  for (int k = ka; k < kb; ++k) tp_pair1<NP, S + 1, true, CNT, LUT>(c, Hw, P, inc, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], jt0 + k);
+  if constexpr (S + 1 < NP) tp_diag1<NP, CNT, LUT, S + 1>(c, Bt, Hw, P, inc, i0, jt0, k0, km);
 }
 
 // The diagonal of a self-correlation row, segment S: partners j in [i0 + 128 S, i0 + 128 (S + 1))
 // (tile-relative [ka, kb)).  Point k of a thread is i0 + 128 k + t, so for these partners points
-// k < S are all active (j > i), point S is masked (j >= jb) and points k > S take no part.
-template <int NP, bool CNT, bool LUT, int S>
-__device__ __forceinline__ void tp_diag_seg(const TPLoopCtx& c, const float* __restrict__ Bt, const uint32_t (&Hw)[NP / 2],
-                                            TPPoint (&P)[NP], const uint32_t (&inc)[NP], int jt0, int ka, int kb) {
-#pragma unroll 1
-  for (int k = ka; k < kb; ++k) {
-    const float x2 = Bt[3 * k], y2 = Bt[3 * k + 1], z2 = Bt[3 * k + 2];
-#pragma unroll
-    for (int q = 0; q <= S; ++q) {
-      const uint32_t b4 = tp_b4<LUT>(c.L, c.eb, c.Es, tp_dot(P[q], x2, y2, z2));
-      const bool on = q < S || jt0 + k >= P[q].jb;
-      red_shared(Hw[q / 2] + b4 * 32u, on ? inc[q] : 0u);
-      if (CNT) {
-        P[q].acc += on ? (int32_t)b4 : 0;
-        P[q].cnt += on ? 1 : 0;
-      }
-    }
-  }
-}
+// k < S are all active (j > i), point S is masked (j >= jb) and points k > S take no part: the
+// grouped loop over points 0..S with the mask on point S.
 template <int NP, bool CNT, bool LUT, int S = 0>
-__device__ __forceinline__ void tp_diag(const TPLoopCtx& c, const float* __restrict__ Bt, const uint32_t (&Hw)[NP / 2],
-                                        TPPoint (&P)[NP], const uint32_t (&inc)[NP], int i0, int jt0, int k0, int km) {
+__device__ __forceinline__ void tp_diag(const TPParams& p, const TPLoopCtx& c, const float* __restrict__ Bt,
+                                        const uint32_t (&Hw)[NP / 2], TPPoint (&P)[NP], const uint32_t (&inc)[NP], int i0, int jt0,
+                                        int k0, int km) {
   const int ka = max(k0, i0 + S * TP_THREADS - jt0), kb = min(km, i0 + (S + 1) * TP_THREADS - jt0);
-  if (ka < kb) tp_diag_seg<NP, CNT, LUT, S>(c, Bt, Hw, P, inc, jt0, ka, kb);
-  if constexpr (S + 1 < NP) tp_diag<NP, CNT, LUT, S + 1>(c, Bt, Hw, P, inc, i0, jt0, k0, km);
+  if (ka < kb) tp_pairs_grp<NP, S + 1, true, CNT, LUT>(p, c, Bt, Hw, P, inc, ka, kb, jt0);
+  if constexpr (S + 1 < NP) tp_diag<NP, CNT, LUT, S + 1>(p, c, Bt, Hw, P, inc, i0, jt0, k0, km);
 }
 
 // Pairs of the staged tile Bt (partners jt0 + k) for k in [k0, k1): [k0, km) with per-point masks
 // (partners below jall = min(i0 + NP * 128, N) in a self-correlation row: its diagonal, in
 // segments), [km, k1) for all points.
-template <int NP, bool CNT, bool LUT>
+template <int NP, bool CNT, bool LUT, bool GDIAG = true>
 __device__ __forceinline__ void tp_tile_pairs(const TPParams& p, const TPLoopCtx& c, const float* __restrict__ Bt,
                                               const uint32_t (&Hw)[NP / 2], TPPoint (&P)[NP], const uint32_t (&inc)[NP],
                                               int jt0, int k0, int k1, int jall, int i0) {
   const int km = min(max(jall - jt0, k0), k1);
-  if (k0 < km) tp_diag<NP, CNT, LUT>(c, Bt, Hw, P, inc, i0, jt0, k0, km);
+  if (k0 < km) {
+    if (GDIAG) tp_diag<NP, CNT, LUT>(p, c, Bt, Hw, P, inc, i0, jt0, k0, km);
+    else tp_diag1<NP, CNT, LUT>(c, Bt, Hw, P, inc, i0, jt0, k0, km);
+  }
   tp_pairs_all<NP, CNT, LUT>(p, c, Bt, Hw, P, inc, km, k1);
 }
 template <int NP>
@@ -404,7 +466,7 @@ __device__ __forceinline__ void tp_lane_hist(const TPParams& p, const TPSmem& S,
 // One work item: the points i0 + t + 128 k (k < NP) of histogram h against partners [jr0, jr1)
 // (already clipped to the block's [jlo, N)), streamed tile by tile through the ring.  The tables
 // are staged and the histogram zeroed by the caller.
-template <int NP, int V, bool LUT>
+template <int NP, int V, bool LUT, bool GDIAG = true>
 __device__ __forceinline__ void tp_item_loop(const TPParams& p, const TPSmem& S, TPPoint (&P)[NP], const uint32_t (&inc)[NP],
                                              int h, int i0, int jr0, int jr1) {
   constexpr bool CNT = (V & (V_L | V_PROF)) != 0;
@@ -429,7 +491,7 @@ __device__ __forceinline__ void tp_item_loop(const TPParams& p, const TPSmem& S,
       cp_async_wait<0>();
     }
     __syncthreads();
-    tp_tile_pairs<NP, CNT, LUT>(p, c, S.B + (t & 1) * 3 * TP_TILE, Hw, P, inc, jt0, max(jr0, jt0) - jt0,
+    tp_tile_pairs<NP, CNT, LUT, GDIAG>(p, c, S.B + (t & 1) * 3 * TP_TILE, Hw, P, inc, jt0, max(jr0, jt0) - jt0,
                                 min(jr1, jt0 + TP_TILE) - jt0, jall, i0);
     __syncthreads();  // slot t & 1 is refilled by the stage of tile t + 2
   }
@@ -950,7 +1012,7 @@ __device__ void tpacf_fi_warp(const TPParams& p, const TPSmem& S, const FaultRec
 // Replica CTA (h, point block) of the FI kernel, whole partner loops, fast part.  The faulted
 // abstract thread (if this CTA holds it) takes no part in the fast loop (increment 0, no exit
 // checks); returns (point index, N0 duplicate) of it in the warp that holds it, else (-1, 0).
-template <bool FT, bool LUT>
+template <bool FT, bool LUT, bool GDIAG = true>
 __device__ __forceinline__ int2 tp_replica_fast(const TPFIParams& q, const TPSmem& S, const FaultRec& f, unsigned long long* hist,
                                                 hk_control* cb, int h, int blk, bool faulted) {
   constexpr int NP = HK_TP_NP_FI;
@@ -974,7 +1036,7 @@ __device__ __forceinline__ int2 tp_replica_fast(const TPFIParams& q, const TPSme
   tp_zero_hist<NP>(p, S);
   __syncthreads();
   const int jlo = h <= p.nr ? i0 + 1 : 0;
-  tp_item_loop<NP, V, LUT>(p, S, P, inc, h, i0, jlo, p.n);
+  tp_item_loop<NP, V, LUT, GDIAG>(p, S, P, inc, h, i0, jlo, p.n);
 #pragma unroll
   for (int k = 0; k < NP; ++k) {
     if (!P[k].valid || k == fk) continue;

@@ -22,7 +22,8 @@
 #define HK_MIX_MQ_VPT 2  // voxels per CUDA thread of the MRI-Q role
 #endif
 #ifndef HK_MIX_MINB
-#define HK_MIX_MINB 5  // 5 CTAs per SM: 96 registers (6 CTAs: 80 registers, spills; measured 7 % slower)
+#define HK_MIX_MINB 4  // 4 CTAs per SM: 128 registers, no spills (5 CTAs: 96 registers with 12-16 B of spills,
+                       // measured 3.7 % slower per mixed step; 6 CTAs: 80 registers, 7 % slower)
 #endif
 
 namespace hk {

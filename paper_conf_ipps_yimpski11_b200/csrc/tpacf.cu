@@ -29,41 +29,45 @@
 
 namespace hk {
 
-// One thread per bucket q: the dot interval of the bucket is found by stepping from
-// fl(1 - u_lo) / fl(1 - u_hi) to the exact extremes (negative-u buckets have their bit order
-// reversed); inf / NaN buckets are set directly.
-__global__ void tpacf_lut_kernel(const float* __restrict__ edges, int nb, uint8_t* __restrict__ lut, int* ok) {
+// One thread per bucket q.  Buckets in u-value order: ord(q) = 1024 + q for u >= +0 (q < 1024),
+// 2047 - q for u <= -0 (bit order reversed).  Because fl(1 - .) is monotone non-increasing, every
+// dot of bucket q is below edge e iff bucket(fl(1 - e)) comes before q (then dot < e for all of
+// them), and above it iff that bucket comes after q; so bmin(q) = bin(dmax(q)) is the number of
+// edges whose u-bucket precedes q, and bin = bmin + (dot < edge[bmin]) holds exactly when no two
+// edges share a bucket (checked; the edges are strictly decreasing, so their bucket ordinals are
+// non-decreasing).  Exponent-0xff buckets: +inf u (dot = -inf) follows the same rule (every finite
+// edge precedes it); NaN u (dot NaN) has bin 0; -inf u (dot = +inf) precedes every bucket.
+// Block 0 also writes the validity flag (no separate memset).
+__device__ __forceinline__ int tp_bucket_ord(uint32_t q) { return q < 1024u ? 1024 + (int)q : 2047 - (int)q; }
+__global__ void __launch_bounds__(256) tpacf_lut_kernel(const float* __restrict__ edges, int nb, uint8_t* __restrict__ lut, int* ok) {
+  __shared__ int eo[32];
+  __shared__ int bad;
   const int q = blockIdx.x * blockDim.x + threadIdx.x;
+  if (threadIdx.x == 0) bad = 0;
+  __syncthreads();
+  if (threadIdx.x <= nb && threadIdx.x < 32) {
+    const float e = edges[threadIdx.x];
+    const float u = __fsub_rn(1.0f, e);
+    eo[threadIdx.x] = tp_bucket_ord(fb(u) >> 21);
+    if (u != u) atomicExch(&bad, 1);  // a NaN edge: no table
+  }
+  __syncthreads();
+  if (threadIdx.x < nb && threadIdx.x < 31 && eo[threadIdx.x] >= eo[threadIdx.x + 1]) atomicExch(&bad, 1);
+  __syncthreads();
+  if (blockIdx.x == 0 && threadIdx.x == 0) *ok = bad ? 0 : 1;
   if (q >= TP_LUT) return;
-  const uint32_t lo_bits = (uint32_t)q << 21, hi_bits = lo_bits | 0x1fffffu;
-  const bool neg = (lo_bits & 0x80000000u) != 0;
-  const uint32_t ex = (lo_bits >> 23) & 0xffu;
+  const uint32_t uq = (uint32_t)q;
+  const uint32_t ex = (uq >> 2) & 0xffu;
   int bmin = 0;
-  bool good = true;
-  if (ex == 0xffu) {
-    // u = +-inf or NaN.  u = +inf <=> dot = -inf: bin = #{edges > -inf}, the compare value -inf
-    // (or edge[nb] = -inf) adds nothing; u = -inf <=> dot = +inf: bin 0; NaN u <=> NaN dot: bin 0
-    // (every compare false).  FADD returns the canonical NaN 0x7fffffff, so the +inf bucket
-    // (bits 0x7f800000-0x7f9fffff) never holds a NaN u.
-    const bool plus_inf = !neg && (lo_bits & 0x7fffffu) == 0;
-    bmin = plus_inf ? bin_def(edges, nb, __int_as_float(0xff800000)) : 0;
+  if (ex == 0xffu && (uq & 0x400u) == 0 && (uq & 0x3u) != 0) {
+    bmin = 0;  // positive NaN buckets (0x7fa00000 .. 0x7fffffff): dot NaN -> bin 0
+  } else if (ex == 0xffu && (uq & 0x400u) != 0) {
+    bmin = 0;  // -inf / negative-NaN buckets: dot = +inf or NaN -> bin 0
   } else {
-    // [ulo, uhi] in value order (for negative u the bit order is reversed)
-    const float ua = bf(lo_bits), ub = bf(hi_bits);
-    const float ulo = neg ? ub : ua, uhi = neg ? ua : ub;
-    // largest dot with fl(1 - dot) >= ulo, smallest dot with fl(1 - dot) <= uhi
-    float dmax = __fsub_rn(1.0f, ulo);
-    for (int k = 0; k < 64 && __fsub_rn(1.0f, nup(dmax)) >= ulo; ++k) dmax = nup(dmax);
-    for (int k = 0; k < 64 && __fsub_rn(1.0f, dmax) < ulo; ++k) dmax = ndown(dmax);
-    float dmin = __fsub_rn(1.0f, uhi);
-    for (int k = 0; k < 64 && __fsub_rn(1.0f, ndown(dmin)) <= uhi; ++k) dmin = ndown(dmin);
-    for (int k = 0; k < 64 && __fsub_rn(1.0f, dmin) > uhi; ++k) dmin = nup(dmin);
-    bmin = bin_def(edges, nb, dmax);
-    const int bmax = bin_def(edges, nb, dmin);
-    good = (__fsub_rn(1.0f, dmax) >= ulo) && (__fsub_rn(1.0f, dmin) <= uhi) && (bmax - bmin <= 1);
+    const int o = tp_bucket_ord(uq);
+    for (int k = 0; k <= nb && k < 32; ++k) bmin += eo[k] < o ? 1 : 0;
   }
   lut[q] = (uint8_t)(4 * bmin);  // byte offset of E[bmin] (E padded with -inf beyond nb)
-  if (!good) atomicExch(ok, 0);
 }
 #ifdef HK_TP_SR_TRACE
 __device__ unsigned long long g_tp_trace[4096][4];  // debug builds: (smid, start ns, end ns, piece)
@@ -72,7 +76,7 @@ extern "C" __attribute__((visibility("default"))) int hk_debug_trace(void* out) 
 }
 #endif
 template <int V>
-__global__ void __launch_bounds__(TP_THREADS, HK_TP_MINB_SR) tpacf_kernel(const TPParams p, const TPSR q) {
+__global__ void __launch_bounds__(TP_THREADS, V == 0 ? HK_TP_MINB_SR : HK_TP_MINB_SR_FT) tpacf_kernel(const TPParams p, const TPSR q) {
 #ifdef HK_TP_SR_TRACE
   unsigned long long t0;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
@@ -267,8 +271,6 @@ size_t tpacf_ws_bytes(const hk_tpacf_args& a) {
 
 cudaError_t tpacf_lut_build(const hk_tpacf_args& a, void* ws, cudaStream_t s) {
   int* ok = reinterpret_cast<int*>(reinterpret_cast<char*>(ws) + TP_LUT);
-  cudaError_t e = cudaMemsetAsync(ok, 1, sizeof(int), s);
-  if (e != cudaSuccess) return e;
   tpacf_lut_kernel<<<TP_LUT / 256, 256, 0, s>>>(a.edges, a.n_bins, reinterpret_cast<uint8_t*>(ws), ok);
   count_launch();
   return cudaGetLastError();

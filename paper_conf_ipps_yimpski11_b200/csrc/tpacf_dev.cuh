@@ -16,7 +16,10 @@ namespace hk {
 #define HK_TP_MINB 6     // replicas: 37 KB of shared memory per CTA -> 6 CTAs per SM, 80 registers
 #endif
 #ifndef HK_TP_MINB_SR
-#define HK_TP_MINB_SR 6  // single run: 37 KB per CTA -> 6 CTAs per SM, 80 registers
+#define HK_TP_MINB_SR 6  // single run BASE: 37 KB per CTA -> 6 CTAs per SM, 80 registers
+#endif
+#ifndef HK_TP_MINB_SR_FT
+#define HK_TP_MINB_SR_FT 5  // single run with detectors: 96 registers (at 80 the NL / L state spills)
 #endif
 #ifndef HK_TP_GROUP
 #define HK_TP_GROUP 0  // partners per group of the unmasked loop (0: 4 for NP >= 4, else 8)
@@ -88,23 +91,6 @@ __device__ __forceinline__ uint32_t tp_b4(const uint8_t* __restrict__, uint32_t,
 __device__ __forceinline__ void red_shared(uint32_t addr, uint32_t v) {
   asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(addr), "r"(v) : "memory");
 }
-
-__device__ __forceinline__ float nup(float x) {
-  const uint32_t b = fb(x);
-  if ((b & 0x7fffffffu) == 0) return bf(1u);
-  return (b & 0x80000000u) ? bf(b - 1) : bf(b + 1);
-}
-__device__ __forceinline__ float ndown(float x) {
-  const uint32_t b = fb(x);
-  if ((b & 0x7fffffffu) == 0) return bf(0x80000001u);
-  return (b & 0x80000000u) ? bf(b + 1) : bf(b - 1);
-}
-__device__ __forceinline__ int32_t bin_def(const float* edges, int nb, float dot) {
-  int32_t b = 0;
-  for (int e = 0; e <= nb; ++e) b += (dot < edges[e]) ? 1 : 0;
-  return b;
-}
-
 
 // ---------------------------------------------------------------------------------------------
 // Shared memory: L[2048] u8 | E[32] f32 | B[2][3 * TP_TILE] f32 (packed x, y, z) |

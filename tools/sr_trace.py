@@ -40,3 +40,5 @@ for q in (0.0, 0.5, 0.9, 1.0):
 slow = np.argsort(-dur)[:10]
 print("slowest rows:", row[slow].tolist(), "pieces:", ((b[slow, 3] >> 16) & 0xffff).tolist(), [round(x, 1) for x in dur[slow]])
 print("mean dur by h:", {int(h): round(float(dur[(row // 8) == h].mean()), 1) for h in range(9)})
+rank = np.arange(n) // 148
+print("mean dur by launch rank (blockIdx // 148):", {int(k): round(float(dur[rank == k].mean()), 1) for k in range(int(rank.max()) + 1)})

@@ -5,7 +5,8 @@ import torch
 import workloads as W
 from paper_conf_ipps_yimpski11_b200 import hauberk as hk
 dev = torch.device("cuda", 0)
-which = sys.argv[1:] or ["cp", "mriq", "tpacf"]
+which = [a for a in sys.argv[1:] if not a.startswith("--v=")] or ["cp", "mriq", "tpacf"]
+variants = [int(a[4:]) for a in sys.argv[1:] if a.startswith("--v=")]  # e.g. --v=1 --v=3 (default BASE, FT)
 for name in which:
     if name == "cp":
         d = hk.CPDevice.from_problem(W.cp_config4(bx=16, by=16, unroll=8), dev)
@@ -15,7 +16,7 @@ for name in which:
         d = hk.TPACFDevice.from_problem(W.tpacf_config3(), dev)
     R = hk.profile_ranges(d)
     cb = hk.new_control(dev)
-    for v in (hk.HK_BASE, hk.HK_FT):
+    for v in (variants or (hk.HK_BASE, hk.HK_FT)):
         hk.run(d, v, R, cb)
     torch.cuda.synchronize()
     print(name, "ok")

@@ -21,6 +21,10 @@
 #ifndef HK_MIX_MQ_VPT
 #define HK_MIX_MQ_VPT 2  // voxels per CUDA thread of the MRI-Q role
 #endif
+#ifndef HK_MIX_GDIAG
+#define HK_MIX_GDIAG true  // TPACF role: the diagonal as grouped loops (at 96 registers the grouped form
+                           // cost the main loop its interleaved schedule; at 128 it is 1.4 % faster)
+#endif
 #ifndef HK_MIX_MINB
 #define HK_MIX_MINB 4  // 4 CTAs per SM: 128 registers, no spills (5 CTAs: 96 registers with 12-16 B of spills,
                        // measured 3.7 % slower per mixed step; 6 CTAs: 80 registers, 7 % slower)
@@ -77,7 +81,7 @@ __device__ __forceinline__ void mix_mq_slot(const MixParams& q, unsigned char* s
 template <bool FT, bool LUT>
 __device__ __forceinline__ void mix_tp_faulted(const TPFIParams& q, const TPSmem& S, const FaultRec& f, unsigned long long* hist,
                                                hk_control* cb, int h, int blk) {
-  const int2 fi = tp_replica_fast<FT, LUT, false>(q, S, f, hist, cb, h, blk, true);
+  const int2 fi = tp_replica_fast<FT, LUT, HK_MIX_GDIAG>(q, S, f, hist, cb, h, blk, true);
   if (fi.x < 0) return;
   TPParams p = q.base;
   p.hist = hist;
@@ -117,8 +121,8 @@ __device__ __forceinline__ void mix_tp_slot(const MixParams& q, unsigned char* s
     if (lut) mix_tp_faulted<FT, true>(q.t, S, f, hist, cb, h, blk);
     else mix_tp_faulted<FT, false>(q.t, S, f, hist, cb, h, blk);
   } else {
-    if (lut) tp_replica_fast<FT, true, false>(q.t, S, f, hist, cb, h, blk, false);
-    else tp_replica_fast<FT, false, false>(q.t, S, f, hist, cb, h, blk, false);
+    if (lut) tp_replica_fast<FT, true, HK_MIX_GDIAG>(q.t, S, f, hist, cb, h, blk, false);
+    else tp_replica_fast<FT, false, HK_MIX_GDIAG>(q.t, S, f, hist, cb, h, blk, false);
   }
 }
 

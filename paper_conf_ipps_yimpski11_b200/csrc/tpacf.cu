@@ -76,13 +76,13 @@ extern "C" __attribute__((visibility("default"))) int hk_debug_trace(void* out) 
 }
 #endif
 template <int V>
-__global__ void __launch_bounds__(TP_THREADS, V == 0 ? HK_TP_MINB_SR : HK_TP_MINB_SR_FT) tpacf_kernel(const TPParams p, const TPSR q) {
+__global__ void __launch_bounds__(TP_SR_T, V == 0 ? HK_TP_MINB_SR : HK_TP_MINB_SR_FT) tpacf_kernel(const TPParams p, const TPSR q) {
 #ifdef HK_TP_SR_TRACE
   unsigned long long t0;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
 #endif
   __shared__ int3 s_pc;
-  const TPSmem S = tp_carve(hk_tp_dsmem, p.nb + 2, HK_TP_NP_SR);
+  const TPSmem S = tp_carve(hk_tp_dsmem, p.nb + 2, HK_TP_NP_SR, TP_SR_T);
   tp_stage_tables(p, S);
   if (threadIdx.x < 32) {
     const int3 pc = tp_sr_locate(p, q, (int)blockIdx.x);
@@ -232,7 +232,7 @@ __global__ void __launch_bounds__(128) tpacf_replay_all_kernel(const TPReplayPar
 // ============================================================================================
 // Host launchers
 // ============================================================================================
-static int tp_nblk(int n, int np) { return (n + np * TP_THREADS - 1) / (np * TP_THREADS); }
+static int tp_nblk(int n, int np, int T = TP_THREADS) { return (n + np * T - 1) / (np * T); }
 
 static TPParams tp_params(const hk_tpacf_args& a, const DevRanges& R, int ndet, hk_control* cb, float* samples,
                           void* ws) {
@@ -249,7 +249,7 @@ static TPParams tp_params(const hk_tpacf_args& a, const DevRanges& R, int ndet, 
   p.nr = a.n_rand;
   p.nb = a.n_bins;
   p.ndet = ndet;
-  p.nblk = tp_nblk(a.n, HK_TP_NP_SR);
+  p.nblk = tp_nblk(a.n, HK_TP_NP_SR, TP_SR_T);
   p.g0 = 0;
   p.g1 = (1 + 2 * a.n_rand) * a.n;
   p.z = opaque_zero();
@@ -262,7 +262,7 @@ static TPParams tp_params(const hk_tpacf_args& a, const DevRanges& R, int ndet, 
 // Workspace (tpacf_ws_bytes): table [TP_LUT] u8 | ok flag (16 B) | row_done [nrows] (padded to 16 B) |
 // accg [nh * N] | cntg [nh * N]  (nrows = nh * blocks of 128 * HK_TP_NP_SR points)
 static size_t tp_ws_head() { return (size_t)TP_LUT + 16; }
-static int tp_nrows(const hk_tpacf_args& a) { return (1 + 2 * a.n_rand) * tp_nblk(a.n, HK_TP_NP_SR); }
+static int tp_nrows(const hk_tpacf_args& a) { return (1 + 2 * a.n_rand) * tp_nblk(a.n, HK_TP_NP_SR, TP_SR_T); }
 static size_t tp_rows_bytes(const hk_tpacf_args& a) { return ((size_t)tp_nrows(a) * sizeof(int) + 15) / 16 * 16; }
 size_t tpacf_ws_bytes(const hk_tpacf_args& a) {
   const size_t nt = (size_t)(1 + 2 * a.n_rand) * (size_t)a.n;
@@ -288,14 +288,14 @@ void tpacf_release_caches() {}
 template <int V>
 static cudaError_t launch_tp_v(const hk_tpacf_args& a, TPParams p, void* ws, cudaStream_t s) {
   constexpr bool CNT = (V & (V_L | V_PROF)) != 0;
-  const size_t smem = tp_smem_bytes(p.nb + 2, HK_TP_NP_SR);
+  const size_t smem = tp_smem_bytes(p.nb + 2, HK_TP_NP_SR, TP_SR_T);
   cudaError_t e = cudaFuncSetAttribute(tpacf_kernel<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   if (p.g1 <= p.g0) return cudaSuccess;
   int dev = 0, nsm = 0, per_sm = 0;
   if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
   if ((e = cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess) return e;
-  if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tpacf_kernel<V>, TP_THREADS, smem)) != cudaSuccess) return e;
+  if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tpacf_kernel<V>, TP_SR_T, smem)) != cudaSuccess) return e;
   char* w = reinterpret_cast<char*>(ws);
   TPSR q;
   q.nrows = tp_nrows(a);
@@ -325,7 +325,7 @@ static cudaError_t launch_tp_v(const hk_tpacf_args& a, TPParams p, void* ws, cud
   }
   if (CNT && (e = cudaMemsetAsync(w + tp_ws_head(), 0, tpacf_ws_bytes(a) - tp_ws_head(), s)) != cudaSuccess) return e;
   TimedScope ts(HK_TPACF, 0, tp_pairs(a) * (double)(p.g1 - p.g0) / (double)((1 + 2 * p.nr) * p.n), s);
-  tpacf_kernel<V><<<(unsigned)grid, TP_THREADS, smem, s>>>(p, q);
+  tpacf_kernel<V><<<(unsigned)grid, TP_SR_T, smem, s>>>(p, q);
   count_launch();
   return cudaGetLastError();
 }

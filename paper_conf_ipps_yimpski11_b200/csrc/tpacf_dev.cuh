@@ -15,8 +15,11 @@ namespace hk {
 #ifndef HK_TP_MINB
 #define HK_TP_MINB 6     // replicas: 37 KB of shared memory per CTA -> 6 CTAs per SM, 80 registers
 #endif
+#ifndef HK_TP_SR_T
+#define HK_TP_SR_T 128  // single run: threads per CTA (128: six CTAs per SM; 256 / 512 measured slower)
+#endif
 #ifndef HK_TP_MINB_SR
-#define HK_TP_MINB_SR 6  // single run BASE: 37 KB per CTA -> 6 CTAs per SM, 80 registers
+#define HK_TP_MINB_SR (HK_TP_SR_T == 128 ? 6 : 1)  // single run BASE: CTAs per SM (128 threads: 37 KB, 80 registers)
 #endif
 #ifndef HK_TP_STASH
 #define HK_TP_STASH 0x2  // single-run variants (bit V) that keep the points' exit state in local memory:
@@ -24,13 +27,15 @@ namespace hk {
                          // 77.8 -> 67.6 us); FT and FT_L measured 2 us slower with it
 #endif
 #ifndef HK_TP_MINB_SR_FT
-#define HK_TP_MINB_SR_FT 5  // single run with detectors: 96 registers (at 80 the NL / L state spills)
+#define HK_TP_MINB_SR_FT (HK_TP_SR_T == 128 ? 5 : 1)  // with detectors: 96 registers at 128 threads (at 80 the
+                                                       // NL / L state spills)
 #endif
 #ifndef HK_TP_GROUP
 #define HK_TP_GROUP 0  // partners per group of the unmasked loop (0: 4 for NP >= 4, else 8)
 #endif
 constexpr int TP_THREADS = 128;
 constexpr int TP_WARPS = TP_THREADS / 32;
+constexpr int TP_SR_T = HK_TP_SR_T;
 constexpr int TP_TILE = 512;                // partners per shared-memory tile (6 KB)
 constexpr int TP_LUT = 2048;                // u-buckets: sign, 8 exponent bits, 2 mantissa bits
 
@@ -109,17 +114,18 @@ struct TPSmem {
   uint32_t* part;  // [TP_WARPS * NP/2 * nb2] flush scratch (the ring may hold a prefetched tile)
   int* flag;
 };
-__host__ __device__ inline size_t tp_smem_bytes(int nb2, int np) {
-  return (size_t)TP_LUT + 32 * 4 + 2 * 3 * TP_TILE * 4 + (size_t)TP_WARPS * (np / 2) * nb2 * 33 * 4 + 16;
+// (T = threads of the CTA: 128 for the replica kernels, HK_TP_SR_T for the single run)
+__host__ __device__ inline size_t tp_smem_bytes(int nb2, int np, int T = TP_THREADS) {
+  return (size_t)TP_LUT + 32 * 4 + 2 * 3 * TP_TILE * 4 + (size_t)(T / 32) * (np / 2) * nb2 * 33 * 4 + 16;
 }
-__device__ __forceinline__ TPSmem tp_carve(unsigned char* base, int nb2, int np) {
+__device__ __forceinline__ TPSmem tp_carve(unsigned char* base, int nb2, int np, int T = TP_THREADS) {
   TPSmem S;
   S.L = base;
   S.E = reinterpret_cast<float*>(base + TP_LUT);
   S.B = reinterpret_cast<float*>(base + TP_LUT + 128);
   S.H = reinterpret_cast<uint32_t*>(base + TP_LUT + 128 + 2 * 3 * TP_TILE * 4);
-  S.part = reinterpret_cast<uint32_t*>(base + TP_LUT + 128 + 2 * 3 * TP_TILE * 4 + (size_t)TP_WARPS * (np / 2) * nb2 * 128);
-  S.flag = reinterpret_cast<int*>(reinterpret_cast<unsigned char*>(S.part) + (size_t)TP_WARPS * (np / 2) * nb2 * 4);
+  S.part = reinterpret_cast<uint32_t*>(base + TP_LUT + 128 + 2 * 3 * TP_TILE * 4 + (size_t)(T / 32) * (np / 2) * nb2 * 128);
+  S.flag = reinterpret_cast<int*>(reinterpret_cast<unsigned char*>(S.part) + (size_t)(T / 32) * (np / 2) * nb2 * 4);
   return S;
 }
 __device__ __forceinline__ void cp_async4(void* dst, const void* src) {
@@ -138,27 +144,28 @@ __device__ __forceinline__ void tp_stage_tables(const TPParams& p, const TPSmem&
   if (threadIdx.x < 32) S.E[threadIdx.x] = threadIdx.x <= p.nb ? p.edges[threadIdx.x] : __int_as_float(0xff800000);
   cp_async_commit();
 }
-template <int NP>
+template <int NP, int T = TP_THREADS>
 __device__ __forceinline__ void tp_zero_hist(const TPParams& p, const TPSmem& S) {
-  const int nh = TP_WARPS * (NP / 2) * (p.nb + 2) * 32;
-  for (int k = threadIdx.x; k < nh; k += TP_THREADS) S.H[k] = 0u;
+  const int nh = (T / 32) * (NP / 2) * (p.nb + 2) * 32;
+  for (int k = threadIdx.x; k < nh; k += T) S.H[k] = 0u;
 }
 // Partners [j0, j0 + cnt) of set sb into ring slot `slot` (cnt <= TP_TILE; 4-byte async copies).
+template <int T = TP_THREADS>
 __device__ __forceinline__ void tp_stage_tile(const TPParams& p, const TPSmem& S, int sb, int j0, int cnt, int slot) {
   const float* src = p.pts + 3 * ((int64_t)sb * p.n + j0);
   float* dst = S.B + slot * 3 * TP_TILE;
-  for (int k = threadIdx.x; k < 3 * cnt; k += TP_THREADS) cp_async4(dst + k, src + k);
+  for (int k = threadIdx.x; k < 3 * cnt; k += T) cp_async4(dst + k, src + k);
   cp_async_commit();
 }
 
 // Reduce the lane-private histograms (both 16-bit halves of every word) and add them to
 // hist[base + b]: each (warp, word, bin) row of 32 counters is summed (rotated start: no bank
 // conflicts), the rows of a bin combined in shared memory, then one u64 atomic per non-zero bin.
-template <int NP>
+template <int NP, int T = TP_THREADS>
 __device__ __forceinline__ void tp_flush(const TPParams& p, const TPSmem& S, unsigned long long* hist, int base) {
-  const int nb2 = p.nb + 2, rows = TP_WARPS * (NP / 2);
+  const int nb2 = p.nb + 2, rows = (T / 32) * (NP / 2);
   uint32_t* part = S.part;
-  for (int t = threadIdx.x; t < rows * nb2; t += TP_THREADS) {
+  for (int t = threadIdx.x; t < rows * nb2; t += T) {
     const uint32_t* row = S.H + (size_t)t * 32;
     uint32_t s = 0;
 #pragma unroll 8
@@ -411,39 +418,39 @@ __device__ __forceinline__ void tp_pairs_all(const TPParams& p, const TPLoopCtx&
 
 // The diagonal, one partner at a time (GDIAG = false: the fused kernel of mix.cu, where the
 // grouped form below costs the main loop its interleaved schedule — measured).
-template <int NP, bool CNT, bool LUT, int S = 0>
+template <int NP, bool CNT, bool LUT, int S = 0, int STR = TP_THREADS>
 __device__ __forceinline__ void tp_diag1(const TPLoopCtx& c, const float* __restrict__ Bt, const uint32_t (&Hw)[NP / 2],
                                          TPPoint (&P)[NP], const uint32_t (&inc)[NP], int i0, int jt0, int k0, int km) {
-  const int ka = max(k0, i0 + S * TP_THREADS - jt0), kb = min(km, i0 + (S + 1) * TP_THREADS - jt0);
+  const int ka = max(k0, i0 + S * STR - jt0), kb = min(km, i0 + (S + 1) * STR - jt0);
 #pragma unroll 1
   for (int k = ka; k < kb; ++k) tp_pair1<NP, S + 1, true, CNT, LUT>(c, Hw, P, inc, Bt[3 * k], Bt[3 * k + 1], Bt[3 * k + 2], jt0 + k);
-  if constexpr (S + 1 < NP) tp_diag1<NP, CNT, LUT, S + 1>(c, Bt, Hw, P, inc, i0, jt0, k0, km);
+  if constexpr (S + 1 < NP) tp_diag1<NP, CNT, LUT, S + 1, STR>(c, Bt, Hw, P, inc, i0, jt0, k0, km);
 }
 
-// The diagonal of a self-correlation row, segment S: partners j in [i0 + 128 S, i0 + 128 (S + 1))
-// (tile-relative [ka, kb)).  Point k of a thread is i0 + 128 k + t, so for these partners points
-// k < S are all active (j > i), point S is masked (j >= jb) and points k > S take no part: the
-// grouped loop over points 0..S with the mask on point S.
-template <int NP, bool CNT, bool LUT, int S = 0>
+// The diagonal of a self-correlation row, segment S: partners j in [i0 + STR S, i0 + STR (S + 1))
+// (tile-relative [ka, kb)).  Point k of a thread is i0 + STR k + t (STR = the CTA's threads), so for
+// these partners points k < S are all active (j > i), point S is masked (j >= jb) and points k > S
+// take no part: the grouped loop over points 0..S with the mask on point S.
+template <int NP, bool CNT, bool LUT, int S = 0, int STR = TP_THREADS>
 __device__ __forceinline__ void tp_diag(const TPParams& p, const TPLoopCtx& c, const float* __restrict__ Bt,
                                         const uint32_t (&Hw)[NP / 2], TPPoint (&P)[NP], const uint32_t (&inc)[NP], int i0, int jt0,
                                         int k0, int km) {
-  const int ka = max(k0, i0 + S * TP_THREADS - jt0), kb = min(km, i0 + (S + 1) * TP_THREADS - jt0);
+  const int ka = max(k0, i0 + S * STR - jt0), kb = min(km, i0 + (S + 1) * STR - jt0);
   if (ka < kb) tp_pairs_grp<NP, S + 1, true, CNT, LUT>(p, c, Bt, Hw, P, inc, ka, kb, jt0);
-  if constexpr (S + 1 < NP) tp_diag<NP, CNT, LUT, S + 1>(p, c, Bt, Hw, P, inc, i0, jt0, k0, km);
+  if constexpr (S + 1 < NP) tp_diag<NP, CNT, LUT, S + 1, STR>(p, c, Bt, Hw, P, inc, i0, jt0, k0, km);
 }
 
 // Pairs of the staged tile Bt (partners jt0 + k) for k in [k0, k1): [k0, km) with per-point masks
-// (partners below jall = min(i0 + NP * 128, N) in a self-correlation row: its diagonal, in
+// (partners below jall = min(i0 + NP * STR, N) in a self-correlation row: its diagonal, in
 // segments), [km, k1) for all points.
-template <int NP, bool CNT, bool LUT, bool GDIAG = true>
+template <int NP, bool CNT, bool LUT, bool GDIAG = true, int STR = TP_THREADS>
 __device__ __forceinline__ void tp_tile_pairs(const TPParams& p, const TPLoopCtx& c, const float* __restrict__ Bt,
                                               const uint32_t (&Hw)[NP / 2], TPPoint (&P)[NP], const uint32_t (&inc)[NP],
                                               int jt0, int k0, int k1, int jall, int i0) {
   const int km = min(max(jall - jt0, k0), k1);
   if (k0 < km) {
-    if (GDIAG) tp_diag<NP, CNT, LUT>(p, c, Bt, Hw, P, inc, i0, jt0, k0, km);
-    else tp_diag1<NP, CNT, LUT>(c, Bt, Hw, P, inc, i0, jt0, k0, km);
+    if (GDIAG) tp_diag<NP, CNT, LUT, 0, STR>(p, c, Bt, Hw, P, inc, i0, jt0, k0, km);
+    else tp_diag1<NP, CNT, LUT, 0, STR>(c, Bt, Hw, P, inc, i0, jt0, k0, km);
   }
   tp_pairs_all<NP, CNT, LUT>(p, c, Bt, Hw, P, inc, km, k1);
 }
@@ -457,7 +464,7 @@ __device__ __forceinline__ void tp_lane_hist(const TPParams& p, const TPSmem& S,
 // One work item: the points i0 + t + 128 k (k < NP) of histogram h against partners [jr0, jr1)
 // (already clipped to the block's [jlo, N)), streamed tile by tile through the ring.  The tables
 // are staged and the histogram zeroed by the caller.
-template <int NP, int V, bool LUT, bool GDIAG = true>
+template <int NP, int V, bool LUT, bool GDIAG = true, int T = TP_THREADS>
 __device__ __forceinline__ void tp_item_loop(const TPParams& p, const TPSmem& S, TPPoint (&P)[NP], const uint32_t (&inc)[NP],
                                              int h, int i0, int jr0, int jr1) {
   constexpr bool CNT = (V & (V_L | V_PROF)) != 0;
@@ -465,39 +472,39 @@ __device__ __forceinline__ void tp_item_loop(const TPParams& p, const TPSmem& S,
   const int js = jr0 & ~3;  // tiles start on 4-partner boundaries (16-byte aligned groups in smem)
   const int nt = jr1 > jr0 ? (jr1 - js + TP_TILE - 1) / TP_TILE : 0;
   // partners below jall need per-point masks (self rows: j >= i + 1), the rest do not
-  const int jall = h <= p.nr ? min(i0 + NP * TP_THREADS, p.n) : 0;
+  const int jall = h <= p.nr ? min(i0 + NP * T, p.n) : 0;
   const uint32_t lane = lane_id(), warp = threadIdx.x >> 5;
   uint32_t Hw[NP / 2];
 #pragma unroll
   for (int w = 0; w < NP / 2; ++w) Hw[w] = smem_u32(S.H + (((size_t)warp * (NP / 2) + w) * (p.nb + 2)) * 32 + lane);
   const TPLoopCtx c{S.L, smem_u32(S.E), S.E};
-  if (nt > 0) tp_stage_tile(p, S, sb, js, min(TP_TILE, jr1 - js), 0);
+  if (nt > 0) tp_stage_tile<T>(p, S, sb, js, min(TP_TILE, jr1 - js), 0);
   for (int t = 0; t < nt; ++t) {
     const int jt0 = js + t * TP_TILE;
     if (t + 1 < nt) {
       const int jn = jt0 + TP_TILE;
-      tp_stage_tile(p, S, sb, jn, min(TP_TILE, jr1 - jn), (t + 1) & 1);
+      tp_stage_tile<T>(p, S, sb, jn, min(TP_TILE, jr1 - jn), (t + 1) & 1);
       cp_async_wait<1>();
     } else {
       cp_async_wait<0>();
     }
     __syncthreads();
-    tp_tile_pairs<NP, CNT, LUT, GDIAG>(p, c, S.B + (t & 1) * 3 * TP_TILE, Hw, P, inc, jt0, max(jr0, jt0) - jt0,
-                                min(jr1, jt0 + TP_TILE) - jt0, jall, i0);
+    tp_tile_pairs<NP, CNT, LUT, GDIAG, T>(p, c, S.B + (t & 1) * 3 * TP_TILE, Hw, P, inc, jt0, max(jr0, jt0) - jt0,
+                                          min(jr1, jt0 + TP_TILE) - jt0, jall, i0);
     __syncthreads();  // slot t & 1 is refilled by the stage of tile t + 2
   }
 }
 
-template <int NP>
+template <int NP, int T = TP_THREADS>
 __device__ __forceinline__ void tp_points(const TPParams& p, const unsigned long long* hist, int h, int blk, int64_t g0,
                                           int64_t g1, TPPoint (&P)[NP], bool nl) {
-  const int i0 = blk * NP * TP_THREADS;
+  const int i0 = blk * NP * T;
   const int64_t gb = (int64_t)h * p.n;
 #pragma unroll
   for (int k = 0; k < NP; ++k) {
-    const int i = i0 + k * TP_THREADS + threadIdx.x;
+    const int i = i0 + k * T + threadIdx.x;
     const bool v = i < p.n && gb + i >= g0 && gb + i < g1;
-    const int idup = (int)((blk ^ p.z) * (NP * TP_THREADS) + k * TP_THREADS + (threadIdx.x ^ p.z));
+    const int idup = (int)((blk ^ p.z) * (NP * T) + k * T + (threadIdx.x ^ p.z));
     P[k] = nl ? tp_prologue<true>(p, hist, h, i, idup, (int)((uint32_t)h ^ p.z), v)
               : tp_prologue<false>(p, hist, h, i, idup, (int)((uint32_t)h ^ p.z), v);
   }
@@ -526,10 +533,10 @@ __host__ __device__ __forceinline__ int64_t tp_sr_row(int n, int nr, int nblk, i
   constexpr int NP = HK_TP_NP_SR;
   *h = row / nblk;
   *blk = row - *h * nblk;
-  const int i0 = *blk * NP * TP_THREADS;
+  const int i0 = *blk * NP * TP_SR_T;
   const int64_t gb = (int64_t)*h * n;
   const int64_t a = gb + i0 > g0 ? gb + i0 : g0;
-  const int64_t e = gb + i0 + NP * TP_THREADS < gb + n ? gb + i0 + NP * TP_THREADS : gb + n;
+  const int64_t e = gb + i0 + NP * TP_SR_T < gb + n ? gb + i0 + NP * TP_SR_T : gb + n;
   const int64_t pts = (e < g1 ? e : g1) - a;
   *jlo = *h <= nr ? i0 + 1 : 0;
   return (pts > 0 && *jlo < n) ? pts * (int64_t)(n - *jlo) : 0;
@@ -584,16 +591,16 @@ __device__ __forceinline__ void tp_sr_piece(const TPParams& p, const TPSmem& S, 
   constexpr bool NL = (V & V_NL) != 0, L = (V & V_L) != 0, PROF = (V & V_PROF) != 0, CNT = L || PROF;
   int h, blk, jlo;
   tp_sr_row(p.n, p.nr, p.nblk, p.g0, p.g1, pc.x, &h, &blk, &jlo);
-  const int i0 = blk * NP * TP_THREADS;
+  const int i0 = blk * NP * TP_SR_T;
   const int64_t gb = (int64_t)h * p.n;
   const int64_t len = p.n - jlo;
   const int j0 = jlo + (int)(len * pc.y / pc.z), j1 = jlo + (int)(len * (pc.y + 1) / pc.z);
   TPPoint P[NP];
-  tp_points<NP>(p, p.hist, h, blk, p.g0, p.g1, P, NL);
+  tp_points<NP, TP_SR_T>(p, p.hist, h, blk, p.g0, p.g1, P, NL);
   uint32_t inc[NP];
 #pragma unroll
   for (int k = 0; k < NP; ++k) inc[k] = P[k].valid ? ((k & 1) ? 0x10000u : 1u) : 0u;
-  tp_zero_hist<NP>(p, S);
+  tp_zero_hist<NP, TP_SR_T>(p, S);
   // The points' state the pair loop does not touch (index, checksum, alarm bits, the NL-protected
   // loop-invariant values) waits in local memory while the loop runs, so the loop keeps its
   // registers for independent table lookups (HK_TP_STASH; the values are written once before and
@@ -608,7 +615,7 @@ __device__ __forceinline__ void tp_sr_piece(const TPParams& p, const TPSmem& S, 
     }
   }
   __syncthreads();
-  tp_item_loop<NP, V, LUT>(p, S, P, inc, h, i0, j0, j1);
+  tp_item_loop<NP, V, LUT, true, TP_SR_T>(p, S, P, inc, h, i0, j0, j1);
   if constexpr (STASH) {
 #pragma unroll
     for (int k = 0; k < NP; ++k) {
@@ -657,7 +664,7 @@ __device__ __forceinline__ void tp_sr_piece(const TPParams& p, const TPSmem& S, 
       if (P[k].valid) fold_alarm(p.cb, P[k].alarm, (uint32_t)(gb + P[k].i));
   }
   __syncthreads();
-  tp_flush<NP>(p, S, p.hist, h * (p.nb + 2));
+  tp_flush<NP, TP_SR_T>(p, S, p.hist, h * (p.nb + 2));
 }
 
 // FI & FT (or FI-only) replicas (blockIdx.y = launch slot)

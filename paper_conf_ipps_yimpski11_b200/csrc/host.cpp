@@ -183,13 +183,12 @@ static hk_status run_bench(int b, const void* args, int variant, const hk_ranges
   if (b == HK_CP) {
     const hk_cp_args* a = (const hk_cp_args*)args;
     ndet = std::min(ndet, a->unroll);
-    HK_CUDA(cudaMemsetAsync(a->grid, 0, sizeof(float) * (size_t)a->nx * a->ny, s), "memset grid");
+    // no zeroing: a whole run stores every grid point once, which equals R18's "+=" on a zeroed grid
     HK_CUDA(cp_launch(vf, *a, R, ndet, d_cb, d_samples, s), "cp kernel");
   } else if (b == HK_MRIQ) {
     const hk_mriq_args* a = (const hk_mriq_args*)args;
     ndet = std::min(ndet, 2);
-    HK_CUDA(cudaMemsetAsync(a->qr, 0, sizeof(float) * (size_t)a->n_vox, s), "memset qr");
-    HK_CUDA(cudaMemsetAsync(a->qi, 0, sizeof(float) * (size_t)a->n_vox, s), "memset qi");
+    // no zeroing: a whole run stores every voxel's Qr, Qi once (R18's "+=" on zeroed outputs)
     HK_CUDA(mriq_launch(vf, *a, R, ndet, d_cb, d_samples, s), "mriq kernels");
   } else {
     const hk_tpacf_args* a = (const hk_tpacf_args*)args;

@@ -116,7 +116,7 @@ __device__ __forceinline__ void mix_tp_slot(const MixParams& q, unsigned char* s
   __syncthreads();
   unsigned long long* hist = q.t.hist0 + (int64_t)r * q.t.hist_elems;
   hk_control* cb = q.t.cb0 + r;
-  const bool lut = *p0.lut_ok != 0;
+  const bool lut = *p0.lut_ok != 0 && tp_dsbase_ok();
   if (rank < 0) {
     if (lut) mix_tp_faulted<FT, true>(q.t, S, f, hist, cb, h, blk);
     else mix_tp_faulted<FT, false>(q.t, S, f, hist, cb, h, blk);

@@ -81,8 +81,9 @@ __global__ void __launch_bounds__(TP_SR_T, V == 0 ? HK_TP_MINB_SR : HK_TP_MINB_S
   unsigned long long t0;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
 #endif
-  __shared__ int3 s_pc;
+  // the piece descriptor lives past the carve (no static shared memory: tp_dsbase_ok)
   const TPSmem S = tp_carve(hk_tp_dsmem, p.nb + 2, HK_TP_NP_SR, TP_SR_T);
+  int3& s_pc = *reinterpret_cast<int3*>(hk_tp_dsmem + tp_smem_bytes(p.nb + 2, HK_TP_NP_SR, TP_SR_T));
   tp_stage_tables(p, S);
   if (threadIdx.x < 32) {
     const int3 pc = tp_sr_locate(p, q, (int)blockIdx.x);
@@ -92,7 +93,7 @@ __global__ void __launch_bounds__(TP_SR_T, V == 0 ? HK_TP_MINB_SR : HK_TP_MINB_S
   __syncthreads();
   const int3 pc = s_pc;
   if (pc.x < 0) return;
-  if (*p.lut_ok) tp_sr_piece<V, true>(p, S, q, pc);
+  if (*p.lut_ok && tp_dsbase_ok()) tp_sr_piece<V, true>(p, S, q, pc);
   else tp_sr_piece<V, false>(p, S, q, pc);
 #ifdef HK_TP_SR_TRACE
   __syncthreads();
@@ -136,7 +137,7 @@ __global__ void __launch_bounds__(TP_THREADS, HK_TP_MINB) tpacf_fi_kernel(const 
   __syncthreads();
   unsigned long long* hist = q.hist0 + (int64_t)r * q.hist_elems;
   hk_control* cb = q.cb0 + r;
-  if (*p0.lut_ok) tp_replica_cta<KIND, FT, true>(q, S, f, hist, cb, h, blk, faulted);
+  if (*p0.lut_ok && tp_dsbase_ok()) tp_replica_cta<KIND, FT, true>(q, S, f, hist, cb, h, blk, faulted);
   else tp_replica_cta<KIND, FT, false>(q, S, f, hist, cb, h, blk, faulted);
 }
 
@@ -288,7 +289,7 @@ void tpacf_release_caches() {}
 template <int V>
 static cudaError_t launch_tp_v(const hk_tpacf_args& a, TPParams p, void* ws, cudaStream_t s) {
   constexpr bool CNT = (V & (V_L | V_PROF)) != 0;
-  const size_t smem = tp_smem_bytes(p.nb + 2, HK_TP_NP_SR, TP_SR_T);
+  const size_t smem = tp_smem_bytes(p.nb + 2, HK_TP_NP_SR, TP_SR_T) + 16;  // + the piece descriptor
   cudaError_t e = cudaFuncSetAttribute(tpacf_kernel<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   if (p.g1 <= p.g0) return cudaSuccess;

@@ -81,18 +81,24 @@ __device__ __forceinline__ uint32_t tp_b4_lut(const uint8_t* __restrict__ L, uin
   asm("ld.shared.f32 %0, [%1];" : "=f"(e) : "r"(eb + b4));
   return (dot < e) ? b4 + 4u : b4;
 }
-// Every TPACF kernel carves its TPSmem from the start of dynamic shared memory, so the table and
-// the edges sit at link-time constant shared addresses: the pair loops index them from the symbol
-// ([reg + imm] addressing, no base register add per lookup).
+// Every TPACF kernel carves its TPSmem from the start of dynamic shared memory and declares no
+// static shared memory, so in a launch without clusters the table sits at the shared address
+// TP_DSBASE (the first KB of the CTA's window is the system's) and the edges at TP_DSBASE + TP_LUT:
+// the pair loops address both as [reg + immediate] (no base add per lookup; the kernels check
+// tp_dsbase_ok() once and otherwise take the binary search).  The compare-and-step is one PTX
+// select so the compiler forms the histogram address as one LEA of the stepped value.
 extern __shared__ __align__(128) unsigned char hk_tp_dsmem[];
+constexpr uint32_t TP_DSBASE = 0x400;
+__device__ __forceinline__ bool tp_dsbase_ok() { return (uint32_t)__cvta_generic_to_shared(hk_tp_dsmem) == TP_DSBASE; }
 __device__ __forceinline__ uint32_t tp_b4_fixed(float dot) {
-  const uint32_t base = (uint32_t)__cvta_generic_to_shared(hk_tp_dsmem);
   const float u = __fsub_rn(1.0f, dot);
-  uint32_t b4;
+  uint32_t b4, r;
   float e;
-  asm("ld.shared.u8 %0, [%1];" : "=r"(b4) : "r"(base + (fb(u) >> 21)));
-  asm("ld.shared.f32 %0, [%1];" : "=f"(e) : "r"(base + (uint32_t)TP_LUT + b4));
-  return (dot < e) ? b4 + 4u : b4;
+  asm("ld.shared.u8 %0, [%1+%2];" : "=r"(b4) : "r"(fb(u) >> 21), "n"(TP_DSBASE));
+  asm("ld.shared.f32 %0, [%1+%2];" : "=f"(e) : "r"(b4), "n"(TP_DSBASE + TP_LUT));
+  asm("{\n\t.reg .pred p;\n\tsetp.lt.f32 p, %1, %2;\n\tadd.u32 %0, %3, 4;\n\tselp.u32 %0, %0, %3, p;\n\t}"
+      : "=r"(r) : "f"(dot), "f"(e), "r"(b4));
+  return r;
 }
 template <bool LUT>
 __device__ __forceinline__ uint32_t tp_b4(const uint8_t* __restrict__, uint32_t, const float* Es, float dot) {

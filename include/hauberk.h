@@ -85,8 +85,9 @@ typedef struct {
 } hk_control;
 
 /* CP (K1; Fig. 9).  atoms: [n_atoms] (x, y, z, q); atoms_ws: [n_atoms] float4 scratch
- * for the (x, y, dz^2, q) pre-pass (both 16-byte aligned); grid: [ny][nx] output, zeroed by the
- * callee.  Requires nx % (bx*unroll) == 0, ny % by == 0, bx*by <= 256 and a multiple of 32,
+ * for the (x, y, dz^2, q) pre-pass (both 16-byte aligned); grid: [ny][nx] output, every point
+ * written by a whole run (the abstract program's "+=" onto a zeroed grid, R18; hauberk_run_part
+ * zeroes its rows and adds).  Requires nx % (bx*unroll) == 0, ny % by == 0, bx*by <= 256 and a multiple of 32,
  * unroll in {1,2,4,8} (campaigns: unroll 4 or 8).  Detector d (maxvar = d + 1) checks the
  * self-accumulator E_{unroll-1} for d = 0, then E_0, E_1, ... (A6, DESIGN R12). */
 typedef struct {
@@ -95,7 +96,8 @@ typedef struct {
 } hk_cp_args;
 
 /* MRI-Q (K2).  x,y,z: [n_vox]; kx..phi_i: [n_k]; kv_ws: [n_k] float4 scratch (PhiMag output);
- * qr, qi: [n_vox] outputs (zeroed by the callee). */
+ * qr, qi: [n_vox] outputs, every voxel written by a whole run (R18's "+=" onto zeroed outputs;
+ * hauberk_run_part zeroes its voxels and adds). */
 typedef struct {
   const float *x, *y, *z; int32_t n_vox, n_k;
   const float *kx, *ky, *kz, *phi_r, *phi_i; float* kv_ws; float *qr, *qi; int32_t exact;

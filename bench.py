@@ -485,9 +485,9 @@ def main():
                     "measured": f"library CUDA events on the fused launch's stream inside the {args.steps} timed steps",
                     "peak_source": f"{N_SM} SMs x {MUFU_PER_SM_CLK} MUFU / {LANES_PER_SM_CLK} lanes per clk/SM x "
                                    f"{sm_mhz_peak:.0f} MHz ({clk_src})",
-                    "limiter_ncu": "instruction issue (profiles/r02_ncu_mix_summary.txt): 85.6M warp instructions per MRI-Q + "
-                                   "TPACF replica pair = 73.5 us at one instruction per clock per SM sub-partition; "
-                                   "83.7 % of issue slots active"}
+                    "limiter_ncu": "instruction issue (profiles/r02_ncu_mix_summary.txt): 85.8M warp instructions per MRI-Q + "
+                                   "TPACF replica pair = 73.7 us at one instruction per clock per SM sub-partition; "
+                                   "83.6 % of issue slots active"}
         tr_key = "mix_fi_kernel"
         n_rep = [sum(1 for st in range(args.steps)
                      for n in range(*(lambda f, c: (f, f + c))(*par.step_slice(st, rank, world, args.per_rank))) if n % 3 == b)

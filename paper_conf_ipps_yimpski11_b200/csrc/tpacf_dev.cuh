@@ -646,6 +646,9 @@ __device__ __forceinline__ void tp_sr_piece(const TPParams& p, const TPSmem& S, 
           atomicAdd(p.accg + gb + P[k].i, P[k].acc);
           atomicAdd(p.cntg + gb + P[k].i, P[k].cnt);
         }
+      // the histogram flush overlaps the combine atomics' round trip (the loop's last barrier
+      // already ordered every ATOMS of the piece)
+      tp_flush<NP, TP_SR_T>(p, S, p.hist, h * (p.nb + 2));
       __syncthreads();  // every thread's combine atomics issued
       if (threadIdx.x == 0) {
         __threadfence();
@@ -669,8 +672,10 @@ __device__ __forceinline__ void tp_sr_piece(const TPParams& p, const TPSmem& S, 
     for (int k = 0; k < NP; ++k)
       if (P[k].valid) fold_alarm(p.cb, P[k].alarm, (uint32_t)(gb + P[k].i));
   }
-  __syncthreads();
-  tp_flush<NP, TP_SR_T>(p, S, p.hist, h * (p.nb + 2));
+  if (!CNT || pc.z == 1) {
+    __syncthreads();
+    tp_flush<NP, TP_SR_T>(p, S, p.hist, h * (p.nb + 2));
+  }
 }
 
 // FI & FT (or FI-only) replicas (blockIdx.y = launch slot)

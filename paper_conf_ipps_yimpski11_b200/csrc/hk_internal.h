@@ -33,10 +33,13 @@ cudaError_t mriq_launch(int vflags, const hk_mriq_args& a, const DevRanges& R, i
                         float* samples, cudaStream_t s);
 // TPACF: abstract threads [g0, g1) (g1 < 0: all); ws = tpacf_ws_bytes(a) bytes (bin table, single-run
 // schedule counters, per-thread (acc, cnt) partial sums)
+// Zeroes a.hist itself (in the table kernel) before adding the run's counts into it.
 cudaError_t tpacf_launch(int vflags, const hk_tpacf_args& a, const DevRanges& R, int ndet, hk_control* cb,
                          float* samples, void* ws, cudaStream_t s, int32_t g0 = 0, int32_t g1 = -1);
 size_t tpacf_ws_bytes(const hk_tpacf_args& a);
-cudaError_t tpacf_lut_build(const hk_tpacf_args& a, void* ws, cudaStream_t s);
+// Builds the bucket table in ws; the same launch zeroes the word ranges [z0, z0 + n0), [z1, z1 + n1).
+cudaError_t tpacf_lut_build(const hk_tpacf_args& a, void* ws, cudaStream_t s, uint32_t* z0 = nullptr, int64_t n0 = 0,
+                            uint32_t* z1 = nullptr, int64_t n1 = 0);
 void tpacf_release_caches();
 cudaError_t cp_prepass_launch(const hk_cp_args& a, cudaStream_t s);
 cudaError_t mriq_phimag_launch(const hk_mriq_args& a, bool nl, hk_control* cb, cudaStream_t s);

@@ -37,12 +37,16 @@ namespace hk {
 // edges share a bucket (checked; the edges are strictly decreasing, so their bucket ordinals are
 // non-decreasing).  Exponent-0xff buckets: +inf u (dot = -inf) follows the same rule (every finite
 // edge precedes it); NaN u (dot NaN) has bin 0; -inf u (dot = +inf) precedes every bucket.
-// Block 0 also writes the validity flag (no separate memset).
+// Block 0 also writes the validity flag, and the grid zeroes up to two word ranges for the run that
+// follows (its histogram and its partial-sum workspace: no separate memsets).
 __device__ __forceinline__ int tp_bucket_ord(uint32_t q) { return q < 1024u ? 1024 + (int)q : 2047 - (int)q; }
-__global__ void __launch_bounds__(256) tpacf_lut_kernel(const float* __restrict__ edges, int nb, uint8_t* __restrict__ lut, int* ok) {
+__global__ void __launch_bounds__(256) tpacf_lut_kernel(const float* __restrict__ edges, int nb, uint8_t* __restrict__ lut, int* ok,
+                                                         uint32_t* z0, int64_t n0, uint32_t* z1, int64_t n1) {
   __shared__ int eo[32];
   __shared__ int bad;
   const int q = blockIdx.x * blockDim.x + threadIdx.x;
+  for (int64_t k = q; k < n0; k += TP_LUT) z0[k] = 0u;
+  for (int64_t k = q; k < n1; k += TP_LUT) z1[k] = 0u;
   if (threadIdx.x == 0) bad = 0;
   __syncthreads();
   if (threadIdx.x <= nb && threadIdx.x < 32) {
@@ -270,9 +274,10 @@ size_t tpacf_ws_bytes(const hk_tpacf_args& a) {
   return tp_ws_head() + tp_rows_bytes(a) + nt * 8;
 }
 
-cudaError_t tpacf_lut_build(const hk_tpacf_args& a, void* ws, cudaStream_t s) {
+cudaError_t tpacf_lut_build(const hk_tpacf_args& a, void* ws, cudaStream_t s, uint32_t* z0, int64_t n0, uint32_t* z1,
+                            int64_t n1) {
   int* ok = reinterpret_cast<int*>(reinterpret_cast<char*>(ws) + TP_LUT);
-  tpacf_lut_kernel<<<TP_LUT / 256, 256, 0, s>>>(a.edges, a.n_bins, reinterpret_cast<uint8_t*>(ws), ok);
+  tpacf_lut_kernel<<<TP_LUT / 256, 256, 0, s>>>(a.edges, a.n_bins, reinterpret_cast<uint8_t*>(ws), ok, z0, n0, z1, n1);
   count_launch();
   return cudaGetLastError();
 }
@@ -324,7 +329,8 @@ static cudaError_t launch_tp_v(const hk_tpacf_args& a, TPParams p, void* ws, cud
     grid += tp_sr_pieces(wr, wcum, p.n - jlo, q.slots, total);
     wcum += wr;
   }
-  if (CNT && (e = cudaMemsetAsync(w + tp_ws_head(), 0, tpacf_ws_bytes(a) - tp_ws_head(), s)) != cudaSuccess) return e;
+  // (the histogram and, for CNT, the workspace's counters and partial sums were zeroed by the table
+  // kernel: tpacf_launch)
   TimedScope ts(HK_TPACF, 0, tp_pairs(a) * (double)(p.g1 - p.g0) / (double)((1 + 2 * p.nr) * p.n), s);
   tpacf_kernel<V><<<(unsigned)grid, TP_SR_T, smem, s>>>(p, q);
   count_launch();
@@ -334,7 +340,12 @@ static cudaError_t launch_tp_v(const hk_tpacf_args& a, TPParams p, void* ws, cud
 // Abstract threads [g0, g1) (g1 < 0: all) of one run, their counts added into hist (sharding).
 cudaError_t tpacf_launch(int vflags, const hk_tpacf_args& a, const DevRanges& R, int ndet, hk_control* cb, float* samples,
                          void* ws, cudaStream_t s, int32_t g0, int32_t g1) {
-  cudaError_t e = tpacf_lut_build(a, ws, s);
+  // the table kernel also zeroes the histogram and (detector variants) the partial-sum workspace
+  const bool cnt = (vflags & (V_L | V_PROF)) != 0;
+  uint32_t* ws_tail = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(ws) + tp_ws_head());
+  const int64_t ws_words = cnt ? (int64_t)((tpacf_ws_bytes(a) - tp_ws_head()) / 4) : 0;
+  const int64_t hist_words = 2 * (int64_t)(1 + 2 * a.n_rand) * (a.n_bins + 2);
+  cudaError_t e = tpacf_lut_build(a, ws, s, reinterpret_cast<uint32_t*>(a.hist), hist_words, ws_tail, ws_words);
   if (e != cudaSuccess) return e;
   TPParams p = tp_params(a, R, ndet, cb, samples, ws);
   p.g0 = g0;

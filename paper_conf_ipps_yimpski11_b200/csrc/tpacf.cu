@@ -293,7 +293,6 @@ void tpacf_release_caches() {}
 
 template <int V>
 static cudaError_t launch_tp_v(const hk_tpacf_args& a, TPParams p, void* ws, cudaStream_t s) {
-  constexpr bool CNT = (V & (V_L | V_PROF)) != 0;
   const size_t smem = tp_smem_bytes(p.nb + 2, HK_TP_NP_SR, TP_SR_T) + 16;  // + the piece descriptor
   cudaError_t e = cudaFuncSetAttribute(tpacf_kernel<V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;

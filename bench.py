@@ -253,6 +253,14 @@ def _trimmed_mean(xs, frac=0.1):
     return sum(core) / len(core)
 
 
+def _nccl_version():
+    try:
+        v = torch.cuda.nccl.version()
+        return ".".join(str(x) for x in v) if isinstance(v, (tuple, list)) else str(v)
+    except Exception:  # noqa: BLE001 - diagnostics only
+        return None
+
+
 def main():
     args = parse()
     if args.impl == "reference":
@@ -644,6 +652,10 @@ def main():
                        "per_rank_injections_per_step": args.per_rank, "parallelism": f"campaign-sharded x{world}",
                        "l2": "flushed between steps (512 MiB write, outside the events)"},
             "clocks": clk,
+            # the process group the counters were all-reduced over (a multi-GPU run shows its NCCL ranks)
+            "dist": {"backend": (backend if world > 1 else "none"),
+                     "world_size": (dist.get_world_size() if dist.is_initialized() else 1),
+                     "nccl_version": _nccl_version() if (world > 1 and backend == "nccl") else None},
             "e2e": {"value": round(e2e_value, 2), "unit": "injections/s", "h2d_bytes_per_step": int(h2d),
                     "d2h_bytes_per_step": 3 * 5 * 8, "steps": e2e_steps},
             "gpu_launches": int(launches),

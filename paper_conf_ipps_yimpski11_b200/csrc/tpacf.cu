@@ -80,7 +80,7 @@ extern "C" __attribute__((visibility("default"))) int hk_debug_trace(void* out) 
 }
 #endif
 template <int V>
-__global__ void __launch_bounds__(TP_SR_T, V == 0 ? HK_TP_MINB_SR : HK_TP_MINB_SR_FT) tpacf_kernel(const TPParams p, const TPSR q) {
+__global__ void __launch_bounds__(TP_SR_T, V == 0 ? HK_TP_MINB_SR : (V == V_NL ? HK_TP_MINB_SR_NL : HK_TP_MINB_SR_FT)) tpacf_kernel(const TPParams p, const TPSR q) {
 #ifdef HK_TP_SR_TRACE
   unsigned long long t0;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));

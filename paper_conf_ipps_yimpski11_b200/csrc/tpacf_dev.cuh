@@ -26,6 +26,10 @@ namespace hk {
                          // FT_NL (its loop otherwise runs out of registers for independent lookups,
                          // 77.8 -> 67.6 us); FT and FT_L measured 2 us slower with it
 #endif
+#ifndef HK_TP_MINB_SR_NL
+#define HK_TP_MINB_SR_NL (HK_TP_SR_T == 128 ? 6 : 1)  // FT_NL (its exit state in local memory, HK_TP_STASH):
+                                                       // 80 registers, 6 CTAs per SM (61.4 vs 63.5 us at 5)
+#endif
 #ifndef HK_TP_MINB_SR_FT
 #define HK_TP_MINB_SR_FT (HK_TP_SR_T == 128 ? 5 : 1)  // with detectors: 96 registers at 128 threads (at 80 the
                                                        // NL / L state spills)

@@ -380,3 +380,27 @@ def test_fused_replicas_equal_separate_launches(monkeypatch, variant, exact, per
         assert np.array_equal(r1[k], r0[k]), k
     assert np.array_equal(c1, c0)
     assert (r1["bench"] == 1).sum() > 700 and (r1["bench"] == 2).sum() > 700
+
+
+# ---------------------------------------------------------------------------------- perf guard
+def test_tpacf_single_run_takes_the_table_path():
+    """The TPACF loops address the bucket table and the edges at the constant shared address 0x400
+     and fall back to the binary search when a kernel's dynamic shared memory starts
+    elsewhere (a static __shared__ variable, a cluster launch).  The fallback is correct but slower;
+    this guards the config-3 single run against silently taking it (BASE ~60 us on B200)."""
+    d = _mk(2, W.tpacf_config3())
+    R = hk.profile_ranges(d)
+    cb = hk.new_control(torch.device(DEV))
+    flush = torch.empty(128 * 1024 * 1024, dtype=torch.float32, device=DEV)
+    hk.timing_enable(True)
+    ks = []
+    for r in range(12):
+        flush.zero_()
+        hk.run(d, hk.HK_BASE, R, cb)
+        torch.cuda.synchronize()
+        ms, _, _ = hk.timing_read(d.bench, 0)
+        if r >= 2:
+            ks.append(ms)
+    hk.timing_enable(False)
+    med = float(np.median(ks))
+    assert med < 0.085, f"TPACF BASE single run {med * 1e3:.1f} us: the table path was not taken?"
